@@ -1,0 +1,31 @@
+# Builds libbk.so (sm_100a CUDA + C++ runtime, C ABI), the oracle and the input generators.
+NVCC   ?= nvcc
+ARCH   := -gencode arch=compute_100a,code=sm_100a
+NVFLAGS := -std=c++17 -O3 -lineinfo $(ARCH) -Xcompiler -fPIC,-fvisibility=hidden -Xptxas -v
+PKG    := paper_conf_ipps_mokhtaris14_b200
+CSRC   := $(PKG)/csrc
+OBJS   := build/kernels_stage.o build/kernels_compute.o build/bk_runtime.o
+
+all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so
+
+build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh include/bk.h
+	@mkdir -p build
+	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
+
+$(PKG)/libbk.so: $(OBJS)
+	$(NVCC) -shared $(ARCH) -cudart static -o $@ $(OBJS)
+
+oracle/libbkoracle.so: oracle/oracle.c oracle/oracle.h
+	gcc -O2 -ffp-contract=off -fPIC -shared -Wall -o $@ oracle/oracle.c -lm
+
+gen/libbkgen.so: gen/gen.c gen/gen.h
+	gcc -O2 -fopenmp -fPIC -shared -Wall -o $@ gen/gen.c -lm
+
+build/probe: tools/probe.cu
+	@mkdir -p build
+	$(NVCC) -O3 $(ARCH) -o $@ $<
+
+clean:
+	rm -rf build $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so
+
+.PHONY: all clean

@@ -1,0 +1,220 @@
+/* bk.h — C ABI of libbk, the B200-native BigKernel streaming path.
+ *
+ * What it implements (§III): a kernel over an arbitrarily large,
+ * record-partitioned host data set ("segments") runs as a four-stage pipeline —
+ *   (1) prefetch address generation on the GPU,
+ *   (2) assembly of exactly the accessed bytes in thread-interleaved order,
+ *   (3) transfer over the host link,
+ *   (4) the compute kernel over the staged chunk,
+ * with several buffer instances so the stages of consecutive chunks overlap.
+ * The programmer registers the host array once and calls bk_run once; there are no
+ * programmer-managed buffers, chunks or transfers.
+ *
+ * Plain C: no CUDA, PyTorch or C++ types in any signature. A CUDA stream is passed as an
+ * opaque `void*` (a cudaStream_t / CUstream; NULL = legacy default stream). Every function
+ * returns a bk_status (0 = OK, negative = error); no exception or CUDA error escapes.
+ * bk_last_error() returns a thread-local detail string for the most recent failure.
+ * A context is single-threaded: use one context per GPU (several per process are allowed).
+ */
+#ifndef BK_H
+#define BK_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define BK_ABI_VERSION 1
+#if defined(__GNUC__)
+#define BK_API __attribute__((visibility("default")))
+#else
+#define BK_API
+#endif
+
+typedef enum {
+  BK_OK = 0,
+  BK_E_INVAL = -1,        /* bad argument, malformed offsets, key out of range */
+  BK_E_NOMEM = -2,        /* device or pinned allocation failed / window too small */
+  BK_E_CUDA = -3,         /* CUDA runtime/driver error (detail in bk_last_error) */
+  BK_E_STATE = -4,        /* call out of order (run before register, ...) */
+  BK_E_RANGE = -5,        /* one record's accessed bytes exceed the chunk budget (A18) */
+  BK_E_CAPACITY = -6,     /* output or table too small; required size written back */
+  BK_E_UNSUPPORTED = -7   /* kernel id / gather mode not supported by this build */
+} bk_status;
+
+/* Built-in compute kernels (north_star: kernels selected by kernel_id). */
+typedef enum {
+  BK_K_WORDCOUNT = 1,   /* C1: word -> count table        out: bk_out_wordcount */
+  BK_K_GREP = 2,        /* C2: ordered indices of records whose key contains a pattern bk_out_grep */
+  BK_K_KMEANS = 3,      /* C3: assignment + per-cluster partial sums      bk_out_kmeans */
+  BK_K_PARTITION = 4,   /* C4: stable hash partition into B buckets                    bk_out_partition */
+  BK_K_GROUPBY = 5,     /* C5: group-by count / sum                                    bk_out_groupby */
+  BK_K_LAYOUT_DUMP = 100 /* test only: copy one chunk's staged bytes + lane table back       bk_out_layout */
+} bk_kernel_id;
+
+/* Stage-2/3 implementations. */
+typedef enum {
+  BK_GATHER_AUTO = 0,   /* ZC for sparse access, DENSE when every byte is accessed */
+  BK_GATHER_ZC = 1,     /* GPU kernel reads the accessed bytes from pinned, mapped host memory
+                           (16-B loads) and writes the interleaved tiles to HBM: stages 2+3 fused */
+  BK_GATHER_CPU = 2,    /* reserved: host-thread assembly into pinned staging + DMA (not in this build) */
+  BK_GATHER_DENSE = 3   /* one contiguous DMA of the chunk's records (copy engine), then an
+                           HBM->HBM re-layout kernel (fetch-all) */
+} bk_gather_mode;
+
+typedef struct bk_config {
+  uint32_t struct_size;   /* = sizeof(bk_config) */
+  int32_t device;         /* CUDA ordinal the context binds to */
+  uint64_t window_bytes;  /* device working-set cap for ALL streaming buffers (slots, offsets
+                             slices, lane tables); 0 = 2 GiB. Resident aggregates are outside it. */
+  uint32_t n_slots;       /* ring depth N >= 2 ("at minimum two"); 0 = 4 */
+  uint32_t gather_mode;   /* bk_gather_mode */
+  uint64_t chunk_bytes;   /* accessed (payload) bytes per chunk; 0 = auto (fits a slot, >= ~32 chunks) */
+  uint32_t lanes;         /* lanes (compute threads) per chunk, multiple of 32; 0 = auto */
+  uint32_t host_threads;  /* reserved for BK_GATHER_CPU */
+  uint64_t record_size;   /* fixed record length when record_offsets == NULL */
+  uint32_t flags;         /* BK_FLAG_* */
+  uint32_t _reserved;
+} bk_config;
+
+#define BK_FLAG_PROFILE 1u  /* time every stage of every chunk with CUDA events (bk_stats.ms_*) */
+
+typedef struct bk_ctx bk_ctx;
+
+/* Allocates the context, its streams, events and the staging ring (window_bytes) on
+ * cfg->device. *out_ctx is owned by the caller and freed by bk_destroy. */
+BK_API int bk_create(const bk_config* cfg, bk_ctx** out_ctx);
+
+/* Maps a host data set (P:355-360 streamingMap). host_ptr[0..nbytes) and, if given,
+ * record_offsets[0..n_records) are BORROWED until bk_destroy or the next registration.
+ * record_offsets: u64 record start offsets relative to host_ptr, off[0] == 0, non-decreasing,
+ * each <= nbytes; record i = [off[i], off[i+1]) with off[n] := nbytes; empty records are legal.
+ * record_offsets == NULL: fixed records of cfg.record_size bytes (nbytes % record_size == 0,
+ * n_records must equal nbytes / record_size). Memory is pinned ONCE here (cudaHostRegister,
+ * mapped + portable) unless already pinned; pre-pinned memory is left as is.
+ * Validation is O(n) once: BK_E_INVAL on malformed offsets. */
+BK_API int bk_register_segments(bk_ctx* ctx, const void* host_ptr, uint64_t nbytes,
+                         const uint64_t* record_offsets, uint64_t n_records);
+
+/* Runs built-in kernel `kernel_id` over every registered record through the pipeline.
+ * Ordered after prior work on `stream`; returns when `out` is valid (blocking) and also
+ * records completion on `stream`. `out` points to the kernel's caller-owned in/out struct
+ * (bk_out_*), whose first two fields are {struct_size, kernel_id}. */
+BK_API int bk_run(bk_ctx* ctx, int kernel_id, void* stream, void* out);
+
+/* NULL-safe. Unpins what bk_register_segments pinned, frees device memory. */
+BK_API int bk_destroy(bk_ctx* ctx);
+
+BK_API const char* bk_strerror(int status);
+BK_API const char* bk_last_error(void);
+
+/* ---- per-kernel in/out structs (host pointers unless stated) ---- */
+typedef struct bk_out_header { uint32_t struct_size; int32_t kernel_id; } bk_out_header;
+
+typedef struct bk_out_wordcount {
+  bk_out_header h;
+  uint64_t table_slots;     /* in: device hash-table slots (power of two); 0 = 2^20 */
+  uint64_t cap;             /* in: capacity of the three arrays below */
+  uint64_t* word_off;       /* out: offset (rel. host_ptr) of one occurrence of each distinct word */
+  uint32_t* word_len;       /* out: its length */
+  uint64_t* word_count;     /* out: its count (unordered; compare as a multiset) */
+  uint64_t n_words;         /* out: distinct words (> cap -> BK_E_CAPACITY) */
+  uint64_t total_words;     /* out */
+} bk_out_wordcount;
+
+typedef struct bk_out_grep {
+  bk_out_header h;
+  const uint8_t* pattern;   /* in: <= 32 bytes; empty matches every record */
+  uint32_t pattern_len;
+  uint32_t _pad;
+  uint64_t first_index;     /* in: added to every index (the shard's first global record) */
+  uint64_t cap;             /* in: capacity of idx */
+  uint64_t* idx;            /* out: ascending matching record indices */
+  uint64_t n_match;         /* out (> cap -> BK_E_CAPACITY) */
+} bk_out_grep;
+
+typedef struct bk_out_kmeans {
+  bk_out_header h;
+  const float* centroids;   /* in: K x 16 fp32 */
+  uint32_t K;               /* in: 1..256 */
+  uint32_t _pad;
+  uint64_t first_index;     /* in: global index of record 0 (checksum) */
+  uint64_t* count;          /* out: K */
+  double* sum;              /* out: K x 16 */
+  uint64_t chk;             /* out: sum_i mix64((i<<8) ^ cid_i) mod 2^64 */
+  int32_t* cid;             /* out, optional (NULL): per-record cluster id, written back to the
+                               host through mapped memory (P:563-572 writes to mapped data) */
+} bk_out_kmeans;
+
+typedef struct bk_out_partition {
+  bk_out_header h;
+  uint32_t n_buckets;       /* in: power of two, 1..4096 */
+  uint32_t _pad;
+  uint64_t* out_records;    /* out: n_records x 16 B, chunk-major runs, each chunk bucket-sorted and stable */
+  uint64_t* chunk_counts;   /* out: n_chunks x n_buckets run lengths */
+  uint64_t chunk_cap;       /* in: capacity of chunk_counts in chunks */
+  uint64_t n_chunks;        /* out */
+  uint64_t* bucket_count;   /* out: n_buckets totals */
+} bk_out_partition;
+
+typedef struct bk_out_groupby {
+  bk_out_header h;
+  uint32_t G;               /* in: number of keys (dense 0..G-1), <= 65536 */
+  uint32_t _pad;
+  uint64_t* count;          /* out: G */
+  uint64_t* qty;            /* out: G */
+  double* amount;           /* out: G */
+} bk_out_groupby;
+
+typedef struct bk_out_layout {
+  bk_out_header h;
+  uint32_t n_ext;           /* in: 0 = whole record, else extents (<= 8) */
+  uint32_t ext_off[8];
+  uint32_t ext_len[8];
+  uint64_t chunk;           /* in: which chunk to dump */
+  uint8_t* stage;           /* out: staged bytes (stage_cap) */
+  uint64_t stage_cap;
+  uint64_t* lane_first;     /* out: lanes entries each (lane_cap) */
+  uint64_t* lane_nrec;
+  uint64_t* lane_bytes;
+  uint64_t lane_cap;
+  uint64_t stage_size;      /* out */
+  uint32_t lanes;           /* out */
+  uint32_t _pad;
+  uint64_t chunk_lo, chunk_hi, n_chunks; /* out */
+} bk_out_layout;
+
+typedef struct bk_stats {
+  uint32_t struct_size;
+  uint32_t gather_mode;       /* mode the last run used */
+  uint64_t n_chunks;
+  uint64_t chunk_budget;      /* accessed bytes per chunk */
+  uint32_t lanes;             /* lanes per chunk */
+  uint32_t n_slots;
+  uint64_t slot_bytes;        /* device bytes per ring slot */
+  uint64_t bytes_accessed;    /* sum of accessed bytes = algorithmic payload (I3) */
+  uint64_t bytes_h2d;         /* payload bytes that crossed the link (DENSE: whole records) */
+  uint64_t bytes_meta;        /* offsets slices shipped to the device */
+  uint64_t bytes_padding;     /* staged - accessed (HBM only, never on the link; A9) */
+  uint64_t bytes_d2h;
+  uint64_t kernel_launches;   /* this library's kernel launches in the last run */
+  double ms_run;              /* wall time of the last bk_run */
+  double ms_register;         /* pin + validate time of the last registration */
+  double ms_device;           /* CUDA-event time of the last run on its compute stream */
+  double ms_h2d;              /* BK_FLAG_PROFILE: summed per-chunk busy time of the H2D copies */
+  double ms_addrgen;          /*   ... of stage 1 (address generation) */
+  double ms_gather;           /*   ... of stage 2 (+3 in ZC mode): gather / re-layout kernels */
+  double ms_compute;          /*   ... of stage 4 (compute kernels) */
+  uint64_t n_gather;          /*   number of gather launches timed */
+} bk_stats;
+
+BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);
+
+/* ABI self-check for bindings: writes sizeof of bk_config, bk_out_wordcount, bk_out_grep,
+ * bk_out_kmeans, bk_out_partition, bk_out_groupby, bk_out_layout, bk_stats (in that order,
+ * up to n entries) and returns BK_ABI_VERSION. Needs no GPU. */
+BK_API int bk_abi_sizes(uint32_t* sizes, int n);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

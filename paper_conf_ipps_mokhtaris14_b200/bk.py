@@ -1,0 +1,256 @@
+"""Thin ctypes binding of libbk (include/bk.h): argument marshalling only.
+
+Every step of the streaming path runs inside libbk.so (sm_100a kernels + C++ runtime). There
+is no CPU fallback: if the library is missing or no GPU is present the calls raise.
+Names follow the C ABI: bk_create / bk_register_segments / bk_run / bk_destroy.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbk.so")
+
+BK_OK, BK_E_INVAL, BK_E_NOMEM, BK_E_CUDA, BK_E_STATE, BK_E_RANGE, BK_E_CAPACITY, BK_E_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
+BK_K_WORDCOUNT, BK_K_GREP, BK_K_KMEANS, BK_K_PARTITION, BK_K_GROUPBY, BK_K_LAYOUT_DUMP = 1, 2, 3, 4, 5, 100
+BK_GATHER_AUTO, BK_GATHER_ZC, BK_GATHER_CPU, BK_GATHER_DENSE = 0, 1, 2, 3
+BK_FLAG_PROFILE = 1
+GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE}
+
+u32, i32, u64, P = C.c_uint32, C.c_int32, C.c_uint64, C.c_void_p
+
+
+class bk_config(C.Structure):
+    _fields_ = [("struct_size", u32), ("device", i32), ("window_bytes", u64), ("n_slots", u32),
+                ("gather_mode", u32), ("chunk_bytes", u64), ("lanes", u32), ("host_threads", u32),
+                ("record_size", u64), ("flags", u32), ("_reserved", u32)]
+
+
+class bk_out_header(C.Structure):
+    _fields_ = [("struct_size", u32), ("kernel_id", i32)]
+
+
+class bk_out_wordcount(C.Structure):
+    _fields_ = [("h", bk_out_header), ("table_slots", u64), ("cap", u64), ("word_off", P), ("word_len", P),
+                ("word_count", P), ("n_words", u64), ("total_words", u64)]
+
+
+class bk_out_grep(C.Structure):
+    _fields_ = [("h", bk_out_header), ("pattern", P), ("pattern_len", u32), ("_pad", u32), ("first_index", u64),
+                ("cap", u64), ("idx", P), ("n_match", u64)]
+
+
+class bk_out_kmeans(C.Structure):
+    _fields_ = [("h", bk_out_header), ("centroids", P), ("K", u32), ("_pad", u32), ("first_index", u64),
+                ("count", P), ("sum", P), ("chk", u64), ("cid", P)]
+
+
+class bk_out_partition(C.Structure):
+    _fields_ = [("h", bk_out_header), ("n_buckets", u32), ("_pad", u32), ("out_records", P), ("chunk_counts", P),
+                ("chunk_cap", u64), ("n_chunks", u64), ("bucket_count", P)]
+
+
+class bk_out_groupby(C.Structure):
+    _fields_ = [("h", bk_out_header), ("G", u32), ("_pad", u32), ("count", P), ("qty", P), ("amount", P)]
+
+
+class bk_out_layout(C.Structure):
+    _fields_ = [("h", bk_out_header), ("n_ext", u32), ("ext_off", u32 * 8), ("ext_len", u32 * 8), ("chunk", u64),
+                ("stage", P), ("stage_cap", u64), ("lane_first", P), ("lane_nrec", P), ("lane_bytes", P),
+                ("lane_cap", u64), ("stage_size", u64), ("lanes", u32), ("_pad", u32), ("chunk_lo", u64),
+                ("chunk_hi", u64), ("n_chunks", u64)]
+
+
+class bk_stats(C.Structure):
+    _fields_ = [("struct_size", u32), ("gather_mode", u32), ("n_chunks", u64), ("chunk_budget", u64), ("lanes", u32),
+                ("n_slots", u32), ("slot_bytes", u64), ("bytes_accessed", u64), ("bytes_h2d", u64),
+                ("bytes_meta", u64), ("bytes_padding", u64), ("bytes_d2h", u64), ("kernel_launches", u64),
+                ("ms_run", C.c_double), ("ms_register", C.c_double), ("ms_device", C.c_double),
+                ("ms_h2d", C.c_double), ("ms_addrgen", C.c_double), ("ms_gather", C.c_double),
+                ("ms_compute", C.c_double), ("n_gather", u64)]
+
+
+ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,
+               bk_out_layout, bk_stats]
+EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_destroy", "bk_strerror", "bk_last_error",
+           "bk_get_stats", "bk_abi_sizes"]
+
+_lib = None
+
+
+class BkError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        detail = lib().bk_last_error().decode(errors="replace")
+        super().__init__(f"{where}: {lib().bk_strerror(status).decode()} ({status}): {detail}")
+
+
+def lib() -> C.CDLL:
+    """Load libbk.so. Fails loudly when it is missing: there is no fallback path."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} not built; run `make` or __graft_entry__.build()")
+        l = C.CDLL(LIB_PATH)
+        l.bk_create.argtypes = [C.POINTER(bk_config), C.POINTER(P)]
+        l.bk_register_segments.argtypes = [P, P, u64, P, u64]
+        l.bk_run.argtypes = [P, C.c_int, P, P]
+        l.bk_destroy.argtypes = [P]
+        l.bk_strerror.argtypes = [C.c_int]
+        l.bk_strerror.restype = C.c_char_p
+        l.bk_last_error.argtypes = []
+        l.bk_last_error.restype = C.c_char_p
+        l.bk_get_stats.argtypes = [P, C.POINTER(bk_stats)]
+        l.bk_abi_sizes.argtypes = [C.POINTER(u32), C.c_int]
+        for name in ("bk_create", "bk_register_segments", "bk_run", "bk_destroy", "bk_get_stats", "bk_abi_sizes"):
+            getattr(l, name).restype = C.c_int
+        _lib = l
+    return _lib
+
+
+def check(status: int, where: str) -> None:
+    if status != BK_OK:
+        raise BkError(status, where)
+
+
+def abi_sizes() -> list[int]:
+    a = (u32 * 8)()
+    lib().bk_abi_sizes(a, 8)
+    return list(a)
+
+
+def _ptr(a) -> int | None:
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        assert a.flags["C_CONTIGUOUS"]
+        return a.ctypes.data
+    return int(a)
+
+
+def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_mode: int | str = 0,
+              chunk_bytes: int = 0, lanes: int = 0, record_size: int = 0, host_threads: int = 0,
+              profile: bool = False) -> int:
+    if isinstance(gather_mode, str):
+        gather_mode = GATHER_NAMES[gather_mode]
+    cfg = bk_config(C.sizeof(bk_config), device, window_bytes, n_slots, gather_mode, chunk_bytes, lanes,
+                    host_threads, record_size, BK_FLAG_PROFILE if profile else 0, 0)
+    ctx = P()
+    check(lib().bk_create(C.byref(cfg), C.byref(ctx)), "bk_create")
+    return ctx.value
+
+
+def bk_register_segments(ctx: int, data, offsets=None, nbytes: int | None = None, n_records: int | None = None) -> None:
+    """data: uint8 ndarray (or raw host address with nbytes); offsets: uint64 ndarray or None."""
+    nb = nbytes if nbytes is not None else int(data.nbytes)
+    if offsets is not None:
+        assert offsets.dtype == np.uint64
+        n = len(offsets) if n_records is None else n_records
+    else:
+        n = n_records if n_records is not None else 0
+    check(lib().bk_register_segments(ctx, _ptr(data), nb, _ptr(offsets) if offsets is not None and len(offsets) else None, n),
+          "bk_register_segments")
+
+
+def bk_run(ctx: int, kernel_id: int, stream, out) -> None:
+    check(lib().bk_run(ctx, kernel_id, stream, C.byref(out)), "bk_run")
+
+
+def bk_destroy(ctx: int) -> None:
+    check(lib().bk_destroy(ctx), "bk_destroy")
+
+
+def bk_get_stats(ctx: int) -> dict:
+    s = bk_stats()
+    s.struct_size = C.sizeof(bk_stats)
+    check(lib().bk_get_stats(ctx, C.byref(s)), "bk_get_stats")
+    return {k: getattr(s, k) for k, _ in bk_stats._fields_ if k != "struct_size"}
+
+
+def _hdr(cls, kid):
+    o = cls()
+    o.h.struct_size = C.sizeof(cls)
+    o.h.kernel_id = kid
+    return o
+
+
+class Context:
+    """Owning wrapper: one context per GPU; marshals the per-kernel in/out structs."""
+
+    def __init__(self, **cfg):
+        self.ctx = bk_create(**cfg)
+        self._keep = []
+
+    def close(self):
+        if self.ctx:
+            bk_destroy(self.ctx)
+            self.ctx = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def register(self, data, offsets=None, n_records=None, nbytes=None):
+        self._keep = [data, offsets]
+        bk_register_segments(self.ctx, data, offsets, nbytes=nbytes, n_records=n_records)
+
+    def stats(self) -> dict:
+        return bk_get_stats(self.ctx)
+
+    def wordcount(self, cap: int = 1 << 20, table_slots: int = 0, stream=None):
+        o = _hdr(bk_out_wordcount, BK_K_WORDCOUNT)
+        off = np.empty(cap, np.uint64); ln = np.empty(cap, np.uint32); cnt = np.empty(cap, np.uint64)
+        o.table_slots, o.cap, o.word_off, o.word_len, o.word_count = table_slots, cap, _ptr(off), _ptr(ln), _ptr(cnt)
+        bk_run(self.ctx, BK_K_WORDCOUNT, stream, o)
+        n = o.n_words
+        return off[:n], ln[:n], cnt[:n]
+
+    def grep(self, pattern: bytes = b"bigk", first_index: int = 0, cap: int | None = None, stream=None, out=None):
+        o = _hdr(bk_out_grep, BK_K_GREP)
+        pat = np.frombuffer(pattern, np.uint8) if pattern else np.zeros(1, np.uint8)
+        idx = out if out is not None else np.empty(max(cap or 1 << 20, 1), np.uint64)
+        o.pattern, o.pattern_len, o.first_index, o.cap, o.idx = _ptr(pat), len(pattern), first_index, len(idx), _ptr(idx)
+        bk_run(self.ctx, BK_K_GREP, stream, o)
+        return idx[: o.n_match]
+
+    def groupby(self, G: int = 4096, stream=None):
+        o = _hdr(bk_out_groupby, BK_K_GROUPBY)
+        cnt = np.empty(G, np.uint64); qty = np.empty(G, np.uint64); amt = np.empty(G, np.float64)
+        o.G, o.count, o.qty, o.amount = G, _ptr(cnt), _ptr(qty), _ptr(amt)
+        bk_run(self.ctx, BK_K_GROUPBY, stream, o)
+        return cnt, qty, amt
+
+    def kmeans(self, mu: np.ndarray, first_index: int = 0, stream=None):
+        mu = np.ascontiguousarray(mu, np.float32).reshape(-1, 16)
+        K = mu.shape[0]
+        o = _hdr(bk_out_kmeans, BK_K_KMEANS)
+        cnt = np.empty(K, np.uint64); s = np.empty((K, 16), np.float64)
+        o.centroids, o.K, o.first_index, o.count, o.sum, o.cid = _ptr(mu), K, first_index, _ptr(cnt), _ptr(s), None
+        bk_run(self.ctx, BK_K_KMEANS, stream, o)
+        return cnt, s, int(o.chk)
+
+    def layout_dump(self, chunk: int, extents=None, stage_cap: int = 1 << 26, lane_cap: int = 1 << 20, stream=None):
+        o = _hdr(bk_out_layout, BK_K_LAYOUT_DUMP)
+        extents = extents or []
+        o.n_ext = len(extents)
+        for i, (eo, el) in enumerate(extents):
+            o.ext_off[i], o.ext_len[i] = eo, el
+        stage = np.empty(stage_cap, np.uint8)
+        lf = np.empty(lane_cap, np.uint64); ln = np.empty(lane_cap, np.uint64); lb = np.empty(lane_cap, np.uint64)
+        o.chunk, o.stage, o.stage_cap = chunk, _ptr(stage), stage_cap
+        o.lane_first, o.lane_nrec, o.lane_bytes, o.lane_cap = _ptr(lf), _ptr(ln), _ptr(lb), lane_cap
+        bk_run(self.ctx, BK_K_LAYOUT_DUMP, stream, o)
+        L = o.lanes
+        return dict(stage=stage[: o.stage_size].copy(), lane_first=lf[:L].copy(), lane_nrec=ln[:L].copy(),
+                    lane_bytes=lb[:L].copy(), lanes=L, lo=o.chunk_lo, hi=o.chunk_hi, n_chunks=o.n_chunks)

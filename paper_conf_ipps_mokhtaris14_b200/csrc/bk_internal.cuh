@@ -1,0 +1,104 @@
+// bk_internal.cuh — shared device/host definitions of libbk (product path only; never the oracle).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace bk {
+
+constexpr int kWarp = 32;
+constexpr int kMaxExt = 8;
+
+// Lane descriptor written by stage 1 (address generation), 16 B. Lane t owns records
+// [first, first + nrec) of the chunk (each thread a contiguous record range) and
+// nbytes accessed bytes, staged as ceil(nbytes/16) 16-byte words.
+struct LaneDesc {
+  uint64_t first;
+  uint32_t nrec;
+  uint32_t nbytes;
+};
+
+// Access spec of a kernel: the bytes of each record its compute touches.
+struct Access {
+  uint32_t whole;        // 1: every byte of the record
+  uint32_t n_ext;        // else: extents relative to the record start, in access order
+  uint32_t ext_off[kMaxExt];
+  uint32_t ext_len[kMaxExt];
+  uint32_t E;            // sum of ext_len (accessed bytes per record) when !whole
+  uint64_t rec_size;     // fixed record length, 0 = variable (offsets)
+};
+
+// One chunk = records [lo, hi) (whole records only, A3).
+struct Chunk {
+  uint64_t lo, hi;
+  uint64_t base_byte;    // start offset of record lo (relative to the data set)
+  uint64_t end_byte;     // end offset of record hi-1
+  uint32_t L;            // lanes
+  uint32_t ntiles;       // L / 32
+  uint64_t accessed;     // A(lo, hi)
+};
+
+// Device error bits (sticky, read back at the end of bk_run).
+enum : int {
+  kErrStageOverflow = 1,
+  kErrTableFull = 2,
+  kErrKeyRange = 4,
+  kErrWordTooLong = 8,
+  kErrOutOverflow = 16,
+};
+
+__host__ __device__ inline uint64_t mix64(uint64_t x) {
+  x ^= x >> 30; x *= 0xbf58476d1ce4e5b9ULL;
+  x ^= x >> 27; x *= 0x94d049bb133111ebULL;
+  x ^= x >> 31;
+  return x;
+}
+
+// ---- launchers (kernels_stage.cu) ----
+// Stage 1: lane plan + per-tile word counts, then tile bases (exclusive scan of 512*K_w).
+// staged_sum accumulates the staged bytes of every chunk (padding statistics).
+void launch_addrgen(const Chunk& c, const Access& a, const uint64_t* meta, LaneDesc* lanes,
+                    uint32_t* tileK, uint64_t* tile_base, uint64_t stage_cap, int* err,
+                    unsigned long long* staged_sum, cudaStream_t s);
+// Stage 2 (+3 when zero_copy: src is pinned, mapped host memory): gather the accessed bytes
+// into warp tiles. src points at byte c.base_byte of the data set, same alignment mod 16.
+void launch_gather(const Chunk& c, const Access& a, const uint8_t* src, const uint64_t* meta,
+                   const LaneDesc* lanes, const uint64_t* tile_base, uint8_t* stage, uint64_t stage_cap,
+                   int zero_copy, cudaStream_t s);
+
+// ---- compute kernels (kernels_compute.cu) ----
+struct WcEntry {            // 32 B open-addressing slot
+  unsigned long long key1;  // 0 = empty
+  unsigned long long key2;  // 0 = being published
+  unsigned long long count;
+  unsigned long long offlen; // occurrence offset (40 bits) | length (24 bits)
+};
+void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+               const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask,
+               unsigned long long* used, int* err, cudaStream_t s);
+void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,
+                       uint32_t* len, uint64_t* cnt, uint64_t cap, cudaStream_t s);
+
+struct GrepParams {
+  uint8_t pat[32];
+  uint32_t plen;
+  uint64_t first_index;
+  uint64_t cap;
+};
+// three launches: block counts, one-block scan (+ running base), ordered write
+void launch_grep(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* running,
+                 unsigned long long* blkbase, uint64_t* out_idx, int* err, cudaStream_t s);
+
+size_t groupby_smem(uint32_t G);
+void launch_groupby(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                    uint32_t G, unsigned long long* count, unsigned long long* qty, double* amount, int* err,
+                    int grid, cudaStream_t s);
+
+size_t kmeans_smem(uint32_t K);
+void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                   const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
+                   unsigned long long* chk, int grid, cudaStream_t s);
+
+cudaError_t configure_compute_kernels();
+
+}  // namespace bk

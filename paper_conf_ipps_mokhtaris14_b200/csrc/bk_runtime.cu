@@ -1,0 +1,869 @@
+// bk_runtime.cu — host runtime of libbk: context, registration (pin once), chunk planner,
+// ring of N staging slots driven by events across copy / assembly / compute streams, and the
+// C ABI of include/bk.h.
+//
+// Paper mapping (Fig. 3, §III, §IV.C):
+//   * pinned buffers      -> the data set itself is pinned + mapped ONCE at
+//                                        registration; device staging is allocated once at create;
+//   * wait_addrReady / signal_dataReady flags -> cudaEvents per slot;
+//   * "at minimum two" buffer instances, addr-gen n syncs with compute n-3
+//                                     -> a ring of N slots; chunk c reuses slot c % N only after
+//                                        the compute of chunk c - N recorded slot_free;
+//   * CPU assembly thread per block -> replaced by a GPU gather kernel that reads
+//                                        pinned host memory directly (zero-copy) or by a DMA of
+//                                        the whole chunk followed by an HBM re-layout kernel.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/bk.h"
+#include "bk_internal.cuh"
+
+using namespace bk;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return code;
+}
+
+#define BK_CUDA(expr)                                                                        \
+  do {                                                                                       \
+    cudaError_t e_ = (expr);                                                                 \
+    if (e_ != cudaSuccess)                                                                   \
+      return fail(BK_E_CUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+
+constexpr uint64_t kAlign = 256;
+inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+struct Slot {
+  uint8_t* raw = nullptr;       // DENSE: the chunk's record bytes as DMA'd
+  uint8_t* stage = nullptr;     // interleaved warp tiles
+  uint64_t* meta = nullptr;     // offsets slice off[lo .. hi-1]
+  LaneDesc* lanes = nullptr;
+  uint32_t* tileK = nullptr;
+  uint64_t* tile_base = nullptr;
+  cudaEvent_t copied = nullptr, ready = nullptr, freed = nullptr;
+  bool used = false;
+};
+
+// Resident (outside the window) per-kernel device buffers, grown on demand.
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t bytes) {
+    if (bytes <= cap) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e == cudaSuccess) cap = bytes;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+}  // namespace
+
+struct bk_ctx {
+  bk_config cfg{};
+  cudaStream_t s_copy = nullptr, s_asm = nullptr, s_comp = nullptr;
+  cudaEvent_t ev_begin = nullptr, ev_end = nullptr;
+  cudaEvent_t t_begin = nullptr, t_end = nullptr;   // timing events on s_comp (device time of a run)
+  std::vector<cudaEvent_t> prof;                   // BK_FLAG_PROFILE: per chunk x stage begin/end
+  std::vector<int> prof_stage;                     // stage id of each event pair
+  size_t prof_used = 0;
+  uint8_t* window = nullptr;    // the whole streaming working set (cfg.window_bytes)
+  std::vector<Slot> slots;
+  // registration
+  const uint8_t* host = nullptr;
+  uint64_t nbytes = 0;
+  const uint64_t* off = nullptr;
+  uint64_t n = 0;
+  bool pinned_data = false, pinned_off = false, registered = false;
+  const uint8_t* host_dev = nullptr;   // device alias of the mapped data set
+  uint64_t max_rec = 0, min_rec = 0;
+  // device scratch / resident buffers
+  int* d_err = nullptr;
+  unsigned long long* d_ctr = nullptr;  // [0] staged sum, [1] wc used, [2] wc n_out, [3] grep running, [4] kmeans chk
+  DevBuf b_table, b_out1, b_out2, b_out3, b_blk, b_blk2, b_agg1, b_agg2, b_agg3, b_mu;
+  int n_launch = 0;
+  bk_stats st{};
+};
+
+namespace {
+
+bool is_pinned(const void* p) {
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeHost;
+}
+
+uint64_t rec_start(const bk_ctx* c, uint64_t r) {
+  if (!c->off) return r * c->cfg.record_size;
+  return r < c->n ? c->off[r] : c->nbytes;
+}
+
+struct Plan {
+  Access a{};
+  int zero_copy = 0;
+  uint64_t budget = 0;                 // plan bytes per chunk
+  uint32_t L = 0;
+  uint64_t max_acc_rec = 0;            // max accessed bytes of one record
+  uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0;
+  std::vector<uint64_t> bounds;        // chunk record bounds
+};
+
+// plan bytes of records [lo, r): what the budget limits (DESIGN.md §Chunk plan)
+uint64_t plan_bytes(const bk_ctx* c, const Plan& p, uint64_t lo, uint64_t r) {
+  if (!p.zero_copy || p.a.whole) return rec_start(c, r) - rec_start(c, lo);
+  return (r - lo) * p.a.E;
+}
+
+int make_chunks(const bk_ctx* c, Plan& p) {
+  p.bounds.clear();
+  p.bounds.push_back(0);
+  uint64_t lo = 0;
+  const bool fixed_per = !c->off || (p.zero_copy && !p.a.whole);
+  const uint64_t per = !c->off ? (p.zero_copy && !p.a.whole ? p.a.E : c->cfg.record_size) : p.a.E;
+  while (lo < c->n) {
+    uint64_t hi;
+    if (fixed_per) {
+      if (per > p.budget) return fail(BK_E_RANGE, "record (%llu B) exceeds chunk budget (%llu B)",
+                                      (unsigned long long)per, (unsigned long long)p.budget);
+      hi = per ? std::min<uint64_t>(c->n, lo + p.budget / per) : c->n;
+    } else {
+      const uint64_t limit = c->off[lo] + p.budget;
+      if (c->nbytes <= limit) {
+        hi = c->n;
+      } else {
+        // first r > lo with off[r] > limit, then hi = r - 1
+        const uint64_t* it = std::upper_bound(c->off + lo + 1, c->off + c->n, limit);
+        hi = (uint64_t)(it - c->off) - 1;
+      }
+      if (hi == lo) return fail(BK_E_RANGE, "record %llu (%llu B) exceeds chunk budget (%llu B)",
+                                (unsigned long long)lo, (unsigned long long)(rec_start(c, lo + 1) - rec_start(c, lo)),
+                                (unsigned long long)p.budget);
+    }
+    p.bounds.push_back(hi);
+    lo = hi;
+  }
+  return BK_OK;
+}
+
+// Bytes one slot needs for a plan: raw + stage + meta + lanes + tiles (+ alignment).
+uint64_t slot_need(const Plan& p) {
+  const uint64_t ntiles = p.L / 32;
+  return align_up(p.raw_cap, kAlign) + align_up(p.stage_cap, kAlign) + align_up(p.meta_cap * 8, kAlign) +
+         align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign) + align_up(ntiles * 4, kAlign) +
+         align_up((ntiles + 1) * 8, kAlign);
+}
+
+void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) {
+  p.budget = budget;
+  // largest accessed byte count of any chunk of this plan (dense mode plans by whole records,
+  // so with sparse or duplicated extents accessed != planned bytes)
+  uint64_t acc = 0, maxrecs = 0;
+  for (size_t i = 0; i + 1 < p.bounds.size(); ++i) {
+    const uint64_t lo = p.bounds[i], hi = p.bounds[i + 1];
+    const uint64_t a = p.a.whole ? rec_start(c, hi) - rec_start(c, lo) : (hi - lo) * p.a.E;
+    acc = std::max(acc, a);
+    maxrecs = std::max(maxrecs, hi - lo);
+  }
+  uint32_t L = c->cfg.lanes;
+  if (!L) {
+    uint64_t l = (acc + lane_target - 1) / lane_target;
+    l = (l + 31) / 32 * 32;
+    L = (uint32_t)std::max<uint64_t>(32, std::min<uint64_t>(l, 1u << 22));
+  }
+  p.L = L;
+  // staged <= A + L*(max record + 32): DESIGN.md §Stage-1 bound
+  p.stage_cap = align_up(acc + (uint64_t)L * (p.max_acc_rec + 32) + 512, 512);
+  p.raw_cap = p.zero_copy ? 0 : budget + 64;
+  p.meta_cap = c->off ? maxrecs + 1 : 0;
+}
+
+int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p) {
+  p.a = a;
+  int mode = (int)c->cfg.gather_mode;
+  if (mode == BK_GATHER_AUTO) mode = a.whole ? BK_GATHER_DENSE : BK_GATHER_ZC;
+  if (mode == BK_GATHER_CPU) return fail(BK_E_UNSUPPORTED, "BK_GATHER_CPU is not in this build");
+  if (mode != BK_GATHER_ZC && mode != BK_GATHER_DENSE) return fail(BK_E_INVAL, "bad gather_mode %d", mode);
+  p.zero_copy = mode == BK_GATHER_ZC;
+  p.max_acc_rec = a.whole ? c->max_rec : a.E;
+  const uint64_t slot = c->cfg.window_bytes / c->cfg.n_slots;
+  // total plan bytes
+  const uint64_t total = (p.zero_copy && !a.whole) ? c->n * a.E : c->nbytes;
+  uint64_t budget = c->cfg.chunk_bytes;
+  bool autob = budget == 0;
+  if (autob) {
+    // >= ~32 chunks so pipeline fill/drain is a few percent, >= 1 MiB each, and fit a slot
+    budget = std::max<uint64_t>(total / 32, 1ull << 20);
+    budget = std::min<uint64_t>(budget, slot);
+  }
+  for (int iter = 0; iter < 64; ++iter) {
+    p.budget = budget;
+    int rc = make_chunks(c, p);
+    if (rc) return rc;
+    size_plan(c, p, budget, lane_target);
+    if (slot_need(p) <= slot) return BK_OK;
+    if (!autob) break;
+    budget = budget * 3 / 4;
+    if (budget < p.max_acc_rec || budget < 16) break;
+  }
+  return fail(BK_E_NOMEM, "window of %llu B (%u slots) cannot hold a chunk of %llu B (need %llu B per slot)",
+              (unsigned long long)c->cfg.window_bytes, c->cfg.n_slots, (unsigned long long)budget,
+              (unsigned long long)slot_need(p));
+}
+
+void carve(bk_ctx* c, const Plan& p) {
+  const uint64_t slot = c->cfg.window_bytes / c->cfg.n_slots;
+  const uint64_t ntiles = p.L / 32;
+  for (uint32_t i = 0; i < c->cfg.n_slots; ++i) {
+    uint8_t* q = c->window + i * slot;
+    Slot& s = c->slots[i];
+    s.raw = p.raw_cap ? q : nullptr;
+    q += align_up(p.raw_cap, kAlign);
+    s.stage = q;
+    q += align_up(p.stage_cap, kAlign);
+    s.meta = reinterpret_cast<uint64_t*>(q);
+    q += align_up(p.meta_cap * 8, kAlign);
+    s.lanes = reinterpret_cast<LaneDesc*>(q);
+    q += align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign);
+    s.tileK = reinterpret_cast<uint32_t*>(q);
+    q += align_up(ntiles * 4, kAlign);
+    s.tile_base = reinterpret_cast<uint64_t*>(q);
+    s.used = false;
+  }
+}
+
+Chunk chunk_of(const bk_ctx* c, const Plan& p, size_t i) {
+  Chunk ch{};
+  ch.lo = p.bounds[i];
+  ch.hi = p.bounds[i + 1];
+  ch.base_byte = rec_start(c, ch.lo);
+  ch.end_byte = rec_start(c, ch.hi);
+  ch.L = p.L;
+  ch.ntiles = p.L / 32;
+  ch.accessed = p.a.whole ? ch.end_byte - ch.base_byte : (ch.hi - ch.lo) * p.a.E;
+  return ch;
+}
+
+// BK_FLAG_PROFILE: bracket one stage of one chunk with timing events on its stream.
+enum { kStH2D = 0, kStAddrgen = 1, kStGather = 2, kStCompute = 3, kNStages = 4 };
+int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin) {
+  if (!(c->cfg.flags & BK_FLAG_PROFILE)) return BK_OK;
+  if (begin) {
+    if (c->prof_used + 2 > c->prof.size()) {
+      for (int k = 0; k < 64; ++k) {
+        cudaEvent_t e;
+        BK_CUDA(cudaEventCreate(&e));
+        c->prof.push_back(e);
+        if (c->prof.size() % 2 == 0) c->prof_stage.push_back(0);
+      }
+    }
+    c->prof_stage[c->prof_used / 2] = stage;
+    BK_CUDA(cudaEventRecord(c->prof[c->prof_used], s));
+  } else {
+    BK_CUDA(cudaEventRecord(c->prof[c->prof_used + 1], s));
+    c->prof_used += 2;
+  }
+  return BK_OK;
+}
+#define BK_PROF(stage, stream, begin) do { int r_ = prof_mark(c, stage, stream, begin); if (r_) return r_; } while (0)
+
+// Stages 1-3 of chunk i into slot s (on s_copy / s_asm); records s.ready.
+int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
+  const Chunk ch = chunk_of(c, p, i);
+  Access a = p.a;
+  a.rec_size = c->off ? 0 : c->cfg.record_size;
+  if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+  BK_PROF(kStH2D, c->s_copy, true);
+  if (c->off && ch.hi > ch.lo) {
+    BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
+    c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+  }
+  if (p.zero_copy) {
+    BK_PROF(kStH2D, c->s_copy, false);
+    BK_PROF(kStAddrgen, c->s_copy, true);
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_copy);
+    BK_PROF(kStAddrgen, c->s_copy, false);
+    BK_PROF(kStGather, c->s_copy, true);
+    launch_gather(ch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1,
+                  c->s_copy);
+    BK_PROF(kStGather, c->s_copy, false);
+    c->n_launch += 3;
+    c->st.bytes_h2d += ch.accessed;
+  } else {
+    const uint64_t raw_off = ((uintptr_t)(c->host + ch.base_byte)) & 15;
+    const uint64_t bytes = ch.end_byte - ch.base_byte;
+    if (bytes) BK_CUDA(cudaMemcpyAsync(s.raw + raw_off, c->host + ch.base_byte, bytes, cudaMemcpyHostToDevice, c->s_copy));
+    BK_PROF(kStH2D, c->s_copy, false);
+    BK_CUDA(cudaEventRecord(s.copied, c->s_copy));
+    BK_CUDA(cudaStreamWaitEvent(c->s_asm, s.copied, 0));
+    BK_PROF(kStAddrgen, c->s_asm, true);
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
+    BK_PROF(kStAddrgen, c->s_asm, false);
+    BK_PROF(kStGather, c->s_asm, true);
+    launch_gather(ch, a, s.raw + raw_off, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 0, c->s_asm);
+    BK_PROF(kStGather, c->s_asm, false);
+    c->n_launch += 3;
+    c->st.bytes_h2d += bytes;
+  }
+  c->st.bytes_accessed += ch.accessed;
+  BK_CUDA(cudaEventRecord(s.ready, p.zero_copy ? c->s_copy : c->s_asm));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, s.ready, 0));
+  s.used = true;
+  return BK_OK;
+}
+
+void note_plan(bk_ctx* c, const Plan& p) {
+  c->st.gather_mode = p.zero_copy ? BK_GATHER_ZC : BK_GATHER_DENSE;
+  c->st.chunk_budget = p.budget;
+  c->st.lanes = p.L;
+}
+
+int check_err(bk_ctx* c) {
+  int herr = 0;
+  BK_CUDA(cudaMemcpy(&herr, c->d_err, sizeof(int), cudaMemcpyDeviceToHost));
+  if (herr & kErrStageOverflow) return fail(BK_E_RANGE, "staged chunk exceeded its slot (internal bound violated)");
+  if (herr & kErrKeyRange) return fail(BK_E_INVAL, "a group-by key is >= G");
+  if (herr & kErrTableFull) return fail(BK_E_CAPACITY, "word-count hash table full; raise table_slots");
+  if (herr & kErrWordTooLong) return fail(BK_E_RANGE, "a word is longer than 2^24 bytes or offset >= 2^40");
+  return BK_OK;
+}
+
+// ---- the pipeline driver: stage chunk i+?, compute chunk i, with N slots in flight ----
+template <class Compute>
+int pipeline(bk_ctx* c, const Plan& p, Compute&& compute) {
+  const size_t C = p.bounds.size() - 1;
+  c->st.n_chunks = C;
+  note_plan(c, p);
+  for (size_t i = 0; i < C; ++i) {
+    Slot& s = c->slots[i % c->cfg.n_slots];
+    int rc = stage_chunk(c, p, i, s);
+    if (rc) return rc;
+    BK_PROF(kStCompute, c->s_comp, true);
+    rc = compute(chunk_of(c, p, i), s);
+    if (rc) return rc;
+    BK_PROF(kStCompute, c->s_comp, false);
+    BK_CUDA(cudaEventRecord(s.freed, c->s_comp));
+  }
+  return BK_OK;
+}
+
+Access whole_access() {
+  Access a{};
+  a.whole = 1;
+  return a;
+}
+Access field_access(uint32_t off, uint32_t len) {
+  Access a{};
+  a.whole = 0;
+  a.n_ext = 1;
+  a.ext_off[0] = off;
+  a.ext_len[0] = len;
+  a.E = len;
+  return a;
+}
+
+int begin_run(bk_ctx* c, void* stream) {
+  BK_CUDA(cudaSetDevice(c->cfg.device));
+  BK_CUDA(cudaMemsetAsync(c->d_err, 0, sizeof(int), c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->d_ctr, 0, 8 * sizeof(unsigned long long), c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_begin, 0));
+  BK_CUDA(cudaEventRecord(c->t_begin, c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_begin, c->s_comp));
+  BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->ev_begin, 0));
+  BK_CUDA(cudaStreamWaitEvent(c->s_asm, c->ev_begin, 0));
+  for (auto& s : c->slots) s.used = false;
+  c->n_launch = 0;
+  c->prof_used = 0;
+  c->st.bytes_accessed = c->st.bytes_h2d = c->st.bytes_meta = c->st.bytes_padding = c->st.bytes_d2h = 0;
+  return BK_OK;
+}
+
+int end_run(bk_ctx* c, void* stream) {
+  BK_CUDA(cudaEventRecord(c->t_end, c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_end, c->s_comp));
+  BK_CUDA(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_end, 0));
+  BK_CUDA(cudaStreamSynchronize(c->s_comp));
+  unsigned long long staged = 0;
+  BK_CUDA(cudaMemcpy(&staged, c->d_ctr + 0, 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_padding = staged >= c->st.bytes_accessed ? staged - c->st.bytes_accessed : 0;
+  float ms = 0;
+  BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
+  c->st.ms_device = ms;
+  double acc[kNStages] = {0, 0, 0, 0};
+  uint64_t cnt[kNStages] = {0, 0, 0, 0};
+  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
+    float e = 0;
+    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
+    acc[c->prof_stage[i / 2]] += e;
+    cnt[c->prof_stage[i / 2]] += 1;
+  }
+  c->st.ms_h2d = acc[kStH2D];
+  c->st.ms_addrgen = acc[kStAddrgen];
+  c->st.ms_gather = acc[kStGather];
+  c->st.ms_compute = acc[kStCompute];
+  c->st.n_gather = cnt[kStGather];
+  return check_err(c);
+}
+
+// ------------------------------------------------------------------ kernels
+int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
+  uint64_t slots = o->table_slots ? o->table_slots : (1ull << 20);
+  if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
+  Plan p;
+  int rc = plan_run(c, whole_access(), 512, p);
+  if (rc) return rc;
+  carve(c, p);
+  BK_CUDA(c->b_table.ensure(slots * sizeof(WcEntry)));
+  const uint64_t ocap = std::min<uint64_t>(o->cap, slots);
+  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(ocap, 1) * 4));
+  BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  if ((rc = begin_run(c, stream))) return rc;
+  BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
+  WcEntry* table = (WcEntry*)c->b_table.p;
+  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+    launch_wc(ch, s.stage, s.lanes, s.tile_base, s.meta, c->off ? 0 : c->cfg.record_size, table, slots - 1,
+              c->d_ctr + 1, c->d_err, c->s_comp);
+    c->n_launch += 1;
+    return BK_OK;
+  });
+  if (rc) return rc;
+  launch_wc_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
+                    (uint64_t*)c->b_out3.p, ocap, c->s_comp);
+  c->n_launch += 1;
+  if ((rc = end_run(c, stream))) return rc;
+  unsigned long long nw = 0;
+  BK_CUDA(cudaMemcpy(&nw, c->d_ctr + 2, 8, cudaMemcpyDeviceToHost));
+  o->n_words = nw;
+  if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
+  if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
+                                  (unsigned long long)slots);
+  if (nw) {
+    BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->word_count, c->b_out3.p, nw * 8, cudaMemcpyDeviceToHost));
+  }
+  uint64_t tot = 0;
+  for (uint64_t i = 0; i < nw; ++i) tot += o->word_count[i];
+  o->total_words = tot;
+  c->st.bytes_d2h = nw * 20;
+  return BK_OK;
+}
+
+int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
+  if (o->pattern_len > 32) return fail(BK_E_INVAL, "pattern longer than 32 bytes");
+  if (o->pattern_len && !o->pattern) return fail(BK_E_INVAL, "NULL pattern");
+  if (c->min_rec < 48) return fail(BK_E_INVAL, "grep needs records of >= 48 bytes (key at +16..+48)");
+  Plan p;
+  int rc = plan_run(c, field_access(16, 32), 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  const uint32_t nblk = (p.L + 255) / 256;
+  const uint64_t cap = std::min<uint64_t>(o->cap, c->n);
+  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(cap, 1) * 8));
+  BK_CUDA(c->b_blk.ensure((uint64_t)nblk * 4));
+  BK_CUDA(c->b_blk2.ensure((uint64_t)nblk * 8));
+  GrepParams gp{};
+  if (o->pattern_len) memcpy(gp.pat, o->pattern, o->pattern_len);
+  gp.plen = o->pattern_len;
+  gp.first_index = o->first_index;
+  gp.cap = cap;
+  if ((rc = begin_run(c, stream))) return rc;
+  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+    launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p, c->d_ctr + 3,
+                (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, c->s_comp);
+    c->n_launch += 3;
+    return BK_OK;
+  });
+  if (rc) return rc;
+  if ((rc = end_run(c, stream))) return rc;
+  unsigned long long m = 0;
+  BK_CUDA(cudaMemcpy(&m, c->d_ctr + 3, 8, cudaMemcpyDeviceToHost));
+  o->n_match = m;
+  if (m > o->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)o->cap);
+  if (m) BK_CUDA(cudaMemcpy(o->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_d2h = m * 8;
+  return BK_OK;
+}
+
+int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
+  const uint32_t G = o->G;
+  if (G == 0 || G > 8192) return fail(BK_E_INVAL, "G must be in 1..8192");
+  if (c->min_rec < 16) return fail(BK_E_INVAL, "group-by records must be >= 16 bytes");
+  const bool dense16 = !c->off && c->cfg.record_size == 16;
+  Plan p;
+  int rc = plan_run(c, dense16 ? whole_access() : field_access(0, 16), 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  BK_CUDA(c->b_agg1.ensure((uint64_t)G * 8));
+  BK_CUDA(c->b_agg2.ensure((uint64_t)G * 8));
+  BK_CUDA(c->b_agg3.ensure((uint64_t)G * 8));
+  int dev_sms = 148, per_sm = 1;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  per_sm = std::max<int>(1, (int)((200 * 1024) / std::max<size_t>(groupby_smem(G), 1)));
+  per_sm = std::min(per_sm, 4);
+  if ((rc = begin_run(c, stream))) return rc;
+  BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)G * 8, c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)G * 8, c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)G * 8, c->s_comp));
+  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * per_sm));
+  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+    launch_groupby(ch, s.stage, s.lanes, s.tile_base, G, (unsigned long long*)c->b_agg1.p,
+                   (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, c->s_comp);
+    c->n_launch += 1;
+    return BK_OK;
+  });
+  if (rc) return rc;
+  if ((rc = end_run(c, stream))) return rc;
+  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->qty, c->b_agg2.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->amount, c->b_agg3.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_d2h = (uint64_t)G * 24;
+  return BK_OK;
+}
+
+int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
+  const uint32_t K = o->K;
+  if (K == 0 || K > 256 || !o->centroids) return fail(BK_E_INVAL, "K must be in 1..256 with centroids");
+  if (o->cid) return fail(BK_E_UNSUPPORTED, "cid write-back is not in this build");
+  if (c->min_rec < 64) return fail(BK_E_INVAL, "k-means records must hold 16 fp32 (>= 64 bytes)");
+  const bool dense64 = !c->off && c->cfg.record_size == 64;
+  Plan p;
+  int rc = plan_run(c, dense64 ? whole_access() : field_access(0, 64), 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  BK_CUDA(c->b_mu.ensure((uint64_t)K * 64));
+  BK_CUDA(c->b_agg1.ensure((uint64_t)K * 8));
+  BK_CUDA(c->b_agg3.ensure((uint64_t)K * 16 * 8));
+  int dev_sms = 148;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  if ((rc = begin_run(c, stream))) return rc;
+  BK_CUDA(cudaMemcpyAsync(c->b_mu.p, o->centroids, (uint64_t)K * 64, cudaMemcpyHostToDevice, c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
+  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
+  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+    launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
+                  (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4, grid, c->s_comp);
+    c->n_launch += 1;
+    return BK_OK;
+  });
+  if (rc) return rc;
+  if ((rc = end_run(c, stream))) return rc;
+  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->sum, c->b_agg3.p, (uint64_t)K * 128, cudaMemcpyDeviceToHost));
+  unsigned long long chk = 0;
+  BK_CUDA(cudaMemcpy(&chk, c->d_ctr + 4, 8, cudaMemcpyDeviceToHost));
+  o->chk = chk;
+  c->st.bytes_d2h = (uint64_t)K * 136;
+  return BK_OK;
+}
+
+int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
+  Access a{};
+  if (o->n_ext == 0) {
+    a = whole_access();
+  } else {
+    if (o->n_ext > (uint32_t)kMaxExt) return fail(BK_E_INVAL, "n_ext > %d", kMaxExt);
+    a.whole = 0;
+    a.n_ext = o->n_ext;
+    for (uint32_t e = 0; e < o->n_ext; ++e) {
+      a.ext_off[e] = o->ext_off[e];
+      a.ext_len[e] = o->ext_len[e];
+      a.E += o->ext_len[e];
+      if ((uint64_t)o->ext_off[e] + o->ext_len[e] > c->min_rec)
+        return fail(BK_E_INVAL, "extent %u exceeds the shortest record", e);
+    }
+  }
+  Plan p;
+  int rc = plan_run(c, a, 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  o->n_chunks = p.bounds.size() - 1;
+  o->lanes = p.L;
+  if (o->chunk >= o->n_chunks) return fail(BK_E_INVAL, "chunk %llu >= %llu chunks", (unsigned long long)o->chunk,
+                                           (unsigned long long)o->n_chunks);
+  if ((rc = begin_run(c, stream))) return rc;
+  Slot& s = c->slots[0];
+  if ((rc = stage_chunk(c, p, o->chunk, s))) return rc;
+  const Chunk ch = chunk_of(c, p, o->chunk);
+  o->chunk_lo = ch.lo;
+  o->chunk_hi = ch.hi;
+  if ((rc = end_run(c, stream))) return rc;
+  uint64_t size = 0;
+  BK_CUDA(cudaMemcpy(&size, s.tile_base + ch.ntiles, 8, cudaMemcpyDeviceToHost));
+  o->stage_size = size;
+  if (size > o->stage_cap || p.L > o->lane_cap) return fail(BK_E_CAPACITY, "stage %llu / lanes %u", size, p.L);
+  BK_CUDA(cudaMemcpy(o->stage, s.stage, size, cudaMemcpyDeviceToHost));
+  std::vector<LaneDesc> ld(p.L);
+  BK_CUDA(cudaMemcpy(ld.data(), s.lanes, (uint64_t)p.L * sizeof(LaneDesc), cudaMemcpyDeviceToHost));
+  for (uint32_t t = 0; t < p.L; ++t) {
+    o->lane_first[t] = ld[t].first;
+    o->lane_nrec[t] = ld[t].nrec;
+    o->lane_bytes[t] = ld[t].nbytes;
+  }
+  return BK_OK;
+}
+
+void unregister(bk_ctx* c) {
+  if (c->pinned_data && c->host) cudaHostUnregister((void*)c->host);
+  if (c->pinned_off && c->off) cudaHostUnregister((void*)c->off);
+  c->pinned_data = c->pinned_off = c->registered = false;
+  c->host = nullptr;
+  c->off = nullptr;
+  c->host_dev = nullptr;
+  c->n = c->nbytes = 0;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* bk_strerror(int status) {
+  switch (status) {
+    case BK_OK: return "ok";
+    case BK_E_INVAL: return "invalid argument";
+    case BK_E_NOMEM: return "out of memory / window too small";
+    case BK_E_CUDA: return "CUDA error";
+    case BK_E_STATE: return "bad call order";
+    case BK_E_RANGE: return "record exceeds chunk budget";
+    case BK_E_CAPACITY: return "output capacity too small";
+    case BK_E_UNSUPPORTED: return "unsupported";
+    default: return "unknown status";
+  }
+}
+
+const char* bk_last_error(void) { return g_last_error.c_str(); }
+
+int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
+  if (!cfg || !out_ctx) return fail(BK_E_INVAL, "NULL argument");
+  if (cfg->struct_size != sizeof(bk_config)) return fail(BK_E_INVAL, "bk_config size %u != %zu", cfg->struct_size, sizeof(bk_config));
+  *out_ctx = nullptr;
+  bk_ctx* c = new (std::nothrow) bk_ctx();
+  if (!c) return fail(BK_E_NOMEM, "host allocation");
+  c->cfg = *cfg;
+  if (!c->cfg.window_bytes) c->cfg.window_bytes = 2ull << 30;
+  if (!c->cfg.n_slots) c->cfg.n_slots = 4;
+  if (c->cfg.n_slots < 2 || c->cfg.n_slots > 64) { delete c; return fail(BK_E_INVAL, "n_slots must be in 2..64"); }
+  if (c->cfg.lanes % 32) { delete c; return fail(BK_E_INVAL, "lanes must be a multiple of 32"); }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || c->cfg.device < 0 || c->cfg.device >= ndev) {
+    cudaGetLastError();
+    delete c;
+    return fail(BK_E_CUDA, "no CUDA device %d", cfg->device);
+  }
+  c->cfg.window_bytes = c->cfg.window_bytes / (c->cfg.n_slots * kAlign) * (c->cfg.n_slots * kAlign);
+  auto cleanup = [&](int rc) { bk_destroy(c); return rc; };
+  if (cudaSetDevice(c->cfg.device) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaSetDevice"));
+  if (configure_compute_kernels() != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
+  if (cudaStreamCreateWithFlags(&c->s_copy, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->s_asm, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->s_comp, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_begin, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_end, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreate(&c->t_begin) != cudaSuccess || cudaEventCreate(&c->t_end) != cudaSuccess)
+    return cleanup(fail(BK_E_CUDA, "stream/event creation"));
+  if (cudaMalloc(&c->window, c->cfg.window_bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return cleanup(fail(BK_E_NOMEM, "cudaMalloc window %llu B", (unsigned long long)c->cfg.window_bytes));
+  }
+  if (cudaMalloc(&c->d_err, 256) != cudaSuccess || cudaMalloc(&c->d_ctr, 8 * sizeof(unsigned long long)) != cudaSuccess)
+    return cleanup(fail(BK_E_NOMEM, "cudaMalloc scratch"));
+  c->slots.resize(c->cfg.n_slots);
+  for (auto& s : c->slots) {
+    if (cudaEventCreateWithFlags(&s.copied, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&s.ready, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&s.freed, cudaEventDisableTiming) != cudaSuccess)
+      return cleanup(fail(BK_E_CUDA, "slot events"));
+  }
+  c->st.struct_size = sizeof(bk_stats);
+  c->st.n_slots = c->cfg.n_slots;
+  c->st.slot_bytes = c->cfg.window_bytes / c->cfg.n_slots;
+  *out_ctx = c;
+  return BK_OK;
+}
+
+int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const uint64_t* off, uint64_t n) {
+  if (!c) return fail(BK_E_INVAL, "NULL ctx");
+  if (!host_ptr && nbytes) return fail(BK_E_INVAL, "NULL host_ptr");
+  const auto t0 = std::chrono::steady_clock::now();
+  if (cudaSetDevice(c->cfg.device) != cudaSuccess) return fail(BK_E_CUDA, "cudaSetDevice");
+  unregister(c);
+  uint64_t maxr = 0, minr = ~0ull;
+  if (off) {
+    if (n && off[0] != 0) return fail(BK_E_INVAL, "record_offsets[0] != 0");
+    for (uint64_t i = 0; i < n; ++i) {
+      const uint64_t e = i + 1 < n ? off[i + 1] : nbytes;
+      if (e < off[i] || e > nbytes) return fail(BK_E_INVAL, "record_offsets not non-decreasing / > nbytes at %llu", (unsigned long long)i);
+      maxr = std::max(maxr, e - off[i]);
+      minr = std::min(minr, e - off[i]);
+    }
+    if (!n && nbytes) return fail(BK_E_INVAL, "bytes without records");
+  } else if (n == 0 && nbytes == 0) {
+    maxr = minr = 0;  // empty data set
+  } else {
+    const uint64_t rs = c->cfg.record_size;
+    if (!rs) return fail(BK_E_INVAL, "record_offsets == NULL needs cfg.record_size");
+    if (nbytes % rs) return fail(BK_E_INVAL, "nbytes %% record_size != 0");
+    if (n != nbytes / rs) return fail(BK_E_INVAL, "n_records != nbytes / record_size");
+    maxr = minr = rs;
+  }
+  if (!n) minr = 0;
+  c->max_rec = maxr;
+  c->min_rec = n ? minr : ~0ull;
+  if (nbytes) {
+    if (is_pinned(host_ptr)) {
+      c->pinned_data = false;
+    } else {
+      cudaError_t e = cudaHostRegister((void*)host_ptr, nbytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+      if (e != cudaSuccess) return fail(BK_E_CUDA, "cudaHostRegister(data, %llu): %s", (unsigned long long)nbytes, cudaGetErrorString(e));
+      c->pinned_data = true;
+    }
+    void* dptr = nullptr;
+    cudaError_t e = cudaHostGetDevicePointer(&dptr, (void*)host_ptr, 0);
+    if (e != cudaSuccess) {
+      if (c->pinned_data) cudaHostUnregister((void*)host_ptr);
+      c->pinned_data = false;
+      return fail(BK_E_CUDA, "cudaHostGetDevicePointer (memory pinned without cudaHostRegisterMapped?): %s", cudaGetErrorString(e));
+    }
+    c->host_dev = (const uint8_t*)dptr;
+  }
+  if (off && n) {
+    if (is_pinned(off)) {
+      c->pinned_off = false;
+    } else {
+      cudaError_t e = cudaHostRegister((void*)off, n * 8, cudaHostRegisterMapped | cudaHostRegisterPortable);
+      if (e != cudaSuccess) return fail(BK_E_CUDA, "cudaHostRegister(offsets): %s", cudaGetErrorString(e));
+      c->pinned_off = true;
+    }
+  }
+  c->host = (const uint8_t*)host_ptr;
+  c->nbytes = nbytes;
+  c->off = off;
+  c->n = n;
+  c->registered = true;
+  c->st.ms_register = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return BK_OK;
+}
+
+int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
+  if (!c || !out) return fail(BK_E_INVAL, "NULL argument");
+  if (!c->registered) return fail(BK_E_STATE, "bk_run before bk_register_segments");
+  const bk_out_header* h = (const bk_out_header*)out;
+  if (h->kernel_id != kernel_id) return fail(BK_E_INVAL, "out->kernel_id %d != %d", h->kernel_id, kernel_id);
+  const auto t0 = std::chrono::steady_clock::now();
+  int rc;
+  switch (kernel_id) {
+    case BK_K_WORDCOUNT:
+      if (h->struct_size != sizeof(bk_out_wordcount)) return fail(BK_E_INVAL, "bk_out_wordcount size");
+      rc = run_wordcount(c, (bk_out_wordcount*)out, stream);
+      break;
+    case BK_K_GREP:
+      if (h->struct_size != sizeof(bk_out_grep)) return fail(BK_E_INVAL, "bk_out_grep size");
+      rc = run_grep(c, (bk_out_grep*)out, stream);
+      break;
+    case BK_K_KMEANS:
+      if (h->struct_size != sizeof(bk_out_kmeans)) return fail(BK_E_INVAL, "bk_out_kmeans size");
+      rc = run_kmeans(c, (bk_out_kmeans*)out, stream);
+      break;
+    case BK_K_GROUPBY:
+      if (h->struct_size != sizeof(bk_out_groupby)) return fail(BK_E_INVAL, "bk_out_groupby size");
+      rc = run_groupby(c, (bk_out_groupby*)out, stream);
+      break;
+    case BK_K_LAYOUT_DUMP:
+      if (h->struct_size != sizeof(bk_out_layout)) return fail(BK_E_INVAL, "bk_out_layout size");
+      rc = run_layout(c, (bk_out_layout*)out, stream);
+      break;
+    case BK_K_PARTITION:
+      return fail(BK_E_UNSUPPORTED, "partition is not in this build yet");
+    default:
+      return fail(BK_E_UNSUPPORTED, "unknown kernel_id %d", kernel_id);
+  }
+  if (rc) {
+    // leave the context usable: drain whatever was queued
+    cudaStreamSynchronize(c->s_copy);
+    cudaStreamSynchronize(c->s_asm);
+    cudaStreamSynchronize(c->s_comp);
+    cudaGetLastError();
+    return rc;
+  }
+  c->st.kernel_launches = (uint64_t)c->n_launch;
+  c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return BK_OK;
+}
+
+int bk_get_stats(const bk_ctx* c, bk_stats* s) {
+  if (!c || !s) return fail(BK_E_INVAL, "NULL argument");
+  if (s->struct_size != sizeof(bk_stats)) return fail(BK_E_INVAL, "bk_stats size");
+  *s = c->st;
+  return BK_OK;
+}
+
+int bk_abi_sizes(uint32_t* sizes, int n) {
+  const uint32_t v[8] = {sizeof(bk_config), sizeof(bk_out_wordcount), sizeof(bk_out_grep), sizeof(bk_out_kmeans),
+                         sizeof(bk_out_partition), sizeof(bk_out_groupby), sizeof(bk_out_layout), sizeof(bk_stats)};
+  for (int i = 0; i < n && i < 8; ++i) sizes[i] = v[i];
+  return BK_ABI_VERSION;
+}
+
+int bk_destroy(bk_ctx* c) {
+  if (!c) return BK_OK;
+  cudaSetDevice(c->cfg.device);
+  if (c->s_comp) cudaStreamSynchronize(c->s_comp);
+  if (c->s_copy) cudaStreamSynchronize(c->s_copy);
+  if (c->s_asm) cudaStreamSynchronize(c->s_asm);
+  unregister(c);
+  for (auto& s : c->slots) {
+    if (s.copied) cudaEventDestroy(s.copied);
+    if (s.ready) cudaEventDestroy(s.ready);
+    if (s.freed) cudaEventDestroy(s.freed);
+  }
+  for (DevBuf* b : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_agg1, &c->b_agg2,
+                    &c->b_agg3, &c->b_mu})
+    b->release();
+  if (c->window) cudaFree(c->window);
+  if (c->d_err) cudaFree(c->d_err);
+  if (c->d_ctr) cudaFree(c->d_ctr);
+  if (c->ev_begin) cudaEventDestroy(c->ev_begin);
+  if (c->ev_end) cudaEventDestroy(c->ev_end);
+  if (c->t_begin) cudaEventDestroy(c->t_begin);
+  if (c->t_end) cudaEventDestroy(c->t_end);
+  for (cudaEvent_t e : c->prof) cudaEventDestroy(e);
+  if (c->s_copy) cudaStreamDestroy(c->s_copy);
+  if (c->s_asm) cudaStreamDestroy(c->s_asm);
+  if (c->s_comp) cudaStreamDestroy(c->s_comp);
+  cudaGetLastError();
+  delete c;
+  return BK_OK;
+}
+
+}  // extern "C"

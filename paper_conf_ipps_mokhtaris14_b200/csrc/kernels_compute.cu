@@ -1,0 +1,446 @@
+// kernels_compute.cu — pipeline stage 4 (Fig. 3):
+// the compute kernels read their lane's words from the staged warp tiles (one coalesced
+// 512-B access per warp per word, the point of the interleaved layout) and
+// reduce with warp-level aggregation and block-level shared-memory tables before touching
+// global memory (north_star: warp shuffles + block-level atomics).
+#include "bk_internal.cuh"
+
+namespace bk {
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+__device__ __forceinline__ uint4 lane_word(const uint8_t* tile, uint32_t k, int lane) {
+  return __ldcs(reinterpret_cast<const uint4*>(tile + ((size_t)k * 32 + lane) * 16));
+}
+
+// ------------------------------------------------------------------------------------------
+// C1 word count (centralized hash table).
+// A word is a maximal run of non-delimiter bytes inside one record (reading A10/A19).
+// Identity = (two independent 64-bit hashes, length); the table stores one occurrence offset
+// so the host can recover the bytes.
+
+__device__ __forceinline__ bool is_delim(uint32_t ch) { return ch == 0x20 || (ch - 0x09u) <= 4u; }
+
+__device__ void wc_insert(WcEntry* table, uint64_t mask, unsigned long long key1, unsigned long long key2,
+                          unsigned long long offlen, unsigned long long cnt, unsigned long long* used, int* err) {
+  uint64_t slot = key1 & mask;
+  for (uint64_t probe = 0; probe <= mask; ++probe, slot = (slot + 1) & mask) {
+    WcEntry* e = &table[slot];
+    unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(&e->key1);
+    if (k == 0) {
+      k = atomicCAS(&e->key1, 0ull, key1);
+      if (k == 0) {  // claimed: publish occurrence, then key2
+        e->offlen = offlen;
+        __threadfence();
+        atomicExch(&e->key2, key2);
+        atomicAdd(&e->count, cnt);
+        atomicAdd(used, 1ull);
+        return;
+      }
+    }
+    if (k == key1) {
+      unsigned long long k2;
+      while ((k2 = *reinterpret_cast<volatile unsigned long long*>(&e->key2)) == 0) {
+      }
+      if (k2 == key2) {
+        atomicAdd(&e->count, cnt);
+        return;
+      }
+    }
+  }
+  atomicOr(err, kErrTableFull);
+}
+
+__device__ __forceinline__ void wc_emit(WcEntry* table, uint64_t mask, uint64_t h1, uint64_t h2, uint32_t len,
+                                        uint64_t occ, unsigned long long* used, int* err) {
+  const unsigned long long key1 = mix64(h1 ^ ((uint64_t)len * 0x9E3779B97F4A7C15ull)) | 1ull;
+  const unsigned long long key2 = mix64(h2 + len) | 1ull;
+  if (len >= (1u << 24) || occ >= (1ull << 40)) atomicOr(err, kErrWordTooLong);
+  const unsigned long long offlen = (occ << 24) | len;
+  const unsigned act = __activemask();
+  const unsigned m = __match_any_sync(act, key1) & __match_any_sync(act, key2);
+  const int lane = threadIdx.x & 31;
+  if (lane == __ffs(m) - 1) wc_insert(table, mask, key1, key2, offlen, __popc(m), used, err);
+}
+
+__global__ void __launch_bounds__(256) k_wc(Chunk c, const uint8_t* __restrict__ stage,
+                                            const LaneDesc* __restrict__ lanes,
+                                            const uint64_t* __restrict__ tile_base,
+                                            const uint64_t* __restrict__ meta, uint64_t rec_size,
+                                            WcEntry* table, uint64_t mask, unsigned long long* used, int* err) {
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= c.L) return;
+  const int lane = t & 31;
+  const LaneDesc d = lanes[t];
+  const uint8_t* tile = stage + tile_base[t >> 5];
+  auto rstart = [&](uint64_t r) -> uint64_t {
+    if (rec_size) return r * rec_size;
+    return r == c.hi ? c.end_byte : meta[r - c.lo];
+  };
+  const uint64_t lane_start = rstart(d.first);
+  const uint64_t rend = d.first + d.nrec;
+  uint64_t r = d.first + 1;
+  uint64_t next_b = r < rend ? rstart(r) - lane_start : ~0ull;
+  bool in_word = false;
+  uint64_t h1 = 0, h2 = 0, wstart = 0;
+  uint32_t wlen = 0;
+  const uint32_t W = (d.nbytes + 15) >> 4;
+  for (uint32_t k = 0; k < W; ++k) {
+    const uint4 v = lane_word(tile, k, lane);
+    const uint32_t wd[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const uint64_t pos = (uint64_t)k * 16 + q;
+      if (pos >= d.nbytes) break;
+      while (pos == next_b) {  // record boundary (several if records are empty)
+        if (in_word) { wc_emit(table, mask, h1, h2, wlen, lane_start + wstart, used, err); in_word = false; }
+        ++r;
+        next_b = r < rend ? rstart(r) - lane_start : ~0ull;
+      }
+      const uint32_t ch = (wd[q >> 2] >> (8 * (q & 3))) & 0xff;
+      if (is_delim(ch)) {
+        if (in_word) { wc_emit(table, mask, h1, h2, wlen, lane_start + wstart, used, err); in_word = false; }
+      } else {
+        if (!in_word) { in_word = true; wstart = pos; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
+        h1 = (h1 ^ ch) * 0x100000001b3ull;
+        h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
+        h2 ^= h2 >> 29;
+        ++wlen;
+      }
+    }
+  }
+  if (in_word) wc_emit(table, mask, h1, h2, wlen, lane_start + wstart, used, err);
+}
+
+__global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, unsigned long long* n_out,
+                             uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t cap) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < slots; i += (uint64_t)gridDim.x * blockDim.x) {
+    const WcEntry e = table[i];
+    if (e.key1 == 0) continue;
+    const unsigned long long p = atomicAdd(n_out, 1ull);
+    if (p < cap) {
+      off[p] = e.offlen >> 24;
+      len[p] = (uint32_t)(e.offlen & 0xffffff);
+      cnt[p] = e.count;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// C2 grep (MCA analogue): key = first strnlen(32) bytes of the record's 32-byte key
+// field (staged as words 2j, 2j+1 of the lane); match iff the pattern is a substring. Output
+// indices are ascending: per chunk, block counts -> one-block scan (+ running base) -> write.
+
+struct Key32 { uint64_t q[8]; };  // q[4..7] = 0: windows past byte 31 read zeros
+
+__device__ __forceinline__ uint64_t window8(const Key32& k, int x) {  // bytes [x, x+8), x constant
+  const int i = x >> 3, s = (x & 7) * 8;
+  if (s == 0) return k.q[i];
+  return (k.q[i] >> s) | (k.q[i + 1] << (64 - s));
+}
+
+__device__ __forceinline__ uint32_t strnlen32(const Key32& k) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint64_t v = k.q[i];
+    const uint64_t z = (v - 0x0101010101010101ull) & ~v & 0x8080808080808080ull;  // first zero byte
+    if (z) return 8 * i + (__ffsll((long long)z) - 1) / 8;
+  }
+  return 32;
+}
+
+__device__ __forceinline__ bool grep_match(const Key32& k, const GrepParams& p, const uint64_t* pw,
+                                           const uint64_t* pm) {
+  if (p.plen == 0) return true;
+  const int kl = (int)strnlen32(k);
+  const int plen = (int)p.plen;
+  bool hit = false;
+#pragma unroll
+  for (int x = 0; x < 32; ++x) {
+    bool ok = x + plen <= kl && (window8(k, x) & pm[0]) == pw[0];
+    if (plen > 8) ok = ok && (window8(k, x + 8) & pm[1]) == pw[1];
+    if (plen > 16) ok = ok && (window8(k, x + 16) & pm[2]) == pw[2];
+    if (plen > 24) ok = ok && (window8(k, x + 24) & pm[3]) == pw[3];
+    hit = hit || ok;
+  }
+  return hit;
+}
+
+__device__ __forceinline__ Key32 load_key(const uint8_t* tile, uint32_t j, int lane) {
+  const uint4 a = lane_word(tile, 2 * j, lane);
+  const uint4 b = lane_word(tile, 2 * j + 1, lane);
+  Key32 k;
+  k.q[0] = (uint64_t)a.x | ((uint64_t)a.y << 32);
+  k.q[1] = (uint64_t)a.z | ((uint64_t)a.w << 32);
+  k.q[2] = (uint64_t)b.x | ((uint64_t)b.y << 32);
+  k.q[3] = (uint64_t)b.z | ((uint64_t)b.w << 32);
+  k.q[4] = k.q[5] = k.q[6] = k.q[7] = 0;
+  return k;
+}
+
+__device__ __forceinline__ void pattern_words(const GrepParams& p, uint64_t* pw, uint64_t* pm) {
+#pragma unroll
+  for (int b = 0; b < 4; ++b) {
+    uint64_t w = 0, m = 0;
+    for (int i = 0; i < 8; ++i) {
+      const int x = 8 * b + i;
+      if (x < (int)p.plen) { w |= (uint64_t)p.pat[x] << (8 * i); m |= 0xffull << (8 * i); }
+    }
+    pw[b] = w;
+    pm[b] = m;
+  }
+}
+
+__device__ __forceinline__ uint32_t block_sum(uint32_t v, uint32_t* sh) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  v = __reduce_add_sync(kFull, v);
+  if (lane == 0) sh[wid] = v;
+  __syncthreads();
+  uint32_t s = 0;
+  if (threadIdx.x == 0)
+    for (int i = 0; i < (int)(blockDim.x >> 5); ++i) s += sh[i];
+  return s;
+}
+
+__global__ void __launch_bounds__(256) k_grep_count(Chunk c, const uint8_t* __restrict__ stage,
+                                                    const LaneDesc* __restrict__ lanes,
+                                                    const uint64_t* __restrict__ tile_base, GrepParams p,
+                                                    uint32_t* __restrict__ blkcnt) {
+  __shared__ uint32_t sh[8];
+  uint64_t pw[4], pm[4];
+  pattern_words(p, pw, pm);
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t cnt = 0;
+  if (t < c.L) {
+    const LaneDesc d = lanes[t];
+    const uint8_t* tile = stage + tile_base[t >> 5];
+    for (uint32_t j = 0; j < d.nrec; ++j) cnt += grep_match(load_key(tile, j, t & 31), p, pw, pm);
+  }
+  const uint32_t s = block_sum(cnt, sh);
+  if (threadIdx.x == 0) blkcnt[blockIdx.x] = s;
+}
+
+__global__ void __launch_bounds__(1024) k_grep_scan(uint32_t* __restrict__ blkcnt, uint32_t nblk,
+                                                    unsigned long long* running, unsigned long long* blkbase) {
+  __shared__ unsigned long long warp_sums[32];
+  __shared__ unsigned long long carry;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (threadIdx.x == 0) carry = *running;
+  __syncthreads();
+  for (uint32_t base = 0; base < nblk; base += 1024) {
+    const uint32_t i = base + threadIdx.x;
+    const unsigned long long v = i < nblk ? blkcnt[i] : 0;
+    unsigned long long x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long y = __shfl_up_sync(kFull, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) warp_sums[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      unsigned long long s = warp_sums[lane];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(kFull, s, o);
+        if (lane >= o) s += y;
+      }
+      warp_sums[lane] = s;
+    }
+    __syncthreads();
+    const unsigned long long excl = carry + (wid ? warp_sums[wid - 1] : 0) + x - v;
+    if (i < nblk) blkbase[i] = excl;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = excl + v;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *running = carry;
+}
+
+__global__ void __launch_bounds__(256) k_grep_write(Chunk c, const uint8_t* __restrict__ stage,
+                                                    const LaneDesc* __restrict__ lanes,
+                                                    const uint64_t* __restrict__ tile_base, GrepParams p,
+                                                    const unsigned long long* __restrict__ blkbase,
+                                                    uint64_t* __restrict__ out, int* err) {
+  __shared__ uint32_t warp_tot[8];
+  uint64_t pw[4], pm[4];
+  pattern_words(p, pw, pm);
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  LaneDesc d{0, 0, 0};
+  const uint8_t* tile = nullptr;
+  uint32_t cnt = 0;
+  if (t < c.L) {
+    d = lanes[t];
+    tile = stage + tile_base[t >> 5];
+    for (uint32_t j = 0; j < d.nrec; ++j) cnt += grep_match(load_key(tile, j, lane), p, pw, pm);
+  }
+  if (__syncthreads_or(cnt) == 0) return;  // most blocks of a 1%-selective filter
+  uint32_t x = cnt;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(kFull, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) warp_tot[wid] = x;
+  __syncthreads();
+  uint32_t before = 0;
+  for (int i = 0; i < wid; ++i) before += warp_tot[i];
+  unsigned long long pos = blkbase[blockIdx.x] + before + x - cnt;
+  if (cnt) {
+    for (uint32_t j = 0; j < d.nrec; ++j) {
+      if (grep_match(load_key(tile, j, lane), p, pw, pm)) {
+        if (pos < p.cap) out[pos] = p.first_index + d.first + j;
+        else atomicOr(err, kErrOutOverflow);
+        ++pos;
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// C5 group-by: records {u32 key, u32 qty, f64 amount} staged one word per record.
+// Block-private shared-memory table (count, qty, amount), flushed once per block.
+
+__global__ void __launch_bounds__(256) k_groupby(Chunk c, const uint8_t* __restrict__ stage,
+                                                 const LaneDesc* __restrict__ lanes,
+                                                 const uint64_t* __restrict__ tile_base, uint32_t G,
+                                                 unsigned long long* gcount, unsigned long long* gqty,
+                                                 double* gamount, int* err) {
+  extern __shared__ unsigned char smem_raw[];
+  double* s_amt = reinterpret_cast<double*>(smem_raw);
+  unsigned int* s_cnt = reinterpret_cast<unsigned int*>(s_amt + G);
+  unsigned int* s_qty = s_cnt + G;
+  for (uint32_t g = threadIdx.x; g < G; g += blockDim.x) { s_amt[g] = 0.0; s_cnt[g] = 0; s_qty[g] = 0; }
+  __syncthreads();
+  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t - threadIdx.x < c.L; t += gridDim.x * blockDim.x) {
+    if (t < c.L) {
+      const LaneDesc d = lanes[t];
+      const uint8_t* tile = stage + tile_base[t >> 5];
+      for (uint32_t j = 0; j < d.nrec; ++j) {
+        const uint4 v = lane_word(tile, j, t & 31);
+        const uint32_t key = v.x;
+        if (key >= G) { atomicOr(err, kErrKeyRange); continue; }
+        const double amt = __hiloint2double((int)v.w, (int)v.z);
+        atomicAdd(&s_cnt[key], 1u);
+        atomicAdd(&s_qty[key], v.y);
+        atomicAdd(&s_amt[key], amt);
+      }
+    }
+  }
+  __syncthreads();
+  for (uint32_t g = threadIdx.x; g < G; g += blockDim.x) {
+    if (s_cnt[g]) {
+      atomicAdd(&gcount[g], (unsigned long long)s_cnt[g]);
+      atomicAdd(&gqty[g], (unsigned long long)s_qty[g]);
+      atomicAdd(&gamount[g], s_amt[g]);
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// C3 k-means step (P:289-305 clusterKernel/findClosestCluster): fp32 distance in the exact
+// order of DESIGN.md reading A13 (__fsub_rn, __fmaf_rn, j ascending), argmin with ties to the
+// lowest k; per-block shared sums (fp64) and counts, flushed once per block.
+
+__global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restrict__ stage,
+                                                const LaneDesc* __restrict__ lanes,
+                                                const uint64_t* __restrict__ tile_base,
+                                                const float* __restrict__ mu, uint32_t K, uint64_t first_index,
+                                                unsigned long long* gcount, double* gsum,
+                                                unsigned long long* gchk) {
+  extern __shared__ unsigned char smem_raw[];
+  double* s_sum = reinterpret_cast<double*>(smem_raw);          // K*16
+  float* s_mu = reinterpret_cast<float*>(s_sum + (size_t)K * 16);  // K*16
+  unsigned int* s_cnt = reinterpret_cast<unsigned int*>(s_mu + (size_t)K * 16);
+  for (uint32_t i = threadIdx.x; i < K * 16; i += blockDim.x) { s_sum[i] = 0.0; s_mu[i] = mu[i]; }
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) s_cnt[i] = 0;
+  __syncthreads();
+  unsigned long long chk = 0;
+  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t - threadIdx.x < c.L; t += gridDim.x * blockDim.x) {
+    if (t >= c.L) continue;
+    const LaneDesc d = lanes[t];
+    const uint8_t* tile = stage + tile_base[t >> 5];
+    for (uint32_t j = 0; j < d.nrec; ++j) {
+      float x[16];
+#pragma unroll
+      for (int w = 0; w < 4; ++w) {
+        const uint4 v = lane_word(tile, 4 * j + w, t & 31);
+        x[4 * w + 0] = __uint_as_float(v.x);
+        x[4 * w + 1] = __uint_as_float(v.y);
+        x[4 * w + 2] = __uint_as_float(v.z);
+        x[4 * w + 3] = __uint_as_float(v.w);
+      }
+      uint32_t best = 0;
+      float bestd = 0.0f;
+      for (uint32_t k = 0; k < K; ++k) {
+        float acc = 0.0f;
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+          const float df = __fsub_rn(x[q], s_mu[k * 16 + q]);
+          acc = __fmaf_rn(df, df, acc);
+        }
+        if (k == 0 || acc < bestd) { bestd = acc; best = k; }
+      }
+      atomicAdd(&s_cnt[best], 1u);
+#pragma unroll
+      for (int q = 0; q < 16; ++q) atomicAdd(&s_sum[best * 16 + q], (double)x[q]);
+      chk += mix64(((first_index + d.first + j) << 8) ^ (uint64_t)best);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) chk += __shfl_xor_sync(kFull, chk, o);  // wraps mod 2^64
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < K * 16; i += blockDim.x)
+    if (s_sum[i] != 0.0) atomicAdd(&gsum[i], s_sum[i]);
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
+    if (s_cnt[i]) atomicAdd(&gcount[i], (unsigned long long)s_cnt[i]);
+  if ((threadIdx.x & 31) == 0) atomicAdd(gchk, chk);
+}
+
+}  // namespace
+
+void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+               const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
+               int* err, cudaStream_t s) {
+  k_wc<<<(c.L + 255) / 256, 256, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
+}
+
+void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,
+                       uint32_t* len, uint64_t* cnt, uint64_t cap, cudaStream_t s) {
+  k_wc_compact<<<148 * 4, 256, 0, s>>>(table, slots, n_out, off, len, cnt, cap);
+}
+
+void launch_grep(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* running, unsigned long long* blkbase,
+                 uint64_t* out_idx, int* err, cudaStream_t s) {
+  const uint32_t nblk = (c.L + 255) / 256;
+  k_grep_count<<<nblk, 256, 0, s>>>(c, stage, lanes, tile_base, p, blkcnt);
+  k_grep_scan<<<1, 1024, 0, s>>>(blkcnt, nblk, running, blkbase);
+  k_grep_write<<<nblk, 256, 0, s>>>(c, stage, lanes, tile_base, p, blkbase, out_idx, err);
+}
+
+size_t groupby_smem(uint32_t G) { return (size_t)G * 16; }
+
+void launch_groupby(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                    uint32_t G, unsigned long long* count, unsigned long long* qty, double* amount, int* err,
+                    int grid, cudaStream_t s) {
+  k_groupby<<<grid, 256, groupby_smem(G), s>>>(c, stage, lanes, tile_base, G, count, qty, amount, err);
+}
+
+size_t kmeans_smem(uint32_t K) { return (size_t)K * 16 * 8 + (size_t)K * 16 * 4 + (size_t)K * 4; }
+
+void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                   const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
+                   unsigned long long* chk, int grid, cudaStream_t s) {
+  k_kmeans<<<grid, 256, kmeans_smem(K), s>>>(c, stage, lanes, tile_base, mu, K, first_index, count, sum, chk);
+}
+
+cudaError_t configure_compute_kernels() {
+  cudaError_t e = cudaFuncSetAttribute(k_groupby, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_kmeans, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+}
+
+}  // namespace bk

@@ -1,0 +1,248 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle on the same seeded inputs.
+
+Bit-exact for counts, indices, words and staged bytes; fp64 sums within 1e-5 relative
+(north_star). Sizes span many chunks, several tiles per chunk and ragged tails.
+"""
+import struct
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from paper_conf_ipps_mokhtaris14_b200 import bk
+
+pytestmark = pytest.mark.gpu
+
+MIB = 1 << 20
+
+
+def wc_multiset_gpu(buf: np.ndarray, off_, ln, cnt):
+    b = buf.tobytes()
+    return sorted((b[int(o): int(o) + int(l)], int(c)) for o, l, c in zip(off_, ln, cnt))
+
+
+# ------------------------------------------------------------------ layout (stages 1-2)
+LAYOUT_CASES = [
+    # name, extents, fixed record size
+    ("wc_text", None, 0),
+    ("grep_key", [(16, 32)], 0),
+    ("sparse64", [(0, 16)], 64),
+    ("kmeans64", None, 64),
+    ("dup_extents", [(8, 4), (0, 12), (8, 4)], 16),
+    ("grep_multi", [(16, 8), (40, 8)], 0),
+]
+
+
+def layout_data(name):
+    if name == "wc_text":
+        buf, off = gen.text(cap_bytes=300_000)
+        return buf, off, 0
+    if name in ("grep_key", "grep_multi"):
+        buf, off = gen.grep_records(n=5000)
+        return buf, off, 0
+    if name == "sparse64":
+        return gen.groupby(n=7001, stride=64), None, 64
+    if name == "kmeans64":
+        return gen.points(n=3001).view(np.uint8).reshape(-1), None, 64
+    return gen.groupby(n=4099, stride=16), None, 16
+
+
+@pytest.mark.parametrize("name,extents,rs", LAYOUT_CASES)
+@pytest.mark.parametrize("mode", ["zc", "dense"])
+@pytest.mark.parametrize("lanes", [32, 160])
+def test_layout_dump_matches_oracle(name, extents, rs, mode, lanes):
+    buf, off, rs = layout_data(name)
+    n = len(off) if off is not None else len(buf) // rs
+    chunk = 12_000
+    with bk.Context(window_bytes=8 * MIB, n_slots=2, gather_mode=mode, chunk_bytes=chunk, lanes=lanes,
+                    record_size=rs) as ctx:
+        ctx.register(buf, off, n_records=n)
+        # the plan budget counts accessed bytes in zc mode, whole records in dense mode
+        plan_ext = extents if mode == "zc" else None
+        bounds = oracle.plan_chunks(off, n, len(buf), rs, plan_ext, chunk)
+        first = ctx.layout_dump(0, extents)
+        assert first["n_chunks"] == len(bounds) - 1 >= 3
+        for c in sorted({0, 1, len(bounds) // 2, len(bounds) - 2}):
+            got = ctx.layout_dump(c, extents)
+            assert (got["lo"], got["hi"]) == (int(bounds[c]), int(bounds[c + 1]))
+            stage, lf, ln, lb = oracle.layout(buf, off, n, len(buf), rs, extents, got["lo"], got["hi"], got["lanes"])
+            assert np.array_equal(got["lane_first"], lf)
+            assert np.array_equal(got["lane_nrec"], ln)
+            assert np.array_equal(got["lane_bytes"], lb)
+            assert got["stage"].tobytes() == stage.tobytes()
+
+
+# ------------------------------------------------------------------ C1 word count
+@pytest.mark.parametrize("mode", ["dense", "zc"])
+@pytest.mark.parametrize("window,slots", [(256 * 1024, 2), (1 * MIB, 4), (8 * MIB, 3)])
+def test_wordcount_small(mode, window, slots):
+    buf, off = gen.text(cap_bytes=2 * MIB)
+    want = oracle.wc(buf, off)
+    with bk.Context(window_bytes=window, n_slots=slots, gather_mode=mode) as ctx:
+        ctx.register(buf, off)
+        got = wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 18))
+        assert ctx.stats()["n_chunks"] >= 2
+    assert got == want
+
+
+def test_wordcount_adversarial():
+    recs = [b"  a\tb\r\n", b"", b"", b"\x00\x80 z", b"ab", b"cd", b"tail without newline", b" ", b"x" * 300,
+            b"dup dup\n"] * 37
+    buf = np.frombuffer(b"".join(recs), np.uint8)
+    off = np.cumsum([0] + [len(r) for r in recs[:-1]]).astype(np.uint64)
+    want = oracle.wc(buf, off)
+    for mode in ("zc", "dense"):
+        with bk.Context(window_bytes=64 * 1024, n_slots=2, gather_mode=mode, chunk_bytes=1500, lanes=32) as ctx:
+            ctx.register(buf, off)
+            assert wc_multiset_gpu(buf, *ctx.wordcount(cap=4096)) == want
+
+
+def test_wordcount_full_c1_config():
+    """configs[0]: 64 MiB text, 8 MiB window, 1 GPU — whole result bit-exact vs the oracle."""
+    buf, off = gen.text(cap_bytes=64 * MIB)
+    want = oracle.wc(buf, off)
+    with bk.Context(window_bytes=8 * MIB) as ctx:
+        ctx.register(buf, off)
+        got = wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 20))
+        st = ctx.stats()
+    assert got == want
+    assert st["bytes_accessed"] == len(buf)        # I3: every byte accessed once
+    assert st["n_chunks"] >= 8                      # out-of-core: data > window
+
+
+# ------------------------------------------------------------------ C2 grep
+def grep_rec(key: bytes, payload: bytes = b"") -> bytes:
+    k = key[:32].ljust(32, b"\x00")
+    return struct.pack("<IIQ", 48 + len(payload), 0, 0) + k + payload
+
+
+def test_grep_adversarial():
+    recs = [grep_rec(b"bigkxxxx"), grep_rec(b"xxxxbigk"), grep_rec(b"a" * 28 + b"bigk"), grep_rec(b"big\x00k"),
+            grep_rec(b"bi"), grep_rec(b"xbigkx", b"bigkbigk" + b"q" * 7), grep_rec(b""), grep_rec(b"q" * 32, b"z")] * 53
+    buf = np.frombuffer(b"".join(recs), np.uint8)
+    off = np.cumsum([0] + [len(r) for r in recs[:-1]]).astype(np.uint64)
+    for pat in (b"bigk", b"", b"a", b"q" * 32, b"aaaaaaaaaaaabigk", b"x" * 33):
+        if len(pat) > 32:
+            with bk.Context(window_bytes=1 * MIB) as ctx:
+                ctx.register(buf, off)
+                with pytest.raises(bk.BkError):
+                    ctx.grep(pat)
+            continue
+        want = oracle.grep(buf, off, pat)
+        for mode in ("zc", "dense"):
+            with bk.Context(window_bytes=256 * 1024, n_slots=2, gather_mode=mode, chunk_bytes=2048, lanes=64) as ctx:
+                ctx.register(buf, off)
+                got = ctx.grep(pat, cap=len(off))
+            assert np.array_equal(got, want), (pat, mode)
+
+
+@pytest.mark.parametrize("mode", ["zc", "dense"])
+def test_grep_medium(mode):
+    buf, off = gen.grep_records(max_bytes=64 * MIB)
+    want = oracle.grep(buf, off, b"bigk", first=1000)
+    with bk.Context(window_bytes=16 * MIB, gather_mode=mode) as ctx:
+        ctx.register(buf, off)
+        got = ctx.grep(b"bigk", first_index=1000, cap=len(off))
+        st = ctx.stats()
+    assert np.array_equal(got, want)
+    assert st["n_chunks"] >= 8
+    if mode == "zc":
+        assert st["bytes_accessed"] == 32 * len(off) == st["bytes_h2d"]   # I3: only the key bytes
+
+
+def test_grep_capacity_error():
+    buf, off = gen.grep_records(n=20000)
+    with bk.Context(window_bytes=4 * MIB) as ctx:
+        ctx.register(buf, off)
+        with pytest.raises(bk.BkError) as e:
+            ctx.grep(b"", cap=100)
+        assert e.value.status == bk.BK_E_CAPACITY
+
+
+def test_grep_full_c2_config():
+    """configs[1] in bench.py's launch configuration: 16 GiB, 2 GiB window, zc gather.
+    The oracle computes the whole answer (single-threaded C, ~10 s)."""
+    buf, off = gen.grep_records(max_bytes=16 << 30)
+    with bk.Context(window_bytes=2 << 30) as ctx:
+        ctx.register(buf, off)
+        got = ctx.grep(b"bigk", cap=len(off) // 50)
+        st = ctx.stats()
+    want = oracle.grep(buf, off, b"bigk")
+    assert np.array_equal(got, want)
+    assert st["n_chunks"] >= 16 and st["bytes_accessed"] == 32 * len(off)
+
+
+# ------------------------------------------------------------------ C5 group-by
+@pytest.mark.parametrize("stride,zipf,mode", [(16, False, "dense"), (16, True, "zc"), (64, False, "zc"),
+                                              (64, True, "dense")])
+def test_groupby(stride, zipf, mode):
+    n = 3_000_001
+    buf = gen.groupby(n=n, stride=stride, zipf=zipf)
+    wc_, wq, wa = oracle.groupby(buf, n, stride, 4096)
+    with bk.Context(window_bytes=16 * MIB, gather_mode=mode, record_size=stride) as ctx:
+        ctx.register(buf, None, n_records=n)
+        c, q, a = ctx.groupby(4096)
+        assert ctx.stats()["n_chunks"] >= 4
+    assert np.array_equal(c, wc_) and np.array_equal(q, wq)
+    np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
+
+
+def test_groupby_key_out_of_range():
+    buf = gen.groupby(n=1000, G=4096)
+    with bk.Context(window_bytes=1 * MIB, record_size=16) as ctx:
+        ctx.register(buf, None, n_records=1000)
+        with pytest.raises(bk.BkError) as e:
+            ctx.groupby(G=100)
+        assert e.value.status == bk.BK_E_INVAL
+
+
+# ------------------------------------------------------------------ C3 k-means
+@pytest.mark.parametrize("mode,K", [("dense", 64), ("zc", 64), ("dense", 7)])
+def test_kmeans(mode, K):
+    n = 400_003
+    x = gen.points(n=n)
+    mu = x[:K].copy()
+    wc_, ws, wchk, _ = oracle.kmeans(x, mu, first=5)
+    with bk.Context(window_bytes=8 * MIB, gather_mode=mode, record_size=64) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=n)
+        c, s, chk = ctx.kmeans(mu, first_index=5)
+    assert np.array_equal(c, wc_) and chk == wchk
+    # |gpu - ref| <= 1e-5 * sum |x| (data are positive, so this is relative)
+    np.testing.assert_allclose(s, ws, rtol=1e-5, atol=0)
+
+
+# ------------------------------------------------------------------ invariants + API errors
+def test_invariance_across_window_slots_lanes_modes():
+    buf, off = gen.text(cap_bytes=1 * MIB)
+    want = oracle.wc(buf, off)
+    for window, slots, lanes, mode in [(128 * 1024, 2, 0, "zc"), (300_000, 3, 64, "dense"), (4 * MIB, 8, 0, "zc"),
+                                       (4 * MIB, 2, 1024, "dense")]:
+        with bk.Context(window_bytes=window, n_slots=slots, lanes=lanes, gather_mode=mode) as ctx:
+            ctx.register(buf, off)
+            assert wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 17)) == want, (window, slots, lanes, mode)
+
+
+def test_api_errors():
+    buf, off = gen.text(cap_bytes=100_000)
+    with bk.Context(window_bytes=1 * MIB) as ctx:
+        with pytest.raises(bk.BkError) as e:
+            ctx.wordcount()
+        assert e.value.status == bk.BK_E_STATE
+        bad = off.copy()
+        bad[5], bad[6] = bad[6], bad[5]
+        with pytest.raises(bk.BkError) as e:
+            ctx.register(buf, bad)
+        assert e.value.status == bk.BK_E_INVAL
+    with bk.Context(window_bytes=1 * MIB, chunk_bytes=10) as ctx:   # a line is longer than the budget
+        ctx.register(buf, off)
+        with pytest.raises(bk.BkError) as e:
+            ctx.wordcount()
+        assert e.value.status == bk.BK_E_RANGE
+    with pytest.raises(bk.BkError):
+        bk.Context(n_slots=1)
+    # empty data set
+    with bk.Context(window_bytes=1 * MIB) as ctx:
+        ctx.register(np.zeros(0, np.uint8), np.zeros(0, np.uint64))
+        o, l, c = ctx.wordcount(cap=16)
+        assert len(c) == 0
