@@ -4,7 +4,7 @@ ARCH   := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -std=c++17 -O3 -lineinfo $(ARCH) -Xcompiler -fPIC,-fvisibility=hidden -Xptxas -v
 PKG    := paper_conf_ipps_mokhtaris14_b200
 CSRC   := $(PKG)/csrc
-OBJS   := build/kernels_stage.o build/kernels_compute.o build/bk_runtime.o
+OBJS   := build/kernels_stage.o build/kernels_compute.o build/bk_runtime.o build/host_gather.o
 
 all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so
 
@@ -12,8 +12,12 @@ build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh include/bk.h
 	@mkdir -p build
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
 
+build/host_gather.o: $(CSRC)/host_gather.cpp $(CSRC)/host_gather.h $(CSRC)/bk_internal.cuh
+	@mkdir -p build
+	g++ -std=c++17 -O3 -march=x86-64-v3 -fPIC -fvisibility=hidden -Wall -I/usr/local/cuda/include -c $< -o $@
+
 $(PKG)/libbk.so: $(OBJS)
-	$(NVCC) -shared $(ARCH) -cudart static -o $@ $(OBJS)
+	$(NVCC) -shared $(ARCH) -cudart static -o $@ $(OBJS) -lpthread
 
 oracle/libbkoracle.so: oracle/oracle.c oracle/oracle.h
 	gcc -O2 -ffp-contract=off -fPIC -shared -Wall -o $@ oracle/oracle.c -lm

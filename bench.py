@@ -48,10 +48,11 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "kmeans"])
-    ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense"])
+    ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense", "cpu", "hybrid"])
     ap.add_argument("--gib", type=float, default=None, help="per-GPU data size override (GiB)")
     ap.add_argument("--window-mib", type=int, default=None)
     ap.add_argument("--slots", type=int, default=0)
+    ap.add_argument("--host-threads", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-profile", action="store_true", help="disable per-stage event timing")
     return ap.parse_args()
@@ -212,6 +213,7 @@ def main():
     shard = make_shard(args.workload, gib, rank, world)
     peak_h2d = measure_h2d_peak(torch, dev)
     ctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
+                     host_threads=args.host_threads,
                      profile=not args.no_profile, record_size=shard["rec_size"])
     t0 = time.perf_counter()
     ctx.register(shard["buf"], shard["off"], n_records=shard["n"])
@@ -280,28 +282,42 @@ def main():
     link_bytes = (st["bytes_h2d"] + st["bytes_meta"]) * world * args.steps
     link_gbs = link_bytes / t_dev / 1e9
 
-    # ---- roofline of the dominant kernel (stage busy times from events on its own stream)
+    # ---- roofline of the dominant stage (busy times from CUDA events on each stage's own stream)
     peaks = load_peaks()
-    stage_ms = {"gather": st["ms_gather"], "compute": st["ms_compute"], "addrgen": st["ms_addrgen"]}
+    stage_ms = {"gather": st["ms_gather"], "compute": st["ms_compute"], "addrgen": st["ms_addrgen"],
+                "h2d": st["ms_h2d"]}
     dom = max(stage_ms, key=stage_ms.get)
-    launches_dom = max(st["n_gather"], 1) if dom == "gather" else st["n_chunks"]
-    avg_ms = stage_ms[dom] / max(launches_dom, 1)
-    if dom == "gather" and st["gather_mode"] == bk.BK_GATHER_ZC:
-        per_launch = st["bytes_accessed"] / launches_dom      # bytes pulled over PCIe per gather launch
+    n_zc = max(st["n_gather"], 1)
+    if dom == "h2d":
+        # copy-engine DMA of packed (CPU) or raw (DENSE) chunks + offsets slices: host-link bound
+        launches = st["n_chunks"]
+        per_launch = (st["bytes_h2d"] - (st["bytes_accessed"] * (st["n_gather"] / max(st["n_chunks"], 1))
+                                          if st["gather_mode"] == bk.BK_GATHER_HYBRID else 0)
+                      + st["bytes_meta"]) / launches
+        roof = {"kernel": "cudaMemcpyAsync H2D of staged chunks (stage 3, copy engine)", "bound": "host_link",
+                "peak": peak_h2d, "unit": "GB/s"}
+    elif dom == "gather" and st["gather_mode"] in (bk.BK_GATHER_ZC, bk.BK_GATHER_HYBRID):
+        launches = n_zc
+        zc_chunks = n_zc
+        per_launch = st["bytes_accessed"] / st["n_chunks"]      # accessed bytes per chunk pulled over PCIe
         roof = {"kernel": "k_gather_field/whole<zero-copy> (stages 2+3)", "bound": "host_link",
-                "achieved": per_launch / (avg_ms * 1e-3) / 1e9, "peak": peak_h2d, "unit": "GB/s",
-                "peak_source": "pinned H2D cudaMemcpyAsync measured live in this run (MEASURED_PEAKS.json has no host-link entry)"}
+                "peak": peak_h2d, "unit": "GB/s"}
     else:
+        launches = n_zc if dom == "gather" else st["n_chunks"]
         # HBM-bound kernels: re-layout reads the raw chunk and writes the tiles; compute reads the tiles
-        per_launch = (st["bytes_h2d"] + st["bytes_accessed"] + st["bytes_padding"]) / launches_dom \
-            if dom == "gather" else (st["bytes_accessed"] + st["bytes_padding"]) / launches_dom
-        roof = {"kernel": f"{dom} ({args.workload})", "bound": "hbm", "achieved": per_launch / (avg_ms * 1e-3) / 1e9,
-                "peak": peaks.get("hbm_gbs", 6650.0), "unit": "GB/s",
-                "peak_source": "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6650 GB/s"}
+        per_launch = ((st["bytes_h2d"] + st["bytes_accessed"] + st["bytes_padding"]) if dom == "gather"
+                      else (st["bytes_accessed"] + st["bytes_padding"])) / max(launches, 1)
+        roof = {"kernel": f"{dom} ({args.workload})", "bound": "hbm", "peak": peaks.get("hbm_gbs", 6650.0),
+                "unit": "GB/s"}
+    avg_ms = stage_ms[dom] / max(launches, 1)
+    roof["achieved"] = per_launch / (avg_ms * 1e-3) / 1e9
+    roof["peak_source"] = ("pinned H2D cudaMemcpyAsync measured live in this run (MEASURED_PEAKS.json has no "
+                           "host-link entry)") if roof["bound"] == "host_link" else (
+        "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6650 GB/s")
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["traffic"] = None
     roof["avg_launch_ms"] = avg_ms
-    roof["launches_per_step"] = launches_dom
+    roof["launches_per_step"] = launches
 
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
@@ -309,7 +325,8 @@ def main():
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded counter RNG, gen/)",
         "config": {"workload": args.workload, "desc": WORKLOADS[args.workload][2],
                    "bytes_per_gpu": nbytes, "records_per_gpu": shard["n"], "window_bytes": window,
-                   "gather_mode": {1: "zc", 3: "dense"}.get(st["gather_mode"], "?"), "n_chunks": st["n_chunks"],
+                   "gather_mode": {1: "zc", 2: "cpu", 3: "dense", 4: "hybrid"}.get(st["gather_mode"], "?"),
+                   "chunks_cpu_assembled": st["n_chunks_cpu"], "n_chunks": st["n_chunks"],
                    "lanes_per_chunk": st["lanes"], "chunk_budget_bytes": st["chunk_budget"],
                    "l2": "inputs (>=64 MiB per GPU, host-resident) exceed the 126 MB L2; streamed from host each step",
                    "parallelism": f"dp{world} (contiguous record shards, one PCIe link per GPU)"},
@@ -318,7 +335,8 @@ def main():
                  "frac": round(link_gbs / (peak_h2d * world), 4),
                  "bytes_per_step_per_gpu": st["bytes_h2d"] + st["bytes_meta"],
                  "payload_bytes": st["bytes_h2d"], "meta_bytes": st["bytes_meta"], "padding_bytes_hbm": st["bytes_padding"]},
-        "stages_ms_per_step": {k: round(st[k], 3) for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute", "ms_device")},
+        "stages_ms_per_step": {k: round(st[k], 3) for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute",
+                                                             "ms_device", "ms_cpu_gather")},
         "e2e": {"value": round(total_bytes / t_wall / 1e9, 3), "unit": "GB/s",
                 "h2d_bytes_per_step": (st["bytes_h2d"] + st["bytes_meta"]) * world,
                 "d2h_bytes_per_step": st["bytes_d2h"] * world,

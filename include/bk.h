@@ -53,12 +53,15 @@ typedef enum {
 
 /* Stage-2/3 implementations. */
 typedef enum {
-  BK_GATHER_AUTO = 0,   /* ZC for sparse access, DENSE when every byte is accessed */
+  BK_GATHER_AUTO = 0,   /* HYBRID for sparse access, DENSE when every byte is accessed */
   BK_GATHER_ZC = 1,     /* GPU kernel reads the accessed bytes from pinned, mapped host memory
                            (16-B loads) and writes the interleaved tiles to HBM: stages 2+3 fused */
-  BK_GATHER_CPU = 2,    /* reserved: host-thread assembly into pinned staging + DMA (not in this build) */
-  BK_GATHER_DENSE = 3   /* one contiguous DMA of the chunk's records (copy engine), then an
+  BK_GATHER_CPU = 2,    /* a host thread pool packs exactly the accessed bytes into pinned staging in
+                           the warp-tile layout (the paper's CPU assembly), then one DMA */
+  BK_GATHER_DENSE = 3,  /* one contiguous DMA of the chunk's records (copy engine), then an
                            HBM->HBM re-layout kernel (fetch-all) */
+  BK_GATHER_HYBRID = 4  /* per chunk: GPU zero-copy gather while fewer than (n_slots-1)/2 are in
+                           flight, otherwise CPU assembly; both share the link */
 } bk_gather_mode;
 
 typedef struct bk_config {
@@ -70,7 +73,7 @@ typedef struct bk_config {
   uint32_t gather_mode;   /* bk_gather_mode */
   uint64_t chunk_bytes;   /* accessed (payload) bytes per chunk; 0 = auto (fits a slot, >= ~32 chunks) */
   uint32_t lanes;         /* lanes (compute threads) per chunk, multiple of 32; 0 = auto */
-  uint32_t host_threads;  /* reserved for BK_GATHER_CPU */
+  uint32_t host_threads;  /* CPU-assembly pool size (BK_GATHER_CPU / HYBRID); 0 = all hardware threads */
   uint64_t record_size;   /* fixed record length when record_offsets == NULL */
   uint32_t flags;         /* BK_FLAG_* */
   uint32_t _reserved;
@@ -205,6 +208,8 @@ typedef struct bk_stats {
   double ms_gather;           /*   ... of stage 2 (+3 in ZC mode): gather / re-layout kernels */
   double ms_compute;          /*   ... of stage 4 (compute kernels) */
   uint64_t n_gather;          /*   number of gather launches timed */
+  uint64_t n_chunks_cpu;      /* chunks assembled by the host pool (CPU / HYBRID) */
+  double ms_cpu_gather;       /* host time spent assembling them */
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);

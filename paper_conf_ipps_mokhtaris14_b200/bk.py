@@ -16,9 +16,9 @@ LIB_PATH = os.path.join(_HERE, "libbk.so")
 
 BK_OK, BK_E_INVAL, BK_E_NOMEM, BK_E_CUDA, BK_E_STATE, BK_E_RANGE, BK_E_CAPACITY, BK_E_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
 BK_K_WORDCOUNT, BK_K_GREP, BK_K_KMEANS, BK_K_PARTITION, BK_K_GROUPBY, BK_K_LAYOUT_DUMP = 1, 2, 3, 4, 5, 100
-BK_GATHER_AUTO, BK_GATHER_ZC, BK_GATHER_CPU, BK_GATHER_DENSE = 0, 1, 2, 3
+BK_GATHER_AUTO, BK_GATHER_ZC, BK_GATHER_CPU, BK_GATHER_DENSE, BK_GATHER_HYBRID = 0, 1, 2, 3, 4
 BK_FLAG_PROFILE = 1
-GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE}
+GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE, "hybrid": BK_GATHER_HYBRID}
 
 u32, i32, u64, P = C.c_uint32, C.c_int32, C.c_uint64, C.c_void_p
 
@@ -70,7 +70,7 @@ class bk_stats(C.Structure):
                 ("bytes_meta", u64), ("bytes_padding", u64), ("bytes_d2h", u64), ("kernel_launches", u64),
                 ("ms_run", C.c_double), ("ms_register", C.c_double), ("ms_device", C.c_double),
                 ("ms_h2d", C.c_double), ("ms_addrgen", C.c_double), ("ms_gather", C.c_double),
-                ("ms_compute", C.c_double), ("n_gather", u64)]
+                ("ms_compute", C.c_double), ("n_gather", u64), ("n_chunks_cpu", u64), ("ms_cpu_gather", C.c_double)]
 
 
 ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,

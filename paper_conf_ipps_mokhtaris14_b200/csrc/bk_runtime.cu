@@ -25,6 +25,7 @@
 
 #include "../../include/bk.h"
 #include "bk_internal.cuh"
+#include "host_gather.h"
 
 using namespace bk;
 
@@ -88,6 +89,7 @@ struct DevBuf {
 struct bk_ctx {
   bk_config cfg{};
   cudaStream_t s_copy = nullptr, s_asm = nullptr, s_comp = nullptr;
+  std::vector<cudaStream_t> s_slot;  // per-slot compute streams for commutative kernels
   cudaEvent_t ev_begin = nullptr, ev_end = nullptr;
   cudaEvent_t t_begin = nullptr, t_end = nullptr;   // timing events on s_comp (device time of a run)
   std::vector<cudaEvent_t> prof;                   // BK_FLAG_PROFILE: per chunk x stage begin/end
@@ -107,6 +109,14 @@ struct bk_ctx {
   int* d_err = nullptr;
   unsigned long long* d_ctr = nullptr;  // [0] staged sum, [1] wc used, [2] wc n_out, [3] grep running, [4] kmeans chk
   DevBuf b_table, b_out1, b_out2, b_out3, b_blk, b_blk2, b_agg1, b_agg2, b_agg3, b_mu;
+  // CPU assembly (BK_GATHER_CPU / HYBRID): thread pool + pinned host staging ring
+  HostPool* pool = nullptr;
+  std::vector<uint8_t*> hstage;
+  std::vector<cudaEvent_t> h_done;
+  std::vector<bool> h_used;
+  uint64_t hstage_cap = 0;
+  uint64_t h_next = 0;
+  std::vector<uint64_t> scratch_first, scratch_tiles;
   int n_launch = 0;
   bk_stats st{};
 };
@@ -129,7 +139,8 @@ uint64_t rec_start(const bk_ctx* c, uint64_t r) {
 
 struct Plan {
   Access a{};
-  int zero_copy = 0;
+  int mode = BK_GATHER_DENSE;          // resolved gather mode
+  int zero_copy = 0;                   // plan budget counts accessed bytes (every mode but DENSE)
   uint64_t budget = 0;                 // plan bytes per chunk
   uint32_t L = 0;
   uint64_t max_acc_rec = 0;            // max accessed bytes of one record
@@ -209,10 +220,14 @@ void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) 
 int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p) {
   p.a = a;
   int mode = (int)c->cfg.gather_mode;
-  if (mode == BK_GATHER_AUTO) mode = a.whole ? BK_GATHER_DENSE : BK_GATHER_ZC;
-  if (mode == BK_GATHER_CPU) return fail(BK_E_UNSUPPORTED, "BK_GATHER_CPU is not in this build");
-  if (mode != BK_GATHER_ZC && mode != BK_GATHER_DENSE) return fail(BK_E_INVAL, "bad gather_mode %d", mode);
-  p.zero_copy = mode == BK_GATHER_ZC;
+  // AUTO (counters in profiles/): whole-record access -> DENSE (copy engine at
+  // 55.5 GB/s beats zero-copy's 51.4); sparse access -> HYBRID (host assembly packs exactly the
+  // accessed bytes; the zero-copy gather is request-rate bound and only adds capacity on top).
+  if (mode == BK_GATHER_AUTO) mode = a.whole ? BK_GATHER_DENSE : BK_GATHER_HYBRID;
+  if (mode != BK_GATHER_ZC && mode != BK_GATHER_DENSE && mode != BK_GATHER_CPU && mode != BK_GATHER_HYBRID)
+    return fail(BK_E_INVAL, "bad gather_mode %d", mode);
+  p.mode = mode;
+  p.zero_copy = mode != BK_GATHER_DENSE;
   p.max_acc_rec = a.whole ? c->max_rec : a.E;
   const uint64_t slot = c->cfg.window_bytes / c->cfg.n_slots;
   // total plan bytes
@@ -295,22 +310,84 @@ int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin) {
 }
 #define BK_PROF(stage, stream, begin) do { int r_ = prof_mark(c, stage, stream, begin); if (r_) return r_; } while (0)
 
+int ensure_host_side(bk_ctx* c, const Plan& p) {
+  if (!c->pool) {
+    int th = (int)c->cfg.host_threads;
+    if (th <= 0) th = (int)std::max(1u, std::thread::hardware_concurrency());
+    c->pool = new (std::nothrow) HostPool(th);
+    if (!c->pool) return fail(BK_E_NOMEM, "host pool");
+  }
+  const size_t NH = 3;
+  if (c->hstage_cap < p.stage_cap || c->hstage.size() != NH) {
+    for (auto* h : c->hstage) cudaFreeHost(h);
+    c->hstage.assign(NH, nullptr);
+    for (auto& h : c->hstage) BK_CUDA(cudaHostAlloc((void**)&h, p.stage_cap, cudaHostAllocPortable));
+    c->hstage_cap = p.stage_cap;
+    if (c->h_done.empty()) {
+      c->h_done.assign(NH, nullptr);
+      for (auto& e : c->h_done) BK_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
+  }
+  c->h_used.assign(NH, false);
+  c->h_next = 0;
+  return BK_OK;
+}
+
+// CPU assembly of chunk i (stage 2 on the host pool) + one DMA of the packed tiles (stage 3).
+int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
+  const Chunk ch = chunk_of(c, p, i);
+  Access a = p.a;
+  a.rec_size = c->off ? 0 : c->cfg.record_size;
+  const size_t hs = c->h_next++ % c->hstage.size();
+  if (c->h_used[hs]) BK_CUDA(cudaEventSynchronize(c->h_done[hs]));   // its previous DMA finished
+  const auto t0 = std::chrono::steady_clock::now();
+  HostData d{c->host, c->off, c->n, c->nbytes, c->cfg.record_size};
+  const uint64_t size = host_gather_chunk(*c->pool, d, a, ch, c->hstage[hs], p.stage_cap, c->scratch_first,
+                                          c->scratch_tiles);
+  c->st.ms_cpu_gather += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  if (size == UINT64_MAX) return fail(BK_E_RANGE, "host-staged chunk exceeds its slot (internal bound violated)");
+  if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+  BK_PROF(kStH2D, c->s_copy, true);
+  if (c->off && a.whole && ch.hi > ch.lo) {  // record boundaries for whole-record kernels
+    BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
+    c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+  }
+  if (size) BK_CUDA(cudaMemcpyAsync(s.stage, c->hstage[hs], size, cudaMemcpyHostToDevice, c->s_copy));
+  BK_CUDA(cudaEventRecord(c->h_done[hs], c->s_copy));
+  c->h_used[hs] = true;
+  BK_PROF(kStH2D, c->s_copy, false);
+  BK_PROF(kStAddrgen, c->s_copy, true);
+  launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_copy);
+  BK_PROF(kStAddrgen, c->s_copy, false);
+  c->n_launch += 2;
+  c->st.bytes_h2d += size;   // payload + tile padding (A9: padding crosses the link only in this mode)
+  c->st.bytes_accessed += ch.accessed;
+  c->st.n_chunks_cpu += 1;
+  BK_CUDA(cudaEventRecord(s.ready, c->s_copy));
+  s.used = true;
+  return BK_OK;
+}
+
 // Stages 1-3 of chunk i into slot s (on s_copy / s_asm); records s.ready.
 int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   const Chunk ch = chunk_of(c, p, i);
   Access a = p.a;
   a.rec_size = c->off ? 0 : c->cfg.record_size;
-  if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
-  BK_PROF(kStH2D, c->s_copy, true);
-  if (c->off && ch.hi > ch.lo) {
-    BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
-    c->st.bytes_meta += (ch.hi - ch.lo) * 8;
-  }
   if (p.zero_copy) {
-    BK_PROF(kStH2D, c->s_copy, false);
-    BK_PROF(kStAddrgen, c->s_copy, true);
-    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_copy);
-    BK_PROF(kStAddrgen, c->s_copy, false);
+    // Stage 1 on s_asm (offsets slice by DMA + lane plan) runs ahead, overlapping the previous
+    // chunk's zero-copy gather on s_copy; the gather waits only for its own plan.
+    if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_asm, s.freed, 0));
+    BK_PROF(kStH2D, c->s_asm, true);
+    if (c->off && ch.hi > ch.lo) {
+      BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_asm));
+      c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+    }
+    BK_PROF(kStH2D, c->s_asm, false);
+    BK_PROF(kStAddrgen, c->s_asm, true);
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
+    BK_PROF(kStAddrgen, c->s_asm, false);
+    BK_CUDA(cudaEventRecord(s.copied, c->s_asm));
+    BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.copied, 0));
     BK_PROF(kStGather, c->s_copy, true);
     launch_gather(ch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1,
                   c->s_copy);
@@ -318,6 +395,12 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     c->n_launch += 3;
     c->st.bytes_h2d += ch.accessed;
   } else {
+    if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+    BK_PROF(kStH2D, c->s_copy, true);
+    if (c->off && ch.hi > ch.lo) {
+      BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
+      c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+    }
     const uint64_t raw_off = ((uintptr_t)(c->host + ch.base_byte)) & 15;
     const uint64_t bytes = ch.end_byte - ch.base_byte;
     if (bytes) BK_CUDA(cudaMemcpyAsync(s.raw + raw_off, c->host + ch.base_byte, bytes, cudaMemcpyHostToDevice, c->s_copy));
@@ -335,13 +418,12 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   }
   c->st.bytes_accessed += ch.accessed;
   BK_CUDA(cudaEventRecord(s.ready, p.zero_copy ? c->s_copy : c->s_asm));
-  BK_CUDA(cudaStreamWaitEvent(c->s_comp, s.ready, 0));
   s.used = true;
   return BK_OK;
 }
 
 void note_plan(bk_ctx* c, const Plan& p) {
-  c->st.gather_mode = p.zero_copy ? BK_GATHER_ZC : BK_GATHER_DENSE;
+  c->st.gather_mode = (uint32_t)p.mode;
   c->st.chunk_budget = p.budget;
   c->st.lanes = p.L;
 }
@@ -356,22 +438,47 @@ int check_err(bk_ctx* c) {
   return BK_OK;
 }
 
-// ---- the pipeline driver: stage chunk i+?, compute chunk i, with N slots in flight ----
+// ---- the pipeline driver: chunk i goes through slot i % N; stages 1-3 on the copy/assembly
+// streams, stage 4 on the compute stream. `concurrent`: the kernel's updates commute (atomic
+// aggregation), so chunk i's compute runs on slot stream i % N and may overlap chunk i-1's;
+// otherwise (grep's ordered output) every compute is serialised on s_comp.
 template <class Compute>
-int pipeline(bk_ctx* c, const Plan& p, Compute&& compute) {
+int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
   const size_t C = p.bounds.size() - 1;
   c->st.n_chunks = C;
   note_plan(c, p);
+  std::vector<cudaEvent_t> zc_inflight;
+  // zero-copy chunks in flight in HYBRID mode: one keeps the GPU gather busy while the host pool
+  // assembles the next chunk (sweep in profiles/r01_hybrid_sweep.md)
+  const size_t zc_depth = std::max<size_t>(1, (c->cfg.n_slots - 1) / 2);
+  if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
+    int rc = ensure_host_side(c, p);
+    if (rc) return rc;
+  }
   for (size_t i = 0; i < C; ++i) {
     Slot& s = c->slots[i % c->cfg.n_slots];
-    int rc = stage_chunk(c, p, i, s);
+    cudaStream_t cs = concurrent ? c->s_slot[i % c->cfg.n_slots] : c->s_comp;
+    bool cpu = p.mode == BK_GATHER_CPU;
+    if (p.mode == BK_GATHER_HYBRID) {
+      // GPU zero-copy gathers run asynchronously; keep up to zc_depth of them in flight and let
+      // the host pool assemble the next chunk whenever the GPU side is saturated.
+      while (!zc_inflight.empty() && cudaEventQuery(zc_inflight.front()) == cudaSuccess) zc_inflight.erase(zc_inflight.begin());
+      cudaGetLastError();
+      cpu = zc_inflight.size() >= zc_depth;
+    }
+    int rc = cpu ? stage_chunk_cpu(c, p, i, s) : stage_chunk(c, p, i, s);
     if (rc) return rc;
-    BK_PROF(kStCompute, c->s_comp, true);
-    rc = compute(chunk_of(c, p, i), s);
+    if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(s.ready);
+    BK_CUDA(cudaStreamWaitEvent(cs, s.ready, 0));
+    BK_PROF(kStCompute, cs, true);
+    rc = compute(chunk_of(c, p, i), s, cs);
     if (rc) return rc;
-    BK_PROF(kStCompute, c->s_comp, false);
-    BK_CUDA(cudaEventRecord(s.freed, c->s_comp));
+    BK_PROF(kStCompute, cs, false);
+    BK_CUDA(cudaEventRecord(s.freed, cs));
   }
+  if (concurrent)  // join: finalize on s_comp after every slot's last compute
+    for (auto& s : c->slots)
+      if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_comp, s.freed, 0));
   return BK_OK;
 }
 
@@ -404,6 +511,8 @@ int begin_run(bk_ctx* c, void* stream) {
   c->n_launch = 0;
   c->prof_used = 0;
   c->st.bytes_accessed = c->st.bytes_h2d = c->st.bytes_meta = c->st.bytes_padding = c->st.bytes_d2h = 0;
+  c->st.n_chunks_cpu = 0;
+  c->st.ms_cpu_gather = 0;
   return BK_OK;
 }
 
@@ -450,9 +559,9 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   if ((rc = begin_run(c, stream))) return rc;
   BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
   WcEntry* table = (WcEntry*)c->b_table.p;
-  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
     launch_wc(ch, s.stage, s.lanes, s.tile_base, s.meta, c->off ? 0 : c->cfg.record_size, table, slots - 1,
-              c->d_ctr + 1, c->d_err, c->s_comp);
+              c->d_ctr + 1, c->d_err, cs);
     c->n_launch += 1;
     return BK_OK;
   });
@@ -498,9 +607,9 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
   gp.first_index = o->first_index;
   gp.cap = cap;
   if ((rc = begin_run(c, stream))) return rc;
-  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+  rc = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
     launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p, c->d_ctr + 3,
-                (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, c->s_comp);
+                (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, cs);
     c->n_launch += 3;
     return BK_OK;
   });
@@ -536,9 +645,9 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
   BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)G * 8, c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)G * 8, c->s_comp));
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * per_sm));
-  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
     launch_groupby(ch, s.stage, s.lanes, s.tile_base, G, (unsigned long long*)c->b_agg1.p,
-                   (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, c->s_comp);
+                   (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, cs);
     c->n_launch += 1;
     return BK_OK;
   });
@@ -571,9 +680,9 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
-  rc = pipeline(c, p, [&](const Chunk& ch, Slot& s) {
+  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
     launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
-                  (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4, grid, c->s_comp);
+                  (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4, grid, cs);
     c->n_launch += 1;
     return BK_OK;
   });
@@ -614,7 +723,13 @@ int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
                                            (unsigned long long)o->n_chunks);
   if ((rc = begin_run(c, stream))) return rc;
   Slot& s = c->slots[0];
-  if ((rc = stage_chunk(c, p, o->chunk, s))) return rc;
+  if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
+    if ((rc = ensure_host_side(c, p))) return rc;
+    if ((rc = stage_chunk_cpu(c, p, o->chunk, s))) return rc;
+  } else if ((rc = stage_chunk(c, p, o->chunk, s))) {
+    return rc;
+  }
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, s.ready, 0));
   const Chunk ch = chunk_of(c, p, o->chunk);
   o->chunk_lo = ch.lo;
   o->chunk_hi = ch.hi;
@@ -699,6 +814,9 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
   if (cudaMalloc(&c->d_err, 256) != cudaSuccess || cudaMalloc(&c->d_ctr, 8 * sizeof(unsigned long long)) != cudaSuccess)
     return cleanup(fail(BK_E_NOMEM, "cudaMalloc scratch"));
   c->slots.resize(c->cfg.n_slots);
+  c->s_slot.assign(c->cfg.n_slots, nullptr);
+  for (auto& st : c->s_slot)
+    if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "slot streams"));
   for (auto& s : c->slots) {
     if (cudaEventCreateWithFlags(&s.copied, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&s.ready, cudaEventDisableTiming) != cudaSuccess ||
@@ -813,6 +931,7 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
     cudaStreamSynchronize(c->s_copy);
     cudaStreamSynchronize(c->s_asm);
     cudaStreamSynchronize(c->s_comp);
+    for (auto st : c->s_slot) cudaStreamSynchronize(st);
     cudaGetLastError();
     return rc;
   }
@@ -841,6 +960,8 @@ int bk_destroy(bk_ctx* c) {
   if (c->s_comp) cudaStreamSynchronize(c->s_comp);
   if (c->s_copy) cudaStreamSynchronize(c->s_copy);
   if (c->s_asm) cudaStreamSynchronize(c->s_asm);
+  for (auto st : c->s_slot)
+    if (st) cudaStreamSynchronize(st);
   unregister(c);
   for (auto& s : c->slots) {
     if (s.copied) cudaEventDestroy(s.copied);
@@ -858,9 +979,14 @@ int bk_destroy(bk_ctx* c) {
   if (c->t_begin) cudaEventDestroy(c->t_begin);
   if (c->t_end) cudaEventDestroy(c->t_end);
   for (cudaEvent_t e : c->prof) cudaEventDestroy(e);
+  delete c->pool;
+  for (auto* h : c->hstage) cudaFreeHost(h);
+  for (auto e : c->h_done) cudaEventDestroy(e);
   if (c->s_copy) cudaStreamDestroy(c->s_copy);
   if (c->s_asm) cudaStreamDestroy(c->s_asm);
   if (c->s_comp) cudaStreamDestroy(c->s_comp);
+  for (auto st : c->s_slot)
+    if (st) cudaStreamDestroy(st);
   cudaGetLastError();
   delete c;
   return BK_OK;

@@ -1,0 +1,189 @@
+// host_gather.cpp — CPU assembly of one chunk into the warp-tile layout (see host_gather.h).
+// The lane rule and the tile layout are the ones k_addrgen / k_gather_* implement on the GPU
+// (DESIGN.md §1, §2 A4); tests/test_gpu_parity.py checks the staged bytes of every gather mode
+// against the layout definition.
+#include "host_gather.h"
+
+#include <immintrin.h>
+
+#include <algorithm>
+#include <cstring>
+
+namespace bk {
+
+HostPool::HostPool(int threads) {
+  if (threads < 1) threads = 1;
+  for (int i = 0; i + 1 < threads; ++i) workers_.emplace_back([this, i] { loop(i); });
+}
+
+HostPool::~HostPool() {
+  {
+    std::lock_guard<std::mutex> g(m_);
+    stop_ = true;
+  }
+  cv_.notify_all();
+  for (auto& t : workers_) t.join();
+}
+
+void HostPool::loop(int tid) {
+  uint64_t seen = 0;
+  for (;;) {
+    std::function<void(int)> job;
+    {
+      std::unique_lock<std::mutex> l(m_);
+      cv_.wait(l, [&] { return stop_ || gen_ != seen; });
+      if (stop_) return;
+      seen = gen_;
+      job = job_;
+    }
+    job(tid);
+    {
+      std::lock_guard<std::mutex> g(m_);
+      if (--pending_ == 0) done_.notify_all();
+    }
+  }
+}
+
+void HostPool::run(const std::function<void(int)>& f) {
+  {
+    std::lock_guard<std::mutex> g(m_);
+    job_ = f;
+    pending_ = (int)workers_.size();
+    ++gen_;
+  }
+  cv_.notify_all();
+  f((int)workers_.size());
+  std::unique_lock<std::mutex> l(m_);
+  done_.wait(l, [&] { return pending_ == 0; });
+}
+
+namespace {
+
+inline uint64_t rstart(const HostData& d, uint64_t r) {
+  if (!d.off) return r * d.rec_size;
+  return r < d.n ? d.off[r] : d.nbytes;
+}
+
+// A(lo, r) of the access spec (k_addrgen's acc_bytes)
+inline uint64_t acc(const HostData& d, const Access& a, const Chunk& c, uint64_t r) {
+  if (!a.whole) return (r - c.lo) * a.E;
+  if (!d.off) return (r - c.lo) * d.rec_size;
+  return (r == c.hi ? c.end_byte : d.off[r]) - c.base_byte;
+}
+
+// first(t) = min{ r in [lo,hi] : A(lo,r) >= floor(t*A/L) } (k_addrgen's lane_first)
+inline uint64_t lane_first(const HostData& d, const Access& a, const Chunk& c, uint64_t t) {
+  if (t >= c.L) return c.hi;
+  const uint64_t target = t * c.accessed / c.L;
+  if (a.whole && d.off) {
+    uint64_t lo = c.lo, hi = c.hi;
+    while (lo < hi) {
+      const uint64_t mid = lo + (hi - lo) / 2;
+      if (acc(d, a, c, mid) >= target) hi = mid; else lo = mid + 1;
+    }
+    return lo;
+  }
+  const uint64_t per = a.whole ? d.rec_size : a.E;
+  if (per == 0) return c.lo;
+  const uint64_t k = (target + per - 1) / per;
+  return std::min(c.lo + k, c.hi);
+}
+
+}  // namespace
+
+uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* stage,
+                           uint64_t cap, std::vector<uint64_t>& first, std::vector<uint64_t>& tbase) {
+  const uint32_t L = c.L, T = c.ntiles;
+  first.resize((size_t)L + 1);
+  tbase.resize((size_t)T + 1);
+  const int P = pool.size();
+  // 1. lane bounds and per-tile K_w (parallel over tiles)
+  pool.run([&](int tid) {
+    const uint64_t per = (T + P - 1) / P;
+    for (uint64_t w = tid * per; w < std::min<uint64_t>(T, (tid + 1) * per); ++w) {
+      uint64_t K = 0, prev = lane_first(d, a, c, (uint32_t)(w * 32));
+      first[w * 32] = prev;
+      for (uint32_t i = 0; i < 32; ++i) {
+        const uint64_t t = w * 32 + i;
+        const uint64_t nx = lane_first(d, a, c, t + 1);
+        first[t + 1] = nx;
+        const uint64_t b = acc(d, a, c, nx) - acc(d, a, c, prev);
+        K = std::max<uint64_t>(K, (b + 15) / 16);
+        prev = nx;
+      }
+      tbase[w] = K;
+    }
+  });
+  // 2. exclusive scan of 512 * K_w
+  uint64_t size = 0;
+  for (uint32_t w = 0; w < T; ++w) {
+    const uint64_t K = tbase[w];
+    tbase[w] = size;
+    size += 512 * K;
+  }
+  tbase[T] = size;
+  if (size > cap) return UINT64_MAX;
+  // 3. fill: each tile is assembled in a thread-local buffer (lane-outer: every lane's records are
+  // read in address order, scattered 16-B stores stay in L1), then streamed to the pinned staging
+  // slot with non-temporal 16-B stores (no read-for-ownership; the CPU never reads it again).
+  const bool fast = !a.whole && a.n_ext == 1 && (a.E % 16) == 0 && a.E > 0;
+  const uint32_t EW = a.E / 16, eo = a.n_ext ? a.ext_off[0] : 0;
+  std::atomic<uint32_t> next{0};
+  pool.run([&](int) {
+    std::vector<__m128i> tl;
+    for (;;) {
+      const uint32_t w0 = next.fetch_add(16);
+      if (w0 >= T) break;
+      for (uint32_t w = w0; w < std::min(T, w0 + 16); ++w) {
+        const uint64_t K = (tbase[w + 1] - tbase[w]) / 512;
+        if (tl.size() < K * 32) tl.resize(K * 32);
+        uint8_t* tile = reinterpret_cast<uint8_t*>(tl.data());
+        memset(tile, 0, K * 512);
+        if (fast) {
+          // the tile's lanes are consecutive record ranges: walk them in address order with a
+          // software prefetch kPf records ahead across lane boundaries (lanes are only ~8 records)
+          constexpr uint64_t kPf = 16;
+          const uint64_t r0 = first[(uint64_t)w * 32], r1 = first[(uint64_t)w * 32 + 32];
+          auto rsrc = [&](uint64_t r) { return d.base + (d.off ? d.off[r] : r * d.rec_size) + eo; };
+          for (uint64_t r = r0; r < std::min(r1, r0 + kPf); ++r) __builtin_prefetch(rsrc(r));
+          int i = 0;
+          uint64_t lane_end = first[(uint64_t)w * 32 + 1], k = 0;
+          for (uint64_t r = r0; r < r1; ++r) {
+            while (r >= lane_end) {  // next non-empty lane
+              ++i;
+              k = 0;
+              lane_end = first[(uint64_t)w * 32 + i + 1];
+            }
+            if (r + kPf < r1) __builtin_prefetch(rsrc(r + kPf));
+            const uint8_t* srcp = rsrc(r);
+            for (uint32_t m = 0; m < EW; ++m, ++k) memcpy(tile + (k * 32 + i) * 16, srcp + 16 * m, 16);
+          }
+        }
+        for (int i = 0; i < 32 && !fast; ++i) {
+          const uint64_t t = (uint64_t)w * 32 + i;
+          const uint64_t f = first[t], nr = first[t + 1] - f;
+          if (a.whole) {
+            const uint64_t nb = acc(d, a, c, first[t + 1]) - acc(d, a, c, f);
+            const uint8_t* src = d.base + rstart(d, f);
+            for (uint64_t b = 0, k = 0; b < nb; b += 16, ++k)
+              memcpy(tile + (k * 32 + i) * 16, src + b, std::min<uint64_t>(16, nb - b));
+          } else {
+            uint64_t b = 0;
+            for (uint64_t j = 0; j < nr; ++j) {
+              const uint64_t rs = rstart(d, f + j);
+              for (uint32_t e = 0; e < a.n_ext; ++e)
+                for (uint32_t x = 0; x < a.ext_len[e]; ++x, ++b)
+                  tile[((b / 16) * 32 + i) * 16 + b % 16] = d.base[rs + a.ext_off[e] + x];
+            }
+          }
+        }
+        __m128i* dst = reinterpret_cast<__m128i*>(stage + tbase[w]);
+        for (uint64_t q = 0; q < K * 32; ++q) _mm_stream_si128(dst + q, tl[q]);
+      }
+    }
+    _mm_sfence();
+  });
+  return size;
+}
+
+}  // namespace bk

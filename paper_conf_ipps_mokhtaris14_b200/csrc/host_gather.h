@@ -1,0 +1,49 @@
+// host_gather.h — CPU assembly (stage 2 on the host, PAPER.md P:273-275, P:421-441, P:691-695,
+// §IV.B): a persistent thread pool packs exactly the accessed bytes of a chunk into a
+// pinned staging buffer in the same warp-tile layout the GPU gather produces, so stage 3 is one
+// large DMA of payload bytes only. Product code (libbk): shares no code with the CPU reference under tests.
+#pragma once
+#include <stdint.h>
+
+#include <atomic>
+#include <condition_variable>
+#include <functional>
+#include <mutex>
+#include <thread>
+#include <vector>
+
+#include "bk_internal.cuh"
+
+namespace bk {
+
+class HostPool {
+ public:
+  explicit HostPool(int threads);
+  ~HostPool();
+  int size() const { return (int)workers_.size() + 1; }
+  // Runs f(tid) on every worker and on the caller (tid = size()-1); returns when all finished.
+  void run(const std::function<void(int)>& f);
+
+ private:
+  void loop(int tid);
+  std::vector<std::thread> workers_;
+  std::mutex m_;
+  std::condition_variable cv_, done_;
+  std::function<void(int)> job_;
+  uint64_t gen_ = 0;
+  int pending_ = 0;
+  bool stop_ = false;
+};
+
+struct HostData {
+  const uint8_t* base;     // registered data set
+  const uint64_t* off;     // record offsets (NULL = fixed records)
+  uint64_t n, nbytes, rec_size;
+};
+
+// Packs chunk c into `stage` (capacity cap) with the lane rule of k_addrgen and the tile layout
+// of k_gather_*; returns the staged size, or UINT64_MAX if it would exceed cap.
+uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* stage,
+                           uint64_t cap, std::vector<uint64_t>& first_scratch, std::vector<uint64_t>& tile_scratch);
+
+}  // namespace bk

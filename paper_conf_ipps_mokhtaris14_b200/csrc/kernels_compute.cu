@@ -52,65 +52,145 @@ __device__ void wc_insert(WcEntry* table, uint64_t mask, unsigned long long key1
   atomicOr(err, kErrTableFull);
 }
 
-__device__ __forceinline__ void wc_emit(WcEntry* table, uint64_t mask, uint64_t h1, uint64_t h2, uint32_t len,
-                                        uint64_t occ, unsigned long long* used, int* err) {
-  const unsigned long long key1 = mix64(h1 ^ ((uint64_t)len * 0x9E3779B97F4A7C15ull)) | 1ull;
-  const unsigned long long key2 = mix64(h2 + len) | 1ull;
-  if (len >= (1u << 24) || occ >= (1ull << 40)) atomicOr(err, kErrWordTooLong);
-  const unsigned long long offlen = (occ << 24) | len;
-  const unsigned act = __activemask();
-  const unsigned m = __match_any_sync(act, key1) & __match_any_sync(act, key2);
-  const int lane = threadIdx.x & 31;
-  if (lane == __ffs(m) - 1) wc_insert(table, mask, key1, key2, offlen, __popc(m), used, err);
-}
+// Per-block shared-memory pre-aggregation (Zipf text: most occurrences hit a few hot words).
+constexpr int kWcBlock = 128;   // 4 warps: small blocks spread a chunk's few lanes over more SMs
+constexpr int kWcTab = 1024;    // block table slots
+constexpr int kWcQ = 160;       // per-warp queue of finished words (static smem < 48 KB)
 
-__global__ void __launch_bounds__(256) k_wc(Chunk c, const uint8_t* __restrict__ stage,
-                                            const LaneDesc* __restrict__ lanes,
-                                            const uint64_t* __restrict__ tile_base,
-                                            const uint64_t* __restrict__ meta, uint64_t rec_size,
-                                            WcEntry* table, uint64_t mask, unsigned long long* used, int* err) {
-  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-  if (t >= c.L) return;
-  const int lane = t & 31;
-  const LaneDesc d = lanes[t];
-  const uint8_t* tile = stage + tile_base[t >> 5];
-  auto rstart = [&](uint64_t r) -> uint64_t {
-    if (rec_size) return r * rec_size;
-    return r == c.hi ? c.end_byte : meta[r - c.lo];
-  };
-  const uint64_t lane_start = rstart(d.first);
-  const uint64_t rend = d.first + d.nrec;
-  uint64_t r = d.first + 1;
-  uint64_t next_b = r < rend ? rstart(r) - lane_start : ~0ull;
-  bool in_word = false;
-  uint64_t h1 = 0, h2 = 0, wstart = 0;
-  uint32_t wlen = 0;
-  const uint32_t W = (d.nbytes + 15) >> 4;
-  for (uint32_t k = 0; k < W; ++k) {
-    const uint4 v = lane_word(tile, k, lane);
-    const uint32_t wd[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      const uint64_t pos = (uint64_t)k * 16 + q;
-      if (pos >= d.nbytes) break;
-      while (pos == next_b) {  // record boundary (several if records are empty)
-        if (in_word) { wc_emit(table, mask, h1, h2, wlen, lane_start + wstart, used, err); in_word = false; }
-        ++r;
-        next_b = r < rend ? rstart(r) - lane_start : ~0ull;
+struct WcShared {
+  unsigned long long k1[kWcTab], k2[kWcTab], ol[kWcTab];
+  unsigned int cnt[kWcTab];
+  unsigned long long qk1[kWcBlock / 32][kWcQ], qk2[kWcBlock / 32][kWcQ], qol[kWcBlock / 32][kWcQ];
+  int qn[kWcBlock / 32];
+};
+
+__device__ void tab_insert(WcShared& sh, WcEntry* table, uint64_t mask, unsigned long long k1,
+                           unsigned long long k2, unsigned long long ol, unsigned int cnt,
+                           unsigned long long* used, int* err) {
+  uint32_t s = (uint32_t)(k1 >> 20) & (kWcTab - 1);
+  for (int p = 0; p < 16; ++p, s = (s + 1) & (kWcTab - 1)) {
+    unsigned long long cur = atomicCAS(&sh.k1[s], 0ull, k1);
+    if (cur == 0) {  // claimed: publish occurrence + key2 (readers spin until key2 != 0)
+      sh.ol[s] = ol;
+      __threadfence_block();
+      atomicExch(&sh.k2[s], k2);
+      atomicAdd(&sh.cnt[s], cnt);
+      return;
+    }
+    if (cur == k1) {
+      unsigned long long c2;
+      while ((c2 = *reinterpret_cast<volatile unsigned long long*>(&sh.k2[s])) == 0) {
       }
-      const uint32_t ch = (wd[q >> 2] >> (8 * (q & 3))) & 0xff;
-      if (is_delim(ch)) {
-        if (in_word) { wc_emit(table, mask, h1, h2, wlen, lane_start + wstart, used, err); in_word = false; }
-      } else {
-        if (!in_word) { in_word = true; wstart = pos; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
-        h1 = (h1 ^ ch) * 0x100000001b3ull;
-        h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
-        h2 ^= h2 >> 29;
-        ++wlen;
+      if (c2 == k2) {
+        atomicAdd(&sh.cnt[s], cnt);
+        return;
       }
     }
   }
-  if (in_word) wc_emit(table, mask, h1, h2, wlen, lane_start + wstart, used, err);
+  wc_insert(table, mask, k1, k2, ol, cnt, used, err);  // block table crowded: go global
+}
+
+// Insert the warp's queued words, 32 at a time, duplicates within a round merged by match_any.
+__device__ __forceinline__ void wc_flush_queue(WcShared& sh, int w, int lane, WcEntry* table, uint64_t mask,
+                                               unsigned long long* used, int* err) {
+  __syncwarp();
+  const int n = min(*reinterpret_cast<volatile int*>(&sh.qn[w]), kWcQ);
+  for (int base = 0; base < n; base += 32) {
+    const int i = base + lane;
+    const bool v = i < n;
+    const unsigned long long k1 = v ? sh.qk1[w][i] : 0, k2 = v ? sh.qk2[w][i] : 0, ol = v ? sh.qol[w][i] : 0;
+    const unsigned m = __match_any_sync(kFull, k1) & __match_any_sync(kFull, k2);
+    if (v && lane == __ffs(m) - 1) tab_insert(sh, table, mask, k1, k2, ol, __popc(m), used, err);
+  }
+  __syncwarp();
+  if (lane == 0) sh.qn[w] = 0;
+  __syncwarp();
+}
+
+__device__ __forceinline__ void wc_push(WcShared& sh, int w, WcEntry* table, uint64_t mask, uint64_t h1,
+                                        uint64_t h2, uint32_t len, uint64_t occ, unsigned long long* used,
+                                        int* err) {
+  const unsigned long long k1 = mix64(h1 ^ ((uint64_t)len * 0x9E3779B97F4A7C15ull)) | 1ull;
+  const unsigned long long k2 = mix64(h2 + len) | 1ull;
+  if (len >= (1u << 24) || occ >= (1ull << 40)) atomicOr(err, kErrWordTooLong);
+  const unsigned long long ol = (occ << 24) | len;
+  const int i = atomicAdd(&sh.qn[w], 1);
+  if (i < kWcQ) {
+    sh.qk1[w][i] = k1;
+    sh.qk2[w][i] = k2;
+    sh.qol[w][i] = ol;
+  } else {
+    tab_insert(sh, table, mask, k1, k2, ol, 1, used, err);  // queue full this step (tiny words)
+  }
+}
+
+// Thread per lane tokenises its bytes (record boundaries from the offsets slice); finished words
+// go to a per-warp shared queue that the whole warp drains after every 16-byte step, so global
+// latency is never on a per-byte critical path.
+__global__ void __launch_bounds__(kWcBlock) k_wc(Chunk c, const uint8_t* __restrict__ stage,
+                                                 const LaneDesc* __restrict__ lanes,
+                                                 const uint64_t* __restrict__ tile_base,
+                                                 const uint64_t* __restrict__ meta, uint64_t rec_size,
+                                                 WcEntry* table, uint64_t mask, unsigned long long* used, int* err) {
+  __shared__ WcShared sh;
+  for (int i = threadIdx.x; i < kWcTab; i += blockDim.x) { sh.k1[i] = 0; sh.k2[i] = 0; sh.cnt[i] = 0; }
+  if (threadIdx.x < kWcBlock / 32) sh.qn[threadIdx.x] = 0;
+  __syncthreads();
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const bool live = t < c.L;   // L % 32 == 0: whole warps are live or not
+  if (live) {
+    const LaneDesc d = lanes[t];
+    const uint8_t* tile = stage + tile_base[t >> 5];
+    auto rstart = [&](uint64_t r) -> uint64_t {
+      if (rec_size) return r * rec_size;
+      return r == c.hi ? c.end_byte : meta[r - c.lo];
+    };
+    const uint64_t lane_start = rstart(d.first);
+    const uint64_t rend = d.first + d.nrec;
+    uint64_t r = d.first + 1;
+    uint32_t next_b = r < rend ? (uint32_t)(rstart(r) - lane_start) : 0xffffffffu;
+    bool in_word = false;
+    uint64_t h1 = 0, h2 = 0;
+    uint32_t wstart = 0, wlen = 0;
+    const uint32_t W = (d.nbytes + 15) >> 4;
+    const uint32_t Kw = __reduce_max_sync(kFull, W);
+    for (uint32_t k = 0; k < Kw; ++k) {
+      if (k < W) {
+        const uint4 v = lane_word(tile, k, lane);
+        const uint32_t lim = min(16u, d.nbytes - 16 * k);
+#pragma unroll 1
+        for (uint32_t q = 0; q < lim; ++q) {
+          const uint32_t pos = 16 * k + q;
+          const uint32_t wd = q < 8 ? (q < 4 ? v.x : v.y) : (q < 12 ? v.z : v.w);
+          const uint32_t ch = (wd >> (8 * (q & 3))) & 0xff;
+          bool boundary = pos == next_b;
+          while (pos == next_b) {  // several if records are empty
+            ++r;
+            next_b = r < rend ? (uint32_t)(rstart(r) - lane_start) : 0xffffffffu;
+          }
+          const bool delim = is_delim(ch);
+          if (in_word && (delim || boundary)) {
+            wc_push(sh, w, table, mask, h1, h2, wlen, lane_start + wstart, used, err);
+            in_word = false;
+          }
+          if (!delim) {
+            if (!in_word) { in_word = true; wstart = pos; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
+            h1 = (h1 ^ ch) * 0x100000001b3ull;
+            h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
+            h2 ^= h2 >> 29;
+            ++wlen;
+          }
+        }
+      }
+      wc_flush_queue(sh, w, lane, table, mask, used, err);
+    }
+    if (in_word) wc_push(sh, w, table, mask, h1, h2, wlen, lane_start + wstart, used, err);
+    wc_flush_queue(sh, w, lane, table, mask, used, err);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < kWcTab; i += blockDim.x)
+    if (sh.k1[i]) wc_insert(table, mask, sh.k1[i], sh.k2[i], sh.ol[i], sh.cnt[i], used, err);
 }
 
 __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, unsigned long long* n_out,
@@ -404,7 +484,8 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
 void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                int* err, cudaStream_t s) {
-  k_wc<<<(c.L + 255) / 256, 256, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
+  k_wc<<<(c.L + kWcBlock - 1) / kWcBlock, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask,
+                                                           used, err);
 }
 
 void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,

@@ -49,7 +49,7 @@ def layout_data(name):
 
 
 @pytest.mark.parametrize("name,extents,rs", LAYOUT_CASES)
-@pytest.mark.parametrize("mode", ["zc", "dense"])
+@pytest.mark.parametrize("mode", ["zc", "dense", "cpu"])
 @pytest.mark.parametrize("lanes", [32, 160])
 def test_layout_dump_matches_oracle(name, extents, rs, mode, lanes):
     buf, off, rs = layout_data(name)
@@ -59,7 +59,7 @@ def test_layout_dump_matches_oracle(name, extents, rs, mode, lanes):
                     record_size=rs) as ctx:
         ctx.register(buf, off, n_records=n)
         # the plan budget counts accessed bytes in zc mode, whole records in dense mode
-        plan_ext = extents if mode == "zc" else None
+        plan_ext = None if mode == "dense" else extents
         bounds = oracle.plan_chunks(off, n, len(buf), rs, plan_ext, chunk)
         first = ctx.layout_dump(0, extents)
         assert first["n_chunks"] == len(bounds) - 1 >= 3
@@ -74,7 +74,7 @@ def test_layout_dump_matches_oracle(name, extents, rs, mode, lanes):
 
 
 # ------------------------------------------------------------------ C1 word count
-@pytest.mark.parametrize("mode", ["dense", "zc"])
+@pytest.mark.parametrize("mode", ["dense", "zc", "cpu", "hybrid"])
 @pytest.mark.parametrize("window,slots", [(256 * 1024, 2), (1 * MIB, 4), (8 * MIB, 3)])
 def test_wordcount_small(mode, window, slots):
     buf, off = gen.text(cap_bytes=2 * MIB)
@@ -92,7 +92,7 @@ def test_wordcount_adversarial():
     buf = np.frombuffer(b"".join(recs), np.uint8)
     off = np.cumsum([0] + [len(r) for r in recs[:-1]]).astype(np.uint64)
     want = oracle.wc(buf, off)
-    for mode in ("zc", "dense"):
+    for mode in ("zc", "dense", "cpu", "hybrid"):
         with bk.Context(window_bytes=64 * 1024, n_slots=2, gather_mode=mode, chunk_bytes=1500, lanes=32) as ctx:
             ctx.register(buf, off)
             assert wc_multiset_gpu(buf, *ctx.wordcount(cap=4096)) == want
@@ -130,14 +130,14 @@ def test_grep_adversarial():
                     ctx.grep(pat)
             continue
         want = oracle.grep(buf, off, pat)
-        for mode in ("zc", "dense"):
+        for mode in ("zc", "dense", "cpu", "hybrid"):
             with bk.Context(window_bytes=256 * 1024, n_slots=2, gather_mode=mode, chunk_bytes=2048, lanes=64) as ctx:
                 ctx.register(buf, off)
                 got = ctx.grep(pat, cap=len(off))
             assert np.array_equal(got, want), (pat, mode)
 
 
-@pytest.mark.parametrize("mode", ["zc", "dense"])
+@pytest.mark.parametrize("mode", ["zc", "dense", "cpu", "hybrid"])
 def test_grep_medium(mode):
     buf, off = gen.grep_records(max_bytes=64 * MIB)
     want = oracle.grep(buf, off, b"bigk", first=1000)
@@ -149,6 +149,11 @@ def test_grep_medium(mode):
     assert st["n_chunks"] >= 8
     if mode == "zc":
         assert st["bytes_accessed"] == 32 * len(off) == st["bytes_h2d"]   # I3: only the key bytes
+    if mode == "cpu":
+        assert st["n_chunks_cpu"] == st["n_chunks"] and st["bytes_meta"] == 0
+        assert 32 * len(off) <= st["bytes_h2d"] <= 32 * len(off) * 1.05  # packed keys + tile padding
+    if mode == "hybrid":
+        assert 0 < st["n_chunks_cpu"] < st["n_chunks"]
 
 
 def test_grep_capacity_error():
@@ -175,7 +180,7 @@ def test_grep_full_c2_config():
 
 # ------------------------------------------------------------------ C5 group-by
 @pytest.mark.parametrize("stride,zipf,mode", [(16, False, "dense"), (16, True, "zc"), (64, False, "zc"),
-                                              (64, True, "dense")])
+                                              (64, True, "dense"), (64, False, "cpu"), (16, True, "hybrid")])
 def test_groupby(stride, zipf, mode):
     n = 3_000_001
     buf = gen.groupby(n=n, stride=stride, zipf=zipf)
@@ -198,7 +203,7 @@ def test_groupby_key_out_of_range():
 
 
 # ------------------------------------------------------------------ C3 k-means
-@pytest.mark.parametrize("mode,K", [("dense", 64), ("zc", 64), ("dense", 7)])
+@pytest.mark.parametrize("mode,K", [("dense", 64), ("zc", 64), ("dense", 7), ("cpu", 64), ("hybrid", 33)])
 def test_kmeans(mode, K):
     n = 400_003
     x = gen.points(n=n)
@@ -217,7 +222,8 @@ def test_invariance_across_window_slots_lanes_modes():
     buf, off = gen.text(cap_bytes=1 * MIB)
     want = oracle.wc(buf, off)
     for window, slots, lanes, mode in [(128 * 1024, 2, 0, "zc"), (300_000, 3, 64, "dense"), (4 * MIB, 8, 0, "zc"),
-                                       (4 * MIB, 2, 1024, "dense")]:
+                                       (4 * MIB, 2, 1024, "dense"), (512 * 1024, 4, 96, "cpu"),
+                                       (1 * MIB, 6, 0, "hybrid")]:
         with bk.Context(window_bytes=window, n_slots=slots, lanes=lanes, gather_mode=mode) as ctx:
             ctx.register(buf, off)
             assert wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 17)) == want, (window, slots, lanes, mode)
