@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "kmeans"])
+    ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "kmeans", "partition"])
     ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense", "cpu", "hybrid"])
     ap.add_argument("--gib", type=float, default=None, help="per-GPU data size override (GiB)")
     ap.add_argument("--window-mib", type=int, default=None)
@@ -66,6 +66,8 @@ WORKLOADS = {
     "wordcount": (64 / 1024, 8, "C1 word count: Zipf(1.0) text lines, 65,536-word vocabulary"),
     "groupby": (16.0, 2048, "C5 group-by sum: {u32 key<4096, u32 qty, f64 amount} 16-B records"),
     "kmeans": (16.0, 2048, "C3 k-means step: 16-dim fp32 points, K=64, Forgy init"),
+    "partition": (8.0, 2048, "C4 stable hash partition: {u64 key, u64 value} 16-B records into 1024 buckets, "
+                             "bucket-sorted chunks written back to host (full duplex)"),
 }
 
 
@@ -85,6 +87,11 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
         n = nbytes // 16
         buf = gen.groupby(gen.SEED_GROUPBY, first=rank * n, n=n)
         return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=16)
+    if workload == "partition":
+        n = nbytes // 16
+        kv = gen.kv(gen.SEED_KV, first=rank * n, n=n)
+        return dict(buf=kv.view(np.uint8).reshape(-1), off=None, n=n, first=rank * n, rec_size=16,
+                    out=np.empty((n, 2), np.uint64))
     n = nbytes // 64
     x = gen.points(gen.SEED_KMEANS, first=rank * n, n=n)
     return dict(buf=x.view(np.uint8).reshape(-1), off=None, n=n, first=rank * n, rec_size=64,
@@ -176,6 +183,9 @@ def oracle_sample(workload: str, shard: dict, target_s: float):
         elif workload == "groupby":
             end = nrec * 16
             oracle.groupby(buf[:end], nrec, 16, 4096)
+        elif workload == "partition":
+            end = nrec * 16
+            oracle.partition(buf[:end].view(np.uint64).reshape(-1, 2), 1024)
         else:
             end = nrec * 64
             oracle.kmeans(buf[:end].view(np.float32), shard["mu"])
@@ -205,10 +215,16 @@ def main():
     import torch.distributed as dist
     from paper_conf_ipps_mokhtaris14_b200 import bk
 
+    # one process per GPU; BK_BENCH_BACKEND=gloo lets several ranks share one GPU for a smoke test
+    backend = os.environ.get("BK_BENCH_BACKEND", "nccl")
+    local = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
 
     shard = make_shard(args.workload, gib, rank, world)
     peak_h2d = measure_h2d_peak(torch, dev)
@@ -224,27 +240,32 @@ def main():
     cap = max(shard["n"] // 50, 1 << 16)
     idx_out = np.empty(cap, np.uint64)
 
+    from paper_conf_ipps_mokhtaris14_b200 import merge
+
     def one_step():
+        """One pass of the whole hot path over this rank's shard, then the merge (N>1)."""
+        cs = stream.cuda_stream
         if args.workload == "grep":
-            res = ctx.grep(b"bigk", first_index=shard["first"], stream=stream.cuda_stream, out=idx_out)
-            cnt = torch.tensor([len(res)], dtype=torch.int64, device=dev)
-            if world > 1:  # exchange: every rank learns where its ascending run lands globally
-                allc = torch.empty(world, dtype=torch.int64, device=dev)
-                dist.all_gather_into_tensor(allc, cnt)
-                cnt = allc
-            return cnt
+            res = ctx.grep(b"bigk", first_index=shard["first"], stream=cs, out=idx_out)
+            return merge.merge_grep_offsets(len(res)) if world > 1 else (0, len(res))
         if args.workload == "wordcount":
-            o, l, c = ctx.wordcount(cap=1 << 20, stream=stream.cuda_stream)
-            t = torch.tensor([int(c.sum())], dtype=torch.int64, device=dev)
-        elif args.workload == "groupby":
-            c, q, a = ctx.groupby(4096, stream=stream.cuda_stream)
+            o, l, c = ctx.wordcount(cap=1 << 20, stream=cs)
+            if world > 1:
+                b = shard["buf"]
+                return merge.merge_wordcount({b[int(x): int(x) + int(y)].tobytes(): int(z) for x, y, z in zip(o, l, c)})
+            return int(c.sum())
+        if args.workload == "partition":
+            out, cc, bc = ctx.partition(1024, out=shard["out"], stream=cs)
+            return merge.merge_partition_offsets(bc) if world > 1 else bc
+        if args.workload == "groupby":
+            c, q, a = ctx.groupby(4096, stream=cs)
             t = torch.from_numpy(np.stack([c.astype(np.float64), q.astype(np.float64), a])).to(dev)
         else:
-            c, s, chk = ctx.kmeans(shard["mu"], first_index=shard["first"], stream=stream.cuda_stream)
-            t = torch.from_numpy(np.concatenate([c.astype(np.float64), s.reshape(-1)])).to(dev)
-        if world > 1:  # merge of per-GPU aggregates (NCCL over NVLink)
-            dist.all_reduce(t)
-        return t
+            c, s_, chk = ctx.kmeans(shard["mu"], first_index=shard["first"], stream=cs)
+            t = torch.from_numpy(np.concatenate([c.astype(np.float64), s_.reshape(-1)])).to(dev)
+            if world > 1:
+                merge.merge_checksum(chk)
+        return merge.merge_sum(t) if world > 1 else t
 
     for _ in range(args.warmup):
         one_step()
@@ -271,8 +292,8 @@ def main():
     dev_ms = [a.elapsed_time(b) for a, b in ev]
     t_dev = sum(dev_ms) / 1e3
     t_wall = sum(wall)
-    if world > 1:
-        tt = torch.tensor([t_dev, t_wall], dtype=torch.float64, device=dev)
+    if world > 1:  # max over ranks
+        tt = torch.tensor([t_dev, t_wall], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t_dev, t_wall = tt.tolist()
     st = stats[-1]

@@ -203,6 +203,7 @@ class Context:
 
     def register(self, data, offsets=None, n_records=None, nbytes=None):
         self._keep = [data, offsets]
+        self.n = len(offsets) if offsets is not None else (n_records or 0)
         bk_register_segments(self.ctx, data, offsets, nbytes=nbytes, n_records=n_records)
 
     def stats(self) -> dict:
@@ -239,6 +240,18 @@ class Context:
         o.centroids, o.K, o.first_index, o.count, o.sum, o.cid = _ptr(mu), K, first_index, _ptr(cnt), _ptr(s), None
         bk_run(self.ctx, BK_K_KMEANS, stream, o)
         return cnt, s, int(o.chk)
+
+    def partition(self, n_buckets: int = 1024, out=None, chunk_cap: int = 1 << 16, stream=None):
+        """Returns (out u64[n,2] chunk-major bucket-sorted runs, chunk_counts u64[C,B], bucket_count u64[B])."""
+        o = _hdr(bk_out_partition, BK_K_PARTITION)
+        out = out if out is not None else np.empty((self.n, 2), np.uint64)
+        cc = np.empty(chunk_cap * n_buckets, np.uint64)
+        bc = np.empty(n_buckets, np.uint64)
+        o.n_buckets, o.out_records, o.chunk_counts, o.chunk_cap, o.bucket_count = (
+            n_buckets, _ptr(out) if self.n else None, _ptr(cc), chunk_cap, _ptr(bc))
+        bk_run(self.ctx, BK_K_PARTITION, stream, o)
+        C = o.n_chunks
+        return out, cc[: C * n_buckets].reshape(C, n_buckets), bc
 
     def layout_dump(self, chunk: int, extents=None, stage_cap: int = 1 << 26, lane_cap: int = 1 << 20, stream=None):
         o = _hdr(bk_out_layout, BK_K_LAYOUT_DUMP)

@@ -101,4 +101,12 @@ void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, 
 
 cudaError_t configure_compute_kernels();
 
+// ---- C4 partition (kernels_partition.cu): 4 launches per chunk ----
+size_t partition_smem(uint32_t B);
+uint32_t partition_blocks(const Chunk& c);
+void launch_partition(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                      int bits, uint32_t* hist, uint32_t* colpre, unsigned long long* total,
+                      unsigned long long* base, uint8_t* out, cudaStream_t s);
+cudaError_t configure_partition_kernels();
+
 }  // namespace bk

@@ -60,6 +60,7 @@ struct Slot {
   LaneDesc* lanes = nullptr;
   uint32_t* tileK = nullptr;
   uint64_t* tile_base = nullptr;
+  uint8_t* out = nullptr;       // per-chunk output (partition: the bucket-sorted chunk)
   cudaEvent_t copied = nullptr, ready = nullptr, freed = nullptr;
   bool used = false;
 };
@@ -117,6 +118,12 @@ struct bk_ctx {
   uint64_t hstage_cap = 0;
   uint64_t h_next = 0;
   std::vector<uint64_t> scratch_first, scratch_tiles;
+  // partition: D2H stream, per-slot "kernels done" events, resident totals, pinned output cache
+  cudaStream_t s_d2h = nullptr;
+  std::vector<cudaEvent_t> ev_part;
+  DevBuf b_hist, b_colpre, b_totals, b_base;
+  void* out_pinned = nullptr;
+  uint64_t out_pinned_bytes = 0;
   int n_launch = 0;
   bk_stats st{};
 };
@@ -144,7 +151,7 @@ struct Plan {
   uint64_t budget = 0;                 // plan bytes per chunk
   uint32_t L = 0;
   uint64_t max_acc_rec = 0;            // max accessed bytes of one record
-  uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0;
+  uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
   std::vector<uint64_t> bounds;        // chunk record bounds
 };
 
@@ -190,7 +197,7 @@ uint64_t slot_need(const Plan& p) {
   const uint64_t ntiles = p.L / 32;
   return align_up(p.raw_cap, kAlign) + align_up(p.stage_cap, kAlign) + align_up(p.meta_cap * 8, kAlign) +
          align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign) + align_up(ntiles * 4, kAlign) +
-         align_up((ntiles + 1) * 8, kAlign);
+         align_up((ntiles + 1) * 8, kAlign) + align_up(p.out_cap, kAlign);
 }
 
 void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) {
@@ -217,7 +224,7 @@ void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) 
   p.meta_cap = c->off ? maxrecs + 1 : 0;
 }
 
-int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p) {
+int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, bool out_per_chunk = false) {
   p.a = a;
   int mode = (int)c->cfg.gather_mode;
   // AUTO (counters in profiles/): whole-record access -> DENSE (copy engine at
@@ -244,6 +251,7 @@ int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p) {
     int rc = make_chunks(c, p);
     if (rc) return rc;
     size_plan(c, p, budget, lane_target);
+    p.out_cap = out_per_chunk ? budget : 0;
     if (slot_need(p) <= slot) return BK_OK;
     if (!autob) break;
     budget = budget * 3 / 4;
@@ -271,6 +279,8 @@ void carve(bk_ctx* c, const Plan& p) {
     s.tileK = reinterpret_cast<uint32_t*>(q);
     q += align_up(ntiles * 4, kAlign);
     s.tile_base = reinterpret_cast<uint64_t*>(q);
+    q += align_up((ntiles + 1) * 8, kAlign);
+    s.out = p.out_cap ? q : nullptr;
     s.used = false;
   }
 }
@@ -471,10 +481,11 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
     if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(s.ready);
     BK_CUDA(cudaStreamWaitEvent(cs, s.ready, 0));
     BK_PROF(kStCompute, cs, true);
-    rc = compute(chunk_of(c, p, i), s, cs);
+    cudaStream_t rel = cs;   // stream whose completion frees the slot (partition: its D2H)
+    rc = compute(chunk_of(c, p, i), s, cs, rel);
     if (rc) return rc;
     BK_PROF(kStCompute, cs, false);
-    BK_CUDA(cudaEventRecord(s.freed, cs));
+    BK_CUDA(cudaEventRecord(s.freed, rel));
   }
   if (concurrent)  // join: finalize on s_comp after every slot's last compute
     for (auto& s : c->slots)
@@ -559,7 +570,7 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   if ((rc = begin_run(c, stream))) return rc;
   BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
   WcEntry* table = (WcEntry*)c->b_table.p;
-  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
+  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
     launch_wc(ch, s.stage, s.lanes, s.tile_base, s.meta, c->off ? 0 : c->cfg.record_size, table, slots - 1,
               c->d_ctr + 1, c->d_err, cs);
     c->n_launch += 1;
@@ -607,7 +618,7 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
   gp.first_index = o->first_index;
   gp.cap = cap;
   if ((rc = begin_run(c, stream))) return rc;
-  rc = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
+  rc = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
     launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p, c->d_ctr + 3,
                 (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, cs);
     c->n_launch += 3;
@@ -645,7 +656,7 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
   BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)G * 8, c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)G * 8, c->s_comp));
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * per_sm));
-  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
+  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
     launch_groupby(ch, s.stage, s.lanes, s.tile_base, G, (unsigned long long*)c->b_agg1.p,
                    (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, cs);
     c->n_launch += 1;
@@ -680,7 +691,7 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
-  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs) {
+  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
     launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
                   (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4, grid, cs);
     c->n_launch += 1;
@@ -694,6 +705,71 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(cudaMemcpy(&chk, c->d_ctr + 4, 8, cudaMemcpyDeviceToHost));
   o->chk = chk;
   c->st.bytes_d2h = (uint64_t)K * 136;
+  return BK_OK;
+}
+
+int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
+  const uint32_t B = o->n_buckets;
+  if (B == 0 || B > 4096 || (B & (B - 1))) return fail(BK_E_INVAL, "n_buckets must be a power of two in 1..4096");
+  if (c->off || c->cfg.record_size != 16) return fail(BK_E_INVAL, "partition needs fixed 16-byte {key, value} records");
+  if (c->n && !o->out_records) return fail(BK_E_INVAL, "NULL out_records");
+  int bits = 0;
+  while ((1u << bits) < B) ++bits;
+  Plan p;
+  int rc = plan_run(c, whole_access(), 256, p, true);
+  if (rc) return rc;
+  carve(c, p);
+  const uint64_t C = p.bounds.size() - 1;
+  o->n_chunks = C;
+  if (C > o->chunk_cap) return fail(BK_E_CAPACITY, "%llu chunks > chunk_cap %llu", (unsigned long long)C,
+                                    (unsigned long long)o->chunk_cap);
+  uint32_t nblk_max = 1;
+  for (uint64_t i = 0; i < C; ++i) nblk_max = std::max(nblk_max, partition_blocks(chunk_of(c, p, i)));
+  BK_CUDA(c->b_hist.ensure((uint64_t)nblk_max * B * 4));
+  BK_CUDA(c->b_colpre.ensure((uint64_t)nblk_max * B * 4));
+  BK_CUDA(c->b_totals.ensure(std::max<uint64_t>(C, 1) * B * 8));
+  BK_CUDA(c->b_base.ensure((uint64_t)B * 8));
+  // the caller's output is written by DMA: pin it once and keep it pinned across runs
+  const uint64_t out_bytes = c->n * 16;
+  if (out_bytes && (c->out_pinned != o->out_records || c->out_pinned_bytes != out_bytes)) {
+    if (c->out_pinned) cudaHostUnregister(c->out_pinned);
+    c->out_pinned = nullptr;
+    if (!is_pinned(o->out_records)) {
+      BK_CUDA(cudaHostRegister(o->out_records, out_bytes, cudaHostRegisterPortable));
+      c->out_pinned = o->out_records;
+      c->out_pinned_bytes = out_bytes;
+    }
+  }
+  if ((rc = begin_run(c, stream))) return rc;
+  BK_CUDA(cudaStreamWaitEvent(c->s_d2h, c->ev_begin, 0));
+  size_t ci = 0;
+  rc = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
+    launch_partition(ch, s.stage, s.lanes, s.tile_base, bits, (uint32_t*)c->b_hist.p, (uint32_t*)c->b_colpre.p,
+                     (unsigned long long*)c->b_totals.p + ci * B, (unsigned long long*)c->b_base.p, s.out, cs);
+    c->n_launch += 4;
+    cudaEvent_t e = c->ev_part[ci % c->ev_part.size()];
+    BK_CUDA(cudaEventRecord(e, cs));
+    BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
+    const uint64_t bytes = (ch.hi - ch.lo) * 16;
+    if (bytes)
+      BK_CUDA(cudaMemcpyAsync((uint8_t*)o->out_records + ch.lo * 16, s.out, bytes, cudaMemcpyDeviceToHost, c->s_d2h));
+    c->st.bytes_d2h += bytes;
+    rel = c->s_d2h;
+    ++ci;
+    return (int)BK_OK;
+  });
+  if (rc) return rc;
+  BK_CUDA(cudaEventRecord(c->ev_end, c->s_d2h));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
+  if ((rc = end_run(c, stream))) return rc;
+  std::vector<uint64_t> tot(C * B);
+  if (C) BK_CUDA(cudaMemcpy(tot.data(), c->b_totals.p, C * B * 8, cudaMemcpyDeviceToHost));
+  for (uint32_t b = 0; b < B; ++b) o->bucket_count[b] = 0;
+  for (uint64_t i = 0; i < C; ++i)
+    for (uint32_t b = 0; b < B; ++b) {
+      o->chunk_counts[i * B + b] = tot[i * B + b];
+      o->bucket_count[b] += tot[i * B + b];
+    }
   return BK_OK;
 }
 
@@ -814,6 +890,11 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
   if (cudaMalloc(&c->d_err, 256) != cudaSuccess || cudaMalloc(&c->d_ctr, 8 * sizeof(unsigned long long)) != cudaSuccess)
     return cleanup(fail(BK_E_NOMEM, "cudaMalloc scratch"));
   c->slots.resize(c->cfg.n_slots);
+  if (cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "d2h stream"));
+  if (configure_partition_kernels() != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
+  c->ev_part.assign(c->cfg.n_slots, nullptr);
+  for (auto& e : c->ev_part)
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
   c->s_slot.assign(c->cfg.n_slots, nullptr);
   for (auto& st : c->s_slot)
     if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "slot streams"));
@@ -922,7 +1003,9 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
       rc = run_layout(c, (bk_out_layout*)out, stream);
       break;
     case BK_K_PARTITION:
-      return fail(BK_E_UNSUPPORTED, "partition is not in this build yet");
+      if (h->struct_size != sizeof(bk_out_partition)) return fail(BK_E_INVAL, "bk_out_partition size");
+      rc = run_partition(c, (bk_out_partition*)out, stream);
+      break;
     default:
       return fail(BK_E_UNSUPPORTED, "unknown kernel_id %d", kernel_id);
   }
@@ -980,6 +1063,13 @@ int bk_destroy(bk_ctx* c) {
   if (c->t_end) cudaEventDestroy(c->t_end);
   for (cudaEvent_t e : c->prof) cudaEventDestroy(e);
   delete c->pool;
+  if (c->s_d2h) {
+    cudaStreamSynchronize(c->s_d2h);
+    cudaStreamDestroy(c->s_d2h);
+  }
+  for (auto e : c->ev_part) cudaEventDestroy(e);
+  if (c->out_pinned) cudaHostUnregister(c->out_pinned);
+  for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base}) b->release();
   for (auto* h : c->hstage) cudaFreeHost(h);
   for (auto e : c->h_done) cudaEventDestroy(e);
   if (c->s_copy) cudaStreamDestroy(c->s_copy);

@@ -217,6 +217,48 @@ def test_kmeans(mode, K):
     np.testing.assert_allclose(s, ws, rtol=1e-5, atol=0)
 
 
+# ------------------------------------------------------------------ C4 partition
+def global_from_runs(out, cc):
+    """Stable global partition from chunk-major bucket-sorted runs: bucket b = chunk 0's run of b,
+    then chunk 1's, ... (chunks ascend in record order)."""
+    C, B = cc.shape
+    starts = np.zeros((C, B), np.int64)
+    lo = 0
+    for c in range(C):
+        starts[c] = lo + np.concatenate([[0], np.cumsum(cc[c].astype(np.int64))[:-1]])
+        lo += int(cc[c].sum())
+    parts = [out[starts[c, b]: starts[c, b] + int(cc[c, b])] for b in range(B) for c in range(C) if cc[c, b]]
+    return np.concatenate(parts) if parts else out[:0]
+
+
+@pytest.mark.parametrize("B,mode,n", [(1024, "dense", 1_000_003), (1024, "zc", 300_001), (1, "dense", 100_000),
+                                      (4096, "cpu", 200_000), (16, "hybrid", 500_000)])
+def test_partition(B, mode, n):
+    kv = gen.kv(n=n)
+    wboff, wout = oracle.partition(kv, B)
+    with bk.Context(window_bytes=8 * MIB, gather_mode=mode, record_size=16) as ctx:
+        ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=n)
+        out, cc, bc = ctx.partition(B)
+        st = ctx.stats()
+    assert cc.shape[0] == st["n_chunks"] >= 2
+    assert np.array_equal(np.concatenate([[0], np.cumsum(bc)]).astype(np.uint64), wboff)
+    assert np.array_equal(global_from_runs(out, cc), wout)
+    assert st["bytes_d2h"] == 16 * n
+
+
+def test_partition_duplicate_keys_and_errors():
+    kv = np.array([[7, i] for i in range(5000)] + [[9, i] for i in range(5000, 7000)], np.uint64)
+    with bk.Context(window_bytes=1 * MIB, record_size=16) as ctx:
+        ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=len(kv))
+        out, cc, bc = ctx.partition(1024)
+        assert np.array_equal(global_from_runs(out, cc), oracle.partition(kv, 1024)[1])
+        with pytest.raises(bk.BkError):
+            ctx.partition(1000)
+        with pytest.raises(bk.BkError) as e:
+            ctx.partition(1024, chunk_cap=1)
+        assert e.value.status == bk.BK_E_CAPACITY
+
+
 # ------------------------------------------------------------------ invariants + API errors
 def test_invariance_across_window_slots_lanes_modes():
     buf, off = gen.text(cap_bytes=1 * MIB)
