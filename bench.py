@@ -47,13 +47,15 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "kmeans", "partition"])
+    ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "groupby_sparse", "kmeans",
+                                                             "partition"])
     ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense", "cpu", "hybrid"])
     ap.add_argument("--gib", type=float, default=None, help="per-GPU data size override (GiB)")
     ap.add_argument("--window-mib", type=int, default=None)
     ap.add_argument("--slots", type=int, default=0)
     ap.add_argument("--host-threads", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-dbuf", action="store_true", help="skip the double-buffering baseline measurement")
     ap.add_argument("--no-profile", action="store_true", help="disable per-stage event timing")
     return ap.parse_args()
 
@@ -65,6 +67,8 @@ WORKLOADS = {
                          "pattern 'bigk' (1% planted), ordered match indices"),
     "wordcount": (64 / 1024, 8, "C1 word count: Zipf(1.0) text lines, 65,536-word vocabulary"),
     "groupby": (16.0, 2048, "C5 group-by sum: {u32 key<4096, u32 qty, f64 amount} 16-B records"),
+    "groupby_sparse": (16.0, 2048, "C5 sparse variant: the same 16 B inside 64-B records (25% read, like Table I "
+                                   "MCA-indexed P:929)"),
     "kmeans": (16.0, 2048, "C3 k-means step: 16-dim fp32 points, K=64, Forgy init"),
     "partition": (8.0, 2048, "C4 stable hash partition: {u64 key, u64 value} 16-B records into 1024 buckets, "
                              "bucket-sorted chunks written back to host (full duplex)"),
@@ -83,10 +87,11 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
     if workload == "wordcount":
         buf, off = gen.text(gen.SEED_WC + rank, cap_bytes=nbytes)
         return dict(buf=buf, off=off, n=len(off), first=0, rec_size=0)
-    if workload == "groupby":
-        n = nbytes // 16
-        buf = gen.groupby(gen.SEED_GROUPBY, first=rank * n, n=n)
-        return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=16)
+    if workload in ("groupby", "groupby_sparse"):
+        stride = 16 if workload == "groupby" else 64
+        n = nbytes // stride
+        buf = gen.groupby(gen.SEED_GROUPBY, first=rank * n, n=n, stride=stride)
+        return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=stride)
     if workload == "partition":
         n = nbytes // 16
         kv = gen.kv(gen.SEED_KV, first=rank * n, n=n)
@@ -180,9 +185,9 @@ def oracle_sample(workload: str, shard: dict, target_s: float):
         elif workload == "wordcount":
             end = int(off[nrec]) if nrec < len(off) else len(buf)
             oracle.wc(buf[:end], off[:nrec])
-        elif workload == "groupby":
-            end = nrec * 16
-            oracle.groupby(buf[:end], nrec, 16, 4096)
+        elif workload in ("groupby", "groupby_sparse"):
+            end = nrec * shard["rec_size"]
+            oracle.groupby(buf[:end], nrec, shard["rec_size"], 4096)
         elif workload == "partition":
             end = nrec * 16
             oracle.partition(buf[:end].view(np.uint64).reshape(-1, 2), 1024)
@@ -257,7 +262,7 @@ def main():
         if args.workload == "partition":
             out, cc, bc = ctx.partition(1024, out=shard["out"], stream=cs)
             return merge.merge_partition_offsets(bc) if world > 1 else bc
-        if args.workload == "groupby":
+        if args.workload in ("groupby", "groupby_sparse"):
             c, q, a = ctx.groupby(4096, stream=cs)
             t = torch.from_numpy(np.stack([c.astype(np.float64), q.astype(np.float64), a])).to(dev)
         else:
@@ -367,6 +372,38 @@ def main():
         "clocks": clk.summary(),
         "register_s": round(reg_s, 3),
     }
+    if args.workload in ("grep", "groupby", "groupby_sparse") and not args.no_dbuf:
+        # the paper's GPU double-buffering baseline (variant iv) on the same data, window and box
+        dctx = bk.Context(device=local, window_bytes=window, baseline_dbuf=True, profile=False,
+                          record_size=shard["rec_size"])
+        dctx.register(shard["buf"], shard["off"], n_records=shard["n"])
+        dsteps = max(1, min(args.steps, 3))
+
+        def dstep():
+            if args.workload == "grep":
+                dctx.grep(b"bigk", first_index=shard["first"], stream=stream.cuda_stream, out=idx_out)
+            else:
+                dctx.groupby(4096, stream=stream.cuda_stream)
+
+        dstep()
+        torch.cuda.synchronize()
+        a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a_.record(stream)
+        for _ in range(dsteps):
+            dstep()
+        b_.record(stream)
+        b_.synchronize()
+        dt = a_.elapsed_time(b_) / 1e3
+        if world > 1:
+            tt = torch.tensor([dt], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            dt = tt.item()
+        dv = nbytes * world * dsteps / dt / 1e9
+        line["baseline_dbuf"] = {"value": round(dv, 3), "unit": "GB/s", "steps": dsteps,
+                                 "what": "cudaMemcpyAsync double buffering of whole-record chunks (2 x window/2, "
+                                         "2 streams) + the same computation per thread-range (PAPER.md P:329-339, P:994-996)",
+                                 "bigkernel_speedup": round(value / dv, 3)}
+        dctx.close()
     if rank == 0 and not args.no_cpu_baseline:
         gbs, sample, secs = oracle_sample(args.workload, shard, 10.0)
         line["cpu_baseline"] = {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",

@@ -80,6 +80,10 @@ typedef struct bk_config {
 } bk_config;
 
 #define BK_FLAG_PROFILE 1u  /* time every stage of every chunk with CUDA events (bk_stats.ms_*) */
+#define BK_FLAG_BASELINE_DBUF 2u  /* run the paper's GPU double-buffering baseline instead (P:329-339,
+                                     P:994-996): raw whole-record chunks into 2 buffers (window/2 each)
+                                     on 2 streams, kernel over contiguous per-thread record ranges.
+                                     BK_K_GREP and BK_K_GROUPBY only; results identical. */
 
 typedef struct bk_ctx bk_ctx;
 

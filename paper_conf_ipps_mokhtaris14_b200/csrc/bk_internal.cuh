@@ -109,4 +109,14 @@ void launch_partition(const Chunk& c, const uint8_t* stage, const LaneDesc* lane
                       unsigned long long* base, uint8_t* out, cudaStream_t s);
 cudaError_t configure_partition_kernels();
 
+// ---- the paper's double-buffering baseline (kernels_baseline.cu) ----
+uint32_t dbuf_blocks();
+void launch_dbuf_grep(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
+                      uint64_t end_byte, uint64_t rec_size, const GrepParams& p, uint32_t* blkcnt,
+                      unsigned long long* running, unsigned long long* blkbase, uint64_t* out, cudaStream_t s);
+void launch_dbuf_groupby(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t base_byte, uint64_t rec_size,
+                         uint32_t G, unsigned long long* count, unsigned long long* qty, double* amount, int* err,
+                         cudaStream_t s);
+cudaError_t configure_baseline_kernels();
+
 }  // namespace bk

@@ -773,6 +773,116 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
   return BK_OK;
 }
 
+// ---- BK_FLAG_BASELINE_DBUF: the traditional chunked loop with two buffers ----
+int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
+  if (kid != BK_K_GREP && kid != BK_K_GROUPBY) return fail(BK_E_UNSUPPORTED, "dbuf baseline: grep / group-by only");
+  Plan p;
+  p.a = whole_access();
+  p.mode = BK_GATHER_DENSE;
+  p.zero_copy = 0;
+  const uint64_t half = c->cfg.window_bytes / 2 / kAlign * kAlign;
+  uint64_t budget = std::max<uint64_t>(std::min<uint64_t>(half, std::max<uint64_t>(c->nbytes / 32, 1ull << 20)), 1);
+  uint64_t meta_cap = 0;
+  for (int it = 0;; ++it) {
+    p.budget = budget;
+    int rc = make_chunks(c, p);
+    if (rc) return rc;
+    uint64_t maxrecs = 0;
+    for (size_t i = 0; i + 1 < p.bounds.size(); ++i) maxrecs = std::max<uint64_t>(maxrecs, p.bounds[i + 1] - p.bounds[i]);
+    meta_cap = c->off ? maxrecs + 1 : 0;
+    if (align_up(budget + 64, kAlign) + meta_cap * 8 <= half) break;
+    if (it > 64 || budget < 64) return fail(BK_E_NOMEM, "window too small for the dbuf baseline");
+    budget = budget * 3 / 4;
+  }
+  uint8_t* buf[2] = {c->window, c->window + half};
+  uint64_t* meta[2] = {reinterpret_cast<uint64_t*>(buf[0] + align_up(budget + 64, kAlign)),
+                       reinterpret_cast<uint64_t*>(buf[1] + align_up(budget + 64, kAlign))};
+  cudaStream_t sb[2] = {c->s_copy, c->s_asm};
+  const size_t C = p.bounds.size() - 1;
+  int rc;
+  GrepParams gp{};
+  bk_out_grep* og = (bk_out_grep*)out;
+  bk_out_groupby* ob = (bk_out_groupby*)out;
+  const uint32_t nb = dbuf_blocks();
+  if (kid == BK_K_GREP) {
+    if (og->pattern_len > 32) return fail(BK_E_INVAL, "pattern longer than 32 bytes");
+    if (c->min_rec < 48) return fail(BK_E_INVAL, "grep needs records of >= 48 bytes");
+    if (og->pattern_len) memcpy(gp.pat, og->pattern, og->pattern_len);
+    gp.plen = og->pattern_len;
+    gp.first_index = og->first_index;
+    gp.cap = std::min<uint64_t>(og->cap, c->n);
+    BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(gp.cap, 1) * 8));
+    BK_CUDA(c->b_blk.ensure((uint64_t)nb * 4 * 2));
+    BK_CUDA(c->b_blk2.ensure((uint64_t)nb * 8 * 2));
+  } else {
+    if (ob->G == 0 || ob->G > 8192) return fail(BK_E_INVAL, "G must be in 1..8192");
+    if (c->off || c->cfg.record_size < 16) return fail(BK_E_INVAL, "group-by needs fixed records >= 16 B");
+    BK_CUDA(c->b_agg1.ensure((uint64_t)ob->G * 8));
+    BK_CUDA(c->b_agg2.ensure((uint64_t)ob->G * 8));
+    BK_CUDA(c->b_agg3.ensure((uint64_t)ob->G * 8));
+  }
+  if ((rc = begin_run(c, stream))) return rc;
+  if (kid == BK_K_GROUPBY) {
+    BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+    BK_CUDA(cudaEventRecord(c->ev_begin, c->s_comp));
+    BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->ev_begin, 0));
+    BK_CUDA(cudaStreamWaitEvent(c->s_asm, c->ev_begin, 0));
+  }
+  c->st.n_chunks = C;
+  c->st.gather_mode = BK_GATHER_DENSE;
+  c->st.chunk_budget = budget;
+  cudaEvent_t scanned[2] = {c->slots[0].ready, c->slots[1].ready};
+  for (size_t i = 0; i < C; ++i) {
+    const int b = (int)(i & 1);
+    cudaStream_t st = sb[b];
+    const uint64_t lo = p.bounds[i], hi = p.bounds[i + 1];
+    const uint64_t base = rec_start(c, lo), end = rec_start(c, hi);
+    const uint64_t raw_off = ((uintptr_t)(c->host + base)) & 15;
+    BK_PROF(kStH2D, st, true);
+    if (end > base) BK_CUDA(cudaMemcpyAsync(buf[b] + raw_off, c->host + base, end - base, cudaMemcpyHostToDevice, st));
+    if (c->off && hi > lo) {
+      BK_CUDA(cudaMemcpyAsync(meta[b], c->off + lo, (hi - lo) * 8, cudaMemcpyHostToDevice, st));
+      c->st.bytes_meta += (hi - lo) * 8;
+    }
+    BK_PROF(kStH2D, st, false);
+    c->st.bytes_h2d += end - base;
+    BK_PROF(kStCompute, st, true);
+    if (kid == BK_K_GREP) {
+      // chunk i's output offset follows chunk i-1's scan (ordered results across the two streams)
+      if (i > 0) BK_CUDA(cudaStreamWaitEvent(st, scanned[1 - b], 0));
+      launch_dbuf_grep(buf[b] + raw_off, c->off ? meta[b] : nullptr, lo, hi, base, end, c->cfg.record_size, gp,
+                       (uint32_t*)c->b_blk.p + b * nb, c->d_ctr + 3, (unsigned long long*)c->b_blk2.p + b * nb,
+                       (uint64_t*)c->b_out1.p, st);
+      BK_CUDA(cudaEventRecord(scanned[b], st));
+      c->n_launch += 3;
+    } else {
+      launch_dbuf_groupby(buf[b] + raw_off, lo, hi, base, c->cfg.record_size, ob->G, (unsigned long long*)c->b_agg1.p,
+                          (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, st);
+      c->n_launch += 1;
+    }
+    BK_PROF(kStCompute, st, false);
+  }
+  for (cudaStream_t st : sb) {
+    BK_CUDA(cudaEventRecord(c->ev_end, st));
+    BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
+  }
+  if ((rc = end_run(c, stream))) return rc;
+  if (kid == BK_K_GREP) {
+    unsigned long long m = 0;
+    BK_CUDA(cudaMemcpy(&m, c->d_ctr + 3, 8, cudaMemcpyDeviceToHost));
+    og->n_match = m;
+    if (m > og->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)og->cap);
+    if (m) BK_CUDA(cudaMemcpy(og->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));
+  } else {
+    BK_CUDA(cudaMemcpy(ob->count, c->b_agg1.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(ob->qty, c->b_agg2.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(ob->amount, c->b_agg3.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
+  }
+  return BK_OK;
+}
+
 int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
   Access a{};
   if (o->n_ext == 0) {
@@ -891,7 +1001,8 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
     return cleanup(fail(BK_E_NOMEM, "cudaMalloc scratch"));
   c->slots.resize(c->cfg.n_slots);
   if (cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "d2h stream"));
-  if (configure_partition_kernels() != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
+  if (configure_partition_kernels() != cudaSuccess || configure_baseline_kernels() != cudaSuccess)
+    return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
   c->ev_part.assign(c->cfg.n_slots, nullptr);
   for (auto& e : c->ev_part)
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
@@ -981,6 +1092,17 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
   if (h->kernel_id != kernel_id) return fail(BK_E_INVAL, "out->kernel_id %d != %d", h->kernel_id, kernel_id);
   const auto t0 = std::chrono::steady_clock::now();
   int rc;
+  if (c->cfg.flags & BK_FLAG_BASELINE_DBUF) {
+    rc = run_dbuf(c, kernel_id, out, stream);
+    if (rc) {
+      cudaDeviceSynchronize();
+      cudaGetLastError();
+      return rc;
+    }
+    c->st.kernel_launches = (uint64_t)c->n_launch;
+    c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return BK_OK;
+  }
   switch (kernel_id) {
     case BK_K_WORDCOUNT:
       if (h->struct_size != sizeof(bk_out_wordcount)) return fail(BK_E_INVAL, "bk_out_wordcount size");

@@ -259,6 +259,26 @@ def test_partition_duplicate_keys_and_errors():
         assert e.value.status == bk.BK_E_CAPACITY
 
 
+# ------------------------------------------------------------------ the double-buffering baseline
+def test_dbuf_baseline_grep_and_groupby_match_oracle():
+    """BK_FLAG_BASELINE_DBUF (the paper's variant iv) must give the same results (I2)."""
+    buf, off = gen.grep_records(max_bytes=24 * MIB)
+    want = oracle.grep(buf, off, b"bigk", first=7)
+    with bk.Context(window_bytes=4 * MIB, baseline_dbuf=True) as ctx:
+        ctx.register(buf, off)
+        got = ctx.grep(b"bigk", first_index=7, cap=len(off))
+        assert ctx.stats()["n_chunks"] >= 8
+    assert np.array_equal(got, want)
+    n = 2_000_003
+    g = gen.groupby(n=n, zipf=True)
+    wc_, wq, wa = oracle.groupby(g, n, 16, 4096)
+    with bk.Context(window_bytes=4 * MIB, baseline_dbuf=True, record_size=16) as ctx:
+        ctx.register(g, None, n_records=n)
+        c, q, a = ctx.groupby(4096)
+    assert np.array_equal(c, wc_) and np.array_equal(q, wq)
+    np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
+
+
 # ------------------------------------------------------------------ invariants + API errors
 def test_invariance_across_window_slots_lanes_modes():
     buf, off = gen.text(cap_bytes=1 * MIB)
