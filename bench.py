@@ -38,6 +38,7 @@ import gen  # noqa: E402
 
 GIB = 1 << 30
 MIB = 1 << 20
+HUGE = True  # data sets in 2 MiB-aligned mappings with transparent huge pages (--pages)
 METRIC = "input GB/s streamed out-of-core at 1/2/4/8 B200; % of host-link roofline"
 
 
@@ -54,6 +55,10 @@ def parse():
     ap.add_argument("--window-mib", type=int, default=None)
     ap.add_argument("--slots", type=int, default=0)
     ap.add_argument("--host-threads", type=int, default=0)
+    ap.add_argument("--lane-bytes", type=int, default=0)
+    ap.add_argument("--zc-share", type=int, default=0, help="HYBRID zero-copy share of chunks, per mille")
+    ap.add_argument("--pages", default="numpy", choices=["huge", "4k", "numpy"],
+                    help="host data set pages: THP-backed mapping, 4 KiB mapping, or plain numpy")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-dbuf", action="store_true", help="skip the double-buffering baseline measurement")
     ap.add_argument("--no-profile", action="store_true", help="disable per-stage event timing")
@@ -82,7 +87,8 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
         first = 0
         for r in range(rank):
             first += gen.grep_count_for_bytes(gen.SEED_GREP, first, nbytes)
-        buf, off = gen.grep_records(gen.SEED_GREP, first=first, max_bytes=nbytes)
+        buf, off = gen.grep_records(gen.SEED_GREP, first=first, max_bytes=nbytes,
+                                    out=gen.alloc(nbytes, huge=HUGE) if HUGE is not None else None)
         return dict(buf=buf, off=off, n=len(off), first=first, rec_size=0)
     if workload == "wordcount":
         buf, off = gen.text(gen.SEED_WC + rank, cap_bytes=nbytes)
@@ -90,7 +96,8 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
     if workload in ("groupby", "groupby_sparse"):
         stride = 16 if workload == "groupby" else 64
         n = nbytes // stride
-        buf = gen.groupby(gen.SEED_GROUPBY, first=rank * n, n=n, stride=stride)
+        buf = gen.groupby(gen.SEED_GROUPBY, first=rank * n, n=n, stride=stride,
+                          out=gen.alloc(n * stride, huge=HUGE) if HUGE is not None else None)
         return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=stride)
     if workload == "partition":
         n = nbytes // 16
@@ -206,7 +213,9 @@ def oracle_sample(workload: str, shard: dict, target_s: float):
 
 # ------------------------------------------------------------------------------ main arms
 def main():
+    global HUGE
     args = parse()
+    HUGE = {"huge": True, "4k": False, "numpy": None}[args.pages]
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -234,7 +243,7 @@ def main():
     shard = make_shard(args.workload, gib, rank, world)
     peak_h2d = measure_h2d_peak(torch, dev)
     ctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
-                     host_threads=args.host_threads,
+                     host_threads=args.host_threads, lane_bytes=args.lane_bytes, zc_share_pm=args.zc_share,
                      profile=not args.no_profile, record_size=shard["rec_size"])
     t0 = time.perf_counter()
     ctx.register(shard["buf"], shard["off"], n_records=shard["n"])

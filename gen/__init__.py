@@ -52,6 +52,10 @@ def lib():
         l.gen_kv.argtypes = [u64, u64, u64, p, C.c_int]
         l.gen_groupby.restype = None
         l.gen_groupby.argtypes = [u64, u64, u64, C.c_uint32, C.c_uint32, C.c_int, p, C.c_int]
+        l.gen_alloc.restype = p
+        l.gen_alloc.argtypes = [u64, C.c_int, C.POINTER(p), C.POINTER(u64)]
+        l.gen_free.restype = None
+        l.gen_free.argtypes = [p, u64]
         _lib = l
     return _lib
 
@@ -63,6 +67,26 @@ def _threads(threads):
 def _ptr(a: np.ndarray) -> int:
     assert a.flags["C_CONTIGUOUS"]
     return a.ctypes.data
+
+
+class _Mapping:
+    """Owner of a gen_alloc mapping; numpy views keep it (their ultimate .base) alive."""
+
+    def __init__(self, p: int, n: int, base: int, ln: int):
+        self.__array_interface__ = {"data": (p, False), "shape": (n,), "typestr": "|u1", "version": 3}
+        self._region = (base, ln)
+
+    def __del__(self):
+        lib().gen_free(*self._region)
+
+
+def alloc(nbytes: int, huge: bool = True) -> np.ndarray:
+    """uint8 array of nbytes in a 2 MiB-aligned mapping (transparent huge pages when huge)."""
+    base, ln = C.c_void_p(), C.c_uint64()
+    p = lib().gen_alloc(max(nbytes, 1), int(huge), C.byref(base), C.byref(ln))
+    if not p:
+        raise MemoryError(nbytes)
+    return np.asarray(_Mapping(p, nbytes, base.value, ln.value))
 
 
 def R(seed: int, stream: int, i: int) -> int:

@@ -5,6 +5,7 @@
 #include <math.h>
 #include <stdlib.h>
 #include <string.h>
+#include <sys/mman.h>
 
 static inline uint64_t mix64(uint64_t x) {
   x ^= x >> 30; x *= 0xbf58476d1ce4e5b9ULL;
@@ -176,3 +177,18 @@ void gen_groupby(uint64_t seed, uint64_t first, uint64_t n, uint32_t G, uint32_t
   }
   free(cdf);
 }
+
+/* ---------------- host buffers (2 MiB aligned, optionally transparent huge pages) ---------------- */
+void* gen_alloc(uint64_t bytes, int huge, void** base_out, uint64_t* len_out) {
+  const uint64_t A = 2ull << 20;
+  uint64_t len = bytes + A;
+  void* base = mmap(NULL, len, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+  if (base == MAP_FAILED) return NULL;
+  uint8_t* p = (uint8_t*)(((uintptr_t)base + A - 1) & ~(uintptr_t)(A - 1));
+  if (huge) madvise(p, (bytes + A - 1) & ~(A - 1), MADV_HUGEPAGE);
+  *base_out = base;
+  *len_out = len;
+  return p;
+}
+
+void gen_free(void* base, uint64_t len) { munmap(base, len); }

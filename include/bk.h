@@ -60,8 +60,8 @@ typedef enum {
                            the warp-tile layout (the paper's CPU assembly), then one DMA */
   BK_GATHER_DENSE = 3,  /* one contiguous DMA of the chunk's records (copy engine), then an
                            HBM->HBM re-layout kernel (fetch-all) */
-  BK_GATHER_HYBRID = 4  /* per chunk: GPU zero-copy gather while fewer than (n_slots-1)/2 are in
-                           flight, otherwise CPU assembly; both share the link */
+  BK_GATHER_HYBRID = 4  /* chunks split between the GPU zero-copy gather and CPU assembly, running
+                           concurrently and sharing the link (see zc_share_pm) */
 } bk_gather_mode;
 
 typedef struct bk_config {
@@ -76,6 +76,10 @@ typedef struct bk_config {
   uint32_t host_threads;  /* CPU-assembly pool size (BK_GATHER_CPU / HYBRID); 0 = all hardware threads */
   uint64_t record_size;   /* fixed record length when record_offsets == NULL */
   uint32_t flags;         /* BK_FLAG_* */
+  uint32_t lane_bytes;    /* target accessed bytes per lane when lanes == 0; 0 = the kernel's default */
+  uint32_t zc_share_pm;   /* HYBRID: 0 = adaptive split (a zero-copy chunk is issued whenever fewer
+                             than (n_slots-1)/2 are in flight); else per-mille of chunks gathered
+                             zero-copy, deterministic: chunk i is zero-copy iff floor((i+1)s) > floor(i s) */
   uint32_t _reserved;
 } bk_config;
 

@@ -27,7 +27,8 @@ u32, i32, u64, P = C.c_uint32, C.c_int32, C.c_uint64, C.c_void_p
 class bk_config(C.Structure):
     _fields_ = [("struct_size", u32), ("device", i32), ("window_bytes", u64), ("n_slots", u32),
                 ("gather_mode", u32), ("chunk_bytes", u64), ("lanes", u32), ("host_threads", u32),
-                ("record_size", u64), ("flags", u32), ("_reserved", u32)]
+                ("record_size", u64), ("flags", u32), ("lane_bytes", u32),
+                ("zc_share_pm", u32), ("_reserved", u32)]
 
 
 class bk_out_header(C.Structure):
@@ -134,12 +135,14 @@ def _ptr(a) -> int | None:
 
 def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_mode: int | str = 0,
               chunk_bytes: int = 0, lanes: int = 0, record_size: int = 0, host_threads: int = 0,
-              profile: bool = False, baseline_dbuf: bool = False) -> int:
+              profile: bool = False, baseline_dbuf: bool = False, lane_bytes: int = 0,
+              zc_share_pm: int = 0) -> int:
     if isinstance(gather_mode, str):
         gather_mode = GATHER_NAMES[gather_mode]
     cfg = bk_config(C.sizeof(bk_config), device, window_bytes, n_slots, gather_mode, chunk_bytes, lanes,
                     host_threads, record_size,
-                    (BK_FLAG_PROFILE if profile else 0) | (BK_FLAG_BASELINE_DBUF if baseline_dbuf else 0), 0)
+                    (BK_FLAG_PROFILE if profile else 0) | (BK_FLAG_BASELINE_DBUF if baseline_dbuf else 0), lane_bytes,
+                    zc_share_pm, 0)
     ctx = P()
     check(lib().bk_create(C.byref(cfg), C.byref(ctx)), "bk_create")
     return ctx.value

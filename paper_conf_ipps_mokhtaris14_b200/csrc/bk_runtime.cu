@@ -85,6 +85,19 @@ struct DevBuf {
   }
 };
 
+// A run plan: depends only on the registration, the access spec and the config, so it is
+// computed once and cached per context (plan_cache) until the next registration.
+struct Plan {
+  Access a{};
+  int mode = BK_GATHER_DENSE;          // resolved gather mode
+  int zero_copy = 0;                   // plan budget counts accessed bytes (every mode but DENSE)
+  uint64_t budget = 0;                 // plan bytes per chunk
+  uint32_t L = 0;
+  uint64_t max_acc_rec = 0;            // max accessed bytes of one record
+  uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
+  std::vector<uint64_t> bounds;        // chunk record bounds
+};
+
 }  // namespace
 
 struct bk_ctx {
@@ -126,6 +139,7 @@ struct bk_ctx {
   uint64_t out_pinned_bytes = 0;
   int n_launch = 0;
   bk_stats st{};
+  std::vector<std::pair<std::string, Plan>> plan_cache;
 };
 
 namespace {
@@ -143,17 +157,6 @@ uint64_t rec_start(const bk_ctx* c, uint64_t r) {
   if (!c->off) return r * c->cfg.record_size;
   return r < c->n ? c->off[r] : c->nbytes;
 }
-
-struct Plan {
-  Access a{};
-  int mode = BK_GATHER_DENSE;          // resolved gather mode
-  int zero_copy = 0;                   // plan budget counts accessed bytes (every mode but DENSE)
-  uint64_t budget = 0;                 // plan bytes per chunk
-  uint32_t L = 0;
-  uint64_t max_acc_rec = 0;            // max accessed bytes of one record
-  uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
-  std::vector<uint64_t> bounds;        // chunk record bounds
-};
 
 // plan bytes of records [lo, r): what the budget limits (DESIGN.md §Chunk plan)
 uint64_t plan_bytes(const bk_ctx* c, const Plan& p, uint64_t lo, uint64_t r) {
@@ -218,19 +221,41 @@ void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) 
     L = (uint32_t)std::max<uint64_t>(32, std::min<uint64_t>(l, 1u << 22));
   }
   p.L = L;
-  // staged <= A + L*(max record + 32): DESIGN.md §Stage-1 bound
+  // staged <= A + L*(max record + 32): DESIGN.md §Stage-1 bound. For whole variable-length records
+  // (word count) that worst case is ~2x the payload, so size the slot from the exact staged size of
+  // every chunk instead (the k_addrgen lane rule evaluated on the host over the offsets).
   p.stage_cap = align_up(acc + (uint64_t)L * (p.max_acc_rec + 32) + 512, 512);
+  if (p.a.whole && c->off && p.bounds.size() > 1) {
+    HostData d{c->host, c->off, c->n, c->nbytes, 0};
+    Access a = p.a;
+    a.rec_size = 0;
+    uint64_t mx = 0;
+    for (size_t i = 0; i + 1 < p.bounds.size(); ++i) {
+      Chunk ch{};
+      ch.lo = p.bounds[i];
+      ch.hi = p.bounds[i + 1];
+      ch.base_byte = rec_start(c, ch.lo);
+      ch.end_byte = rec_start(c, ch.hi);
+      ch.L = L;
+      ch.ntiles = L / 32;
+      ch.accessed = ch.end_byte - ch.base_byte;
+      mx = std::max(mx, host_staged_size(d, a, ch));
+    }
+    p.stage_cap = align_up(mx + 512, 512);
+  }
   p.raw_cap = p.zero_copy ? 0 : budget + 64;
   p.meta_cap = c->off ? maxrecs + 1 : 0;
 }
 
-int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, bool out_per_chunk = false) {
+int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, bool out_per_chunk,
+                      int auto_mode) {
   p.a = a;
+  if (c->cfg.lane_bytes) lane_target = c->cfg.lane_bytes;
   int mode = (int)c->cfg.gather_mode;
   // AUTO (counters in profiles/): whole-record access -> DENSE (copy engine at
   // 55.5 GB/s beats zero-copy's 51.4); sparse access -> HYBRID (host assembly packs exactly the
   // accessed bytes; the zero-copy gather is request-rate bound and only adds capacity on top).
-  if (mode == BK_GATHER_AUTO) mode = a.whole ? BK_GATHER_DENSE : BK_GATHER_HYBRID;
+  if (mode == BK_GATHER_AUTO) mode = auto_mode != BK_GATHER_AUTO ? auto_mode : a.whole ? BK_GATHER_DENSE : BK_GATHER_HYBRID;
   if (mode != BK_GATHER_ZC && mode != BK_GATHER_DENSE && mode != BK_GATHER_CPU && mode != BK_GATHER_HYBRID)
     return fail(BK_E_INVAL, "bad gather_mode %d", mode);
   p.mode = mode;
@@ -260,6 +285,23 @@ int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, bool out
   return fail(BK_E_NOMEM, "window of %llu B (%u slots) cannot hold a chunk of %llu B (need %llu B per slot)",
               (unsigned long long)c->cfg.window_bytes, c->cfg.n_slots, (unsigned long long)budget,
               (unsigned long long)slot_need(p));
+}
+
+int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, bool out_per_chunk = false,
+             int auto_mode = BK_GATHER_AUTO) {
+  char key[256];
+  snprintf(key, sizeof key, "%u/%u/%u/%u/%u/%u/%u/%u/%u/%u/%d/%d", a.whole, a.n_ext, a.ext_off[0], a.ext_len[0],
+           a.ext_off[1], a.ext_len[1], a.ext_off[2], a.ext_len[2], a.E, lane_target, (int)out_per_chunk, auto_mode);
+  std::string k(key);
+  for (uint32_t e = 3; e < a.n_ext; ++e) k += "/" + std::to_string(a.ext_off[e]) + ":" + std::to_string(a.ext_len[e]);
+  for (auto& kv : c->plan_cache)
+    if (kv.first == k) {
+      p = kv.second;
+      return BK_OK;
+    }
+  const int rc = plan_run_uncached(c, a, lane_target, p, out_per_chunk, auto_mode);
+  if (rc == BK_OK) c->plan_cache.emplace_back(k, p);
+  return rc;
 }
 
 void carve(bk_ctx* c, const Plan& p) {
@@ -458,8 +500,6 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
   c->st.n_chunks = C;
   note_plan(c, p);
   std::vector<cudaEvent_t> zc_inflight;
-  // zero-copy chunks in flight in HYBRID mode: one keeps the GPU gather busy while the host pool
-  // assembles the next chunk (sweep in profiles/r01_hybrid_sweep.md)
   const size_t zc_depth = std::max<size_t>(1, (c->cfg.n_slots - 1) / 2);
   if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
     int rc = ensure_host_side(c, p);
@@ -469,10 +509,16 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
     Slot& s = c->slots[i % c->cfg.n_slots];
     cudaStream_t cs = concurrent ? c->s_slot[i % c->cfg.n_slots] : c->s_comp;
     bool cpu = p.mode == BK_GATHER_CPU;
-    if (p.mode == BK_GATHER_HYBRID) {
-      // GPU zero-copy gathers run asynchronously; keep up to zc_depth of them in flight and let
-      // the host pool assemble the next chunk whenever the GPU side is saturated.
-      while (!zc_inflight.empty() && cudaEventQuery(zc_inflight.front()) == cudaSuccess) zc_inflight.erase(zc_inflight.begin());
+    if (p.mode == BK_GATHER_HYBRID && c->cfg.zc_share_pm) {
+      // deterministic split (profiling, reproducibility): chunk i is zero-copy iff
+      // floor((i+1) s) > floor(i s)
+      const uint64_t pm = std::min<uint32_t>(c->cfg.zc_share_pm, 1000);
+      cpu = ((i + 1) * pm) / 1000 == (i * pm) / 1000;
+    } else if (p.mode == BK_GATHER_HYBRID) {
+      // adaptive split (default): the GPU zero-copy gathers run asynchronously; keep one in flight
+      // and let the host pool assemble the next chunk while it is busy (profiles/r01_hybrid_sweep.md)
+      while (!zc_inflight.empty() && cudaEventQuery(zc_inflight.front()) == cudaSuccess)
+        zc_inflight.erase(zc_inflight.begin());
       cudaGetLastError();
       cpu = zc_inflight.size() >= zc_depth;
     }
@@ -559,7 +605,9 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   uint64_t slots = o->table_slots ? o->table_slots : (1ull << 20);
   if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
   Plan p;
-  int rc = plan_run(c, whole_access(), 512, p);
+  // word count is compute-bound (thread-per-lane scan + table updates): AUTO picks ZC, which needs
+  // no raw buffer, so the window holds twice the text in flight; 256-B lanes (profiles/r01_wc_sweep.md)
+  int rc = plan_run(c, whole_access(), 256, p, false, BK_GATHER_ZC);
   if (rc) return rc;
   carve(c, p);
   BK_CUDA(c->b_table.ensure(slots * sizeof(WcEntry)));
@@ -1081,6 +1129,7 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
   c->off = off;
   c->n = n;
   c->registered = true;
+  c->plan_cache.clear();
   c->st.ms_register = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return BK_OK;
 }

@@ -91,6 +91,21 @@ inline uint64_t lane_first(const HostData& d, const Access& a, const Chunk& c, u
 
 }  // namespace
 
+uint64_t host_staged_size(const HostData& d, const Access& a, const Chunk& c) {
+  uint64_t size = 0;
+  uint64_t prev = lane_first(d, a, c, 0);
+  for (uint32_t w = 0; w < c.ntiles; ++w) {
+    uint64_t K = 0;
+    for (uint32_t i = 0; i < 32; ++i) {
+      const uint64_t nx = lane_first(d, a, c, (uint64_t)w * 32 + i + 1);
+      K = std::max<uint64_t>(K, (acc(d, a, c, nx) - acc(d, a, c, prev) + 15) / 16);
+      prev = nx;
+    }
+    size += 512 * K;
+  }
+  return size;
+}
+
 uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* stage,
                            uint64_t cap, std::vector<uint64_t>& first, std::vector<uint64_t>& tbase) {
   const uint32_t L = c.L, T = c.ntiles;

@@ -43,6 +43,9 @@ struct HostData {
 
 // Packs chunk c into `stage` (capacity cap) with the lane rule of k_addrgen and the tile layout
 // of k_gather_*; returns the staged size, or UINT64_MAX if it would exceed cap.
+// Exact staged size of chunk c (512 * sum of tile word counts) under the k_addrgen lane rule.
+uint64_t host_staged_size(const HostData& d, const Access& a, const Chunk& c);
+
 uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* stage,
                            uint64_t cap, std::vector<uint64_t>& first_scratch, std::vector<uint64_t>& tile_scratch);
 

@@ -56,6 +56,7 @@ __device__ void wc_insert(WcEntry* table, uint64_t mask, unsigned long long key1
 constexpr int kWcBlock = 128;   // 4 warps: small blocks spread a chunk's few lanes over more SMs
 constexpr int kWcTab = 1024;    // block table slots
 constexpr int kWcQ = 160;       // per-warp queue of finished words (static smem < 48 KB)
+constexpr int kWcProbes = 2;   // block table = hot-word cache: a crowded slot sends the word to the global table
 
 struct WcShared {
   unsigned long long k1[kWcTab], k2[kWcTab], ol[kWcTab];
@@ -68,7 +69,7 @@ __device__ void tab_insert(WcShared& sh, WcEntry* table, uint64_t mask, unsigned
                            unsigned long long k2, unsigned long long ol, unsigned int cnt,
                            unsigned long long* used, int* err) {
   uint32_t s = (uint32_t)(k1 >> 20) & (kWcTab - 1);
-  for (int p = 0; p < 16; ++p, s = (s + 1) & (kWcTab - 1)) {
+  for (int p = 0; p < kWcProbes; ++p, s = (s + 1) & (kWcTab - 1)) {
     unsigned long long cur = atomicCAS(&sh.k1[s], 0ull, k1);
     if (cur == 0) {  // claimed: publish occurrence + key2 (readers spin until key2 != 0)
       sh.ol[s] = ol;
