@@ -47,7 +47,9 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference", "dbuf", "sbuf"],
+                    help="ours | reference (CPU oracle) | dbuf / sbuf (the paper's GPU double / single "
+                         "buffering variants, for ablations)")
     ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "groupby_sparse", "kmeans",
                                                              "partition"])
     ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense", "cpu", "hybrid"])
@@ -243,6 +245,7 @@ def main():
     shard = make_shard(args.workload, gib, rank, world)
     peak_h2d = measure_h2d_peak(torch, dev)
     ctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
+                     baseline_dbuf=args.impl == "dbuf", baseline_sbuf=args.impl == "sbuf",
                      host_threads=args.host_threads, lane_bytes=args.lane_bytes, zc_share_pm=args.zc_share,
                      profile=not args.no_profile, record_size=shard["rec_size"])
     t0 = time.perf_counter()
@@ -381,7 +384,9 @@ def main():
         "clocks": clk.summary(),
         "register_s": round(reg_s, 3),
     }
-    if args.workload in ("grep", "groupby", "groupby_sparse") and not args.no_dbuf:
+    if args.impl != "ours":
+        line["impl"] = args.impl
+    if args.workload in ("grep", "groupby", "groupby_sparse") and not args.no_dbuf and args.impl == "ours":
         # the paper's GPU double-buffering baseline (variant iv) on the same data, window and box
         dctx = bk.Context(device=local, window_bytes=window, baseline_dbuf=True, profile=False,
                           record_size=shard["rec_size"])

@@ -88,6 +88,8 @@ typedef struct bk_config {
                                      P:994-996): raw whole-record chunks into 2 buffers (window/2 each)
                                      on 2 streams, kernel over contiguous per-thread record ranges.
                                      BK_K_GREP and BK_K_GROUPBY only; results identical. */
+#define BK_FLAG_BASELINE_SBUF 4u  /* the single-buffer variant: one buffer of the whole window,
+                                     copy then compute, no overlap */
 
 typedef struct bk_ctx bk_ctx;
 

@@ -828,7 +828,8 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
   p.a = whole_access();
   p.mode = BK_GATHER_DENSE;
   p.zero_copy = 0;
-  const uint64_t half = c->cfg.window_bytes / 2 / kAlign * kAlign;
+  const bool single = (c->cfg.flags & BK_FLAG_BASELINE_SBUF) != 0;
+  const uint64_t half = c->cfg.window_bytes / (single ? 1 : 2) / kAlign * kAlign;
   uint64_t budget = std::max<uint64_t>(std::min<uint64_t>(half, std::max<uint64_t>(c->nbytes / 32, 1ull << 20)), 1);
   uint64_t meta_cap = 0;
   for (int it = 0;; ++it) {
@@ -842,10 +843,10 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     if (it > 64 || budget < 64) return fail(BK_E_NOMEM, "window too small for the dbuf baseline");
     budget = budget * 3 / 4;
   }
-  uint8_t* buf[2] = {c->window, c->window + half};
+  uint8_t* buf[2] = {c->window, c->window + (single ? 0 : half)};
   uint64_t* meta[2] = {reinterpret_cast<uint64_t*>(buf[0] + align_up(budget + 64, kAlign)),
                        reinterpret_cast<uint64_t*>(buf[1] + align_up(budget + 64, kAlign))};
-  cudaStream_t sb[2] = {c->s_copy, c->s_asm};
+  cudaStream_t sb[2] = {c->s_copy, single ? c->s_copy : c->s_asm};
   const size_t C = p.bounds.size() - 1;
   int rc;
   GrepParams gp{};
@@ -1141,7 +1142,7 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
   if (h->kernel_id != kernel_id) return fail(BK_E_INVAL, "out->kernel_id %d != %d", h->kernel_id, kernel_id);
   const auto t0 = std::chrono::steady_clock::now();
   int rc;
-  if (c->cfg.flags & BK_FLAG_BASELINE_DBUF) {
+  if (c->cfg.flags & (BK_FLAG_BASELINE_DBUF | BK_FLAG_BASELINE_SBUF)) {
     rc = run_dbuf(c, kernel_id, out, stream);
     if (rc) {
       cudaDeviceSynchronize();
