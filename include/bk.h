@@ -154,8 +154,9 @@ typedef struct bk_out_kmeans {
   uint64_t* count;          /* out: K */
   double* sum;              /* out: K x 16 */
   uint64_t chk;             /* out: sum_i mix64((i<<8) ^ cid_i) mod 2^64 */
-  int32_t* cid;             /* out, optional (NULL): per-record cluster id, written back to the
-                               host through mapped memory (P:563-572 writes to mapped data) */
+  int32_t* cid;             /* out, optional (NULL): n_records cluster ids written back to the host
+                               (P:563-572 writes to mapped data): per chunk into the slot,
+                               then DMA'd on a D2H stream; the array is pinned once and cached */
 } bk_out_kmeans;
 
 typedef struct bk_out_partition {

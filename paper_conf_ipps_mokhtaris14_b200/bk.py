@@ -239,12 +239,16 @@ class Context:
         bk_run(self.ctx, BK_K_GROUPBY, stream, o)
         return cnt, qty, amt
 
-    def kmeans(self, mu: np.ndarray, first_index: int = 0, stream=None):
+    def kmeans(self, mu: np.ndarray, first_index: int = 0, stream=None, cid=None):
+        """(count u64[K], sum f64[K,16], chk); cid: optional int32[n] written back per record."""
         mu = np.ascontiguousarray(mu, np.float32).reshape(-1, 16)
         K = mu.shape[0]
         o = _hdr(bk_out_kmeans, BK_K_KMEANS)
         cnt = np.empty(K, np.uint64); s = np.empty((K, 16), np.float64)
-        o.centroids, o.K, o.first_index, o.count, o.sum, o.cid = _ptr(mu), K, first_index, _ptr(cnt), _ptr(s), None
+        if cid is not None:
+            assert cid.dtype == np.int32 and len(cid) >= self.n
+        o.centroids, o.K, o.first_index, o.count, o.sum = _ptr(mu), K, first_index, _ptr(cnt), _ptr(s)
+        o.cid = _ptr(cid) if cid is not None and self.n else None
         bk_run(self.ctx, BK_K_KMEANS, stream, o)
         return cnt, s, int(o.chk)
 

@@ -97,7 +97,7 @@ void launch_groupby(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes,
 size_t kmeans_smem(uint32_t K);
 void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                    const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
-                   unsigned long long* chk, int grid, cudaStream_t s);
+                   unsigned long long* chk, int32_t* cid_out, int grid, cudaStream_t s);
 
 cudaError_t configure_compute_kernels();
 

@@ -247,7 +247,7 @@ void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) 
   p.meta_cap = c->off ? maxrecs + 1 : 0;
 }
 
-int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, bool out_per_chunk,
+int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t out_per_rec,
                       int auto_mode) {
   p.a = a;
   if (c->cfg.lane_bytes) lane_target = c->cfg.lane_bytes;
@@ -276,7 +276,9 @@ int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p,
     int rc = make_chunks(c, p);
     if (rc) return rc;
     size_plan(c, p, budget, lane_target);
-    p.out_cap = out_per_chunk ? budget : 0;
+    uint64_t maxrecs = 0;  // per-chunk output buffer: out_per_rec bytes per record (partition, cid)
+    for (size_t i = 0; i + 1 < p.bounds.size(); ++i) maxrecs = std::max<uint64_t>(maxrecs, p.bounds[i + 1] - p.bounds[i]);
+    p.out_cap = maxrecs * out_per_rec;
     if (slot_need(p) <= slot) return BK_OK;
     if (!autob) break;
     budget = budget * 3 / 4;
@@ -287,7 +289,7 @@ int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p,
               (unsigned long long)slot_need(p));
 }
 
-int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, bool out_per_chunk = false,
+int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t out_per_chunk = 0,
              int auto_mode = BK_GATHER_AUTO) {
   char key[256];
   snprintf(key, sizeof key, "%u/%u/%u/%u/%u/%u/%u/%u/%u/%u/%d/%d", a.whole, a.n_ext, a.ext_off[0], a.ext_len[0],
@@ -607,7 +609,7 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   Plan p;
   // word count is compute-bound (thread-per-lane scan + table updates): AUTO picks ZC, which needs
   // no raw buffer, so the window holds twice the text in flight; 256-B lanes (profiles/r01_wc_sweep.md)
-  int rc = plan_run(c, whole_access(), 256, p, false, BK_GATHER_ZC);
+  int rc = plan_run(c, whole_access(), 256, p, 0, BK_GATHER_ZC);
   if (rc) return rc;
   carve(c, p);
   BK_CUDA(c->b_table.ensure(slots * sizeof(WcEntry)));
@@ -719,16 +721,33 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
   return BK_OK;
 }
 
+// The caller's per-record output (partition records, k-means cid) is written by DMA: pin it once
+// and keep it pinned across runs (one cached registration per context).
+int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes) {
+  if (!bytes || (c->out_pinned == ptr && c->out_pinned_bytes == bytes)) return BK_OK;
+  if (c->out_pinned) cudaHostUnregister(c->out_pinned);
+  c->out_pinned = nullptr;
+  c->out_pinned_bytes = 0;
+  if (!is_pinned(ptr)) {
+    BK_CUDA(cudaHostRegister(ptr, bytes, cudaHostRegisterPortable));
+    c->out_pinned = ptr;
+    c->out_pinned_bytes = bytes;
+  }
+  return BK_OK;
+}
+
 int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   const uint32_t K = o->K;
   if (K == 0 || K > 256 || !o->centroids) return fail(BK_E_INVAL, "K must be in 1..256 with centroids");
-  if (o->cid) return fail(BK_E_UNSUPPORTED, "cid write-back is not in this build");
   if (c->min_rec < 64) return fail(BK_E_INVAL, "k-means records must hold 16 fp32 (>= 64 bytes)");
   const bool dense64 = !c->off && c->cfg.record_size == 64;
   Plan p;
-  int rc = plan_run(c, dense64 ? whole_access() : field_access(0, 64), 256, p);
+  // cid write-back (P:563-572 writes to mapped data; "sets its clusterId"): 4 B per
+  // record per chunk in the slot, DMA'd back on the D2H stream while the next chunks stream in
+  int rc = plan_run(c, dense64 ? whole_access() : field_access(0, 64), 256, p, o->cid ? 4 : 0);
   if (rc) return rc;
   carve(c, p);
+  if (o->cid && (rc = ensure_out_pinned(c, o->cid, c->n * 4))) return rc;
   BK_CUDA(c->b_mu.ensure((uint64_t)K * 64));
   BK_CUDA(c->b_agg1.ensure((uint64_t)K * 8));
   BK_CUDA(c->b_agg3.ensure((uint64_t)K * 16 * 8));
@@ -739,20 +758,35 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
-  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+  if (o->cid) BK_CUDA(cudaStreamWaitEvent(c->s_d2h, c->ev_begin, 0));
+  size_t ci = 0;
+  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
     launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
-                  (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4, grid, cs);
+                  (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4,
+                  o->cid ? (int32_t*)s.out : nullptr, grid, cs);
     c->n_launch += 1;
-    return BK_OK;
+    if (o->cid && ch.hi > ch.lo) {
+      cudaEvent_t e = c->ev_part[ci++ % c->ev_part.size()];
+      BK_CUDA(cudaEventRecord(e, cs));
+      BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
+      BK_CUDA(cudaMemcpyAsync(o->cid + ch.lo, s.out, (ch.hi - ch.lo) * 4, cudaMemcpyDeviceToHost, c->s_d2h));
+      c->st.bytes_d2h += (ch.hi - ch.lo) * 4;
+      rel = c->s_d2h;
+    }
+    return (int)BK_OK;
   });
   if (rc) return rc;
+  if (o->cid) {
+    BK_CUDA(cudaEventRecord(c->ev_end, c->s_d2h));
+    BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
+  }
   if ((rc = end_run(c, stream))) return rc;
   BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDeviceToHost));
   BK_CUDA(cudaMemcpy(o->sum, c->b_agg3.p, (uint64_t)K * 128, cudaMemcpyDeviceToHost));
   unsigned long long chk = 0;
   BK_CUDA(cudaMemcpy(&chk, c->d_ctr + 4, 8, cudaMemcpyDeviceToHost));
   o->chk = chk;
-  c->st.bytes_d2h = (uint64_t)K * 136;
+  c->st.bytes_d2h += (uint64_t)K * 136;
   return BK_OK;
 }
 
@@ -764,7 +798,7 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
   int bits = 0;
   while ((1u << bits) < B) ++bits;
   Plan p;
-  int rc = plan_run(c, whole_access(), 256, p, true);
+  int rc = plan_run(c, whole_access(), 256, p, 16);
   if (rc) return rc;
   carve(c, p);
   const uint64_t C = p.bounds.size() - 1;
@@ -777,17 +811,7 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
   BK_CUDA(c->b_colpre.ensure((uint64_t)nblk_max * B * 4));
   BK_CUDA(c->b_totals.ensure(std::max<uint64_t>(C, 1) * B * 8));
   BK_CUDA(c->b_base.ensure((uint64_t)B * 8));
-  // the caller's output is written by DMA: pin it once and keep it pinned across runs
-  const uint64_t out_bytes = c->n * 16;
-  if (out_bytes && (c->out_pinned != o->out_records || c->out_pinned_bytes != out_bytes)) {
-    if (c->out_pinned) cudaHostUnregister(c->out_pinned);
-    c->out_pinned = nullptr;
-    if (!is_pinned(o->out_records)) {
-      BK_CUDA(cudaHostRegister(o->out_records, out_bytes, cudaHostRegisterPortable));
-      c->out_pinned = o->out_records;
-      c->out_pinned_bytes = out_bytes;
-    }
-  }
+  if ((rc = ensure_out_pinned(c, o->out_records, c->n * 16))) return rc;
   if ((rc = begin_run(c, stream))) return rc;
   BK_CUDA(cudaStreamWaitEvent(c->s_d2h, c->ev_begin, 0));
   size_t ci = 0;

@@ -430,7 +430,7 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
                                                 const uint64_t* __restrict__ tile_base,
                                                 const float* __restrict__ mu, uint32_t K, uint64_t first_index,
                                                 unsigned long long* gcount, double* gsum,
-                                                unsigned long long* gchk) {
+                                                unsigned long long* gchk, int32_t* __restrict__ cid_out) {
   extern __shared__ unsigned char smem_raw[];
   double* s_sum = reinterpret_cast<double*>(smem_raw);          // K*16
   float* s_mu = reinterpret_cast<float*>(s_sum + (size_t)K * 16);  // K*16
@@ -468,6 +468,7 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
 #pragma unroll
       for (int q = 0; q < 16; ++q) atomicAdd(&s_sum[best * 16 + q], (double)x[q]);
       chk += mix64(((first_index + d.first + j) << 8) ^ (uint64_t)best);
+      if (cid_out) cid_out[d.first + j - c.lo] = (int32_t)best;
     }
   }
 #pragma unroll
@@ -515,8 +516,9 @@ size_t kmeans_smem(uint32_t K) { return (size_t)K * 16 * 8 + (size_t)K * 16 * 4 
 
 void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                    const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
-                   unsigned long long* chk, int grid, cudaStream_t s) {
-  k_kmeans<<<grid, 256, kmeans_smem(K), s>>>(c, stage, lanes, tile_base, mu, K, first_index, count, sum, chk);
+                   unsigned long long* chk, int32_t* cid_out, int grid, cudaStream_t s) {
+  k_kmeans<<<grid, 256, kmeans_smem(K), s>>>(c, stage, lanes, tile_base, mu, K, first_index, count, sum, chk,
+                                              cid_out);
 }
 
 cudaError_t configure_compute_kernels() {

@@ -279,6 +279,79 @@ def test_dbuf_baseline_grep_and_groupby_match_oracle():
     np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
 
 
+# ------------------------------------------------------------------ f1: k-means cid write-back
+@pytest.mark.parametrize("mode", ["dense", "zc", "hybrid"])
+def test_kmeans_cid_writeback(mode):
+    n = 300_007
+    x = gen.points(n=n)
+    mu = x[:64].copy()
+    wc_, ws, wchk, wcid = oracle.kmeans(x, mu, want_cid=True)
+    cid = np.full(n, -1, np.int32)
+    with bk.Context(window_bytes=4 * MIB, gather_mode=mode, record_size=64) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=n)
+        c, s, chk = ctx.kmeans(mu, cid=cid)
+        assert ctx.stats()["bytes_d2h"] >= 4 * n
+        c2, _, _ = ctx.kmeans(mu)   # without write-back on the same context
+    assert np.array_equal(cid, wcid) and np.array_equal(c, wc_) and chk == wchk and np.array_equal(c2, wc_)
+
+
+# ------------------------------------------------------------------ bench-scale sizes (sampled / properties)
+def mix64_np(x):
+    x = x.astype(np.uint64)
+    x ^= x >> np.uint64(30); x *= np.uint64(0xBF58476D1CE4E5B9)
+    x ^= x >> np.uint64(27); x *= np.uint64(0x94D049BB133111EB)
+    x ^= x >> np.uint64(31)
+    return x
+
+
+def test_kmeans_bench_scale_sampled():
+    """C3 per-GPU share at 2 GPUs would be 5e8 points; here 2.5e8 (16 GiB, bench.py's default
+    k-means size) in bench.py's launch configuration (2 GiB window, AUTO). Checked: every cid the
+    oracle computes for 200k sampled points, Sum count = n, count = bincount(cid), the checksum
+    recomputed from the written-back cids, and column sums."""
+    n = 250_000_000
+    x = gen.points(n=n)
+    mu = gen.points(n=64)
+    cid = np.empty(n, np.int32)
+    with bk.Context(window_bytes=2 << 30, record_size=64) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=n)
+        c, s, chk = ctx.kmeans(mu, cid=cid)
+    rng = np.random.default_rng(5)
+    idx = np.sort(rng.choice(n, 200_000, replace=False))
+    _, _, _, scid = oracle.kmeans(x[idx], mu, want_cid=True)
+    assert np.array_equal(cid[idx], scid)
+    assert int(c.sum()) == n and np.array_equal(c, np.bincount(cid, minlength=64).astype(np.uint64))
+    i = np.arange(n, dtype=np.uint64)
+    assert int(mix64_np((i << np.uint64(8)) ^ cid.astype(np.uint64)).sum(dtype=np.uint64)) == chk
+    np.testing.assert_allclose(s.sum(0), x.sum(0, dtype=np.float64), rtol=1e-9)
+
+
+def test_partition_bench_scale():
+    """C4 per-GPU share (64 GiB / 8 GPUs = 8 GiB, 2^29 records), 1024 buckets: whole result bit-exact."""
+    n = 1 << 29
+    kv = gen.kv(n=n)
+    with bk.Context(window_bytes=2 << 30, record_size=16) as ctx:
+        ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=n)
+        out, cc, bc = ctx.partition(1024)
+    del ctx
+    wboff, wout = oracle.partition(kv, 1024)
+    assert np.array_equal(np.concatenate([[0], np.cumsum(bc)]).astype(np.uint64), wboff)
+    assert np.array_equal(global_from_runs(out, cc), wout)
+
+
+def test_groupby_bench_scale():
+    """C5 at 32 GiB through a 2 GiB window (16x out-of-core), whole result vs the oracle."""
+    n = 2 << 30
+    g = gen.groupby(n=n)
+    with bk.Context(window_bytes=2 << 30, record_size=16) as ctx:
+        ctx.register(g, None, n_records=n)
+        c, q, a = ctx.groupby(4096)
+        assert ctx.stats()["n_chunks"] >= 16
+    wc_, wq, wa = oracle.groupby(g, n, 16, 4096)
+    assert np.array_equal(c, wc_) and np.array_equal(q, wq)
+    np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
+
+
 # ------------------------------------------------------------------ invariants + API errors
 def test_invariance_across_window_slots_lanes_modes():
     buf, off = gen.text(cap_bytes=1 * MIB)
