@@ -6,7 +6,7 @@ PKG    := paper_conf_ipps_mokhtaris14_b200
 CSRC   := $(PKG)/csrc
 OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/bk_runtime.o build/host_gather.o
 
-all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so
+all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so baselines/libbkmt.so
 
 build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh include/bk.h
 	@mkdir -p build
@@ -33,3 +33,6 @@ clean:
 	rm -rf build $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so
 
 .PHONY: all clean
+
+baselines/libbkmt.so: baselines/cpu_mt.c
+	gcc -O3 -march=x86-64-v3 -ffp-contract=off -fopenmp -fPIC -shared -o $@ $< -lm

@@ -1,0 +1,57 @@
+"""The paper's multithreaded CPU variant (ii), bench-only (ctypes over
+baselines/libbkmt.so, OpenMP on all host cores). Not the oracle, not part of libbk."""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libbkmt.so")
+_SRC = os.path.join(_HERE, "cpu_mt.c")
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+            subprocess.check_call(["gcc", "-O3", "-march=x86-64-v3", "-ffp-contract=off", "-fopenmp", "-fPIC",
+                                   "-shared", _SRC, "-o", _SO, "-lm"])
+        l = C.CDLL(_SO)
+        p, u64, u32 = C.c_void_p, C.c_uint64, C.c_uint32
+        l.mt_threads.restype = C.c_int
+        l.mt_grep.restype = C.c_int64
+        l.mt_grep.argtypes = [p, u64, p, u64, p, u32, p, u64]
+        l.mt_groupby.argtypes = [p, u64, u32, u32, p, p, p]
+        l.mt_kmeans.argtypes = [p, u64, p, u32, p, p]
+        _lib = l
+    return _lib
+
+
+def threads() -> int:
+    return lib().mt_threads()
+
+
+def grep(buf, off, pattern: bytes = b"bigk"):
+    pat = np.frombuffer(pattern, np.uint8) if pattern else np.zeros(1, np.uint8)
+    idx = np.empty(max(len(off), 1), np.uint64)
+    m = lib().mt_grep(buf.ctypes.data, len(buf), off.ctypes.data, len(off), pat.ctypes.data, len(pattern),
+                      idx.ctypes.data, len(idx))
+    return idx[:m]
+
+
+def groupby(buf, n, stride=16, G=4096):
+    c = np.empty(G, np.uint64); q = np.empty(G, np.uint64); a = np.empty(G, np.float64)
+    lib().mt_groupby(buf.ctypes.data, n, stride, G, c.ctypes.data, q.ctypes.data, a.ctypes.data)
+    return c, q, a
+
+
+def kmeans(x, mu):
+    mu = np.ascontiguousarray(mu, np.float32)
+    K = mu.shape[0]
+    c = np.empty(K, np.uint64); s = np.empty((K, 16), np.float64)
+    lib().mt_kmeans(x.ctypes.data, len(x), mu.ctypes.data, K, c.ctypes.data, s.ctypes.data)
+    return c, s

@@ -1,0 +1,103 @@
+/* cpu_mt.c — the paper's multithreaded CPU variant (ii), the comparison
+ * point of its "3.0x over multithreaded CPU" claim. Bench-only baseline: OpenMP over all
+ * host cores, each thread a contiguous record range, per-thread partial results merged at the end.
+ * Not the oracle (oracle/ stays single-threaded and unoptimised) and not part of libbk. */
+#include <math.h>
+#include <omp.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+int mt_threads(void) { return omp_get_max_threads(); }
+
+/* grep: returns the match count; indices are written in ascending order (per-thread buffers). */
+int64_t mt_grep(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uint64_t n, const uint8_t* pat,
+                uint32_t plen, uint64_t* idx, uint64_t cap) {
+  int T = omp_get_max_threads();
+  uint64_t* cnt = calloc(T + 1, sizeof(uint64_t));
+  uint64_t** loc = calloc(T, sizeof(uint64_t*));
+#pragma omp parallel num_threads(T)
+  {
+    int t = omp_get_thread_num();
+    uint64_t lo = n * t / T, hi = n * (t + 1) / T, m = 0, capl = 1024;
+    uint64_t* buf = malloc(capl * 8);
+    for (uint64_t r = lo; r < hi; ++r) {
+      const uint8_t* key = d + off[r] + 16;
+      uint32_t kl = 0;
+      while (kl < 32 && key[kl]) ++kl;
+      int hit = plen == 0;
+      for (uint32_t p = 0; !hit && p + plen <= kl; ++p) hit = memcmp(key + p, pat, plen) == 0;
+      if (hit) {
+        if (m == capl) { capl *= 2; buf = realloc(buf, capl * 8); }
+        buf[m++] = r;
+      }
+    }
+    loc[t] = buf;
+    cnt[t + 1] = m;
+  }
+  for (int t = 0; t < T; ++t) cnt[t + 1] += cnt[t];
+#pragma omp parallel for num_threads(T)
+  for (int t = 0; t < T; ++t) {
+    for (uint64_t i = cnt[t]; i < cnt[t + 1] && i < cap; ++i) idx[i] = loc[t][i - cnt[t]];
+    free(loc[t]);
+  }
+  int64_t total = (int64_t)cnt[T];
+  free(cnt);
+  free(loc);
+  (void)nbytes;
+  return total;
+}
+
+void mt_groupby(const uint8_t* recs, uint64_t n, uint32_t stride, uint32_t G, uint64_t* count, uint64_t* qty,
+                double* amount) {
+  memset(count, 0, 8 * G);
+  memset(qty, 0, 8 * G);
+  memset(amount, 0, 8 * G);
+#pragma omp parallel
+  {
+    uint64_t* c = calloc(G, 8);
+    uint64_t* q = calloc(G, 8);
+    double* a = calloc(G, 8);
+#pragma omp for schedule(static)
+    for (uint64_t i = 0; i < n; ++i) {
+      uint32_t k, qq;
+      double aa;
+      memcpy(&k, recs + i * stride, 4);
+      memcpy(&qq, recs + i * stride + 4, 4);
+      memcpy(&aa, recs + i * stride + 8, 8);
+      if (k < G) { c[k] += 1; q[k] += qq; a[k] += aa; }
+    }
+#pragma omp critical
+    for (uint32_t g = 0; g < G; ++g) { count[g] += c[g]; qty[g] += q[g]; amount[g] += a[g]; }
+    free(c);
+    free(q);
+    free(a);
+  }
+}
+
+void mt_kmeans(const float* x, uint64_t n, const float* mu, uint32_t K, uint64_t* count, double* sum) {
+  memset(count, 0, 8 * K);
+  memset(sum, 0, 8 * K * 16);
+#pragma omp parallel
+  {
+    uint64_t* c = calloc(K, 8);
+    double* s = calloc((size_t)K * 16, 8);
+#pragma omp for schedule(static)
+    for (uint64_t i = 0; i < n; ++i) {
+      const float* p = x + i * 16;
+      uint32_t best = 0;
+      float bd = 0;
+      for (uint32_t k = 0; k < K; ++k) {
+        float acc = 0;
+        for (int j = 0; j < 16; ++j) { float t = p[j] - mu[k * 16 + j]; acc = fmaf(t, t, acc); }
+        if (k == 0 || acc < bd) { bd = acc; best = k; }
+      }
+      c[best] += 1;
+      for (int j = 0; j < 16; ++j) s[best * 16 + j] += p[j];
+    }
+#pragma omp critical
+    for (uint32_t k = 0; k < K * 16; ++k) { sum[k] += s[k]; if (k < K) count[k] += c[k]; }
+    free(c);
+    free(s);
+  }
+}

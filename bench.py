@@ -418,6 +418,25 @@ def main():
                                          "2 streams) + the same computation per thread-range (PAPER.md P:329-339, P:994-996)",
                                  "bigkernel_speedup": round(value / dv, 3)}
         dctx.close()
+    if rank == 0 and not args.no_cpu_baseline and args.impl == "ours" and args.workload in (
+            "grep", "groupby", "groupby_sparse", "kmeans"):
+        # the paper's multithreaded CPU variant (ii) on all host cores, same shard (kmeans: 1/16 sample)
+        import baselines
+        t0 = time.perf_counter()
+        if args.workload == "grep":
+            baselines.grep(shard["buf"], shard["off"])
+            mt_bytes = nbytes
+        elif args.workload == "kmeans":
+            m = shard["n"] // 16
+            baselines.kmeans(shard["buf"][: m * 64].view(np.float32).reshape(-1, 16), shard["mu"])
+            mt_bytes = m * 64
+        else:
+            baselines.groupby(shard["buf"], shard["n"], shard["rec_size"], 4096)
+            mt_bytes = nbytes
+        mt = mt_bytes / (time.perf_counter() - t0) / 1e9
+        line["cpu_mt_baseline"] = {"value": round(mt, 3), "unit": "GB/s", "cores": baselines.threads(),
+                                   "what": "paper variant (ii): OpenMP over all host cores (baselines/cpu_mt.c)",
+                                   "bigkernel_speedup": round(value / mt, 3)}
     if rank == 0 and not args.no_cpu_baseline:
         gbs, sample, secs = oracle_sample(args.workload, shard, 10.0)
         line["cpu_baseline"] = {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",

@@ -54,15 +54,14 @@ __device__ void wc_insert(WcEntry* table, uint64_t mask, unsigned long long key1
 
 // Per-block shared-memory pre-aggregation (Zipf text: most occurrences hit a few hot words).
 constexpr int kWcBlock = 128;   // 4 warps: small blocks spread a chunk's few lanes over more SMs
-constexpr int kWcTab = 1024;    // block table slots
-constexpr int kWcQ = 160;       // per-warp queue of finished words (static smem < 48 KB)
-constexpr int kWcProbes = 2;   // block table = hot-word cache: a crowded slot sends the word to the global table
+constexpr int kWcTab = 512;     // block table slots (a hot-word cache)
+constexpr int kWcQ = 256;       // per-warp queue of finished words
+constexpr int kWcProbes = 2;    // a crowded block-table slot sends the word to the global table
 
 struct WcShared {
   unsigned long long k1[kWcTab], k2[kWcTab], ol[kWcTab];
   unsigned int cnt[kWcTab];
   unsigned long long qk1[kWcBlock / 32][kWcQ], qk2[kWcBlock / 32][kWcQ], qol[kWcBlock / 32][kWcQ];
-  int qn[kWcBlock / 32];
 };
 
 __device__ void tab_insert(WcShared& sh, WcEntry* table, uint64_t mask, unsigned long long k1,
@@ -91,43 +90,34 @@ __device__ void tab_insert(WcShared& sh, WcEntry* table, uint64_t mask, unsigned
   wc_insert(table, mask, k1, k2, ol, cnt, used, err);  // block table crowded: go global
 }
 
-// Insert the warp's queued words, 32 at a time, duplicates within a round merged by match_any.
-__device__ __forceinline__ void wc_flush_queue(WcShared& sh, int w, int lane, WcEntry* table, uint64_t mask,
-                                               unsigned long long* used, int* err) {
+// Insert the warp's n queued words, 32 at a time: finalise the identity here (every lane busy),
+// merge duplicates within a round by match_any, insert into the block table.
+__device__ __forceinline__ void wc_flush_queue(WcShared& sh, int w, int lane, int n, WcEntry* table,
+                                               uint64_t mask, unsigned long long* used, int* err) {
   __syncwarp();
-  const int n = min(*reinterpret_cast<volatile int*>(&sh.qn[w]), kWcQ);
   for (int base = 0; base < n; base += 32) {
     const int i = base + lane;
     const bool v = i < n;
-    const unsigned long long k1 = v ? sh.qk1[w][i] : 0, k2 = v ? sh.qk2[w][i] : 0, ol = v ? sh.qol[w][i] : 0;
+    unsigned long long k1 = 0, k2 = 0, ol = 0;
+    if (v) {
+      ol = sh.qol[w][i];
+      const uint64_t len = ol & 0xffffff;
+      k1 = mix64(sh.qk1[w][i] ^ (len * 0x9E3779B97F4A7C15ull)) | 1ull;
+      k2 = mix64(sh.qk2[w][i] + len) | 1ull;
+    }
     const unsigned m = __match_any_sync(kFull, k1) & __match_any_sync(kFull, k2);
     if (v && lane == __ffs(m) - 1) tab_insert(sh, table, mask, k1, k2, ol, __popc(m), used, err);
   }
   __syncwarp();
-  if (lane == 0) sh.qn[w] = 0;
-  __syncwarp();
 }
 
-__device__ __forceinline__ void wc_push(WcShared& sh, int w, WcEntry* table, uint64_t mask, uint64_t h1,
-                                        uint64_t h2, uint32_t len, uint64_t occ, unsigned long long* used,
-                                        int* err) {
-  const unsigned long long k1 = mix64(h1 ^ ((uint64_t)len * 0x9E3779B97F4A7C15ull)) | 1ull;
-  const unsigned long long k2 = mix64(h2 + len) | 1ull;
-  if (len >= (1u << 24) || occ >= (1ull << 40)) atomicOr(err, kErrWordTooLong);
-  const unsigned long long ol = (occ << 24) | len;
-  const int i = atomicAdd(&sh.qn[w], 1);
-  if (i < kWcQ) {
-    sh.qk1[w][i] = k1;
-    sh.qk2[w][i] = k2;
-    sh.qol[w][i] = ol;
-  } else {
-    tab_insert(sh, table, mask, k1, k2, ol, 1, used, err);  // queue full this step (tiny words)
-  }
-}
+constexpr int kWcSub = 4;  // sub-threads per lane
 
-// Thread per lane tokenises its bytes (record boundaries from the offsets slice); finished words
-// go to a per-warp shared queue that the whole warp drains after every 16-byte step, so global
-// latency is never on a per-byte critical path.
+// kWcSub threads share one lane: sub-thread q owns the words that START in its quarter
+// [q*span, (q+1)*span) of the lane's bytes and finishes its last word past the quarter end
+// (classic parallel tokenisation; record boundaries from the offsets slice). Every 16-byte step
+// is branch-free across the warp: a word ending at a byte takes a queue slot from a ballot, and
+// its identity is finalised in the flush, so per-word work never rides on the per-byte path.
 __global__ void __launch_bounds__(kWcBlock) k_wc(Chunk c, const uint8_t* __restrict__ stage,
                                                  const LaneDesc* __restrict__ lanes,
                                                  const uint64_t* __restrict__ tile_base,
@@ -135,59 +125,105 @@ __global__ void __launch_bounds__(kWcBlock) k_wc(Chunk c, const uint8_t* __restr
                                                  WcEntry* table, uint64_t mask, unsigned long long* used, int* err) {
   __shared__ WcShared sh;
   for (int i = threadIdx.x; i < kWcTab; i += blockDim.x) { sh.k1[i] = 0; sh.k2[i] = 0; sh.cnt[i] = 0; }
-  if (threadIdx.x < kWcBlock / 32) sh.qn[threadIdx.x] = 0;
   __syncthreads();
-  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t t = g / kWcSub, q = g % kWcSub;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const bool live = t < c.L;   // L % 32 == 0: whole warps are live or not
-  if (live) {
-    const LaneDesc d = lanes[t];
-    const uint8_t* tile = stage + tile_base[t >> 5];
+  const unsigned lt = (1u << lane) - 1;
+  const bool live_warp = (g & ~31u) / kWcSub < c.L;
+  if (live_warp) {
+    const bool live = t < c.L;
+    LaneDesc d{0, 0, 0};
+    if (live) d = lanes[t];
+    const uint8_t* tile = live ? stage + tile_base[t >> 5] : stage;
+    const int col = t & 31;
     auto rstart = [&](uint64_t r) -> uint64_t {
       if (rec_size) return r * rec_size;
       return r == c.hi ? c.end_byte : meta[r - c.lo];
     };
-    const uint64_t lane_start = rstart(d.first);
+    const uint64_t lane_start = live ? rstart(d.first) : 0;
     const uint64_t rend = d.first + d.nrec;
-    uint64_t r = d.first + 1;
+    const uint32_t span = ((d.nbytes + kWcSub - 1) / kWcSub + 15) & ~15u;
+    uint32_t pos0 = min(d.nbytes, q * span);
+    const uint32_t range_end = min(d.nbytes, (q + 1) * span);
+    // first record boundary strictly after pos0 (binary search over the lane's records)
+    uint64_t r;
+    {
+      uint64_t lo = d.first + 1, hi = rend;
+      while (lo < hi) {
+        const uint64_t mid = (lo + hi) / 2;
+        if (rstart(mid) - lane_start <= pos0) lo = mid + 1; else hi = mid;
+      }
+      r = lo;
+    }
+    const bool at_boundary = pos0 > 0 && r > d.first + 1 && rstart(r - 1) - lane_start == pos0;
     uint32_t next_b = r < rend ? (uint32_t)(rstart(r) - lane_start) : 0xffffffffu;
+    auto byte_at = [&](uint32_t p) -> uint32_t {
+      const uint4 v = lane_word(tile, p >> 4, col);
+      const uint32_t j = p & 15;
+      const uint32_t wd = j < 8 ? (j < 4 ? v.x : v.y) : (j < 12 ? v.z : v.w);
+      return (wd >> (8 * (j & 3))) & 0xff;
+    };
+    // a word running into pos0 belongs to the previous sub-thread: start in "skip" state
+    bool skip = live && q > 0 && pos0 < d.nbytes && !at_boundary && !is_delim(byte_at(pos0 - 1));
     bool in_word = false;
     uint64_t h1 = 0, h2 = 0;
     uint32_t wstart = 0, wlen = 0;
-    const uint32_t W = (d.nbytes + 15) >> 4;
-    const uint32_t Kw = __reduce_max_sync(kFull, W);
-    for (uint32_t k = 0; k < Kw; ++k) {
-      if (k < W) {
-        const uint4 v = lane_word(tile, k, lane);
-        const uint32_t lim = min(16u, d.nbytes - 16 * k);
-#pragma unroll 1
-        for (uint32_t q = 0; q < lim; ++q) {
-          const uint32_t pos = 16 * k + q;
-          const uint32_t wd = q < 8 ? (q < 4 ? v.x : v.y) : (q < 12 ? v.z : v.w);
-          const uint32_t ch = (wd >> (8 * (q & 3))) & 0xff;
-          bool boundary = pos == next_b;
-          while (pos == next_b) {  // several if records are empty
-            ++r;
-            next_b = r < rend ? (uint32_t)(rstart(r) - lane_start) : 0xffffffffu;
-          }
-          const bool delim = is_delim(ch);
-          if (in_word && (delim || boundary)) {
-            wc_push(sh, w, table, mask, h1, h2, wlen, lane_start + wstart, used, err);
-            in_word = false;
-          }
-          if (!delim) {
-            if (!in_word) { in_word = true; wstart = pos; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
-            h1 = (h1 ^ ch) * 0x100000001b3ull;
-            h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
-            h2 ^= h2 >> 29;
-            ++wlen;
-          }
+    int qn = 0;  // warp-uniform queue fill
+    auto emit = [&](bool end) {
+      const unsigned m = __ballot_sync(kFull, end);
+      if (m) {
+        if (end) {
+          const uint64_t occ = lane_start + wstart;
+          if (wlen >= (1u << 24) || occ >= (1ull << 40)) atomicOr(err, kErrWordTooLong);
+          const int i = qn + __popc(m & lt);
+          sh.qk1[w][i] = h1;
+          sh.qk2[w][i] = h2;
+          sh.qol[w][i] = (occ << 24) | wlen;
+        }
+        qn += __popc(m);
+        if (qn > kWcQ - 32) {
+          wc_flush_queue(sh, w, lane, qn, table, mask, used, err);
+          qn = 0;
         }
       }
-      wc_flush_queue(sh, w, lane, table, mask, used, err);
+    };
+    uint32_t k = pos0 >> 4;
+    bool go = live && pos0 < range_end;
+    while (__any_sync(kFull, go)) {
+      const uint4 v = go ? lane_word(tile, k, col) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        const uint32_t pos = 16 * k + j;
+        // a byte is ours while inside the quarter, or past it while finishing our last word
+        const bool valid = go && pos >= pos0 && pos < d.nbytes && (pos < range_end || in_word || skip);
+        const uint32_t wd = j < 8 ? (j < 4 ? v.x : v.y) : (j < 12 ? v.z : v.w);
+        const uint32_t ch = (wd >> (8 * (j & 3))) & 0xff;
+        const bool boundary = valid && pos == next_b;
+        if (boundary) {
+          do {  // several records may start here if some are empty
+            ++r;
+            next_b = r < rend ? (uint32_t)(rstart(r) - lane_start) : 0xffffffffu;
+          } while (next_b == pos);
+        }
+        const bool delim = is_delim(ch);
+        if (valid && (delim || boundary)) skip = false;
+        const bool end = valid && in_word && (delim || boundary);
+        emit(end);
+        if (end) in_word = false;
+        if (valid && !delim && !skip && (in_word || pos < range_end)) {
+          if (!in_word) { in_word = true; wstart = pos; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
+          h1 = (h1 ^ ch) * 0x100000001b3ull;
+          h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
+          h2 ^= h2 >> 29;
+          ++wlen;
+        }
+      }
+      ++k;
+      go = go && 16 * k < d.nbytes && (16 * k < range_end || in_word || skip);
     }
-    if (in_word) wc_push(sh, w, table, mask, h1, h2, wlen, lane_start + wstart, used, err);
-    wc_flush_queue(sh, w, lane, table, mask, used, err);
+    emit(in_word && live);
+    if (qn) wc_flush_queue(sh, w, lane, qn, table, mask, used, err);
   }
   __syncthreads();
   for (int i = threadIdx.x; i < kWcTab; i += blockDim.x)
@@ -486,8 +522,9 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
 void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                int* err, cudaStream_t s) {
-  k_wc<<<(c.L + kWcBlock - 1) / kWcBlock, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask,
-                                                           used, err);
+  const uint32_t threads = c.L * kWcSub;
+  k_wc<<<(threads + kWcBlock - 1) / kWcBlock, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table,
+                                                                mask, used, err);
 }
 
 void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,

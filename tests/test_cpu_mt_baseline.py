@@ -1,0 +1,22 @@
+"""The multithreaded CPU baseline (paper variant ii) computes the same results as the oracle."""
+import numpy as np
+
+import baselines
+import gen
+import oracle
+
+
+def test_mt_baseline_matches_oracle():
+    buf, off = gen.grep_records(max_bytes=4 << 20)
+    assert np.array_equal(baselines.grep(buf, off), oracle.grep(buf, off))
+    g = gen.groupby(n=300_001, zipf=True)
+    c, q, a = baselines.groupby(g, 300_001)
+    wc, wq, wa = oracle.groupby(g, 300_001, 16, 4096)
+    assert np.array_equal(c, wc) and np.array_equal(q, wq)
+    np.testing.assert_allclose(a, wa, rtol=1e-9)
+    x = gen.points(n=50_000)
+    c, s = baselines.kmeans(x, x[:64])
+    kc, ks, _, _ = oracle.kmeans(x, x[:64])
+    assert np.array_equal(c, kc)
+    np.testing.assert_allclose(s, ks, rtol=1e-9)
+    assert baselines.threads() >= 1
