@@ -83,11 +83,15 @@ typedef struct bk_config {
   uint32_t _reserved;
 } bk_config;
 
-#define BK_FLAG_PROFILE 1u  /* time every stage of every chunk with CUDA events (bk_stats.ms_*) */
+#define BK_FLAG_PROFILE 1u  /* time every stage of every chunk with CUDA events (bk_stats.ms_*); implies
+                               eager issue (no CUDA-graph replay: graph event nodes carry no timestamps) */
 #define BK_FLAG_BASELINE_DBUF 2u  /* run the paper's GPU double-buffering baseline instead (P:329-339,
                                      P:994-996): raw whole-record chunks into 2 buffers (window/2 each)
                                      on 2 streams, kernel over contiguous per-thread record ranges.
                                      BK_K_GREP and BK_K_GROUPBY only; results identical. */
+#define BK_FLAG_NO_GRAPH 8u  /* issue every pipeline eagerly instead of capturing/replaying a CUDA graph
+                               (ZC / DENSE pipelines are otherwise captured on their first run per
+                               kernel, parameters and plan, and replayed by later runs) */
 #define BK_FLAG_BASELINE_SBUF 4u  /* the single-buffer variant: one buffer of the whole window,
                                      copy then compute, no overlap */
 

@@ -96,6 +96,18 @@ struct Plan {
   uint64_t max_acc_rec = 0;            // max accessed bytes of one record
   uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
   std::vector<uint64_t> bounds;        // chunk record bounds
+  std::string key;                     // plan-cache key (also part of the graph key)
+};
+
+// A captured pipeline (CUDA graph) for one (kernel, parameters, plan, output pointers), replayed
+// by later bk_run calls with the same key instead of re-issuing ~10 launches/copies per chunk.
+struct GraphEntry {
+  std::string key;
+  cudaGraphExec_t exec = nullptr;
+  bk_stats st{};
+  int n_launch = 0;
+  size_t prof_used = 0;
+  std::vector<int> prof_stage;
 };
 
 }  // namespace
@@ -140,6 +152,10 @@ struct bk_ctx {
   int n_launch = 0;
   bk_stats st{};
   std::vector<std::pair<std::string, Plan>> plan_cache;
+  std::vector<GraphEntry> graphs;
+  cudaEvent_t ev_fork = nullptr;
+  std::vector<cudaEvent_t> ev_join;
+  float* h_mu = nullptr;   // pinned copy of the k-means centroids (graph memcpy source)
 };
 
 namespace {
@@ -302,6 +318,7 @@ int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t
       return BK_OK;
     }
   const int rc = plan_run_uncached(c, a, lane_target, p, out_per_chunk, auto_mode);
+  p.key = k;
   if (rc == BK_OK) c->plan_cache.emplace_back(k, p);
   return rc;
 }
@@ -602,6 +619,141 @@ int end_run(bk_ctx* c, void* stream) {
   return check_err(c);
 }
 
+// ---- run_device: fork/join all streams around a pipeline; capture it as a CUDA graph once per key
+std::vector<cudaStream_t> side_streams(bk_ctx* c) {
+  std::vector<cudaStream_t> v{c->s_copy, c->s_asm, c->s_d2h};
+  for (auto st : c->s_slot) v.push_back(st);
+  return v;
+}
+
+int device_begin(bk_ctx* c) {
+  BK_CUDA(cudaMemsetAsync(c->d_err, 0, sizeof(int), c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->d_ctr, 0, 8 * sizeof(unsigned long long), c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_fork, c->s_comp));
+  for (auto st : side_streams(c)) BK_CUDA(cudaStreamWaitEvent(st, c->ev_fork, 0));
+  return BK_OK;
+}
+
+int device_end(bk_ctx* c) {
+  const auto ss = side_streams(c);
+  for (size_t i = 0; i < ss.size(); ++i) {
+    BK_CUDA(cudaEventRecord(c->ev_join[i], ss[i]));
+    BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_join[i], 0));
+  }
+  return BK_OK;
+}
+
+void host_reset(bk_ctx* c) {
+  for (auto& s : c->slots) s.used = false;
+  c->n_launch = 0;
+  c->prof_used = 0;
+  c->st.bytes_accessed = c->st.bytes_h2d = c->st.bytes_meta = c->st.bytes_padding = c->st.bytes_d2h = 0;
+  c->st.n_chunks_cpu = 0;
+  c->st.ms_cpu_gather = 0;
+}
+
+int prof_reserve(bk_ctx* c, size_t pairs) {
+  if (!(c->cfg.flags & BK_FLAG_PROFILE)) return BK_OK;
+  while (c->prof.size() < 2 * pairs) {
+    cudaEvent_t e;
+    BK_CUDA(cudaEventCreate(&e));
+    c->prof.push_back(e);
+    if (c->prof.size() % 2 == 0) c->prof_stage.push_back(0);
+  }
+  return BK_OK;
+}
+
+int end_host(bk_ctx* c, void* stream) {
+  BK_CUDA(cudaEventRecord(c->t_end, c->s_comp));   // outside any graph: graph event nodes carry no timestamps
+  BK_CUDA(cudaEventRecord(c->ev_end, c->s_comp));
+  BK_CUDA(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_end, 0));
+  BK_CUDA(cudaStreamSynchronize(c->s_comp));
+  unsigned long long staged = 0;
+  BK_CUDA(cudaMemcpy(&staged, c->d_ctr + 0, 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_padding = staged >= c->st.bytes_accessed ? staged - c->st.bytes_accessed : 0;
+  float ms = 0;
+  BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
+  c->st.ms_device = ms;
+  double acc[kNStages] = {0, 0, 0, 0};
+  uint64_t cnt[kNStages] = {0, 0, 0, 0};
+  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
+    float e = 0;
+    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
+    acc[c->prof_stage[i / 2]] += e;
+    cnt[c->prof_stage[i / 2]] += 1;
+  }
+  c->st.ms_h2d = acc[kStH2D];
+  c->st.ms_addrgen = acc[kStAddrgen];
+  c->st.ms_gather = acc[kStGather];
+  c->st.ms_compute = acc[kStCompute];
+  c->st.n_gather = cnt[kStGather];
+  return check_err(c);
+}
+
+// Runs `enqueue` (which issues one whole pipeline on the context's streams) ordered after `stream`.
+// ZC / DENSE pipelines are fully static for a given key, so the first run captures them as a
+// CUDA graph and later runs replay it (BK_FLAG_NO_GRAPH forces eager issue).
+template <class Enqueue>
+int run_device(bk_ctx* c, void* stream, const std::string& key, bool graphable, size_t n_chunks, Enqueue&& enqueue) {
+  BK_CUDA(cudaSetDevice(c->cfg.device));
+  host_reset(c);
+  BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_begin, 0));
+  BK_CUDA(cudaEventRecord(c->t_begin, c->s_comp));
+  int rc;
+  // per-stage profiling events must be real stream events (timestamps), so BK_FLAG_PROFILE issues eagerly
+  if (!graphable || (c->cfg.flags & (BK_FLAG_NO_GRAPH | BK_FLAG_PROFILE))) {
+    if ((rc = device_begin(c)) || (rc = enqueue()) || (rc = device_end(c))) return rc;
+    return end_host(c, stream);
+  }
+  GraphEntry* ge = nullptr;
+  for (auto& g : c->graphs)
+    if (g.key == key) ge = &g;
+  if (ge) {
+    const double reg = c->st.ms_register;
+    c->st = ge->st;
+    c->st.ms_register = reg;
+    c->n_launch = ge->n_launch;
+    c->prof_used = ge->prof_used;
+    for (size_t i = 0; i < ge->prof_stage.size(); ++i) c->prof_stage[i] = ge->prof_stage[i];
+  } else {
+    if ((rc = prof_reserve(c, 4 * n_chunks + 8))) return rc;
+    BK_CUDA(cudaStreamBeginCapture(c->s_comp, cudaStreamCaptureModeThreadLocal));
+    rc = device_begin(c);
+    if (!rc) rc = enqueue();
+    if (!rc) rc = device_end(c);
+    cudaGraph_t graph = nullptr;
+    const cudaError_t e = cudaStreamEndCapture(c->s_comp, &graph);
+    if (rc) {
+      if (graph) cudaGraphDestroy(graph);
+      cudaGetLastError();
+      return rc;
+    }
+    if (e != cudaSuccess) return fail(BK_E_CUDA, "graph capture: %s", cudaGetErrorString(e));
+    GraphEntry g;
+    g.key = key;
+    const cudaError_t ie = cudaGraphInstantiate(&g.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (ie != cudaSuccess) return fail(BK_E_CUDA, "cudaGraphInstantiate: %s", cudaGetErrorString(ie));
+    g.st = c->st;
+    g.n_launch = c->n_launch;
+    g.prof_used = c->prof_used;
+    g.prof_stage.assign(c->prof_stage.begin(), c->prof_stage.begin() + std::min(c->prof_stage.size(), c->prof_used / 2));
+    c->graphs.push_back(std::move(g));
+    ge = &c->graphs.back();
+  }
+  BK_CUDA(cudaGraphLaunch(ge->exec, c->s_comp));
+  return end_host(c, stream);
+}
+
+void drop_graphs(bk_ctx* c) {
+  for (auto& g : c->graphs)
+    if (g.exec) cudaGraphExecDestroy(g.exec);
+  c->graphs.clear();
+}
+
+bool graphable(const Plan& p) { return p.mode == BK_GATHER_ZC || p.mode == BK_GATHER_DENSE; }
+
 // ------------------------------------------------------------------ kernels
 int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   uint64_t slots = o->table_slots ? o->table_slots : (1ull << 20);
@@ -617,20 +769,23 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
   BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(ocap, 1) * 4));
   BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
-  if ((rc = begin_run(c, stream))) return rc;
-  BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
   WcEntry* table = (WcEntry*)c->b_table.p;
-  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
-    launch_wc(ch, s.stage, s.lanes, s.tile_base, s.meta, c->off ? 0 : c->cfg.record_size, table, slots - 1,
-              c->d_ctr + 1, c->d_err, cs);
+  const std::string key = "wc/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
+    int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_wc(ch, s.stage, s.lanes, s.tile_base, s.meta, c->off ? 0 : c->cfg.record_size, table, slots - 1,
+                c->d_ctr + 1, c->d_err, cs);
+      c->n_launch += 1;
+      return BK_OK;
+    });
+    if (r) return r;
+    launch_wc_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
+                      (uint64_t*)c->b_out3.p, ocap, c->s_comp);
     c->n_launch += 1;
-    return BK_OK;
+    return (int)BK_OK;
   });
   if (rc) return rc;
-  launch_wc_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
-                    (uint64_t*)c->b_out3.p, ocap, c->s_comp);
-  c->n_launch += 1;
-  if ((rc = end_run(c, stream))) return rc;
   unsigned long long nw = 0;
   BK_CUDA(cudaMemcpy(&nw, c->d_ctr + 2, 8, cudaMemcpyDeviceToHost));
   o->n_words = nw;
@@ -667,15 +822,18 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
   gp.plen = o->pattern_len;
   gp.first_index = o->first_index;
   gp.cap = cap;
-  if ((rc = begin_run(c, stream))) return rc;
-  rc = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
-    launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p, c->d_ctr + 3,
-                (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, cs);
-    c->n_launch += 3;
-    return BK_OK;
+  std::string key = "grep/" + std::to_string(gp.plen) + "/" + std::to_string(gp.first_index) + "/" +
+                    std::to_string(gp.cap) + "/" + p.key + "/";
+  for (uint32_t i = 0; i < gp.plen; ++i) key += std::to_string(gp.pat[i]) + ",";
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+    return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p, c->d_ctr + 3,
+                  (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, cs);
+      c->n_launch += 3;
+      return BK_OK;
+    });
   });
   if (rc) return rc;
-  if ((rc = end_run(c, stream))) return rc;
   unsigned long long m = 0;
   BK_CUDA(cudaMemcpy(&m, c->d_ctr + 3, 8, cudaMemcpyDeviceToHost));
   o->n_match = m;
@@ -701,19 +859,20 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
   cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
   per_sm = std::max<int>(1, (int)((200 * 1024) / std::max<size_t>(groupby_smem(G), 1)));
   per_sm = std::min(per_sm, 4);
-  if ((rc = begin_run(c, stream))) return rc;
-  BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)G * 8, c->s_comp));
-  BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)G * 8, c->s_comp));
-  BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)G * 8, c->s_comp));
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * per_sm));
-  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
-    launch_groupby(ch, s.stage, s.lanes, s.tile_base, G, (unsigned long long*)c->b_agg1.p,
-                   (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, cs);
-    c->n_launch += 1;
-    return BK_OK;
+  rc = run_device(c, stream, "groupby/" + std::to_string(G) + "/" + p.key, graphable(p), p.bounds.size() - 1,
+                  [&]() -> int {
+    BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)G * 8, c->s_comp));
+    return pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_groupby(ch, s.stage, s.lanes, s.tile_base, G, (unsigned long long*)c->b_agg1.p,
+                     (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, cs);
+      c->n_launch += 1;
+      return BK_OK;
+    });
   });
   if (rc) return rc;
-  if ((rc = end_run(c, stream))) return rc;
   BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
   BK_CUDA(cudaMemcpy(o->qty, c->b_agg2.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
   BK_CUDA(cudaMemcpy(o->amount, c->b_agg3.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
@@ -753,14 +912,17 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(c->b_agg3.ensure((uint64_t)K * 16 * 8));
   int dev_sms = 148;
   cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
-  if ((rc = begin_run(c, stream))) return rc;
-  BK_CUDA(cudaMemcpyAsync(c->b_mu.p, o->centroids, (uint64_t)K * 64, cudaMemcpyHostToDevice, c->s_comp));
+  if (!c->h_mu) BK_CUDA(cudaHostAlloc((void**)&c->h_mu, 256 * 64, cudaHostAllocPortable));
+  memcpy(c->h_mu, o->centroids, (size_t)K * 64);   // the graph copies from this pinned buffer
+  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
+  const std::string key = "kmeans/" + std::to_string(K) + "/" + std::to_string(o->first_index) + "/" +
+                          std::to_string((uintptr_t)o->cid) + "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+  BK_CUDA(cudaMemcpyAsync(c->b_mu.p, c->h_mu, (uint64_t)K * 64, cudaMemcpyHostToDevice, c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
-  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
-  if (o->cid) BK_CUDA(cudaStreamWaitEvent(c->s_d2h, c->ev_begin, 0));
   size_t ci = 0;
-  rc = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
+  int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
     launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
                   (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4,
                   o->cid ? (int32_t*)s.out : nullptr, grid, cs);
@@ -775,12 +937,9 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
     }
     return (int)BK_OK;
   });
+  return r;
+  });
   if (rc) return rc;
-  if (o->cid) {
-    BK_CUDA(cudaEventRecord(c->ev_end, c->s_d2h));
-    BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
-  }
-  if ((rc = end_run(c, stream))) return rc;
   BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDeviceToHost));
   BK_CUDA(cudaMemcpy(o->sum, c->b_agg3.p, (uint64_t)K * 128, cudaMemcpyDeviceToHost));
   unsigned long long chk = 0;
@@ -812,10 +971,10 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
   BK_CUDA(c->b_totals.ensure(std::max<uint64_t>(C, 1) * B * 8));
   BK_CUDA(c->b_base.ensure((uint64_t)B * 8));
   if ((rc = ensure_out_pinned(c, o->out_records, c->n * 16))) return rc;
-  if ((rc = begin_run(c, stream))) return rc;
-  BK_CUDA(cudaStreamWaitEvent(c->s_d2h, c->ev_begin, 0));
+  const std::string key = "part/" + std::to_string(B) + "/" + std::to_string((uintptr_t)o->out_records) + "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
   size_t ci = 0;
-  rc = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
+  return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
     launch_partition(ch, s.stage, s.lanes, s.tile_base, bits, (uint32_t*)c->b_hist.p, (uint32_t*)c->b_colpre.p,
                      (unsigned long long*)c->b_totals.p + ci * B, (unsigned long long*)c->b_base.p, s.out, cs);
     c->n_launch += 4;
@@ -830,10 +989,8 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
     ++ci;
     return (int)BK_OK;
   });
+  });
   if (rc) return rc;
-  BK_CUDA(cudaEventRecord(c->ev_end, c->s_d2h));
-  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
-  if ((rc = end_run(c, stream))) return rc;
   std::vector<uint64_t> tot(C * B);
   if (C) BK_CUDA(cudaMemcpy(tot.data(), c->b_totals.p, C * B * 8, cudaMemcpyDeviceToHost));
   for (uint32_t b = 0; b < B; ++b) o->bucket_count[b] = 0;
@@ -1076,6 +1233,11 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
   if (cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "d2h stream"));
   if (configure_partition_kernels() != cudaSuccess || configure_baseline_kernels() != cudaSuccess)
     return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
+  if (cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess)
+    return cleanup(fail(BK_E_CUDA, "events"));
+  c->ev_join.assign(3 + c->cfg.n_slots, nullptr);
+  for (auto& e : c->ev_join)
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
   c->ev_part.assign(c->cfg.n_slots, nullptr);
   for (auto& e : c->ev_part)
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
@@ -1155,6 +1317,7 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
   c->n = n;
   c->registered = true;
   c->plan_cache.clear();
+  drop_graphs(c);
   c->st.ms_register = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return BK_OK;
 }
@@ -1258,6 +1421,10 @@ int bk_destroy(bk_ctx* c) {
   if (c->t_begin) cudaEventDestroy(c->t_begin);
   if (c->t_end) cudaEventDestroy(c->t_end);
   for (cudaEvent_t e : c->prof) cudaEventDestroy(e);
+  drop_graphs(c);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  for (auto e : c->ev_join) cudaEventDestroy(e);
+  if (c->h_mu) cudaFreeHost(c->h_mu);
   delete c->pool;
   if (c->s_d2h) {
     cudaStreamSynchronize(c->s_d2h);

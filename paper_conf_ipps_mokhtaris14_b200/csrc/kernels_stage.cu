@@ -183,13 +183,26 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
     uint8_t* tile = stage + tile_base[w];
     const uint32_t K = (uint32_t)((tile_base[w + 1] - tile_base[w]) >> 9);
     const uint4* in = reinterpret_cast<const uint4*>(abase);
-    uint4 cur = lane < (int)NW ? ld16<kHost>(in + lane) : make_uint4(0, 0, 0, 0);
+    // kDepth 512-B warp loads in flight per warp (PCIe latency x bandwidth needs ~100 KB in
+    // flight chip-wide; a chunk may have only a few hundred tiles)
+    constexpr int kDepth = 4;
+    uint4 ring[kDepth];
+#pragma unroll
+    for (int i = 0; i < kDepth; ++i) {
+      const uint32_t jj = i * 32 + lane;
+      ring[i] = jj < NW ? ld16<kHost>(in + jj) : make_uint4(0, 0, 0, 0);
+    }
     for (uint32_t blk = 0; blk * 32 < NW; ++blk) {
-      const uint32_t jn = (blk + 1) * 32 + lane;
-      const uint4 nxt = jn < NW ? ld16<kHost>(in + jn) : make_uint4(0, 0, 0, 0);
+      const uint4 cur = ring[0];
       uint4 hi = shfl_down_u4(cur, 1);
-      const uint4 n0 = shfl_u4(nxt, 0);
+      const uint4 n0 = shfl_u4(ring[1], 0);
       if (lane == 31) hi = n0;
+#pragma unroll
+      for (int i = 0; i + 1 < kDepth; ++i) ring[i] = ring[i + 1];
+      {
+        const uint32_t jn = (blk + kDepth) * 32 + lane;
+        ring[kDepth - 1] = jn < NW ? ld16<kHost>(in + jn) : make_uint4(0, 0, 0, 0);
+      }
       const uint32_t j = blk * 32 + lane;
       // ta = last lane whose first word is <= j (sw is non-decreasing over lanes)
       int ta = 0;
@@ -217,7 +230,6 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
           if (swt == j && tt > 0) t = tt - 1; else active = false;
         }
       }
-      cur = nxt;
     }
     zero_holes(tile, K, W, lane);
   }

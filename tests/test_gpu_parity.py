@@ -352,6 +352,46 @@ def test_groupby_bench_scale():
     np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
 
 
+# ------------------------------------------------------------------ CUDA-graph replay == eager issue
+@pytest.mark.parametrize("no_graph", [False, True])
+def test_repeated_runs_graph_replay(no_graph):
+    """The first run of a static (ZC/DENSE) pipeline is captured as a CUDA graph, later runs replay
+    it; results and stats must equal the eager path on every repetition."""
+    buf, off = gen.text(cap_bytes=3 * MIB)
+    want = oracle.wc(buf, off)
+    gb, goff = gen.grep_records(max_bytes=8 * MIB)
+    gwant = oracle.grep(gb, goff, b"bigk")
+    n = 200_000
+    x = gen.points(n=n)
+    kc, ks, kchk, kcid = oracle.kmeans(x, x[:64], want_cid=True)
+    kv = gen.kv(n=300_000)
+    wboff, wout = oracle.partition(kv, 256)
+    with bk.Context(window_bytes=1 * MIB, no_graph=no_graph) as ctx:
+        ctx.register(buf, off)
+        for _ in range(3):
+            assert wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 17)) == want
+            st = ctx.stats()
+            assert st["bytes_accessed"] == len(buf) and st["n_chunks"] >= 4
+    with bk.Context(window_bytes=2 * MIB, gather_mode="zc", no_graph=no_graph) as ctx:
+        ctx.register(gb, goff)
+        for pat in (b"bigk", b"zz", b"bigk"):
+            got = ctx.grep(pat, cap=len(goff))
+            assert np.array_equal(got, oracle.grep(gb, goff, pat))
+    with bk.Context(window_bytes=2 * MIB, record_size=64, no_graph=no_graph) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=n)
+        for _ in range(2):
+            cid = np.full(n, -1, np.int32)
+            c, s, chk = ctx.kmeans(x[:64], cid=cid)
+            assert np.array_equal(cid, kcid) and chk == kchk and np.array_equal(c, kc)
+    with bk.Context(window_bytes=2 * MIB, record_size=16, no_graph=no_graph) as ctx:
+        ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=len(kv))
+        out = np.empty_like(kv)
+        for _ in range(2):
+            out[:] = 0
+            o, cc, bc = ctx.partition(256, out=out)
+            assert np.array_equal(global_from_runs(o, cc), wout)
+
+
 # ------------------------------------------------------------------ invariants + API errors
 def test_invariance_across_window_slots_lanes_modes():
     buf, off = gen.text(cap_bytes=1 * MIB)
