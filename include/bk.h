@@ -48,7 +48,9 @@ typedef enum {
   BK_K_KMEANS = 3,      /* C3: assignment + per-cluster partial sums      bk_out_kmeans */
   BK_K_PARTITION = 4,   /* C4: stable hash partition into B buckets                    bk_out_partition */
   BK_K_GROUPBY = 5,     /* C5: group-by count / sum                                    bk_out_groupby */
-  BK_K_LAYOUT_DUMP = 100 /* test only: copy one chunk's staged bytes + lane table back       bk_out_layout */
+  BK_K_LAYOUT_DUMP = 100, /* test only: copy one chunk's staged bytes + lane table back      bk_out_layout */
+  BK_K_PATTERN_STATS = 101 /* stage 1 in address mode + online pattern recognition over
+                              every lane's element-address stream; Table II accounting     bk_out_pattern */
 } bk_kernel_id;
 
 /* Stage-2/3 implementations. */
@@ -201,6 +203,28 @@ typedef struct bk_out_layout {
   uint64_t chunk_lo, chunk_hi, n_chunks; /* out */
 } bk_out_layout;
 
+typedef struct bk_out_pattern {
+  bk_out_header h;
+  uint32_t n_ext;           /* in: access spec, 0 = whole record, else extents (<= 8) */
+  uint32_t ext_off[8];
+  uint32_t ext_len[8];
+  uint32_t elem_bytes;      /* in: element size of the address stream (1 = every byte, 4 = fp32 ...) */
+  uint32_t T;               /* in: temporary address buffer entries, 2..16 */
+  uint32_t pmax;            /* in: longest stride period tried, 1..4 */
+  uint32_t _pad;
+  uint64_t chunk;           /* in: chunk whose per-lane results are dumped (UINT64_MAX: none) */
+  int32_t* lane_p;          /* out (dump): per lane period, 0 = explicit addresses */
+  int64_t* lane_strides;    /* out (dump): 4 per lane */
+  uint64_t* lane_base;      /* out (dump): first address (offset in the data set) */
+  uint64_t* lane_count;     /* out (dump): addresses generated */
+  uint64_t lane_cap;        /* in: capacity of the dump arrays in lanes */
+  uint32_t lanes;           /* out: lanes per chunk */
+  uint32_t _pad2;
+  uint64_t n_lanes, n_pattern_lanes, n_addresses, n_explicit_addresses; /* out: totals over all chunks */
+  uint64_t address_bytes;   /* out: 8 B per address if every address were sent (the paper's addrBuf) */
+  uint64_t pattern_bytes;   /* out: descriptors for pattern lanes + 8 B per explicit fallback address */
+} bk_out_pattern;
+
 typedef struct bk_stats {
   uint32_t struct_size;
   uint32_t gather_mode;       /* mode the last run used */
@@ -230,7 +254,7 @@ typedef struct bk_stats {
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);
 
 /* ABI self-check for bindings: writes sizeof of bk_config, bk_out_wordcount, bk_out_grep,
- * bk_out_kmeans, bk_out_partition, bk_out_groupby, bk_out_layout, bk_stats (in that order,
+ * bk_out_kmeans, bk_out_partition, bk_out_groupby, bk_out_layout, bk_stats, bk_out_pattern (in that order,
  * up to n entries) and returns BK_ABI_VERSION. Needs no GPU. */
 BK_API int bk_abi_sizes(uint32_t* sizes, int n);
 

@@ -46,6 +46,8 @@ def lib():
         l.oracle_layout.argtypes = [p, p, u64, u64, u64, u32, p, p, u64, u64, u32, p, p, p, p, u64]
         l.oracle_pattern.restype = C.c_int
         l.oracle_pattern.argtypes = [p, u32, u32, p]
+        l.oracle_pattern_online.restype = C.c_int
+        l.oracle_pattern_online.argtypes = [p, u64, u32, u32, p]
         _lib = l
     return _lib
 
@@ -165,6 +167,16 @@ def layout(buf, off, n: int, nbytes: int, rec_size: int, extents, lo: int, hi: i
         assert size2 == size
         stage = stage[:size]
     return stage, lf, ln, lb
+
+
+def pattern_online(addrs, T: int = 8, pmax: int = 4):
+    """O-P online: detect on the first T addresses, verify the rest; (base, strides) or None."""
+    a = np.ascontiguousarray(addrs, np.uint64)
+    st = np.empty(max(pmax, 1), np.int64)
+    p = lib().oracle_pattern_online(_p(a) if len(a) else None, len(a), T, pmax, _p(st))
+    if p == 0:
+        return None
+    return int(a[0]), [int(v) for v in st[:p]]
 
 
 def pattern(addrs, pmax: int = 4):

@@ -265,6 +265,15 @@ int64_t oracle_layout(const uint8_t* d, const uint64_t* off, uint64_t n, uint64_
 }
 
 /* ------------------------------------------------------------------ O-P pattern */
+int oracle_pattern_online(const uint64_t* a, uint64_t n, uint32_t T, uint32_t pmax, int64_t* strides) {
+  uint32_t first = n < T ? (uint32_t)n : T;
+  int p = oracle_pattern(a, first, pmax, strides);
+  if (p == 0) return 0;
+  for (uint64_t k = first; k < n; ++k)   /* verify each subsequently generated address */
+    if ((int64_t)(a[k] - a[k - 1]) != strides[(k - 1) % (uint64_t)p]) return 0;
+  return p;
+}
+
 int oracle_pattern(const uint64_t* a, uint32_t n, uint32_t pmax, int64_t* strides) {
   if (n < 2) return 0;
   for (uint32_t p = 1; p <= pmax && p + 1 < n; ++p) { /* >= 1 delta beyond the first period verifies it */

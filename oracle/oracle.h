@@ -87,6 +87,12 @@ int64_t oracle_layout(const uint8_t* d, const uint64_t* off, uint64_t n, uint64_
  * the first period (n-1 > p: 'verifies that each subsequently generated address follows'). Returns p (base = a[0]) or 0. */
 int oracle_pattern(const uint64_t* a, uint32_t n, uint32_t pmax, int64_t* strides);
 
+/* Online form of the same detector: detect on the first T addresses only ("a few
+ * addresses, storing them in a private temporary address buffer"), then verify that every later
+ * address follows the pattern; the first mismatch abandons it (fallback to explicit addresses).
+ * Returns p or 0. */
+int oracle_pattern_online(const uint64_t* a, uint64_t n, uint32_t T, uint32_t pmax, int64_t* strides);
+
 #ifdef __cplusplus
 }
 #endif

@@ -77,8 +77,17 @@ class bk_stats(C.Structure):
                 ("ms_compute", C.c_double), ("n_gather", u64), ("n_chunks_cpu", u64), ("ms_cpu_gather", C.c_double)]
 
 
+class bk_out_pattern(C.Structure):
+    _fields_ = [("h", bk_out_header), ("n_ext", u32), ("ext_off", u32 * 8), ("ext_len", u32 * 8), ("elem_bytes", u32),
+                ("T", u32), ("pmax", u32), ("_pad", u32), ("chunk", u64), ("lane_p", P), ("lane_strides", P),
+                ("lane_base", P), ("lane_count", P), ("lane_cap", u64), ("lanes", u32), ("_pad2", u32),
+                ("n_lanes", u64), ("n_pattern_lanes", u64), ("n_addresses", u64), ("n_explicit_addresses", u64),
+                ("address_bytes", u64), ("pattern_bytes", u64)]
+
+
+BK_K_PATTERN_STATS = 101
 ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,
-               bk_out_layout, bk_stats]
+               bk_out_layout, bk_stats, bk_out_pattern]
 EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_destroy", "bk_strerror", "bk_last_error",
            "bk_get_stats", "bk_abi_sizes"]
 
@@ -121,8 +130,8 @@ def check(status: int, where: str) -> None:
 
 
 def abi_sizes() -> list[int]:
-    a = (u32 * 8)()
-    lib().bk_abi_sizes(a, 8)
+    a = (u32 * len(ABI_STRUCTS))()
+    lib().bk_abi_sizes(a, len(ABI_STRUCTS))
     return list(a)
 
 
@@ -265,6 +274,27 @@ class Context:
         bk_run(self.ctx, BK_K_PARTITION, stream, o)
         C = o.n_chunks
         return out, cc[: C * n_buckets].reshape(C, n_buckets), bc
+
+    def pattern_stats(self, extents=None, elem_bytes: int = 1, T: int = 8, pmax: int = 4, chunk: int | None = None,
+                      lane_cap: int = 1 << 20, stream=None):
+        """Stage 1 in address mode + online pattern recognition over every lane.
+        Returns the totals dict and, for `chunk`, per-lane (p, strides[4], base, count)."""
+        o = _hdr(bk_out_pattern, BK_K_PATTERN_STATS)
+        extents = extents or []
+        o.n_ext = len(extents)
+        for i, (eo, el) in enumerate(extents):
+            o.ext_off[i], o.ext_len[i] = eo, el
+        o.elem_bytes, o.T, o.pmax = elem_bytes, T, pmax
+        p_ = np.empty(lane_cap, np.int32); st = np.empty((lane_cap, 4), np.int64)
+        base = np.empty(lane_cap, np.uint64); cnt = np.empty(lane_cap, np.uint64)
+        o.chunk = chunk if chunk is not None else (1 << 64) - 1
+        o.lane_p, o.lane_strides, o.lane_base, o.lane_count, o.lane_cap = _ptr(p_), _ptr(st), _ptr(base), _ptr(cnt), lane_cap
+        bk_run(self.ctx, BK_K_PATTERN_STATS, stream, o)
+        tot = {k: getattr(o, k) for k in ("n_lanes", "n_pattern_lanes", "n_addresses", "n_explicit_addresses",
+                                          "address_bytes", "pattern_bytes", "lanes")}
+        L = o.lanes
+        lanes = (p_[:L].copy(), st[:L].copy(), base[:L].copy(), cnt[:L].copy()) if chunk is not None else None
+        return tot, lanes
 
     def layout_dump(self, chunk: int, extents=None, stage_cap: int = 1 << 26, lane_cap: int = 1 << 20, stream=None):
         o = _hdr(bk_out_layout, BK_K_LAYOUT_DUMP)

@@ -119,4 +119,9 @@ void launch_dbuf_groupby(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t 
                          cudaStream_t s);
 cudaError_t configure_baseline_kernels();
 
+// ---- online pattern recognition of stage 1 (kernels_pattern.cu, NEXT f2) ----
+void launch_addr_patterns(const Chunk& c, const Access& a, const uint64_t* meta, const LaneDesc* lanes, uint32_t elem,
+                          uint32_t T, uint32_t pmax, int32_t* lane_p, int64_t* lane_strides, uint64_t* lane_base,
+                          uint64_t* lane_count, unsigned long long* totals, int dump, cudaStream_t s);
+
 }  // namespace bk

@@ -1113,24 +1113,83 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
   return BK_OK;
 }
 
-int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
-  Access a{};
-  if (o->n_ext == 0) {
+// caller-given access spec (test / experiment kernels): n_ext == 0 = whole record
+int parse_access(const bk_ctx* c, uint32_t n_ext, const uint32_t* eo, const uint32_t* el, Access& a) {
+  a = Access{};
+  if (n_ext == 0) {
     a = whole_access();
-  } else {
-    if (o->n_ext > (uint32_t)kMaxExt) return fail(BK_E_INVAL, "n_ext > %d", kMaxExt);
-    a.whole = 0;
-    a.n_ext = o->n_ext;
-    for (uint32_t e = 0; e < o->n_ext; ++e) {
-      a.ext_off[e] = o->ext_off[e];
-      a.ext_len[e] = o->ext_len[e];
-      a.E += o->ext_len[e];
-      if ((uint64_t)o->ext_off[e] + o->ext_len[e] > c->min_rec)
-        return fail(BK_E_INVAL, "extent %u exceeds the shortest record", e);
-    }
+    return BK_OK;
   }
+  if (n_ext > (uint32_t)kMaxExt) return fail(BK_E_INVAL, "n_ext > %d", kMaxExt);
+  a.n_ext = n_ext;
+  for (uint32_t e = 0; e < n_ext; ++e) {
+    a.ext_off[e] = eo[e];
+    a.ext_len[e] = el[e];
+    a.E += el[e];
+    if ((uint64_t)eo[e] + el[e] > c->min_rec) return fail(BK_E_INVAL, "extent %u exceeds the shortest record", e);
+  }
+  return BK_OK;
+}
+
+// BK_K_PATTERN_STATS: stage 1 in address mode with online pattern recognition, every chunk
+int run_pattern(bk_ctx* c, bk_out_pattern* o, void* stream) {
+  Access a;
+  int rc = parse_access(c, o->n_ext, o->ext_off, o->ext_len, a);
+  if (rc) return rc;
+  if (o->elem_bytes == 0 || o->T < 2 || o->T > 16 || o->pmax < 1 || o->pmax > 4)
+    return fail(BK_E_INVAL, "elem_bytes >= 1, T in 2..16, pmax in 1..4");
   Plan p;
-  int rc = plan_run(c, a, 256, p);
+  if ((rc = plan_run(c, a, 256, p))) return rc;
+  carve(c, p);
+  a.rec_size = c->off ? 0 : c->cfg.record_size;
+  o->lanes = p.L;
+  const bool want_dump = o->chunk != UINT64_MAX;
+  if (want_dump && (o->chunk >= p.bounds.size() - 1 || p.L > o->lane_cap))
+    return fail(BK_E_INVAL, "dump chunk / lane_cap");
+  BK_CUDA(c->b_out1.ensure((uint64_t)p.L * 4));
+  BK_CUDA(c->b_out2.ensure((uint64_t)p.L * 32));
+  BK_CUDA(c->b_out3.ensure((uint64_t)p.L * 16));
+  BK_CUDA(c->b_blk2.ensure(8 * 8));
+  if ((rc = begin_run(c, stream))) return rc;
+  BK_CUDA(cudaMemsetAsync(c->b_blk2.p, 0, 64, c->s_copy));
+  Slot& s = c->slots[0];
+  for (size_t i = 0; i + 1 < p.bounds.size(); ++i) {  // one stream, one slot: stage 1 only
+    const Chunk ch = chunk_of(c, p, i);
+    if (c->off && ch.hi > ch.lo)
+      BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_copy);
+    uint64_t* dumps = (uint64_t*)c->b_out3.p;
+    launch_addr_patterns(ch, a, s.meta, s.lanes, o->elem_bytes, o->T, o->pmax, (int32_t*)c->b_out1.p,
+                         (int64_t*)c->b_out2.p, dumps, dumps + p.L, (unsigned long long*)c->b_blk2.p,
+                         want_dump && i == o->chunk, c->s_copy);
+    c->n_launch += 3;
+  }
+  BK_CUDA(cudaEventRecord(c->ev_end, c->s_copy));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
+  if ((rc = end_run(c, stream))) return rc;
+  unsigned long long tot[5];
+  BK_CUDA(cudaMemcpy(tot, c->b_blk2.p, sizeof tot, cudaMemcpyDeviceToHost));
+  o->n_lanes = tot[0];
+  o->n_pattern_lanes = tot[1];
+  o->n_addresses = tot[2];
+  o->n_explicit_addresses = tot[3];
+  o->address_bytes = 8 * tot[2];
+  o->pattern_bytes = tot[4] + 8 * tot[3];
+  if (want_dump) {
+    BK_CUDA(cudaMemcpy(o->lane_p, c->b_out1.p, (uint64_t)p.L * 4, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->lane_strides, c->b_out2.p, (uint64_t)p.L * 32, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->lane_base, c->b_out3.p, (uint64_t)p.L * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->lane_count, (uint64_t*)c->b_out3.p + p.L, (uint64_t)p.L * 8, cudaMemcpyDeviceToHost));
+  }
+  return BK_OK;
+}
+
+int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
+  Access a;
+  int rc = parse_access(c, o->n_ext, o->ext_off, o->ext_len, a);
+  if (rc) return rc;
+  Plan p;
+  rc = plan_run(c, a, 256, p);
   if (rc) return rc;
   carve(c, p);
   o->n_chunks = p.bounds.size() - 1;
@@ -1357,6 +1416,10 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
       if (h->struct_size != sizeof(bk_out_groupby)) return fail(BK_E_INVAL, "bk_out_groupby size");
       rc = run_groupby(c, (bk_out_groupby*)out, stream);
       break;
+    case BK_K_PATTERN_STATS:
+      if (h->struct_size != sizeof(bk_out_pattern)) return fail(BK_E_INVAL, "bk_out_pattern size");
+      rc = run_pattern(c, (bk_out_pattern*)out, stream);
+      break;
     case BK_K_LAYOUT_DUMP:
       if (h->struct_size != sizeof(bk_out_layout)) return fail(BK_E_INVAL, "bk_out_layout size");
       rc = run_layout(c, (bk_out_layout*)out, stream);
@@ -1390,9 +1453,10 @@ int bk_get_stats(const bk_ctx* c, bk_stats* s) {
 }
 
 int bk_abi_sizes(uint32_t* sizes, int n) {
-  const uint32_t v[8] = {sizeof(bk_config), sizeof(bk_out_wordcount), sizeof(bk_out_grep), sizeof(bk_out_kmeans),
-                         sizeof(bk_out_partition), sizeof(bk_out_groupby), sizeof(bk_out_layout), sizeof(bk_stats)};
-  for (int i = 0; i < n && i < 8; ++i) sizes[i] = v[i];
+  const uint32_t v[9] = {sizeof(bk_config),        sizeof(bk_out_wordcount), sizeof(bk_out_grep),
+                         sizeof(bk_out_kmeans),    sizeof(bk_out_partition), sizeof(bk_out_groupby),
+                         sizeof(bk_out_layout),    sizeof(bk_stats),         sizeof(bk_out_pattern)};
+  for (int i = 0; i < n && i < 9; ++i) sizes[i] = v[i];
   return BK_ABI_VERSION;
 }
 

@@ -127,6 +127,30 @@ def test_pattern_paper_example():
         assert base == g[key]["base"] and strides == g[key]["strides"]
 
 
+def test_pattern_online_detect_then_verify():
+    g = golden("pattern_example.json")
+    # the paper's example, extended: the detected stride holds for every later address
+    a = list(range(100, 100 + 5 * 40, 5))
+    assert oracle.pattern_online(a, T=4) == (100, [5])
+    assert oracle.pattern_online(g["decimal_reading"]["addrs"], T=8) == (100, [5])
+    # a late mismatch abandons the pattern ("If it does not, then address generation
+    # is started again, this time without attempting to identify a pattern")
+    assert oracle.pattern_online(a[:30] + [a[29] + 7] + a[31:], T=4) is None
+    # detection sees only the first T: a longer true period is missed (fallback), unlike the
+    # whole-list detector
+    b = [0, 1, 2, 3, 10, 11, 12, 13, 20, 21, 22, 23]
+    assert oracle.pattern(b) == (0, [1, 1, 1, 7])
+    assert oracle.pattern_online(b, T=4) is None
+    assert oracle.pattern_online(b, T=8) == (0, [1, 1, 1, 7])
+    # byte addresses of a contiguous text lane (WC, 1-byte elements) and fp32 fields of 64-B
+    # records (K-means, 4-byte elements) reduce to one stride
+    assert oracle.pattern_online(list(range(1000, 1300)), T=8) == (1000, [1])
+    assert oracle.pattern_online([r * 64 + 4 * j for r in range(10) for j in range(16)], T=8) == (0, [4])
+    # sparse group-by: {key, qty, amount} = 4 + 4 + 8 bytes at +0 of 64-B records, 4-byte elements
+    assert oracle.pattern_online([r * 64 + e for r in range(20) for e in (0, 4, 8, 12)], T=8) == (0, [4, 4, 4, 52])
+    assert oracle.pattern_online([7], T=8) is None and oracle.pattern_online([], T=8) is None
+
+
 def test_pattern_fallback_and_multi_stride():
     assert oracle.pattern([10, 13, 20, 27, 40]) is None  # no period <= 4 fits -> explicit list
     assert oracle.pattern([0, 4, 8, 64, 68, 72, 128], pmax=4) == (0, [4, 4, 56])
