@@ -35,6 +35,10 @@ struct Chunk {
   uint32_t L;            // lanes
   uint32_t ntiles;       // L / 32
   uint64_t accessed;     // A(lo, hi)
+  // gather source bounds, in bytes around src: [src - guard_lo, src + guard_hi) is readable
+  // (zero-copy: the registered data set; DENSE: the raw slot). Aligned 16-B words that would
+  // straddle a bound are assembled from in-range bytes only.
+  uint64_t guard_lo, guard_hi;
 };
 
 // Device error bits (sticky, read back at the end of bk_run).

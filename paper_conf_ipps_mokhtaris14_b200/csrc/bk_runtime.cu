@@ -460,7 +460,10 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     BK_CUDA(cudaEventRecord(s.copied, c->s_asm));
     BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.copied, 0));
     BK_PROF(kStGather, c->s_copy, true);
-    launch_gather(ch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1,
+    Chunk gch = ch;   // readable source: the registered data set
+    gch.guard_lo = ch.base_byte;
+    gch.guard_hi = c->nbytes - ch.base_byte;
+    launch_gather(gch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1,
                   c->s_copy);
     BK_PROF(kStGather, c->s_copy, false);
     c->n_launch += 3;
@@ -482,7 +485,10 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
     BK_PROF(kStAddrgen, c->s_asm, false);
     BK_PROF(kStGather, c->s_asm, true);
-    launch_gather(ch, a, s.raw + raw_off, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 0, c->s_asm);
+    Chunk gch = ch;   // readable source: the raw slot (256-B aligned, 64 B of slack)
+    gch.guard_lo = raw_off;
+    gch.guard_hi = p.raw_cap - raw_off;
+    launch_gather(gch, a, s.raw + raw_off, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 0, c->s_asm);
     BK_PROF(kStGather, c->s_asm, false);
     c->n_launch += 3;
     c->st.bytes_h2d += bytes;

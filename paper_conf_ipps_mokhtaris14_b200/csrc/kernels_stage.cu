@@ -113,6 +113,18 @@ __device__ __forceinline__ uint4 ld16(const uint4* p) {
   return __ldcs(p);
 }
 
+// 16-B aligned load limited to the readable source range [lo, hi): interior words are one vector
+// load; a word straddling a bound (data-set edges only) is assembled from in-range bytes.
+template <bool kHost>
+__device__ __forceinline__ uint4 ld16b(const uint4* p, const uint8_t* lo, const uint8_t* hi) {
+  const uint8_t* b = reinterpret_cast<const uint8_t*>(p);
+  if (b >= lo && b + 16 <= hi) return ld16<kHost>(p);
+  uint32_t w[4] = {0, 0, 0, 0};
+  for (int q = 0; q < 16; ++q)
+    if (b + q >= lo && b + q < hi) w[q >> 2] |= (uint32_t)b[q] << (8 * (q & 3));
+  return make_uint4(w[0], w[1], w[2], w[3]);
+}
+
 // out bytes q = concat(a, b)[s + q], s in [0, 16)
 __device__ __forceinline__ uint4 shift_bytes(uint4 a, uint4 b, uint32_t s) {
   const uint32_t bs = (s & 3) * 8;
@@ -167,6 +179,8 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
                                                       const uint64_t* __restrict__ tile_base,
                                                       uint8_t* __restrict__ stage, uint64_t cap) {
   if (tile_base[c.ntiles] > cap) return;  // stage-1 flagged an overflow: never write past the slot
+  const uint8_t* glo = src - c.guard_lo;
+  const uint8_t* ghi = src + c.guard_hi;
   const int lane = threadIdx.x & 31;
   const uint32_t nw_grid = gridDim.x * (blockDim.x >> 5);
   for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < c.ntiles; w += nw_grid) {
@@ -190,7 +204,7 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
 #pragma unroll
     for (int i = 0; i < kDepth; ++i) {
       const uint32_t jj = i * 32 + lane;
-      ring[i] = jj < NW ? ld16<kHost>(in + jj) : make_uint4(0, 0, 0, 0);
+      ring[i] = jj < NW ? ld16b<kHost>(in + jj, glo, ghi) : make_uint4(0, 0, 0, 0);
     }
     for (uint32_t blk = 0; blk * 32 < NW; ++blk) {
       const uint4 cur = ring[0];
@@ -201,7 +215,7 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
       for (int i = 0; i + 1 < kDepth; ++i) ring[i] = ring[i + 1];
       {
         const uint32_t jn = (blk + kDepth) * 32 + lane;
-        ring[kDepth - 1] = jn < NW ? ld16<kHost>(in + jn) : make_uint4(0, 0, 0, 0);
+        ring[kDepth - 1] = jn < NW ? ld16b<kHost>(in + jn, glo, ghi) : make_uint4(0, 0, 0, 0);
       }
       const uint32_t j = blk * 32 + lane;
       // ta = last lane whose first word is <= j (sw is non-decreasing over lanes)
@@ -245,6 +259,8 @@ __global__ void __launch_bounds__(256) k_gather_field(Chunk c, Access a, const u
                                                       const uint64_t* __restrict__ tile_base,
                                                       uint8_t* __restrict__ stage, uint64_t cap) {
   if (tile_base[c.ntiles] > cap) return;  // stage-1 flagged an overflow: never write past the slot
+  const uint8_t* glo = src - c.guard_lo;
+  const uint8_t* ghi = src + c.guard_hi;
   const int lane = threadIdx.x & 31;
   const int g = lane / G, q = lane % G;
   const uint32_t EW = a.E >> 4;
@@ -284,7 +300,7 @@ __global__ void __launch_bounds__(256) k_gather_field(Chunk c, Access a, const u
         const uintptr_t ab = (uintptr_t)p & ~(uintptr_t)15;
         s = (uint32_t)((uintptr_t)p - ab);
         const uint32_t NI = (s + a.E + 15) >> 4;
-        if ((uint32_t)q < NI) v = ld16<kHost>(reinterpret_cast<const uint4*>(ab) + q);
+        if ((uint32_t)q < NI) v = ld16b<kHost>(reinterpret_cast<const uint4*>(ab) + q, glo, ghi);
       }
       const uint4 hi = shfl_down_u4(v, 1, G);
       if (valid && (uint32_t)q < EW) {
@@ -305,6 +321,8 @@ __global__ void __launch_bounds__(256) k_gather_bytes(Chunk c, Access a, const u
                                                       const uint64_t* __restrict__ tile_base,
                                                       uint8_t* __restrict__ stage, uint64_t cap) {
   if (tile_base[c.ntiles] > cap) return;  // stage-1 flagged an overflow: never write past the slot
+  const uint8_t* glo = src - c.guard_lo;
+  const uint8_t* ghi = src + c.guard_hi;
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
   if (t >= c.L) return;
   const int lane = t & 31;

@@ -1,0 +1,33 @@
+"""Small out-of-core runs of every kernel and gather mode, for compute-sanitizer (SURVEY §4:
+memcheck / racecheck / synccheck with tiny windows so many chunks and slot reuse occur)."""
+import sys
+
+sys.path.insert(0, "/root/repo")
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+from paper_conf_ipps_mokhtaris14_b200 import bk  # noqa: E402
+
+buf, off = gen.text(cap_bytes=1 << 19)
+for mode in ("zc", "dense", "cpu"):
+    with bk.Context(window_bytes=96 << 10, n_slots=3, gather_mode=mode, no_graph=True) as ctx:
+        ctx.register(buf, off)
+        ctx.wordcount(cap=1 << 16)
+gb, goff = gen.grep_records(n=20000)
+for mode in ("zc", "hybrid"):
+    with bk.Context(window_bytes=256 << 10, n_slots=3, gather_mode=mode) as ctx:
+        ctx.register(gb, goff)
+        ctx.grep(b"bigk", cap=20000)
+g = gen.groupby(n=100_000, stride=64)
+with bk.Context(window_bytes=512 << 10, record_size=64) as ctx:
+    ctx.register(g, None, n_records=100_000)
+    ctx.groupby(4096)
+x = gen.points(n=50_000)
+with bk.Context(window_bytes=512 << 10, record_size=64) as ctx:
+    ctx.register(x.view(np.uint8).reshape(-1), None, n_records=50_000)
+    ctx.kmeans(x[:64], cid=np.empty(50_000, np.int32))
+kv = gen.kv(n=100_000)
+with bk.Context(window_bytes=1 << 20, record_size=16) as ctx:
+    ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=100_000)
+    ctx.partition(1024)
+print("sanitize run done")
