@@ -94,6 +94,8 @@ typedef struct bk_config {
 #define BK_FLAG_NO_GRAPH 8u  /* issue every pipeline eagerly instead of capturing/replaying a CUDA graph
                                (ZC / DENSE pipelines are otherwise captured on their first run per
                                kernel, parameters and plan, and replayed by later runs) */
+#define BK_FLAG_TEST_DELAYS 16u  /* test only: random spin kernels before every stage on every stream and
+                                   host sleeps before CPU assembly, to expose missing ordering */
 #define BK_FLAG_BASELINE_SBUF 4u  /* the single-buffer variant: one buffer of the whole window,
                                      copy then compute, no overlap */
 

@@ -21,6 +21,7 @@ BK_FLAG_PROFILE = 1
 BK_FLAG_BASELINE_DBUF = 2
 BK_FLAG_BASELINE_SBUF = 4
 BK_FLAG_NO_GRAPH = 8
+BK_FLAG_TEST_DELAYS = 16
 GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE, "hybrid": BK_GATHER_HYBRID}
 
 u32, i32, u64, P = C.c_uint32, C.c_int32, C.c_uint64, C.c_void_p
@@ -147,13 +148,15 @@ def _ptr(a) -> int | None:
 def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_mode: int | str = 0,
               chunk_bytes: int = 0, lanes: int = 0, record_size: int = 0, host_threads: int = 0,
               profile: bool = False, baseline_dbuf: bool = False, lane_bytes: int = 0,
-              zc_share_pm: int = 0, baseline_sbuf: bool = False, no_graph: bool = False) -> int:
+              zc_share_pm: int = 0, baseline_sbuf: bool = False, no_graph: bool = False,
+              test_delays: bool = False) -> int:
     if isinstance(gather_mode, str):
         gather_mode = GATHER_NAMES[gather_mode]
     cfg = bk_config(C.sizeof(bk_config), device, window_bytes, n_slots, gather_mode, chunk_bytes, lanes,
                     host_threads, record_size,
                     (BK_FLAG_PROFILE if profile else 0) | (BK_FLAG_BASELINE_DBUF if baseline_dbuf else 0) |
-                    (BK_FLAG_BASELINE_SBUF if baseline_sbuf else 0) | (BK_FLAG_NO_GRAPH if no_graph else 0),
+                    (BK_FLAG_BASELINE_SBUF if baseline_sbuf else 0) | (BK_FLAG_NO_GRAPH if no_graph else 0) |
+                    (BK_FLAG_TEST_DELAYS if test_delays else 0),
                     lane_bytes,
                     zc_share_pm, 0)
     ctx = P()

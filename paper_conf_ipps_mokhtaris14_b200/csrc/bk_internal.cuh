@@ -58,6 +58,8 @@ __host__ __device__ inline uint64_t mix64(uint64_t x) {
 }
 
 // ---- launchers (kernels_stage.cu) ----
+// test-only: a one-thread kernel that spins `cycles` SM clocks (BK_FLAG_TEST_DELAYS)
+void launch_spin(long long cycles, cudaStream_t s);
 // Stage 1: lane plan + per-tile word counts, then tile bases (exclusive scan of 512*K_w).
 // staged_sum accumulates the staged bytes of every chunk (padding statistics).
 void launch_addrgen(const Chunk& c, const Access& a, const uint64_t* meta, LaneDesc* lanes,

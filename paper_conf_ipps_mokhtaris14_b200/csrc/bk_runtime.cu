@@ -21,6 +21,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "../../include/bk.h"
@@ -156,6 +157,7 @@ struct bk_ctx {
   cudaEvent_t ev_fork = nullptr;
   std::vector<cudaEvent_t> ev_join;
   float* h_mu = nullptr;   // pinned copy of the k-means centroids (graph memcpy source)
+  uint64_t test_rng = 0x9E3779B97F4A7C15ull;   // BK_FLAG_TEST_DELAYS
 };
 
 namespace {
@@ -381,6 +383,17 @@ int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin) {
 }
 #define BK_PROF(stage, stream, begin) do { int r_ = prof_mark(c, stage, stream, begin); if (r_) return r_; } while (0)
 
+// BK_FLAG_TEST_DELAYS: a random spin kernel (0..~100 us) on the stream before every stage, so a
+// missing event dependency between stages shows up as wrong results (SURVEY §4 delay injection).
+uint64_t test_rand(bk_ctx* c) {
+  c->test_rng = c->test_rng * 6364136223846793005ull + 1442695040888963407ull;
+  return c->test_rng >> 33;
+}
+#define BK_DELAY(stream)                                                        \
+  do {                                                                          \
+    if (c->cfg.flags & BK_FLAG_TEST_DELAYS) launch_spin((long long)(test_rand(c) % 200000), stream); \
+  } while (0)
+
 int ensure_host_side(bk_ctx* c, const Plan& p) {
   if (!c->pool) {
     int th = (int)c->cfg.host_threads;
@@ -411,6 +424,8 @@ int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   a.rec_size = c->off ? 0 : c->cfg.record_size;
   const size_t hs = c->h_next++ % c->hstage.size();
   if (c->h_used[hs]) BK_CUDA(cudaEventSynchronize(c->h_done[hs]));   // its previous DMA finished
+  if (c->cfg.flags & BK_FLAG_TEST_DELAYS)   // host-side jitter before the assembly
+    std::this_thread::sleep_for(std::chrono::microseconds(test_rand(c) % 200));
   const auto t0 = std::chrono::steady_clock::now();
   HostData d{c->host, c->off, c->n, c->nbytes, c->cfg.record_size};
   const uint64_t size = host_gather_chunk(*c->pool, d, a, ch, c->hstage[hs], p.stage_cap, c->scratch_first,
@@ -418,7 +433,8 @@ int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   c->st.ms_cpu_gather += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   if (size == UINT64_MAX) return fail(BK_E_RANGE, "host-staged chunk exceeds its slot (internal bound violated)");
   if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
-  BK_PROF(kStH2D, c->s_copy, true);
+  BK_DELAY(c->s_copy);
+    BK_PROF(kStH2D, c->s_copy, true);
   if (c->off && a.whole && ch.hi > ch.lo) {  // record boundaries for whole-record kernels
     BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
     c->st.bytes_meta += (ch.hi - ch.lo) * 8;
@@ -448,6 +464,7 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     // Stage 1 on s_asm (offsets slice by DMA + lane plan) runs ahead, overlapping the previous
     // chunk's zero-copy gather on s_copy; the gather waits only for its own plan.
     if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_asm, s.freed, 0));
+    BK_DELAY(c->s_asm);
     BK_PROF(kStH2D, c->s_asm, true);
     if (c->off && ch.hi > ch.lo) {
       BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_asm));
@@ -459,6 +476,7 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     BK_PROF(kStAddrgen, c->s_asm, false);
     BK_CUDA(cudaEventRecord(s.copied, c->s_asm));
     BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.copied, 0));
+    BK_DELAY(c->s_copy);
     BK_PROF(kStGather, c->s_copy, true);
     Chunk gch = ch;   // readable source: the registered data set
     gch.guard_lo = ch.base_byte;
@@ -470,6 +488,7 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     c->st.bytes_h2d += ch.accessed;
   } else {
     if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+    BK_DELAY(c->s_copy);
     BK_PROF(kStH2D, c->s_copy, true);
     if (c->off && ch.hi > ch.lo) {
       BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
@@ -484,6 +503,7 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     BK_PROF(kStAddrgen, c->s_asm, true);
     launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
     BK_PROF(kStAddrgen, c->s_asm, false);
+    BK_DELAY(c->s_asm);
     BK_PROF(kStGather, c->s_asm, true);
     Chunk gch = ch;   // readable source: the raw slot (256-B aligned, 64 B of slack)
     gch.guard_lo = raw_off;
@@ -551,6 +571,7 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
     if (rc) return rc;
     if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(s.ready);
     BK_CUDA(cudaStreamWaitEvent(cs, s.ready, 0));
+    BK_DELAY(cs);
     BK_PROF(kStCompute, cs, true);
     cudaStream_t rel = cs;   // stream whose completion frees the slot (partition: its D2H)
     rc = compute(chunk_of(c, p, i), s, cs, rel);

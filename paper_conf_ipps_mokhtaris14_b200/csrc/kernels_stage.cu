@@ -350,6 +350,14 @@ __global__ void __launch_bounds__(256) k_gather_bytes(Chunk c, Access a, const u
 
 }  // namespace
 
+__global__ void k_spin(long long cycles) {
+  const long long t0 = clock64();
+  while (clock64() - t0 < cycles) {
+  }
+}
+
+void launch_spin(long long cycles, cudaStream_t s) { k_spin<<<1, 1, 0, s>>>(cycles); }
+
 void launch_addrgen(const Chunk& c, const Access& a, const uint64_t* meta, LaneDesc* lanes, uint32_t* tileK,
                     uint64_t* tile_base, uint64_t stage_cap, int* err, unsigned long long* staged_sum,
                     cudaStream_t s) {

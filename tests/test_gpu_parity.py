@@ -427,3 +427,28 @@ def test_api_errors():
         ctx.register(np.zeros(0, np.uint8), np.zeros(0, np.uint64))
         o, l, c = ctx.wordcount(cap=16)
         assert len(c) == 0
+
+
+# ------------------------------------------------------------------ delay injection
+@pytest.mark.parametrize("mode", ["zc", "dense", "cpu", "hybrid"])
+def test_results_survive_random_stage_delays(mode):
+    """Random spin kernels before every stage on every stream (and host sleeps before CPU
+    assembly) reorder the stages' timing; with a 2-slot ring any missing event dependency
+    (slot reuse before its compute finished, compute before its gather) corrupts results."""
+    buf, off = gen.text(cap_bytes=1 * MIB)
+    want = oracle.wc(buf, off)
+    gb, goff = gen.grep_records(max_bytes=4 * MIB)
+    gwant = oracle.grep(gb, goff, b"bigk")
+    kv = gen.kv(n=200_000)
+    wboff, wout = oracle.partition(kv, 1024)
+    with bk.Context(window_bytes=256 * 1024, n_slots=2, gather_mode=mode, test_delays=True, no_graph=True) as ctx:
+        ctx.register(buf, off)
+        assert wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 17)) == want
+        assert ctx.stats()["n_chunks"] >= 8
+    with bk.Context(window_bytes=256 * 1024, n_slots=2, gather_mode=mode, test_delays=True) as ctx:
+        ctx.register(gb, goff)
+        assert np.array_equal(ctx.grep(b"bigk", cap=len(goff)), gwant)
+    with bk.Context(window_bytes=512 * 1024, n_slots=2, gather_mode=mode, test_delays=True, record_size=16) as ctx:
+        ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=len(kv))
+        out, cc, bc = ctx.partition(1024)
+        assert np.array_equal(global_from_runs(out, cc), wout)
