@@ -242,6 +242,9 @@ def main():
         else:
             dist.init_process_group(backend)
 
+    # ranks on one node share the host cores for CPU assembly (one pool per rank)
+    if not args.host_threads:
+        args.host_threads = max(1, (os.cpu_count() or 1) // int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
     shard = make_shard(args.workload, gib, rank, world)
     peak_h2d = measure_h2d_peak(torch, dev)
     ctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
