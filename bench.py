@@ -329,7 +329,8 @@ def main():
             one_step(pctx)
         pst = pctx.stats()
         pctx.close()
-        for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute", "n_gather", "ms_cpu_gather"):
+        for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute", "n_gather", "ms_cpu_gather", "ms_xfer_busy",
+                  "ms_compute_busy", "ms_overlap"):
             st[k] = pst[k]
         st["profiled_ms_device"] = pst["ms_device"]
     total_bytes = nbytes * world * args.steps
@@ -372,6 +373,16 @@ def main():
         "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6650 GB/s")
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["traffic"] = None
+    if roof["kernel"].startswith("k_gather_field") and args.workload == "grep":
+        # the zero-copy key gather is PCIe read-request bound, not byte bound: one read request per
+        # 128-B line a 32-B key touches (8-aligned keys: 1 + 3/16 = 1.1875 requests per record).
+        # Peak = the request rate the phase-0 probe measured for one field per 256-B record
+        # (profiles/r01_box_probe.txt: zc_sparse rec 256 -> 0.562 G records/s, one request each).
+        recs_per_launch = shard["n"] / st["n_chunks"]
+        req_rate = recs_per_launch * 1.1875 / (avg_ms * 1e-3)
+        roof["request_rate"] = {"bound": "pcie_read_requests", "achieved": req_rate / 1e9, "peak": 0.562,
+                                "unit": "G requests/s", "frac": req_rate / 0.562e9,
+                                "peak_source": "profiles/r01_box_probe.txt zc_sparse (256-B stride, 1 request/record)"}
     roof["avg_launch_ms"] = avg_ms
     roof["launches_per_step"] = launches
 
@@ -396,6 +407,15 @@ def main():
                                "profiled_ms_device": round(st.get("profiled_ms_device", 0.0), 3),
                                "note": "per-stage busy sums from a profiled eager pass (CUDA events per stage "
                                        "per chunk); ms_device from the timed (graph-replayed when static) pass"},
+        "overlap": {"xfer_busy_ms": round(st.get("ms_xfer_busy", 0.0), 3),
+                    "compute_busy_ms": round(st.get("ms_compute_busy", 0.0), 3),
+                    "overlap_ms": round(st.get("ms_overlap", 0.0), 3),
+                    "overlap_frac": round(st.get("ms_overlap", 0.0) / max(min(st.get("ms_xfer_busy", 0.0),
+                                                                              st.get("ms_compute_busy", 0.0)), 1e-9), 4),
+                    "link_busy_frac": round(st.get("ms_xfer_busy", 0.0) / max(st.get("profiled_ms_device", 0.0), 1e-9), 4),
+                    "how": "unions of per-chunk CUDA-event intervals of the transfer stages (DMA copies, zero-copy "
+                           "gathers) and of the compute kernels, profiled pass; overlap_frac = |xfer n compute| / "
+                           "min(xfer, compute); link_busy_frac = xfer union / device time"},
         "e2e": {"value": round(total_bytes / t_wall / 1e9, 3), "unit": "GB/s",
                 "h2d_bytes_per_step": (st["bytes_h2d"] + st["bytes_meta"]) * world,
                 "d2h_bytes_per_step": st["bytes_d2h"] * world,

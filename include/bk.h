@@ -251,6 +251,9 @@ typedef struct bk_stats {
   uint64_t n_gather;          /*   number of gather launches timed */
   uint64_t n_chunks_cpu;      /* chunks assembled by the host pool (CPU / HYBRID) */
   double ms_cpu_gather;       /* host time spent assembling them */
+  double ms_xfer_busy;        /* BK_FLAG_PROFILE: union of the transfer intervals (DMA copies, zero-copy gathers) */
+  double ms_compute_busy;     /*   union of the compute-kernel intervals */
+  double ms_overlap;          /*   length of their intersection (copy/compute overlap) */
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);

@@ -75,7 +75,8 @@ class bk_stats(C.Structure):
                 ("bytes_meta", u64), ("bytes_padding", u64), ("bytes_d2h", u64), ("kernel_launches", u64),
                 ("ms_run", C.c_double), ("ms_register", C.c_double), ("ms_device", C.c_double),
                 ("ms_h2d", C.c_double), ("ms_addrgen", C.c_double), ("ms_gather", C.c_double),
-                ("ms_compute", C.c_double), ("n_gather", u64), ("n_chunks_cpu", u64), ("ms_cpu_gather", C.c_double)]
+                ("ms_compute", C.c_double), ("n_gather", u64), ("n_chunks_cpu", u64), ("ms_cpu_gather", C.c_double),
+                ("ms_xfer_busy", C.c_double), ("ms_compute_busy", C.c_double), ("ms_overlap", C.c_double)]
 
 
 class bk_out_pattern(C.Structure):

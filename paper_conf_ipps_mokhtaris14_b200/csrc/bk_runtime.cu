@@ -361,7 +361,8 @@ Chunk chunk_of(const bk_ctx* c, const Plan& p, size_t i) {
 }
 
 // BK_FLAG_PROFILE: bracket one stage of one chunk with timing events on its stream.
-enum { kStH2D = 0, kStAddrgen = 1, kStGather = 2, kStCompute = 3, kNStages = 4 };
+// stage ids of the profiling events: transfer = {H2D, Gather (zero-copy)}, compute = {Compute}
+enum { kStH2D = 0, kStAddrgen = 1, kStGather = 2, kStCompute = 3, kStRelayout = 4, kNStages = 5 };
 int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin) {
   if (!(c->cfg.flags & BK_FLAG_PROFILE)) return BK_OK;
   if (begin) {
@@ -504,12 +505,12 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
     BK_PROF(kStAddrgen, c->s_asm, false);
     BK_DELAY(c->s_asm);
-    BK_PROF(kStGather, c->s_asm, true);
+    BK_PROF(kStRelayout, c->s_asm, true);
     Chunk gch = ch;   // readable source: the raw slot (256-B aligned, 64 B of slack)
     gch.guard_lo = raw_off;
     gch.guard_hi = p.raw_cap - raw_off;
     launch_gather(gch, a, s.raw + raw_off, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 0, c->s_asm);
-    BK_PROF(kStGather, c->s_asm, false);
+    BK_PROF(kStRelayout, c->s_asm, false);
     c->n_launch += 3;
     c->st.bytes_h2d += bytes;
   }
@@ -619,6 +620,52 @@ int begin_run(bk_ctx* c, void* stream) {
   return BK_OK;
 }
 
+// Per-stage busy sums and, from the interval of every (stage, chunk) event pair relative to the
+// run start, the union of transfer intervals, the union of compute intervals and their overlap
+// (the north_star's copy/compute overlap, measured with CUDA events instead of nsys).
+int stage_stats(bk_ctx* c) {
+  double acc[kNStages] = {0, 0, 0, 0, 0};
+  uint64_t cnt[kNStages] = {0, 0, 0, 0, 0};
+  std::vector<std::pair<double, double>> xfer, comp;
+  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
+    float e = 0, b0 = 0;
+    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
+    BK_CUDA(cudaEventElapsedTime(&b0, c->t_begin, c->prof[i]));
+    const int stg = c->prof_stage[i / 2];
+    acc[stg] += e;
+    cnt[stg] += 1;
+    if (stg == kStH2D || stg == kStGather) xfer.emplace_back(b0, b0 + e);
+    if (stg == kStCompute) comp.emplace_back(b0, b0 + e);
+  }
+  auto merge = [](std::vector<std::pair<double, double>> v) {
+    std::sort(v.begin(), v.end());
+    std::vector<std::pair<double, double>> u;
+    for (auto& x : v) {
+      if (!u.empty() && x.first <= u.back().second) u.back().second = std::max(u.back().second, x.second);
+      else u.push_back(x);
+    }
+    return u;
+  };
+  const auto ux = merge(xfer), uc = merge(comp);
+  double bx = 0, bc = 0, ov = 0;
+  for (auto& x : ux) bx += x.second - x.first;
+  for (auto& x : uc) bc += x.second - x.first;
+  for (size_t i = 0, j = 0; i < ux.size() && j < uc.size();) {  // intersection of two sorted unions
+    const double lo = std::max(ux[i].first, uc[j].first), hi = std::min(ux[i].second, uc[j].second);
+    if (hi > lo) ov += hi - lo;
+    if (ux[i].second < uc[j].second) ++i; else ++j;
+  }
+  c->st.ms_h2d = acc[kStH2D];
+  c->st.ms_addrgen = acc[kStAddrgen];
+  c->st.ms_gather = acc[kStGather] + acc[kStRelayout];
+  c->st.ms_compute = acc[kStCompute];
+  c->st.n_gather = cnt[kStGather] + cnt[kStRelayout];
+  c->st.ms_xfer_busy = bx;
+  c->st.ms_compute_busy = bc;
+  c->st.ms_overlap = ov;
+  return BK_OK;
+}
+
 int end_run(bk_ctx* c, void* stream) {
   BK_CUDA(cudaEventRecord(c->t_end, c->s_comp));
   BK_CUDA(cudaEventRecord(c->ev_end, c->s_comp));
@@ -630,19 +677,8 @@ int end_run(bk_ctx* c, void* stream) {
   float ms = 0;
   BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
   c->st.ms_device = ms;
-  double acc[kNStages] = {0, 0, 0, 0};
-  uint64_t cnt[kNStages] = {0, 0, 0, 0};
-  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
-    float e = 0;
-    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
-    acc[c->prof_stage[i / 2]] += e;
-    cnt[c->prof_stage[i / 2]] += 1;
-  }
-  c->st.ms_h2d = acc[kStH2D];
-  c->st.ms_addrgen = acc[kStAddrgen];
-  c->st.ms_gather = acc[kStGather];
-  c->st.ms_compute = acc[kStCompute];
-  c->st.n_gather = cnt[kStGather];
+  int rc = stage_stats(c);
+  if (rc) return rc;
   return check_err(c);
 }
 
@@ -701,19 +737,8 @@ int end_host(bk_ctx* c, void* stream) {
   float ms = 0;
   BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
   c->st.ms_device = ms;
-  double acc[kNStages] = {0, 0, 0, 0};
-  uint64_t cnt[kNStages] = {0, 0, 0, 0};
-  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
-    float e = 0;
-    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
-    acc[c->prof_stage[i / 2]] += e;
-    cnt[c->prof_stage[i / 2]] += 1;
-  }
-  c->st.ms_h2d = acc[kStH2D];
-  c->st.ms_addrgen = acc[kStAddrgen];
-  c->st.ms_gather = acc[kStGather];
-  c->st.ms_compute = acc[kStCompute];
-  c->st.n_gather = cnt[kStGather];
+  int rc = stage_stats(c);
+  if (rc) return rc;
   return check_err(c);
 }
 
