@@ -172,6 +172,29 @@ def measure_h2d_peak(torch, dev) -> float:
     return best
 
 
+def measure_bidir_peak(torch, dev) -> float:
+    """Each-direction GB/s with H2D and D2H of 1 GiB running at once (partition's full-duplex roof)."""
+    h_in = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
+    h_out = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
+    d_in = torch.empty(GIB, dtype=torch.uint8, device=dev)
+    d_out = torch.empty(GIB, dtype=torch.uint8, device=dev)
+    s1, s2 = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+    best = 0.0
+    for _ in range(3):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with torch.cuda.stream(s1):
+            for o in range(0, GIB, 256 * MIB):
+                d_in[o:o + 256 * MIB].copy_(h_in[o:o + 256 * MIB], non_blocking=True)
+        with torch.cuda.stream(s2):
+            for o in range(0, GIB, 256 * MIB):
+                h_out[o:o + 256 * MIB].copy_(d_out[o:o + 256 * MIB], non_blocking=True)
+        torch.cuda.synchronize()
+        best = max(best, GIB / (time.perf_counter() - t0) / 1e9)
+    del h_in, h_out, d_in, d_out
+    return best
+
+
 def load_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -247,6 +270,7 @@ def main():
         args.host_threads = max(1, (os.cpu_count() or 1) // int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
     shard = make_shard(args.workload, gib, rank, world)
     peak_h2d = measure_h2d_peak(torch, dev)
+    peak_bidir = measure_bidir_peak(torch, dev) if args.workload == "partition" else None
     ctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
                      baseline_dbuf=args.impl == "dbuf", baseline_sbuf=args.impl == "sbuf",
                      host_threads=args.host_threads, lane_bytes=args.lane_bytes, zc_share_pm=args.zc_share,
@@ -398,6 +422,10 @@ def main():
                    "l2": "inputs (>=64 MiB per GPU, host-resident) exceed the 126 MB L2; streamed from host each step",
                    "parallelism": f"dp{world} (contiguous record shards, one PCIe link per GPU)"},
         "records_per_s": total_recs / t_dev,
+        "link_full_duplex": None if peak_bidir is None else {
+            "peak_each_way_gbs": round(peak_bidir, 3), "achieved_each_way_gbs": round(link_gbs, 3),
+            "frac": round(link_gbs / (peak_bidir * world), 4),
+            "note": "partition streams n x 16 B in and the bucket-sorted n x 16 B back out concurrently"},
         "link": {"algorithmic_gbs": round(link_gbs, 3), "peak_h2d_gbs_per_gpu": round(peak_h2d, 3),
                  "frac": round(link_gbs / (peak_h2d * world), 4),
                  "bytes_per_step_per_gpu": st["bytes_h2d"] + st["bytes_meta"],
