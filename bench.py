@@ -51,7 +51,7 @@ def parse():
                     help="ours | reference (CPU oracle) | dbuf / sbuf (the paper's GPU double / single "
                          "buffering variants, for ablations)")
     ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "groupby_sparse", "kmeans",
-                                                             "partition"])
+                                                             "partition", "kmer"])
     ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense", "cpu", "hybrid"])
     ap.add_argument("--gib", type=float, default=None, help="per-GPU data size override (GiB)")
     ap.add_argument("--window-mib", type=int, default=None)
@@ -77,6 +77,8 @@ WORKLOADS = {
     "groupby_sparse": (16.0, 2048, "C5 sparse variant: the same 16 B inside 64-B records (25% read, like Table I "
                                    "MCA-indexed P:929)"),
     "kmeans": (16.0, 2048, "C3 k-means step: 16-dim fp32 points, K=64, Forgy init"),
+    "kmer": (4.0, 2048, "f4 k-mer counting (k=31) over 256-B DNA read records, 96-base sequence at +16 (37.5% "
+                        "read, Table I DNA: 36%), reads of a seeded 2^25-base genome, 0.05% substitutions, 0.2% N"),
     "partition": (8.0, 2048, "C4 stable hash partition: {u64 key, u64 value} 16-B records into 1024 buckets, "
                              "bucket-sorted chunks written back to host (full duplex)"),
 }
@@ -101,6 +103,10 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
         buf = gen.groupby(gen.SEED_GROUPBY, first=rank * n, n=n, stride=stride,
                           out=gen.alloc(n * stride, huge=HUGE) if HUGE is not None else None)
         return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=stride)
+    if workload == "kmer":
+        n = nbytes // 256
+        buf = gen.dna(gen.SEED_DNA, first=rank * n, n=n, genome_len=1 << 25, err_pm=0, n_pm=2)
+        return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=256)
     if workload == "partition":
         n = nbytes // 16
         kv = gen.kv(gen.SEED_KV, first=rank * n, n=n)
@@ -220,6 +226,9 @@ def oracle_sample(workload: str, shard: dict, target_s: float):
         elif workload in ("groupby", "groupby_sparse"):
             end = nrec * shard["rec_size"]
             oracle.groupby(buf[:end], nrec, shard["rec_size"], 4096)
+        elif workload == "kmer":
+            end = nrec * 256
+            oracle.kmer(buf[:end], nrec, 31)
         elif workload == "partition":
             end = nrec * 16
             oracle.partition(buf[:end].view(np.uint64).reshape(-1, 2), 1024)
@@ -281,6 +290,10 @@ def main():
     stream = torch.cuda.current_stream()
     nbytes = len(shard["buf"])
 
+    kmer_out = (np.empty(1 << 27, np.uint64), np.empty(1 << 27, np.uint64)) if args.workload == "kmer" else None
+    if kmer_out is not None:   # touch once: the result D2H must not pay first-touch page faults per step
+        kmer_out[0].fill(0)
+        kmer_out[1].fill(0)
     cap = max(shard["n"] // 50, 1 << 16)
     idx_out = np.empty(cap, np.uint64)
 
@@ -298,6 +311,10 @@ def main():
                 b = shard["buf"]
                 return merge.merge_wordcount({b[int(x): int(x) + int(y)].tobytes(): int(z) for x, y, z in zip(o, l, c)})
             return int(c.sum())
+        if args.workload == "kmer":
+            km, ct, total = ctx.kmer(k=31, table_slots=1 << 28, stream=cs, out=kmer_out)
+            t = torch.tensor([total, len(km)], dtype=torch.int64, device=dev)
+            return merge.merge_sum(t) if world > 1 else t
         if args.workload == "partition":
             out, cc, bc = ctx.partition(1024, out=shard["out"], stream=cs)
             return merge.merge_partition_offsets(bc) if world > 1 else bc

@@ -21,6 +21,7 @@ SEED_GREP = 0xB16C0002
 SEED_KMEANS = 0xB16C0003
 SEED_KV = 0xB16C0004
 SEED_GROUPBY = 0xB16C0005
+SEED_DNA = 0xB16C0006
 
 _lib = None
 
@@ -52,6 +53,8 @@ def lib():
         l.gen_kv.argtypes = [u64, u64, u64, p, C.c_int]
         l.gen_groupby.restype = None
         l.gen_groupby.argtypes = [u64, u64, u64, C.c_uint32, C.c_uint32, C.c_int, p, C.c_int]
+        l.gen_dna.restype = None
+        l.gen_dna.argtypes = [u64, u64, u64, u64, C.c_uint32, C.c_uint32, p, C.c_int]
         l.gen_alloc.restype = p
         l.gen_alloc.argtypes = [u64, C.c_int, C.POINTER(p), C.POINTER(u64)]
         l.gen_free.restype = None
@@ -67,6 +70,14 @@ def _threads(threads):
 def _ptr(a: np.ndarray) -> int:
     assert a.flags["C_CONTIGUOUS"]
     return a.ctypes.data
+
+
+def dna(seed: int = SEED_DNA, first: int = 0, n: int = 1 << 16, genome_len: int = 1 << 20, err_pm: int = 1,
+        n_pm: int = 2, out: np.ndarray | None = None, threads: int = 0):
+    """f4: n x 256-B read records (96-base sequence at +16) sampled from a seeded genome."""
+    buf = out if out is not None else np.empty(n * 256, np.uint8)
+    lib().gen_dna(seed, first, n, genome_len, err_pm, n_pm, _ptr(buf), _threads(threads))
+    return buf
 
 
 class _Mapping:

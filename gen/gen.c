@@ -192,3 +192,36 @@ void* gen_alloc(uint64_t bytes, int huge, void** base_out, uint64_t* len_out) {
 }
 
 void gen_free(void* base, uint64_t len) { munmap(base, len); }
+
+/* ---------------- f4: DNA reads (Table I DNA assembly: fixed-length fragments, 36% read) ----------------
+ * Record (256 B): [u64 id][u32 genome_pos][u32 flags][char seq[96] ACGT/N][char qual[144]].
+ * A seeded random genome of genome_len bases; read i = the 96 bases at a random position with
+ * substitution errors (err_pm per mille) and 'N' calls (n_pm per mille). */
+static inline uint8_t genome_base(uint64_t seed, uint64_t p) {
+  return (uint8_t)("ACGT"[(gen_R(seed, 20, p >> 5) >> (2 * (p & 31))) & 3]);
+}
+
+void gen_dna(uint64_t seed, uint64_t first, uint64_t n, uint64_t genome_len, uint32_t err_pm, uint32_t n_pm,
+             uint8_t* buf, int threads) {
+#pragma omp parallel for schedule(static) num_threads(threads > 0 ? threads : 1)
+  for (uint64_t k = 0; k < n; ++k) {
+    const uint64_t i = first + k;
+    uint8_t* r = buf + k * 256;
+    const uint64_t pos = gen_R(seed, 21, i) % (genome_len - 96);
+    const uint32_t pos32 = (uint32_t)pos, flags = 0;
+    memcpy(r, &i, 8);
+    memcpy(r + 8, &pos32, 4);
+    memcpy(r + 12, &flags, 4);
+    for (int j = 0; j < 96; ++j) {
+      uint8_t b = genome_base(seed, pos + j);
+      const uint64_t e = gen_R(seed, 22, i * 96 + j) % 1000;
+      if (e < n_pm) b = 'N';
+      else if (e < n_pm + err_pm) b = (uint8_t)("ACGT"[gen_R(seed, 23, i * 96 + j) & 3]);
+      r[16 + j] = b;
+    }
+    for (int j = 112; j < 256; j += 8) {
+      uint64_t q = gen_R(seed, 24, i * 32 + j / 8);
+      for (int t = 0; t < 8; ++t) { r[j + t] = (uint8_t)(33 + (q & 0xff) % 42); q >>= 8; }
+    }
+  }
+}

@@ -47,6 +47,11 @@ void gen_kv(uint64_t seed, uint64_t first, uint64_t n, uint64_t* kv, int threads
 void gen_groupby(uint64_t seed, uint64_t first, uint64_t n, uint32_t G, uint32_t stride, int zipf,
                  uint8_t* buf, int threads);
 
+/* f4 — DNA reads: 256-B records, 96-base sequence at +16 (ACGT, 'N' calls), sampled from a seeded
+ * genome of genome_len bases with err_pm / n_pm per-mille substitution / N rates. */
+void gen_dna(uint64_t seed, uint64_t first, uint64_t n, uint64_t genome_len, uint32_t err_pm, uint32_t n_pm,
+             uint8_t* buf, int threads);
+
 /* 2 MiB-aligned anonymous mapping for large data sets; huge != 0 asks for transparent huge pages
  * (madvise). Free with gen_free(base, len). */
 void* gen_alloc(uint64_t bytes, int huge, void** base_out, uint64_t* len_out);

@@ -48,6 +48,7 @@ typedef enum {
   BK_K_KMEANS = 3,      /* C3: assignment + per-cluster partial sums      bk_out_kmeans */
   BK_K_PARTITION = 4,   /* C4: stable hash partition into B buckets                    bk_out_partition */
   BK_K_GROUPBY = 5,     /* C5: group-by count / sum                                    bk_out_groupby */
+  BK_K_KMER = 6,        /* f4: k-mer counting over fixed-length DNA reads           bk_out_kmer */
   BK_K_LAYOUT_DUMP = 100, /* test only: copy one chunk's staged bytes + lane table back      bk_out_layout */
   BK_K_PATTERN_STATS = 101 /* stage 1 in address mode + online pattern recognition over
                               every lane's element-address stream; Table II accounting     bk_out_pattern */
@@ -204,6 +205,20 @@ typedef struct bk_out_layout {
   uint32_t _pad;
   uint64_t chunk_lo, chunk_hi, n_chunks; /* out */
 } bk_out_layout;
+
+typedef struct bk_out_kmer {
+  bk_out_header h;
+  uint32_t k;               /* in: 1..31 */
+  uint32_t seq_off;         /* in: sequence field offset in every record */
+  uint32_t seq_len;         /* in: sequence field length, a multiple of 16 */
+  uint32_t _pad;
+  uint64_t table_slots;     /* in: device table slots (power of two); 0 = 2^24 */
+  uint64_t cap;             /* in: capacity of kmer / count */
+  uint64_t* kmer;           /* out: distinct k-mers, 2-bit packed (A=0 C=1 G=2 T=3), unordered */
+  uint64_t* count;          /* out */
+  uint64_t n_kmers;         /* out: distinct (> cap -> BK_E_CAPACITY) */
+  uint64_t total;           /* out: k-mer occurrences */
+} bk_out_kmer;
 
 typedef struct bk_out_pattern {
   bk_out_header h;

@@ -46,6 +46,8 @@ def lib():
         l.oracle_layout.argtypes = [p, p, u64, u64, u64, u32, p, p, u64, u64, u32, p, p, p, p, u64]
         l.oracle_pattern.restype = C.c_int
         l.oracle_pattern.argtypes = [p, u32, u32, p]
+        l.oracle_kmer.restype = i64
+        l.oracle_kmer.argtypes = [p, u64, u32, u32, u32, u32, p, p, u64]
         l.oracle_pattern_online.restype = C.c_int
         l.oracle_pattern_online.argtypes = [p, u64, u32, u32, p]
         _lib = l
@@ -126,6 +128,18 @@ def groupby(recs, n: int, stride: int = 16, G: int = 4096):
     if rc:
         raise ValueError("key >= G")
     return count, qty, amt
+
+
+def kmer(recs, n: int, k: int = 31, rec_size: int = 256, seq_off: int = 16, seq_len: int = 96):
+    """O6: (kmers u64 ascending, counts u64)."""
+    r = _u8(recs)
+    cap = 1 << 16
+    while True:
+        km = np.empty(cap, np.uint64); ct = np.empty(cap, np.uint64)
+        V = lib().oracle_kmer(_p(r) if len(r) else None, n, rec_size, seq_off, seq_len, k, _p(km), _p(ct), cap)
+        if V >= 0:
+            return km[:V].copy(), ct[:V].copy()
+        cap = -V
 
 
 def _ext(extents):

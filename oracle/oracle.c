@@ -160,6 +160,46 @@ int oracle_groupby(const uint8_t* recs, uint64_t n, uint32_t stride, uint32_t G,
   return 0;
 }
 
+/* ------------------------------------------------------------------ O6 k-mers */
+static int cmp_u64(const void* a, const void* b) {
+  const uint64_t x = *(const uint64_t*)a, y = *(const uint64_t*)b;
+  return x < y ? -1 : x > y;
+}
+
+int64_t oracle_kmer(const uint8_t* recs, uint64_t n, uint32_t rec_size, uint32_t seq_off, uint32_t seq_len,
+                    uint32_t k, uint64_t* kmer, uint64_t* count, uint64_t cap) {
+  /* 1. every k-mer occurrence, record by record, window by window */
+  uint64_t cap_occ = 1024, m = 0;
+  uint64_t* occ = (uint64_t*)malloc(cap_occ * 8);
+  for (uint64_t r = 0; r < n; ++r) {
+    const uint8_t* s = recs + r * rec_size + seq_off;
+    for (uint32_t j = 0; j + k <= seq_len; ++j) {
+      uint64_t v = 0;
+      int ok = 1;
+      for (uint32_t q = 0; q < k && ok; ++q) {
+        int code = s[j + q] == 'A' ? 0 : s[j + q] == 'C' ? 1 : s[j + q] == 'G' ? 2 : s[j + q] == 'T' ? 3 : -1;
+        if (code < 0) ok = 0;
+        else v = v * 4 + (uint64_t)code;
+      }
+      if (!ok) continue;
+      if (m == cap_occ) { cap_occ *= 2; occ = (uint64_t*)realloc(occ, cap_occ * 8); }
+      occ[m++] = v;
+    }
+  }
+  /* 2. sort, 3. count runs */
+  qsort(occ, m, 8, cmp_u64);
+  int64_t V = 0;
+  for (uint64_t i = 0; i < m;) {
+    uint64_t j = i + 1;
+    while (j < m && occ[j] == occ[i]) ++j;
+    if ((uint64_t)V < cap) { kmer[V] = occ[i]; count[V] = j - i; }
+    ++V;
+    i = j;
+  }
+  free(occ);
+  return (uint64_t)V > cap ? -V : V;
+}
+
 /* ------------------------------------------------------------------ O-L layout */
 /* accessed bytes of record r under the access spec */
 static int64_t rec_access(const uint64_t* off, uint64_t n, uint64_t nbytes, uint64_t rec_size,

@@ -55,6 +55,14 @@ int oracle_partition(const uint64_t* kv, uint64_t n, uint32_t B, uint64_t* boff,
 int oracle_groupby(const uint8_t* recs, uint64_t n, uint32_t stride, uint32_t G,
                    uint64_t* count, uint64_t* qty, double* amount);
 
+/* O6 k-mer counting (NEXT f4; DNA assembly's k-mer table, Table I): for every
+ * record the sequence field rec[seq_off .. seq_off+seq_len), every window of k consecutive bases
+ * in {A,C,G,T} (a base outside the set breaks windows) is the 2-bit value sum code(b_j) 4^(k-1-j),
+ * A=0 C=1 G=2 T=3. Writes the distinct k-mers ascending with their counts; returns V or -V if
+ * V > cap. 1 <= k <= 31. */
+int64_t oracle_kmer(const uint8_t* recs, uint64_t n, uint32_t rec_size, uint32_t seq_off, uint32_t seq_len,
+                    uint32_t k, uint64_t* kmer, uint64_t* count, uint64_t cap);
+
 /* ---- O-L: staged layout (stage 1 address generation + stage 2 assembly) ----
  * Access spec: n_ext == 0 means the WHOLE record; else n_ext extents (ext_off[e], ext_len[e])
  * relative to the record start, all inside every record (the addresses the

@@ -87,9 +87,15 @@ class bk_out_pattern(C.Structure):
                 ("address_bytes", u64), ("pattern_bytes", u64)]
 
 
+class bk_out_kmer(C.Structure):
+    _fields_ = [("h", bk_out_header), ("k", u32), ("seq_off", u32), ("seq_len", u32), ("_pad", u32),
+                ("table_slots", u64), ("cap", u64), ("kmer", P), ("count", P), ("n_kmers", u64), ("total", u64)]
+
+
 BK_K_PATTERN_STATS = 101
+BK_K_KMER = 6
 ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,
-               bk_out_layout, bk_stats, bk_out_pattern]
+               bk_out_layout, bk_stats, bk_out_pattern, bk_out_kmer]
 EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_destroy", "bk_strerror", "bk_last_error",
            "bk_get_stats", "bk_abi_sizes"]
 
@@ -278,6 +284,21 @@ class Context:
         bk_run(self.ctx, BK_K_PARTITION, stream, o)
         C = o.n_chunks
         return out, cc[: C * n_buckets].reshape(C, n_buckets), bc
+
+    def kmer(self, k: int = 31, seq_off: int = 16, seq_len: int = 96, table_slots: int = 0, cap: int = 1 << 22,
+             stream=None, out=None):
+        """f4: (kmers u64, counts u64) unordered, and the total number of k-mer occurrences.
+        out: optional preallocated (kmers, counts) arrays of equal length (the capacity)."""
+        o = _hdr(bk_out_kmer, BK_K_KMER)
+        if out is not None:
+            km, ct = out
+            cap = min(len(km), len(ct))
+        else:
+            km = np.empty(cap, np.uint64); ct = np.empty(cap, np.uint64)
+        o.k, o.seq_off, o.seq_len, o.table_slots, o.cap, o.kmer, o.count = k, seq_off, seq_len, table_slots, cap, \
+            _ptr(km), _ptr(ct)
+        bk_run(self.ctx, BK_K_KMER, stream, o)
+        return km[: o.n_kmers], ct[: o.n_kmers], int(o.total)
 
     def pattern_stats(self, extents=None, elem_bytes: int = 1, T: int = 8, pmax: int = 4, chunk: int | None = None,
                       lane_cap: int = 1 << 20, stream=None):

@@ -125,6 +125,17 @@ void launch_dbuf_groupby(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t 
                          cudaStream_t s);
 cudaError_t configure_baseline_kernels();
 
+// ---- f4: k-mer counting over DNA reads (kernels_kmer.cu) ----
+struct KmerEntry {            // 16 B exact-key slot
+  unsigned long long key;     // k-mer + 1 (0 = empty)
+  unsigned long long count;
+};
+void launch_kmer(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base, uint32_t k,
+                 uint32_t seq_words, KmerEntry* table, uint64_t mask, unsigned long long* used,
+                 unsigned long long* total, int* err, cudaStream_t s);
+void launch_kmer_compact(const KmerEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* kmer,
+                         uint64_t* cnt, uint64_t cap, cudaStream_t s);
+
 // ---- online pattern recognition of stage 1 (kernels_pattern.cu, NEXT f2) ----
 void launch_addr_patterns(const Chunk& c, const Access& a, const uint64_t* meta, const LaneDesc* lanes, uint32_t elem,
                           uint32_t T, uint32_t pmax, int32_t* lane_p, int64_t* lane_strides, uint64_t* lane_base,

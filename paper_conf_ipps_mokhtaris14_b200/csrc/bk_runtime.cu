@@ -148,8 +148,7 @@ struct bk_ctx {
   cudaStream_t s_d2h = nullptr;
   std::vector<cudaEvent_t> ev_part;
   DevBuf b_hist, b_colpre, b_totals, b_base;
-  void* out_pinned = nullptr;
-  uint64_t out_pinned_bytes = 0;
+  std::vector<std::pair<void*, uint64_t>> out_pinned;  // caller output arrays this context pinned
   int n_launch = 0;
   bk_stats st{};
   std::vector<std::pair<std::string, Plan>> plan_cache;
@@ -935,15 +934,16 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
 // The caller's per-record output (partition records, k-means cid) is written by DMA: pin it once
 // and keep it pinned across runs (one cached registration per context).
 int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes) {
-  if (!bytes || (c->out_pinned == ptr && c->out_pinned_bytes == bytes)) return BK_OK;
-  if (c->out_pinned) cudaHostUnregister(c->out_pinned);
-  c->out_pinned = nullptr;
-  c->out_pinned_bytes = 0;
-  if (!is_pinned(ptr)) {
-    BK_CUDA(cudaHostRegister(ptr, bytes, cudaHostRegisterPortable));
-    c->out_pinned = ptr;
-    c->out_pinned_bytes = bytes;
+  if (!bytes) return BK_OK;
+  for (auto& e : c->out_pinned)
+    if (e.first == ptr && e.second == bytes) return BK_OK;
+  if (is_pinned(ptr)) return BK_OK;
+  if (c->out_pinned.size() >= 4) {  // keep at most four cached registrations (oldest out)
+    cudaHostUnregister(c->out_pinned.front().first);
+    c->out_pinned.erase(c->out_pinned.begin());
   }
+  BK_CUDA(cudaHostRegister(ptr, bytes, cudaHostRegisterPortable));
+  c->out_pinned.emplace_back(ptr, bytes);
   return BK_OK;
 }
 
@@ -998,6 +998,56 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(cudaMemcpy(&chk, c->d_ctr + 4, 8, cudaMemcpyDeviceToHost));
   o->chk = chk;
   c->st.bytes_d2h += (uint64_t)K * 136;
+  return BK_OK;
+}
+
+// f4: k-mer counting (FIELD access to the sequence; the table is resident, outside the window)
+int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
+  const uint64_t slots = o->table_slots ? o->table_slots : (1ull << 24);
+  if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
+  if (o->k < 1 || o->k > 31) return fail(BK_E_INVAL, "k must be in 1..31");
+  if (o->seq_len == 0 || o->seq_len % 16) return fail(BK_E_INVAL, "seq_len must be a positive multiple of 16");
+  if ((uint64_t)o->seq_off + o->seq_len > c->min_rec) return fail(BK_E_INVAL, "sequence field exceeds a record");
+  Plan p;
+  int rc = plan_run(c, field_access(o->seq_off, o->seq_len), 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  BK_CUDA(c->b_table.ensure(slots * sizeof(KmerEntry)));
+  const uint64_t ocap = std::min<uint64_t>(o->cap, slots);
+  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  KmerEntry* table = (KmerEntry*)c->b_table.p;
+  const std::string key = "kmer/" + std::to_string(o->k) + "/" + std::to_string(slots) + "/" + std::to_string(ocap) +
+                          "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(KmerEntry), c->s_comp));
+    int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_kmer(ch, s.stage, s.lanes, s.tile_base, o->k, o->seq_len / 16, table, slots - 1, c->d_ctr + 1,
+                  c->d_ctr + 5, c->d_err, cs);
+      c->n_launch += 1;
+      return BK_OK;
+    });
+    if (r) return r;
+    launch_kmer_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint64_t*)c->b_out3.p, ocap, c->s_comp);
+    c->n_launch += 1;
+    return (int)BK_OK;
+  });
+  if (rc) return rc;
+  unsigned long long nk = 0, tot = 0;
+  BK_CUDA(cudaMemcpy(&nk, c->d_ctr + 2, 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(&tot, c->d_ctr + 5, 8, cudaMemcpyDeviceToHost));
+  o->n_kmers = nk;
+  o->total = tot;
+  if (nk > o->cap) return fail(BK_E_CAPACITY, "%llu distinct k-mers > cap %llu", nk, (unsigned long long)o->cap);
+  if (nk * 10 > slots * 7) return fail(BK_E_CAPACITY, "k-mer table load %llu/%llu too high; raise table_slots", nk,
+                                       (unsigned long long)slots);
+  if (nk) {
+    // the result arrays are large (16 B per distinct k-mer): pin them once so the copy runs at DMA speed
+    if ((rc = ensure_out_pinned(c, o->kmer, o->cap * 8)) || (rc = ensure_out_pinned(c, o->count, o->cap * 8))) return rc;
+    BK_CUDA(cudaMemcpy(o->kmer, c->b_out1.p, nk * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->count, c->b_out3.p, nk * 8, cudaMemcpyDeviceToHost));
+  }
+  c->st.bytes_d2h = nk * 16;
   return BK_OK;
 }
 
@@ -1468,6 +1518,10 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
       if (h->struct_size != sizeof(bk_out_groupby)) return fail(BK_E_INVAL, "bk_out_groupby size");
       rc = run_groupby(c, (bk_out_groupby*)out, stream);
       break;
+    case BK_K_KMER:
+      if (h->struct_size != sizeof(bk_out_kmer)) return fail(BK_E_INVAL, "bk_out_kmer size");
+      rc = run_kmer(c, (bk_out_kmer*)out, stream);
+      break;
     case BK_K_PATTERN_STATS:
       if (h->struct_size != sizeof(bk_out_pattern)) return fail(BK_E_INVAL, "bk_out_pattern size");
       rc = run_pattern(c, (bk_out_pattern*)out, stream);
@@ -1505,10 +1559,11 @@ int bk_get_stats(const bk_ctx* c, bk_stats* s) {
 }
 
 int bk_abi_sizes(uint32_t* sizes, int n) {
-  const uint32_t v[9] = {sizeof(bk_config),        sizeof(bk_out_wordcount), sizeof(bk_out_grep),
-                         sizeof(bk_out_kmeans),    sizeof(bk_out_partition), sizeof(bk_out_groupby),
-                         sizeof(bk_out_layout),    sizeof(bk_stats),         sizeof(bk_out_pattern)};
-  for (int i = 0; i < n && i < 9; ++i) sizes[i] = v[i];
+  const uint32_t v[10] = {sizeof(bk_config),     sizeof(bk_out_wordcount), sizeof(bk_out_grep),
+                          sizeof(bk_out_kmeans), sizeof(bk_out_partition), sizeof(bk_out_groupby),
+                          sizeof(bk_out_layout), sizeof(bk_stats),         sizeof(bk_out_pattern),
+                          sizeof(bk_out_kmer)};
+  for (int i = 0; i < n && i < 10; ++i) sizes[i] = v[i];
   return BK_ABI_VERSION;
 }
 
@@ -1547,7 +1602,7 @@ int bk_destroy(bk_ctx* c) {
     cudaStreamDestroy(c->s_d2h);
   }
   for (auto e : c->ev_part) cudaEventDestroy(e);
-  if (c->out_pinned) cudaHostUnregister(c->out_pinned);
+  for (auto& e : c->out_pinned) cudaHostUnregister(e.first);
   for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base}) b->release();
   for (auto* h : c->hstage) cudaFreeHost(h);
   for (auto e : c->h_done) cudaEventDestroy(e);

@@ -1,0 +1,106 @@
+// kernels_kmer.cu — f4, the second workload family: k-mer counting over fixed-length DNA read
+// records (the paper's DNA assembly builds a k-mer hash table; Table I P:927:
+// fixed-length records, 36% read). Stage 1-3 stage only the sequence field (FIELD access); here
+// each thread walks its lane's reads base by base (the warp in lockstep: reads have one length),
+// rolls the 2-bit k-mer (A=0 C=1 G=2 T=3; any other byte breaks the window) and counts it in an
+// exact-key open-addressing table (key = k-mer + 1, no hashing collisions in identity). Equal
+// k-mers of one warp step are merged with __match_any_sync; an existing key costs one load and a
+// fire-and-forget atomic add.
+#include "bk_internal.cuh"
+
+namespace bk {
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+__device__ __forceinline__ void kmer_insert(KmerEntry* table, uint64_t mask, unsigned long long key, unsigned cnt,
+                                            unsigned long long* used, int* err) {
+  uint64_t slot = mix64(key) & mask;
+  for (uint64_t probe = 0; probe <= mask; ++probe, slot = (slot + 1) & mask) {
+    unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(&table[slot].key);
+    if (k == 0) {
+      k = atomicCAS(&table[slot].key, 0ull, key);
+      if (k == 0) atomicAdd(used, 1ull);
+    }
+    if (k == 0 || k == key) {
+      atomicAdd(&table[slot].count, (unsigned long long)cnt);
+      return;
+    }
+  }
+  atomicOr(err, kErrTableFull);
+}
+
+__global__ void __launch_bounds__(256) k_kmer(Chunk c, const uint8_t* __restrict__ stage,
+                                              const LaneDesc* __restrict__ lanes,
+                                              const uint64_t* __restrict__ tile_base, uint32_t k, uint32_t seq_words,
+                                              KmerEntry* table, uint64_t mask, unsigned long long* used,
+                                              unsigned long long* total, int* err) {
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= c.L) return;  // whole warps
+  const int lane = t & 31;
+  const LaneDesc d = lanes[t];
+  const uint8_t* tile = stage + tile_base[t >> 5];
+  const uint32_t R = __reduce_max_sync(kFull, d.nrec);
+  const uint64_t kmask = k == 32 ? ~0ull : ((1ull << (2 * k)) - 1);
+  unsigned long long mine = 0;
+  for (uint32_t j = 0; j < R; ++j) {
+    const bool rec = j < d.nrec;
+    uint64_t v = 0;
+    uint32_t valid = 0;
+    for (uint32_t w = 0; w < seq_words; ++w) {
+      uint4 q = make_uint4(0, 0, 0, 0);
+      if (rec) q = *reinterpret_cast<const uint4*>(tile + ((size_t)(j * seq_words + w) * 32 + lane) * 16);
+      const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+      for (int b = 0; b < 16; ++b) {
+        const uint32_t ch = (wd[b >> 2] >> (8 * (b & 3))) & 0xff;
+        const int code = ch == 'A' ? 0 : ch == 'C' ? 1 : ch == 'G' ? 2 : ch == 'T' ? 3 : -1;
+        if (code < 0) {
+          valid = 0;
+          v = 0;
+        } else {
+          v = ((v << 2) | (uint64_t)code) & kmask;
+          ++valid;
+        }
+        const bool emit = rec && valid >= k;
+        const unsigned act = __ballot_sync(kFull, emit);
+        if (act) {
+          const unsigned long long key = v + 1;
+          const unsigned m = __match_any_sync(kFull, emit ? key : 0ull);
+          if (emit && lane == __ffs(m & act) - 1) kmer_insert(table, mask, key, __popc(m & act), used, err);
+          mine += emit;
+        }
+      }
+    }
+  }
+  mine = __reduce_add_sync(kFull, (unsigned)mine);
+  if (lane == 0 && mine) atomicAdd(total, mine);
+}
+
+__global__ void k_kmer_compact(const KmerEntry* __restrict__ table, uint64_t slots, unsigned long long* n_out,
+                               uint64_t* kmer, uint64_t* cnt, uint64_t cap) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < slots; i += (uint64_t)gridDim.x * blockDim.x) {
+    const KmerEntry e = table[i];
+    if (e.key == 0) continue;
+    const unsigned long long p = atomicAdd(n_out, 1ull);
+    if (p < cap) {
+      kmer[p] = e.key - 1;
+      cnt[p] = e.count;
+    }
+  }
+}
+
+}  // namespace
+
+void launch_kmer(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base, uint32_t k,
+                 uint32_t seq_words, KmerEntry* table, uint64_t mask, unsigned long long* used,
+                 unsigned long long* total, int* err, cudaStream_t s) {
+  k_kmer<<<(c.L + 255) / 256, 256, 0, s>>>(c, stage, lanes, tile_base, k, seq_words, table, mask, used, total, err);
+}
+
+void launch_kmer_compact(const KmerEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* kmer,
+                         uint64_t* cnt, uint64_t cap, cudaStream_t s) {
+  k_kmer_compact<<<148 * 4, 256, 0, s>>>(table, slots, n_out, kmer, cnt, cap);
+}
+
+}  // namespace bk
