@@ -4,11 +4,11 @@ ARCH   := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -std=c++17 -O3 -lineinfo $(ARCH) -Xcompiler -fPIC,-fvisibility=hidden -Xptxas -v
 PKG    := paper_conf_ipps_mokhtaris14_b200
 CSRC   := $(PKG)/csrc
-OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/kernels_pattern.o build/kernels_kmer.o build/bk_runtime.o build/host_gather.o
+OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/kernels_pattern.o build/kernels_kmer.o build/runtime_plan.o build/runtime_pipeline.o build/runtime_kernels.o build/runtime_api.o build/host_gather.o
 
 all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so baselines/libbkmt.so
 
-build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh include/bk.h
+build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh $(CSRC)/runtime.cuh include/bk.h
 	@mkdir -p build
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
 

@@ -1,0 +1,314 @@
+// runtime.cuh — internal host-side definitions of libbk's runtime (context, plan, ring slots,
+// CUDA-graph cache) shared by the runtime translation units:
+//   runtime_plan.cu      chunk + lane planning, slot carving (a1)
+//   runtime_pipeline.cu  stages 1-3 per chunk, event ring, fork/join, stats, graphs (a2-a4, a6)
+//   runtime_kernels.cu   the per-kernel drivers (a5, a7) and the experiment kernels
+//   runtime_api.cu       the C ABI of include/bk.h (a0: create / register / run / destroy)
+//
+//
+// Paper mapping (Fig. 3, §III, §IV.C):
+//   * pinned buffers      -> the data set itself is pinned + mapped ONCE at
+//                                        registration; device staging is allocated once at create;
+//   * wait_addrReady / signal_dataReady flags -> cudaEvents per slot;
+//   * "at minimum two" buffer instances, addr-gen n syncs with compute n-3
+//                                     -> a ring of N slots; chunk c reuses slot c % N only after
+//                                        the compute of chunk c - N recorded slot_free;
+//   * CPU assembly thread per block -> replaced by a GPU gather kernel that reads
+//                                        pinned host memory directly (zero-copy) or by a DMA of
+//                                        the whole chunk followed by an HBM re-layout kernel.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <thread>
+#include <utility>
+#include <vector>
+
+#include "../../include/bk.h"
+#include "bk_internal.cuh"
+#include "host_gather.h"
+
+namespace bk {
+namespace rt {
+
+// Sets the thread-local detail string of bk_last_error() and returns `code`.
+int fail(int code, const char* fmt, ...);
+
+#define BK_CUDA(expr)                                                                        \
+  do {                                                                                       \
+    cudaError_t e_ = (expr);                                                                 \
+    if (e_ != cudaSuccess)                                                                   \
+      return ::bk::rt::fail(BK_E_CUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+
+constexpr uint64_t kAlign = 256;
+inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+struct Slot {
+  uint8_t* raw = nullptr;       // DENSE: the chunk's record bytes as DMA'd
+  uint8_t* stage = nullptr;     // interleaved warp tiles
+  uint64_t* meta = nullptr;     // offsets slice off[lo .. hi-1]
+  LaneDesc* lanes = nullptr;
+  uint32_t* tileK = nullptr;
+  uint64_t* tile_base = nullptr;
+  uint8_t* out = nullptr;       // per-chunk output (partition: the bucket-sorted chunk)
+  cudaEvent_t copied = nullptr, ready = nullptr, freed = nullptr;
+  bool used = false;
+};
+
+// Resident (outside the window) per-kernel device buffers, grown on demand.
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t bytes) {
+    if (bytes <= cap) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e == cudaSuccess) cap = bytes;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+// A run plan: depends only on the registration, the access spec and the config, so it is
+// computed once and cached per context (plan_cache) until the next registration.
+struct Plan {
+  Access a{};
+  int mode = BK_GATHER_DENSE;          // resolved gather mode
+  int zero_copy = 0;                   // plan budget counts accessed bytes (every mode but DENSE)
+  uint64_t budget = 0;                 // plan bytes per chunk
+  uint32_t L = 0;
+  uint64_t max_acc_rec = 0;            // max accessed bytes of one record
+  uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
+  std::vector<uint64_t> bounds;        // chunk record bounds
+  std::string key;                     // plan-cache key (also part of the graph key)
+};
+
+// A captured pipeline (CUDA graph) for one (kernel, parameters, plan, output pointers), replayed
+// by later bk_run calls with the same key instead of re-issuing ~10 launches/copies per chunk.
+struct GraphEntry {
+  std::string key;
+  cudaGraphExec_t exec = nullptr;
+  bk_stats st{};
+  int n_launch = 0;
+  size_t prof_used = 0;
+  std::vector<int> prof_stage;
+};
+
+}  // namespace rt
+}  // namespace bk
+
+struct bk_ctx {  // the opaque context of include/bk.h
+  bk_config cfg{};
+  cudaStream_t s_copy = nullptr, s_asm = nullptr, s_comp = nullptr;
+  std::vector<cudaStream_t> s_slot;  // per-slot compute streams for commutative kernels
+  cudaEvent_t ev_begin = nullptr, ev_end = nullptr;
+  cudaEvent_t t_begin = nullptr, t_end = nullptr;   // timing events on s_comp (device time of a run)
+  std::vector<cudaEvent_t> prof;                   // BK_FLAG_PROFILE: per chunk x stage begin/end
+  std::vector<int> prof_stage;                     // stage id of each event pair
+  size_t prof_used = 0;
+  uint8_t* window = nullptr;    // the whole streaming working set (cfg.window_bytes)
+  std::vector<bk::rt::Slot> slots;
+  // registration
+  const uint8_t* host = nullptr;
+  uint64_t nbytes = 0;
+  const uint64_t* off = nullptr;
+  uint64_t n = 0;
+  bool pinned_data = false, pinned_off = false, registered = false;
+  const uint8_t* host_dev = nullptr;   // device alias of the mapped data set
+  uint64_t max_rec = 0, min_rec = 0;
+  // device scratch / resident buffers
+  int* d_err = nullptr;
+  unsigned long long* d_ctr = nullptr;  // [0] staged sum, [1] wc used, [2] wc n_out, [3] grep running, [4] kmeans chk
+  bk::rt::DevBuf b_table, b_out1, b_out2, b_out3, b_blk, b_blk2, b_agg1, b_agg2, b_agg3, b_mu;
+  // CPU assembly (BK_GATHER_CPU / HYBRID): thread pool + pinned host staging ring
+  bk::HostPool* pool = nullptr;
+  std::vector<uint8_t*> hstage;
+  std::vector<cudaEvent_t> h_done;
+  std::vector<bool> h_used;
+  uint64_t hstage_cap = 0;
+  uint64_t h_next = 0;
+  std::vector<uint64_t> scratch_first, scratch_tiles;
+  // partition: D2H stream, per-slot "kernels done" events, resident totals, pinned output cache
+  cudaStream_t s_d2h = nullptr;
+  std::vector<cudaEvent_t> ev_part;
+  bk::rt::DevBuf b_hist, b_colpre, b_totals, b_base;
+  std::vector<std::pair<void*, uint64_t>> out_pinned;  // caller output arrays this context pinned
+  int n_launch = 0;
+  bk_stats st{};
+  std::vector<std::pair<std::string, bk::rt::Plan>> plan_cache;
+  std::vector<bk::rt::GraphEntry> graphs;
+  cudaEvent_t ev_fork = nullptr;
+  std::vector<cudaEvent_t> ev_join;
+  float* h_mu = nullptr;   // pinned copy of the k-means centroids (graph memcpy source)
+  uint64_t test_rng = 0x9E3779B97F4A7C15ull;   // BK_FLAG_TEST_DELAYS
+};
+
+
+namespace bk {
+namespace rt {
+
+// ---- planning (runtime_plan.cu)
+bool is_pinned(const void* p);
+uint64_t rec_start(const bk_ctx* c, uint64_t r);
+int make_chunks(const bk_ctx* c, Plan& p);
+int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t out_per_chunk = 0,
+             int auto_mode = BK_GATHER_AUTO);
+void carve(bk_ctx* c, const Plan& p);
+Chunk chunk_of(const bk_ctx* c, const Plan& p, size_t i);
+Access whole_access();
+Access field_access(uint32_t off, uint32_t len);
+int parse_access(const bk_ctx* c, uint32_t n_ext, const uint32_t* eo, const uint32_t* el, Access& a);
+
+// ---- pipeline (runtime_pipeline.cu)
+enum { kStH2D = 0, kStAddrgen = 1, kStGather = 2, kStCompute = 3, kStRelayout = 4, kNStages = 5 };
+int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin);
+#define BK_PROF(stage, stream, begin) do { int r_ = prof_mark(c, stage, stream, begin); if (r_) return r_; } while (0)
+uint64_t test_rand(bk_ctx* c);
+#define BK_DELAY(stream)                                                                      \
+  do {                                                                                        \
+    if (c->cfg.flags & BK_FLAG_TEST_DELAYS) launch_spin((long long)(::bk::rt::test_rand(c) % 200000), stream); \
+  } while (0)
+int ensure_host_side(bk_ctx* c, const Plan& p);
+int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s);
+int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s);
+void note_plan(bk_ctx* c, const Plan& p);
+int check_err(bk_ctx* c);
+int begin_run(bk_ctx* c, void* stream);
+int end_run(bk_ctx* c, void* stream);
+int device_begin(bk_ctx* c);
+int device_end(bk_ctx* c);
+void host_reset(bk_ctx* c);
+int prof_reserve(bk_ctx* c, size_t pairs);
+int end_host(bk_ctx* c, void* stream);
+void drop_graphs(bk_ctx* c);
+bool graphable(const Plan& p);
+int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes);
+void unregister(bk_ctx* c);
+
+template <class Compute>
+int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
+  const size_t C = p.bounds.size() - 1;
+  c->st.n_chunks = C;
+  note_plan(c, p);
+  std::vector<cudaEvent_t> zc_inflight;
+  const size_t zc_depth = std::max<size_t>(1, (c->cfg.n_slots - 1) / 2);
+  if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
+    int rc = ensure_host_side(c, p);
+    if (rc) return rc;
+  }
+  for (size_t i = 0; i < C; ++i) {
+    Slot& s = c->slots[i % c->cfg.n_slots];
+    cudaStream_t cs = concurrent ? c->s_slot[i % c->cfg.n_slots] : c->s_comp;
+    bool cpu = p.mode == BK_GATHER_CPU;
+    if (p.mode == BK_GATHER_HYBRID && c->cfg.zc_share_pm) {
+      // deterministic split (profiling, reproducibility): chunk i is zero-copy iff
+      // floor((i+1) s) > floor(i s)
+      const uint64_t pm = std::min<uint32_t>(c->cfg.zc_share_pm, 1000);
+      cpu = ((i + 1) * pm) / 1000 == (i * pm) / 1000;
+    } else if (p.mode == BK_GATHER_HYBRID) {
+      // adaptive split (default): the GPU zero-copy gathers run asynchronously; keep one in flight
+      // and let the host pool assemble the next chunk while it is busy (profiles/r01_hybrid_sweep.md)
+      while (!zc_inflight.empty() && cudaEventQuery(zc_inflight.front()) == cudaSuccess)
+        zc_inflight.erase(zc_inflight.begin());
+      cudaGetLastError();
+      cpu = zc_inflight.size() >= zc_depth;
+    }
+    int rc = cpu ? stage_chunk_cpu(c, p, i, s) : stage_chunk(c, p, i, s);
+    if (rc) return rc;
+    if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(s.ready);
+    BK_CUDA(cudaStreamWaitEvent(cs, s.ready, 0));
+    BK_DELAY(cs);
+    BK_PROF(kStCompute, cs, true);
+    cudaStream_t rel = cs;   // stream whose completion frees the slot (partition: its D2H)
+    rc = compute(chunk_of(c, p, i), s, cs, rel);
+    if (rc) return rc;
+    BK_PROF(kStCompute, cs, false);
+    BK_CUDA(cudaEventRecord(s.freed, rel));
+  }
+  if (concurrent)  // join: finalize on s_comp after every slot's last compute
+    for (auto& s : c->slots)
+      if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_comp, s.freed, 0));
+  return BK_OK;
+}
+
+
+template <class Enqueue>
+int run_device(bk_ctx* c, void* stream, const std::string& key, bool graphable, size_t n_chunks, Enqueue&& enqueue) {
+  BK_CUDA(cudaSetDevice(c->cfg.device));
+  host_reset(c);
+  BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_begin, 0));
+  BK_CUDA(cudaEventRecord(c->t_begin, c->s_comp));
+  int rc;
+  // per-stage profiling events must be real stream events (timestamps), so BK_FLAG_PROFILE issues eagerly
+  if (!graphable || (c->cfg.flags & (BK_FLAG_NO_GRAPH | BK_FLAG_PROFILE))) {
+    if ((rc = device_begin(c)) || (rc = enqueue()) || (rc = device_end(c))) return rc;
+    return end_host(c, stream);
+  }
+  GraphEntry* ge = nullptr;
+  for (auto& g : c->graphs)
+    if (g.key == key) ge = &g;
+  if (ge) {
+    const double reg = c->st.ms_register;
+    c->st = ge->st;
+    c->st.ms_register = reg;
+    c->n_launch = ge->n_launch;
+    c->prof_used = ge->prof_used;
+    for (size_t i = 0; i < ge->prof_stage.size(); ++i) c->prof_stage[i] = ge->prof_stage[i];
+  } else {
+    if ((rc = prof_reserve(c, 4 * n_chunks + 8))) return rc;
+    BK_CUDA(cudaStreamBeginCapture(c->s_comp, cudaStreamCaptureModeThreadLocal));
+    rc = device_begin(c);
+    if (!rc) rc = enqueue();
+    if (!rc) rc = device_end(c);
+    cudaGraph_t graph = nullptr;
+    const cudaError_t e = cudaStreamEndCapture(c->s_comp, &graph);
+    if (rc) {
+      if (graph) cudaGraphDestroy(graph);
+      cudaGetLastError();
+      return rc;
+    }
+    if (e != cudaSuccess) return fail(BK_E_CUDA, "graph capture: %s", cudaGetErrorString(e));
+    GraphEntry g;
+    g.key = key;
+    const cudaError_t ie = cudaGraphInstantiate(&g.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (ie != cudaSuccess) return fail(BK_E_CUDA, "cudaGraphInstantiate: %s", cudaGetErrorString(ie));
+    g.st = c->st;
+    g.n_launch = c->n_launch;
+    g.prof_used = c->prof_used;
+    g.prof_stage.assign(c->prof_stage.begin(), c->prof_stage.begin() + std::min(c->prof_stage.size(), c->prof_used / 2));
+    c->graphs.push_back(std::move(g));
+    ge = &c->graphs.back();
+  }
+  BK_CUDA(cudaGraphLaunch(ge->exec, c->s_comp));
+  return end_host(c, stream);
+}
+
+
+// ---- kernel drivers (runtime_kernels.cu)
+int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream);
+int run_grep(bk_ctx* c, bk_out_grep* o, void* stream);
+int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream);
+int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream);
+int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream);
+int run_partition(bk_ctx* c, bk_out_partition* o, void* stream);
+int run_dbuf(bk_ctx* c, int kid, void* out, void* stream);
+int run_pattern(bk_ctx* c, bk_out_pattern* o, void* stream);
+int run_layout(bk_ctx* c, bk_out_layout* o, void* stream);
+
+}  // namespace rt
+}  // namespace bk

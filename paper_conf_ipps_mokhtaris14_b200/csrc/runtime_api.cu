@@ -1,0 +1,308 @@
+// runtime_api.cu — the C ABI of include/bk.h: context creation (streams, events, window), registration
+// (validate offsets once, pin once), run dispatch by kernel id, statistics, destruction.
+#include "runtime.cuh"
+
+namespace bk {
+namespace rt {
+
+namespace {
+thread_local std::string g_last_error;
+}  // namespace
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return code;
+}
+
+const char* last_error() { return g_last_error.c_str(); }
+
+}  // namespace rt
+}  // namespace bk
+
+using namespace bk;
+using namespace bk::rt;
+
+extern "C" {
+
+const char* bk_strerror(int status) {
+  switch (status) {
+    case BK_OK: return "ok";
+    case BK_E_INVAL: return "invalid argument";
+    case BK_E_NOMEM: return "out of memory / window too small";
+    case BK_E_CUDA: return "CUDA error";
+    case BK_E_STATE: return "bad call order";
+    case BK_E_RANGE: return "record exceeds chunk budget";
+    case BK_E_CAPACITY: return "output capacity too small";
+    case BK_E_UNSUPPORTED: return "unsupported";
+    default: return "unknown status";
+  }
+}
+
+const char* bk_last_error(void) { return bk::rt::last_error(); }
+
+int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
+  if (!cfg || !out_ctx) return fail(BK_E_INVAL, "NULL argument");
+  if (cfg->struct_size != sizeof(bk_config)) return fail(BK_E_INVAL, "bk_config size %u != %zu", cfg->struct_size, sizeof(bk_config));
+  *out_ctx = nullptr;
+  bk_ctx* c = new (std::nothrow) bk_ctx();
+  if (!c) return fail(BK_E_NOMEM, "host allocation");
+  c->cfg = *cfg;
+  if (!c->cfg.window_bytes) c->cfg.window_bytes = 2ull << 30;
+  if (!c->cfg.n_slots) c->cfg.n_slots = 4;
+  if (c->cfg.n_slots < 2 || c->cfg.n_slots > 64) { delete c; return fail(BK_E_INVAL, "n_slots must be in 2..64"); }
+  if (c->cfg.lanes % 32) { delete c; return fail(BK_E_INVAL, "lanes must be a multiple of 32"); }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || c->cfg.device < 0 || c->cfg.device >= ndev) {
+    cudaGetLastError();
+    delete c;
+    return fail(BK_E_CUDA, "no CUDA device %d", cfg->device);
+  }
+  c->cfg.window_bytes = c->cfg.window_bytes / (c->cfg.n_slots * kAlign) * (c->cfg.n_slots * kAlign);
+  auto cleanup = [&](int rc) { bk_destroy(c); return rc; };
+  if (cudaSetDevice(c->cfg.device) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaSetDevice"));
+  if (configure_compute_kernels() != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
+  if (cudaStreamCreateWithFlags(&c->s_copy, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->s_asm, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->s_comp, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_begin, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_end, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreate(&c->t_begin) != cudaSuccess || cudaEventCreate(&c->t_end) != cudaSuccess)
+    return cleanup(fail(BK_E_CUDA, "stream/event creation"));
+  if (cudaMalloc(&c->window, c->cfg.window_bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return cleanup(fail(BK_E_NOMEM, "cudaMalloc window %llu B", (unsigned long long)c->cfg.window_bytes));
+  }
+  if (cudaMalloc(&c->d_err, 256) != cudaSuccess || cudaMalloc(&c->d_ctr, 8 * sizeof(unsigned long long)) != cudaSuccess)
+    return cleanup(fail(BK_E_NOMEM, "cudaMalloc scratch"));
+  c->slots.resize(c->cfg.n_slots);
+  if (cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "d2h stream"));
+  if (configure_partition_kernels() != cudaSuccess || configure_baseline_kernels() != cudaSuccess)
+    return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
+  if (cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess)
+    return cleanup(fail(BK_E_CUDA, "events"));
+  c->ev_join.assign(3 + c->cfg.n_slots, nullptr);
+  for (auto& e : c->ev_join)
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
+  c->ev_part.assign(c->cfg.n_slots, nullptr);
+  for (auto& e : c->ev_part)
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
+  c->s_slot.assign(c->cfg.n_slots, nullptr);
+  for (auto& st : c->s_slot)
+    if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "slot streams"));
+  for (auto& s : c->slots) {
+    if (cudaEventCreateWithFlags(&s.copied, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&s.ready, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&s.freed, cudaEventDisableTiming) != cudaSuccess)
+      return cleanup(fail(BK_E_CUDA, "slot events"));
+  }
+  c->st.struct_size = sizeof(bk_stats);
+  c->st.n_slots = c->cfg.n_slots;
+  c->st.slot_bytes = c->cfg.window_bytes / c->cfg.n_slots;
+  *out_ctx = c;
+  return BK_OK;
+}
+
+int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const uint64_t* off, uint64_t n) {
+  if (!c) return fail(BK_E_INVAL, "NULL ctx");
+  if (!host_ptr && nbytes) return fail(BK_E_INVAL, "NULL host_ptr");
+  const auto t0 = std::chrono::steady_clock::now();
+  if (cudaSetDevice(c->cfg.device) != cudaSuccess) return fail(BK_E_CUDA, "cudaSetDevice");
+  unregister(c);
+  uint64_t maxr = 0, minr = ~0ull;
+  if (off) {
+    if (n && off[0] != 0) return fail(BK_E_INVAL, "record_offsets[0] != 0");
+    for (uint64_t i = 0; i < n; ++i) {
+      const uint64_t e = i + 1 < n ? off[i + 1] : nbytes;
+      if (e < off[i] || e > nbytes) return fail(BK_E_INVAL, "record_offsets not non-decreasing / > nbytes at %llu", (unsigned long long)i);
+      maxr = std::max(maxr, e - off[i]);
+      minr = std::min(minr, e - off[i]);
+    }
+    if (!n && nbytes) return fail(BK_E_INVAL, "bytes without records");
+  } else if (n == 0 && nbytes == 0) {
+    maxr = minr = 0;  // empty data set
+  } else {
+    const uint64_t rs = c->cfg.record_size;
+    if (!rs) return fail(BK_E_INVAL, "record_offsets == NULL needs cfg.record_size");
+    if (nbytes % rs) return fail(BK_E_INVAL, "nbytes %% record_size != 0");
+    if (n != nbytes / rs) return fail(BK_E_INVAL, "n_records != nbytes / record_size");
+    maxr = minr = rs;
+  }
+  if (!n) minr = 0;
+  c->max_rec = maxr;
+  c->min_rec = n ? minr : ~0ull;
+  if (nbytes) {
+    if (is_pinned(host_ptr)) {
+      c->pinned_data = false;
+    } else {
+      cudaError_t e = cudaHostRegister((void*)host_ptr, nbytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+      if (e != cudaSuccess) return fail(BK_E_CUDA, "cudaHostRegister(data, %llu): %s", (unsigned long long)nbytes, cudaGetErrorString(e));
+      c->pinned_data = true;
+    }
+    void* dptr = nullptr;
+    cudaError_t e = cudaHostGetDevicePointer(&dptr, (void*)host_ptr, 0);
+    if (e != cudaSuccess) {
+      if (c->pinned_data) cudaHostUnregister((void*)host_ptr);
+      c->pinned_data = false;
+      return fail(BK_E_CUDA, "cudaHostGetDevicePointer (memory pinned without cudaHostRegisterMapped?): %s", cudaGetErrorString(e));
+    }
+    c->host_dev = (const uint8_t*)dptr;
+  }
+  if (off && n) {
+    if (is_pinned(off)) {
+      c->pinned_off = false;
+    } else {
+      cudaError_t e = cudaHostRegister((void*)off, n * 8, cudaHostRegisterMapped | cudaHostRegisterPortable);
+      if (e != cudaSuccess) return fail(BK_E_CUDA, "cudaHostRegister(offsets): %s", cudaGetErrorString(e));
+      c->pinned_off = true;
+    }
+  }
+  c->host = (const uint8_t*)host_ptr;
+  c->nbytes = nbytes;
+  c->off = off;
+  c->n = n;
+  c->registered = true;
+  c->plan_cache.clear();
+  drop_graphs(c);
+  c->st.ms_register = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return BK_OK;
+}
+
+int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
+  if (!c || !out) return fail(BK_E_INVAL, "NULL argument");
+  if (!c->registered) return fail(BK_E_STATE, "bk_run before bk_register_segments");
+  const bk_out_header* h = (const bk_out_header*)out;
+  if (h->kernel_id != kernel_id) return fail(BK_E_INVAL, "out->kernel_id %d != %d", h->kernel_id, kernel_id);
+  const auto t0 = std::chrono::steady_clock::now();
+  int rc;
+  if (c->cfg.flags & (BK_FLAG_BASELINE_DBUF | BK_FLAG_BASELINE_SBUF)) {
+    rc = run_dbuf(c, kernel_id, out, stream);
+    if (rc) {
+      cudaDeviceSynchronize();
+      cudaGetLastError();
+      return rc;
+    }
+    c->st.kernel_launches = (uint64_t)c->n_launch;
+    c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return BK_OK;
+  }
+  switch (kernel_id) {
+    case BK_K_WORDCOUNT:
+      if (h->struct_size != sizeof(bk_out_wordcount)) return fail(BK_E_INVAL, "bk_out_wordcount size");
+      rc = run_wordcount(c, (bk_out_wordcount*)out, stream);
+      break;
+    case BK_K_GREP:
+      if (h->struct_size != sizeof(bk_out_grep)) return fail(BK_E_INVAL, "bk_out_grep size");
+      rc = run_grep(c, (bk_out_grep*)out, stream);
+      break;
+    case BK_K_KMEANS:
+      if (h->struct_size != sizeof(bk_out_kmeans)) return fail(BK_E_INVAL, "bk_out_kmeans size");
+      rc = run_kmeans(c, (bk_out_kmeans*)out, stream);
+      break;
+    case BK_K_GROUPBY:
+      if (h->struct_size != sizeof(bk_out_groupby)) return fail(BK_E_INVAL, "bk_out_groupby size");
+      rc = run_groupby(c, (bk_out_groupby*)out, stream);
+      break;
+    case BK_K_KMER:
+      if (h->struct_size != sizeof(bk_out_kmer)) return fail(BK_E_INVAL, "bk_out_kmer size");
+      rc = run_kmer(c, (bk_out_kmer*)out, stream);
+      break;
+    case BK_K_PATTERN_STATS:
+      if (h->struct_size != sizeof(bk_out_pattern)) return fail(BK_E_INVAL, "bk_out_pattern size");
+      rc = run_pattern(c, (bk_out_pattern*)out, stream);
+      break;
+    case BK_K_LAYOUT_DUMP:
+      if (h->struct_size != sizeof(bk_out_layout)) return fail(BK_E_INVAL, "bk_out_layout size");
+      rc = run_layout(c, (bk_out_layout*)out, stream);
+      break;
+    case BK_K_PARTITION:
+      if (h->struct_size != sizeof(bk_out_partition)) return fail(BK_E_INVAL, "bk_out_partition size");
+      rc = run_partition(c, (bk_out_partition*)out, stream);
+      break;
+    default:
+      return fail(BK_E_UNSUPPORTED, "unknown kernel_id %d", kernel_id);
+  }
+  if (rc) {
+    // leave the context usable: drain whatever was queued
+    cudaStreamSynchronize(c->s_copy);
+    cudaStreamSynchronize(c->s_asm);
+    cudaStreamSynchronize(c->s_comp);
+    for (auto st : c->s_slot) cudaStreamSynchronize(st);
+    cudaGetLastError();
+    return rc;
+  }
+  c->st.kernel_launches = (uint64_t)c->n_launch;
+  c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return BK_OK;
+}
+
+int bk_get_stats(const bk_ctx* c, bk_stats* s) {
+  if (!c || !s) return fail(BK_E_INVAL, "NULL argument");
+  if (s->struct_size != sizeof(bk_stats)) return fail(BK_E_INVAL, "bk_stats size");
+  *s = c->st;
+  return BK_OK;
+}
+
+int bk_abi_sizes(uint32_t* sizes, int n) {
+  const uint32_t v[10] = {sizeof(bk_config),     sizeof(bk_out_wordcount), sizeof(bk_out_grep),
+                          sizeof(bk_out_kmeans), sizeof(bk_out_partition), sizeof(bk_out_groupby),
+                          sizeof(bk_out_layout), sizeof(bk_stats),         sizeof(bk_out_pattern),
+                          sizeof(bk_out_kmer)};
+  for (int i = 0; i < n && i < 10; ++i) sizes[i] = v[i];
+  return BK_ABI_VERSION;
+}
+
+int bk_destroy(bk_ctx* c) {
+  if (!c) return BK_OK;
+  cudaSetDevice(c->cfg.device);
+  if (c->s_comp) cudaStreamSynchronize(c->s_comp);
+  if (c->s_copy) cudaStreamSynchronize(c->s_copy);
+  if (c->s_asm) cudaStreamSynchronize(c->s_asm);
+  for (auto st : c->s_slot)
+    if (st) cudaStreamSynchronize(st);
+  unregister(c);
+  for (auto& s : c->slots) {
+    if (s.copied) cudaEventDestroy(s.copied);
+    if (s.ready) cudaEventDestroy(s.ready);
+    if (s.freed) cudaEventDestroy(s.freed);
+  }
+  for (DevBuf* b : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_agg1, &c->b_agg2,
+                    &c->b_agg3, &c->b_mu})
+    b->release();
+  if (c->window) cudaFree(c->window);
+  if (c->d_err) cudaFree(c->d_err);
+  if (c->d_ctr) cudaFree(c->d_ctr);
+  if (c->ev_begin) cudaEventDestroy(c->ev_begin);
+  if (c->ev_end) cudaEventDestroy(c->ev_end);
+  if (c->t_begin) cudaEventDestroy(c->t_begin);
+  if (c->t_end) cudaEventDestroy(c->t_end);
+  for (cudaEvent_t e : c->prof) cudaEventDestroy(e);
+  drop_graphs(c);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  for (auto e : c->ev_join) cudaEventDestroy(e);
+  if (c->h_mu) cudaFreeHost(c->h_mu);
+  delete c->pool;
+  if (c->s_d2h) {
+    cudaStreamSynchronize(c->s_d2h);
+    cudaStreamDestroy(c->s_d2h);
+  }
+  for (auto e : c->ev_part) cudaEventDestroy(e);
+  for (auto& e : c->out_pinned) cudaHostUnregister(e.first);
+  for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base}) b->release();
+  for (auto* h : c->hstage) cudaFreeHost(h);
+  for (auto e : c->h_done) cudaEventDestroy(e);
+  if (c->s_copy) cudaStreamDestroy(c->s_copy);
+  if (c->s_asm) cudaStreamDestroy(c->s_asm);
+  if (c->s_comp) cudaStreamDestroy(c->s_comp);
+  for (auto st : c->s_slot)
+    if (st) cudaStreamDestroy(st);
+  cudaGetLastError();
+  delete c;
+  return BK_OK;
+}
+
+}  // extern "C"

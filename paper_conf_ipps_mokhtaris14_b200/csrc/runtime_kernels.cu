@@ -1,0 +1,500 @@
+// runtime_kernels.cu — per-kernel drivers: plan, resident buffers, the enqueue lambda for the
+// pipeline, result copies into the caller's out struct; the double-buffering
+// baseline and the experiment kernels (layout dump, pattern statistics).
+#include "runtime.cuh"
+
+namespace bk {
+namespace rt {
+
+// ------------------------------------------------------------------ kernels
+int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
+  uint64_t slots = o->table_slots ? o->table_slots : (1ull << 20);
+  if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
+  Plan p;
+  // word count is compute-bound (thread-per-lane scan + table updates): AUTO picks ZC, which needs
+  // no raw buffer, so the window holds twice the text in flight; 256-B lanes (profiles/r01_wc_sweep.md)
+  int rc = plan_run(c, whole_access(), 256, p, 0, BK_GATHER_ZC);
+  if (rc) return rc;
+  carve(c, p);
+  BK_CUDA(c->b_table.ensure(slots * sizeof(WcEntry)));
+  const uint64_t ocap = std::min<uint64_t>(o->cap, slots);
+  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(ocap, 1) * 4));
+  BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  WcEntry* table = (WcEntry*)c->b_table.p;
+  const std::string key = "wc/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
+    int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_wc(ch, s.stage, s.lanes, s.tile_base, s.meta, c->off ? 0 : c->cfg.record_size, table, slots - 1,
+                c->d_ctr + 1, c->d_err, cs);
+      c->n_launch += 1;
+      return BK_OK;
+    });
+    if (r) return r;
+    launch_wc_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
+                      (uint64_t*)c->b_out3.p, ocap, c->s_comp);
+    c->n_launch += 1;
+    return (int)BK_OK;
+  });
+  if (rc) return rc;
+  unsigned long long nw = 0;
+  BK_CUDA(cudaMemcpy(&nw, c->d_ctr + 2, 8, cudaMemcpyDeviceToHost));
+  o->n_words = nw;
+  if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
+  if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
+                                  (unsigned long long)slots);
+  if (nw) {
+    BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->word_count, c->b_out3.p, nw * 8, cudaMemcpyDeviceToHost));
+  }
+  uint64_t tot = 0;
+  for (uint64_t i = 0; i < nw; ++i) tot += o->word_count[i];
+  o->total_words = tot;
+  c->st.bytes_d2h = nw * 20;
+  return BK_OK;
+}
+
+int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
+  if (o->pattern_len > 32) return fail(BK_E_INVAL, "pattern longer than 32 bytes");
+  if (o->pattern_len && !o->pattern) return fail(BK_E_INVAL, "NULL pattern");
+  if (c->min_rec < 48) return fail(BK_E_INVAL, "grep needs records of >= 48 bytes (key at +16..+48)");
+  Plan p;
+  int rc = plan_run(c, field_access(16, 32), 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  const uint32_t nblk = (p.L + 255) / 256;
+  const uint64_t cap = std::min<uint64_t>(o->cap, c->n);
+  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(cap, 1) * 8));
+  BK_CUDA(c->b_blk.ensure((uint64_t)nblk * 4));
+  BK_CUDA(c->b_blk2.ensure((uint64_t)nblk * 8));
+  GrepParams gp{};
+  if (o->pattern_len) memcpy(gp.pat, o->pattern, o->pattern_len);
+  gp.plen = o->pattern_len;
+  gp.first_index = o->first_index;
+  gp.cap = cap;
+  std::string key = "grep/" + std::to_string(gp.plen) + "/" + std::to_string(gp.first_index) + "/" +
+                    std::to_string(gp.cap) + "/" + p.key + "/";
+  for (uint32_t i = 0; i < gp.plen; ++i) key += std::to_string(gp.pat[i]) + ",";
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+    return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p, c->d_ctr + 3,
+                  (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, cs);
+      c->n_launch += 3;
+      return BK_OK;
+    });
+  });
+  if (rc) return rc;
+  unsigned long long m = 0;
+  BK_CUDA(cudaMemcpy(&m, c->d_ctr + 3, 8, cudaMemcpyDeviceToHost));
+  o->n_match = m;
+  if (m > o->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)o->cap);
+  if (m) BK_CUDA(cudaMemcpy(o->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_d2h = m * 8;
+  return BK_OK;
+}
+
+int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
+  const uint32_t G = o->G;
+  if (G == 0 || G > 8192) return fail(BK_E_INVAL, "G must be in 1..8192");
+  if (c->min_rec < 16) return fail(BK_E_INVAL, "group-by records must be >= 16 bytes");
+  const bool dense16 = !c->off && c->cfg.record_size == 16;
+  Plan p;
+  int rc = plan_run(c, dense16 ? whole_access() : field_access(0, 16), 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  BK_CUDA(c->b_agg1.ensure((uint64_t)G * 8));
+  BK_CUDA(c->b_agg2.ensure((uint64_t)G * 8));
+  BK_CUDA(c->b_agg3.ensure((uint64_t)G * 8));
+  int dev_sms = 148, per_sm = 1;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  per_sm = std::max<int>(1, (int)((200 * 1024) / std::max<size_t>(groupby_smem(G), 1)));
+  per_sm = std::min(per_sm, 4);
+  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * per_sm));
+  rc = run_device(c, stream, "groupby/" + std::to_string(G) + "/" + p.key, graphable(p), p.bounds.size() - 1,
+                  [&]() -> int {
+    BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)G * 8, c->s_comp));
+    return pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_groupby(ch, s.stage, s.lanes, s.tile_base, G, (unsigned long long*)c->b_agg1.p,
+                     (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, cs);
+      c->n_launch += 1;
+      return BK_OK;
+    });
+  });
+  if (rc) return rc;
+  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->qty, c->b_agg2.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->amount, c->b_agg3.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_d2h = (uint64_t)G * 24;
+  return BK_OK;
+}
+
+
+int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
+  const uint32_t K = o->K;
+  if (K == 0 || K > 256 || !o->centroids) return fail(BK_E_INVAL, "K must be in 1..256 with centroids");
+  if (c->min_rec < 64) return fail(BK_E_INVAL, "k-means records must hold 16 fp32 (>= 64 bytes)");
+  const bool dense64 = !c->off && c->cfg.record_size == 64;
+  Plan p;
+  // cid write-back (P:563-572 writes to mapped data; "sets its clusterId"): 4 B per
+  // record per chunk in the slot, DMA'd back on the D2H stream while the next chunks stream in
+  int rc = plan_run(c, dense64 ? whole_access() : field_access(0, 64), 256, p, o->cid ? 4 : 0);
+  if (rc) return rc;
+  carve(c, p);
+  if (o->cid && (rc = ensure_out_pinned(c, o->cid, c->n * 4))) return rc;
+  BK_CUDA(c->b_mu.ensure((uint64_t)K * 64));
+  BK_CUDA(c->b_agg1.ensure((uint64_t)K * 8));
+  BK_CUDA(c->b_agg3.ensure((uint64_t)K * 16 * 8));
+  int dev_sms = 148;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  if (!c->h_mu) BK_CUDA(cudaHostAlloc((void**)&c->h_mu, 256 * 64, cudaHostAllocPortable));
+  memcpy(c->h_mu, o->centroids, (size_t)K * 64);   // the graph copies from this pinned buffer
+  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
+  const std::string key = "kmeans/" + std::to_string(K) + "/" + std::to_string(o->first_index) + "/" +
+                          std::to_string((uintptr_t)o->cid) + "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+  BK_CUDA(cudaMemcpyAsync(c->b_mu.p, c->h_mu, (uint64_t)K * 64, cudaMemcpyHostToDevice, c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
+  size_t ci = 0;
+  int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
+    launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
+                  (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4,
+                  o->cid ? (int32_t*)s.out : nullptr, grid, cs);
+    c->n_launch += 1;
+    if (o->cid && ch.hi > ch.lo) {
+      cudaEvent_t e = c->ev_part[ci++ % c->ev_part.size()];
+      BK_CUDA(cudaEventRecord(e, cs));
+      BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
+      BK_CUDA(cudaMemcpyAsync(o->cid + ch.lo, s.out, (ch.hi - ch.lo) * 4, cudaMemcpyDeviceToHost, c->s_d2h));
+      c->st.bytes_d2h += (ch.hi - ch.lo) * 4;
+      rel = c->s_d2h;
+    }
+    return (int)BK_OK;
+  });
+  return r;
+  });
+  if (rc) return rc;
+  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->sum, c->b_agg3.p, (uint64_t)K * 128, cudaMemcpyDeviceToHost));
+  unsigned long long chk = 0;
+  BK_CUDA(cudaMemcpy(&chk, c->d_ctr + 4, 8, cudaMemcpyDeviceToHost));
+  o->chk = chk;
+  c->st.bytes_d2h += (uint64_t)K * 136;
+  return BK_OK;
+}
+
+// f4: k-mer counting (FIELD access to the sequence; the table is resident, outside the window)
+int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
+  const uint64_t slots = o->table_slots ? o->table_slots : (1ull << 24);
+  if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
+  if (o->k < 1 || o->k > 31) return fail(BK_E_INVAL, "k must be in 1..31");
+  if (o->seq_len == 0 || o->seq_len % 16) return fail(BK_E_INVAL, "seq_len must be a positive multiple of 16");
+  if ((uint64_t)o->seq_off + o->seq_len > c->min_rec) return fail(BK_E_INVAL, "sequence field exceeds a record");
+  Plan p;
+  int rc = plan_run(c, field_access(o->seq_off, o->seq_len), 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  BK_CUDA(c->b_table.ensure(slots * sizeof(KmerEntry)));
+  const uint64_t ocap = std::min<uint64_t>(o->cap, slots);
+  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  KmerEntry* table = (KmerEntry*)c->b_table.p;
+  const std::string key = "kmer/" + std::to_string(o->k) + "/" + std::to_string(slots) + "/" + std::to_string(ocap) +
+                          "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(KmerEntry), c->s_comp));
+    int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_kmer(ch, s.stage, s.lanes, s.tile_base, o->k, o->seq_len / 16, table, slots - 1, c->d_ctr + 1,
+                  c->d_ctr + 5, c->d_err, cs);
+      c->n_launch += 1;
+      return BK_OK;
+    });
+    if (r) return r;
+    launch_kmer_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint64_t*)c->b_out3.p, ocap, c->s_comp);
+    c->n_launch += 1;
+    return (int)BK_OK;
+  });
+  if (rc) return rc;
+  unsigned long long nk = 0, tot = 0;
+  BK_CUDA(cudaMemcpy(&nk, c->d_ctr + 2, 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(&tot, c->d_ctr + 5, 8, cudaMemcpyDeviceToHost));
+  o->n_kmers = nk;
+  o->total = tot;
+  if (nk > o->cap) return fail(BK_E_CAPACITY, "%llu distinct k-mers > cap %llu", nk, (unsigned long long)o->cap);
+  if (nk * 10 > slots * 7) return fail(BK_E_CAPACITY, "k-mer table load %llu/%llu too high; raise table_slots", nk,
+                                       (unsigned long long)slots);
+  if (nk) {
+    // the result arrays are large (16 B per distinct k-mer): pin them once so the copy runs at DMA speed
+    if ((rc = ensure_out_pinned(c, o->kmer, o->cap * 8)) || (rc = ensure_out_pinned(c, o->count, o->cap * 8))) return rc;
+    BK_CUDA(cudaMemcpy(o->kmer, c->b_out1.p, nk * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->count, c->b_out3.p, nk * 8, cudaMemcpyDeviceToHost));
+  }
+  c->st.bytes_d2h = nk * 16;
+  return BK_OK;
+}
+
+int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
+  const uint32_t B = o->n_buckets;
+  if (B == 0 || B > 4096 || (B & (B - 1))) return fail(BK_E_INVAL, "n_buckets must be a power of two in 1..4096");
+  if (c->off || c->cfg.record_size != 16) return fail(BK_E_INVAL, "partition needs fixed 16-byte {key, value} records");
+  if (c->n && !o->out_records) return fail(BK_E_INVAL, "NULL out_records");
+  int bits = 0;
+  while ((1u << bits) < B) ++bits;
+  Plan p;
+  int rc = plan_run(c, whole_access(), 256, p, 16);
+  if (rc) return rc;
+  carve(c, p);
+  const uint64_t C = p.bounds.size() - 1;
+  o->n_chunks = C;
+  if (C > o->chunk_cap) return fail(BK_E_CAPACITY, "%llu chunks > chunk_cap %llu", (unsigned long long)C,
+                                    (unsigned long long)o->chunk_cap);
+  uint32_t nblk_max = 1;
+  for (uint64_t i = 0; i < C; ++i) nblk_max = std::max(nblk_max, partition_blocks(chunk_of(c, p, i)));
+  BK_CUDA(c->b_hist.ensure((uint64_t)nblk_max * B * 4));
+  BK_CUDA(c->b_colpre.ensure((uint64_t)nblk_max * B * 4));
+  BK_CUDA(c->b_totals.ensure(std::max<uint64_t>(C, 1) * B * 8));
+  BK_CUDA(c->b_base.ensure((uint64_t)B * 8));
+  if ((rc = ensure_out_pinned(c, o->out_records, c->n * 16))) return rc;
+  const std::string key = "part/" + std::to_string(B) + "/" + std::to_string((uintptr_t)o->out_records) + "/" + p.key;
+  rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
+  size_t ci = 0;
+  return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
+    launch_partition(ch, s.stage, s.lanes, s.tile_base, bits, (uint32_t*)c->b_hist.p, (uint32_t*)c->b_colpre.p,
+                     (unsigned long long*)c->b_totals.p + ci * B, (unsigned long long*)c->b_base.p, s.out, cs);
+    c->n_launch += 4;
+    cudaEvent_t e = c->ev_part[ci % c->ev_part.size()];
+    BK_CUDA(cudaEventRecord(e, cs));
+    BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
+    const uint64_t bytes = (ch.hi - ch.lo) * 16;
+    if (bytes)
+      BK_CUDA(cudaMemcpyAsync((uint8_t*)o->out_records + ch.lo * 16, s.out, bytes, cudaMemcpyDeviceToHost, c->s_d2h));
+    c->st.bytes_d2h += bytes;
+    rel = c->s_d2h;
+    ++ci;
+    return (int)BK_OK;
+  });
+  });
+  if (rc) return rc;
+  std::vector<uint64_t> tot(C * B);
+  if (C) BK_CUDA(cudaMemcpy(tot.data(), c->b_totals.p, C * B * 8, cudaMemcpyDeviceToHost));
+  for (uint32_t b = 0; b < B; ++b) o->bucket_count[b] = 0;
+  for (uint64_t i = 0; i < C; ++i)
+    for (uint32_t b = 0; b < B; ++b) {
+      o->chunk_counts[i * B + b] = tot[i * B + b];
+      o->bucket_count[b] += tot[i * B + b];
+    }
+  return BK_OK;
+}
+
+// ---- BK_FLAG_BASELINE_DBUF: the traditional chunked loop with two buffers ----
+int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
+  if (kid != BK_K_GREP && kid != BK_K_GROUPBY) return fail(BK_E_UNSUPPORTED, "dbuf baseline: grep / group-by only");
+  Plan p;
+  p.a = whole_access();
+  p.mode = BK_GATHER_DENSE;
+  p.zero_copy = 0;
+  const bool single = (c->cfg.flags & BK_FLAG_BASELINE_SBUF) != 0;
+  const uint64_t half = c->cfg.window_bytes / (single ? 1 : 2) / kAlign * kAlign;
+  uint64_t budget = std::max<uint64_t>(std::min<uint64_t>(half, std::max<uint64_t>(c->nbytes / 32, 1ull << 20)), 1);
+  uint64_t meta_cap = 0;
+  for (int it = 0;; ++it) {
+    p.budget = budget;
+    int rc = make_chunks(c, p);
+    if (rc) return rc;
+    uint64_t maxrecs = 0;
+    for (size_t i = 0; i + 1 < p.bounds.size(); ++i) maxrecs = std::max<uint64_t>(maxrecs, p.bounds[i + 1] - p.bounds[i]);
+    meta_cap = c->off ? maxrecs + 1 : 0;
+    if (align_up(budget + 64, kAlign) + meta_cap * 8 <= half) break;
+    if (it > 64 || budget < 64) return fail(BK_E_NOMEM, "window too small for the dbuf baseline");
+    budget = budget * 3 / 4;
+  }
+  uint8_t* buf[2] = {c->window, c->window + (single ? 0 : half)};
+  uint64_t* meta[2] = {reinterpret_cast<uint64_t*>(buf[0] + align_up(budget + 64, kAlign)),
+                       reinterpret_cast<uint64_t*>(buf[1] + align_up(budget + 64, kAlign))};
+  cudaStream_t sb[2] = {c->s_copy, single ? c->s_copy : c->s_asm};
+  const size_t C = p.bounds.size() - 1;
+  int rc;
+  GrepParams gp{};
+  bk_out_grep* og = (bk_out_grep*)out;
+  bk_out_groupby* ob = (bk_out_groupby*)out;
+  const uint32_t nb = dbuf_blocks();
+  if (kid == BK_K_GREP) {
+    if (og->pattern_len > 32) return fail(BK_E_INVAL, "pattern longer than 32 bytes");
+    if (c->min_rec < 48) return fail(BK_E_INVAL, "grep needs records of >= 48 bytes");
+    if (og->pattern_len) memcpy(gp.pat, og->pattern, og->pattern_len);
+    gp.plen = og->pattern_len;
+    gp.first_index = og->first_index;
+    gp.cap = std::min<uint64_t>(og->cap, c->n);
+    BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(gp.cap, 1) * 8));
+    BK_CUDA(c->b_blk.ensure((uint64_t)nb * 4 * 2));
+    BK_CUDA(c->b_blk2.ensure((uint64_t)nb * 8 * 2));
+  } else {
+    if (ob->G == 0 || ob->G > 8192) return fail(BK_E_INVAL, "G must be in 1..8192");
+    if (c->off || c->cfg.record_size < 16) return fail(BK_E_INVAL, "group-by needs fixed records >= 16 B");
+    BK_CUDA(c->b_agg1.ensure((uint64_t)ob->G * 8));
+    BK_CUDA(c->b_agg2.ensure((uint64_t)ob->G * 8));
+    BK_CUDA(c->b_agg3.ensure((uint64_t)ob->G * 8));
+  }
+  if ((rc = begin_run(c, stream))) return rc;
+  if (kid == BK_K_GROUPBY) {
+    BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+    BK_CUDA(cudaEventRecord(c->ev_begin, c->s_comp));
+    BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->ev_begin, 0));
+    BK_CUDA(cudaStreamWaitEvent(c->s_asm, c->ev_begin, 0));
+  }
+  c->st.n_chunks = C;
+  c->st.gather_mode = BK_GATHER_DENSE;
+  c->st.chunk_budget = budget;
+  cudaEvent_t scanned[2] = {c->slots[0].ready, c->slots[1].ready};
+  for (size_t i = 0; i < C; ++i) {
+    const int b = (int)(i & 1);
+    cudaStream_t st = sb[b];
+    const uint64_t lo = p.bounds[i], hi = p.bounds[i + 1];
+    const uint64_t base = rec_start(c, lo), end = rec_start(c, hi);
+    const uint64_t raw_off = ((uintptr_t)(c->host + base)) & 15;
+    BK_PROF(kStH2D, st, true);
+    if (end > base) BK_CUDA(cudaMemcpyAsync(buf[b] + raw_off, c->host + base, end - base, cudaMemcpyHostToDevice, st));
+    if (c->off && hi > lo) {
+      BK_CUDA(cudaMemcpyAsync(meta[b], c->off + lo, (hi - lo) * 8, cudaMemcpyHostToDevice, st));
+      c->st.bytes_meta += (hi - lo) * 8;
+    }
+    BK_PROF(kStH2D, st, false);
+    c->st.bytes_h2d += end - base;
+    BK_PROF(kStCompute, st, true);
+    if (kid == BK_K_GREP) {
+      // chunk i's output offset follows chunk i-1's scan (ordered results across the two streams)
+      if (i > 0) BK_CUDA(cudaStreamWaitEvent(st, scanned[1 - b], 0));
+      launch_dbuf_grep(buf[b] + raw_off, c->off ? meta[b] : nullptr, lo, hi, base, end, c->cfg.record_size, gp,
+                       (uint32_t*)c->b_blk.p + b * nb, c->d_ctr + 3, (unsigned long long*)c->b_blk2.p + b * nb,
+                       (uint64_t*)c->b_out1.p, st);
+      BK_CUDA(cudaEventRecord(scanned[b], st));
+      c->n_launch += 3;
+    } else {
+      launch_dbuf_groupby(buf[b] + raw_off, lo, hi, base, c->cfg.record_size, ob->G, (unsigned long long*)c->b_agg1.p,
+                          (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, st);
+      c->n_launch += 1;
+    }
+    BK_PROF(kStCompute, st, false);
+  }
+  for (cudaStream_t st : sb) {
+    BK_CUDA(cudaEventRecord(c->ev_end, st));
+    BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
+  }
+  if ((rc = end_run(c, stream))) return rc;
+  if (kid == BK_K_GREP) {
+    unsigned long long m = 0;
+    BK_CUDA(cudaMemcpy(&m, c->d_ctr + 3, 8, cudaMemcpyDeviceToHost));
+    og->n_match = m;
+    if (m > og->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)og->cap);
+    if (m) BK_CUDA(cudaMemcpy(og->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));
+  } else {
+    BK_CUDA(cudaMemcpy(ob->count, c->b_agg1.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(ob->qty, c->b_agg2.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(ob->amount, c->b_agg3.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
+  }
+  return BK_OK;
+}
+
+
+// BK_K_PATTERN_STATS: stage 1 in address mode with online pattern recognition, every chunk
+int run_pattern(bk_ctx* c, bk_out_pattern* o, void* stream) {
+  Access a;
+  int rc = parse_access(c, o->n_ext, o->ext_off, o->ext_len, a);
+  if (rc) return rc;
+  if (o->elem_bytes == 0 || o->T < 2 || o->T > 16 || o->pmax < 1 || o->pmax > 4)
+    return fail(BK_E_INVAL, "elem_bytes >= 1, T in 2..16, pmax in 1..4");
+  Plan p;
+  if ((rc = plan_run(c, a, 256, p))) return rc;
+  carve(c, p);
+  a.rec_size = c->off ? 0 : c->cfg.record_size;
+  o->lanes = p.L;
+  const bool want_dump = o->chunk != UINT64_MAX;
+  if (want_dump && (o->chunk >= p.bounds.size() - 1 || p.L > o->lane_cap))
+    return fail(BK_E_INVAL, "dump chunk / lane_cap");
+  BK_CUDA(c->b_out1.ensure((uint64_t)p.L * 4));
+  BK_CUDA(c->b_out2.ensure((uint64_t)p.L * 32));
+  BK_CUDA(c->b_out3.ensure((uint64_t)p.L * 16));
+  BK_CUDA(c->b_blk2.ensure(8 * 8));
+  if ((rc = begin_run(c, stream))) return rc;
+  BK_CUDA(cudaMemsetAsync(c->b_blk2.p, 0, 64, c->s_copy));
+  Slot& s = c->slots[0];
+  for (size_t i = 0; i + 1 < p.bounds.size(); ++i) {  // one stream, one slot: stage 1 only
+    const Chunk ch = chunk_of(c, p, i);
+    if (c->off && ch.hi > ch.lo)
+      BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_copy);
+    uint64_t* dumps = (uint64_t*)c->b_out3.p;
+    launch_addr_patterns(ch, a, s.meta, s.lanes, o->elem_bytes, o->T, o->pmax, (int32_t*)c->b_out1.p,
+                         (int64_t*)c->b_out2.p, dumps, dumps + p.L, (unsigned long long*)c->b_blk2.p,
+                         want_dump && i == o->chunk, c->s_copy);
+    c->n_launch += 3;
+  }
+  BK_CUDA(cudaEventRecord(c->ev_end, c->s_copy));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
+  if ((rc = end_run(c, stream))) return rc;
+  unsigned long long tot[5];
+  BK_CUDA(cudaMemcpy(tot, c->b_blk2.p, sizeof tot, cudaMemcpyDeviceToHost));
+  o->n_lanes = tot[0];
+  o->n_pattern_lanes = tot[1];
+  o->n_addresses = tot[2];
+  o->n_explicit_addresses = tot[3];
+  o->address_bytes = 8 * tot[2];
+  o->pattern_bytes = tot[4] + 8 * tot[3];
+  if (want_dump) {
+    BK_CUDA(cudaMemcpy(o->lane_p, c->b_out1.p, (uint64_t)p.L * 4, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->lane_strides, c->b_out2.p, (uint64_t)p.L * 32, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->lane_base, c->b_out3.p, (uint64_t)p.L * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(o->lane_count, (uint64_t*)c->b_out3.p + p.L, (uint64_t)p.L * 8, cudaMemcpyDeviceToHost));
+  }
+  return BK_OK;
+}
+
+int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
+  Access a;
+  int rc = parse_access(c, o->n_ext, o->ext_off, o->ext_len, a);
+  if (rc) return rc;
+  Plan p;
+  rc = plan_run(c, a, 256, p);
+  if (rc) return rc;
+  carve(c, p);
+  o->n_chunks = p.bounds.size() - 1;
+  o->lanes = p.L;
+  if (o->chunk >= o->n_chunks) return fail(BK_E_INVAL, "chunk %llu >= %llu chunks", (unsigned long long)o->chunk,
+                                           (unsigned long long)o->n_chunks);
+  if ((rc = begin_run(c, stream))) return rc;
+  Slot& s = c->slots[0];
+  if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
+    if ((rc = ensure_host_side(c, p))) return rc;
+    if ((rc = stage_chunk_cpu(c, p, o->chunk, s))) return rc;
+  } else if ((rc = stage_chunk(c, p, o->chunk, s))) {
+    return rc;
+  }
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, s.ready, 0));
+  const Chunk ch = chunk_of(c, p, o->chunk);
+  o->chunk_lo = ch.lo;
+  o->chunk_hi = ch.hi;
+  if ((rc = end_run(c, stream))) return rc;
+  uint64_t size = 0;
+  BK_CUDA(cudaMemcpy(&size, s.tile_base + ch.ntiles, 8, cudaMemcpyDeviceToHost));
+  o->stage_size = size;
+  if (size > o->stage_cap || p.L > o->lane_cap) return fail(BK_E_CAPACITY, "stage %llu / lanes %u", size, p.L);
+  BK_CUDA(cudaMemcpy(o->stage, s.stage, size, cudaMemcpyDeviceToHost));
+  std::vector<LaneDesc> ld(p.L);
+  BK_CUDA(cudaMemcpy(ld.data(), s.lanes, (uint64_t)p.L * sizeof(LaneDesc), cudaMemcpyDeviceToHost));
+  for (uint32_t t = 0; t < p.L; ++t) {
+    o->lane_first[t] = ld[t].first;
+    o->lane_nrec[t] = ld[t].nrec;
+    o->lane_bytes[t] = ld[t].nbytes;
+  }
+  return BK_OK;
+}
+
+
+}  // namespace rt
+}  // namespace bk

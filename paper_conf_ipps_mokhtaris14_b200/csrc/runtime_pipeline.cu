@@ -1,0 +1,362 @@
+// runtime_pipeline.cu — stages 1-3 of a chunk (ZC / DENSE on the GPU, CPU assembly on the host pool),
+// profiling and delay-injection hooks, fork/join of the context's streams, stage statistics and
+// the CUDA-graph cache.
+#include "runtime.cuh"
+
+namespace bk {
+namespace rt {
+
+int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin) {
+  if (!(c->cfg.flags & BK_FLAG_PROFILE)) return BK_OK;
+  if (begin) {
+    if (c->prof_used + 2 > c->prof.size()) {
+      for (int k = 0; k < 64; ++k) {
+        cudaEvent_t e;
+        BK_CUDA(cudaEventCreate(&e));
+        c->prof.push_back(e);
+        if (c->prof.size() % 2 == 0) c->prof_stage.push_back(0);
+      }
+    }
+    c->prof_stage[c->prof_used / 2] = stage;
+    BK_CUDA(cudaEventRecord(c->prof[c->prof_used], s));
+  } else {
+    BK_CUDA(cudaEventRecord(c->prof[c->prof_used + 1], s));
+    c->prof_used += 2;
+  }
+  return BK_OK;
+}
+
+uint64_t test_rand(bk_ctx* c) {
+  c->test_rng = c->test_rng * 6364136223846793005ull + 1442695040888963407ull;
+  return c->test_rng >> 33;
+}
+
+int ensure_host_side(bk_ctx* c, const Plan& p) {
+  if (!c->pool) {
+    int th = (int)c->cfg.host_threads;
+    if (th <= 0) th = (int)std::max(1u, std::thread::hardware_concurrency());
+    c->pool = new (std::nothrow) HostPool(th);
+    if (!c->pool) return fail(BK_E_NOMEM, "host pool");
+  }
+  const size_t NH = 3;
+  if (c->hstage_cap < p.stage_cap || c->hstage.size() != NH) {
+    for (auto* h : c->hstage) cudaFreeHost(h);
+    c->hstage.assign(NH, nullptr);
+    for (auto& h : c->hstage) BK_CUDA(cudaHostAlloc((void**)&h, p.stage_cap, cudaHostAllocPortable));
+    c->hstage_cap = p.stage_cap;
+    if (c->h_done.empty()) {
+      c->h_done.assign(NH, nullptr);
+      for (auto& e : c->h_done) BK_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
+  }
+  c->h_used.assign(NH, false);
+  c->h_next = 0;
+  return BK_OK;
+}
+
+// CPU assembly of chunk i (stage 2 on the host pool) + one DMA of the packed tiles (stage 3).
+int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
+  const Chunk ch = chunk_of(c, p, i);
+  Access a = p.a;
+  a.rec_size = c->off ? 0 : c->cfg.record_size;
+  const size_t hs = c->h_next++ % c->hstage.size();
+  if (c->h_used[hs]) BK_CUDA(cudaEventSynchronize(c->h_done[hs]));   // its previous DMA finished
+  if (c->cfg.flags & BK_FLAG_TEST_DELAYS)   // host-side jitter before the assembly
+    std::this_thread::sleep_for(std::chrono::microseconds(test_rand(c) % 200));
+  const auto t0 = std::chrono::steady_clock::now();
+  HostData d{c->host, c->off, c->n, c->nbytes, c->cfg.record_size};
+  const uint64_t size = host_gather_chunk(*c->pool, d, a, ch, c->hstage[hs], p.stage_cap, c->scratch_first,
+                                          c->scratch_tiles);
+  c->st.ms_cpu_gather += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  if (size == UINT64_MAX) return fail(BK_E_RANGE, "host-staged chunk exceeds its slot (internal bound violated)");
+  if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+  BK_DELAY(c->s_copy);
+    BK_PROF(kStH2D, c->s_copy, true);
+  if (c->off && a.whole && ch.hi > ch.lo) {  // record boundaries for whole-record kernels
+    BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
+    c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+  }
+  if (size) BK_CUDA(cudaMemcpyAsync(s.stage, c->hstage[hs], size, cudaMemcpyHostToDevice, c->s_copy));
+  BK_CUDA(cudaEventRecord(c->h_done[hs], c->s_copy));
+  c->h_used[hs] = true;
+  BK_PROF(kStH2D, c->s_copy, false);
+  BK_PROF(kStAddrgen, c->s_copy, true);
+  launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_copy);
+  BK_PROF(kStAddrgen, c->s_copy, false);
+  c->n_launch += 2;
+  c->st.bytes_h2d += size;   // payload + tile padding (A9: padding crosses the link only in this mode)
+  c->st.bytes_accessed += ch.accessed;
+  c->st.n_chunks_cpu += 1;
+  BK_CUDA(cudaEventRecord(s.ready, c->s_copy));
+  s.used = true;
+  return BK_OK;
+}
+
+// Stages 1-3 of chunk i into slot s (on s_copy / s_asm); records s.ready.
+int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
+  const Chunk ch = chunk_of(c, p, i);
+  Access a = p.a;
+  a.rec_size = c->off ? 0 : c->cfg.record_size;
+  if (p.zero_copy) {
+    // Stage 1 on s_asm (offsets slice by DMA + lane plan) runs ahead, overlapping the previous
+    // chunk's zero-copy gather on s_copy; the gather waits only for its own plan.
+    if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_asm, s.freed, 0));
+    BK_DELAY(c->s_asm);
+    BK_PROF(kStH2D, c->s_asm, true);
+    if (c->off && ch.hi > ch.lo) {
+      BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_asm));
+      c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+    }
+    BK_PROF(kStH2D, c->s_asm, false);
+    BK_PROF(kStAddrgen, c->s_asm, true);
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
+    BK_PROF(kStAddrgen, c->s_asm, false);
+    BK_CUDA(cudaEventRecord(s.copied, c->s_asm));
+    BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.copied, 0));
+    BK_DELAY(c->s_copy);
+    BK_PROF(kStGather, c->s_copy, true);
+    Chunk gch = ch;   // readable source: the registered data set
+    gch.guard_lo = ch.base_byte;
+    gch.guard_hi = c->nbytes - ch.base_byte;
+    launch_gather(gch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1,
+                  c->s_copy);
+    BK_PROF(kStGather, c->s_copy, false);
+    c->n_launch += 3;
+    c->st.bytes_h2d += ch.accessed;
+  } else {
+    if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+    BK_DELAY(c->s_copy);
+    BK_PROF(kStH2D, c->s_copy, true);
+    if (c->off && ch.hi > ch.lo) {
+      BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_copy));
+      c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+    }
+    const uint64_t raw_off = ((uintptr_t)(c->host + ch.base_byte)) & 15;
+    const uint64_t bytes = ch.end_byte - ch.base_byte;
+    if (bytes) BK_CUDA(cudaMemcpyAsync(s.raw + raw_off, c->host + ch.base_byte, bytes, cudaMemcpyHostToDevice, c->s_copy));
+    BK_PROF(kStH2D, c->s_copy, false);
+    BK_CUDA(cudaEventRecord(s.copied, c->s_copy));
+    BK_CUDA(cudaStreamWaitEvent(c->s_asm, s.copied, 0));
+    BK_PROF(kStAddrgen, c->s_asm, true);
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
+    BK_PROF(kStAddrgen, c->s_asm, false);
+    BK_DELAY(c->s_asm);
+    BK_PROF(kStRelayout, c->s_asm, true);
+    Chunk gch = ch;   // readable source: the raw slot (256-B aligned, 64 B of slack)
+    gch.guard_lo = raw_off;
+    gch.guard_hi = p.raw_cap - raw_off;
+    launch_gather(gch, a, s.raw + raw_off, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 0, c->s_asm);
+    BK_PROF(kStRelayout, c->s_asm, false);
+    c->n_launch += 3;
+    c->st.bytes_h2d += bytes;
+  }
+  c->st.bytes_accessed += ch.accessed;
+  BK_CUDA(cudaEventRecord(s.ready, p.zero_copy ? c->s_copy : c->s_asm));
+  s.used = true;
+  return BK_OK;
+}
+
+void note_plan(bk_ctx* c, const Plan& p) {
+  c->st.gather_mode = (uint32_t)p.mode;
+  c->st.chunk_budget = p.budget;
+  c->st.lanes = p.L;
+}
+
+int check_err(bk_ctx* c) {
+  int herr = 0;
+  BK_CUDA(cudaMemcpy(&herr, c->d_err, sizeof(int), cudaMemcpyDeviceToHost));
+  if (herr & kErrStageOverflow) return fail(BK_E_RANGE, "staged chunk exceeded its slot (internal bound violated)");
+  if (herr & kErrKeyRange) return fail(BK_E_INVAL, "a group-by key is >= G");
+  if (herr & kErrTableFull) return fail(BK_E_CAPACITY, "word-count hash table full; raise table_slots");
+  if (herr & kErrWordTooLong) return fail(BK_E_RANGE, "a word is longer than 2^24 bytes or offset >= 2^40");
+  return BK_OK;
+}
+
+// ---- the pipeline driver: chunk i goes through slot i % N; stages 1-3 on the copy/assembly
+// streams, stage 4 on the compute stream. `concurrent`: the kernel's updates commute (atomic
+// aggregation), so chunk i's compute runs on slot stream i % N and may overlap chunk i-1's;
+// otherwise (grep's ordered output) every compute is serialised on s_comp.
+
+int begin_run(bk_ctx* c, void* stream) {
+  BK_CUDA(cudaSetDevice(c->cfg.device));
+  BK_CUDA(cudaMemsetAsync(c->d_err, 0, sizeof(int), c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->d_ctr, 0, 8 * sizeof(unsigned long long), c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
+  BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_begin, 0));
+  BK_CUDA(cudaEventRecord(c->t_begin, c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_begin, c->s_comp));
+  BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->ev_begin, 0));
+  BK_CUDA(cudaStreamWaitEvent(c->s_asm, c->ev_begin, 0));
+  for (auto& s : c->slots) s.used = false;
+  c->n_launch = 0;
+  c->prof_used = 0;
+  c->st.bytes_accessed = c->st.bytes_h2d = c->st.bytes_meta = c->st.bytes_padding = c->st.bytes_d2h = 0;
+  c->st.n_chunks_cpu = 0;
+  c->st.ms_cpu_gather = 0;
+  return BK_OK;
+}
+
+// Per-stage busy sums and, from the interval of every (stage, chunk) event pair relative to the
+// run start, the union of transfer intervals, the union of compute intervals and their overlap
+// (the north_star's copy/compute overlap, measured with CUDA events instead of nsys).
+int stage_stats(bk_ctx* c) {
+  double acc[kNStages] = {0, 0, 0, 0, 0};
+  uint64_t cnt[kNStages] = {0, 0, 0, 0, 0};
+  std::vector<std::pair<double, double>> xfer, comp;
+  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
+    float e = 0, b0 = 0;
+    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
+    BK_CUDA(cudaEventElapsedTime(&b0, c->t_begin, c->prof[i]));
+    const int stg = c->prof_stage[i / 2];
+    acc[stg] += e;
+    cnt[stg] += 1;
+    if (stg == kStH2D || stg == kStGather) xfer.emplace_back(b0, b0 + e);
+    if (stg == kStCompute) comp.emplace_back(b0, b0 + e);
+  }
+  auto merge = [](std::vector<std::pair<double, double>> v) {
+    std::sort(v.begin(), v.end());
+    std::vector<std::pair<double, double>> u;
+    for (auto& x : v) {
+      if (!u.empty() && x.first <= u.back().second) u.back().second = std::max(u.back().second, x.second);
+      else u.push_back(x);
+    }
+    return u;
+  };
+  const auto ux = merge(xfer), uc = merge(comp);
+  double bx = 0, bc = 0, ov = 0;
+  for (auto& x : ux) bx += x.second - x.first;
+  for (auto& x : uc) bc += x.second - x.first;
+  for (size_t i = 0, j = 0; i < ux.size() && j < uc.size();) {  // intersection of two sorted unions
+    const double lo = std::max(ux[i].first, uc[j].first), hi = std::min(ux[i].second, uc[j].second);
+    if (hi > lo) ov += hi - lo;
+    if (ux[i].second < uc[j].second) ++i; else ++j;
+  }
+  c->st.ms_h2d = acc[kStH2D];
+  c->st.ms_addrgen = acc[kStAddrgen];
+  c->st.ms_gather = acc[kStGather] + acc[kStRelayout];
+  c->st.ms_compute = acc[kStCompute];
+  c->st.n_gather = cnt[kStGather] + cnt[kStRelayout];
+  c->st.ms_xfer_busy = bx;
+  c->st.ms_compute_busy = bc;
+  c->st.ms_overlap = ov;
+  return BK_OK;
+}
+
+int end_run(bk_ctx* c, void* stream) {
+  BK_CUDA(cudaEventRecord(c->t_end, c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_end, c->s_comp));
+  BK_CUDA(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_end, 0));
+  BK_CUDA(cudaStreamSynchronize(c->s_comp));
+  unsigned long long staged = 0;
+  BK_CUDA(cudaMemcpy(&staged, c->d_ctr + 0, 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_padding = staged >= c->st.bytes_accessed ? staged - c->st.bytes_accessed : 0;
+  float ms = 0;
+  BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
+  c->st.ms_device = ms;
+  int rc = stage_stats(c);
+  if (rc) return rc;
+  return check_err(c);
+}
+
+// ---- run_device: fork/join all streams around a pipeline; capture it as a CUDA graph once per key
+std::vector<cudaStream_t> side_streams(bk_ctx* c) {
+  std::vector<cudaStream_t> v{c->s_copy, c->s_asm, c->s_d2h};
+  for (auto st : c->s_slot) v.push_back(st);
+  return v;
+}
+
+int device_begin(bk_ctx* c) {
+  BK_CUDA(cudaMemsetAsync(c->d_err, 0, sizeof(int), c->s_comp));
+  BK_CUDA(cudaMemsetAsync(c->d_ctr, 0, 8 * sizeof(unsigned long long), c->s_comp));
+  BK_CUDA(cudaEventRecord(c->ev_fork, c->s_comp));
+  for (auto st : side_streams(c)) BK_CUDA(cudaStreamWaitEvent(st, c->ev_fork, 0));
+  return BK_OK;
+}
+
+int device_end(bk_ctx* c) {
+  const auto ss = side_streams(c);
+  for (size_t i = 0; i < ss.size(); ++i) {
+    BK_CUDA(cudaEventRecord(c->ev_join[i], ss[i]));
+    BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_join[i], 0));
+  }
+  return BK_OK;
+}
+
+void host_reset(bk_ctx* c) {
+  for (auto& s : c->slots) s.used = false;
+  c->n_launch = 0;
+  c->prof_used = 0;
+  c->st.bytes_accessed = c->st.bytes_h2d = c->st.bytes_meta = c->st.bytes_padding = c->st.bytes_d2h = 0;
+  c->st.n_chunks_cpu = 0;
+  c->st.ms_cpu_gather = 0;
+}
+
+int prof_reserve(bk_ctx* c, size_t pairs) {
+  if (!(c->cfg.flags & BK_FLAG_PROFILE)) return BK_OK;
+  while (c->prof.size() < 2 * pairs) {
+    cudaEvent_t e;
+    BK_CUDA(cudaEventCreate(&e));
+    c->prof.push_back(e);
+    if (c->prof.size() % 2 == 0) c->prof_stage.push_back(0);
+  }
+  return BK_OK;
+}
+
+int end_host(bk_ctx* c, void* stream) {
+  BK_CUDA(cudaEventRecord(c->t_end, c->s_comp));   // outside any graph: graph event nodes carry no timestamps
+  BK_CUDA(cudaEventRecord(c->ev_end, c->s_comp));
+  BK_CUDA(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_end, 0));
+  BK_CUDA(cudaStreamSynchronize(c->s_comp));
+  unsigned long long staged = 0;
+  BK_CUDA(cudaMemcpy(&staged, c->d_ctr + 0, 8, cudaMemcpyDeviceToHost));
+  c->st.bytes_padding = staged >= c->st.bytes_accessed ? staged - c->st.bytes_accessed : 0;
+  float ms = 0;
+  BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
+  c->st.ms_device = ms;
+  int rc = stage_stats(c);
+  if (rc) return rc;
+  return check_err(c);
+}
+
+// Runs `enqueue` (which issues one whole pipeline on the context's streams) ordered after `stream`.
+// ZC / DENSE pipelines are fully static for a given key, so the first run captures them as a
+// CUDA graph and later runs replay it (BK_FLAG_NO_GRAPH forces eager issue).
+
+void drop_graphs(bk_ctx* c) {
+  for (auto& g : c->graphs)
+    if (g.exec) cudaGraphExecDestroy(g.exec);
+  c->graphs.clear();
+}
+
+bool graphable(const Plan& p) { return p.mode == BK_GATHER_ZC || p.mode == BK_GATHER_DENSE; }
+
+
+// The caller's per-record output (partition records, k-means cid) is written by DMA: pin it once
+// and keep it pinned across runs (one cached registration per context).
+int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes) {
+  if (!bytes) return BK_OK;
+  for (auto& e : c->out_pinned)
+    if (e.first == ptr && e.second == bytes) return BK_OK;
+  if (is_pinned(ptr)) return BK_OK;
+  if (c->out_pinned.size() >= 4) {  // keep at most four cached registrations (oldest out)
+    cudaHostUnregister(c->out_pinned.front().first);
+    c->out_pinned.erase(c->out_pinned.begin());
+  }
+  BK_CUDA(cudaHostRegister(ptr, bytes, cudaHostRegisterPortable));
+  c->out_pinned.emplace_back(ptr, bytes);
+  return BK_OK;
+}
+
+void unregister(bk_ctx* c) {
+  if (c->pinned_data && c->host) cudaHostUnregister((void*)c->host);
+  if (c->pinned_off && c->off) cudaHostUnregister((void*)c->off);
+  c->pinned_data = c->pinned_off = c->registered = false;
+  c->host = nullptr;
+  c->off = nullptr;
+  c->host_dev = nullptr;
+  c->n = c->nbytes = 0;
+}
+
+
+}  // namespace rt
+}  // namespace bk
