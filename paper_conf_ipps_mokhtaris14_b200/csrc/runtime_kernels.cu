@@ -156,26 +156,25 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   const std::string key = "kmeans/" + std::to_string(K) + "/" + std::to_string(o->first_index) + "/" +
                           std::to_string((uintptr_t)o->cid) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
-  BK_CUDA(cudaMemcpyAsync(c->b_mu.p, c->h_mu, (uint64_t)K * 64, cudaMemcpyHostToDevice, c->s_comp));
-  BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
-  BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
-  size_t ci = 0;
-  int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
-    launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
-                  (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4,
-                  o->cid ? (int32_t*)s.out : nullptr, grid, cs);
-    c->n_launch += 1;
-    if (o->cid && ch.hi > ch.lo) {
-      cudaEvent_t e = c->ev_part[ci++ % c->ev_part.size()];
-      BK_CUDA(cudaEventRecord(e, cs));
-      BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
-      BK_CUDA(cudaMemcpyAsync(o->cid + ch.lo, s.out, (ch.hi - ch.lo) * 4, cudaMemcpyDeviceToHost, c->s_d2h));
-      c->st.bytes_d2h += (ch.hi - ch.lo) * 4;
-      rel = c->s_d2h;
-    }
-    return (int)BK_OK;
-  });
-  return r;
+    BK_CUDA(cudaMemcpyAsync(c->b_mu.p, c->h_mu, (uint64_t)K * 64, cudaMemcpyHostToDevice, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)K * 128, c->s_comp));
+    size_t ci = 0;
+    return pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
+      launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
+                    (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4,
+                    o->cid ? (int32_t*)s.out : nullptr, grid, cs);
+      c->n_launch += 1;
+      if (o->cid && ch.hi > ch.lo) {  // write-back of this chunk's cids, full duplex with the H2D stream
+        cudaEvent_t e = c->ev_part[ci++ % c->ev_part.size()];
+        BK_CUDA(cudaEventRecord(e, cs));
+        BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
+        BK_CUDA(cudaMemcpyAsync(o->cid + ch.lo, s.out, (ch.hi - ch.lo) * 4, cudaMemcpyDeviceToHost, c->s_d2h));
+        c->st.bytes_d2h += (ch.hi - ch.lo) * 4;
+        rel = c->s_d2h;
+      }
+      return (int)BK_OK;
+    });
   });
   if (rc) return rc;
   BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDeviceToHost));
@@ -261,22 +260,22 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
   if ((rc = ensure_out_pinned(c, o->out_records, c->n * 16))) return rc;
   const std::string key = "part/" + std::to_string(B) + "/" + std::to_string((uintptr_t)o->out_records) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
-  size_t ci = 0;
-  return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
-    launch_partition(ch, s.stage, s.lanes, s.tile_base, bits, (uint32_t*)c->b_hist.p, (uint32_t*)c->b_colpre.p,
-                     (unsigned long long*)c->b_totals.p + ci * B, (unsigned long long*)c->b_base.p, s.out, cs);
-    c->n_launch += 4;
-    cudaEvent_t e = c->ev_part[ci % c->ev_part.size()];
-    BK_CUDA(cudaEventRecord(e, cs));
-    BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
-    const uint64_t bytes = (ch.hi - ch.lo) * 16;
-    if (bytes)
-      BK_CUDA(cudaMemcpyAsync((uint8_t*)o->out_records + ch.lo * 16, s.out, bytes, cudaMemcpyDeviceToHost, c->s_d2h));
-    c->st.bytes_d2h += bytes;
-    rel = c->s_d2h;
-    ++ci;
-    return (int)BK_OK;
-  });
+    size_t ci = 0;
+    return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
+      launch_partition(ch, s.stage, s.lanes, s.tile_base, bits, (uint32_t*)c->b_hist.p, (uint32_t*)c->b_colpre.p,
+                       (unsigned long long*)c->b_totals.p + ci * B, (unsigned long long*)c->b_base.p, s.out, cs);
+      c->n_launch += 4;
+      cudaEvent_t e = c->ev_part[ci % c->ev_part.size()];
+      BK_CUDA(cudaEventRecord(e, cs));
+      BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
+      const uint64_t bytes = (ch.hi - ch.lo) * 16;
+      if (bytes)
+        BK_CUDA(cudaMemcpyAsync((uint8_t*)o->out_records + ch.lo * 16, s.out, bytes, cudaMemcpyDeviceToHost, c->s_d2h));
+      c->st.bytes_d2h += bytes;
+      rel = c->s_d2h;
+      ++ci;
+      return (int)BK_OK;
+    });
   });
   if (rc) return rc;
   std::vector<uint64_t> tot(C * B);
