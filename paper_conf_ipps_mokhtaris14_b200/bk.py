@@ -237,9 +237,17 @@ class Context:
     def stats(self) -> dict:
         return bk_get_stats(self.ctx)
 
-    def wordcount(self, cap: int = 1 << 20, table_slots: int = 0, stream=None):
+    def wordcount(self, cap: int = 1 << 20, table_slots: int = 0, stream=None, out=None):
+        """(word_off u64, word_len u32, word_count u64) of every distinct word; `out`: optional
+        preallocated (off, len, count) arrays of equal length (the cap), reused across calls."""
         o = _hdr(bk_out_wordcount, BK_K_WORDCOUNT)
-        off = np.empty(cap, np.uint64); ln = np.empty(cap, np.uint32); cnt = np.empty(cap, np.uint64)
+        if out is not None:
+            off, ln, cnt = out
+            assert off.dtype == np.uint64 and ln.dtype == np.uint32 and cnt.dtype == np.uint64
+            assert len(off) == len(ln) == len(cnt)
+            cap = len(off)
+        else:
+            off = np.empty(cap, np.uint64); ln = np.empty(cap, np.uint32); cnt = np.empty(cap, np.uint64)
         o.table_slots, o.cap, o.word_off, o.word_len, o.word_count = table_slots, cap, _ptr(off), _ptr(ln), _ptr(cnt)
         bk_run(self.ctx, BK_K_WORDCOUNT, stream, o)
         n = o.n_words

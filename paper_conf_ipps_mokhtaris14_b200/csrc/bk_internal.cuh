@@ -61,10 +61,12 @@ __host__ __device__ inline uint64_t mix64(uint64_t x) {
 // test-only: a one-thread kernel that spins `cycles` SM clocks (BK_FLAG_TEST_DELAYS)
 void launch_spin(long long cycles, cudaStream_t s);
 // Stage 1: lane plan + per-tile word counts, then tile bases (exclusive scan of 512*K_w).
-// staged_sum accumulates the staged bytes of every chunk (padding statistics).
+// staged_sum accumulates the staged bytes of every chunk (padding statistics). meta_src (whole
+// variable-length records only): the chunk's offsets in mapped host memory, read zero-copy and
+// copied into `meta` on the way (no separate offsets DMA); nullptr = `meta` is already filled.
 void launch_addrgen(const Chunk& c, const Access& a, const uint64_t* meta, LaneDesc* lanes,
                     uint32_t* tileK, uint64_t* tile_base, uint64_t stage_cap, int* err,
-                    unsigned long long* staged_sum, cudaStream_t s);
+                    unsigned long long* staged_sum, cudaStream_t s, const uint64_t* meta_src = nullptr);
 // Stage 2 (+3 when zero_copy: src is pinned, mapped host memory): gather the accessed bytes
 // into warp tiles. src points at byte c.base_byte of the data set, same alignment mod 16.
 void launch_gather(const Chunk& c, const Access& a, const uint8_t* src, const uint64_t* meta,

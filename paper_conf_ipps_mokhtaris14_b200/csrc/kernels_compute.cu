@@ -5,6 +5,8 @@
 // global memory (north_star: warp shuffles + block-level atomics).
 #include "bk_internal.cuh"
 
+#include <cstdlib>
+
 namespace bk {
 namespace {
 
@@ -22,8 +24,9 @@ __device__ __forceinline__ uint4 lane_word(const uint8_t* tile, uint32_t k, int 
 
 __device__ __forceinline__ bool is_delim(uint32_t ch) { return ch == 0x20 || (ch - 0x09u) <= 4u; }
 
-__device__ void wc_insert(WcEntry* table, uint64_t mask, unsigned long long key1, unsigned long long key2,
-                          unsigned long long offlen, unsigned long long cnt, unsigned long long* used, int* err) {
+__device__ __noinline__ void wc_insert(WcEntry* table, uint64_t mask, unsigned long long key1, unsigned long long key2,
+                                       unsigned long long offlen, unsigned long long cnt, unsigned long long* used,
+                                       int* err) {
   uint64_t slot = key1 & mask;
   for (uint64_t probe = 0; probe <= mask; ++probe, slot = (slot + 1) & mask) {
     WcEntry* e = &table[slot];
@@ -50,6 +53,12 @@ __device__ void wc_insert(WcEntry* table, uint64_t mask, unsigned long long key1
     }
   }
   atomicOr(err, kErrTableFull);
+}
+
+// The common case of a global update: the word is already at its home slot. One 16-B L2 read of
+// (key1, key2) and a fire-and-forget add; anything else takes the full probe/claim path.
+__device__ __forceinline__ bool wc_home_hit(const ulonglong2 home, unsigned long long key1, unsigned long long key2) {
+  return home.x == key1 && home.y == key2;
 }
 
 // Per-block shared-memory pre-aggregation (Zipf text: most occurrences hit a few hot words).
@@ -87,12 +96,15 @@ __device__ void tab_insert(WcShared& sh, WcEntry* table, uint64_t mask, unsigned
       }
     }
   }
-  wc_insert(table, mask, k1, k2, ol, cnt, used, err);  // block table crowded: go global
+  // block table crowded: go global
+  const ulonglong2 home = __ldcg(reinterpret_cast<const ulonglong2*>(&table[k1 & mask]));
+  if (wc_home_hit(home, k1, k2)) atomicAdd(&table[k1 & mask].count, (unsigned long long)cnt);
+  else wc_insert(table, mask, k1, k2, ol, cnt, used, err);
 }
 
 // Insert the warp's n queued words, 32 at a time: finalise the identity here (every lane busy),
 // merge duplicates within a round by match_any, insert into the block table.
-__device__ __forceinline__ void wc_flush_queue(WcShared& sh, int w, int lane, int n, WcEntry* table,
+__device__ __noinline__ void wc_flush_queue(WcShared& sh, int w, int lane, int n, WcEntry* table,
                                                uint64_t mask, unsigned long long* used, int* err) {
   __syncwarp();
   for (int base = 0; base < n; base += 32) {
@@ -111,13 +123,13 @@ __device__ __forceinline__ void wc_flush_queue(WcShared& sh, int w, int lane, in
   __syncwarp();
 }
 
-constexpr int kWcSub = 4;  // sub-threads per lane
 
 // kWcSub threads share one lane: sub-thread q owns the words that START in its quarter
 // [q*span, (q+1)*span) of the lane's bytes and finishes its last word past the quarter end
 // (classic parallel tokenisation; record boundaries from the offsets slice). Every 16-byte step
 // is branch-free across the warp: a word ending at a byte takes a queue slot from a ballot, and
 // its identity is finalised in the flush, so per-word work never rides on the per-byte path.
+template <int kWcSub>  // sub-threads per lane
 __global__ void __launch_bounds__(kWcBlock) k_wc(Chunk c, const uint8_t* __restrict__ stage,
                                                  const LaneDesc* __restrict__ lanes,
                                                  const uint64_t* __restrict__ tile_base,
@@ -226,8 +238,24 @@ __global__ void __launch_bounds__(kWcBlock) k_wc(Chunk c, const uint8_t* __restr
     if (qn) wc_flush_queue(sh, w, lane, qn, table, mask, used, err);
   }
   __syncthreads();
-  for (int i = threadIdx.x; i < kWcTab; i += blockDim.x)
-    if (sh.k1[i]) wc_insert(table, mask, sh.k1[i], sh.k2[i], sh.ol[i], sh.cnt[i], used, err);
+  // flush the block table: all of this thread's home-slot reads in flight at once, then adds
+  constexpr int kPer = kWcTab / kWcBlock;
+  unsigned long long k1[kPer], k2[kPer];
+  ulonglong2 home[kPer];
+#pragma unroll
+  for (int m = 0; m < kPer; ++m) {
+    const int i = threadIdx.x + m * kWcBlock;
+    k1[m] = sh.k1[i];
+    k2[m] = sh.k2[i];
+    home[m] = k1[m] ? __ldcg(reinterpret_cast<const ulonglong2*>(&table[k1[m] & mask])) : make_ulonglong2(0, 0);
+  }
+#pragma unroll
+  for (int m = 0; m < kPer; ++m) {
+    const int i = threadIdx.x + m * kWcBlock;
+    if (!k1[m]) continue;
+    if (wc_home_hit(home[m], k1[m], k2[m])) atomicAdd(&table[k1[m] & mask].count, (unsigned long long)sh.cnt[i]);
+    else wc_insert(table, mask, k1[m], k2[m], sh.ol[i], sh.cnt[i], used, err);
+  }
 }
 
 __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, unsigned long long* n_out,
@@ -522,9 +550,13 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
 void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                int* err, cudaStream_t s) {
-  const uint32_t threads = c.L * kWcSub;
-  k_wc<<<(threads + kWcBlock - 1) / kWcBlock, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table,
-                                                                mask, used, err);
+  static const int sub = getenv("BK_WC_SUB") ? atoi(getenv("BK_WC_SUB")) : 8;
+  const uint32_t threads = c.L * sub;
+  const uint32_t grid = (threads + kWcBlock - 1) / kWcBlock;
+  if (sub == 16) k_wc<16><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
+  else if (sub == 8) k_wc<8><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
+  else if (sub == 2) k_wc<2><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
+  else k_wc<4><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
 }
 
 void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,

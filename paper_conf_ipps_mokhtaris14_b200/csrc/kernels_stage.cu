@@ -13,6 +13,8 @@
 // kernel is also stage 3 (the transfer): it pulls the bytes over PCIe with 16-byte loads.
 #include "bk_internal.cuh"
 
+#include <algorithm>
+
 namespace bk {
 namespace {
 
@@ -48,18 +50,64 @@ __device__ __forceinline__ uint64_t lane_first(const Chunk& c, const Access& a, 
   return c.lo + k < c.hi ? c.lo + k : c.hi;
 }
 
+// Whole variable-length records: the same rule evaluated from the records' side, so no lane
+// needs a binary search (a chain of ~log2(n) dependent loads). With A_j = A(lo, lo+j),
+//   first(t) = lo+j  <=>  A_{j-1} < floor(t*A/L) <= A_j  <=>  ceil((A_{j-1}+1)L/A) <= t < ceil((A_j+1)L/A)
+// (j = 0: from t = 0). One thread per record boundary j in [0, n] writes lanes[t].first for its t
+// range. `src` holds off[lo..hi-1] (HBM, or the registered offsets read zero-copy, in which case
+// they are also copied to `meta_out` for the later stages).
+__global__ void __launch_bounds__(256) k_lane_first(Chunk c, const uint64_t* __restrict__ src,
+                                                    uint64_t* __restrict__ meta_out, LaneDesc* __restrict__ lanes) {
+  const uint64_t n = c.hi - c.lo;
+  const uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  const int lane = threadIdx.x & 31;
+  uint64_t Aj = 0;
+  if (j < n) {
+    const uint64_t o = __ldcs(src + j);
+    if (meta_out) meta_out[j] = o;
+    Aj = o - c.base_byte;
+  } else if (j == n) {
+    Aj = c.end_byte - c.base_byte;
+  }
+  uint64_t Ap = __shfl_up_sync(kFull, Aj, 1);
+  if (lane == 0 && j > 0 && j <= n) Ap = __ldcs(src + j - 1) - c.base_byte;
+  if (j > n) return;
+  const uint64_t A = c.accessed, L = c.L;
+  uint64_t t0, t1;
+  if (A == 0) {
+    t0 = 0;
+    t1 = j == 0 ? L : 0;
+  } else {
+    t0 = j == 0 ? 0 : ((Ap + 1) * L + A - 1) / A;
+    t1 = ((Aj + 1) * L + A - 1) / A;
+    if (t1 > L) t1 = L;
+  }
+  for (uint64_t t = t0; t < t1; ++t) lanes[t].first = c.lo + j;
+}
+
+template <bool kPre>  // kPre: lanes[].first already written by k_lane_first
 __global__ void __launch_bounds__(256) k_addrgen(Chunk c, Access a, const uint64_t* __restrict__ meta,
                                                  LaneDesc* __restrict__ lanes, uint32_t* __restrict__ tileK) {
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
   if (t >= c.L) return;  // L % 32 == 0: whole warps leave together
-  const uint64_t f0 = lane_first(c, a, meta, t);
-  const uint64_t f1 = lane_first(c, a, meta, t + 1);
+  uint64_t f0, f1;
+  if (kPre) {
+    f0 = lanes[t].first;
+    f1 = t + 1 < c.L ? lanes[t + 1].first : c.hi;
+  } else {
+    f0 = lane_first(c, a, meta, t);
+    f1 = lane_first(c, a, meta, t + 1);
+  }
   const uint64_t nb = acc_bytes(c, a, meta, f1) - acc_bytes(c, a, meta, f0);
-  LaneDesc d;
-  d.first = f0;
-  d.nrec = (uint32_t)(f1 - f0);
-  d.nbytes = (uint32_t)nb;
-  lanes[t] = d;
+  if (kPre) {  // leave .first alone: the neighbouring lane reads it
+    *reinterpret_cast<uint2*>(&lanes[t].nrec) = make_uint2((uint32_t)(f1 - f0), (uint32_t)nb);
+  } else {
+    LaneDesc d;
+    d.first = f0;
+    d.nrec = (uint32_t)(f1 - f0);
+    d.nbytes = (uint32_t)nb;
+    lanes[t] = d;
+  }
   const uint32_t K = __reduce_max_sync(kFull, (uint32_t)((nb + 15) >> 4));
   if ((t & 31) == 0) tileK[t >> 5] = K;
 }
@@ -177,13 +225,16 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
                                                       const uint64_t* __restrict__ meta,
                                                       const LaneDesc* __restrict__ lanes,
                                                       const uint64_t* __restrict__ tile_base,
-                                                      uint8_t* __restrict__ stage, uint64_t cap) {
+                                                      uint8_t* __restrict__ stage, uint64_t cap, uint32_t U) {
   if (tile_base[c.ntiles] > cap) return;  // stage-1 flagged an overflow: never write past the slot
   const uint8_t* glo = src - c.guard_lo;
   const uint8_t* ghi = src + c.guard_hi;
   const int lane = threadIdx.x & 31;
   const uint32_t nw_grid = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < c.ntiles; w += nw_grid) {
+  // U warps per tile: warp u streams the tile's 512-B blocks [u*NB/U, (u+1)*NB/U), so a chunk
+  // with few tiles still spreads its loads over every SM.
+  for (uint32_t vw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); vw < c.ntiles * U; vw += nw_grid) {
+    const uint32_t w = vw / U, u = vw % U;
     const LaneDesc d = lanes[(size_t)w * 32 + lane];
     const uint64_t rel = rec_off(c, a, meta, d.first) - c.base_byte;
     const uint64_t rel0 = __shfl_sync(kFull, rel, 0);
@@ -200,22 +251,28 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
     // kDepth 512-B warp loads in flight per warp (PCIe latency x bandwidth needs ~100 KB in
     // flight chip-wide; a chunk may have only a few hundred tiles)
     constexpr int kDepth = 4;
+    const uint32_t NB = (NW + 31) >> 5;
+    const uint32_t b0 = (uint32_t)((uint64_t)u * NB / U), b1 = (uint32_t)((uint64_t)(u + 1) * NB / U);
+    const uint32_t jend = min(NW, b1 * 32);  // words of this warp's range
     uint4 ring[kDepth];
 #pragma unroll
     for (int i = 0; i < kDepth; ++i) {
-      const uint32_t jj = i * 32 + lane;
-      ring[i] = jj < NW ? ld16b<kHost>(in + jj, glo, ghi) : make_uint4(0, 0, 0, 0);
+      const uint32_t jj = (b0 + i) * 32 + lane;
+      ring[i] = jj < jend ? ld16b<kHost>(in + jj, glo, ghi) : make_uint4(0, 0, 0, 0);
     }
-    for (uint32_t blk = 0; blk * 32 < NW; ++blk) {
+    // the word after the range: the high half of lane 31's shift window in the last block
+    const uint4 extra = (lane == 0 && b1 > b0 && b1 * 32 < NW) ? ld16b<kHost>(in + b1 * 32, glo, ghi)
+                                                              : make_uint4(0, 0, 0, 0);
+    for (uint32_t blk = b0; blk < b1; ++blk) {
       const uint4 cur = ring[0];
       uint4 hi = shfl_down_u4(cur, 1);
-      const uint4 n0 = shfl_u4(ring[1], 0);
+      const uint4 n0 = shfl_u4(blk + 1 < b1 ? ring[1] : extra, 0);
       if (lane == 31) hi = n0;
 #pragma unroll
       for (int i = 0; i + 1 < kDepth; ++i) ring[i] = ring[i + 1];
       {
         const uint32_t jn = (blk + kDepth) * 32 + lane;
-        ring[kDepth - 1] = jn < NW ? ld16b<kHost>(in + jn, glo, ghi) : make_uint4(0, 0, 0, 0);
+        ring[kDepth - 1] = jn < jend ? ld16b<kHost>(in + jn, glo, ghi) : make_uint4(0, 0, 0, 0);
       }
       const uint32_t j = blk * 32 + lane;
       // ta = last lane whose first word is <= j (sw is non-decreasing over lanes)
@@ -245,7 +302,7 @@ __global__ void __launch_bounds__(256) k_gather_whole(Chunk c, Access a, const u
         }
       }
     }
-    zero_holes(tile, K, W, lane);
+    if (u == 0) zero_holes(tile, K, W, lane);
   }
 }
 
@@ -360,8 +417,15 @@ void launch_spin(long long cycles, cudaStream_t s) { k_spin<<<1, 1, 0, s>>>(cycl
 
 void launch_addrgen(const Chunk& c, const Access& a, const uint64_t* meta, LaneDesc* lanes, uint32_t* tileK,
                     uint64_t* tile_base, uint64_t stage_cap, int* err, unsigned long long* staged_sum,
-                    cudaStream_t s) {
-  k_addrgen<<<(c.L + 255) / 256, 256, 0, s>>>(c, a, meta, lanes, tileK);
+                    cudaStream_t s, const uint64_t* meta_src) {
+  if (a.whole && a.rec_size == 0) {
+    const uint64_t nb = c.hi - c.lo + 1;
+    k_lane_first<<<(uint32_t)((nb + 255) / 256), 256, 0, s>>>(c, meta_src ? meta_src : meta,
+                                                               meta_src ? const_cast<uint64_t*>(meta) : nullptr, lanes);
+    k_addrgen<true><<<(c.L + 255) / 256, 256, 0, s>>>(c, a, meta, lanes, tileK);
+  } else {
+    k_addrgen<false><<<(c.L + 255) / 256, 256, 0, s>>>(c, a, meta, lanes, tileK);
+  }
   k_tile_scan<<<1, 1024, 0, s>>>(tileK, c.ntiles, tile_base, stage_cap, err, staged_sum);
 }
 
@@ -378,7 +442,11 @@ static void gather_impl(const Chunk& c, const Access& a, const uint8_t* src, con
   if (grid > grid_cap) grid = grid_cap;
   if (grid == 0) return;
   if (a.whole) {
-    k_gather_whole<kHost><<<grid, 256, 0, s>>>(c, a, src, meta, lanes, tile_base, stage, cap);
+    // split tiles over up to 8 warps until the chunk fills the grid cap's warps
+    const uint32_t U = (uint32_t)std::min<uint64_t>(8, std::max<uint64_t>(1, (8ull * grid_cap + warps - 1) / warps));
+    uint64_t g2 = ((uint64_t)warps * U + 7) / 8;
+    k_gather_whole<kHost><<<(uint32_t)std::min<uint64_t>(g2, grid_cap), 256, 0, s>>>(c, a, src, meta, lanes,
+                                                                                       tile_base, stage, cap, U);
     return;
   }
   const bool fast = a.n_ext == 1 && (a.E & 15) == 0 && a.E > 0;

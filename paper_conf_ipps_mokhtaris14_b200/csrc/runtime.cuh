@@ -58,6 +58,13 @@ struct Slot {
   uint32_t* tileK = nullptr;
   uint64_t* tile_base = nullptr;
   uint8_t* out = nullptr;       // per-chunk output (partition: the bucket-sorted chunk)
+  // descriptor sets (meta, lanes, tileK, tile_base); ZC plans keep two so that stage 1 of chunk
+  // i+N can run while chunk i still computes from the other set. meta..tile_base above point at
+  // the set of the chunk being issued.
+  uint64_t* meta_set[2] = {nullptr, nullptr};
+  LaneDesc* lanes_set[2] = {nullptr, nullptr};
+  uint32_t* tileK_set[2] = {nullptr, nullptr};
+  uint64_t* tile_base_set[2] = {nullptr, nullptr};
   cudaEvent_t copied = nullptr, ready = nullptr, freed = nullptr;
   bool used = false;
 };
@@ -92,6 +99,7 @@ struct Plan {
   uint32_t L = 0;
   uint64_t max_acc_rec = 0;            // max accessed bytes of one record
   uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
+  uint32_t desc_sets = 1;              // descriptor sets per slot (2: ZC, stage 1 runs a chunk ahead)
   std::vector<uint64_t> bounds;        // chunk record bounds
   std::string key;                     // plan-cache key (also part of the graph key)
 };
@@ -114,6 +122,7 @@ struct bk_ctx {  // the opaque context of include/bk.h
   bk_config cfg{};
   cudaStream_t s_copy = nullptr, s_asm = nullptr, s_comp = nullptr;
   std::vector<cudaStream_t> s_slot;  // per-slot compute streams for commutative kernels
+  std::vector<cudaStream_t> s_stage; // per-slot zero-copy staging streams (stages 1-3 of slot k's chunks)
   cudaEvent_t ev_begin = nullptr, ev_end = nullptr;
   cudaEvent_t t_begin = nullptr, t_end = nullptr;   // timing events on s_comp (device time of a run)
   std::vector<cudaEvent_t> prof;                   // BK_FLAG_PROFILE: per chunk x stage begin/end
@@ -128,10 +137,13 @@ struct bk_ctx {  // the opaque context of include/bk.h
   uint64_t n = 0;
   bool pinned_data = false, pinned_off = false, registered = false;
   const uint8_t* host_dev = nullptr;   // device alias of the mapped data set
+  const uint64_t* off_dev = nullptr;   // device alias of the mapped offsets (nullptr: not mapped)
   uint64_t max_rec = 0, min_rec = 0;
   // device scratch / resident buffers
   int* d_err = nullptr;
   unsigned long long* d_ctr = nullptr;  // [0] staged sum, [1] wc used, [2] wc n_out, [3] grep running, [4] kmeans chk
+  // pinned mirror of d_ctr[0..7] and d_err (at [8]), copied by the run's tail before its one sync
+  unsigned long long* h_ctr = nullptr;
   bk::rt::DevBuf b_table, b_out1, b_out2, b_out3, b_blk, b_blk2, b_agg1, b_agg2, b_agg3, b_mu;
   // CPU assembly (BK_GATHER_CPU / HYBRID): thread pool + pinned host staging ring
   bk::HostPool* pool = nullptr;

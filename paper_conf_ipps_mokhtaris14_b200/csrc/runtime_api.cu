@@ -79,13 +79,15 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
   }
   if (cudaMalloc(&c->d_err, 256) != cudaSuccess || cudaMalloc(&c->d_ctr, 8 * sizeof(unsigned long long)) != cudaSuccess)
     return cleanup(fail(BK_E_NOMEM, "cudaMalloc scratch"));
+  if (cudaHostAlloc(&c->h_ctr, 9 * sizeof(unsigned long long), cudaHostAllocDefault) != cudaSuccess)
+    return cleanup(fail(BK_E_NOMEM, "cudaHostAlloc counters"));
   c->slots.resize(c->cfg.n_slots);
   if (cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "d2h stream"));
   if (configure_partition_kernels() != cudaSuccess || configure_baseline_kernels() != cudaSuccess)
     return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
   if (cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess)
     return cleanup(fail(BK_E_CUDA, "events"));
-  c->ev_join.assign(3 + c->cfg.n_slots, nullptr);
+  c->ev_join.assign(3 + 2 * c->cfg.n_slots, nullptr);
   for (auto& e : c->ev_join)
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
   c->ev_part.assign(c->cfg.n_slots, nullptr);
@@ -93,6 +95,9 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "events"));
   c->s_slot.assign(c->cfg.n_slots, nullptr);
   for (auto& st : c->s_slot)
+    if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "slot streams"));
+  c->s_stage.assign(c->cfg.n_slots, nullptr);
+  for (auto& st : c->s_stage)
     if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "slot streams"));
   for (auto& s : c->slots) {
     if (cudaEventCreateWithFlags(&s.copied, cudaEventDisableTiming) != cudaSuccess ||
@@ -160,6 +165,9 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
       if (e != cudaSuccess) return fail(BK_E_CUDA, "cudaHostRegister(offsets): %s", cudaGetErrorString(e));
       c->pinned_off = true;
     }
+    void* odev = nullptr;  // caller-pinned offsets may be unmapped: then stage 1 DMAs them instead
+    c->off_dev = cudaHostGetDevicePointer(&odev, (void*)off, 0) == cudaSuccess ? (const uint64_t*)odev : nullptr;
+    cudaGetLastError();
   }
   c->host = (const uint8_t*)host_ptr;
   c->nbytes = nbytes;
@@ -232,6 +240,7 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
     cudaStreamSynchronize(c->s_asm);
     cudaStreamSynchronize(c->s_comp);
     for (auto st : c->s_slot) cudaStreamSynchronize(st);
+    for (auto st : c->s_stage) cudaStreamSynchronize(st);
     cudaGetLastError();
     return rc;
   }
@@ -264,6 +273,8 @@ int bk_destroy(bk_ctx* c) {
   if (c->s_asm) cudaStreamSynchronize(c->s_asm);
   for (auto st : c->s_slot)
     if (st) cudaStreamSynchronize(st);
+  for (auto st : c->s_stage)
+    if (st) cudaStreamSynchronize(st);
   unregister(c);
   for (auto& s : c->slots) {
     if (s.copied) cudaEventDestroy(s.copied);
@@ -276,6 +287,7 @@ int bk_destroy(bk_ctx* c) {
   if (c->window) cudaFree(c->window);
   if (c->d_err) cudaFree(c->d_err);
   if (c->d_ctr) cudaFree(c->d_ctr);
+  if (c->h_ctr) cudaFreeHost(c->h_ctr);
   if (c->ev_begin) cudaEventDestroy(c->ev_begin);
   if (c->ev_end) cudaEventDestroy(c->ev_end);
   if (c->t_begin) cudaEventDestroy(c->t_begin);
@@ -299,6 +311,8 @@ int bk_destroy(bk_ctx* c) {
   if (c->s_asm) cudaStreamDestroy(c->s_asm);
   if (c->s_comp) cudaStreamDestroy(c->s_comp);
   for (auto st : c->s_slot)
+    if (st) cudaStreamDestroy(st);
+  for (auto st : c->s_stage)
     if (st) cudaStreamDestroy(st);
   cudaGetLastError();
   delete c;

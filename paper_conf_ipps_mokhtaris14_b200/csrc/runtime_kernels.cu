@@ -39,7 +39,7 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   });
   if (rc) return rc;
   unsigned long long nw = 0;
-  BK_CUDA(cudaMemcpy(&nw, c->d_ctr + 2, 8, cudaMemcpyDeviceToHost));
+  nw = c->h_ctr[2];
   o->n_words = nw;
   if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
   if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
@@ -87,7 +87,7 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
   });
   if (rc) return rc;
   unsigned long long m = 0;
-  BK_CUDA(cudaMemcpy(&m, c->d_ctr + 3, 8, cudaMemcpyDeviceToHost));
+  m = c->h_ctr[3];
   o->n_match = m;
   if (m > o->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)o->cap);
   if (m) BK_CUDA(cudaMemcpy(o->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));
@@ -180,7 +180,7 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDeviceToHost));
   BK_CUDA(cudaMemcpy(o->sum, c->b_agg3.p, (uint64_t)K * 128, cudaMemcpyDeviceToHost));
   unsigned long long chk = 0;
-  BK_CUDA(cudaMemcpy(&chk, c->d_ctr + 4, 8, cudaMemcpyDeviceToHost));
+  chk = c->h_ctr[4];
   o->chk = chk;
   c->st.bytes_d2h += (uint64_t)K * 136;
   return BK_OK;
@@ -219,8 +219,8 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   });
   if (rc) return rc;
   unsigned long long nk = 0, tot = 0;
-  BK_CUDA(cudaMemcpy(&nk, c->d_ctr + 2, 8, cudaMemcpyDeviceToHost));
-  BK_CUDA(cudaMemcpy(&tot, c->d_ctr + 5, 8, cudaMemcpyDeviceToHost));
+  nk = c->h_ctr[2];
+  tot = c->h_ctr[5];
   o->n_kmers = nk;
   o->total = tot;
   if (nk > o->cap) return fail(BK_E_CAPACITY, "%llu distinct k-mers > cap %llu", nk, (unsigned long long)o->cap);
@@ -388,7 +388,7 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
   if ((rc = end_run(c, stream))) return rc;
   if (kid == BK_K_GREP) {
     unsigned long long m = 0;
-    BK_CUDA(cudaMemcpy(&m, c->d_ctr + 3, 8, cudaMemcpyDeviceToHost));
+    m = c->h_ctr[3];
     og->n_match = m;
     if (m > og->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)og->cap);
     if (m) BK_CUDA(cudaMemcpy(og->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));

@@ -98,31 +98,51 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   Access a = p.a;
   a.rec_size = c->off ? 0 : c->cfg.record_size;
   if (p.zero_copy) {
-    // Stage 1 on s_asm (offsets slice by DMA + lane plan) runs ahead, overlapping the previous
-    // chunk's zero-copy gather on s_copy; the gather waits only for its own plan.
-    if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_asm, s.freed, 0));
-    BK_DELAY(c->s_asm);
-    BK_PROF(kStH2D, c->s_asm, true);
+    // ZC mode: stages 1-3 of slot k's chunks on slot k's own staging stream, so consecutive
+    // chunks' zero-copy gathers overlap (one gather's ramp-up and tail hide under the next one's
+    // transfer). HYBRID: stage 1 on s_asm runs ahead, and the gathers share s_copy with the DMAs
+    // of CPU-assembled chunks so chunks become ready in order (grep's compute is ordered).
+    const bool per_slot = p.mode != BK_GATHER_HYBRID;
+    cudaStream_t s1 = per_slot ? c->s_stage[i % c->cfg.n_slots] : c->s_asm;
+    cudaStream_t ss = per_slot ? s1 : c->s_copy;
+    // two descriptor sets: stage 1 of this chunk writes the set chunk i-2N used, whose compute
+    // ended before chunk i-N's gather started (that gather waited for it, earlier on this stream)
+    const int set = p.desc_sets == 2 ? (int)((i / c->cfg.n_slots) & 1) : 0;
+    s.meta = s.meta_set[set];
+    s.lanes = s.lanes_set[set];
+    s.tileK = s.tileK_set[set];
+    s.tile_base = s.tile_base_set[set];
+    const bool early = per_slot && p.desc_sets == 2;   // stage 1 need not wait for the slot
+    if (s.used && !early) BK_CUDA(cudaStreamWaitEvent(s1, s.freed, 0));
+    BK_DELAY(s1);
+    // whole variable-length records: stage 1 reads the offsets zero-copy itself (no DMA in the chain)
+    const bool meta_zc = a.whole && c->off && c->off_dev;
+    BK_PROF(kStH2D, s1, true);
     if (c->off && ch.hi > ch.lo) {
-      BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, c->s_asm));
+      if (!meta_zc)
+        BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, s1));
       c->st.bytes_meta += (ch.hi - ch.lo) * 8;
     }
-    BK_PROF(kStH2D, c->s_asm, false);
-    BK_PROF(kStAddrgen, c->s_asm, true);
-    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_asm);
-    BK_PROF(kStAddrgen, c->s_asm, false);
-    BK_CUDA(cudaEventRecord(s.copied, c->s_asm));
-    BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.copied, 0));
-    BK_DELAY(c->s_copy);
-    BK_PROF(kStGather, c->s_copy, true);
+    BK_PROF(kStH2D, s1, false);
+    BK_PROF(kStAddrgen, s1, true);
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, s1,
+                   meta_zc ? c->off_dev + ch.lo : nullptr);
+    BK_PROF(kStAddrgen, s1, false);
+    if (!per_slot) {
+      BK_CUDA(cudaEventRecord(s.copied, s1));
+      BK_CUDA(cudaStreamWaitEvent(ss, s.copied, 0));
+    }
+    if (s.used && early) BK_CUDA(cudaStreamWaitEvent(ss, s.freed, 0));   // the stage buffer
+    BK_DELAY(ss);
+    BK_PROF(kStGather, ss, true);
     Chunk gch = ch;   // readable source: the registered data set
     gch.guard_lo = ch.base_byte;
     gch.guard_hi = c->nbytes - ch.base_byte;
-    launch_gather(gch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1,
-                  c->s_copy);
-    BK_PROF(kStGather, c->s_copy, false);
+    launch_gather(gch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1, ss);
+    BK_PROF(kStGather, ss, false);
     c->n_launch += 3;
     c->st.bytes_h2d += ch.accessed;
+    BK_CUDA(cudaEventRecord(s.ready, ss));
   } else {
     if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
     BK_DELAY(c->s_copy);
@@ -151,7 +171,7 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     c->st.bytes_h2d += bytes;
   }
   c->st.bytes_accessed += ch.accessed;
-  BK_CUDA(cudaEventRecord(s.ready, p.zero_copy ? c->s_copy : c->s_asm));
+  if (!p.zero_copy) BK_CUDA(cudaEventRecord(s.ready, c->s_asm));
   s.used = true;
   return BK_OK;
 }
@@ -162,9 +182,8 @@ void note_plan(bk_ctx* c, const Plan& p) {
   c->st.lanes = p.L;
 }
 
-int check_err(bk_ctx* c) {
-  int herr = 0;
-  BK_CUDA(cudaMemcpy(&herr, c->d_err, sizeof(int), cudaMemcpyDeviceToHost));
+int check_err(bk_ctx* c) {  // after end_host: the error bits arrived with the run's tail copy
+  const int herr = (int)(uint32_t)c->h_ctr[8];
   if (herr & kErrStageOverflow) return fail(BK_E_RANGE, "staged chunk exceeded its slot (internal bound violated)");
   if (herr & kErrKeyRange) return fail(BK_E_INVAL, "a group-by key is >= G");
   if (herr & kErrTableFull) return fail(BK_E_CAPACITY, "word-count hash table full; raise table_slots");
@@ -242,26 +261,13 @@ int stage_stats(bk_ctx* c) {
   return BK_OK;
 }
 
-int end_run(bk_ctx* c, void* stream) {
-  BK_CUDA(cudaEventRecord(c->t_end, c->s_comp));
-  BK_CUDA(cudaEventRecord(c->ev_end, c->s_comp));
-  BK_CUDA(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_end, 0));
-  BK_CUDA(cudaStreamSynchronize(c->s_comp));
-  unsigned long long staged = 0;
-  BK_CUDA(cudaMemcpy(&staged, c->d_ctr + 0, 8, cudaMemcpyDeviceToHost));
-  c->st.bytes_padding = staged >= c->st.bytes_accessed ? staged - c->st.bytes_accessed : 0;
-  float ms = 0;
-  BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
-  c->st.ms_device = ms;
-  int rc = stage_stats(c);
-  if (rc) return rc;
-  return check_err(c);
-}
+int end_run(bk_ctx* c, void* stream) { return end_host(c, stream); }
 
 // ---- run_device: fork/join all streams around a pipeline; capture it as a CUDA graph once per key
 std::vector<cudaStream_t> side_streams(bk_ctx* c) {
   std::vector<cudaStream_t> v{c->s_copy, c->s_asm, c->s_d2h};
   for (auto st : c->s_slot) v.push_back(st);
+  for (auto st : c->s_stage) v.push_back(st);
   return v;
 }
 
@@ -303,12 +309,15 @@ int prof_reserve(bk_ctx* c, size_t pairs) {
 }
 
 int end_host(bk_ctx* c, void* stream) {
+  // the run's tail: counters + error bits into pinned memory, then ONE host sync per run
+  c->h_ctr[8] = 0;
+  BK_CUDA(cudaMemcpyAsync(c->h_ctr, c->d_ctr, 8 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->s_comp));
+  BK_CUDA(cudaMemcpyAsync(c->h_ctr + 8, c->d_err, sizeof(int), cudaMemcpyDeviceToHost, c->s_comp));
   BK_CUDA(cudaEventRecord(c->t_end, c->s_comp));   // outside any graph: graph event nodes carry no timestamps
   BK_CUDA(cudaEventRecord(c->ev_end, c->s_comp));
   BK_CUDA(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_end, 0));
   BK_CUDA(cudaStreamSynchronize(c->s_comp));
-  unsigned long long staged = 0;
-  BK_CUDA(cudaMemcpy(&staged, c->d_ctr + 0, 8, cudaMemcpyDeviceToHost));
+  const unsigned long long staged = c->h_ctr[0];
   c->st.bytes_padding = staged >= c->st.bytes_accessed ? staged - c->st.bytes_accessed : 0;
   float ms = 0;
   BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
@@ -354,6 +363,7 @@ void unregister(bk_ctx* c) {
   c->host = nullptr;
   c->off = nullptr;
   c->host_dev = nullptr;
+  c->off_dev = nullptr;
   c->n = c->nbytes = 0;
 }
 

@@ -59,9 +59,9 @@ int make_chunks(const bk_ctx* c, Plan& p) {
 // Bytes one slot needs for a plan: raw + stage + meta + lanes + tiles (+ alignment).
 uint64_t slot_need(const Plan& p) {
   const uint64_t ntiles = p.L / 32;
-  return align_up(p.raw_cap, kAlign) + align_up(p.stage_cap, kAlign) + align_up(p.meta_cap * 8, kAlign) +
-         align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign) + align_up(ntiles * 4, kAlign) +
-         align_up((ntiles + 1) * 8, kAlign) + align_up(p.out_cap, kAlign);
+  const uint64_t desc = align_up(p.meta_cap * 8, kAlign) + align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign) +
+                        align_up(ntiles * 4, kAlign) + align_up((ntiles + 1) * 8, kAlign);
+  return align_up(p.raw_cap, kAlign) + align_up(p.stage_cap, kAlign) + p.desc_sets * desc + align_up(p.out_cap, kAlign);
 }
 
 void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) {
@@ -121,6 +121,7 @@ int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p,
     return fail(BK_E_INVAL, "bad gather_mode %d", mode);
   p.mode = mode;
   p.zero_copy = mode != BK_GATHER_DENSE;
+  p.desc_sets = mode == BK_GATHER_ZC ? 2 : 1;
   p.max_acc_rec = a.whole ? c->max_rec : a.E;
   const uint64_t slot = c->cfg.window_bytes / c->cfg.n_slots;
   // total plan bytes
@@ -177,14 +178,27 @@ void carve(bk_ctx* c, const Plan& p) {
     q += align_up(p.raw_cap, kAlign);
     s.stage = q;
     q += align_up(p.stage_cap, kAlign);
-    s.meta = reinterpret_cast<uint64_t*>(q);
-    q += align_up(p.meta_cap * 8, kAlign);
-    s.lanes = reinterpret_cast<LaneDesc*>(q);
-    q += align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign);
-    s.tileK = reinterpret_cast<uint32_t*>(q);
-    q += align_up(ntiles * 4, kAlign);
-    s.tile_base = reinterpret_cast<uint64_t*>(q);
-    q += align_up((ntiles + 1) * 8, kAlign);
+    for (uint32_t d = 0; d < 2; ++d) {
+      if (d == 1 && p.desc_sets < 2) {
+        s.meta_set[1] = s.meta_set[0];
+        s.lanes_set[1] = s.lanes_set[0];
+        s.tileK_set[1] = s.tileK_set[0];
+        s.tile_base_set[1] = s.tile_base_set[0];
+        break;
+      }
+      s.meta_set[d] = reinterpret_cast<uint64_t*>(q);
+      q += align_up(p.meta_cap * 8, kAlign);
+      s.lanes_set[d] = reinterpret_cast<LaneDesc*>(q);
+      q += align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign);
+      s.tileK_set[d] = reinterpret_cast<uint32_t*>(q);
+      q += align_up(ntiles * 4, kAlign);
+      s.tile_base_set[d] = reinterpret_cast<uint64_t*>(q);
+      q += align_up((ntiles + 1) * 8, kAlign);
+    }
+    s.meta = s.meta_set[0];
+    s.lanes = s.lanes_set[0];
+    s.tileK = s.tileK_set[0];
+    s.tile_base = s.tile_base_set[0];
     s.out = p.out_cap ? q : nullptr;
     s.used = false;
   }
