@@ -64,7 +64,10 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-dbuf", action="store_true", help="skip the double-buffering baseline measurement")
     ap.add_argument("--no-profile", action="store_true", help="disable per-stage event timing")
-    return ap.parse_args()
+    args = ap.parse_args()
+    if args.slots == 0 and args.workload == "wordcount":
+        args.slots = 8   # the 8 MiB window: more, smaller chunks in flight (profiles/r01_wc_sweep.md)
+    return args
 
 
 # ------------------------------------------------------------------------------ workloads
@@ -120,45 +123,57 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
 
 # ------------------------------------------------------------------------------ helpers
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """SM clocks + throttle reasons sampled every 10 ms through NVML while the timed region runs
+    (the nvidia-smi query of the profiling recipe, without its ~100 ms start-up, so that short
+    regions are sampled too); one sample is taken on entry and one on exit of the region."""
 
-    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4))
 
     def __init__(self, dev: int):
-        self.dev, self.rows, self.proc = dev, [], None
+        self.dev, self.rows, self.h, self.stop = dev, [], None, threading.Event()
+
+    def _sample(self):
+        import pynvml
+        sm = pynvml.nvmlDeviceGetClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        mx = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        self.rows.append((sm, mx, rs))
+
+    def _loop(self):
+        while not self.stop.wait(0.01):
+            self._sample()
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                                          "-i", str(self.dev), "-lms", "200"], stdout=subprocess.PIPE,
-                                         stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
+            import pynvml
+            pynvml.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES", "")
+            ids = [x for x in vis.split(",") if x.strip()]
+            idx = int(ids[self.dev]) if ids and ids[self.dev].strip().isdigit() else self.dev
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self._sample()
+            self.t = threading.Thread(target=self._loop, daemon=True)
             self.t.start()
-        except OSError:
-            self.proc = None
+        except Exception:
+            self.h = None
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            parts = [p.strip() for p in line.split(",")]
-            if len(parts) == 6:
-                self.rows.append(parts)
-
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            self.proc.wait(timeout=5)
+        if self.h is not None:
+            self.stop.set()
+            self.t.join(timeout=5)
+            try:
+                self._sample()
+            except Exception:
+                pass
 
     def summary(self):
         if not self.rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
-        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[2 + i].lower() == "active"})
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+        reasons = sorted({n for r in self.rows for n, bit in self.REASONS if r[2] & bit})
+        return {"sm_mhz": statistics.median(r[0] for r in self.rows), "sm_max_mhz": max(r[1] for r in self.rows),
+                "reasons": reasons, "samples": len(self.rows), "how": "NVML every 10 ms during the timed steps"}
 
 
 def measure_h2d_peak(torch, dev) -> float:
@@ -438,6 +453,7 @@ def main():
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded counter RNG, gen/)",
         "config": {"workload": args.workload, "desc": WORKLOADS[args.workload][2],
                    "bytes_per_gpu": nbytes, "records_per_gpu": shard["n"], "window_bytes": window,
+                   "n_slots": st["n_slots"],
                    "gather_mode": {1: "zc", 2: "cpu", 3: "dense", 4: "hybrid"}.get(st["gather_mode"], "?"),
                    "chunks_cpu_assembled": st["n_chunks_cpu"], "n_chunks": st["n_chunks"],
                    "lanes_per_chunk": st["lanes"], "chunk_budget_bytes": st["chunk_budget"],

@@ -5,8 +5,6 @@
 // global memory (north_star: warp shuffles + block-level atomics).
 #include "bk_internal.cuh"
 
-#include <cstdlib>
-
 namespace bk {
 namespace {
 
@@ -550,13 +548,9 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
 void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                int* err, cudaStream_t s) {
-  static const int sub = getenv("BK_WC_SUB") ? atoi(getenv("BK_WC_SUB")) : 8;
-  const uint32_t threads = c.L * sub;
-  const uint32_t grid = (threads + kWcBlock - 1) / kWcBlock;
-  if (sub == 16) k_wc<16><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
-  else if (sub == 8) k_wc<8><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
-  else if (sub == 2) k_wc<2><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
-  else k_wc<4><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
+  constexpr int kSub = 8;  // sub-threads per 256-B lane (sweep: 2/4/8/16, profiles/r01_wc_sweep.md)
+  const uint32_t grid = (c.L * kSub + kWcBlock - 1) / kWcBlock;
+  k_wc<kSub><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
 }
 
 void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,
