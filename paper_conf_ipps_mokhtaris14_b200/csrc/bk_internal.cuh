@@ -92,10 +92,15 @@ struct GrepParams {
   uint64_t first_index;
   uint64_t cap;
 };
-// three launches: block counts, one-block scan (+ running base), ordered write
+// three launches per chunk: block counts, one-block scan (reserves the chunk's run [base, base+n)
+// of the match pool with atomicAdd on *cursor, writes chunk_run = {base, n}), ordered write into
+// the pool. Chunks may run concurrently; launch_grep_order then lays the runs out in chunk order.
 void launch_grep(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
-                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* running,
-                 unsigned long long* blkbase, uint64_t* out_idx, int* err, cudaStream_t s);
+                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* cursor,
+                 unsigned long long* blkbase, unsigned long long* chunk_run, uint64_t* out_idx, int* err,
+                 cudaStream_t s);
+void launch_grep_order(const unsigned long long* runs, uint32_t C, const uint64_t* pool, uint64_t* out, uint64_t cap,
+                       cudaStream_t s);
 
 size_t groupby_smem(uint32_t G);
 void launch_groupby(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,

@@ -273,7 +273,10 @@ __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, 
 // ------------------------------------------------------------------------------------------
 // C2 grep (MCA analogue): key = first strnlen(32) bytes of the record's 32-byte key
 // field (staged as words 2j, 2j+1 of the lane); match iff the pattern is a substring. Output
-// indices are ascending: per chunk, block counts -> one-block scan (+ running base) -> write.
+// indices are ascending. Chunks compute in any order (per-slot streams): per chunk, block counts ->
+// one-block scan that reserves the chunk's run in a match pool with one atomicAdd and records
+// (pool offset, count) per chunk -> write; after the last chunk one pass copies the runs into
+// chunk order (k_grep_order).
 
 struct Key32 { uint64_t q[8]; };  // q[4..7] = 0: windows past byte 31 read zeros
 
@@ -365,11 +368,24 @@ __global__ void __launch_bounds__(256) k_grep_count(Chunk c, const uint8_t* __re
 }
 
 __global__ void __launch_bounds__(1024) k_grep_scan(uint32_t* __restrict__ blkcnt, uint32_t nblk,
-                                                    unsigned long long* running, unsigned long long* blkbase) {
+                                                    unsigned long long* cursor, unsigned long long* blkbase,
+                                                    unsigned long long* chunk_run) {
   __shared__ unsigned long long warp_sums[32];
   __shared__ unsigned long long carry;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  if (threadIdx.x == 0) carry = *running;
+  // the chunk's match count, then its run in the pool: [base, base + total)
+  unsigned long long part = 0;
+  for (uint32_t i = threadIdx.x; i < nblk; i += 1024) part += blkcnt[i];
+  part = __reduce_add_sync(kFull, (unsigned)part);
+  if (lane == 0) warp_sums[wid] = part;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long tot = 0;
+    for (int w = 0; w < 32; ++w) tot += warp_sums[w];
+    carry = atomicAdd(cursor, tot);
+    chunk_run[0] = carry;
+    chunk_run[1] = tot;
+  }
   __syncthreads();
   for (uint32_t base = 0; base < nblk; base += 1024) {
     const uint32_t i = base + threadIdx.x;
@@ -398,7 +414,31 @@ __global__ void __launch_bounds__(1024) k_grep_scan(uint32_t* __restrict__ blkcn
     if (threadIdx.x == 1023) carry = excl + v;
     __syncthreads();
   }
-  if (threadIdx.x == 0) *running = carry;
+}
+
+// Block c copies chunk c's run of the pool to its place in chunk order (the sum of the runs of
+// chunks 0..c-1), clipped to cap (overflow was already flagged by k_grep_write).
+__global__ void __launch_bounds__(256) k_grep_order(const unsigned long long* __restrict__ runs, uint32_t C,
+                                                    const uint64_t* __restrict__ pool, uint64_t* __restrict__ out,
+                                                    uint64_t cap) {
+  __shared__ unsigned long long sh[8];
+  __shared__ unsigned long long s_dst;
+  const uint32_t c = blockIdx.x;
+  unsigned long long before = 0;
+  for (uint32_t i = threadIdx.x; i < c; i += blockDim.x) before += runs[2 * i + 1];
+#pragma unroll
+  for (int o = 16; o; o >>= 1) before += __shfl_down_sync(kFull, before, o);
+  if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = before;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += sh[w];
+    s_dst = t;
+  }
+  __syncthreads();
+  const unsigned long long dst = s_dst, src = runs[2 * c], n = runs[2 * c + 1];
+  for (unsigned long long k = threadIdx.x; k < n; k += blockDim.x)
+    if (dst + k < cap && src + k < cap) out[dst + k] = pool[src + k];
 }
 
 __global__ void __launch_bounds__(256) k_grep_write(Chunk c, const uint8_t* __restrict__ stage,
@@ -559,12 +599,17 @@ void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long*
 }
 
 void launch_grep(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
-                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* running, unsigned long long* blkbase,
-                 uint64_t* out_idx, int* err, cudaStream_t s) {
+                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* cursor, unsigned long long* blkbase,
+                 unsigned long long* chunk_run, uint64_t* out_idx, int* err, cudaStream_t s) {
   const uint32_t nblk = (c.L + 255) / 256;
   k_grep_count<<<nblk, 256, 0, s>>>(c, stage, lanes, tile_base, p, blkcnt);
-  k_grep_scan<<<1, 1024, 0, s>>>(blkcnt, nblk, running, blkbase);
+  k_grep_scan<<<1, 1024, 0, s>>>(blkcnt, nblk, cursor, blkbase, chunk_run);
   k_grep_write<<<nblk, 256, 0, s>>>(c, stage, lanes, tile_base, p, blkbase, out_idx, err);
+}
+
+void launch_grep_order(const unsigned long long* runs, uint32_t C, const uint64_t* pool, uint64_t* out, uint64_t cap,
+                       cudaStream_t s) {
+  if (C) k_grep_order<<<C, 256, 0, s>>>(runs, C, pool, out, cap);
 }
 
 size_t groupby_smem(uint32_t G) { return (size_t)G * 16; }

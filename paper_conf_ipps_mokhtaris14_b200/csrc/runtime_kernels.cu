@@ -66,9 +66,13 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
   carve(c, p);
   const uint32_t nblk = (p.L + 255) / 256;
   const uint64_t cap = std::min<uint64_t>(o->cap, c->n);
-  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(cap, 1) * 8));
-  BK_CUDA(c->b_blk.ensure((uint64_t)nblk * 4));
-  BK_CUDA(c->b_blk2.ensure((uint64_t)nblk * 8));
+  const size_t C = p.bounds.size() - 1;
+  const uint32_t N = c->cfg.n_slots;
+  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(cap, 1) * 8));   // matches in chunk order
+  BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(cap, 1) * 8));   // match pool (runs in completion order)
+  BK_CUDA(c->b_out3.ensure(std::max<size_t>(C, 1) * 16));       // per chunk {pool offset, count}
+  BK_CUDA(c->b_blk.ensure((uint64_t)nblk * 4 * N));             // per slot: block counts
+  BK_CUDA(c->b_blk2.ensure((uint64_t)nblk * 8 * N));            // per slot: block bases
   GrepParams gp{};
   if (o->pattern_len) memcpy(gp.pat, o->pattern, o->pattern_len);
   gp.plen = o->pattern_len;
@@ -78,12 +82,21 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
                     std::to_string(gp.cap) + "/" + p.key + "/";
   for (uint32_t i = 0; i < gp.plen; ++i) key += std::to_string(gp.pat[i]) + ",";
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
-    return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
-      launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p, c->d_ctr + 3,
-                  (unsigned long long*)c->b_blk2.p, (uint64_t*)c->b_out1.p, c->d_err, cs);
+    size_t ci = 0;
+    int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      const size_t k = ci % N;   // slot of this chunk: its block counts/bases are private to it
+      launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p + k * nblk, c->d_ctr + 3,
+                  (unsigned long long*)c->b_blk2.p + k * nblk, (unsigned long long*)c->b_out3.p + 2 * ci,
+                  (uint64_t*)c->b_out2.p, c->d_err, cs);
+      ++ci;
       c->n_launch += 3;
       return BK_OK;
     });
+    if (r) return r;
+    launch_grep_order((const unsigned long long*)c->b_out3.p, (uint32_t)C, (const uint64_t*)c->b_out2.p,
+                      (uint64_t*)c->b_out1.p, cap, c->s_comp);
+    c->n_launch += 1;
+    return (int)BK_OK;
   });
   if (rc) return rc;
   unsigned long long m = 0;
