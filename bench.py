@@ -81,7 +81,7 @@ WORKLOADS = {
                                    "MCA-indexed P:929)"),
     "kmeans": (16.0, 2048, "C3 k-means step: 16-dim fp32 points, K=64, Forgy init"),
     "kmer": (4.0, 2048, "f4 k-mer counting (k=31) over 256-B DNA read records, 96-base sequence at +16 (37.5% "
-                        "read, Table I DNA: 36%), reads of a seeded 2^25-base genome, 0.05% substitutions, 0.2% N"),
+                        "read, Table I DNA: 36%), reads of a seeded 2^25-base genome, 0.1% substitutions, 0.2% N"),
     "partition": (8.0, 2048, "C4 stable hash partition: {u64 key, u64 value} 16-B records into 1024 buckets, "
                              "bucket-sorted chunks written back to host (full duplex)"),
 }
@@ -108,7 +108,7 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
         return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=stride)
     if workload == "kmer":
         n = nbytes // 256
-        buf = gen.dna(gen.SEED_DNA, first=rank * n, n=n, genome_len=1 << 25, err_pm=0, n_pm=2)
+        buf = gen.dna(gen.SEED_DNA, first=rank * n, n=n, genome_len=1 << 25, err_pm=1, n_pm=2)
         return dict(buf=buf, off=None, n=n, first=rank * n, rec_size=256)
     if workload == "partition":
         n = nbytes // 16

@@ -42,3 +42,53 @@ def test_kmer_errors():
         with pytest.raises(bk.BkError) as e:
             ctx.kmer(k=31, table_slots=1 << 10)
         assert e.value.status == bk.BK_E_CAPACITY
+
+
+def _windows(seq: np.ndarray, k: int):
+    """All k-windows of a block of reads (uint8 [reads, L]): packed values (A=0 C=1 G=2 T=3, first
+    base most significant) and validity (every base in ACGT). Plain definition, no rolling."""
+    code = np.full(seq.shape, 255, np.uint8)
+    for i, ch in enumerate(b"ACGT"):
+        code[seq == ch] = i
+    ok = code != 255
+    W = seq.shape[1] - k + 1
+    val = np.zeros((seq.shape[0], W), np.uint64)
+    valid = np.ones((seq.shape[0], W), bool)
+    for i in range(k):
+        val <<= np.uint64(2)
+        val |= code[:, i:i + W] & np.uint8(3)
+        valid &= ok[:, i:i + W]
+    return val, valid
+
+
+def test_kmer_bench_scale_sampled():
+    """The bench configuration (4 GiB of reads, 2 GiB window, k = 31, AUTO gather): the total
+    equals the number of valid windows counted from the definition, the counts sum to it, and
+    64 sampled k-mers have exactly the counts a brute-force recount over every read gives."""
+    k, n = 31, (4 << 30) // 256
+    buf = gen.dna(gen.SEED_DNA, first=0, n=n, genome_len=1 << 25, err_pm=1, n_pm=2, threads=16)
+    with bk.Context(window_bytes=2 << 30, record_size=256) as ctx:
+        ctx.register(buf, None, n_records=n)
+        km, ct, total = ctx.kmer(k=k, table_slots=1 << 28, cap=1 << 27)
+    assert int(ct.sum()) == total
+    rng = np.random.default_rng(7)
+    pick = rng.choice(len(km), 64, replace=False)
+    want = {int(km[i]): int(ct[i]) for i in pick}
+    keys = np.array(sorted(want), np.uint64)
+    seqs = buf.reshape(n, 256)[:, 16:112]
+
+    def block(lo):  # numpy releases the GIL: blocks recount in parallel
+        val, valid = _windows(seqs[lo:lo + (1 << 18)], k)
+        v = val[valid]
+        idx = np.searchsorted(keys, v)
+        idx[idx == len(keys)] = 0
+        m = keys[idx] == v
+        return int(valid.sum()), np.bincount(idx[m], minlength=len(keys))
+
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(8) as ex:
+        parts = list(ex.map(block, range(0, n, 1 << 18)))
+    n_valid = sum(p[0] for p in parts)
+    hits = sum(p[1] for p in parts)
+    assert total == n_valid
+    assert {int(key): int(h) for key, h in zip(keys, hits)} == want

@@ -60,3 +60,14 @@ def test_kmer_invariants():
         assert int(ct.sum()) == windows                      # every valid window counted once
         assert np.all(np.diff(km.astype(np.int64)) > 0)     # distinct, ascending
         assert int(km.max()) < 4 ** k
+
+
+def test_window_helper_of_the_bench_scale_test_matches_oracle():
+    """tests/test_gpu_kmer.py recounts sampled k-mers with a numpy helper; pin it to O6 here."""
+    from test_gpu_kmer import _windows
+    n, k = 300, 13
+    buf = gen.dna(n=n, genome_len=1 << 12, err_pm=5, n_pm=20)
+    wk, wc = oracle.kmer(buf, n, k)
+    val, valid = _windows(buf.reshape(n, 256)[:, 16:112], k)
+    u, c = np.unique(val[valid], return_counts=True)
+    assert np.array_equal(u, wk) and np.array_equal(c.astype(np.uint64), wc)
