@@ -201,4 +201,33 @@ uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, c
   return size;
 }
 
+bool host_packable(const Access& a) { return !a.whole && a.n_ext == 1 && a.E > 0 && (a.E % 16) == 0; }
+
+uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* dst,
+                         uint64_t cap) {
+  const uint64_t E = a.E, n = c.hi - c.lo, size = n * E;
+  if (size > cap) return UINT64_MAX;
+  const uint32_t eo = a.ext_off[0], EW = (uint32_t)(E / 16);
+  constexpr uint64_t kGrab = 16384;   // records per grab: a few MB of the data set, read in order
+  constexpr uint64_t kPf = 16;        // software prefetch distance (records)
+  std::atomic<uint64_t> next{0};
+  pool.run([&](int) {
+    auto src = [&](uint64_t r) { return d.base + (d.off ? d.off[r] : r * d.rec_size) + eo; };
+    for (;;) {
+      const uint64_t j0 = next.fetch_add(kGrab);
+      if (j0 >= n) break;
+      const uint64_t j1 = std::min(n, j0 + kGrab);
+      for (uint64_t j = j0; j < std::min(j1, j0 + kPf); ++j) __builtin_prefetch(src(c.lo + j));
+      for (uint64_t j = j0; j < j1; ++j) {
+        if (j + kPf < j1) __builtin_prefetch(src(c.lo + j + kPf));
+        const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
+        __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
+        for (uint32_t m = 0; m < EW; ++m) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
+      }
+    }
+    _mm_sfence();
+  });
+  return size;
+}
+
 }  // namespace bk

@@ -49,4 +49,12 @@ uint64_t host_staged_size(const HostData& d, const Access& a, const Chunk& c);
 uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* stage,
                            uint64_t cap, std::vector<uint64_t>& first_scratch, std::vector<uint64_t>& tile_scratch);
 
+// Single-extent access with E % 16 == 0 (host_packable): packs the chunk's accessed bytes in record
+// order, E bytes per record, into dst (16-B aligned) — a sequential read of the data set and a
+// sequential non-temporal write, the cheapest host gather there is. The warp-tile interleave is then
+// done on the GPU (HBM -> HBM). Returns (hi - lo) * E, or UINT64_MAX if that exceeds cap.
+bool host_packable(const Access& a);
+uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* dst,
+                         uint64_t cap);
+
 }  // namespace bk

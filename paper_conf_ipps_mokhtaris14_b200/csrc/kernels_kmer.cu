@@ -18,10 +18,8 @@ __device__ __forceinline__ void kmer_insert(KmerEntry* table, uint64_t mask, uns
   uint64_t slot = mix64(key) & mask;
   for (uint64_t probe = 0; probe <= mask; ++probe, slot = (slot + 1) & mask) {
     unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(&table[slot].key);
-    if (k == 0) {
-      k = atomicCAS(&table[slot].key, 0ull, key);
-      if (k == 0) atomicAdd(used, 1ull);
-    }
+    if (k == 0) k = atomicCAS(&table[slot].key, 0ull, key);   // claim (the distinct count comes from compaction:
+                                                               // a counter here would serialise every new key)
     if (k == 0 || k == key) {
       atomicAdd(&table[slot].count, (unsigned long long)cnt);
       return;

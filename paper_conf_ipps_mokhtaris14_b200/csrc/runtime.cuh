@@ -100,6 +100,7 @@ struct Plan {
   uint64_t max_acc_rec = 0;            // max accessed bytes of one record
   uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
   uint32_t desc_sets = 1;              // descriptor sets per slot (2: ZC, stage 1 runs a chunk ahead)
+  bool packed = false;                 // CPU chunks: host packs records' bytes, GPU interleaves (raw slot)
   std::vector<uint64_t> bounds;        // chunk record bounds
   std::string key;                     // plan-cache key (also part of the graph key)
 };

@@ -54,6 +54,45 @@ int ensure_host_side(bk_ctx* c, const Plan& p) {
   return BK_OK;
 }
 
+// Packed CPU chunk: the host pool copies each record's accessed bytes in record order (stage 2,
+// gather half), one DMA moves exactly those bytes (stage 3), and the GPU interleaves them into warp
+// tiles HBM -> HBM (stage 2, layout half): the packed chunk is a run of fixed E-byte records read
+// whole, so stage 1 and the whole-record gather produce the same lanes and tiles as the field plan.
+static int stage_chunk_packed(bk_ctx* c, const Plan& p, size_t i, Slot& s, const Chunk& ch, const Access& a,
+                              const HostData& d, size_t hs, std::chrono::steady_clock::time_point t0) {
+  (void)i;
+  const uint64_t size = host_pack_chunk(*c->pool, d, a, ch, c->hstage[hs], p.raw_cap);
+  c->st.ms_cpu_gather += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  if (size == UINT64_MAX) return fail(BK_E_RANGE, "host-packed chunk exceeds its slot (internal bound violated)");
+  if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+  BK_DELAY(c->s_copy);
+  BK_PROF(kStH2D, c->s_copy, true);
+  if (size) BK_CUDA(cudaMemcpyAsync(s.raw, c->hstage[hs], size, cudaMemcpyHostToDevice, c->s_copy));
+  BK_CUDA(cudaEventRecord(c->h_done[hs], c->s_copy));
+  c->h_used[hs] = true;
+  BK_PROF(kStH2D, c->s_copy, false);
+  Chunk pc = ch;              // the packed chunk: records [lo, hi) of E bytes at raw + (r - lo) * E
+  pc.base_byte = ch.lo * a.E;
+  pc.end_byte = ch.hi * a.E;
+  pc.guard_lo = 0;
+  pc.guard_hi = p.raw_cap;
+  Access pa = whole_access();
+  pa.rec_size = a.E;
+  BK_PROF(kStAddrgen, c->s_copy, true);
+  launch_addrgen(pc, pa, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, c->s_copy);
+  BK_PROF(kStAddrgen, c->s_copy, false);
+  BK_PROF(kStRelayout, c->s_copy, true);
+  launch_gather(pc, pa, s.raw, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 0, c->s_copy);
+  BK_PROF(kStRelayout, c->s_copy, false);
+  c->n_launch += 3;
+  c->st.bytes_h2d += size;
+  c->st.bytes_accessed += ch.accessed;
+  c->st.n_chunks_cpu += 1;
+  BK_CUDA(cudaEventRecord(s.ready, c->s_copy));
+  s.used = true;
+  return BK_OK;
+}
+
 // CPU assembly of chunk i (stage 2 on the host pool) + one DMA of the packed tiles (stage 3).
 int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   const Chunk ch = chunk_of(c, p, i);
@@ -65,6 +104,7 @@ int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     std::this_thread::sleep_for(std::chrono::microseconds(test_rand(c) % 200));
   const auto t0 = std::chrono::steady_clock::now();
   HostData d{c->host, c->off, c->n, c->nbytes, c->cfg.record_size};
+  if (p.packed) return stage_chunk_packed(c, p, i, s, ch, a, d, hs, t0);
   const uint64_t size = host_gather_chunk(*c->pool, d, a, ch, c->hstage[hs], p.stage_cap, c->scratch_first,
                                           c->scratch_tiles);
   c->st.ms_cpu_gather += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();

@@ -104,7 +104,9 @@ void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) 
     }
     p.stage_cap = align_up(mx + 512, 512);
   }
-  p.raw_cap = p.zero_copy ? 0 : budget + 64;
+  // DENSE: raw whole records; CPU/HYBRID with a packable access: the host-packed chunk (plan bytes
+  // = accessed bytes there)
+  p.raw_cap = !p.zero_copy || p.packed ? budget + 64 : 0;
   p.meta_cap = c->off ? maxrecs + 1 : 0;
 }
 
@@ -122,6 +124,7 @@ int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p,
   p.mode = mode;
   p.zero_copy = mode != BK_GATHER_DENSE;
   p.desc_sets = mode == BK_GATHER_ZC ? 2 : 1;
+  p.packed = (mode == BK_GATHER_CPU || mode == BK_GATHER_HYBRID) && host_packable(a);
   p.max_acc_rec = a.whole ? c->max_rec : a.E;
   const uint64_t slot = c->cfg.window_bytes / c->cfg.n_slots;
   // total plan bytes

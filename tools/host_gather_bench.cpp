@@ -4,6 +4,7 @@
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
+#include <string>
 #include <vector>
 
 #include "gen.h"
@@ -13,6 +14,7 @@ int main(int argc, char** argv) {
   using namespace bk;
   const double gib = argc > 1 ? atof(argv[1]) : 16;
   const int threads = argc > 2 ? atoi(argv[2]) : 16;
+  const bool pack = argc > 3 && std::string(argv[3]) == "pack";   // host_pack_chunk instead of tiles
   const uint64_t n = gen_grep_count_for_bytes(0xB16C0002, 0, (uint64_t)(gib * (1ull << 30)));
   std::vector<uint64_t> off(n);
   const uint64_t nb = gen_grep_sizes(0xB16C0002, 0, n, off.data());
@@ -32,10 +34,12 @@ int main(int argc, char** argv) {
       c.lo = lo; c.hi = std::min(n, lo + per);
       c.base_byte = off[lo]; c.end_byte = c.hi < n ? off[c.hi] : nb;
       c.L = (uint32_t)(((c.hi - lo) / 8 + 31) / 32 * 32); c.ntiles = c.L / 32; c.accessed = (c.hi - lo) * 32;
-      host_gather_chunk(pool, d, a, c, stage.data(), stage.size(), f, t);
+      if (pack) host_pack_chunk(pool, d, a, c, stage.data(), stage.size());
+      else host_gather_chunk(pool, d, a, c, stage.data(), stage.size(), f, t);
     }
     double s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
-    printf("{\"threads\": %d, \"s\": %.4f, \"grec_s\": %.3f}\n", threads, s, n / s / 1e9);
+    printf("{\"mode\": \"%s\", \"threads\": %d, \"s\": %.4f, \"grec_s\": %.3f}\n", pack ? "pack" : "tiles",
+           threads, s, n / s / 1e9);
   }
   return 0;
 }
