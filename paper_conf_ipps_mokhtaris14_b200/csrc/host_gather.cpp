@@ -208,6 +208,8 @@ uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, con
   const uint64_t E = a.E, n = c.hi - c.lo, size = n * E;
   if (size > cap) return UINT64_MAX;
   const uint32_t eo = a.ext_off[0], EW = (uint32_t)(E / 16);
+  // sweep on the 16-core host (profiles/r01_hybrid_sweep.md): 16-record prefetch distance, grabs of
+  // 4k-16k records; non-temporal vs regular stores are equal inside the pipeline
   constexpr uint64_t kGrab = 16384;   // records per grab: a few MB of the data set, read in order
   constexpr uint64_t kPf = 16;        // software prefetch distance (records)
   std::atomic<uint64_t> next{0};
