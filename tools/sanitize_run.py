@@ -30,4 +30,27 @@ kv = gen.kv(n=100_000)
 with bk.Context(window_bytes=1 << 20, record_size=16) as ctx:
     ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=100_000)
     ctx.partition(1024)
+# later round-1 paths: ZC per-slot staging streams + double-buffered descriptors (graph and eager),
+# host-packed CPU chunks with the GPU interleave, order-independent grep, k-mers, online patterns
+for ng in (False, True):
+    with bk.Context(window_bytes=128 << 10, n_slots=4, gather_mode="zc", no_graph=ng) as ctx:
+        ctx.register(buf, off)
+        ctx.wordcount(cap=1 << 16)
+        ctx.wordcount(cap=1 << 16)
+for mode in ("cpu", "dense"):
+    with bk.Context(window_bytes=256 << 10, n_slots=3, gather_mode=mode) as ctx:
+        ctx.register(gb, goff)
+        ctx.grep(b"bigk", cap=20000)
+for mode in ("cpu", "hybrid"):
+    with bk.Context(window_bytes=512 << 10, record_size=64, gather_mode=mode) as ctx:
+        ctx.register(g, None, n_records=100_000)
+        ctx.groupby(4096)
+d = gen.dna(n=20_000, genome_len=1 << 16, err_pm=2, n_pm=3)
+for mode in ("hybrid", "zc", "cpu"):
+    with bk.Context(window_bytes=1 << 20, record_size=256, gather_mode=mode) as ctx:
+        ctx.register(d, None, n_records=20_000)
+        ctx.kmer(k=31, table_slots=1 << 22)
+with bk.Context(window_bytes=256 << 10) as ctx:
+    ctx.register(buf, off)
+    ctx.pattern_stats(elem_bytes=1, T=8)
 print("sanitize run done")
