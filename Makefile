@@ -8,7 +8,7 @@ OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.
 
 all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so baselines/libbkmt.so
 
-build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh $(CSRC)/runtime.cuh $(CSRC)/host_gather.h include/bk.h
+build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh $(CSRC)/tma.cuh $(CSRC)/runtime.cuh $(CSRC)/host_gather.h include/bk.h
 	@mkdir -p build
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
 

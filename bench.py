@@ -87,6 +87,38 @@ WORKLOADS = {
 }
 
 
+def _cpulist(text: str) -> list[int]:
+    out = []
+    for part in text.strip().split(","):
+        if "-" in part:
+            a, b = part.split("-")
+            out.extend(range(int(a), int(b) + 1))
+        elif part:
+            out.append(int(part))
+    return out
+
+
+def numa_local_cores(torch, local: int) -> list[int] | None:
+    """Host cores for this rank when several ranks share the node: the cores PCIe-local to its GPU
+    (sysfs local_cpulist), split evenly among the ranks whose GPUs share that list, so that first
+    touch of the shard lands on the GPU's NUMA node and the assembly pools do not oversubscribe."""
+    lists = []
+    for d in range(torch.cuda.device_count()):
+        p = torch.cuda.get_device_properties(d)
+        path = f"/sys/bus/pci/devices/{p.pci_domain_id:04x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0/local_cpulist"
+        try:
+            with open(path) as f:
+                cores = _cpulist(f.read())
+        except OSError:
+            return None
+        lists.append(tuple(c for c in cores if c in os.sched_getaffinity(0)))
+    mine = lists[local]
+    peers = [d for d, l in enumerate(lists) if l == mine]
+    k, m = peers.index(local), len(peers)
+    part = list(mine[len(mine) * k // m: len(mine) * (k + 1) // m])
+    return part or None
+
+
 def make_shard(workload: str, gib: float, rank: int, world: int):
     """Rank r's contiguous shard of the weak-scaled data set. Returns dict."""
     nbytes = int(gib * GIB)
@@ -289,7 +321,14 @@ def main():
         else:
             dist.init_process_group(backend)
 
-    # ranks on one node share the host cores for CPU assembly (one pool per rank)
+    # ranks on one node share the host cores for CPU assembly (one pool per rank): bind each rank to
+    # its GPU's NUMA-local share before the shard is generated (first touch) and the pool started
+    if world > 1 and torch.cuda.device_count() > 1:
+        cores = numa_local_cores(torch, local)
+        if cores:
+            os.sched_setaffinity(0, cores)
+            if not args.host_threads:
+                args.host_threads = len(cores)
     if not args.host_threads:
         args.host_threads = max(1, (os.cpu_count() or 1) // int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
     shard = make_shard(args.workload, gib, rank, world)
@@ -392,6 +431,7 @@ def main():
         pst = pctx.stats()
         pctx.close()
         for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute", "n_gather", "ms_cpu_gather", "ms_xfer_busy",
+                  "ms_zc", "n_zc", "ms_relayout", "n_relayout", "n_chunks_zc", "bytes_zc", "records_zc",
                   "ms_compute_busy", "ms_overlap"):
             st[k] = pst[k]
         st["profiled_ms_device"] = pst["ms_device"]
@@ -403,36 +443,34 @@ def main():
 
     # ---- roofline of the dominant stage (busy times from CUDA events on each stage's own stream)
     peaks = load_peaks()
-    stage_ms = {"gather": st["ms_gather"], "compute": st["ms_compute"], "addrgen": st["ms_addrgen"],
-                "h2d": st["ms_h2d"]}
+    stage_ms = {"zc": st["ms_zc"], "relayout": st["ms_relayout"], "compute": st["ms_compute"],
+                "addrgen": st["ms_addrgen"], "h2d": st["ms_h2d"]}
     # dominant stage: transfer (DMA / zero-copy gather) vs compute by the UNION of their busy
     # intervals (per-slot streams run kernels concurrently, so per-launch sums overcount); stage 1
-    # (addrgen) runs a chunk ahead and is off the critical chain, so it is never the roofline kernel
+    # (addrgen) runs a chunk ahead and is off the critical chain, so it is never the roofline kernel.
+    # Inside the transfer side the zero-copy gathers and the copy-engine DMAs are told apart by their
+    # own busy times; the HBM -> HBM interleave of DMA'd chunks is accounted separately (ms_relayout).
     if st.get("ms_compute_busy", 0.0) > st.get("ms_xfer_busy", 0.0):
         dom = "compute"
     else:
-        dom = "gather" if st["ms_gather"] >= st["ms_h2d"] else "h2d"
-    n_zc = max(st["n_gather"], 1)
+        dom = "zc" if st["n_chunks_zc"] and st["ms_zc"] >= st["ms_h2d"] else "h2d"
     if dom == "h2d":
         # copy-engine DMA of packed (CPU) or raw (DENSE) chunks + offsets slices: host-link bound
-        launches = st["n_chunks"]
-        per_launch = (st["bytes_h2d"] - (st["bytes_accessed"] * (st["n_gather"] / max(st["n_chunks"], 1))
-                                          if st["gather_mode"] == bk.BK_GATHER_HYBRID else 0)
-                      + st["bytes_meta"]) / launches
+        launches = max(st["n_chunks"] - st["n_chunks_zc"], 1)
+        per_launch = (st["bytes_h2d"] - st["bytes_zc"] + st["bytes_meta"]) / launches
         roof = {"kernel": "cudaMemcpyAsync H2D of staged chunks (stage 3, copy engine)", "bound": "host_link",
                 "peak": peak_h2d, "unit": "GB/s"}
-    elif dom == "gather" and st["gather_mode"] in (bk.BK_GATHER_ZC, bk.BK_GATHER_HYBRID):
-        launches = n_zc
-        zc_chunks = n_zc
-        per_launch = st["bytes_accessed"] / st["n_chunks"]      # accessed bytes per chunk pulled over PCIe
+    elif dom == "zc":
+        # the zero-copy gather kernel (stages 2+3 fused): accessed bytes it pulled over PCIe per launch
+        launches = max(st["n_zc"], 1)
+        per_launch = st["bytes_zc"] / max(st["n_chunks_zc"], 1)
         roof = {"kernel": "k_gather_field/whole<zero-copy> (stages 2+3)", "bound": "host_link",
                 "peak": peak_h2d, "unit": "GB/s"}
     else:
-        launches = n_zc if dom == "gather" else st["n_chunks"]
-        # HBM-bound kernels: re-layout reads the raw chunk and writes the tiles; compute reads the tiles
-        per_launch = ((st["bytes_h2d"] + st["bytes_accessed"] + st["bytes_padding"]) if dom == "gather"
-                      else (st["bytes_accessed"] + st["bytes_padding"])) / max(launches, 1)
-        if dom == "compute" and args.workload == "kmer" and box.get("kmer_windows"):
+        launches = st["n_chunks"]
+        # HBM-bound compute: reads the staged tiles (payload + padding)
+        per_launch = (st["bytes_accessed"] + st["bytes_padding"]) / max(launches, 1)
+        if args.workload == "kmer" and box.get("kmer_windows"):
             # + the hash-table traffic: one 16-B entry read and one 8-B count update per k-mer window
             per_launch += 24 * box["kmer_windows"] / max(launches, 1)
         roof = {"kernel": f"{dom} ({args.workload})", "bound": "hbm", "peak": peaks.get("hbm_gbs", 6650.0),
@@ -446,12 +484,12 @@ def main():
         "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6650 GB/s")
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["traffic"] = None
-    if roof["kernel"].startswith("k_gather_field") and args.workload == "grep":
+    if dom == "zc" and args.workload == "grep":
         # the zero-copy key gather is PCIe read-request bound, not byte bound: one read request per
         # 128-B line a 32-B key touches (8-aligned keys: 1 + 3/16 = 1.1875 requests per record).
         # Peak = the request rate the phase-0 probe measured for one field per 256-B record
         # (profiles/r01_box_probe.txt: zc_sparse rec 256 -> 0.562 G records/s, one request each).
-        recs_per_launch = shard["n"] / st["n_chunks"]
+        recs_per_launch = st["records_zc"] / max(st["n_chunks_zc"], 1)
         req_rate = recs_per_launch * 1.1875 / (avg_ms * 1e-3)
         roof["request_rate"] = {"bound": "pcie_read_requests", "achieved": req_rate / 1e9, "peak": 0.562,
                                 "unit": "G requests/s", "frac": req_rate / 0.562e9,
@@ -480,8 +518,10 @@ def main():
                  "frac": round(link_gbs / (peak_h2d * world), 4),
                  "bytes_per_step_per_gpu": st["bytes_h2d"] + st["bytes_meta"],
                  "payload_bytes": st["bytes_h2d"], "meta_bytes": st["bytes_meta"], "padding_bytes_hbm": st["bytes_padding"]},
-        "stages_ms_per_step": {**{k: round(st[k], 3) for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute",
-                                                                "ms_device", "ms_cpu_gather")},
+        "stages_ms_per_step": {**{k: round(st[k], 3) for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_zc",
+                                                                "ms_relayout", "ms_compute", "ms_device",
+                                                                "ms_cpu_gather")},
+                               "n_zc": st["n_zc"], "n_relayout": st["n_relayout"],
                                "profiled_ms_device": round(st.get("profiled_ms_device", 0.0), 3),
                                "note": "per-stage busy sums from a profiled eager pass (CUDA events per stage "
                                        "per chunk); ms_device from the timed (graph-replayed when static) pass"},

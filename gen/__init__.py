@@ -64,7 +64,7 @@ def lib():
 
 
 def _threads(threads):
-    return threads if threads else (os.cpu_count() or 1)
+    return threads if threads else (len(os.sched_getaffinity(0)) or 1)
 
 
 def _ptr(a: np.ndarray) -> int:

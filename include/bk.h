@@ -269,6 +269,13 @@ typedef struct bk_stats {
   double ms_xfer_busy;        /* BK_FLAG_PROFILE: union of the transfer intervals (DMA copies, zero-copy gathers) */
   double ms_compute_busy;     /*   union of the compute-kernel intervals */
   double ms_overlap;          /*   length of their intersection (copy/compute overlap) */
+  double ms_zc;               /* BK_FLAG_PROFILE: busy time of the zero-copy gathers alone (stages 2+3 over PCIe) */
+  uint64_t n_zc;              /*   number of zero-copy gather launches timed */
+  double ms_relayout;         /*   busy time of the HBM -> HBM interleave kernels (DENSE raw chunks, packed CPU chunks) */
+  uint64_t n_relayout;        /*   number of interleave launches timed */
+  uint64_t n_chunks_zc;       /* chunks gathered zero-copy in the last run */
+  uint64_t bytes_zc;          /* accessed bytes those chunks pulled over PCIe */
+  uint64_t records_zc;        /* records in those chunks */
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);

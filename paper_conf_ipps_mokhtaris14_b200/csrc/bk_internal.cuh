@@ -92,25 +92,30 @@ struct GrepParams {
   uint64_t first_index;
   uint64_t cap;
 };
-// three launches per chunk: block counts, one-block scan (reserves the chunk's run [base, base+n)
-// of the match pool with atomicAdd on *cursor, writes chunk_run = {base, n}), ordered write into
-// the pool. Chunks may run concurrently; launch_grep_order then lays the runs out in chunk order.
+// three launches per chunk: per-tile counts + per-lane match masks, a one-block scan (reserves the
+// chunk's run [base, base+n) of the match pool with atomicAdd on *cursor, writes chunk_run =
+// {base, n} and each tile's output base), ordered write into the pool. Chunks may run
+// concurrently; launch_grep_order then lays the runs out in chunk order. tilecnt / tilebase_out
+// hold c.ntiles entries, lanemask c.L.
+size_t grep_count_smem();
 void launch_grep(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
-                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* cursor,
-                 unsigned long long* blkbase, unsigned long long* chunk_run, uint64_t* out_idx, int* err,
-                 cudaStream_t s);
+                 const GrepParams& p, uint32_t* tilecnt, uint32_t* lanemask, unsigned long long* cursor,
+                 unsigned long long* tilebase_out, unsigned long long* chunk_run, uint64_t* out_idx, int* err,
+                 int grid, bool tma, cudaStream_t s);
 void launch_grep_order(const unsigned long long* runs, uint32_t C, const uint64_t* pool, uint64_t* out, uint64_t cap,
                        cudaStream_t s);
 
-size_t groupby_smem(uint32_t G);
+// tma: stage-4 reads through bulk copies into shared memory (tma.cuh); false: plain 16-B loads
+// (chunks computed while zero-copy gathers run, profiles/r01_tma.md)
+size_t groupby_smem(uint32_t G, bool tma);
 void launch_groupby(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                     uint32_t G, unsigned long long* count, unsigned long long* qty, double* amount, int* err,
-                    int grid, cudaStream_t s);
+                    int grid, bool tma, cudaStream_t s);
 
-size_t kmeans_smem(uint32_t K);
+size_t kmeans_smem(uint32_t K, bool tma);
 void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                    const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
-                   unsigned long long* chk, int32_t* cid_out, int grid, cudaStream_t s);
+                   unsigned long long* chk, int32_t* cid_out, int grid, bool tma, cudaStream_t s);
 
 cudaError_t configure_compute_kernels();
 

@@ -4,6 +4,10 @@
 // reduce with warp-level aggregation and block-level shared-memory tables before touching
 // global memory (north_star: warp shuffles + block-level atomics).
 #include "bk_internal.cuh"
+#include "tma.cuh"
+
+#include <algorithm>
+#include <cstdlib>
 
 namespace bk {
 namespace {
@@ -273,110 +277,104 @@ __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, 
 // ------------------------------------------------------------------------------------------
 // C2 grep (MCA analogue): key = first strnlen(32) bytes of the record's 32-byte key
 // field (staged as words 2j, 2j+1 of the lane); match iff the pattern is a substring. Output
-// indices are ascending. Chunks compute in any order (per-slot streams): per chunk, block counts ->
-// one-block scan that reserves the chunk's run in a match pool with one atomicAdd and records
-// (pool offset, count) per chunk -> write; after the last chunk one pass copies the runs into
-// chunk order (k_grep_order).
+// indices are ascending. Chunks compute in any order (per-slot streams). Per chunk:
+//   k_grep_count  each warp streams its tiles through shared memory (WarpTileStream) and writes
+//                 per-lane match masks (bit j = record j of the lane) and per-tile match counts;
+//   k_grep_scan   one block: the chunk's match count, its run [base, base+n) of a match pool
+//                 (one atomicAdd), and each tile's output base;
+//   k_grep_write  one warp per tile turns the masks into ascending record indices (no key re-read).
+// After the last chunk one pass copies the runs into chunk order (k_grep_order).
 
-struct Key32 { uint64_t q[8]; };  // q[4..7] = 0: windows past byte 31 read zeros
+struct Key32 { uint32_t w[8]; };   // the key field, little-endian words
 
-__device__ __forceinline__ uint64_t window8(const Key32& k, int x) {  // bytes [x, x+8), x constant
-  const int i = x >> 3, s = (x & 7) * 8;
-  if (s == 0) return k.q[i];
-  return (k.q[i] >> s) | (k.q[i + 1] << (64 - s));
-}
-
-__device__ __forceinline__ uint32_t strnlen32(const Key32& k) {
+// bit x set iff key byte x == the byte replicated in `rep` (SWAR compare of 4 bytes per word; the
+// 0/1 byte flags at bits 0, 8, 16, 24 are gathered to bits 24..27 by one multiply)
+__device__ __forceinline__ uint32_t eqmask32(const Key32& k, uint32_t rep) {
+  uint32_t m = 0;
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const uint64_t v = k.q[i];
-    const uint64_t z = (v - 0x0101010101010101ull) & ~v & 0x8080808080808080ull;  // first zero byte
-    if (z) return 8 * i + (__ffsll((long long)z) - 1) / 8;
+  for (int i = 0; i < 8; ++i) {
+    const uint32_t t = __vcmpeq4(k.w[i], rep) & 0x01010101u;
+    m |= ((t * 0x01020408u) >> 24) << (4 * i);
   }
-  return 32;
+  return m;
 }
 
-__device__ __forceinline__ bool grep_match(const Key32& k, const GrepParams& p, const uint64_t* pw,
-                                           const uint64_t* pm) {
+// Match bits of every start position: bit x set iff x + plen <= kl and key[x + i] == pat[i] for
+// all i < plen, i.e. AND_i (eqmask(pat[i]) >> i) restricted to the positions that fit in the key.
+__device__ __forceinline__ bool grep_match(const Key32& k, const GrepParams& p) {
   if (p.plen == 0) return true;
-  const int kl = (int)strnlen32(k);
+  const uint32_t z = eqmask32(k, 0u);
+  const int kl = z ? __ffs((int)z) - 1 : 32;   // strnlen(key, 32)
   const int plen = (int)p.plen;
-  bool hit = false;
+  if (kl < plen) return false;
+  const int fit = kl - plen + 1;               // start positions 0 .. kl - plen
+  uint32_t M = fit >= 32 ? 0xffffffffu : ((1u << fit) - 1);
 #pragma unroll
-  for (int x = 0; x < 32; ++x) {
-    bool ok = x + plen <= kl && (window8(k, x) & pm[0]) == pw[0];
-    if (plen > 8) ok = ok && (window8(k, x + 8) & pm[1]) == pw[1];
-    if (plen > 16) ok = ok && (window8(k, x + 16) & pm[2]) == pw[2];
-    if (plen > 24) ok = ok && (window8(k, x + 24) & pm[3]) == pw[3];
-    hit = hit || ok;
+  for (int i = 0; i < 32; ++i) {   // unrolled: pattern bytes come from the constant bank, not a stack copy
+    if (i >= plen || !M) break;
+    M &= eqmask32(k, (uint32_t)p.pat[i] * 0x01010101u) >> i;
   }
-  return hit;
+  return M != 0;
 }
 
-__device__ __forceinline__ Key32 load_key(const uint8_t* tile, uint32_t j, int lane) {
-  const uint4 a = lane_word(tile, 2 * j, lane);
-  const uint4 b = lane_word(tile, 2 * j + 1, lane);
-  Key32 k;
-  k.q[0] = (uint64_t)a.x | ((uint64_t)a.y << 32);
-  k.q[1] = (uint64_t)a.z | ((uint64_t)a.w << 32);
-  k.q[2] = (uint64_t)b.x | ((uint64_t)b.y << 32);
-  k.q[3] = (uint64_t)b.z | ((uint64_t)b.w << 32);
-  k.q[4] = k.q[5] = k.q[6] = k.q[7] = 0;
-  return k;
+__device__ __forceinline__ Key32 key_at(const uint8_t* row0, int lane) {  // rows 2j, 2j+1 (smem or HBM)
+  const uint4 a = *reinterpret_cast<const uint4*>(row0 + lane * 16);
+  const uint4 b = *reinterpret_cast<const uint4*>(row0 + 512 + lane * 16);
+  return Key32{{a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w}};
 }
 
-__device__ __forceinline__ void pattern_words(const GrepParams& p, uint64_t* pw, uint64_t* pm) {
-#pragma unroll
-  for (int b = 0; b < 4; ++b) {
-    uint64_t w = 0, m = 0;
-    for (int i = 0; i < 8; ++i) {
-      const int x = 8 * b + i;
-      if (x < (int)p.plen) { w |= (uint64_t)p.pat[x] << (8 * i); m |= 0xffull << (8 * i); }
+constexpr int kGrepThreads = 256;
+constexpr uint32_t kGrepRows = 8;    // rows per piece: 4 keys of 2 words
+
+template <bool kTma>
+__global__ void __launch_bounds__(kGrepThreads) k_grep_count(Chunk c, const uint8_t* __restrict__ stage,
+                                                             const LaneDesc* __restrict__ lanes,
+                                                             const uint64_t* __restrict__ tile_base, GrepParams p,
+                                                             uint32_t* __restrict__ tilecnt,
+                                                             uint32_t* __restrict__ lanemask) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  constexpr uint32_t nwarp = kGrepThreads / 32;
+  const uint32_t wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  WarpTileStream<kTma> ts = warp_stream<kTma>(smem_raw, nwarp, kGrepRows, stage, tile_base, c.ntiles);
+  ts.begin(blockIdx.x * nwarp + wid);
+  uint32_t mask = 0, cnt = 0;
+  while (ts.valid()) {
+    const uint32_t nrec = lanes[(size_t)ts.w * 32 + lane].nrec;
+    if (ts.p == 0) mask = cnt = 0;
+    uint32_t nw, np, nK;
+    const uint8_t* piece = ts.acquire(nw, np, nK);
+    const uint32_t r0 = ts.p * kGrepRows;
+    const uint32_t j1 = min(min(ts.K, r0 + kGrepRows) / 2, nrec);
+    for (uint32_t j = r0 / 2; j < j1; ++j) {
+      const uint32_t m = grep_match(key_at(piece + (size_t)(2 * j - r0) * 512, lane), p);
+      cnt += m;
+      if (j < 32) mask |= m << j;
     }
-    pw[b] = w;
-    pm[b] = m;
+    if ((ts.p + 1) * kGrepRows >= ts.K) {   // last piece of the tile
+      lanemask[(size_t)ts.w * 32 + lane] = mask;
+      const uint32_t tot = __reduce_add_sync(kFull, cnt);
+      if (lane == 0) tilecnt[ts.w] = tot;
+    }
+    ts.release(nw, np, nK);
   }
 }
 
-__device__ __forceinline__ uint32_t block_sum(uint32_t v, uint32_t* sh) {
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  v = __reduce_add_sync(kFull, v);
-  if (lane == 0) sh[wid] = v;
-  __syncthreads();
-  uint32_t s = 0;
-  if (threadIdx.x == 0)
-    for (int i = 0; i < (int)(blockDim.x >> 5); ++i) s += sh[i];
-  return s;
-}
-
-__global__ void __launch_bounds__(256) k_grep_count(Chunk c, const uint8_t* __restrict__ stage,
-                                                    const LaneDesc* __restrict__ lanes,
-                                                    const uint64_t* __restrict__ tile_base, GrepParams p,
-                                                    uint32_t* __restrict__ blkcnt) {
-  __shared__ uint32_t sh[8];
-  uint64_t pw[4], pm[4];
-  pattern_words(p, pw, pm);
-  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-  uint32_t cnt = 0;
-  if (t < c.L) {
-    const LaneDesc d = lanes[t];
-    const uint8_t* tile = stage + tile_base[t >> 5];
-    for (uint32_t j = 0; j < d.nrec; ++j) cnt += grep_match(load_key(tile, j, t & 31), p, pw, pm);
-  }
-  const uint32_t s = block_sum(cnt, sh);
-  if (threadIdx.x == 0) blkcnt[blockIdx.x] = s;
-}
-
-__global__ void __launch_bounds__(1024) k_grep_scan(uint32_t* __restrict__ blkcnt, uint32_t nblk,
-                                                    unsigned long long* cursor, unsigned long long* blkbase,
+// tiles with no staged rows were never visited by k_grep_count: they count zero
+__global__ void __launch_bounds__(1024) k_grep_scan(const uint32_t* __restrict__ tilecnt,
+                                                    const uint64_t* __restrict__ tile_base, uint32_t ntiles,
+                                                    unsigned long long* cursor, unsigned long long* tilebase_out,
                                                     unsigned long long* chunk_run) {
   __shared__ unsigned long long warp_sums[32];
   __shared__ unsigned long long carry;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  auto count = [&](uint32_t i) -> unsigned long long {
+    return i < ntiles && tile_base[i + 1] > tile_base[i] ? tilecnt[i] : 0ull;
+  };
   // the chunk's match count, then its run in the pool: [base, base + total)
   unsigned long long part = 0;
-  for (uint32_t i = threadIdx.x; i < nblk; i += 1024) part += blkcnt[i];
-  part = __reduce_add_sync(kFull, (unsigned)part);
+  for (uint32_t i = threadIdx.x; i < ntiles; i += 1024) part += count(i);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(kFull, part, o);
   if (lane == 0) warp_sums[wid] = part;
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -387,9 +385,9 @@ __global__ void __launch_bounds__(1024) k_grep_scan(uint32_t* __restrict__ blkcn
     chunk_run[1] = tot;
   }
   __syncthreads();
-  for (uint32_t base = 0; base < nblk; base += 1024) {
+  for (uint32_t base = 0; base < ntiles; base += 1024) {
     const uint32_t i = base + threadIdx.x;
-    const unsigned long long v = i < nblk ? blkcnt[i] : 0;
+    const unsigned long long v = count(i);
     unsigned long long x = v;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -409,7 +407,7 @@ __global__ void __launch_bounds__(1024) k_grep_scan(uint32_t* __restrict__ blkcn
     }
     __syncthreads();
     const unsigned long long excl = carry + (wid ? warp_sums[wid - 1] : 0) + x - v;
-    if (i < nblk) blkbase[i] = excl;
+    if (i < ntiles) tilebase_out[i] = excl;
     __syncthreads();
     if (threadIdx.x == 1023) carry = excl + v;
     __syncthreads();
@@ -441,76 +439,89 @@ __global__ void __launch_bounds__(256) k_grep_order(const unsigned long long* __
     if (dst + k < cap && src + k < cap) out[dst + k] = pool[src + k];
 }
 
+// One warp per tile: lane t's matches go to tilebase_out[w] + (matches of lanes before t), in
+// record order. Lanes of more than 32 records (a lane_bytes override) re-test their keys from HBM.
 __global__ void __launch_bounds__(256) k_grep_write(Chunk c, const uint8_t* __restrict__ stage,
                                                     const LaneDesc* __restrict__ lanes,
                                                     const uint64_t* __restrict__ tile_base, GrepParams p,
-                                                    const unsigned long long* __restrict__ blkbase,
+                                                    const unsigned long long* __restrict__ tilebase_out,
+                                                    const uint32_t* __restrict__ lanemask,
                                                     uint64_t* __restrict__ out, int* err) {
-  __shared__ uint32_t warp_tot[8];
-  uint64_t pw[4], pm[4];
-  pattern_words(p, pw, pm);
-  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  LaneDesc d{0, 0, 0};
-  const uint8_t* tile = nullptr;
-  uint32_t cnt = 0;
-  if (t < c.L) {
-    d = lanes[t];
-    tile = stage + tile_base[t >> 5];
-    for (uint32_t j = 0; j < d.nrec; ++j) cnt += grep_match(load_key(tile, j, lane), p, pw, pm);
+  const uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (w >= c.ntiles || tile_base[w + 1] == tile_base[w]) return;   // whole warps leave together
+  const LaneDesc d = lanes[(size_t)w * 32 + lane];
+  const uint8_t* tile = stage + tile_base[w];
+  uint32_t mask = 0, cnt = 0;
+  if (d.nrec <= 32) {
+    mask = d.nrec ? lanemask[(size_t)w * 32 + lane] : 0;
+    cnt = __popc(mask);
+  } else {
+    for (uint32_t j = 0; j < d.nrec; ++j) cnt += grep_match(key_at(tile + (size_t)2 * j * 512, lane), p);
   }
-  if (__syncthreads_or(cnt) == 0) return;  // most blocks of a 1%-selective filter
   uint32_t x = cnt;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
     const uint32_t y = __shfl_up_sync(kFull, x, o);
     if (lane >= o) x += y;
   }
-  if (lane == 31) warp_tot[wid] = x;
-  __syncthreads();
-  uint32_t before = 0;
-  for (int i = 0; i < wid; ++i) before += warp_tot[i];
-  unsigned long long pos = blkbase[blockIdx.x] + before + x - cnt;
-  if (cnt) {
-    for (uint32_t j = 0; j < d.nrec; ++j) {
-      if (grep_match(load_key(tile, j, lane), p, pw, pm)) {
-        if (pos < p.cap) out[pos] = p.first_index + d.first + j;
-        else atomicOr(err, kErrOutOverflow);
-        ++pos;
-      }
-    }
+  unsigned long long pos = tilebase_out[w] + x - cnt;
+  auto emit = [&](uint32_t j) {
+    if (pos < p.cap) out[pos] = p.first_index + d.first + j;
+    else atomicOr(err, kErrOutOverflow);
+    ++pos;
+  };
+  if (d.nrec <= 32) {
+    for (; mask; mask &= mask - 1) emit((uint32_t)__ffs((int)mask) - 1);
+  } else if (cnt) {
+    for (uint32_t j = 0; j < d.nrec; ++j)
+      if (grep_match(key_at(tile + (size_t)2 * j * 512, lane), p)) emit(j);
   }
 }
 
 // ------------------------------------------------------------------------------------------
 // C5 group-by: records {u32 key, u32 qty, f64 amount} staged one word per record.
-// Block-private shared-memory table (count, qty, amount), flushed once per block.
+// Each warp streams its tiles through shared memory with bulk copies (WarpTileStream, tma.cuh:
+// the copy of the next piece is in flight while the warp aggregates the current one) into a
+// block-private shared-memory table (count, qty, amount), flushed once per block.
 
-__global__ void __launch_bounds__(256) k_groupby(Chunk c, const uint8_t* __restrict__ stage,
-                                                 const LaneDesc* __restrict__ lanes,
-                                                 const uint64_t* __restrict__ tile_base, uint32_t G,
-                                                 unsigned long long* gcount, unsigned long long* gqty,
-                                                 double* gamount, int* err) {
-  extern __shared__ unsigned char smem_raw[];
-  double* s_amt = reinterpret_cast<double*>(smem_raw);
+constexpr int kGbThreads = 512;
+
+__host__ __device__ constexpr uint32_t groupby_rows(uint32_t G) { return G <= 4096 ? 8 : 4; }
+
+template <bool kTma>
+__global__ void __launch_bounds__(kGbThreads) k_groupby(Chunk c, const uint8_t* __restrict__ stage,
+                                                        const LaneDesc* __restrict__ lanes,
+                                                        const uint64_t* __restrict__ tile_base, uint32_t G,
+                                                        unsigned long long* gcount, unsigned long long* gqty,
+                                                        double* gamount, int* err) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  constexpr uint32_t nwarp = kGbThreads / 32;
+  const uint32_t rows = groupby_rows(G);
+  const uint32_t wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  WarpTileStream<kTma> ts = warp_stream<kTma>(smem_raw, nwarp, rows, stage, tile_base, c.ntiles);
+  double* s_amt = reinterpret_cast<double*>(smem_raw + stream_smem<kTma>(nwarp, rows));
   unsigned int* s_cnt = reinterpret_cast<unsigned int*>(s_amt + G);
   unsigned int* s_qty = s_cnt + G;
   for (uint32_t g = threadIdx.x; g < G; g += blockDim.x) { s_amt[g] = 0.0; s_cnt[g] = 0; s_qty[g] = 0; }
   __syncthreads();
-  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t - threadIdx.x < c.L; t += gridDim.x * blockDim.x) {
-    if (t < c.L) {
-      const LaneDesc d = lanes[t];
-      const uint8_t* tile = stage + tile_base[t >> 5];
-      for (uint32_t j = 0; j < d.nrec; ++j) {
-        const uint4 v = lane_word(tile, j, t & 31);
-        const uint32_t key = v.x;
-        if (key >= G) { atomicOr(err, kErrKeyRange); continue; }
-        const double amt = __hiloint2double((int)v.w, (int)v.z);
-        atomicAdd(&s_cnt[key], 1u);
-        atomicAdd(&s_qty[key], v.y);
-        atomicAdd(&s_amt[key], amt);
-      }
+  ts.begin(blockIdx.x * nwarp + wid);
+  while (ts.valid()) {
+    const uint32_t nrec = lanes[(size_t)ts.w * 32 + lane].nrec;
+    uint32_t nw, np, nK;
+    const uint8_t* piece = ts.acquire(nw, np, nK);
+    const uint32_t r0 = ts.p * rows;
+    const uint32_t r1 = min(min(ts.K, r0 + rows), nrec);
+    for (uint32_t r = r0; r < r1; ++r) {
+      const uint4 v = *reinterpret_cast<const uint4*>(piece + (size_t)(r - r0) * 512 + lane * 16);
+      const uint32_t key = v.x;
+      if (key >= G) { atomicOr(err, kErrKeyRange); continue; }
+      const double amt = __hiloint2double((int)v.w, (int)v.z);
+      atomicAdd(&s_cnt[key], 1u);
+      atomicAdd(&s_qty[key], v.y);
+      atomicAdd(&s_amt[key], amt);
     }
+    ts.release(nw, np, nK);
   }
   __syncthreads();
   for (uint32_t g = threadIdx.x; g < G; g += blockDim.x) {
@@ -527,29 +538,66 @@ __global__ void __launch_bounds__(256) k_groupby(Chunk c, const uint8_t* __restr
 // order of DESIGN.md reading A13 (__fsub_rn, __fmaf_rn, j ascending), argmin with ties to the
 // lowest k; per-block shared sums (fp64) and counts, flushed once per block.
 
-__global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restrict__ stage,
-                                                const LaneDesc* __restrict__ lanes,
-                                                const uint64_t* __restrict__ tile_base,
-                                                const float* __restrict__ mu, uint32_t K, uint64_t first_index,
-                                                unsigned long long* gcount, double* gsum,
-                                                unsigned long long* gchk, int32_t* __restrict__ cid_out) {
-  extern __shared__ unsigned char smem_raw[];
-  double* s_sum = reinterpret_cast<double*>(smem_raw);          // K*16
-  float* s_mu = reinterpret_cast<float*>(s_sum + (size_t)K * 16);  // K*16
+// Each warp streams its tiles through shared memory (WarpTileStream, 2 points per piece) and
+// evaluates four centroids at a time: four independent fmaf chains, each in the order of A13,
+// compared in ascending k afterwards, so the argmin (ties to the lowest k) is bit-identical to
+// the one-centroid-at-a-time loop while the FMA pipes see four chains to interleave.
+constexpr int kKmThreads = 512;
+constexpr uint32_t kKmRows = 8;   // rows per piece: 2 points of 4 words
+
+// Exact fp32 -> fp64 widening with integer ops for normal numbers and zeros (rebias the exponent,
+// shift the mantissa); subnormals, infinities and NaNs take the conversion instruction. ncu showed
+// the 16 conversions per point saturating the XU pipe (122% of its sustained rate) in k_kmeans.
+__device__ __forceinline__ double widen(float f) {
+  const uint32_t u = __float_as_uint(f);
+  const uint32_t e = (u >> 23) & 0xffu;
+  const uint64_t sign = (uint64_t)(u >> 31) << 63;
+  if (e - 1u < 0xfeu)
+    return __longlong_as_double((long long)(sign | ((uint64_t)(e + 896u) << 52) | ((uint64_t)(u & 0x7fffffu) << 29)));
+  if ((u << 1) == 0) return __longlong_as_double((long long)sign);
+  return (double)f;
+}
+
+__device__ __forceinline__ float km_dist(const float* x, const float* m) {
+  float acc = 0.0f;
+#pragma unroll
+  for (int q = 0; q < 16; ++q) {
+    const float df = __fsub_rn(x[q], m[q]);
+    acc = __fmaf_rn(df, df, acc);
+  }
+  return acc;
+}
+
+template <bool kTma>
+__global__ void __launch_bounds__(kKmThreads) k_kmeans(Chunk c, const uint8_t* __restrict__ stage,
+                                                       const LaneDesc* __restrict__ lanes,
+                                                       const uint64_t* __restrict__ tile_base,
+                                                       const float* __restrict__ mu, uint32_t K, uint64_t first_index,
+                                                       unsigned long long* gcount, double* gsum,
+                                                       unsigned long long* gchk, int32_t* __restrict__ cid_out) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  constexpr uint32_t nwarp = kKmThreads / 32;
+  const uint32_t wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  WarpTileStream<kTma> ts = warp_stream<kTma>(smem_raw, nwarp, kKmRows, stage, tile_base, c.ntiles);
+  double* s_sum = reinterpret_cast<double*>(smem_raw + stream_smem<kTma>(nwarp, kKmRows));   // K*16
+  float* s_mu = reinterpret_cast<float*>(s_sum + (size_t)K * 16);                             // K*16
   unsigned int* s_cnt = reinterpret_cast<unsigned int*>(s_mu + (size_t)K * 16);
   for (uint32_t i = threadIdx.x; i < K * 16; i += blockDim.x) { s_sum[i] = 0.0; s_mu[i] = mu[i]; }
   for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) s_cnt[i] = 0;
   __syncthreads();
   unsigned long long chk = 0;
-  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t - threadIdx.x < c.L; t += gridDim.x * blockDim.x) {
-    if (t >= c.L) continue;
-    const LaneDesc d = lanes[t];
-    const uint8_t* tile = stage + tile_base[t >> 5];
-    for (uint32_t j = 0; j < d.nrec; ++j) {
+  ts.begin(blockIdx.x * nwarp + wid);
+  while (ts.valid()) {
+    const LaneDesc d = lanes[(size_t)ts.w * 32 + lane];
+    uint32_t nw, np, nK;
+    const uint8_t* piece = ts.acquire(nw, np, nK);
+    const uint32_t r0 = ts.p * kKmRows;
+    const uint32_t j1 = min(min(ts.K, r0 + kKmRows) / 4, d.nrec);
+    for (uint32_t j = r0 / 4; j < j1; ++j) {
       float x[16];
 #pragma unroll
       for (int w = 0; w < 4; ++w) {
-        const uint4 v = lane_word(tile, 4 * j + w, t & 31);
+        const uint4 v = *reinterpret_cast<const uint4*>(piece + (size_t)(4 * j + w - r0) * 512 + lane * 16);
         x[4 * w + 0] = __uint_as_float(v.x);
         x[4 * w + 1] = __uint_as_float(v.y);
         x[4 * w + 2] = __uint_as_float(v.z);
@@ -557,21 +605,28 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
       }
       uint32_t best = 0;
       float bestd = 0.0f;
-      for (uint32_t k = 0; k < K; ++k) {
-        float acc = 0.0f;
-#pragma unroll
-        for (int q = 0; q < 16; ++q) {
-          const float df = __fsub_rn(x[q], s_mu[k * 16 + q]);
-          acc = __fmaf_rn(df, df, acc);
-        }
-        if (k == 0 || acc < bestd) { bestd = acc; best = k; }
+      uint32_t k = 0;
+      for (; k + 4 <= K; k += 4) {
+        const float a0 = km_dist(x, s_mu + (k + 0) * 16);
+        const float a1 = km_dist(x, s_mu + (k + 1) * 16);
+        const float a2 = km_dist(x, s_mu + (k + 2) * 16);
+        const float a3 = km_dist(x, s_mu + (k + 3) * 16);
+        if (k == 0 || a0 < bestd) { bestd = a0; best = k; }
+        if (a1 < bestd) { bestd = a1; best = k + 1; }
+        if (a2 < bestd) { bestd = a2; best = k + 2; }
+        if (a3 < bestd) { bestd = a3; best = k + 3; }
+      }
+      for (; k < K; ++k) {
+        const float a0 = km_dist(x, s_mu + k * 16);
+        if (k == 0 || a0 < bestd) { bestd = a0; best = k; }
       }
       atomicAdd(&s_cnt[best], 1u);
 #pragma unroll
-      for (int q = 0; q < 16; ++q) atomicAdd(&s_sum[best * 16 + q], (double)x[q]);
+      for (int q = 0; q < 16; ++q) atomicAdd(&s_sum[best * 16 + q], widen(x[q]));
       chk += mix64(((first_index + d.first + j) << 8) ^ (uint64_t)best);
       if (cid_out) cid_out[d.first + j - c.lo] = (int32_t)best;
     }
+    ts.release(nw, np, nK);
   }
 #pragma unroll
   for (int o = 16; o; o >>= 1) chk += __shfl_xor_sync(kFull, chk, o);  // wraps mod 2^64
@@ -580,7 +635,7 @@ __global__ void __launch_bounds__(256) k_kmeans(Chunk c, const uint8_t* __restri
     if (s_sum[i] != 0.0) atomicAdd(&gsum[i], s_sum[i]);
   for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
     if (s_cnt[i]) atomicAdd(&gcount[i], (unsigned long long)s_cnt[i]);
-  if ((threadIdx.x & 31) == 0) atomicAdd(gchk, chk);
+  if (lane == 0) atomicAdd(gchk, chk);
 }
 
 }  // namespace
@@ -598,13 +653,23 @@ void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long*
   k_wc_compact<<<148 * 4, 256, 0, s>>>(table, slots, n_out, off, len, cnt, cap);
 }
 
+size_t grep_count_smem() { return stream_smem<true>(kGrepThreads / 32, kGrepRows); }
+
+// Stage 4 reads the tiles through TMA bulk copies (persistent warps, double-buffered pieces) unless
+// zero-copy gathers share the chunk's run (`tma` false): then plain loads, one tile per warp.
 void launch_grep(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
-                 const GrepParams& p, uint32_t* blkcnt, unsigned long long* cursor, unsigned long long* blkbase,
-                 unsigned long long* chunk_run, uint64_t* out_idx, int* err, cudaStream_t s) {
-  const uint32_t nblk = (c.L + 255) / 256;
-  k_grep_count<<<nblk, 256, 0, s>>>(c, stage, lanes, tile_base, p, blkcnt);
-  k_grep_scan<<<1, 1024, 0, s>>>(blkcnt, nblk, cursor, blkbase, chunk_run);
-  k_grep_write<<<nblk, 256, 0, s>>>(c, stage, lanes, tile_base, p, blkbase, out_idx, err);
+                 const GrepParams& p, uint32_t* tilecnt, uint32_t* lanemask, unsigned long long* cursor,
+                 unsigned long long* tilebase_out, unsigned long long* chunk_run, uint64_t* out_idx, int* err,
+                 int grid, bool tma, cudaStream_t s) {
+  const uint32_t nwarp = kGrepThreads / 32;
+  const uint32_t tile_blocks = std::max<uint32_t>(1, (c.ntiles + nwarp - 1) / nwarp);
+  if (tma)
+    k_grep_count<true><<<std::min<int>(grid, (int)tile_blocks), kGrepThreads, grep_count_smem(), s>>>(
+        c, stage, lanes, tile_base, p, tilecnt, lanemask);
+  else
+    k_grep_count<false><<<tile_blocks, kGrepThreads, 0, s>>>(c, stage, lanes, tile_base, p, tilecnt, lanemask);
+  k_grep_scan<<<1, 1024, 0, s>>>(tilecnt, tile_base, c.ntiles, cursor, tilebase_out, chunk_run);
+  k_grep_write<<<tile_blocks, 256, 0, s>>>(c, stage, lanes, tile_base, p, tilebase_out, lanemask, out_idx, err);
 }
 
 void launch_grep_order(const unsigned long long* runs, uint32_t C, const uint64_t* pool, uint64_t* out, uint64_t cap,
@@ -612,27 +677,47 @@ void launch_grep_order(const unsigned long long* runs, uint32_t C, const uint64_
   if (C) k_grep_order<<<C, 256, 0, s>>>(runs, C, pool, out, cap);
 }
 
-size_t groupby_smem(uint32_t G) { return (size_t)G * 16; }
+size_t groupby_smem(uint32_t G, bool tma) {
+  return (tma ? stream_smem<true>(kGbThreads / 32, groupby_rows(G)) : 0) + (size_t)G * 16;
+}
 
 void launch_groupby(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                     uint32_t G, unsigned long long* count, unsigned long long* qty, double* amount, int* err,
-                    int grid, cudaStream_t s) {
-  k_groupby<<<grid, 256, groupby_smem(G), s>>>(c, stage, lanes, tile_base, G, count, qty, amount, err);
+                    int grid, bool tma, cudaStream_t s) {
+  // TMA: one 16-warp block per SM (stream buffers + table ~192 KB); plain loads: up to 3 per SM
+  grid = std::min<int>(grid, (int)std::max<uint32_t>(1, (c.ntiles + kGbThreads / 32 - 1) / (kGbThreads / 32)));
+  if (tma)
+    k_groupby<true><<<grid, kGbThreads, groupby_smem(G, true), s>>>(c, stage, lanes, tile_base, G, count, qty, amount,
+                                                                     err);
+  else
+    k_groupby<false><<<grid, kGbThreads, groupby_smem(G, false), s>>>(c, stage, lanes, tile_base, G, count, qty,
+                                                                       amount, err);
 }
 
-size_t kmeans_smem(uint32_t K) { return (size_t)K * 16 * 8 + (size_t)K * 16 * 4 + (size_t)K * 4; }
+size_t kmeans_smem(uint32_t K, bool tma) {
+  return (tma ? stream_smem<true>(kKmThreads / 32, kKmRows) : 0) + (size_t)K * 16 * 8 + (size_t)K * 16 * 4 +
+         (size_t)K * 4;
+}
 
 void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                    const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
-                   unsigned long long* chk, int32_t* cid_out, int grid, cudaStream_t s) {
-  k_kmeans<<<grid, 256, kmeans_smem(K), s>>>(c, stage, lanes, tile_base, mu, K, first_index, count, sum, chk,
-                                              cid_out);
+                   unsigned long long* chk, int32_t* cid_out, int grid, bool tma, cudaStream_t s) {
+  grid = std::min<int>(grid, (int)std::max<uint32_t>(1, (c.ntiles + kKmThreads / 32 - 1) / (kKmThreads / 32)));
+  if (tma)
+    k_kmeans<true><<<grid, kKmThreads, kmeans_smem(K, true), s>>>(c, stage, lanes, tile_base, mu, K, first_index,
+                                                                   count, sum, chk, cid_out);
+  else
+    k_kmeans<false><<<grid, kKmThreads, kmeans_smem(K, false), s>>>(c, stage, lanes, tile_base, mu, K, first_index,
+                                                                     count, sum, chk, cid_out);
 }
 
 cudaError_t configure_compute_kernels() {
-  cudaError_t e = cudaFuncSetAttribute(k_groupby, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_kmeans, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  for (const void* f : {(const void*)k_groupby<true>, (const void*)k_groupby<false>, (const void*)k_kmeans<true>,
+                        (const void*)k_kmeans<false>, (const void*)k_grep_count<true>}) {
+    const cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 }  // namespace bk

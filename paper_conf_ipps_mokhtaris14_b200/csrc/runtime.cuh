@@ -145,7 +145,7 @@ struct bk_ctx {  // the opaque context of include/bk.h
   unsigned long long* d_ctr = nullptr;  // [0] staged sum, [1] wc used, [2] wc n_out, [3] grep running, [4] kmeans chk
   // pinned mirror of d_ctr[0..7] and d_err (at [8]), copied by the run's tail before its one sync
   unsigned long long* h_ctr = nullptr;
-  bk::rt::DevBuf b_table, b_out1, b_out2, b_out3, b_blk, b_blk2, b_agg1, b_agg2, b_agg3, b_mu;
+  bk::rt::DevBuf b_table, b_out1, b_out2, b_out3, b_blk, b_blk2, b_blk3, b_agg1, b_agg2, b_agg3, b_mu;
   // CPU assembly (BK_GATHER_CPU / HYBRID): thread pool + pinned host staging ring
   bk::HostPool* pool = nullptr;
   std::vector<uint8_t*> hstage;
@@ -208,6 +208,9 @@ int prof_reserve(bk_ctx* c, size_t pairs);
 int end_host(bk_ctx* c, void* stream);
 void drop_graphs(bk_ctx* c);
 bool graphable(const Plan& p);
+// Stage 4 stages tiles through TMA bulk copies unless zero-copy gathers run alongside (ZC, HYBRID):
+// those keep the SMs' sysmem path busy and the bulk copies were measured to stall behind them.
+inline bool stage_tma(const Plan& p) { return p.mode == BK_GATHER_DENSE || p.mode == BK_GATHER_CPU; }
 int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes);
 void unregister(bk_ctx* c);
 

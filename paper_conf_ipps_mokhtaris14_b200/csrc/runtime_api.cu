@@ -281,7 +281,7 @@ int bk_destroy(bk_ctx* c) {
     if (s.ready) cudaEventDestroy(s.ready);
     if (s.freed) cudaEventDestroy(s.freed);
   }
-  for (DevBuf* b : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_agg1, &c->b_agg2,
+  for (DevBuf* b : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_blk3, &c->b_agg1, &c->b_agg2,
                     &c->b_agg3, &c->b_mu})
     b->release();
   if (c->window) cudaFree(c->window);

@@ -64,15 +64,19 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
   int rc = plan_run(c, field_access(16, 32), 256, p);
   if (rc) return rc;
   carve(c, p);
-  const uint32_t nblk = (p.L + 255) / 256;
+  const uint32_t ntl = std::max<uint32_t>(p.L / 32, 1);   // tiles per chunk (L % 32 == 0)
   const uint64_t cap = std::min<uint64_t>(o->cap, c->n);
   const size_t C = p.bounds.size() - 1;
   const uint32_t N = c->cfg.n_slots;
   BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(cap, 1) * 8));   // matches in chunk order
   BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(cap, 1) * 8));   // match pool (runs in completion order)
   BK_CUDA(c->b_out3.ensure(std::max<size_t>(C, 1) * 16));       // per chunk {pool offset, count}
-  BK_CUDA(c->b_blk.ensure((uint64_t)nblk * 4 * N));             // per slot: block counts
-  BK_CUDA(c->b_blk2.ensure((uint64_t)nblk * 8 * N));            // per slot: block bases
+  BK_CUDA(c->b_blk.ensure((uint64_t)ntl * 4 * N));              // per slot: tile match counts
+  BK_CUDA(c->b_blk2.ensure((uint64_t)ntl * 8 * N));             // per slot: tile output bases
+  BK_CUDA(c->b_blk3.ensure((uint64_t)ntl * 32 * 4 * N));        // per slot: lane match masks
+  int dev_sms = 148;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  const int grid = dev_sms * 2;   // 2 x 8-warp blocks per SM stream the tiles (64 KB smem each)
   GrepParams gp{};
   if (o->pattern_len) memcpy(gp.pat, o->pattern, o->pattern_len);
   gp.plen = o->pattern_len;
@@ -85,9 +89,9 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
     size_t ci = 0;
     int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
       const size_t k = ci % N;   // slot of this chunk: its block counts/bases are private to it
-      launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p + k * nblk, c->d_ctr + 3,
-                  (unsigned long long*)c->b_blk2.p + k * nblk, (unsigned long long*)c->b_out3.p + 2 * ci,
-                  (uint64_t*)c->b_out2.p, c->d_err, cs);
+      launch_grep(ch, s.stage, s.lanes, s.tile_base, gp, (uint32_t*)c->b_blk.p + k * ntl,
+                  (uint32_t*)c->b_blk3.p + k * ntl * 32, c->d_ctr + 3, (unsigned long long*)c->b_blk2.p + k * ntl,
+                  (unsigned long long*)c->b_out3.p + 2 * ci, (uint64_t*)c->b_out2.p, c->d_err, grid, stage_tma(p), cs);
       ++ci;
       c->n_launch += 3;
       return BK_OK;
@@ -122,8 +126,9 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
   BK_CUDA(c->b_agg3.ensure((uint64_t)G * 8));
   int dev_sms = 148, per_sm = 1;
   cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
-  per_sm = std::max<int>(1, (int)((200 * 1024) / std::max<size_t>(groupby_smem(G), 1)));
-  per_sm = std::min(per_sm, 4);
+  const bool tma = stage_tma(p);
+  per_sm = std::max<int>(1, (int)((220 * 1024) / std::max<size_t>(groupby_smem(G, tma), 1)));
+  per_sm = std::min(per_sm, 3);
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * per_sm));
   rc = run_device(c, stream, "groupby/" + std::to_string(G) + "/" + p.key, graphable(p), p.bounds.size() - 1,
                   [&]() -> int {
@@ -132,7 +137,7 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
     BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)G * 8, c->s_comp));
     return pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
       launch_groupby(ch, s.stage, s.lanes, s.tile_base, G, (unsigned long long*)c->b_agg1.p,
-                     (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, cs);
+                     (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, grid, tma, cs);
       c->n_launch += 1;
       return BK_OK;
     });
@@ -165,7 +170,8 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
   if (!c->h_mu) BK_CUDA(cudaHostAlloc((void**)&c->h_mu, 256 * 64, cudaHostAllocPortable));
   memcpy(c->h_mu, o->centroids, (size_t)K * 64);   // the graph copies from this pinned buffer
-  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * 2));
+  const bool tma = stage_tma(p);   // TMA: one 16-warp block per SM; plain loads: two
+  const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * (tma ? 1 : 2)));
   const std::string key = "kmeans/" + std::to_string(K) + "/" + std::to_string(o->first_index) + "/" +
                           std::to_string((uintptr_t)o->cid) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
@@ -176,7 +182,7 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
     return pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {
       launch_kmeans(ch, s.stage, s.lanes, s.tile_base, (const float*)c->b_mu.p, K, o->first_index,
                     (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4,
-                    o->cid ? (int32_t*)s.out : nullptr, grid, cs);
+                    o->cid ? (int32_t*)s.out : nullptr, grid, tma, cs);
       c->n_launch += 1;
       if (o->cid && ch.hi > ch.lo) {  // write-back of this chunk's cids, full duplex with the H2D stream
         cudaEvent_t e = c->ev_part[ci++ % c->ev_part.size()];

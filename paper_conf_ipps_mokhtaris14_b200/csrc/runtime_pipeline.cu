@@ -182,6 +182,9 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     BK_PROF(kStGather, ss, false);
     c->n_launch += 3;
     c->st.bytes_h2d += ch.accessed;
+    c->st.n_chunks_zc += 1;
+    c->st.bytes_zc += ch.accessed;
+    c->st.records_zc += ch.hi - ch.lo;
     BK_CUDA(cudaEventRecord(s.ready, ss));
   } else {
     if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
@@ -252,6 +255,7 @@ int begin_run(bk_ctx* c, void* stream) {
   c->st.bytes_accessed = c->st.bytes_h2d = c->st.bytes_meta = c->st.bytes_padding = c->st.bytes_d2h = 0;
   c->st.n_chunks_cpu = 0;
   c->st.ms_cpu_gather = 0;
+  c->st.n_chunks_zc = c->st.bytes_zc = c->st.records_zc = 0;
   return BK_OK;
 }
 
@@ -295,6 +299,10 @@ int stage_stats(bk_ctx* c) {
   c->st.ms_gather = acc[kStGather] + acc[kStRelayout];
   c->st.ms_compute = acc[kStCompute];
   c->st.n_gather = cnt[kStGather] + cnt[kStRelayout];
+  c->st.ms_zc = acc[kStGather];
+  c->st.n_zc = cnt[kStGather];
+  c->st.ms_relayout = acc[kStRelayout];
+  c->st.n_relayout = cnt[kStRelayout];
   c->st.ms_xfer_busy = bx;
   c->st.ms_compute_busy = bc;
   c->st.ms_overlap = ov;
@@ -335,6 +343,7 @@ void host_reset(bk_ctx* c) {
   c->st.bytes_accessed = c->st.bytes_h2d = c->st.bytes_meta = c->st.bytes_padding = c->st.bytes_d2h = 0;
   c->st.n_chunks_cpu = 0;
   c->st.ms_cpu_gather = 0;
+  c->st.n_chunks_zc = c->st.bytes_zc = c->st.records_zc = 0;
 }
 
 int prof_reserve(bk_ctx* c, size_t pairs) {

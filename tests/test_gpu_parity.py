@@ -156,6 +156,20 @@ def test_grep_medium(mode):
         assert 0 < st["n_chunks_cpu"] < st["n_chunks"]
 
 
+@pytest.mark.parametrize("lane_bytes", [1024, 1056, 4096])
+def test_grep_long_lanes(lane_bytes):
+    """Lanes of 32, 33 and 128 keys: k_grep_count keeps a 32-record match mask per lane; longer
+    lanes are re-tested from the staged keys by k_grep_write. Same indices as the oracle."""
+    buf, off = gen.grep_records(n=60_000)
+    for pat in (b"bigk", b"", b"a"):
+        want = oracle.grep(buf, off, pat, first=5)
+        for mode in ("zc", "hybrid"):
+            with bk.Context(window_bytes=8 * MIB, gather_mode=mode, lane_bytes=lane_bytes) as ctx:
+                ctx.register(buf, off)
+                got = ctx.grep(pat, first_index=5, cap=len(off))
+            assert np.array_equal(got, want), (pat, mode, lane_bytes)
+
+
 def test_grep_capacity_error():
     buf, off = gen.grep_records(n=20000)
     with bk.Context(window_bytes=4 * MIB) as ctx:
@@ -193,6 +207,20 @@ def test_groupby(stride, zipf, mode):
     np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
 
 
+@pytest.mark.parametrize("G,mode", [(8192, "dense"), (1, "dense"), (8192, "zc"), (4097, "cpu")])
+def test_groupby_group_counts(G, mode):
+    """Table sizes at the edges: G = 8192 halves the TMA pieces (4 rows) to fit the shared table,
+    G = 1 sends every record to one slot; both load paths (TMA in dense/cpu, plain loads in zc)."""
+    n = 1_000_003
+    buf = gen.groupby(n=n, G=G)
+    wc_, wq, wa = oracle.groupby(buf, n, 16, G)
+    with bk.Context(window_bytes=8 * MIB, gather_mode=mode, record_size=16) as ctx:
+        ctx.register(buf, None, n_records=n)
+        c, q, a = ctx.groupby(G)
+    assert np.array_equal(c, wc_) and np.array_equal(q, wq)
+    np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
+
+
 def test_groupby_key_out_of_range():
     buf = gen.groupby(n=1000, G=4096)
     with bk.Context(window_bytes=1 * MIB, record_size=16) as ctx:
@@ -203,7 +231,8 @@ def test_groupby_key_out_of_range():
 
 
 # ------------------------------------------------------------------ C3 k-means
-@pytest.mark.parametrize("mode,K", [("dense", 64), ("zc", 64), ("dense", 7), ("cpu", 64), ("hybrid", 33)])
+@pytest.mark.parametrize("mode,K", [("dense", 64), ("zc", 64), ("dense", 7), ("cpu", 64), ("hybrid", 33),
+                                    ("dense", 1), ("cpu", 256), ("zc", 255)])
 def test_kmeans(mode, K):
     n = 400_003
     x = gen.points(n=n)
