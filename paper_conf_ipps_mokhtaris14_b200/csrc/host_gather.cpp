@@ -204,13 +204,13 @@ uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, c
 bool host_packable(const Access& a) { return !a.whole && a.n_ext == 1 && a.E > 0 && (a.E % 16) == 0; }
 
 uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* dst,
-                         uint64_t cap) {
+                         uint64_t cap, uint64_t grab, bool nt, const std::function<void(uint64_t, uint64_t)>* sink) {
   const uint64_t E = a.E, n = c.hi - c.lo, size = n * E;
   if (size > cap) return UINT64_MAX;
   const uint32_t eo = a.ext_off[0], EW = (uint32_t)(E / 16);
   // sweep on the 16-core host (profiles/r01_hybrid_sweep.md): 16-record prefetch distance, grabs of
-  // 4k-16k records; non-temporal vs regular stores are equal inside the pipeline
-  constexpr uint64_t kGrab = 16384;   // records per grab: a few MB of the data set, read in order
+  // 4k-16k records read in order
+  const uint64_t kGrab = grab ? grab : 16384;
   constexpr uint64_t kPf = 16;        // software prefetch distance (records)
   std::atomic<uint64_t> next{0};
   pool.run([&](int) {
@@ -220,12 +220,23 @@ uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, con
       if (j0 >= n) break;
       const uint64_t j1 = std::min(n, j0 + kGrab);
       for (uint64_t j = j0; j < std::min(j1, j0 + kPf); ++j) __builtin_prefetch(src(c.lo + j));
-      for (uint64_t j = j0; j < j1; ++j) {
-        if (j + kPf < j1) __builtin_prefetch(src(c.lo + j + kPf));
-        const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
-        __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
-        for (uint32_t m = 0; m < EW; ++m) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
+      if (nt) {
+        for (uint64_t j = j0; j < j1; ++j) {
+          if (j + kPf < j1) __builtin_prefetch(src(c.lo + j + kPf));
+          const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
+          __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
+          for (uint32_t m = 0; m < EW; ++m) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
+        }
+        if (sink) _mm_sfence();
+      } else {
+        for (uint64_t j = j0; j < j1; ++j) {
+          if (j + kPf < j1) __builtin_prefetch(src(c.lo + j + kPf));
+          const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
+          __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
+          for (uint32_t m = 0; m < EW; ++m) _mm_storeu_si128(o + m, _mm_loadu_si128(s + m));
+        }
       }
+      if (sink) (*sink)(j0 * E, (j1 - j0) * E);
     }
     _mm_sfence();
   });

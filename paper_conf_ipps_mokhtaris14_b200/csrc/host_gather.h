@@ -53,8 +53,12 @@ uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, c
 // order, E bytes per record, into dst (16-B aligned) — a sequential read of the data set and a
 // sequential non-temporal write, the cheapest host gather there is. The warp-tile interleave is then
 // done on the GPU (HBM -> HBM). Returns (hi - lo) * E, or UINT64_MAX if that exceeds cap.
+// `grab` records per work item (0 = default); `nt`: non-temporal stores; `sink(byte_off, bytes)`, if
+// set, is called by the packing thread as soon as a grab's bytes are in dst (e.g. to DMA them while
+// they are still in the host's caches).
 bool host_packable(const Access& a);
 uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* dst,
-                         uint64_t cap);
+                         uint64_t cap, uint64_t grab = 0, bool nt = true,
+                         const std::function<void(uint64_t, uint64_t)>* sink = nullptr);
 
 }  // namespace bk

@@ -2,6 +2,7 @@
 # Round evidence: GPU tests, every bench line, ncu launch lists and one --set full capture per top kernel.
 mkdir -p gpurun_out
 TAG=${TAG:-r01z}
+{ lscpu; free -g; nproc; } > gpurun_out/${TAG}_host.txt 2>&1
 timeout 900 python -m pytest tests -m gpu -q --timeout 600 --tb=short -p no:cacheprovider > gpurun_out/${TAG}_gpu_tests.log 2>&1
 tail -2 gpurun_out/${TAG}_gpu_tests.log
 timeout 900 python bench.py > gpurun_out/${TAG}_bench_grep.json 2> gpurun_out/${TAG}_bench_grep.err
