@@ -135,6 +135,9 @@ void launch_dbuf_grep(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uin
 void launch_dbuf_groupby(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t base_byte, uint64_t rec_size,
                          uint32_t G, unsigned long long* count, unsigned long long* qty, double* amount, int* err,
                          cudaStream_t s);
+void launch_dbuf_kmeans(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t base_byte, uint64_t rec_size,
+                        const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
+                        unsigned long long* chk, cudaStream_t s);
 cudaError_t configure_baseline_kernels();
 
 // ---- f4: k-mer counting over DNA reads (kernels_kmer.cu) ----

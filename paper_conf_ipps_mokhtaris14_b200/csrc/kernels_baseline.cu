@@ -129,9 +129,62 @@ __global__ void __launch_bounds__(256) k_dbuf_groupby(RawChunk c, uint32_t G, un
     }
 }
 
+// K-means step on raw 64-B+ records (16 fp32 at +0), thread per contiguous record range, the
+// distance / argmin / accumulation rules of k_kmeans (A13) on the original AoS layout.
+__global__ void __launch_bounds__(256) k_dbuf_kmeans(RawChunk c, const float* __restrict__ mu, uint32_t K,
+                                                     uint64_t first_index, unsigned long long* gcount, double* gsum,
+                                                     unsigned long long* gchk) {
+  extern __shared__ unsigned char smem_raw[];
+  double* s_sum = reinterpret_cast<double*>(smem_raw);
+  float* s_mu = reinterpret_cast<float*>(s_sum + (size_t)K * 16);
+  unsigned int* s_cnt = reinterpret_cast<unsigned int*>(s_mu + (size_t)K * 16);
+  for (uint32_t i = threadIdx.x; i < K * 16; i += blockDim.x) { s_sum[i] = 0.0; s_mu[i] = mu[i]; }
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) s_cnt[i] = 0;
+  __syncthreads();
+  uint64_t a, b;
+  my_range(c, a, b);
+  unsigned long long chk = 0;
+  for (uint64_t r = a; r < b; ++r) {
+    const float4* p = reinterpret_cast<const float4*>(c.raw + rstart(c, r));
+    float x[16];
+    for (int w = 0; w < 4; ++w) {
+      const float4 v = p[w];
+      x[4 * w] = v.x; x[4 * w + 1] = v.y; x[4 * w + 2] = v.z; x[4 * w + 3] = v.w;
+    }
+    uint32_t best = 0;
+    float bestd = 0.0f;
+    for (uint32_t k = 0; k < K; ++k) {
+      float acc = 0.0f;
+      for (int q = 0; q < 16; ++q) {
+        const float df = __fsub_rn(x[q], s_mu[k * 16 + q]);
+        acc = __fmaf_rn(df, df, acc);
+      }
+      if (k == 0 || acc < bestd) { bestd = acc; best = k; }
+    }
+    atomicAdd(&s_cnt[best], 1u);
+    for (int q = 0; q < 16; ++q) atomicAdd(&s_sum[best * 16 + q], (double)x[q]);
+    chk += mix64(((first_index + r) << 8) ^ (uint64_t)best);
+  }
+  for (int o = 16; o; o >>= 1) chk += __shfl_xor_sync(kFull, chk, o);
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < K * 16; i += blockDim.x)
+    if (s_sum[i] != 0.0) atomicAdd(&gsum[i], s_sum[i]);
+  for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
+    if (s_cnt[i]) atomicAdd(&gcount[i], (unsigned long long)s_cnt[i]);
+  if ((threadIdx.x & 31) == 0) atomicAdd(gchk, chk);
+}
+
 }  // namespace
 
 uint32_t dbuf_blocks() { return 148 * 4; }
+
+void launch_dbuf_kmeans(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t base_byte, uint64_t rec_size,
+                        const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,
+                        unsigned long long* chk, cudaStream_t s) {
+  RawChunk c{raw, nullptr, lo, hi, base_byte, hi * rec_size, rec_size};
+  const size_t smem = (size_t)K * 16 * 12 + (size_t)K * 4;
+  k_dbuf_kmeans<<<dbuf_blocks(), 256, smem, s>>>(c, mu, K, first_index, count, sum, chk);
+}
 
 void launch_dbuf_grep(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
                       uint64_t end_byte, uint64_t rec_size, const GrepParams& p, uint32_t* blkcnt,
@@ -154,7 +207,9 @@ void launch_dbuf_groupby(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t 
 }
 
 cudaError_t configure_baseline_kernels() {
-  return cudaFuncSetAttribute(k_dbuf_groupby, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  const cudaError_t e = cudaFuncSetAttribute(k_dbuf_groupby, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_dbuf_kmeans, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
 }
 
 }  // namespace bk

@@ -7,7 +7,6 @@
 #include "tma.cuh"
 
 #include <algorithm>
-#include <cstdlib>
 
 namespace bk {
 namespace {

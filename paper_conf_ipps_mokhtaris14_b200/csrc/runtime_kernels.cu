@@ -310,7 +310,8 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
 
 // ---- BK_FLAG_BASELINE_DBUF: the traditional chunked loop with two buffers ----
 int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
-  if (kid != BK_K_GREP && kid != BK_K_GROUPBY) return fail(BK_E_UNSUPPORTED, "dbuf baseline: grep / group-by only");
+  if (kid != BK_K_GREP && kid != BK_K_GROUPBY && kid != BK_K_KMEANS)
+    return fail(BK_E_UNSUPPORTED, "dbuf baseline: grep / group-by / k-means only");
   Plan p;
   p.a = whole_access();
   p.mode = BK_GATHER_DENSE;
@@ -339,8 +340,17 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
   GrepParams gp{};
   bk_out_grep* og = (bk_out_grep*)out;
   bk_out_groupby* ob = (bk_out_groupby*)out;
+  bk_out_kmeans* ok = (bk_out_kmeans*)out;
   const uint32_t nb = dbuf_blocks();
-  if (kid == BK_K_GREP) {
+  if (kid == BK_K_KMEANS) {
+    if (ok->K == 0 || ok->K > 256 || !ok->centroids) return fail(BK_E_INVAL, "K must be in 1..256 with centroids");
+    if (ok->cid) return fail(BK_E_UNSUPPORTED, "dbuf baseline: no k-means cid write-back");
+    if (c->off || c->cfg.record_size < 64) return fail(BK_E_INVAL, "k-means needs fixed records >= 64 B");
+    BK_CUDA(c->b_mu.ensure((uint64_t)ok->K * 64));
+    BK_CUDA(c->b_agg1.ensure((uint64_t)ok->K * 8));
+    BK_CUDA(c->b_agg3.ensure((uint64_t)ok->K * 16 * 8));
+    BK_CUDA(cudaMemcpy(c->b_mu.p, ok->centroids, (uint64_t)ok->K * 64, cudaMemcpyHostToDevice));
+  } else if (kid == BK_K_GREP) {
     if (og->pattern_len > 32) return fail(BK_E_INVAL, "pattern longer than 32 bytes");
     if (c->min_rec < 48) return fail(BK_E_INVAL, "grep needs records of >= 48 bytes");
     if (og->pattern_len) memcpy(gp.pat, og->pattern, og->pattern_len);
@@ -358,10 +368,12 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     BK_CUDA(c->b_agg3.ensure((uint64_t)ob->G * 8));
   }
   if ((rc = begin_run(c, stream))) return rc;
-  if (kid == BK_K_GROUPBY) {
-    BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)ob->G * 8, c->s_comp));
-    BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)ob->G * 8, c->s_comp));
-    BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+  if (kid == BK_K_GROUPBY || kid == BK_K_KMEANS) {
+    const uint64_t n1 = kid == BK_K_GROUPBY ? (uint64_t)ob->G * 8 : (uint64_t)ok->K * 8;
+    const uint64_t n3 = kid == BK_K_GROUPBY ? (uint64_t)ob->G * 8 : (uint64_t)ok->K * 128;
+    BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, n1, c->s_comp));
+    if (kid == BK_K_GROUPBY) BK_CUDA(cudaMemsetAsync(c->b_agg2.p, 0, (uint64_t)ob->G * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(c->b_agg3.p, 0, n3, c->s_comp));
     BK_CUDA(cudaEventRecord(c->ev_begin, c->s_comp));
     BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->ev_begin, 0));
     BK_CUDA(cudaStreamWaitEvent(c->s_asm, c->ev_begin, 0));
@@ -393,6 +405,10 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
                        (uint64_t*)c->b_out1.p, st);
       BK_CUDA(cudaEventRecord(scanned[b], st));
       c->n_launch += 3;
+    } else if (kid == BK_K_KMEANS) {
+      launch_dbuf_kmeans(buf[b] + raw_off, lo, hi, base, c->cfg.record_size, (const float*)c->b_mu.p, ok->K,
+                         ok->first_index, (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4, st);
+      c->n_launch += 1;
     } else {
       launch_dbuf_groupby(buf[b] + raw_off, lo, hi, base, c->cfg.record_size, ob->G, (unsigned long long*)c->b_agg1.p,
                           (unsigned long long*)c->b_agg2.p, (double*)c->b_agg3.p, c->d_err, st);
@@ -411,6 +427,10 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     og->n_match = m;
     if (m > og->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)og->cap);
     if (m) BK_CUDA(cudaMemcpy(og->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));
+  } else if (kid == BK_K_KMEANS) {
+    BK_CUDA(cudaMemcpy(ok->count, c->b_agg1.p, (uint64_t)ok->K * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(ok->sum, c->b_agg3.p, (uint64_t)ok->K * 128, cudaMemcpyDeviceToHost));
+    ok->chk = c->h_ctr[4];
   } else {
     BK_CUDA(cudaMemcpy(ob->count, c->b_agg1.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
     BK_CUDA(cudaMemcpy(ob->qty, c->b_agg2.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));

@@ -289,6 +289,23 @@ def test_partition_duplicate_keys_and_errors():
 
 
 # ------------------------------------------------------------------ the double-buffering baseline
+@pytest.mark.parametrize("sbuf", [False, True])
+def test_dbuf_baseline_kmeans_matches_oracle(sbuf):
+    """The k-means double- (and single-) buffering baseline: same counts, checksum and sums (I2)."""
+    n, K = 300_007, 64
+    x = gen.points(n=n)
+    mu = x[:K].copy()
+    wc_, ws, wchk, _ = oracle.kmeans(x, mu, first=3)
+    with bk.Context(window_bytes=4 * MIB, baseline_dbuf=not sbuf, baseline_sbuf=sbuf, record_size=64) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=n)
+        c, s, chk = ctx.kmeans(mu, first_index=3)
+        assert ctx.stats()["n_chunks"] >= 4
+        with pytest.raises(bk.BkError):   # no cid write-back in the baseline
+            ctx.kmeans(mu, cid=np.empty(n, np.int32))
+    assert np.array_equal(c, wc_) and chk == wchk
+    np.testing.assert_allclose(s, ws, rtol=1e-5, atol=0)
+
+
 def test_dbuf_baseline_grep_and_groupby_match_oracle():
     """BK_FLAG_BASELINE_DBUF (the paper's variant iv) must give the same results (I2)."""
     buf, off = gen.grep_records(max_bytes=24 * MIB)
