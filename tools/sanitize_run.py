@@ -54,3 +54,17 @@ with bk.Context(window_bytes=256 << 10) as ctx:
     ctx.register(buf, off)
     ctx.pattern_stats(elem_bytes=1, T=8)
 print("sanitize run done")
+# TMA-staged stage 4 (dense / cpu), grep masks with long lanes, G = 8192 tables, k-means dbuf baseline
+g16 = gen.groupby(n=200_000, G=8192)
+for mode in ("dense", "cpu", "zc"):
+    with bk.Context(window_bytes=1 << 20, record_size=16, gather_mode=mode) as ctx:
+        ctx.register(g16, None, n_records=200_000)
+        ctx.groupby(8192)
+for mode in ("cpu", "zc"):
+    with bk.Context(window_bytes=1 << 20, gather_mode=mode, lane_bytes=4096) as ctx:
+        ctx.register(gb, goff)
+        ctx.grep(b"a", cap=20000)
+with bk.Context(window_bytes=512 << 10, record_size=64, baseline_dbuf=True) as ctx:
+    ctx.register(x.view(np.uint8).reshape(-1), None, n_records=50_000)
+    ctx.kmeans(x[:7])
+print("sanitize run ok")
