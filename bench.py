@@ -545,7 +545,8 @@ def main():
     }
     if args.impl != "ours":
         line["impl"] = args.impl
-    if args.workload in ("grep", "groupby", "groupby_sparse", "kmeans") and not args.no_dbuf and args.impl == "ours":
+    if args.workload in ("grep", "groupby", "groupby_sparse", "kmeans", "wordcount") and not args.no_dbuf and \
+            args.impl == "ours":
         # the paper's GPU double-buffering baseline (variant iv) on the same data, window and box
         dctx = bk.Context(device=local, window_bytes=window, baseline_dbuf=True, profile=False,
                           record_size=shard["rec_size"])
@@ -557,6 +558,8 @@ def main():
                 dctx.grep(b"bigk", first_index=shard["first"], stream=stream.cuda_stream, out=idx_out)
             elif args.workload == "kmeans":
                 dctx.kmeans(shard["mu"], first_index=shard["first"], stream=stream.cuda_stream)
+            elif args.workload == "wordcount":
+                dctx.wordcount(stream=stream.cuda_stream, out=wc_out)
             else:
                 dctx.groupby(4096, stream=stream.cuda_stream)
 

@@ -91,7 +91,7 @@ typedef struct bk_config {
 #define BK_FLAG_BASELINE_DBUF 2u  /* run the paper's GPU double-buffering baseline instead (P:329-339,
                                      P:994-996): raw whole-record chunks into 2 buffers (window/2 each)
                                      on 2 streams, kernel over contiguous per-thread record ranges.
-                                     BK_K_GREP, BK_K_GROUPBY and BK_K_KMEANS (no cid write-back:
+                                     BK_K_WORDCOUNT, BK_K_GREP, BK_K_GROUPBY and BK_K_KMEANS (no cid write-back:
                                      BK_E_UNSUPPORTED) only; results identical. */
 #define BK_FLAG_NO_GRAPH 8u  /* issue every pipeline eagerly instead of capturing/replaying a CUDA graph
                                (ZC / DENSE pipelines are otherwise captured on their first run per

@@ -83,6 +83,10 @@ struct WcEntry {            // 32 B open-addressing slot
 void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask,
                unsigned long long* used, int* err, cudaStream_t s);
+// double-buffering baseline (variant iv): raw chunk bytes start at absolute offset base_byte
+void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
+                    uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
+                    int* err, cudaStream_t s);
 void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,
                        uint32_t* len, uint64_t* cnt, uint64_t cap, cudaStream_t s);
 

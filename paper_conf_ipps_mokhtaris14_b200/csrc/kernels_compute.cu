@@ -259,6 +259,45 @@ __global__ void __launch_bounds__(kWcBlock) k_wc(Chunk c, const uint8_t* __restr
   }
 }
 
+// The paper's double-buffering baseline for word count (variant iv): the
+// same word identity and table as k_wc, but each thread scans a contiguous record range of the
+// raw DMA'd chunk (AoS text) byte by byte and inserts every word into the global table
+// directly — no lane layout, no block pre-aggregation.
+__global__ void __launch_bounds__(256) k_dbuf_wc(const uint8_t* __restrict__ raw, const uint64_t* __restrict__ meta,
+                                                 uint64_t lo, uint64_t hi, uint64_t base_byte, uint64_t end_byte,
+                                                 uint64_t rec_size, WcEntry* table, uint64_t mask,
+                                                 unsigned long long* used, int* err) {
+  const uint64_t T = (uint64_t)gridDim.x * blockDim.x, t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  const uint64_t n = hi - lo, a = lo + n * t / T, b = lo + n * (t + 1) / T;
+  auto rstart = [&](uint64_t r) -> uint64_t {   // absolute data-set offset of record r
+    if (!meta) return r * rec_size;
+    return r == hi ? end_byte : meta[r - lo];
+  };
+  for (uint64_t r = a; r < b; ++r) {
+    const uint64_t s0 = rstart(r), s1 = rstart(r + 1);
+    uint64_t h1 = 0, h2 = 0, wstart = 0;
+    uint32_t wlen = 0;
+    for (uint64_t pos = s0; pos <= s1; ++pos) {
+      const uint32_t ch = pos < s1 ? raw[pos - base_byte] : 0x20u;   // the record end is a delimiter
+      if (is_delim(ch)) {
+        if (wlen) {
+          if (wlen >= (1u << 24) || wstart >= (1ull << 40)) atomicOr(err, kErrWordTooLong);
+          const unsigned long long k1 = mix64(h1 ^ ((uint64_t)wlen * 0x9E3779B97F4A7C15ull)) | 1ull;
+          const unsigned long long k2 = mix64(h2 + wlen) | 1ull;
+          wc_insert(table, mask, k1, k2, (wstart << 24) | wlen, 1, used, err);
+          wlen = 0;
+        }
+        continue;
+      }
+      if (!wlen) { wstart = pos; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
+      h1 = (h1 ^ ch) * 0x100000001b3ull;
+      h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
+      h2 ^= h2 >> 29;
+      ++wlen;
+    }
+  }
+}
+
 __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, unsigned long long* n_out,
                              uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t cap) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < slots; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -645,6 +684,12 @@ void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, cons
   constexpr int kSub = 8;  // sub-threads per 256-B lane (sweep: 2/4/8/16, profiles/r01_wc_sweep.md)
   const uint32_t grid = (c.L * kSub + kWcBlock - 1) / kWcBlock;
   k_wc<kSub><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
+}
+
+void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
+                    uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
+                    int* err, cudaStream_t s) {
+  k_dbuf_wc<<<148 * 4, 256, 0, s>>>(raw, meta, lo, hi, base_byte, end_byte, rec_size, table, mask, used, err);
 }
 
 void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,

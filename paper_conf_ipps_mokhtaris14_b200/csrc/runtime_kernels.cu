@@ -310,8 +310,8 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
 
 // ---- BK_FLAG_BASELINE_DBUF: the traditional chunked loop with two buffers ----
 int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
-  if (kid != BK_K_GREP && kid != BK_K_GROUPBY && kid != BK_K_KMEANS)
-    return fail(BK_E_UNSUPPORTED, "dbuf baseline: grep / group-by / k-means only");
+  if (kid != BK_K_GREP && kid != BK_K_GROUPBY && kid != BK_K_KMEANS && kid != BK_K_WORDCOUNT)
+    return fail(BK_E_UNSUPPORTED, "dbuf baseline: word count / grep / group-by / k-means only");
   Plan p;
   p.a = whole_access();
   p.mode = BK_GATHER_DENSE;
@@ -341,8 +341,18 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
   bk_out_grep* og = (bk_out_grep*)out;
   bk_out_groupby* ob = (bk_out_groupby*)out;
   bk_out_kmeans* ok = (bk_out_kmeans*)out;
+  bk_out_wordcount* ow = (bk_out_wordcount*)out;
   const uint32_t nb = dbuf_blocks();
-  if (kid == BK_K_KMEANS) {
+  uint64_t wc_slots = 0, wc_ocap = 0;
+  if (kid == BK_K_WORDCOUNT) {
+    wc_slots = ow->table_slots ? ow->table_slots : (1ull << 20);
+    if (wc_slots & (wc_slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
+    wc_ocap = std::min<uint64_t>(ow->cap, wc_slots);
+    BK_CUDA(c->b_table.ensure(wc_slots * sizeof(WcEntry)));
+    BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(wc_ocap, 1) * 8));
+    BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(wc_ocap, 1) * 4));
+    BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(wc_ocap, 1) * 8));
+  } else if (kid == BK_K_KMEANS) {
     if (ok->K == 0 || ok->K > 256 || !ok->centroids) return fail(BK_E_INVAL, "K must be in 1..256 with centroids");
     if (ok->cid) return fail(BK_E_UNSUPPORTED, "dbuf baseline: no k-means cid write-back");
     if (c->off || c->cfg.record_size < 64) return fail(BK_E_INVAL, "k-means needs fixed records >= 64 B");
@@ -368,6 +378,12 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     BK_CUDA(c->b_agg3.ensure((uint64_t)ob->G * 8));
   }
   if ((rc = begin_run(c, stream))) return rc;
+  if (kid == BK_K_WORDCOUNT) {
+    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, wc_slots * sizeof(WcEntry), c->s_comp));
+    BK_CUDA(cudaEventRecord(c->ev_begin, c->s_comp));
+    BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->ev_begin, 0));
+    BK_CUDA(cudaStreamWaitEvent(c->s_asm, c->ev_begin, 0));
+  }
   if (kid == BK_K_GROUPBY || kid == BK_K_KMEANS) {
     const uint64_t n1 = kid == BK_K_GROUPBY ? (uint64_t)ob->G * 8 : (uint64_t)ok->K * 8;
     const uint64_t n3 = kid == BK_K_GROUPBY ? (uint64_t)ob->G * 8 : (uint64_t)ok->K * 128;
@@ -405,6 +421,10 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
                        (uint64_t*)c->b_out1.p, st);
       BK_CUDA(cudaEventRecord(scanned[b], st));
       c->n_launch += 3;
+    } else if (kid == BK_K_WORDCOUNT) {
+      launch_dbuf_wc(buf[b] + raw_off, c->off ? meta[b] : nullptr, lo, hi, base, end, c->cfg.record_size,
+                     (WcEntry*)c->b_table.p, wc_slots - 1, c->d_ctr + 1, c->d_err, st);
+      c->n_launch += 1;
     } else if (kid == BK_K_KMEANS) {
       launch_dbuf_kmeans(buf[b] + raw_off, lo, hi, base, c->cfg.record_size, (const float*)c->b_mu.p, ok->K,
                          ok->first_index, (unsigned long long*)c->b_agg1.p, (double*)c->b_agg3.p, c->d_ctr + 4, st);
@@ -420,6 +440,11 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     BK_CUDA(cudaEventRecord(c->ev_end, st));
     BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
   }
+  if (kid == BK_K_WORDCOUNT) {
+    launch_wc_compact((const WcEntry*)c->b_table.p, wc_slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p,
+                      (uint32_t*)c->b_out2.p, (uint64_t*)c->b_out3.p, wc_ocap, c->s_comp);
+    c->n_launch += 1;
+  }
   if ((rc = end_run(c, stream))) return rc;
   if (kid == BK_K_GREP) {
     unsigned long long m = 0;
@@ -427,6 +452,20 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     og->n_match = m;
     if (m > og->cap) return fail(BK_E_CAPACITY, "%llu matches > cap %llu", m, (unsigned long long)og->cap);
     if (m) BK_CUDA(cudaMemcpy(og->idx, c->b_out1.p, m * 8, cudaMemcpyDeviceToHost));
+  } else if (kid == BK_K_WORDCOUNT) {
+    const unsigned long long nw = c->h_ctr[2];
+    ow->n_words = nw;
+    if (nw > ow->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)ow->cap);
+    if (nw * 2 > wc_slots)
+      return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw, (unsigned long long)wc_slots);
+    if (nw) {
+      BK_CUDA(cudaMemcpy(ow->word_off, c->b_out1.p, nw * 8, cudaMemcpyDeviceToHost));
+      BK_CUDA(cudaMemcpy(ow->word_len, c->b_out2.p, nw * 4, cudaMemcpyDeviceToHost));
+      BK_CUDA(cudaMemcpy(ow->word_count, c->b_out3.p, nw * 8, cudaMemcpyDeviceToHost));
+    }
+    uint64_t tot = 0;
+    for (uint64_t i = 0; i < nw; ++i) tot += ow->word_count[i];
+    ow->total_words = tot;
   } else if (kid == BK_K_KMEANS) {
     BK_CUDA(cudaMemcpy(ok->count, c->b_agg1.p, (uint64_t)ok->K * 8, cudaMemcpyDeviceToHost));
     BK_CUDA(cudaMemcpy(ok->sum, c->b_agg3.p, (uint64_t)ok->K * 128, cudaMemcpyDeviceToHost));

@@ -86,11 +86,18 @@ def test_wordcount_small(mode, window, slots):
     assert got == want
 
 
-def test_wordcount_adversarial():
+def adversarial_text():
+    """Mixed delimiter runs, empty records, bytes 0x00 / >= 0x80 as word bytes, a last record
+    without a newline, a 300-byte word (SURVEY §8(c) adversarial catalogue)."""
     recs = [b"  a\tb\r\n", b"", b"", b"\x00\x80 z", b"ab", b"cd", b"tail without newline", b" ", b"x" * 300,
             b"dup dup\n"] * 37
     buf = np.frombuffer(b"".join(recs), np.uint8)
     off = np.cumsum([0] + [len(r) for r in recs[:-1]]).astype(np.uint64)
+    return buf, off
+
+
+def test_wordcount_adversarial():
+    buf, off = adversarial_text()
     want = oracle.wc(buf, off)
     for mode in ("zc", "dense", "cpu", "hybrid"):
         with bk.Context(window_bytes=64 * 1024, n_slots=2, gather_mode=mode, chunk_bytes=1500, lanes=32) as ctx:
@@ -289,6 +296,18 @@ def test_partition_duplicate_keys_and_errors():
 
 
 # ------------------------------------------------------------------ the double-buffering baseline
+@pytest.mark.parametrize("sbuf", [False, True])
+def test_dbuf_baseline_wordcount_matches_oracle(sbuf):
+    """The word-count double- (and single-) buffering baseline: the same word multiset (I2), also
+    on the adversarial text (empty records, delimiter runs, high bytes)."""
+    buf, off = gen.text(cap_bytes=3 * MIB)
+    for b, o in ((buf, off), adversarial_text()):
+        want = oracle.wc(b, o)
+        with bk.Context(window_bytes=512 * 1024, baseline_dbuf=not sbuf, baseline_sbuf=sbuf) as ctx:
+            ctx.register(b, o)
+            assert wc_multiset_gpu(b, *ctx.wordcount(cap=1 << 17)) == want
+
+
 @pytest.mark.parametrize("sbuf", [False, True])
 def test_dbuf_baseline_kmeans_matches_oracle(sbuf):
     """The k-means double- (and single-) buffering baseline: same counts, checksum and sums (I2)."""
