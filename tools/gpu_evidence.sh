@@ -1,7 +1,7 @@
 #!/bin/bash
 # Round evidence: GPU tests, every bench line, ncu launch lists and one --set full capture per top kernel.
 mkdir -p gpurun_out
-TAG=${TAG:-r01z}
+TAG=${TAG:-r01f}
 { lscpu; free -g; nproc; } > gpurun_out/${TAG}_host.txt 2>&1
 timeout 900 python -m pytest tests -m gpu -q --timeout 600 --tb=short -p no:cacheprovider > gpurun_out/${TAG}_gpu_tests.log 2>&1
 tail -2 gpurun_out/${TAG}_gpu_tests.log
@@ -14,7 +14,8 @@ for w in wordcount groupby groupby_sparse kmeans partition kmer; do
 done
 timeout 600 python bench.py --impl reference --steps 2 --warmup 3 > gpurun_out/${TAG}_bench_reference.json 2> gpurun_out/${TAG}_bench_reference.err; tail -c 300 gpurun_out/${TAG}_bench_reference.json
 B="python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-dbuf"
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches_grep.csv $B > gpurun_out/${TAG}_l1.log 2>&1; tail -1 gpurun_out/${TAG}_l1.log
+# under ncu kernels serialise, so the adaptive HYBRID split would go all zero-copy: pin the bench's split (9 of 33)
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches_grep.csv $B --zc-share 273 > gpurun_out/${TAG}_l1.log 2>&1; tail -1 gpurun_out/${TAG}_l1.log
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches_groupby.csv $B --workload groupby --gib 4 > gpurun_out/${TAG}_l2.log 2>&1; tail -1 gpurun_out/${TAG}_l2.log
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches_wordcount.csv $B --workload wordcount > gpurun_out/${TAG}_l3.log 2>&1; tail -1 gpurun_out/${TAG}_l3.log
 B="$B --no-profile"
