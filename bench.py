@@ -494,6 +494,9 @@ def main():
         roof["request_rate"] = {"bound": "pcie_read_requests", "achieved": req_rate / 1e9, "peak": 0.562,
                                 "unit": "G requests/s", "frac": req_rate / 0.562e9,
                                 "peak_source": "profiles/r01_box_probe.txt zc_sparse (256-B stride, 1 request/record)"}
+        roof["note"] = ("the zero-copy key gather is bound by outstanding PCIe read requests (one per 32-B key, "
+                        "~84 B of read-completion traffic each), not by bytes: frac is against the H2D DMA byte "
+                        "peak, request_rate.frac against the probed request-rate peak (DESIGN.md §6, §9)")
     roof["avg_launch_ms"] = avg_ms
     roof["launches_per_step"] = launches
 
