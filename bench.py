@@ -497,6 +497,17 @@ def main():
         roof["note"] = ("the zero-copy key gather is bound by outstanding PCIe read requests (one per 32-B key, "
                         "~84 B of read-completion traffic each), not by bytes: frac is against the H2D DMA byte "
                         "peak, request_rate.frac against the probed request-rate peak (DESIGN.md §6, §9)")
+    if dom == "compute" and args.workload == "kmer" and box.get("kmer_windows") and st.get("ms_compute_busy"):
+        # k-mer table updates are random 16-B entry accesses in a 4 GiB table: the bound is the HBM
+        # random-update rate, probed on this GPU (profiles/r01_probe_random.txt: read the key of a
+        # random entry, then an 8-B atomic add to its count, 2^28 entries: 16.9 G updates/s).
+        # Launches of consecutive chunks overlap, so the rate uses the union of the compute intervals.
+        rate = box["kmer_windows"] / (st["ms_compute_busy"] * 1e-3) / 1e9
+        roof["random_update"] = {"bound": "hbm_random_update", "achieved": rate, "peak": 16.94,
+                                 "unit": "G updates/s", "frac": rate / 16.94,
+                                 "peak_source": "profiles/r01_probe_random.txt load+atomic, 148x4 blocks",
+                                 "note": "achieved counts every k-mer window; equal k-mers of one warp step are "
+                                         "merged into one update, so it can exceed the probe"}
     roof["avg_launch_ms"] = avg_ms
     roof["launches_per_step"] = launches
 
