@@ -551,7 +551,9 @@ def main():
         "e2e": {"value": round(total_bytes / t_wall / 1e9, 3), "unit": "GB/s",
                 "h2d_bytes_per_step": (st["bytes_h2d"] + st["bytes_meta"]) * world,
                 "d2h_bytes_per_step": st["bytes_d2h"] * world,
-                "note": "host wall clock around the public bk_run call (pinned host data in, results out to host)"},
+                "note": "host wall clock around the public bk_run call (pinned host data in, results out to host); "
+                        "it tracks the device-timed value because the data set never resides on the GPU: every "
+                        "input byte of every step crosses the host link inside bk_run, in both measurements"},
         "roofline": roof,
         "gpu_launches": int(st["kernel_launches"]) * args.steps,
         "clocks": clk.summary(),
