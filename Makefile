@@ -6,7 +6,7 @@ PKG    := paper_conf_ipps_mokhtaris14_b200
 CSRC   := $(PKG)/csrc
 OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/kernels_pattern.o build/kernels_kmer.o build/runtime_plan.o build/runtime_pipeline.o build/runtime_kernels.o build/runtime_api.o build/host_gather.o
 
-all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so baselines/libbkmt.so
+all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so baselines/libbkmt.so tests/user/libbkuser.so
 
 build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh $(CSRC)/tma.cuh $(CSRC)/runtime.cuh $(CSRC)/host_gather.h include/bk.h
 	@mkdir -p build
@@ -25,12 +25,16 @@ oracle/libbkoracle.so: oracle/oracle.c oracle/oracle.h
 gen/libbkgen.so: gen/gen.c gen/gen.h
 	gcc -O2 -fopenmp -fPIC -shared -Wall -o $@ gen/gen.c -lm
 
+# test-only user kernel for bk_run_user (a caller's own stage-4 kernel against include/bk.h)
+tests/user/libbkuser.so: tests/user/user_kernels.cu include/bk.h
+	$(NVCC) -std=c++17 -O3 $(ARCH) -Xcompiler -fPIC -shared -Iinclude -cudart static -o $@ $<
+
 build/probe: tools/probe.cu
 	@mkdir -p build
 	$(NVCC) -O3 $(ARCH) -o $@ $<
 
 clean:
-	rm -rf build $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so
+	rm -rf build $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so tests/user/libbkuser.so
 
 .PHONY: all clean
 

@@ -281,9 +281,64 @@ typedef struct bk_stats {
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);
 
+/* ---- user kernels over the staged chunks (the paper's general programming model) -------------
+ * BigKernel's promise is that ANY data-parallel kernel over a record-partitioned host array runs
+ * out of core without programmer-managed buffers: the programmer states
+ * which bytes of a record the kernel touches (the access spec, what BigKernel's address
+ * generation derives from the kernel's code) and writes the kernel against the
+ * staged, interleaved layout. bk_run_user runs stages 1-3 exactly as for the built-in kernels and
+ * calls back, once per chunk, so that the caller enqueues its own stage-4 kernel. */
+typedef struct bk_access {
+  uint32_t struct_size;     /* = sizeof(bk_access) */
+  uint32_t n_ext;           /* 0 = the whole record; else 1..8 extents, in access order (duplicates
+                               and overlaps allowed: every listed byte is staged) */
+  uint32_t ext_off[8];      /* extent offset relative to the record start */
+  uint32_t ext_len[8];      /* extent length; every record must contain every extent (BK_E_INVAL) */
+  uint32_t lane_bytes;      /* target accessed bytes per lane (compute thread); 0 = 256 */
+  uint32_t _reserved;
+} bk_access;
+
+/* One staged chunk, as seen by the caller's stage-4 kernel. All pointers are DEVICE pointers,
+ * valid for work enqueued on the callback's stream during the callback; libbk recycles the slot
+ * once that work has completed. Layout: lane t (0 <= t < lanes) owns records
+ * [lanes_desc[t].first, +nrec) of the data set; its accessed bytes, concatenated in record order
+ * then access order, are staged as 16-B words, word k at
+ *   stage + tile_base[t / 32] + (k * 32 + t % 32) * 16,
+ * zero-padded to the tile's longest lane. */
+typedef struct bk_lane { uint64_t first; uint32_t nrec; uint32_t nbytes; } bk_lane;
+typedef struct bk_chunk_view {
+  uint32_t struct_size;       /* = sizeof(bk_chunk_view) */
+  uint32_t lanes;             /* L, a multiple of 32 (tiles = L / 32) */
+  uint64_t chunk_index;       /* 0 .. n_chunks-1; chunks may be computed concurrently, in any order */
+  uint64_t n_chunks;
+  uint64_t first_record;      /* the chunk is records [first_record, first_record + n_records) */
+  uint64_t n_records;
+  const uint8_t* stage;       /* device: the warp tiles */
+  const bk_lane* lane_desc;   /* device: L lane descriptors */
+  const uint64_t* tile_base;  /* device: L/32 + 1 tile offsets (tile_base[L/32] = staged bytes) */
+  const uint64_t* offsets;    /* device: record start offsets (relative to host_ptr) of the chunk's
+                                 records, n_records entries, when the access is whole variable-length
+                                 records; NULL otherwise (records then have a fixed accessed size) */
+  uint64_t end_offset;        /* end of the chunk's last record (relative to host_ptr) */
+} bk_chunk_view;
+
+/* Called on the bk_run_user thread once per chunk, after that chunk's stages 1-3 are ordered on
+ * `stream` (a cudaStream_t): enqueue stage-4 work on `stream` only, do not synchronise it, and
+ * return 0. A non-zero return aborts the run with BK_E_INVAL (work already enqueued completes). */
+typedef int (*bk_chunk_fn)(const bk_chunk_view* view, void* stream, void* user);
+
+/* Streams the registered data set through stages 1-3 under `access` and calls `fn` per chunk;
+ * ordered after prior work on `stream`, returns when every chunk's enqueued work has completed.
+ * Gather mode, window and ring depth come from the context's bk_config (AUTO: DENSE for whole
+ * records, HYBRID for sparse extents). Errors: BK_E_INVAL (NULL fn / access, bad extents, fn
+ * returned non-zero), BK_E_STATE (nothing registered), BK_E_RANGE (a record's accessed bytes exceed
+ * a chunk), BK_E_CUDA. Not available with BK_FLAG_BASELINE_* (BK_E_UNSUPPORTED). */
+BK_API int bk_run_user(bk_ctx* ctx, const bk_access* access, bk_chunk_fn fn, void* user, void* stream);
+
 /* ABI self-check for bindings: writes sizeof of bk_config, bk_out_wordcount, bk_out_grep,
- * bk_out_kmeans, bk_out_partition, bk_out_groupby, bk_out_layout, bk_stats, bk_out_pattern (in that order,
- * up to n entries) and returns BK_ABI_VERSION. Needs no GPU. */
+ * bk_out_kmeans, bk_out_partition, bk_out_groupby, bk_out_layout, bk_stats, bk_out_pattern,
+ * bk_out_kmer, bk_access, bk_chunk_view (in that order, up to n entries) and returns
+ * BK_ABI_VERSION. Needs no GPU. */
 BK_API int bk_abi_sizes(uint32_t* sizes, int n);
 
 #ifdef __cplusplus

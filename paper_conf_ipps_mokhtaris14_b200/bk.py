@@ -94,12 +94,30 @@ class bk_out_kmer(C.Structure):
                 ("table_slots", u64), ("cap", u64), ("kmer", P), ("count", P), ("n_kmers", u64), ("total", u64)]
 
 
+class bk_access(C.Structure):
+    _fields_ = [("struct_size", u32), ("n_ext", u32), ("ext_off", u32 * 8), ("ext_len", u32 * 8), ("lane_bytes", u32),
+                ("_reserved", u32)]
+
+
+class bk_lane(C.Structure):
+    _fields_ = [("first", u64), ("nrec", u32), ("nbytes", u32)]
+
+
+class bk_chunk_view(C.Structure):
+    _fields_ = [("struct_size", u32), ("lanes", u32), ("chunk_index", u64), ("n_chunks", u64),
+                ("first_record", u64), ("n_records", u64), ("stage", P), ("lane_desc", P), ("tile_base", P),
+                ("offsets", P), ("end_offset", u64)]
+
+
+# int (*bk_chunk_fn)(const bk_chunk_view* view, void* stream, void* user)
+bk_chunk_fn = C.CFUNCTYPE(C.c_int, C.POINTER(bk_chunk_view), P, P)
+
 BK_K_PATTERN_STATS = 101
 BK_K_KMER = 6
 ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,
-               bk_out_layout, bk_stats, bk_out_pattern, bk_out_kmer]
-EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_destroy", "bk_strerror", "bk_last_error",
-           "bk_get_stats", "bk_abi_sizes"]
+               bk_out_layout, bk_stats, bk_out_pattern, bk_out_kmer, bk_access, bk_chunk_view]
+EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_strerror",
+           "bk_last_error", "bk_get_stats", "bk_abi_sizes"]
 
 _lib = None
 
@@ -128,7 +146,9 @@ def lib() -> C.CDLL:
         l.bk_last_error.restype = C.c_char_p
         l.bk_get_stats.argtypes = [P, C.POINTER(bk_stats)]
         l.bk_abi_sizes.argtypes = [C.POINTER(u32), C.c_int]
-        for name in ("bk_create", "bk_register_segments", "bk_run", "bk_destroy", "bk_get_stats", "bk_abi_sizes"):
+        l.bk_run_user.argtypes = [P, C.POINTER(bk_access), P, P, P]
+        for name in ("bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_get_stats",
+                     "bk_abi_sizes"):
             getattr(l, name).restype = C.c_int
         _lib = l
     return _lib
@@ -330,6 +350,22 @@ class Context:
         L = o.lanes
         lanes = (p_[:L].copy(), st[:L].copy(), base[:L].copy(), cnt[:L].copy()) if chunk is not None else None
         return tot, lanes
+
+    def run_user(self, fn, user=None, extents=None, lane_bytes: int = 0, stream=None):
+        """bk_run_user: stages 1-3 under `extents` ([(offset, length), ...]; None = whole records),
+        then fn(view*, stream, user) per chunk enqueues the caller's own stage-4 kernel. `fn` is a
+        native bk_chunk_fn (e.g. a symbol of the caller's CUDA library) or a bk_chunk_fn wrapper;
+        `user` an opaque pointer (int address or ctypes object) handed back to it."""
+        a = bk_access()
+        a.struct_size = C.sizeof(bk_access)
+        extents = extents or []
+        a.n_ext = len(extents)
+        for i, (eo, el) in enumerate(extents):
+            a.ext_off[i], a.ext_len[i] = eo, el
+        a.lane_bytes = lane_bytes
+        fp = C.cast(fn, P)
+        up = user if (user is None or isinstance(user, int)) else C.cast(C.pointer(user), P)
+        check(lib().bk_run_user(self.ctx, C.byref(a), fp, up, stream), "bk_run_user")
 
     def layout_dump(self, chunk: int, extents=None, stage_cap: int = 1 << 26, lane_cap: int = 1 << 20, stream=None):
         o = _hdr(bk_out_layout, BK_K_LAYOUT_DUMP)

@@ -325,6 +325,7 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream);
 int run_dbuf(bk_ctx* c, int kid, void* out, void* stream);
 int run_pattern(bk_ctx* c, bk_out_pattern* o, void* stream);
 int run_layout(bk_ctx* c, bk_out_layout* o, void* stream);
+int run_user(bk_ctx* c, const bk_access* a, bk_chunk_fn fn, void* user, void* stream);
 
 }  // namespace rt
 }  // namespace bk

@@ -249,6 +249,28 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
   return BK_OK;
 }
 
+int bk_run_user(bk_ctx* c, const bk_access* a, bk_chunk_fn fn, void* user, void* stream) {
+  if (!c || !a || !fn) return fail(BK_E_INVAL, "NULL argument");
+  if (a->struct_size != sizeof(bk_access)) return fail(BK_E_INVAL, "bk_access size");
+  if (!c->registered) return fail(BK_E_STATE, "bk_run_user before bk_register_segments");
+  if (c->cfg.flags & (BK_FLAG_BASELINE_DBUF | BK_FLAG_BASELINE_SBUF))
+    return fail(BK_E_UNSUPPORTED, "bk_run_user: no double-buffering baseline for user kernels");
+  const auto t0 = std::chrono::steady_clock::now();
+  const int rc = run_user(c, a, fn, user, stream);
+  if (rc) {
+    cudaStreamSynchronize(c->s_copy);
+    cudaStreamSynchronize(c->s_asm);
+    cudaStreamSynchronize(c->s_comp);
+    for (auto st : c->s_slot) cudaStreamSynchronize(st);
+    for (auto st : c->s_stage) cudaStreamSynchronize(st);
+    cudaGetLastError();
+    return rc;
+  }
+  c->st.kernel_launches = (uint64_t)c->n_launch;
+  c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return BK_OK;
+}
+
 int bk_get_stats(const bk_ctx* c, bk_stats* s) {
   if (!c || !s) return fail(BK_E_INVAL, "NULL argument");
   if (s->struct_size != sizeof(bk_stats)) return fail(BK_E_INVAL, "bk_stats size");
@@ -257,11 +279,11 @@ int bk_get_stats(const bk_ctx* c, bk_stats* s) {
 }
 
 int bk_abi_sizes(uint32_t* sizes, int n) {
-  const uint32_t v[10] = {sizeof(bk_config),     sizeof(bk_out_wordcount), sizeof(bk_out_grep),
+  const uint32_t v[12] = {sizeof(bk_config),     sizeof(bk_out_wordcount), sizeof(bk_out_grep),
                           sizeof(bk_out_kmeans), sizeof(bk_out_partition), sizeof(bk_out_groupby),
                           sizeof(bk_out_layout), sizeof(bk_stats),         sizeof(bk_out_pattern),
-                          sizeof(bk_out_kmer)};
-  for (int i = 0; i < n && i < 10; ++i) sizes[i] = v[i];
+                          sizeof(bk_out_kmer),   sizeof(bk_access),        sizeof(bk_chunk_view)};
+  for (int i = 0; i < n && i < 12; ++i) sizes[i] = v[i];
   return BK_ABI_VERSION;
 }
 

@@ -532,6 +532,41 @@ int run_pattern(bk_ctx* c, bk_out_pattern* o, void* stream) {
   return BK_OK;
 }
 
+// bk_run_user: stages 1-3 under the caller's access spec, stage 4 enqueued by the caller per chunk.
+// Always eager (no graph capture): the callback must run on every bk_run_user call.
+int run_user(bk_ctx* c, const bk_access* ua, bk_chunk_fn fn, void* user, void* stream) {
+  if (ua->n_ext > 8) return fail(BK_E_INVAL, "at most 8 extents");
+  Access a;
+  int rc = parse_access(c, ua->n_ext, ua->ext_off, ua->ext_len, a);
+  if (rc) return rc;
+  Plan p;
+  if ((rc = plan_run(c, a, ua->lane_bytes ? ua->lane_bytes : 256, p))) return rc;
+  carve(c, p);
+  static_assert(sizeof(bk_lane) == sizeof(LaneDesc), "bk_lane mirrors LaneDesc");
+  const size_t C = p.bounds.size() - 1;
+  return run_device(c, stream, "user", false, C, [&]() -> int {
+    size_t ci = 0;
+    return pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) -> int {
+      bk_chunk_view v{};
+      v.struct_size = sizeof(bk_chunk_view);
+      v.lanes = ch.L;
+      v.chunk_index = ci++;
+      v.n_chunks = C;
+      v.first_record = ch.lo;
+      v.n_records = ch.hi - ch.lo;
+      v.stage = s.stage;
+      v.lane_desc = reinterpret_cast<const bk_lane*>(s.lanes);
+      v.tile_base = s.tile_base;
+      v.offsets = (a.whole && c->off) ? s.meta : nullptr;
+      v.end_offset = ch.end_byte;
+      const int r = fn(&v, (void*)cs, user);
+      if (r) return fail(BK_E_INVAL, "user chunk function returned %d for chunk %llu", r,
+                         (unsigned long long)v.chunk_index);
+      return (int)BK_OK;
+    });
+  });
+}
+
 int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
   Access a;
   int rc = parse_access(c, o->n_ext, o->ext_off, o->ext_len, a);
