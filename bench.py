@@ -431,7 +431,7 @@ def main():
         pst = pctx.stats()
         pctx.close()
         for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute", "n_gather", "ms_cpu_gather", "ms_xfer_busy",
-                  "ms_zc", "n_zc", "ms_relayout", "n_relayout", "n_chunks_zc", "bytes_zc", "records_zc",
+                  "ms_zc", "n_zc", "ms_relayout", "n_relayout", "n_chunks_zc", "bytes_zc", "records_zc", "ms_d2h", "n_d2h",
                   "ms_compute_busy", "ms_overlap"):
             st[k] = pst[k]
         st["profiled_ms_device"] = pst["ms_device"]
@@ -454,7 +454,17 @@ def main():
         dom = "compute"
     else:
         dom = "zc" if st["n_chunks_zc"] and st["ms_zc"] >= st["ms_h2d"] else "h2d"
-    if dom == "h2d":
+        if st.get("n_d2h") and st.get("ms_d2h", 0.0) > st[{"zc": "ms_zc", "h2d": "ms_h2d"}[dom]]:
+            dom = "d2h"  # write-back (partition's bucket-sorted chunks) is the busier direction
+    stage_ms["d2h"] = st.get("ms_d2h", 0.0)
+    if dom == "d2h":
+        # copy-engine DMA of the per-chunk outputs back to the host, running full duplex with the
+        # H2D stream: against the per-direction peak measured with both directions busy
+        launches = max(st["n_d2h"], 1)
+        per_launch = st["bytes_d2h"] / launches
+        roof = {"kernel": "cudaMemcpyAsync D2H of per-chunk outputs (write-back, copy engine)", "bound": "host_link",
+                "peak": peak_bidir if peak_bidir else peak_h2d, "unit": "GB/s"}
+    elif dom == "h2d":
         # copy-engine DMA of packed (CPU) or raw (DENSE) chunks + offsets slices: host-link bound
         launches = max(st["n_chunks"] - st["n_chunks_zc"], 1)
         per_launch = (st["bytes_h2d"] - st["bytes_zc"] + st["bytes_meta"]) / launches
@@ -480,7 +490,9 @@ def main():
         avg_ms = float("nan")
     roof["achieved"] = per_launch / (avg_ms * 1e-3) / 1e9
     roof["peak_source"] = ("pinned H2D cudaMemcpyAsync measured live in this run (MEASURED_PEAKS.json has no "
-                           "host-link entry)") if roof["bound"] == "host_link" else (
+                           "host-link entry)") if dom in ("h2d", "zc") else (
+        "pinned H2D + D2H cudaMemcpyAsync running concurrently, per direction, measured live in this run"
+        if dom == "d2h" else None) if roof["bound"] == "host_link" else (
         "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6650 GB/s")
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["traffic"] = None
@@ -534,7 +546,7 @@ def main():
                  "payload_bytes": st["bytes_h2d"], "meta_bytes": st["bytes_meta"], "padding_bytes_hbm": st["bytes_padding"]},
         "stages_ms_per_step": {**{k: round(st[k], 3) for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_zc",
                                                                 "ms_relayout", "ms_compute", "ms_device",
-                                                                "ms_cpu_gather")},
+                                                                "ms_cpu_gather", "ms_d2h")},
                                "n_zc": st["n_zc"], "n_relayout": st["n_relayout"],
                                "profiled_ms_device": round(st.get("profiled_ms_device", 0.0), 3),
                                "note": "per-stage busy sums from a profiled eager pass (CUDA events per stage "

@@ -277,6 +277,9 @@ typedef struct bk_stats {
   uint64_t n_chunks_zc;       /* chunks gathered zero-copy in the last run */
   uint64_t bytes_zc;          /* accessed bytes those chunks pulled over PCIe */
   uint64_t records_zc;        /* records in those chunks */
+  double ms_d2h;              /* BK_FLAG_PROFILE: busy time of the device->host write-back copies (partitioned
+                                 chunks, k-means cluster ids); counted in ms_xfer_busy */
+  uint64_t n_d2h;             /*   number of write-back copies timed */
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);

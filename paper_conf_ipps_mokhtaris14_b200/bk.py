@@ -78,7 +78,7 @@ class bk_stats(C.Structure):
                 ("ms_compute", C.c_double), ("n_gather", u64), ("n_chunks_cpu", u64), ("ms_cpu_gather", C.c_double),
                 ("ms_xfer_busy", C.c_double), ("ms_compute_busy", C.c_double), ("ms_overlap", C.c_double),
                 ("ms_zc", C.c_double), ("n_zc", u64), ("ms_relayout", C.c_double), ("n_relayout", u64),
-                ("n_chunks_zc", u64), ("bytes_zc", u64), ("records_zc", u64)]
+                ("n_chunks_zc", u64), ("bytes_zc", u64), ("records_zc", u64), ("ms_d2h", C.c_double), ("n_d2h", u64)]
 
 
 class bk_out_pattern(C.Structure):

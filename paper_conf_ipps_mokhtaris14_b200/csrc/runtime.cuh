@@ -129,6 +129,7 @@ struct bk_ctx {  // the opaque context of include/bk.h
   std::vector<cudaEvent_t> prof;                   // BK_FLAG_PROFILE: per chunk x stage begin/end
   std::vector<int> prof_stage;                     // stage id of each event pair
   size_t prof_used = 0;
+  size_t prof_open[8] = {};                        // event index of each stage's open pair
   uint8_t* window = nullptr;    // the whole streaming working set (cfg.window_bytes)
   std::vector<bk::rt::Slot> slots;
   // registration
@@ -186,7 +187,7 @@ Access field_access(uint32_t off, uint32_t len);
 int parse_access(const bk_ctx* c, uint32_t n_ext, const uint32_t* eo, const uint32_t* el, Access& a);
 
 // ---- pipeline (runtime_pipeline.cu)
-enum { kStH2D = 0, kStAddrgen = 1, kStGather = 2, kStCompute = 3, kStRelayout = 4, kNStages = 5 };
+enum { kStH2D = 0, kStAddrgen = 1, kStGather = 2, kStCompute = 3, kStRelayout = 4, kStD2H = 5, kNStages = 6 };
 int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin);
 #define BK_PROF(stage, stream, begin) do { int r_ = prof_mark(c, stage, stream, begin); if (r_) return r_; } while (0)
 uint64_t test_rand(bk_ctx* c);
@@ -285,7 +286,7 @@ int run_device(bk_ctx* c, void* stream, const std::string& key, bool graphable, 
     c->prof_used = ge->prof_used;
     for (size_t i = 0; i < ge->prof_stage.size(); ++i) c->prof_stage[i] = ge->prof_stage[i];
   } else {
-    if ((rc = prof_reserve(c, 4 * n_chunks + 8))) return rc;
+    if ((rc = prof_reserve(c, 5 * n_chunks + 8))) return rc;
     BK_CUDA(cudaStreamBeginCapture(c->s_comp, cudaStreamCaptureModeThreadLocal));
     rc = device_begin(c);
     if (!rc) rc = enqueue();

@@ -188,7 +188,9 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
         cudaEvent_t e = c->ev_part[ci++ % c->ev_part.size()];
         BK_CUDA(cudaEventRecord(e, cs));
         BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
+        BK_PROF(kStD2H, c->s_d2h, true);
         BK_CUDA(cudaMemcpyAsync(o->cid + ch.lo, s.out, (ch.hi - ch.lo) * 4, cudaMemcpyDeviceToHost, c->s_d2h));
+        BK_PROF(kStD2H, c->s_d2h, false);
         c->st.bytes_d2h += (ch.hi - ch.lo) * 4;
         rel = c->s_d2h;
       }
@@ -288,8 +290,11 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
       BK_CUDA(cudaEventRecord(e, cs));
       BK_CUDA(cudaStreamWaitEvent(c->s_d2h, e, 0));
       const uint64_t bytes = (ch.hi - ch.lo) * 16;
-      if (bytes)
+      if (bytes) {
+        BK_PROF(kStD2H, c->s_d2h, true);
         BK_CUDA(cudaMemcpyAsync((uint8_t*)o->out_records + ch.lo * 16, s.out, bytes, cudaMemcpyDeviceToHost, c->s_d2h));
+        BK_PROF(kStD2H, c->s_d2h, false);
+      }
       c->st.bytes_d2h += bytes;
       rel = c->s_d2h;
       ++ci;

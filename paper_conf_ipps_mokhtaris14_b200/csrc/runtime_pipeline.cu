@@ -9,6 +9,8 @@ namespace rt {
 int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin) {
   if (!(c->cfg.flags & BK_FLAG_PROFILE)) return BK_OK;
   if (begin) {
+    // a pair is claimed at its begin mark and closed through prof_open[stage], so intervals of
+    // different stages may nest (the write-back D2H is issued inside the compute enqueue)
     if (c->prof_used + 2 > c->prof.size()) {
       for (int k = 0; k < 64; ++k) {
         cudaEvent_t e;
@@ -17,11 +19,12 @@ int prof_mark(bk_ctx* c, int stage, cudaStream_t s, bool begin) {
         if (c->prof.size() % 2 == 0) c->prof_stage.push_back(0);
       }
     }
+    c->prof_open[stage] = c->prof_used;
     c->prof_stage[c->prof_used / 2] = stage;
     BK_CUDA(cudaEventRecord(c->prof[c->prof_used], s));
-  } else {
-    BK_CUDA(cudaEventRecord(c->prof[c->prof_used + 1], s));
     c->prof_used += 2;
+  } else {
+    BK_CUDA(cudaEventRecord(c->prof[c->prof_open[stage] + 1], s));
   }
   return BK_OK;
 }
@@ -263,19 +266,26 @@ int begin_run(bk_ctx* c, void* stream) {
 // run start, the union of transfer intervals, the union of compute intervals and their overlap
 // (the north_star's copy/compute overlap, measured with CUDA events instead of nsys).
 int stage_stats(bk_ctx* c) {
-  double acc[kNStages] = {0, 0, 0, 0, 0};
-  uint64_t cnt[kNStages] = {0, 0, 0, 0, 0};
+  double acc[kNStages] = {};
+  uint64_t cnt[kNStages] = {};
   std::vector<std::pair<double, double>> xfer, comp;
+  // BK_TIMELINE=<path>: append every profiled (stage, begin ms, end ms) interval of the run as CSV
+  // (a timeline for analysis where nsys is not available; stage ids as kSt* in runtime.cuh)
+  const char* tl_path = getenv("BK_TIMELINE");
+  FILE* tl = tl_path ? fopen(tl_path, "a") : nullptr;
+  if (tl) fprintf(tl, "# run\n");
   for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
     float e = 0, b0 = 0;
     BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
     BK_CUDA(cudaEventElapsedTime(&b0, c->t_begin, c->prof[i]));
     const int stg = c->prof_stage[i / 2];
+    if (tl) fprintf(tl, "%d,%.4f,%.4f\n", stg, b0, b0 + e);
     acc[stg] += e;
     cnt[stg] += 1;
-    if (stg == kStH2D || stg == kStGather) xfer.emplace_back(b0, b0 + e);
+    if (stg == kStH2D || stg == kStGather || stg == kStD2H) xfer.emplace_back(b0, b0 + e);
     if (stg == kStCompute) comp.emplace_back(b0, b0 + e);
   }
+  if (tl) fclose(tl);
   auto merge = [](std::vector<std::pair<double, double>> v) {
     std::sort(v.begin(), v.end());
     std::vector<std::pair<double, double>> u;
@@ -303,6 +313,8 @@ int stage_stats(bk_ctx* c) {
   c->st.n_zc = cnt[kStGather];
   c->st.ms_relayout = acc[kStRelayout];
   c->st.n_relayout = cnt[kStRelayout];
+  c->st.ms_d2h = acc[kStD2H];
+  c->st.n_d2h = cnt[kStD2H];
   c->st.ms_xfer_busy = bx;
   c->st.ms_compute_busy = bc;
   c->st.ms_overlap = ov;

@@ -457,6 +457,39 @@ def test_repeated_runs_graph_replay(no_graph):
             assert np.array_equal(global_from_runs(o, cc), wout)
 
 
+@pytest.mark.parametrize("mode", ["dense", "zc", "hybrid"])
+def test_profiled_runs(mode):
+    """BK_FLAG_PROFILE (the bench's stage-breakdown pass) issues eagerly with CUDA events around every
+    stage of every chunk, including the write-back D2H copies issued inside the compute enqueue
+    (nested intervals): results equal the oracle and the stage accounting is consistent."""
+    x = gen.points(n=150_000)
+    kc, ks, kchk, kcid = oracle.kmeans(x, x[:64], want_cid=True)
+    kv = gen.kv(n=200_000)
+    wboff, wout = oracle.partition(kv, 512)
+    gb, goff = gen.grep_records(max_bytes=6 * MIB)
+    with bk.Context(window_bytes=2 * MIB, record_size=64, gather_mode=mode, profile=True) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=len(x))
+        cid = np.full(len(x), -1, np.int32)
+        c, s, chk = ctx.kmeans(x[:64], cid=cid)
+        assert np.array_equal(cid, kcid) and chk == kchk and np.array_equal(c, kc)
+        st = ctx.stats()
+        assert st["n_d2h"] == st["n_chunks"] and st["ms_d2h"] > 0 and st["bytes_d2h"] >= 4 * len(x)
+        assert st["ms_compute"] > 0 and 0 < st["ms_xfer_busy"] <= st["ms_device"] * 1.01
+    if mode != "hybrid":
+        with bk.Context(window_bytes=2 * MIB, record_size=16, gather_mode=mode, profile=True) as ctx:
+            ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=len(kv))
+            o, cc, bc = ctx.partition(512)
+            assert np.array_equal(global_from_runs(o, cc), wout)
+            st = ctx.stats()
+            assert st["n_d2h"] == st["n_chunks"] >= 4 and st["ms_d2h"] > 0
+            assert st["ms_overlap"] <= min(st["ms_xfer_busy"], st["ms_compute_busy"]) + 1e-6
+    with bk.Context(window_bytes=2 * MIB, gather_mode=mode, profile=True) as ctx:
+        ctx.register(gb, goff)
+        assert np.array_equal(ctx.grep(b"bigk", cap=len(goff)), oracle.grep(gb, goff, b"bigk"))
+        st = ctx.stats()
+        assert st["n_d2h"] == 0 and st["ms_compute"] > 0 and st["ms_xfer_busy"] > 0
+
+
 # ------------------------------------------------------------------ invariants + API errors
 def test_invariance_across_window_slots_lanes_modes():
     buf, off = gen.text(cap_bytes=1 * MIB)
