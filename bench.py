@@ -248,6 +248,15 @@ def measure_bidir_peak(torch, dev) -> float:
     return best
 
 
+def load_traffic() -> dict:
+    """Per-unit traffic of the roofline kernels from one ncu --set full capture each (committed)."""
+    try:
+        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r01_traffic.json")) as f:
+            return json.load(f)
+    except (OSError, ValueError):
+        return {}
+
+
 def load_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -496,6 +505,20 @@ def main():
         "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6650 GB/s")
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["traffic"] = None
+    tr = load_traffic().get(args.workload)
+    if tr and ((dom == "zc" and tr["unit"] == "record") or (dom == "compute")):
+        # bytes one launch moves, measured by ncu --set full on one launch of the same kernel
+        # (profiles/r01_traffic.json, tools/gpu_traffic.sh), scaled to this run's units per launch
+        if dom == "zc":
+            units = st["records_zc"] / max(st["n_chunks_zc"], 1)
+        elif tr["unit"] == "record":
+            units = shard["n"] / max(st["n_chunks"], 1)
+        else:
+            units = st["bytes_accessed"] / max(st["n_chunks"], 1)
+        roof["traffic"] = tr["traffic_per_unit"] * units
+        roof["traffic_source"] = (f"{tr['what']} of {tr['kernel']}, ncu --set full ({tr['capture']}): "
+                                  f"{tr['traffic_per_unit']:.2f} B per {tr['unit']} x {units:.0f} {tr['unit']}s "
+                                  f"per launch; algorithmic bytes per launch {per_launch:.0f}")
     if dom == "zc" and args.workload == "grep":
         # the zero-copy key gather is PCIe read-request bound, not byte bound: one read request per
         # 128-B line a 32-B key touches (8-aligned keys: 1 + 3/16 = 1.1875 requests per record).
