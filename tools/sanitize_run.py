@@ -67,4 +67,25 @@ for mode in ("cpu", "zc"):
 with bk.Context(window_bytes=512 << 10, record_size=64, baseline_dbuf=True) as ctx:
     ctx.register(x.view(np.uint8).reshape(-1), None, n_records=50_000)
     ctx.kmeans(x[:7])
+# late round 1: profiled runs (nested write-back D2H events), tiny / ragged data sets, user kernels
+with bk.Context(window_bytes=512 << 10, record_size=64, profile=True) as ctx:
+    ctx.register(x.view(np.uint8).reshape(-1), None, n_records=50_000)
+    ctx.kmeans(x[:64], cid=np.empty(50_000, np.int32))
+with bk.Context(window_bytes=1 << 20, record_size=16, profile=True) as ctx:
+    ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=100_000)
+    ctx.partition(256)
+for n in (1, 33):
+    for mode in ("zc", "cpu", "dense", "hybrid"):
+        tb, to = gen.text(cap_recs=n)
+        with bk.Context(window_bytes=1 << 20, gather_mode=mode) as ctx:
+            ctx.register(tb, to[:n])
+            ctx.wordcount(cap=1 << 10)
+        eb, eo = gen.grep_records(n=n)
+        with bk.Context(window_bytes=1 << 20, gather_mode=mode) as ctx:
+            ctx.register(eb, eo)
+            ctx.grep(b"", cap=n)
+        with bk.Context(window_bytes=1 << 20, record_size=16, gather_mode=mode) as ctx:
+            ctx.register(kv[:n].view(np.uint8).reshape(-1), None, n_records=n)
+            if mode != "hybrid":
+                ctx.partition(64)
 print("sanitize run ok")
