@@ -532,6 +532,11 @@ def main():
         roof["note"] = ("the zero-copy key gather is bound by outstanding PCIe read requests (one per 32-B key, "
                         "~84 B of read-completion traffic each), not by bytes: frac is against the H2D DMA byte "
                         "peak, request_rate.frac against the probed request-rate peak (DESIGN.md §6, §9)")
+    if dom == "compute" and args.workload == "wordcount":
+        roof["note"] = ("k_wc is latency-bound, not bandwidth-bound: an 8 MiB window gives ~0.44-MB chunks, "
+                        "0.15 waves of the kernel (6% achieved occupancy, issue IPC 0.43 under ncu); its launches "
+                        "overlap across slots, and dropping it entirely would raise the step by only ~12% "
+                        "(profiles/r01_wc_sweep.md). The step-level link fraction is link.frac")
     if dom == "compute" and args.workload == "kmer" and box.get("kmer_windows") and st.get("ms_compute_busy"):
         # k-mer table updates are random 16-B entry accesses in a 4 GiB table: the bound is the HBM
         # random-update rate, probed on this GPU (profiles/r01_probe_random.txt: read the key of a
