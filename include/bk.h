@@ -344,6 +344,27 @@ BK_API int bk_run_user(bk_ctx* ctx, const bk_access* access, bk_chunk_fn fn, voi
  * BK_ABI_VERSION. Needs no GPU. */
 BK_API int bk_abi_sizes(uint32_t* sizes, int n);
 
+/* ---- C4 output in bucket-major order (host side, optional; SURVEY §8(d) C4 "a bucket-major
+ * materialised copy is an optional, separately timed host pass") -------------------------------
+ * BK_K_PARTITION leaves its result as chunk-major runs (each chunk bucket-sorted and stable,
+ * chunk_counts[c * n_buckets + b] records of bucket b in chunk c), which is already the stable
+ * partition up to a re-ordering of whole runs (chunks ascend in record order). This copies the runs
+ * into the O4 order (bucket, original index) of PAPER.md's data-parallel partition (P:16-17 via
+ * SURVEY O4): dst[bucket_start[b] + k] = k-th record of bucket b, taking chunk 0's run of b, then
+ * chunk 1's, and so on.
+ *   out_records   n x 16 B, the chunk-major runs bk_run wrote (n = sum of chunk_counts)
+ *   chunk_counts  n_chunks x n_buckets, row-major, as bk_run wrote them
+ *   bucket_start  n_buckets destination indices (records) of each bucket's first record, or NULL for
+ *                 the local exclusive scan of the bucket totals (dst then holds exactly n records).
+ *                 Multi-GPU: pass the global offsets of this rank's records (merge.py
+ *                 merge_partition_offsets) so every rank fills its disjoint share of one array.
+ *   dst           destination, 16-B records, caller-owned, must not overlap out_records
+ *   threads       host threads (0 = all cores)
+ * Pure host code, no CUDA call: it may run while the GPU streams the next data set. Returns BK_OK,
+ * or BK_E_INVAL on NULL pointers, n_buckets == 0 or n_chunks * n_buckets overflow. */
+BK_API int bk_partition_materialize(const void* out_records, const uint64_t* chunk_counts, uint64_t n_chunks,
+                                    uint32_t n_buckets, const uint64_t* bucket_start, void* dst, uint32_t threads);
+
 #ifdef __cplusplus
 }
 #endif

@@ -117,7 +117,7 @@ BK_K_KMER = 6
 ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,
                bk_out_layout, bk_stats, bk_out_pattern, bk_out_kmer, bk_access, bk_chunk_view]
 EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_strerror",
-           "bk_last_error", "bk_get_stats", "bk_abi_sizes"]
+           "bk_last_error", "bk_get_stats", "bk_abi_sizes", "bk_partition_materialize"]
 
 _lib = None
 
@@ -147,8 +147,9 @@ def lib() -> C.CDLL:
         l.bk_get_stats.argtypes = [P, C.POINTER(bk_stats)]
         l.bk_abi_sizes.argtypes = [C.POINTER(u32), C.c_int]
         l.bk_run_user.argtypes = [P, C.POINTER(bk_access), P, P, P]
+        l.bk_partition_materialize.argtypes = [P, P, u64, u32, P, P, u32]
         for name in ("bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_get_stats",
-                     "bk_abi_sizes"):
+                     "bk_abi_sizes", "bk_partition_materialize"):
             getattr(l, name).restype = C.c_int
         _lib = l
     return _lib
@@ -207,6 +208,21 @@ def bk_register_segments(ctx: int, data, offsets=None, nbytes: int | None = None
 
 def bk_run(ctx: int, kernel_id: int, stream, out) -> None:
     check(lib().bk_run(ctx, kernel_id, stream, C.byref(out)), "bk_run")
+
+
+def partition_materialize(out: np.ndarray, chunk_counts: np.ndarray, bucket_start: np.ndarray | None = None,
+                          dst: np.ndarray | None = None, threads: int = 0) -> np.ndarray:
+    """bk_partition_materialize: chunk-major runs (Context.partition) -> bucket-major stable order.
+    dst defaults to a new n x 2 u64 array (bucket_start None: local offsets)."""
+    cc = np.ascontiguousarray(chunk_counts, np.uint64)
+    C, B = cc.shape
+    if dst is None:
+        dst = np.empty((int(cc.sum()), 2), np.uint64)
+    bs = None if bucket_start is None else np.ascontiguousarray(bucket_start, np.uint64)
+    check(lib().bk_partition_materialize(_ptr(out) if C else None, _ptr(cc) if C else None, C, B,
+                                         _ptr(bs) if bs is not None else None, _ptr(dst) if C else None, threads),
+          "bk_partition_materialize")
+    return dst
 
 
 def bk_destroy(ctx: int) -> None:

@@ -243,4 +243,50 @@ uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, con
   return size;
 }
 
+// The runs of bucket b sit at chunk_base[c] + sum_{b' < b} counts[c][b'] in the chunk-major array;
+// in the bucket-major order they follow each other in chunk order from bucket_start[b]. Every run
+// is one memcpy; threads take runs in blocks from a shared counter (runs average n / (C * B) records).
+int partition_materialize(const uint8_t* runs, const uint64_t* counts, uint64_t n_chunks, uint32_t n_buckets,
+                          const uint64_t* bucket_start, uint8_t* dst, uint32_t threads) {
+  constexpr uint64_t R = 16;  // bytes per {key, value} record
+  struct Run { uint64_t src, dst, n; };
+  std::vector<uint64_t> bstart(n_buckets), bnext(n_buckets);
+  if (bucket_start) {
+    for (uint32_t b = 0; b < n_buckets; ++b) bstart[b] = bucket_start[b];
+  } else {
+    std::vector<uint64_t> tot(n_buckets, 0);
+    for (uint64_t c = 0; c < n_chunks; ++c)
+      for (uint32_t b = 0; b < n_buckets; ++b) tot[b] += counts[c * n_buckets + b];
+    uint64_t acc = 0;
+    for (uint32_t b = 0; b < n_buckets; ++b) { bstart[b] = acc; acc += tot[b]; }
+  }
+  bnext = bstart;
+  std::vector<Run> work;
+  work.reserve((size_t)std::min<uint64_t>(n_chunks * n_buckets, 1u << 24));
+  uint64_t src = 0;
+  for (uint64_t c = 0; c < n_chunks; ++c)
+    for (uint32_t b = 0; b < n_buckets; ++b) {
+      const uint64_t m = counts[c * n_buckets + b];
+      if (m) work.push_back({src, bnext[b], m});
+      src += m;
+      bnext[b] += m;
+    }
+  unsigned T = threads ? threads : std::max(1u, std::thread::hardware_concurrency());
+  T = (unsigned)std::min<uint64_t>(T, std::max<size_t>(work.size() / 16, 1));
+  std::atomic<size_t> next{0};
+  auto body = [&]() {
+    for (;;) {
+      const size_t i0 = next.fetch_add(16);
+      if (i0 >= work.size()) return;
+      for (size_t i = i0; i < std::min(work.size(), i0 + 16); ++i)
+        memcpy(dst + work[i].dst * R, runs + work[i].src * R, work[i].n * R);
+    }
+  };
+  std::vector<std::thread> pool;
+  for (unsigned t = 1; t < T; ++t) pool.emplace_back(body);
+  body();
+  for (auto& th : pool) th.join();
+  return 0;
+}
+
 }  // namespace bk

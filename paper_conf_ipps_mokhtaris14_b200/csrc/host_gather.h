@@ -61,4 +61,8 @@ uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, con
                          uint64_t cap, uint64_t grab = 0, bool nt = true,
                          const std::function<void(uint64_t, uint64_t)>* sink = nullptr);
 
+// bk_partition_materialize (include/bk.h): chunk-major bucket-sorted runs -> bucket-major order.
+int partition_materialize(const uint8_t* runs, const uint64_t* counts, uint64_t n_chunks, uint32_t n_buckets,
+                          const uint64_t* bucket_start, uint8_t* dst, uint32_t threads);
+
 }  // namespace bk

@@ -278,6 +278,20 @@ int bk_get_stats(const bk_ctx* c, bk_stats* s) {
   return BK_OK;
 }
 
+int bk_partition_materialize(const void* out_records, const uint64_t* chunk_counts, uint64_t n_chunks,
+                             uint32_t n_buckets, const uint64_t* bucket_start, void* dst, uint32_t threads) {
+  if (n_buckets == 0) return fail(BK_E_INVAL, "n_buckets == 0");
+  if (n_chunks && n_chunks > UINT64_MAX / n_buckets) return fail(BK_E_INVAL, "n_chunks * n_buckets overflows");
+  if (n_chunks && (!out_records || !chunk_counts || !dst)) return fail(BK_E_INVAL, "NULL argument");
+  try {
+    partition_materialize(static_cast<const uint8_t*>(out_records), chunk_counts, n_chunks, n_buckets, bucket_start,
+                          static_cast<uint8_t*>(dst), threads);
+  } catch (...) {
+    return fail(BK_E_NOMEM, "partition_materialize: host allocation failed");
+  }
+  return BK_OK;
+}
+
 int bk_abi_sizes(uint32_t* sizes, int n) {
   const uint32_t v[12] = {sizeof(bk_config),     sizeof(bk_out_wordcount), sizeof(bk_out_grep),
                           sizeof(bk_out_kmeans), sizeof(bk_out_partition), sizeof(bk_out_groupby),

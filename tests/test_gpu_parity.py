@@ -402,6 +402,7 @@ def test_partition_bench_scale():
     wboff, wout = oracle.partition(kv, 1024)
     assert np.array_equal(np.concatenate([[0], np.cumsum(bc)]).astype(np.uint64), wboff)
     assert np.array_equal(global_from_runs(out, cc), wout)
+    assert np.array_equal(bk.partition_materialize(out, cc), wout)   # the host bucket-major pass
 
 
 def test_groupby_bench_scale():
