@@ -18,6 +18,7 @@
 //                                        the whole chunk followed by an HBM re-layout kernel.
 #pragma once
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX v3: ranges cost ~ns when no tool is attached
 
 #include <algorithm>
 #include <chrono>
@@ -215,6 +216,22 @@ inline bool stage_tma(const Plan& p) { return p.mode == BK_GATHER_DENSE || p.mod
 int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes);
 void unregister(bk_ctx* c);
 
+// NVTX ranges (SURVEY §5 tracing): bk_run / registration, and per chunk its stage issue ("chunk i
+// zc|cpu|dense") and compute enqueue, so `ncu --nvtx --nvtx-include "bk_run.grep/"` or a timeline
+// tool can select one workload's kernels. They mark host issue time; GPU time is in bk_stats.
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  template <class... A>
+  NvtxRange(const char* fmt, A... a) {
+    char b[96];
+    snprintf(b, sizeof b, fmt, a...);
+    nvtxRangePushA(b);
+  }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
+
 template <class Compute>
 int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
   const size_t C = p.bounds.size() - 1;
@@ -243,14 +260,21 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
       cudaGetLastError();
       cpu = zc_inflight.size() >= zc_depth;
     }
-    int rc = cpu ? stage_chunk_cpu(c, p, i, s) : stage_chunk(c, p, i, s);
+    int rc;
+    {
+      NvtxRange r("chunk %zu %s", i, cpu ? "cpu" : p.zero_copy ? "zc" : "dense");
+      rc = cpu ? stage_chunk_cpu(c, p, i, s) : stage_chunk(c, p, i, s);
+    }
     if (rc) return rc;
     if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(s.ready);
     BK_CUDA(cudaStreamWaitEvent(cs, s.ready, 0));
     BK_DELAY(cs);
     BK_PROF(kStCompute, cs, true);
     cudaStream_t rel = cs;   // stream whose completion frees the slot (partition: its D2H)
-    rc = compute(chunk_of(c, p, i), s, cs, rel);
+    {
+      NvtxRange r("compute %zu", i);
+      rc = compute(chunk_of(c, p, i), s, cs, rel);
+    }
     if (rc) return rc;
     BK_PROF(kStCompute, cs, false);
     BK_CUDA(cudaEventRecord(s.freed, rel));

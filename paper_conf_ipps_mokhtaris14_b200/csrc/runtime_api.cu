@@ -113,6 +113,7 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
 }
 
 int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const uint64_t* off, uint64_t n) {
+  NvtxRange nv("bk_register_segments");
   if (!c) return fail(BK_E_INVAL, "NULL ctx");
   if (!host_ptr && nbytes) return fail(BK_E_INVAL, "NULL host_ptr");
   const auto t0 = std::chrono::steady_clock::now();
@@ -185,6 +186,9 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
   if (!c->registered) return fail(BK_E_STATE, "bk_run before bk_register_segments");
   const bk_out_header* h = (const bk_out_header*)out;
   if (h->kernel_id != kernel_id) return fail(BK_E_INVAL, "out->kernel_id %d != %d", h->kernel_id, kernel_id);
+  static const char* const kNames[] = {"?", "wordcount", "grep", "kmeans", "partition", "groupby", "kmer"};
+  NvtxRange nv("bk_run.%s", kernel_id >= 1 && kernel_id <= 6 ? kNames[kernel_id]
+                             : kernel_id == BK_K_LAYOUT_DUMP ? "layout" : "pattern");
   const auto t0 = std::chrono::steady_clock::now();
   int rc;
   if (c->cfg.flags & (BK_FLAG_BASELINE_DBUF | BK_FLAG_BASELINE_SBUF)) {
@@ -250,6 +254,7 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
 }
 
 int bk_run_user(bk_ctx* c, const bk_access* a, bk_chunk_fn fn, void* user, void* stream) {
+  NvtxRange nv("bk_run_user");
   if (!c || !a || !fn) return fail(BK_E_INVAL, "NULL argument");
   if (a->struct_size != sizeof(bk_access)) return fail(BK_E_INVAL, "bk_access size");
   if (!c->registered) return fail(BK_E_STATE, "bk_run_user before bk_register_segments");
