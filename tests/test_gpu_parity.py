@@ -163,6 +163,27 @@ def test_grep_medium(mode):
         assert 0 < st["n_chunks_cpu"] < st["n_chunks"]
 
 
+@pytest.mark.parametrize("mode", ["zc", "cpu"])
+def test_grep_every_pattern_length(mode):
+    """The SWAR matcher at every pattern length 1..32: each pattern is cut from a real key (so it
+    matches somewhere), from its start, middle or end; indices equal the oracle's."""
+    buf, off = gen.grep_records(n=30_000)
+    b = buf.tobytes()
+    rng = np.random.default_rng(7)
+    with bk.Context(window_bytes=4 * MIB, gather_mode=mode) as ctx:
+        ctx.register(buf, off)
+        for L in range(1, 33):
+            for _ in range(2):
+                r = int(rng.integers(len(off)))
+                key = b[int(off[r]) + 16: int(off[r]) + 48].split(b"\0")[0]
+                if len(key) < L:
+                    key = (key * 8)[:32]   # repeated key bytes: still a plausible pattern, maybe no match
+                s0 = int(rng.integers(0, len(key) - L + 1))
+                pat = key[s0: s0 + L]
+                got = ctx.grep(pat, cap=len(off))
+                assert np.array_equal(got, oracle.grep(buf, off, pat)), (L, pat)
+
+
 @pytest.mark.parametrize("lane_bytes", [1024, 1056, 4096])
 def test_grep_long_lanes(lane_bytes):
     """Lanes of 32, 33 and 128 keys: k_grep_count keeps a 32-record match mask per lane; longer
