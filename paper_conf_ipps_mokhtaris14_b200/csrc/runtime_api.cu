@@ -157,13 +157,17 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
       return fail(BK_E_CUDA, "cudaHostGetDevicePointer (memory pinned without cudaHostRegisterMapped?): %s", cudaGetErrorString(e));
     }
     c->host_dev = (const uint8_t*)dptr;
+    c->host = (const uint8_t*)host_ptr;   // from here on unregister() releases what was pinned
   }
   if (off && n) {
     if (is_pinned(off)) {
       c->pinned_off = false;
     } else {
       cudaError_t e = cudaHostRegister((void*)off, n * 8, cudaHostRegisterMapped | cudaHostRegisterPortable);
-      if (e != cudaSuccess) return fail(BK_E_CUDA, "cudaHostRegister(offsets): %s", cudaGetErrorString(e));
+      if (e != cudaSuccess) {
+        unregister(c);   // do not leak the data set's pinning on a failed registration
+        return fail(BK_E_CUDA, "cudaHostRegister(offsets): %s", cudaGetErrorString(e));
+      }
       c->pinned_off = true;
     }
     void* odev = nullptr;  // caller-pinned offsets may be unmapped: then stage 1 DMAs them instead

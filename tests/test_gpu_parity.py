@@ -512,6 +512,29 @@ def test_profiled_runs(mode):
         assert st["n_d2h"] == 0 and st["ms_compute"] > 0 and st["ms_xfer_busy"] > 0
 
 
+def test_reregistration_and_prepinned_data():
+    """One context, several data sets in turn (each registration releases the previous pinning and
+    drops cached plans / graphs), plus a caller-pinned buffer that libbk must not re-register."""
+    import torch
+    t1, o1 = gen.text(cap_bytes=2 * MIB)
+    gb, goff = gen.grep_records(n=40_000)
+    t2, o2 = gen.text(seed=12345, cap_bytes=1 * MIB)
+    with bk.Context(window_bytes=1 * MIB) as ctx:
+        for _ in range(2):
+            ctx.register(t1, o1)
+            assert wc_multiset_gpu(t1, *ctx.wordcount(cap=1 << 17)) == oracle.wc(t1, o1)
+            ctx.register(gb, goff)
+            assert np.array_equal(ctx.grep(b"bigk", cap=len(goff)), oracle.grep(gb, goff, b"bigk"))
+            ctx.register(t2, o2)
+            assert wc_multiset_gpu(t2, *ctx.wordcount(cap=1 << 17)) == oracle.wc(t2, o2)
+        pinned = torch.empty(len(t1), dtype=torch.uint8, pin_memory=True).numpy()
+        pinned[:] = t1
+        ctx.register(pinned, o1)
+        assert wc_multiset_gpu(pinned, *ctx.wordcount(cap=1 << 17)) == oracle.wc(t1, o1)
+    # the caller's pinned buffer is still valid (not unregistered by libbk) after bk_destroy
+    assert pinned[:16].tobytes() == t1[:16].tobytes()
+
+
 # ------------------------------------------------------------------ invariants + API errors
 def test_invariance_across_window_slots_lanes_modes():
     buf, off = gen.text(cap_bytes=1 * MIB)
