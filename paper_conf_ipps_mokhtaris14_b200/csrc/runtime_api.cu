@@ -27,6 +27,16 @@ const char* last_error() { return g_last_error.c_str(); }
 using namespace bk;
 using namespace bk::rt;
 
+// After a failed run: wait for everything already queued on the context's streams (no copy may
+// still target the caller's buffers, no kernel may still use the slots) and clear the error state.
+static void drain(bk_ctx* c) {
+  for (cudaStream_t st : {c->s_copy, c->s_asm, c->s_comp, c->s_d2h})
+    if (st) cudaStreamSynchronize(st);
+  for (auto st : c->s_slot) cudaStreamSynchronize(st);
+  for (auto st : c->s_stage) cudaStreamSynchronize(st);
+  cudaGetLastError();
+}
+
 extern "C" {
 
 const char* bk_strerror(int status) {
@@ -243,13 +253,7 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
       return fail(BK_E_UNSUPPORTED, "unknown kernel_id %d", kernel_id);
   }
   if (rc) {
-    // leave the context usable: drain whatever was queued
-    cudaStreamSynchronize(c->s_copy);
-    cudaStreamSynchronize(c->s_asm);
-    cudaStreamSynchronize(c->s_comp);
-    for (auto st : c->s_slot) cudaStreamSynchronize(st);
-    for (auto st : c->s_stage) cudaStreamSynchronize(st);
-    cudaGetLastError();
+    drain(c);   // leave the context usable
     return rc;
   }
   c->st.kernel_launches = (uint64_t)c->n_launch;
@@ -267,12 +271,7 @@ int bk_run_user(bk_ctx* c, const bk_access* a, bk_chunk_fn fn, void* user, void*
   const auto t0 = std::chrono::steady_clock::now();
   const int rc = run_user(c, a, fn, user, stream);
   if (rc) {
-    cudaStreamSynchronize(c->s_copy);
-    cudaStreamSynchronize(c->s_asm);
-    cudaStreamSynchronize(c->s_comp);
-    for (auto st : c->s_slot) cudaStreamSynchronize(st);
-    for (auto st : c->s_stage) cudaStreamSynchronize(st);
-    cudaGetLastError();
+    drain(c);
     return rc;
   }
   c->st.kernel_launches = (uint64_t)c->n_launch;
