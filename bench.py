@@ -248,6 +248,11 @@ def measure_bidir_peak(torch, dev) -> float:
     return best
 
 
+# arithmetic type each workload's path computes in (bytes are moved as u8 everywhere)
+DTYPE = {"grep": "u8", "wordcount": "u8 (u64 hashes, u64 counts)", "groupby": "u64 + f64",
+         "groupby_sparse": "u64 + f64", "kmeans": "f32 distances, f64 sums", "partition": "u64", "kmer": "u64"}
+
+
 def load_traffic() -> dict:
     """Per-unit traffic of the roofline kernels from one ncu --set full capture each (committed)."""
     try:
@@ -567,7 +572,7 @@ def main():
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(t_dev / args.steps * 1e3, 3), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded counter RNG, gen/)",
+        "scaling": "weak", "vs_baseline": None, "dtype": DTYPE[args.workload], "data": "synthetic (seeded counter RNG, gen/)",
         "config": {"workload": args.workload, "desc": WORKLOADS[args.workload][2],
                    "bytes_per_gpu": nbytes, "records_per_gpu": shard["n"], "window_bytes": window,
                    "n_slots": st["n_slots"],
@@ -701,7 +706,7 @@ def reference_arm(args, rank, world, gib):
     v = statistics.mean(vals)
     line = {"metric": METRIC, "value": round(v, 4), "unit": "GB/s", "impl": "reference", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded counter RNG, gen/)",
+            "vs_baseline": None, "dtype": DTYPE[args.workload], "data": "synthetic (seeded counter RNG, gen/)",
             "config": {"workload": args.workload, "desc": WORKLOADS[args.workload][2],
                        "bytes_per_gpu": len(shard["buf"]), "records_per_gpu": shard["n"]},
             "ms_per_step": round(secs / args.steps * 1e3, 1),
