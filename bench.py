@@ -603,9 +603,12 @@ def main():
                     "overlap_frac": round(st.get("ms_overlap", 0.0) / max(min(st.get("ms_xfer_busy", 0.0),
                                                                               st.get("ms_compute_busy", 0.0)), 1e-9), 4),
                     "link_busy_frac": round(st.get("ms_xfer_busy", 0.0) / max(st.get("profiled_ms_device", 0.0), 1e-9), 4),
+                    "max_busy_frac": round(max(st.get("ms_xfer_busy", 0.0), st.get("ms_compute_busy", 0.0)) /
+                                           max(st.get("profiled_ms_device", 0.0), 1e-9), 4),
                     "how": "unions of per-chunk CUDA-event intervals of the transfer stages (DMA copies, zero-copy "
                            "gathers) and of the compute kernels, profiled pass; overlap_frac = |xfer n compute| / "
-                           "min(xfer, compute); link_busy_frac = xfer union / device time"},
+                           "min(xfer, compute); link_busy_frac = xfer union / device time; max_busy_frac = max(xfer, compute) "
+                           "union / device time (SURVEY §8(d) overlap)"},
         "e2e": {"value": round(total_bytes / t_wall / 1e9, 3), "unit": "GB/s",
                 "h2d_bytes_per_step": (st["bytes_h2d"] + st["bytes_meta"]) * world,
                 "d2h_bytes_per_step": st["bytes_d2h"] * world,
