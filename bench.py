@@ -536,7 +536,11 @@ def main():
         roof["traffic"] = tr["traffic_per_unit"] * units
         roof["traffic_source"] = (f"{tr['what']} of {tr['kernel']}, ncu --set full ({tr['capture']}): "
                                   f"{tr['traffic_per_unit']:.2f} B per {tr['unit']} x {units:.0f} {tr['unit']}s "
-                                  f"per launch; algorithmic bytes per launch {per_launch:.0f}")
+                                  f"per launch; algorithmic bytes per launch {per_launch:.0f}" +
+                                  ("; a zero-copy read moves whole 32-B sectors (an 8-aligned 32-B key at +16 touches "
+                                   "1.75 of them on average) and every read completion carries PCIe TLP overhead, so "
+                                   "the link traffic is ~2.7x the key bytes by construction, not re-reads"
+                                   if dom == "zc" else ""))
     if dom == "zc" and args.workload == "grep":
         # the zero-copy key gather is PCIe read-request bound, not byte bound: one read request per
         # 128-B line a 32-B key touches (8-aligned keys: 1 + 3/16 = 1.1875 requests per record).
