@@ -537,9 +537,13 @@ def main():
         roof["traffic_source"] = (f"{tr['what']} of {tr['kernel']}, ncu --set full ({tr['capture']}): "
                                   f"{tr['traffic_per_unit']:.2f} B per {tr['unit']} x {units:.0f} {tr['unit']}s "
                                   f"per launch; algorithmic bytes per launch {per_launch:.0f}" +
-                                  ("; a zero-copy read moves whole 32-B sectors (an 8-aligned 32-B key at +16 touches "
-                                   "1.75 of them on average) and every read completion carries PCIe TLP overhead, so "
-                                   "the link traffic is ~2.7x the key bytes by construction, not re-reads"
+                                  ({"grep": "; a zero-copy read moves whole 32-B sectors (an 8-aligned 32-B key at +16 "
+                                            "touches 1.75 of them on average) and every read completion carries PCIe TLP "
+                                            "overhead, so the link traffic is ~2.7x the key bytes by construction, not "
+                                            "re-reads",
+                                    "groupby_sparse": "; each 16-B field is read as a whole 32-B sector of its 64-B "
+                                                      "record plus PCIe TLP overhead per completion, ~4.4x the field "
+                                                      "bytes by construction, not re-reads"}.get(args.workload, "")
                                    if dom == "zc" else ""))
     if dom == "zc" and args.workload == "grep":
         # the zero-copy key gather is PCIe read-request bound, not byte bound: one read request per
