@@ -27,6 +27,9 @@ def lib():
         l.mt_grep.argtypes = [p, u64, p, u64, p, u32, p, u64]
         l.mt_groupby.argtypes = [p, u64, u32, u32, p, p, p]
         l.mt_kmeans.argtypes = [p, u64, p, u32, p, p]
+        l.mt_partition.argtypes = [p, u64, u32, p, p]
+        l.mt_kmer.restype = C.c_int64
+        l.mt_kmer.argtypes = [p, u64, u32, u32, u32, u32, u64, p, p, u64]
         _lib = l
     return _lib
 
@@ -55,3 +58,28 @@ def kmeans(x, mu):
     c = np.empty(K, np.uint64); s = np.empty((K, 16), np.float64)
     lib().mt_kmeans(x.ctypes.data, len(x), mu.ctypes.data, K, c.ctypes.data, s.ctypes.data)
     return c, s
+
+
+def partition(kv, B=1024):
+    """(boff u64[B+1], out u64[n,2]) stable bucket-major, like oracle.partition."""
+    kv = np.ascontiguousarray(kv, np.uint64).reshape(-1, 2)
+    out = np.empty_like(kv)
+    boff = np.empty(B + 1, np.uint64)
+    lib().mt_partition(kv.ctypes.data, len(kv), B, out.ctypes.data, boff.ctypes.data)
+    return boff, out
+
+
+def kmer(recs, n, k=31, rec_size=256, seq_off=16, seq_len=96, slots=None):
+    """(kmers u64 ascending, counts u64), like oracle.kmer."""
+    slots = slots or 1 << max(16, int(2 * n * (seq_len - k + 1)).bit_length())
+    cap = 1 << 16
+    while True:
+        km = np.empty(cap, np.uint64); ct = np.empty(cap, np.uint64)
+        V = lib().mt_kmer(recs.ctypes.data, n, rec_size, seq_off, seq_len, k, slots, km.ctypes.data, ct.ctypes.data,
+                          cap)
+        if V == -1:
+            raise RuntimeError("k-mer table full")
+        if V >= 0:
+            o = np.argsort(km[:V])
+            return km[:V][o], ct[:V][o]
+        cap = -V

@@ -101,3 +101,92 @@ void mt_kmeans(const float* x, uint64_t n, const float* mu, uint32_t K, uint64_t
     free(s);
   }
 }
+
+/* ---- partition (C4): stable bucket-major partition by mix64(key) >> (64 - log2 B) ----------------
+ * Two passes over per-thread contiguous ranges: per-thread bucket histograms, a (bucket, thread)
+ * exclusive scan, then a stable scatter. boff: B+1 bucket offsets. */
+static inline uint64_t mt_mix64(uint64_t x) {
+  x ^= x >> 30; x *= 0xbf58476d1ce4e5b9ull;
+  x ^= x >> 27; x *= 0x94d049bb133111ebull;
+  x ^= x >> 31;
+  return x;
+}
+
+void mt_partition(const uint64_t* kv, uint64_t n, uint32_t B, uint64_t* out, uint64_t* boff) {
+  int bits = 0;
+  while ((1u << bits) < B) ++bits;
+  const int T = omp_get_max_threads();
+  uint64_t* h = calloc((size_t)T * B, 8);
+#pragma omp parallel num_threads(T)
+  {
+    const int t = omp_get_thread_num();
+    const uint64_t lo = n * t / T, hi = n * (t + 1) / T;
+    uint64_t* ht = h + (size_t)t * B;
+    for (uint64_t i = lo; i < hi; ++i) ht[bits ? mt_mix64(kv[2 * i]) >> (64 - bits) : 0]++;
+#pragma omp barrier
+#pragma omp single
+    {
+      uint64_t acc = 0;
+      for (uint32_t b = 0; b < B; ++b) {
+        boff[b] = acc;
+        for (int u = 0; u < T; ++u) { const uint64_t c = h[(size_t)u * B + b]; h[(size_t)u * B + b] = acc; acc += c; }
+      }
+      boff[B] = acc;
+    }
+    for (uint64_t i = lo; i < hi; ++i) {
+      const uint64_t b = bits ? mt_mix64(kv[2 * i]) >> (64 - bits) : 0;
+      const uint64_t p = ht[b]++;
+      out[2 * p] = kv[2 * i];
+      out[2 * p + 1] = kv[2 * i + 1];
+    }
+  }
+  free(h);
+}
+
+/* ---- k-mers (f4): exact-key concurrent open-addressing table (key = 2-bit k-mer + 1) ------------
+ * Returns the number of distinct k-mers written (unordered) to kmer/cnt, or -(needed) if cap is
+ * too small; -1 if the table filled up. */
+int64_t mt_kmer(const uint8_t* recs, uint64_t n, uint32_t rec_size, uint32_t seq_off, uint32_t seq_len, uint32_t k,
+                uint64_t slots, uint64_t* kmer, uint64_t* cnt, uint64_t cap) {
+  uint64_t* key = calloc(slots, 8);
+  uint64_t* val = calloc(slots, 8);
+  const uint64_t mask = slots - 1, kmask = k == 32 ? ~0ull : ((1ull << (2 * k)) - 1);
+  int full = 0;
+#pragma omp parallel for schedule(dynamic, 4096) reduction(| : full)
+  for (uint64_t r = 0; r < n; ++r) {
+    const uint8_t* s = recs + r * rec_size + seq_off;
+    uint64_t v = 0;
+    uint32_t valid = 0;
+    for (uint32_t i = 0; i < seq_len; ++i) {
+      const uint8_t ch = s[i];
+      const int code = ch == 'A' ? 0 : ch == 'C' ? 1 : ch == 'G' ? 2 : ch == 'T' ? 3 : -1;
+      if (code < 0) { valid = 0; v = 0; continue; }
+      v = ((v << 2) | (uint64_t)code) & kmask;
+      if (++valid < k) continue;
+      const uint64_t kk = v + 1;
+      uint64_t slot = mt_mix64(kk) & mask, probe = 0;
+      for (; probe <= mask; ++probe, slot = (slot + 1) & mask) {
+        uint64_t cur = __atomic_load_n(&key[slot], __ATOMIC_RELAXED);
+        if (cur == 0) {
+          uint64_t z = 0;
+          if (__atomic_compare_exchange_n(&key[slot], &z, kk, 0, __ATOMIC_RELAXED, __ATOMIC_RELAXED)) cur = kk;
+          else cur = z;
+        }
+        if (cur == kk) { __atomic_fetch_add(&val[slot], 1, __ATOMIC_RELAXED); break; }
+      }
+      if (probe > mask) full = 1;
+    }
+  }
+  int64_t V = 0;
+  if (!full) {
+    for (uint64_t i = 0; i < slots; ++i)
+      if (key[i]) {
+        if ((uint64_t)V < cap) { kmer[V] = key[i] - 1; cnt[V] = val[i]; }
+        ++V;
+      }
+    if ((uint64_t)V > cap) V = -V;
+  }
+  free(key);
+  free(val);
+  return full ? -1 : V;
+}

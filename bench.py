@@ -670,8 +670,9 @@ def main():
                                  "bigkernel_speedup": round(value / dv, 3)}
         dctx.close()
     if rank == 0 and not args.no_cpu_baseline and args.impl == "ours" and args.workload in (
-            "grep", "groupby", "groupby_sparse", "kmeans"):
-        # the paper's multithreaded CPU variant (ii) on all host cores, same shard (kmeans: 1/16 sample)
+            "grep", "groupby", "groupby_sparse", "kmeans", "partition", "kmer"):
+        # the paper's multithreaded CPU variant (ii) on all host cores, same shard (kmeans: 1/16 sample,
+        # k-mers: 1/4 sample)
         import baselines
         t0 = time.perf_counter()
         if args.workload == "grep":
@@ -681,6 +682,13 @@ def main():
             m = shard["n"] // 16
             baselines.kmeans(shard["buf"][: m * 64].view(np.float32).reshape(-1, 16), shard["mu"])
             mt_bytes = m * 64
+        elif args.workload == "partition":
+            baselines.partition(shard["buf"].view(np.uint64).reshape(-1, 2), 1024)
+            mt_bytes = nbytes
+        elif args.workload == "kmer":
+            m = shard["n"] // 4   # a quarter of the reads, into the same 2^28-slot table size as the GPU's
+            baselines.kmer(shard["buf"][: m * 256], m, k=31, slots=1 << 28)
+            mt_bytes = m * 256
         else:
             baselines.groupby(shard["buf"], shard["n"], shard["rec_size"], 4096)
             mt_bytes = nbytes

@@ -20,3 +20,15 @@ def test_mt_baseline_matches_oracle():
     assert np.array_equal(c, kc)
     np.testing.assert_allclose(s, ks, rtol=1e-9)
     assert baselines.threads() >= 1
+
+
+def test_mt_partition_and_kmer_match_oracle():
+    kv = gen.kv(n=200_003)
+    for B in (1024, 1):
+        boff, out = baselines.partition(kv, B)
+        wboff, wout = oracle.partition(kv, B)
+        assert np.array_equal(boff, wboff) and np.array_equal(out, wout)
+    d = gen.dna(n=5000, genome_len=1 << 14, err_pm=3, n_pm=3)
+    km, ct = baselines.kmer(d, 5000)
+    okm, oct_ = oracle.kmer(d, 5000)
+    assert np.array_equal(km, okm) and np.array_equal(ct, oct_)
