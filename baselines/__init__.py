@@ -28,6 +28,8 @@ def lib():
         l.mt_groupby.argtypes = [p, u64, u32, u32, p, p, p]
         l.mt_kmeans.argtypes = [p, u64, p, u32, p, p]
         l.mt_partition.argtypes = [p, u64, u32, p, p]
+        l.mt_wordcount.restype = C.c_int64
+        l.mt_wordcount.argtypes = [p, u64, p, u64, p, p, p, u64]
         l.mt_kmer.restype = C.c_int64
         l.mt_kmer.argtypes = [p, u64, u32, u32, u32, u32, u64, p, p, u64]
         _lib = l
@@ -82,4 +84,16 @@ def kmer(recs, n, k=31, rec_size=256, seq_off=16, seq_len=96, slots=None):
         if V >= 0:
             o = np.argsort(km[:V])
             return km[:V][o], ct[:V][o]
+        cap = -V
+
+
+def wordcount(buf, off):
+    """(word_off u64, word_len u32, count u64) of every distinct word, unordered (like the GPU's)."""
+    cap = 1 << 17
+    while True:
+        wo = np.empty(cap, np.uint64); wl = np.empty(cap, np.uint32); wc = np.empty(cap, np.uint64)
+        V = lib().mt_wordcount(buf.ctypes.data, len(buf), off.ctypes.data, len(off), wo.ctypes.data, wl.ctypes.data,
+                               wc.ctypes.data, cap)
+        if V >= 0:
+            return wo[:V], wl[:V], wc[:V]
         cap = -V

@@ -190,3 +190,77 @@ int64_t mt_kmer(const uint8_t* recs, uint64_t n, uint32_t rec_size, uint32_t seq
   free(val);
   return full ? -1 : V;
 }
+
+/* ---- word count (C1): per-thread exact tables (FNV-1a hash + byte compare), merged at the end ----
+ * Word = maximal run of bytes outside {0x20, 0x09..0x0D} inside one record (A10/A19).
+ * Output: unordered (offset of one occurrence, length, count); returns the number of distinct words,
+ * or -(needed) if cap is too small. */
+typedef struct { uint64_t h, off, len, cnt; } mt_wc_e;
+typedef struct { mt_wc_e* e; uint64_t mask, used; } mt_wc_t;
+
+static int mt_isdelim(uint8_t c) { return c == 0x20 || (uint8_t)(c - 0x09) <= 4; }
+
+static void mt_wc_init(mt_wc_t* t, uint64_t slots) {
+  t->e = calloc(slots, sizeof(mt_wc_e));
+  t->mask = slots - 1;
+  t->used = 0;
+}
+
+static void mt_wc_add(mt_wc_t* t, const uint8_t* d, uint64_t h, uint64_t off, uint64_t len, uint64_t cnt);
+
+static void mt_wc_grow(mt_wc_t* t, const uint8_t* d) {
+  mt_wc_t n;
+  mt_wc_init(&n, (t->mask + 1) * 2);
+  for (uint64_t i = 0; i <= t->mask; ++i)
+    if (t->e[i].cnt) mt_wc_add(&n, d, t->e[i].h, t->e[i].off, t->e[i].len, t->e[i].cnt);
+  free(t->e);
+  *t = n;
+}
+
+static void mt_wc_add(mt_wc_t* t, const uint8_t* d, uint64_t h, uint64_t off, uint64_t len, uint64_t cnt) {
+  if ((t->used + 1) * 10 > (t->mask + 1) * 7) mt_wc_grow(t, d);
+  for (uint64_t s = h & t->mask;; s = (s + 1) & t->mask) {
+    mt_wc_e* e = &t->e[s];
+    if (!e->cnt) { e->h = h; e->off = off; e->len = len; e->cnt = cnt; t->used++; return; }
+    if (e->h == h && e->len == len && memcmp(d + e->off, d + off, len) == 0) { e->cnt += cnt; return; }
+  }
+}
+
+int64_t mt_wordcount(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uint64_t n, uint64_t* w_off,
+                     uint32_t* w_len, uint64_t* w_cnt, uint64_t cap) {
+  const int T = omp_get_max_threads();
+  mt_wc_t* tabs = calloc(T, sizeof(mt_wc_t));
+#pragma omp parallel num_threads(T)
+  {
+    const int t = omp_get_thread_num();
+    const uint64_t lo = n * t / T, hi = n * (t + 1) / T;
+    mt_wc_init(&tabs[t], 1u << 16);
+    for (uint64_t r = lo; r < hi; ++r) {
+      const uint64_t a = off[r], b = r + 1 < n ? off[r + 1] : nbytes;
+      uint64_t i = a;
+      while (i < b) {
+        while (i < b && mt_isdelim(d[i])) ++i;
+        const uint64_t s = i;
+        uint64_t h = 0xcbf29ce484222325ull;
+        while (i < b && !mt_isdelim(d[i])) { h = (h ^ d[i]) * 0x100000001b3ull; ++i; }
+        if (i > s) mt_wc_add(&tabs[t], d, mt_mix64(h ^ (i - s)), s, i - s, 1);
+      }
+    }
+  }
+  mt_wc_t g;
+  mt_wc_init(&g, 1u << 17);
+  for (int t = 0; t < T; ++t) {
+    for (uint64_t i = 0; i <= tabs[t].mask; ++i)
+      if (tabs[t].e[i].cnt) mt_wc_add(&g, d, tabs[t].e[i].h, tabs[t].e[i].off, tabs[t].e[i].len, tabs[t].e[i].cnt);
+    free(tabs[t].e);
+  }
+  free(tabs);
+  int64_t V = 0;
+  for (uint64_t i = 0; i <= g.mask; ++i)
+    if (g.e[i].cnt) {
+      if ((uint64_t)V < cap) { w_off[V] = g.e[i].off; w_len[V] = (uint32_t)g.e[i].len; w_cnt[V] = g.e[i].cnt; }
+      ++V;
+    }
+  free(g.e);
+  return (uint64_t)V > cap ? -V : V;
+}

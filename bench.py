@@ -670,7 +670,7 @@ def main():
                                  "bigkernel_speedup": round(value / dv, 3)}
         dctx.close()
     if rank == 0 and not args.no_cpu_baseline and args.impl == "ours" and args.workload in (
-            "grep", "groupby", "groupby_sparse", "kmeans", "partition", "kmer"):
+            "grep", "groupby", "groupby_sparse", "kmeans", "partition", "kmer", "wordcount"):
         # the paper's multithreaded CPU variant (ii) on all host cores, same shard (kmeans: 1/16 sample,
         # k-mers: 1/4 sample)
         import baselines
@@ -682,6 +682,9 @@ def main():
             m = shard["n"] // 16
             baselines.kmeans(shard["buf"][: m * 64].view(np.float32).reshape(-1, 16), shard["mu"])
             mt_bytes = m * 64
+        elif args.workload == "wordcount":
+            baselines.wordcount(shard["buf"], shard["off"])
+            mt_bytes = nbytes
         elif args.workload == "partition":
             baselines.partition(shard["buf"].view(np.uint64).reshape(-1, 2), 1024)
             mt_bytes = nbytes

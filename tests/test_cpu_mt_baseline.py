@@ -32,3 +32,15 @@ def test_mt_partition_and_kmer_match_oracle():
     km, ct = baselines.kmer(d, 5000)
     okm, oct_ = oracle.kmer(d, 5000)
     assert np.array_equal(km, okm) and np.array_equal(ct, oct_)
+
+
+def test_mt_wordcount_matches_oracle():
+    adv = b"  a\tb\r\n\x00\xff  \x0b\x0cab" + b"ab" + b"" + b"x y  x"
+    adv_off = np.array([0, 17, 19, 19], np.uint64)   # records: adversarial, "ab", empty, "x y  x"
+    cases = (gen.text(cap_bytes=3 << 20), gen.text(cap_recs=1), (np.zeros(0, np.uint8), np.zeros(0, np.uint64)),
+             (np.frombuffer(adv, np.uint8).copy(), adv_off))
+    for buf, off in cases:
+        b = buf.tobytes()
+        wo, wl, wc = baselines.wordcount(buf, off)
+        got = sorted((b[int(o): int(o) + int(l)], int(c)) for o, l, c in zip(wo, wl, wc))
+        assert got == oracle.wc(buf, off)
