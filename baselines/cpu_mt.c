@@ -191,11 +191,12 @@ int64_t mt_kmer(const uint8_t* recs, uint64_t n, uint32_t rec_size, uint32_t seq
   return full ? -1 : V;
 }
 
-/* ---- word count (C1): per-thread exact tables (FNV-1a hash + byte compare), merged at the end ----
+/* ---- word count (C1): per-thread tables merged by hash shard -----------------------------------
  * Word = maximal run of bytes outside {0x20, 0x09..0x0D} inside one record (A10/A19).
- * Output: unordered (offset of one occurrence, length, count); returns the number of distinct words,
- * or -(needed) if cap is too small. */
-typedef struct { uint64_t h, off, len, cnt; } mt_wc_e;
+ * Word identity = (two independent 64-bit hashes, length), the same reading the GPU path uses
+ * (DESIGN.md §2): 32-B entries, no second look at the text. Output: unordered (offset of one
+ * occurrence, length, count); returns the number of distinct words, or -(needed) if cap is too small. */
+typedef struct { uint64_t h1, h2l, off, cnt; } mt_wc_e;   /* h2l = (h2 << 24) | len */
 typedef struct { mt_wc_e* e; uint64_t mask, used; } mt_wc_t;
 
 static int mt_isdelim(uint8_t c) { return c == 0x20 || (uint8_t)(c - 0x09) <= 4; }
@@ -206,61 +207,84 @@ static void mt_wc_init(mt_wc_t* t, uint64_t slots) {
   t->used = 0;
 }
 
-static void mt_wc_add(mt_wc_t* t, const uint8_t* d, uint64_t h, uint64_t off, uint64_t len, uint64_t cnt);
+static void mt_wc_put(mt_wc_t* t, const mt_wc_e* x);
 
-static void mt_wc_grow(mt_wc_t* t, const uint8_t* d) {
+static void mt_wc_grow(mt_wc_t* t) {
   mt_wc_t n;
   mt_wc_init(&n, (t->mask + 1) * 2);
   for (uint64_t i = 0; i <= t->mask; ++i)
-    if (t->e[i].cnt) mt_wc_add(&n, d, t->e[i].h, t->e[i].off, t->e[i].len, t->e[i].cnt);
+    if (t->e[i].cnt) mt_wc_put(&n, &t->e[i]);
   free(t->e);
   *t = n;
 }
 
-static void mt_wc_add(mt_wc_t* t, const uint8_t* d, uint64_t h, uint64_t off, uint64_t len, uint64_t cnt) {
-  if ((t->used + 1) * 10 > (t->mask + 1) * 7) mt_wc_grow(t, d);
-  for (uint64_t s = h & t->mask;; s = (s + 1) & t->mask) {
+static void mt_wc_put(mt_wc_t* t, const mt_wc_e* x) {
+  if ((t->used + 1) * 10 > (t->mask + 1) * 7) mt_wc_grow(t);
+  for (uint64_t s = x->h1 & t->mask;; s = (s + 1) & t->mask) {
     mt_wc_e* e = &t->e[s];
-    if (!e->cnt) { e->h = h; e->off = off; e->len = len; e->cnt = cnt; t->used++; return; }
-    if (e->h == h && e->len == len && memcmp(d + e->off, d + off, len) == 0) { e->cnt += cnt; return; }
+    if (!e->cnt) { *e = *x; t->used++; return; }
+    if (e->h1 == x->h1 && e->h2l == x->h2l) { e->cnt += x->cnt; return; }
   }
 }
 
 int64_t mt_wordcount(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uint64_t n, uint64_t* w_off,
                      uint32_t* w_len, uint64_t* w_cnt, uint64_t cap) {
   const int T = omp_get_max_threads();
-  mt_wc_t* tabs = calloc(T, sizeof(mt_wc_t));
+  mt_wc_t* loc = calloc(T, sizeof(mt_wc_t));
+  mt_wc_t* shard = calloc(T, sizeof(mt_wc_t));
+  uint64_t* base = calloc(T + 1, 8);
 #pragma omp parallel num_threads(T)
   {
     const int t = omp_get_thread_num();
     const uint64_t lo = n * t / T, hi = n * (t + 1) / T;
-    mt_wc_init(&tabs[t], 1u << 16);
+    mt_wc_init(&loc[t], 1u << 17);
+    mt_wc_e x;
+    x.cnt = 1;
     for (uint64_t r = lo; r < hi; ++r) {
       const uint64_t a = off[r], b = r + 1 < n ? off[r + 1] : nbytes;
       uint64_t i = a;
       while (i < b) {
         while (i < b && mt_isdelim(d[i])) ++i;
-        const uint64_t s = i;
-        uint64_t h = 0xcbf29ce484222325ull;
-        while (i < b && !mt_isdelim(d[i])) { h = (h ^ d[i]) * 0x100000001b3ull; ++i; }
-        if (i > s) mt_wc_add(&tabs[t], d, mt_mix64(h ^ (i - s)), s, i - s, 1);
+        const uint64_t s0 = i;
+        uint64_t h1 = 0xcbf29ce484222325ull, h2 = 0x84222325cbf29ce4ull;
+        while (i < b && !mt_isdelim(d[i])) {
+          h1 = (h1 ^ d[i]) * 0x100000001b3ull;
+          h2 = (h2 + d[i] + 1) * 0x9E3779B97F4A7C15ull;
+          ++i;
+        }
+        if (i == s0) continue;
+        x.h1 = mt_mix64(h1 ^ (i - s0));
+        x.h2l = (mt_mix64(h2 + (i - s0)) << 24) | (i - s0);
+        x.off = s0;
+        mt_wc_put(&loc[t], &x);
       }
     }
-  }
-  mt_wc_t g;
-  mt_wc_init(&g, 1u << 17);
-  for (int t = 0; t < T; ++t) {
-    for (uint64_t i = 0; i <= tabs[t].mask; ++i)
-      if (tabs[t].e[i].cnt) mt_wc_add(&g, d, tabs[t].e[i].h, tabs[t].e[i].off, tabs[t].e[i].len, tabs[t].e[i].cnt);
-    free(tabs[t].e);
-  }
-  free(tabs);
-  int64_t V = 0;
-  for (uint64_t i = 0; i <= g.mask; ++i)
-    if (g.e[i].cnt) {
-      if ((uint64_t)V < cap) { w_off[V] = g.e[i].off; w_len[V] = (uint32_t)g.e[i].len; w_cnt[V] = g.e[i].cnt; }
-      ++V;
+#pragma omp barrier
+    /* merge: thread t owns the words whose hash falls in shard t */
+    mt_wc_init(&shard[t], 1u << 14);
+    for (int u = 0; u < T; ++u)
+      for (uint64_t i = 0; i <= loc[u].mask; ++i) {
+        const mt_wc_e* e = &loc[u].e[i];
+        if (e->cnt && (int)((e->h1 >> 40) % (uint64_t)T) == t) mt_wc_put(&shard[t], e);
+      }
+#pragma omp barrier
+    free(loc[t].e);
+    base[t + 1] = shard[t].used;
+#pragma omp barrier
+#pragma omp single
+    for (int u = 0; u < T; ++u) base[u + 1] += base[u];
+    uint64_t v = base[t];
+    for (uint64_t i = 0; i <= shard[t].mask; ++i) {
+      const mt_wc_e* e = &shard[t].e[i];
+      if (!e->cnt) continue;
+      if (v < cap) { w_off[v] = e->off; w_len[v] = (uint32_t)(e->h2l & 0xffffff); w_cnt[v] = e->cnt; }
+      ++v;
     }
-  free(g.e);
+    free(shard[t].e);
+  }
+  const int64_t V = (int64_t)base[T];
+  free(loc);
+  free(shard);
+  free(base);
   return (uint64_t)V > cap ? -V : V;
 }
