@@ -33,5 +33,7 @@ for w in ("grep", "groupby", "groupby_sparse", "kmeans", "partition", "wordcount
           f"{d2h:.1f} | {comp:.1f} | {slow} ({stages[slow]:.1f}) | {ag / stages[slow]:.1%} |")
 print("\nThe paper's address-generation observation holds on B200 for every workload except word count, "
       "whose stage 1 reads each chunk's offsets zero-copy (one thread per record) and, at 0.44-MB chunks, is "
-      "launch- and latency-dominated; it runs a chunk ahead on double-buffered descriptors, off the "
-      "critical chain (DESIGN.md §1).")
+      "launch- and latency-dominated (these are eager-pass sums). On double-buffered descriptors it runs "
+      "alongside the slot's previous compute; issuing it a whole ring earlier on its own streams (gated "
+      "only by the compute that last used its descriptor set) was measured at 32.1 vs 33.3 GB/s "
+      "(`tools/gpu_lookahead.sh`, reverted), so it does not hold the step back.")
