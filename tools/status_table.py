@@ -1,0 +1,58 @@
+#!/usr/bin/env python3
+"""DESIGN.md §9 / README status rows from the committed bench lines (profiles/r01_bench_*.json).
+
+    python tools/status_table.py design   # the §9 table rows
+    python tools/status_table.py readme   # the README table rows
+"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROWS = [
+    ("grep", "C2 grep 16 GiB (default bench)", "Grep, 16 GiB", "host-packing / PCIe-request-rate bound"),
+    ("groupby", "C5 group-by 16 GiB dense", "Group-by, 16 GiB", ""),
+    ("groupby_sparse", "C5 group-by sparse 16 GiB (64-B records, 25% read)", "Group-by sparse (25% read), 16 GiB", ""),
+    ("kmeans", "C3 k-means 16 GiB, K=64", "K-means, 16 GiB", ""),
+    ("partition", "C4 partition 8 GiB, 1024 buckets (D2H out)", "Partition, 8 GiB", ""),
+    ("wordcount", "C1 word count 64 MiB, 8 MiB window, 8 slots", "Word count, 64 MiB (8 MiB window)", ""),
+    ("kmer", "f4 k-mers 4 GiB (k = 31)", "k-mers, 4 GiB", "random-access bound table updates"),
+]
+
+
+def load(w):
+    return json.load(open(os.path.join(ROOT, "profiles", f"r01_bench_{w}.json")))
+
+
+def gbs(v):
+    return f"{v:.1f} GB/s" if v >= 1 else f"{v:.2g} GB/s"
+
+
+def design():
+    for w, name, _, _ in ROWS:
+        d = load(w)
+        fd = d.get("link_full_duplex")
+        val = f"{d['value']:.1f} each way" if fd else f"{d['value']:.1f}"
+        frac = (f"{d['link']['frac']:.2f} (H2D); {fd['frac']:.2f} of the {fd['peak_each_way_gbs']:.1f} GB/s "
+                f"bidirectional per-direction peak") if fd else f"{d['link']['frac']:.2f}"
+        db = d.get("baseline_dbuf")
+        dbs = f"{db['bigkernel_speedup']:.2f}× ({db['value']:.1f})" if db else "—"
+        mt = d.get("cpu_mt_baseline")
+        print(f"| {name} | {d['config']['gather_mode'].upper()} | {val} | {d['ms_per_step']:.3g} | {frac} | "
+              f"{d['overlap']['overlap_frac']:.2f} | {dbs} | {gbs(mt['value']) if mt else '—'} | "
+              f"{gbs(d['cpu_baseline']['value'])} |")
+
+
+def readme():
+    for w, _, name, note in ROWS:
+        d = load(w)
+        fd = d.get("link_full_duplex")
+        val = f"{d['value']:.1f} each way" if fd else f"{d['value']:.1f}"
+        frac = f"{fd['frac']:.2f} of bidirectional" if fd else f"{d['link']['frac']:.2f}" + (f" ({note})" if note else "")
+        db = d.get("baseline_dbuf")
+        sp = f"{db['bigkernel_speedup']:.2f}×" if db else "—"
+        print(f"| {name} | {val} | {frac} | {sp} |")
+
+
+if __name__ == "__main__":
+    {"design": design, "readme": readme}[sys.argv[1] if len(sys.argv) > 1 else "design"]()
