@@ -23,6 +23,7 @@ def lib():
         l = C.CDLL(_SO)
         p, u64, u32 = C.c_void_p, C.c_uint64, C.c_uint32
         l.mt_threads.restype = C.c_int
+        l.mt_set_threads.argtypes = [C.c_int]
         l.mt_grep.restype = C.c_int64
         l.mt_grep.argtypes = [p, u64, p, u64, p, u32, p, u64]
         l.mt_groupby.argtypes = [p, u64, u32, u32, p, p, p]
@@ -38,6 +39,11 @@ def lib():
 
 def threads() -> int:
     return lib().mt_threads()
+
+
+def set_threads(n: int) -> None:
+    """OpenMP thread count of the baseline (torchrun sets OMP_NUM_THREADS=1 for N > 1 ranks)."""
+    lib().mt_set_threads(int(n))
 
 
 def grep(buf, off, pattern: bytes = b"bigk"):

@@ -9,6 +9,7 @@
 #include <string.h>
 
 int mt_threads(void) { return omp_get_max_threads(); }
+void mt_set_threads(int n) { if (n > 0) omp_set_num_threads(n); }
 
 /* grep: returns the match count; indices are written in ascending order (per-thread buffers). */
 int64_t mt_grep(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uint64_t n, const uint8_t* pat,

@@ -674,6 +674,11 @@ def main():
         # the paper's multithreaded CPU variant (ii) on all host cores, same shard (kmeans: 1/16 sample,
         # k-mers: 1/4 sample)
         import baselines
+        # all host cores (the variant-ii CPU baseline is the whole box's CPU), whatever OMP_NUM_THREADS
+        # torchrun set and whatever NUMA-local affinity this rank's GPU pipeline runs under
+        saved_aff = os.sched_getaffinity(0)
+        os.sched_setaffinity(0, range(os.cpu_count() or 1))
+        baselines.set_threads(os.cpu_count() or 1)
         if args.workload == "wordcount":   # steady state: its per-thread tables persist across calls
             baselines.wordcount(shard["buf"], shard["off"])
         t0 = time.perf_counter()
@@ -698,6 +703,7 @@ def main():
             baselines.groupby(shard["buf"], shard["n"], shard["rec_size"], 4096)
             mt_bytes = nbytes
         mt = mt_bytes / (time.perf_counter() - t0) / 1e9
+        os.sched_setaffinity(0, saved_aff)
         line["cpu_mt_baseline"] = {"value": round(mt, 3), "unit": "GB/s", "cores": baselines.threads(),
                                    "what": "paper variant (ii): OpenMP over all host cores (baselines/cpu_mt.c)",
                                    "bigkernel_speedup": round(value / mt, 3)}
