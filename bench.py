@@ -677,7 +677,10 @@ def main():
         # all host cores (the variant-ii CPU baseline is the whole box's CPU), whatever OMP_NUM_THREADS
         # torchrun set and whatever NUMA-local affinity this rank's GPU pipeline runs under
         saved_aff = os.sched_getaffinity(0)
-        os.sched_setaffinity(0, range(os.cpu_count() or 1))
+        try:
+            os.sched_setaffinity(0, range(os.cpu_count() or 1))
+        except OSError:
+            pass
         baselines.set_threads(os.cpu_count() or 1)
         if args.workload == "wordcount":   # steady state: its per-thread tables persist across calls
             baselines.wordcount(shard["buf"], shard["off"])
