@@ -390,12 +390,12 @@ def mix64_np(x):
     return x
 
 
-def test_kmeans_bench_scale_sampled():
-    """C3 per-GPU share at 2 GPUs would be 5e8 points; here 2.5e8 (16 GiB, bench.py's default
-    k-means size) in bench.py's launch configuration (2 GiB window, AUTO). Checked: every cid the
-    oracle computes for 200k sampled points, Sum count = n, count = bincount(cid), the checksum
-    recomputed from the written-back cids, and column sums."""
-    n = 250_000_000
+@pytest.mark.parametrize("n", [250_000_000, 500_000_000])
+def test_kmeans_bench_scale_sampled(n):
+    """2.5e8 points (16 GiB, bench.py's default k-means size) and 5e8 (32 GiB, C3's per-GPU share at
+    2 GPUs) in bench.py's launch configuration (2 GiB window, AUTO). Checked: every cid the oracle
+    computes for 200k sampled points, Sum count = n, count = bincount(cid), the checksum recomputed
+    from the written-back cids, and column sums."""
     x = gen.points(n=n)
     mu = gen.points(n=64)
     cid = np.empty(n, np.int32)
