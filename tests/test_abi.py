@@ -61,3 +61,26 @@ def test_product_package_never_imports_the_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".cpp", ".h")):
                 txt = open(os.path.join(dirpath, f)).read()
                 assert "oracle" not in txt.replace("never imports the oracle", "").replace("never the oracle", ""), f
+
+
+def test_header_is_plain_c_and_links(tmp_path):
+    """include/bk.h compiles as C99 and C++17, and a plain C program links against libbk.so and calls
+    the GPU-free entry points (no torch, no CUDA headers in the signatures)."""
+    import shutil
+    if not shutil.which("gcc"):
+        pytest.skip("no gcc")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    src = tmp_path / "abi.c"
+    src.write_text(
+        '#include "bk.h"\n#include <stdio.h>\n'
+        "int main(void) { unsigned s[12]; int v = bk_abi_sizes(s, 12);\n"
+        '  printf("%d %u %s\\n", v, s[0], bk_strerror(BK_E_RANGE));\n'
+        "  return bk_destroy(NULL); }\n")
+    exe = tmp_path / "abi"
+    libdir = os.path.join(root, "paper_conf_ipps_mokhtaris14_b200")
+    subprocess.check_call(["gcc", "-std=c99", "-Wall", "-Werror", "-I", os.path.join(root, "include"), str(src),
+                           "-L", libdir, "-l:libbk.so", "-Wl,-rpath," + libdir, "-o", str(exe)])
+    subprocess.check_call(["g++", "-std=c++17", "-Wall", "-Werror", "-fsyntax-only", "-x", "c++",
+                           os.path.join(root, "include", "bk.h")])
+    out = subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()
+    assert int(out[1]) == bk.abi_sizes()[0] and "record" in " ".join(out[2:])
