@@ -64,6 +64,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-dbuf", action="store_true", help="skip the double-buffering baseline measurement")
     ap.add_argument("--no-profile", action="store_true", help="disable per-stage event timing")
+    ap.add_argument("--dump", default=None, help="after the timed steps, run one more step and write this rank's "
+                                                 "(merged) result to DUMP/rank<r>.npz (the N>1 parity tests)")
     args = ap.parse_args()
     if args.slots == 0 and args.workload == "wordcount":
         args.slots = 8   # the 8 MiB window: more, smaller chunks in flight (profiles/r01_wc_sweep.md)
@@ -351,57 +353,82 @@ def main():
     ctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
                      baseline_dbuf=args.impl == "dbuf", baseline_sbuf=args.impl == "sbuf",
                      host_threads=args.host_threads, lane_bytes=args.lane_bytes, zc_share_pm=args.zc_share,
-                     profile=False, record_size=shard["rec_size"])
+                     profile=False, record_size=shard["rec_size"], keep_outputs_pinned=True)
     t0 = time.perf_counter()
     ctx.register(shard["buf"], shard["off"], n_records=shard["n"])
     reg_s = time.perf_counter() - t0
     stream = torch.cuda.current_stream()
     nbytes = len(shard["buf"])
 
-    kmer_out = (np.empty(1 << 27, np.uint64), np.empty(1 << 27, np.uint64)) if args.workload == "kmer" else None
-    if kmer_out is not None:   # touch once: the result D2H must not pay first-touch page faults per step
-        kmer_out[0].fill(0)
-        kmer_out[1].fill(0)
     cap = max(shard["n"] // 50, 1 << 16)
     idx_out = np.empty(cap, np.uint64)
-    wc_out = None
-    if args.workload == "wordcount":   # reused result arrays, touched once (no per-step page faults)
-        wc_out = (np.zeros(1 << 20, np.uint64), np.zeros(1 << 20, np.uint32), np.zeros(1 << 20, np.uint64))
+    # result arrays, allocated (and touched) once and reused by every step: host arrays at N=1 (the
+    # caller reads its result on the host); at N>1 the aggregating kernels write device tensors that
+    # the merge collectives reduce / gather in place (bk.h: result arrays may be device memory)
+    kmer_out = wc_out = agg_out = None
+    if args.workload == "kmer":
+        kcap = 1 << 27
+        kmer_out = ((torch.zeros(kcap, dtype=torch.int64, device=dev), torch.zeros(kcap, dtype=torch.int64, device=dev))
+                    if world > 1 else (np.zeros(kcap, np.uint64), np.zeros(kcap, np.uint64)))
+    if args.workload == "wordcount":
+        wcap = 1 << 20
+        wc_out = ((torch.zeros(wcap, dtype=torch.int64, device=dev), torch.zeros(wcap, dtype=torch.int32, device=dev),
+                   torch.zeros(wcap, dtype=torch.int64, device=dev), torch.zeros(wcap, dtype=torch.int64, device=dev),
+                   torch.zeros(wcap, dtype=torch.int64, device=dev))
+                  if world > 1 else (np.zeros(wcap, np.uint64), np.zeros(wcap, np.uint32), np.zeros(wcap, np.uint64)))
+    if args.workload in ("groupby", "groupby_sparse"):
+        cq = torch.zeros(2, 4096, dtype=torch.int64, device=dev)
+        agg_out = ((cq[0], cq[1], torch.zeros(4096, dtype=torch.float64, device=dev), cq) if world > 1 else
+                   (np.zeros(4096, np.uint64), np.zeros(4096, np.uint64), np.zeros(4096, np.float64)))
+    if args.workload == "kmeans":
+        agg_out = ((torch.zeros(64, dtype=torch.int64, device=dev), torch.zeros(64, 16, dtype=torch.float64, device=dev))
+                   if world > 1 else (np.zeros(64, np.uint64), np.zeros((64, 16), np.float64)))
 
     from paper_conf_ipps_mokhtaris14_b200 import merge
 
     box = {}   # facts of the last step the roofline needs (k-mer windows)
 
     def one_step(ctx=ctx):
-        """One pass of the whole hot path over this rank's shard, then the merge (N>1)."""
+        """One pass of the whole hot path over this rank's shard, then the merge (N>1). Returns this
+        rank's (merged) result, for --dump."""
         cs = stream.cuda_stream
         if args.workload == "grep":
             res = ctx.grep(b"bigk", first_index=shard["first"], stream=cs, out=idx_out)
-            return merge.merge_grep_offsets(len(res)) if world > 1 else (0, len(res))
+            return {"idx": res, "place": merge.merge_grep_offsets(len(res)) if world > 1 else (0, len(res))}
         if args.workload == "wordcount":
-            o, l, c = ctx.wordcount(stream=cs, out=wc_out)
-            if world > 1:
-                b = shard["buf"]
-                return merge.merge_wordcount({b[int(x): int(x) + int(y)].tobytes(): int(z) for x, y, z in zip(o, l, c)})
-            return int(c.sum())
+            r = ctx.wordcount(stream=cs, out=wc_out)
+            if world > 1:   # all-gather of compacted {h1, h2, len, count, rank, off} rows, merged on the GPU
+                rows = merge.merge_wordcount(ctx, *r)
+                return {"rows": rows.cpu().numpy()}
+            return {"off": r[0], "len": r[1], "count": r[2]}
         if args.workload == "kmer":
             km, ct, total = ctx.kmer(k=31, table_slots=1 << 28, stream=cs, out=kmer_out)
             box["kmer_windows"] = total
-            t = torch.tensor([total, len(km)], dtype=torch.int64, device=dev)
-            return merge.merge_sum(t) if world > 1 else t
+            if world > 1:
+                rows = merge.merge_kmer(ctx, km, ct)
+                return {"rows": rows.cpu().numpy()}
+            return {"kmer": km, "count": ct}
         if args.workload == "partition":
             out, cc, bc = ctx.partition(1024, out=shard["out"], stream=cs)
             box["part_cc"] = cc
-            return merge.merge_partition_offsets(bc) if world > 1 else bc
-        if args.workload in ("groupby", "groupby_sparse"):
-            c, q, a = ctx.groupby(4096, stream=cs)
-            t = torch.from_numpy(np.stack([c.astype(np.float64), q.astype(np.float64), a])).to(dev)
-        else:
-            c, s_, chk = ctx.kmeans(shard["mu"], first_index=shard["first"], stream=cs)
-            t = torch.from_numpy(np.concatenate([c.astype(np.float64), s_.reshape(-1)])).to(dev)
             if world > 1:
-                merge.merge_checksum(chk)
-        return merge.merge_sum(t) if world > 1 else t
+                start, boff = merge.merge_partition_offsets(bc)
+                return {"start": start, "boff": boff, "cc": cc}
+            return {"cc": cc, "bc": bc}
+        if args.workload in ("groupby", "groupby_sparse"):
+            c, q, a = ctx.groupby(4096, stream=cs, out=agg_out[:3])
+            if world > 1:   # in place on the device buffers bk_run wrote
+                merge.merge_sum(agg_out[3])
+                merge.merge_sum(a)
+                return {"count": c.cpu().numpy(), "qty": q.cpu().numpy(), "amount": a.cpu().numpy()}
+            return {"count": c, "qty": q, "amount": a}
+        c, s_, chk = ctx.kmeans(shard["mu"], first_index=shard["first"], stream=cs, out=agg_out)
+        if world > 1:
+            merge.merge_sum(c)
+            merge.merge_sum(s_)
+            chk = merge.merge_checksum(chk)
+            return {"count": c.cpu().numpy(), "sum": s_.cpu().numpy(), "chk": chk}
+        return {"count": c, "sum": s_, "chk": chk}
 
     for _ in range(args.warmup):
         one_step()
@@ -445,13 +472,26 @@ def main():
                                       "the host (optional, timed separately, not part of value; destination pre-faulted)"}
         del dst
     st = dict(stats[-1])
+    if args.dump:
+        res = one_step()
+        torch.cuda.synchronize()
+        os.makedirs(args.dump, exist_ok=True)
+        flat = {}
+        for k, v in res.items():
+            if hasattr(v, "cpu"):
+                v = v.cpu().numpy()
+            flat[k] = np.asarray(v)
+        if args.workload == "partition":
+            flat["out"] = shard["out"]
+        np.savez(os.path.join(args.dump, f"rank{rank}.npz"), world=world, rank=rank, first=shard["first"],
+                 n=shard["n"], **flat)
     if not args.no_profile:
         # per-stage CUDA events force eager issue (graph event nodes carry no timestamps), so the
         # stage breakdown comes from a separate profiled pass over the same shard
         pctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
                           baseline_dbuf=args.impl == "dbuf", baseline_sbuf=args.impl == "sbuf",
                           host_threads=args.host_threads, lane_bytes=args.lane_bytes, zc_share_pm=args.zc_share,
-                          profile=True, record_size=shard["rec_size"])
+                          profile=True, record_size=shard["rec_size"], keep_outputs_pinned=True)
         pctx.register(shard["buf"], shard["off"], n_records=shard["n"])
         for _ in range(2):
             one_step(pctx)

@@ -23,7 +23,7 @@
 extern "C" {
 #endif
 
-#define BK_ABI_VERSION 1
+#define BK_ABI_VERSION 2
 #if defined(__GNUC__)
 #define BK_API __attribute__((visibility("default")))
 #else
@@ -100,6 +100,13 @@ typedef struct bk_config {
                                    host sleeps before CPU assembly, to expose missing ordering */
 #define BK_FLAG_BASELINE_SBUF 4u  /* the single-buffer variant: one buffer of the whole window,
                                      copy then compute, no overlap */
+#define BK_FLAG_KEEP_OUTPUTS_PINNED 32u  /* caller-owned per-record output arrays that bk_run writes by DMA
+                                     (bk_out_kmeans.cid, bk_out_partition.out_records, bk_out_kmer.kmer /
+                                     .count) are page-locked (cudaHostRegister) by bk_run. Default: only for
+                                     the duration of that bk_run (each run pays the registration, ~0.1 s per
+                                     GiB). With this flag the registration is cached across runs (at most four
+                                     arrays, oldest released first) and released by bk_unpin_outputs or
+                                     bk_destroy: the caller must keep such arrays allocated until then. */
 
 typedef struct bk_ctx bk_ctx;
 
@@ -113,7 +120,8 @@ BK_API int bk_create(const bk_config* cfg, bk_ctx** out_ctx);
  * each <= nbytes; record i = [off[i], off[i+1]) with off[n] := nbytes; empty records are legal.
  * record_offsets == NULL: fixed records of cfg.record_size bytes (nbytes % record_size == 0,
  * n_records must equal nbytes / record_size). Memory is pinned ONCE here (cudaHostRegister,
- * mapped + portable) unless already pinned; pre-pinned memory is left as is.
+ * mapped + portable + read-only where the device supports it: libbk never writes the data set)
+ * unless already pinned; pre-pinned memory is left as is.
  * Validation is O(n) once: BK_E_INVAL on malformed offsets. */
 BK_API int bk_register_segments(bk_ctx* ctx, const void* host_ptr, uint64_t nbytes,
                          const uint64_t* record_offsets, uint64_t n_records);
@@ -121,11 +129,18 @@ BK_API int bk_register_segments(bk_ctx* ctx, const void* host_ptr, uint64_t nbyt
 /* Runs built-in kernel `kernel_id` over every registered record through the pipeline.
  * Ordered after prior work on `stream`; returns when `out` is valid (blocking) and also
  * records completion on `stream`. `out` points to the kernel's caller-owned in/out struct
- * (bk_out_*), whose first two fields are {struct_size, kernel_id}. */
+ * (bk_out_*), whose first two fields are {struct_size, kernel_id}; struct_size must equal the
+ * sizeof of that kernel's struct (BK_E_INVAL), an unknown kernel_id is BK_E_UNSUPPORTED.
+ * The calling thread's current CUDA device is left unchanged. */
 BK_API int bk_run(bk_ctx* ctx, int kernel_id, void* stream, void* out);
 
-/* NULL-safe. Unpins what bk_register_segments pinned, frees device memory. */
+/* NULL-safe. Unpins what bk_register_segments pinned (and any output arrays kept pinned under
+ * BK_FLAG_KEEP_OUTPUTS_PINNED), frees device memory. */
 BK_API int bk_destroy(bk_ctx* ctx);
+
+/* Releases the output-array registrations cached under BK_FLAG_KEEP_OUTPUTS_PINNED, after which
+ * the caller may free those arrays. BK_E_INVAL on NULL. */
+BK_API int bk_unpin_outputs(bk_ctx* ctx);
 
 BK_API const char* bk_strerror(int status);
 BK_API const char* bk_last_error(void);
@@ -133,15 +148,21 @@ BK_API const char* bk_last_error(void);
 /* ---- per-kernel in/out structs (host pointers unless stated) ---- */
 typedef struct bk_out_header { uint32_t struct_size; int32_t kernel_id; } bk_out_header;
 
+/* Result arrays of the aggregating kernels (word count, group-by, k-means, k-mers) may be HOST or
+ * DEVICE pointers (device memory of the context's GPU): libbk copies with unified addressing, so a
+ * multi-GPU caller can point them at the buffers its NCCL collectives reduce in place (SURVEY
+ * §8(e)) with no host round trip. Host arrays need not be pinned. */
 typedef struct bk_out_wordcount {
   bk_out_header h;
   uint64_t table_slots;     /* in: device hash-table slots (power of two); 0 = 2^20 */
-  uint64_t cap;             /* in: capacity of the three arrays below */
+  uint64_t cap;             /* in: capacity of the arrays below */
   uint64_t* word_off;       /* out: offset (rel. host_ptr) of one occurrence of each distinct word */
   uint32_t* word_len;       /* out: its length */
   uint64_t* word_count;     /* out: its count (unordered; compare as a multiset) */
   uint64_t n_words;         /* out: distinct words (> cap -> BK_E_CAPACITY) */
   uint64_t total_words;     /* out */
+  uint64_t* word_h1;        /* out, optional (NULL): the word's identity, two 64-bit hashes of its bytes */
+  uint64_t* word_h2;        /*   and length — equal across GPUs, the key of the multi-GPU merge (bk_merge_counts) */
 } bk_out_wordcount;
 
 typedef struct bk_out_grep {
@@ -166,7 +187,8 @@ typedef struct bk_out_kmeans {
   uint64_t chk;             /* out: sum_i mix64((i<<8) ^ cid_i) mod 2^64 */
   int32_t* cid;             /* out, optional (NULL): n_records cluster ids written back to the host
                                (P:563-572 writes to mapped data): per chunk into the slot,
-                               then DMA'd on a D2H stream; the array is pinned once and cached */
+                               then DMA'd on a D2H stream (page-locked per run, or cached with
+                               BK_FLAG_KEEP_OUTPUTS_PINNED) */
 } bk_out_kmeans;
 
 typedef struct bk_out_partition {
@@ -182,7 +204,7 @@ typedef struct bk_out_partition {
 
 typedef struct bk_out_groupby {
   bk_out_header h;
-  uint32_t G;               /* in: number of keys (dense 0..G-1), <= 65536 */
+  uint32_t G;               /* in: number of keys (dense 0..G-1), 1..8192 (else BK_E_INVAL) */
   uint32_t _pad;
   uint64_t* count;          /* out: G */
   uint64_t* qty;            /* out: G */
@@ -337,6 +359,23 @@ typedef int (*bk_chunk_fn)(const bk_chunk_view* view, void* stream, void* user);
  * returned non-zero), BK_E_STATE (nothing registered), BK_E_RANGE (a record's accessed bytes exceed
  * a chunk), BK_E_CUDA. Not available with BK_FLAG_BASELINE_* (BK_E_UNSUPPORTED). */
 BK_API int bk_run_user(bk_ctx* ctx, const bk_access* access, bk_chunk_fn fn, void* user, void* stream);
+
+/* ---- multi-GPU merge of count tables (SURVEY §8(e), C1 word count / f4 k-mers) ----------------
+ * Per-GPU tables are all-gathered (NCCL over NVLink, by the caller) into one device buffer; this
+ * merges them by key on the context's GPU. All pointers are DEVICE pointers on that GPU except
+ * seg_rows (host).
+ *   rows       n_seg segments of seg_stride rows each (segment r = rank r's table, padded to the
+ *              longest); segment r holds seg_rows[r] <= seg_stride valid rows. A row is row_u64
+ *              u64 words: words [0, key_u64) are its key, word count_col (>= key_u64) its count.
+ *   out        cap rows of row_u64 words: one per distinct key, the count the sum over all rows of
+ *              that key, every other word copied from its first row in (segment, row) order —
+ *              e.g. the lowest rank's occurrence offset. Rows are in unspecified order.
+ *   *n_out     (host) distinct keys; > cap: BK_E_CAPACITY, out holds cap of them.
+ * Ordered after `stream`; returns when out and *n_out are valid. BK_E_INVAL: NULL pointers,
+ * key_u64 == 0, count_col < key_u64 or >= row_u64, row_u64 > 16, seg_rows[r] > seg_stride. */
+BK_API int bk_merge_counts(bk_ctx* ctx, const uint64_t* rows, uint32_t n_seg, uint64_t seg_stride,
+                           const uint64_t* seg_rows, uint32_t row_u64, uint32_t key_u64, uint32_t count_col,
+                           uint64_t* out, uint64_t cap, uint64_t* n_out, void* stream);
 
 /* ABI self-check for bindings: writes sizeof of bk_config, bk_out_wordcount, bk_out_grep,
  * bk_out_kmeans, bk_out_partition, bk_out_groupby, bk_out_layout, bk_stats, bk_out_pattern,

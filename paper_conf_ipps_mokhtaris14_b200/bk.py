@@ -22,6 +22,7 @@ BK_FLAG_BASELINE_DBUF = 2
 BK_FLAG_BASELINE_SBUF = 4
 BK_FLAG_NO_GRAPH = 8
 BK_FLAG_TEST_DELAYS = 16
+BK_FLAG_KEEP_OUTPUTS_PINNED = 32
 GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE, "hybrid": BK_GATHER_HYBRID}
 
 u32, i32, u64, P = C.c_uint32, C.c_int32, C.c_uint64, C.c_void_p
@@ -40,7 +41,7 @@ class bk_out_header(C.Structure):
 
 class bk_out_wordcount(C.Structure):
     _fields_ = [("h", bk_out_header), ("table_slots", u64), ("cap", u64), ("word_off", P), ("word_len", P),
-                ("word_count", P), ("n_words", u64), ("total_words", u64)]
+                ("word_count", P), ("n_words", u64), ("total_words", u64), ("word_h1", P), ("word_h2", P)]
 
 
 class bk_out_grep(C.Structure):
@@ -117,7 +118,8 @@ BK_K_KMER = 6
 ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,
                bk_out_layout, bk_stats, bk_out_pattern, bk_out_kmer, bk_access, bk_chunk_view]
 EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_strerror",
-           "bk_last_error", "bk_get_stats", "bk_abi_sizes", "bk_partition_materialize"]
+           "bk_last_error", "bk_get_stats", "bk_abi_sizes", "bk_partition_materialize", "bk_unpin_outputs",
+           "bk_merge_counts"]
 
 _lib = None
 
@@ -148,8 +150,10 @@ def lib() -> C.CDLL:
         l.bk_abi_sizes.argtypes = [C.POINTER(u32), C.c_int]
         l.bk_run_user.argtypes = [P, C.POINTER(bk_access), P, P, P]
         l.bk_partition_materialize.argtypes = [P, P, u64, u32, P, P, u32]
+        l.bk_unpin_outputs.argtypes = [P]
+        l.bk_merge_counts.argtypes = [P, P, u32, u64, P, u32, u32, u32, P, u64, C.POINTER(u64), P]
         for name in ("bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_get_stats",
-                     "bk_abi_sizes", "bk_partition_materialize"):
+                     "bk_abi_sizes", "bk_partition_materialize", "bk_unpin_outputs", "bk_merge_counts"):
             getattr(l, name).restype = C.c_int
         _lib = l
     return _lib
@@ -167,11 +171,16 @@ def abi_sizes() -> list[int]:
 
 
 def _ptr(a) -> int | None:
+    """Address of a numpy array, a torch tensor (host or device memory: the aggregating kernels'
+    result arrays may live on the context's GPU, bk.h) or a raw integer address."""
     if a is None:
         return None
     if isinstance(a, np.ndarray):
         assert a.flags["C_CONTIGUOUS"]
         return a.ctypes.data
+    if hasattr(a, "data_ptr"):
+        assert a.is_contiguous()
+        return a.data_ptr()
     return int(a)
 
 
@@ -179,14 +188,15 @@ def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_m
               chunk_bytes: int = 0, lanes: int = 0, record_size: int = 0, host_threads: int = 0,
               profile: bool = False, baseline_dbuf: bool = False, lane_bytes: int = 0,
               zc_share_pm: int = 0, baseline_sbuf: bool = False, no_graph: bool = False,
-              test_delays: bool = False) -> int:
+              test_delays: bool = False, keep_outputs_pinned: bool = False) -> int:
     if isinstance(gather_mode, str):
         gather_mode = GATHER_NAMES[gather_mode]
     cfg = bk_config(C.sizeof(bk_config), device, window_bytes, n_slots, gather_mode, chunk_bytes, lanes,
                     host_threads, record_size,
                     (BK_FLAG_PROFILE if profile else 0) | (BK_FLAG_BASELINE_DBUF if baseline_dbuf else 0) |
                     (BK_FLAG_BASELINE_SBUF if baseline_sbuf else 0) | (BK_FLAG_NO_GRAPH if no_graph else 0) |
-                    (BK_FLAG_TEST_DELAYS if test_delays else 0),
+                    (BK_FLAG_TEST_DELAYS if test_delays else 0) |
+                    (BK_FLAG_KEEP_OUTPUTS_PINNED if keep_outputs_pinned else 0),
                     lane_bytes,
                     zc_share_pm, 0)
     ctx = P()
@@ -275,21 +285,29 @@ class Context:
     def stats(self) -> dict:
         return bk_get_stats(self.ctx)
 
+    def unpin_outputs(self):
+        """bk_unpin_outputs: release output arrays kept pinned (keep_outputs_pinned=True)."""
+        check(lib().bk_unpin_outputs(self.ctx), "bk_unpin_outputs")
+
     def wordcount(self, cap: int = 1 << 20, table_slots: int = 0, stream=None, out=None):
         """(word_off u64, word_len u32, word_count u64) of every distinct word; `out`: optional
-        preallocated (off, len, count) arrays of equal length (the cap), reused across calls."""
+        preallocated (off, len, count) or (off, len, count, h1, h2) arrays of equal length (the cap),
+        numpy or torch (host or device), reused across calls; with h1/h2 the word identities (the
+        multi-GPU merge key) are returned too."""
         o = _hdr(bk_out_wordcount, BK_K_WORDCOUNT)
         if out is not None:
-            off, ln, cnt = out
-            assert off.dtype == np.uint64 and ln.dtype == np.uint32 and cnt.dtype == np.uint64
-            assert len(off) == len(ln) == len(cnt)
-            cap = len(off)
+            assert len(out) in (3, 5) and len({len(a) for a in out}) == 1
+            cap = len(out[0])
         else:
-            off = np.empty(cap, np.uint64); ln = np.empty(cap, np.uint32); cnt = np.empty(cap, np.uint64)
-        o.table_slots, o.cap, o.word_off, o.word_len, o.word_count = table_slots, cap, _ptr(off), _ptr(ln), _ptr(cnt)
+            out = (np.empty(cap, np.uint64), np.empty(cap, np.uint32), np.empty(cap, np.uint64))
+        o.table_slots, o.cap = table_slots, cap
+        o.word_off, o.word_len, o.word_count = _ptr(out[0]), _ptr(out[1]), _ptr(out[2])
+        if len(out) == 5:
+            o.word_h1, o.word_h2 = _ptr(out[3]), _ptr(out[4])
         bk_run(self.ctx, BK_K_WORDCOUNT, stream, o)
+        self.total_words = int(o.total_words)
         n = o.n_words
-        return off[:n], ln[:n], cnt[:n]
+        return tuple(a[:n] for a in out)
 
     def grep(self, pattern: bytes = b"bigk", first_index: int = 0, cap: int | None = None, stream=None, out=None):
         o = _hdr(bk_out_grep, BK_K_GREP)
@@ -299,25 +317,44 @@ class Context:
         bk_run(self.ctx, BK_K_GREP, stream, o)
         return idx[: o.n_match]
 
-    def groupby(self, G: int = 4096, stream=None):
+    def groupby(self, G: int = 4096, stream=None, out=None):
+        """(count u64[G], qty u64[G], amount f64[G]); `out`: optional (count, qty, amount) arrays,
+        numpy or torch (host or device memory of this context's GPU)."""
         o = _hdr(bk_out_groupby, BK_K_GROUPBY)
-        cnt = np.empty(G, np.uint64); qty = np.empty(G, np.uint64); amt = np.empty(G, np.float64)
-        o.G, o.count, o.qty, o.amount = G, _ptr(cnt), _ptr(qty), _ptr(amt)
+        if out is None:
+            out = (np.empty(G, np.uint64), np.empty(G, np.uint64), np.empty(G, np.float64))
+        assert all(len(a) >= G for a in out)
+        o.G, o.count, o.qty, o.amount = G, _ptr(out[0]), _ptr(out[1]), _ptr(out[2])
         bk_run(self.ctx, BK_K_GROUPBY, stream, o)
-        return cnt, qty, amt
+        return out
 
-    def kmeans(self, mu: np.ndarray, first_index: int = 0, stream=None, cid=None):
-        """(count u64[K], sum f64[K,16], chk); cid: optional int32[n] written back per record."""
+    def kmeans(self, mu: np.ndarray, first_index: int = 0, stream=None, cid=None, out=None):
+        """(count u64[K], sum f64[K,16], chk); cid: optional int32[n] (host) written back per record;
+        out: optional (count[K], sum[K*16 or K,16]) arrays, numpy or torch (host or device)."""
         mu = np.ascontiguousarray(mu, np.float32).reshape(-1, 16)
         K = mu.shape[0]
         o = _hdr(bk_out_kmeans, BK_K_KMEANS)
-        cnt = np.empty(K, np.uint64); s = np.empty((K, 16), np.float64)
+        if out is None:
+            out = (np.empty(K, np.uint64), np.empty((K, 16), np.float64))
+        cnt, s = out
         if cid is not None:
             assert cid.dtype == np.int32 and len(cid) >= self.n
         o.centroids, o.K, o.first_index, o.count, o.sum = _ptr(mu), K, first_index, _ptr(cnt), _ptr(s)
         o.cid = _ptr(cid) if cid is not None and self.n else None
         bk_run(self.ctx, BK_K_KMEANS, stream, o)
         return cnt, s, int(o.chk)
+
+    def merge_counts(self, rows, seg_rows, seg_stride: int, row_u64: int, key_u64: int, count_col: int, out,
+                     stream=None) -> int:
+        """bk_merge_counts over DEVICE arrays (torch tensors on this context's GPU): `rows` holds
+        len(seg_rows) segments of seg_stride rows; merged rows go to `out` (cap = its rows).
+        Returns the number of distinct keys."""
+        segs = np.ascontiguousarray(seg_rows, np.uint64)
+        cap = out.numel() // row_u64 if hasattr(out, "numel") else len(out) // row_u64
+        n = u64(0)
+        check(lib().bk_merge_counts(self.ctx, _ptr(rows), len(segs), seg_stride, _ptr(segs), row_u64, key_u64,
+                                    count_col, _ptr(out), cap, C.byref(n), stream), "bk_merge_counts")
+        return int(n.value)
 
     def partition(self, n_buckets: int = 1024, out=None, chunk_cap: int = 1 << 16, stream=None):
         """Returns (out u64[n,2] chunk-major bucket-sorted runs, chunk_counts u64[C,B], bucket_count u64[B])."""

@@ -50,6 +50,20 @@ enum : int {
   kErrOutOverflow = 16,
 };
 
+// SM count of the current device (queried once per device, then cached): grids are sized in
+// multiples of it instead of a hard-coded 148.
+inline int device_sms() {
+  static int cache[64] = {};
+  int d = 0;
+  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return 148;
+  if (!cache[d]) {
+    int n = 0;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, d) != cudaSuccess || n <= 0) n = 148;
+    cache[d] = n;
+  }
+  return cache[d];
+}
+
 __host__ __device__ inline uint64_t mix64(uint64_t x) {
   x ^= x >> 30; x *= 0xbf58476d1ce4e5b9ULL;
   x ^= x >> 27; x *= 0x94d049bb133111ebULL;
@@ -87,8 +101,10 @@ void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, cons
 void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
                     uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                     int* err, cudaStream_t s);
-void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,
-                       uint32_t* len, uint64_t* cnt, uint64_t cap, cudaStream_t s);
+// distinct words -> (occurrence offset, length, count, key1, key2) rows; *total += every count
+void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, unsigned long long* total,
+                       uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1, uint64_t* h2, uint64_t cap,
+                       cudaStream_t s);
 
 struct GrepParams {
   uint8_t pat[32];
@@ -154,6 +170,13 @@ void launch_kmer(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, co
                  unsigned long long* total, int* err, cudaStream_t s);
 void launch_kmer_compact(const KmerEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* kmer,
                          uint64_t* cnt, uint64_t cap, cudaStream_t s);
+
+// ---- multi-GPU merge of count tables (kernels_merge.cu): rows of row_u64 words, key = words
+// [0, key_u64), count at count_col; owner/cnt: `slots` (power of two) scratch entries each
+cudaError_t launch_merge_counts(const uint64_t* rows, uint32_t n_seg, uint64_t seg_stride, const uint64_t* seg_rows,
+                                uint32_t row_u64, uint32_t key_u64, uint32_t count_col, unsigned long long* owner,
+                                unsigned long long* cnt, uint64_t slots, uint64_t* out, uint64_t cap,
+                                unsigned long long* n_out, int* err, cudaStream_t s);
 
 // ---- online pattern recognition of stage 1 (kernels_pattern.cu, NEXT f2) ----
 void launch_addr_patterns(const Chunk& c, const Access& a, const uint64_t* meta, const LaneDesc* lanes, uint32_t elem,

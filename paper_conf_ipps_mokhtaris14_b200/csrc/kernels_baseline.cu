@@ -176,7 +176,7 @@ __global__ void __launch_bounds__(256) k_dbuf_kmeans(RawChunk c, const float* __
 
 }  // namespace
 
-uint32_t dbuf_blocks() { return 148 * 4; }
+uint32_t dbuf_blocks() { return (uint32_t)device_sms() * 4; }
 
 void launch_dbuf_kmeans(const uint8_t* raw, uint64_t lo, uint64_t hi, uint64_t base_byte, uint64_t rec_size,
                         const float* mu, uint32_t K, uint64_t first_index, unsigned long long* count, double* sum,

@@ -299,17 +299,25 @@ __global__ void __launch_bounds__(256) k_dbuf_wc(const uint8_t* __restrict__ raw
 }
 
 __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, unsigned long long* n_out,
-                             uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t cap) {
+                             unsigned long long* total, uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1,
+                             uint64_t* h2, uint64_t cap) {
+  unsigned long long mine = 0;
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < slots; i += (uint64_t)gridDim.x * blockDim.x) {
     const WcEntry e = table[i];
     if (e.key1 == 0) continue;
+    mine += e.count;
     const unsigned long long p = atomicAdd(n_out, 1ull);
     if (p < cap) {
       off[p] = e.offlen >> 24;
       len[p] = (uint32_t)(e.offlen & 0xffffff);
       cnt[p] = e.count;
+      h1[p] = e.key1;
+      h2[p] = e.key2;
     }
   }
+  // total words: one atomic per warp
+  for (int o = 16; o; o >>= 1) mine += __shfl_down_sync(kFull, mine, o);
+  if ((threadIdx.x & 31) == 0 && mine) atomicAdd(total, mine);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -689,12 +697,13 @@ void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, cons
 void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
                     uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                     int* err, cudaStream_t s) {
-  k_dbuf_wc<<<148 * 4, 256, 0, s>>>(raw, meta, lo, hi, base_byte, end_byte, rec_size, table, mask, used, err);
+  k_dbuf_wc<<<device_sms() * 4, 256, 0, s>>>(raw, meta, lo, hi, base_byte, end_byte, rec_size, table, mask, used, err);
 }
 
-void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* off,
-                       uint32_t* len, uint64_t* cnt, uint64_t cap, cudaStream_t s) {
-  k_wc_compact<<<148 * 4, 256, 0, s>>>(table, slots, n_out, off, len, cnt, cap);
+void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, unsigned long long* total,
+                       uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1, uint64_t* h2, uint64_t cap,
+                       cudaStream_t s) {
+  k_wc_compact<<<device_sms() * 4, 256, 0, s>>>(table, slots, n_out, total, off, len, cnt, h1, h2, cap);
 }
 
 size_t grep_count_smem() { return stream_smem<true>(kGrepThreads / 32, kGrepRows); }

@@ -98,7 +98,7 @@ void launch_kmer(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, co
 
 void launch_kmer_compact(const KmerEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* kmer,
                          uint64_t* cnt, uint64_t cap, cudaStream_t s) {
-  k_kmer_compact<<<148 * 4, 256, 0, s>>>(table, slots, n_out, kmer, cnt, cap);
+  k_kmer_compact<<<device_sms() * 4, 256, 0, s>>>(table, slots, n_out, kmer, cnt, cap);
 }
 
 }  // namespace bk

@@ -218,7 +218,7 @@ size_t partition_smem(uint32_t B) { return (size_t)9 * B * 4; }
 
 uint32_t partition_blocks(const Chunk& c) {
   uint32_t nblk = (c.ntiles + 7) / 8;
-  if (nblk > 148 * 2) nblk = 148 * 2;
+  if (nblk > (uint32_t)device_sms() * 2) nblk = (uint32_t)device_sms() * 2;
   return nblk ? nblk : 1;
 }
 

@@ -438,7 +438,7 @@ static void gather_impl(const Chunk& c, const Access& a, const uint8_t* src, con
   // Zero-copy reads are bound by outstanding PCIe read requests (~1k tags), not by warps: one
   // block per SM keeps >1k 16-B requests in flight and leaves the other SMs' slots to the compute
   // kernels of earlier chunks running concurrently. HBM re-layout uses the whole chip.
-  const uint32_t grid_cap = kHost ? 148 : 148 * 8;
+  const uint32_t grid_cap = kHost ? (uint32_t)device_sms() : (uint32_t)device_sms() * 8;
   if (grid > grid_cap) grid = grid_cap;
   if (grid == 0) return;
   if (a.whole) {

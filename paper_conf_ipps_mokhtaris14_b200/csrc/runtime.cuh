@@ -139,6 +139,7 @@ struct bk_ctx {  // the opaque context of include/bk.h
   const uint64_t* off = nullptr;
   uint64_t n = 0;
   bool pinned_data = false, pinned_off = false, registered = false;
+  bool registered_ro = false;          // the data set was registered cudaHostRegisterReadOnly
   const uint8_t* host_dev = nullptr;   // device alias of the mapped data set
   const uint64_t* off_dev = nullptr;   // device alias of the mapped offsets (nullptr: not mapped)
   uint64_t max_rec = 0, min_rec = 0;
@@ -160,7 +161,10 @@ struct bk_ctx {  // the opaque context of include/bk.h
   cudaStream_t s_d2h = nullptr;
   std::vector<cudaEvent_t> ev_part;
   bk::rt::DevBuf b_hist, b_colpre, b_totals, b_base;
-  std::vector<std::pair<void*, uint64_t>> out_pinned;  // caller output arrays this context pinned
+  bk::rt::DevBuf b_h1, b_h2;                 // word-count key hashes (multi-GPU merge keys)
+  bk::rt::DevBuf b_mown, b_mcnt, b_mctr;     // bk_merge_counts scratch (never captured in a graph)
+  std::vector<std::pair<void*, uint64_t>> out_pinned;      // caller output arrays pinned across runs (opt-in)
+  std::vector<std::pair<void*, uint64_t>> out_pinned_run;  // caller output arrays pinned for this run only
   int n_launch = 0;
   bk_stats st{};
   std::vector<std::pair<std::string, bk::rt::Plan>> plan_cache;
@@ -214,6 +218,8 @@ bool graphable(const Plan& p);
 // those keep the SMs' sysmem path busy and the bulk copies were measured to stall behind them.
 inline bool stage_tma(const Plan& p) { return p.mode == BK_GATHER_DENSE || p.mode == BK_GATHER_CPU; }
 int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes);
+void release_run_outputs(bk_ctx* c);
+void release_kept_outputs(bk_ctx* c);
 void unregister(bk_ctx* c);
 
 // NVTX ranges (SURVEY §5 tracing): bk_run / registration, and per chunk its stage issue ("chunk i
@@ -286,9 +292,17 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
 }
 
 
+// Every device address a captured graph may bake in besides those the per-kernel key already names
+// (the window's carving is a function of the plan, which is in the key): the resident DevBufs can be
+// reallocated by a later run with larger parameters, so their current addresses are part of the key
+// and a graph whose buffers moved is never replayed (it would touch freed memory).
+std::string resident_key(const bk_ctx* c);
+constexpr size_t kMaxGraphs = 16;   // cached graphs per context (oldest dropped first)
+
 template <class Enqueue>
-int run_device(bk_ctx* c, void* stream, const std::string& key, bool graphable, size_t n_chunks, Enqueue&& enqueue) {
+int run_device(bk_ctx* c, void* stream, const std::string& key_in, bool graphable, size_t n_chunks, Enqueue&& enqueue) {
   BK_CUDA(cudaSetDevice(c->cfg.device));
+  const std::string key = key_in + "|" + resident_key(c);
   host_reset(c);
   BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
   BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_begin, 0));
@@ -332,6 +346,10 @@ int run_device(bk_ctx* c, void* stream, const std::string& key, bool graphable, 
     g.n_launch = c->n_launch;
     g.prof_used = c->prof_used;
     g.prof_stage.assign(c->prof_stage.begin(), c->prof_stage.begin() + std::min(c->prof_stage.size(), c->prof_used / 2));
+    if (c->graphs.size() >= kMaxGraphs) {
+      if (c->graphs.front().exec) cudaGraphExecDestroy(c->graphs.front().exec);
+      c->graphs.erase(c->graphs.begin());
+    }
     c->graphs.push_back(std::move(g));
     ge = &c->graphs.back();
   }

@@ -37,6 +37,39 @@ static void drain(bk_ctx* c) {
   cudaGetLastError();
 }
 
+// Selects the context's device for the duration of an API call and restores the caller's current
+// device on return (a process may drive contexts on several GPUs from one thread).
+struct DeviceGuard {
+  int prev = -1;
+  bool ok = false;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    ok = cudaSetDevice(dev) == cudaSuccess;
+    cudaGetLastError();
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+    cudaGetLastError();
+  }
+  DeviceGuard(const DeviceGuard&) = delete;
+  DeviceGuard& operator=(const DeviceGuard&) = delete;
+};
+
+// struct_size of the in/out struct bk_run expects for each kernel id (0: unknown id)
+static uint32_t out_size(int kernel_id) {
+  switch (kernel_id) {
+    case BK_K_WORDCOUNT: return sizeof(bk_out_wordcount);
+    case BK_K_GREP: return sizeof(bk_out_grep);
+    case BK_K_KMEANS: return sizeof(bk_out_kmeans);
+    case BK_K_PARTITION: return sizeof(bk_out_partition);
+    case BK_K_GROUPBY: return sizeof(bk_out_groupby);
+    case BK_K_KMER: return sizeof(bk_out_kmer);
+    case BK_K_LAYOUT_DUMP: return sizeof(bk_out_layout);
+    case BK_K_PATTERN_STATS: return sizeof(bk_out_pattern);
+    default: return 0;
+  }
+}
+
 extern "C" {
 
 const char* bk_strerror(int status) {
@@ -74,7 +107,8 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
   }
   c->cfg.window_bytes = c->cfg.window_bytes / (c->cfg.n_slots * kAlign) * (c->cfg.n_slots * kAlign);
   auto cleanup = [&](int rc) { bk_destroy(c); return rc; };
-  if (cudaSetDevice(c->cfg.device) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaSetDevice"));
+  DeviceGuard dg(c->cfg.device);
+  if (!dg.ok) return cleanup(fail(BK_E_CUDA, "cudaSetDevice"));
   if (configure_compute_kernels() != cudaSuccess) return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
   if (cudaStreamCreateWithFlags(&c->s_copy, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->s_asm, cudaStreamNonBlocking) != cudaSuccess ||
@@ -127,7 +161,8 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
   if (!c) return fail(BK_E_INVAL, "NULL ctx");
   if (!host_ptr && nbytes) return fail(BK_E_INVAL, "NULL host_ptr");
   const auto t0 = std::chrono::steady_clock::now();
-  if (cudaSetDevice(c->cfg.device) != cudaSuccess) return fail(BK_E_CUDA, "cudaSetDevice");
+  DeviceGuard dg(c->cfg.device);
+  if (!dg.ok) return fail(BK_E_CUDA, "cudaSetDevice");
   unregister(c);
   uint64_t maxr = 0, minr = ~0ull;
   if (off) {
@@ -155,7 +190,16 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
     if (is_pinned(host_ptr)) {
       c->pinned_data = false;
     } else {
-      cudaError_t e = cudaHostRegister((void*)host_ptr, nbytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+      // read-only where supported: libbk never writes the registered data set
+      int ro = 0;
+      cudaDeviceGetAttribute(&ro, cudaDevAttrHostRegisterReadOnlySupported, c->cfg.device);
+      const unsigned fl = cudaHostRegisterMapped | cudaHostRegisterPortable | (ro ? cudaHostRegisterReadOnly : 0u);
+      cudaError_t e = cudaHostRegister((void*)host_ptr, nbytes, fl);
+      if (e != cudaSuccess && ro) {   // some platforms advertise but refuse it: plain mapped registration
+        cudaGetLastError();
+        e = cudaHostRegister((void*)host_ptr, nbytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+      }
+      c->registered_ro = e == cudaSuccess && ro;
       if (e != cudaSuccess) return fail(BK_E_CUDA, "cudaHostRegister(data, %llu): %s", (unsigned long long)nbytes, cudaGetErrorString(e));
       c->pinned_data = true;
     }
@@ -200,6 +244,11 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
   if (!c->registered) return fail(BK_E_STATE, "bk_run before bk_register_segments");
   const bk_out_header* h = (const bk_out_header*)out;
   if (h->kernel_id != kernel_id) return fail(BK_E_INVAL, "out->kernel_id %d != %d", h->kernel_id, kernel_id);
+  const uint32_t want = out_size(kernel_id);
+  if (!want) return fail(BK_E_UNSUPPORTED, "unknown kernel_id %d", kernel_id);
+  if (h->struct_size != want) return fail(BK_E_INVAL, "out struct_size %u != %u for kernel %d", h->struct_size, want, kernel_id);
+  DeviceGuard dg(c->cfg.device);   // every allocation and launch of this run lands on the context's GPU
+  if (!dg.ok) return fail(BK_E_CUDA, "cudaSetDevice(%d)", c->cfg.device);
   static const char* const kNames[] = {"?", "wordcount", "grep", "kmeans", "partition", "groupby", "kmer"};
   NvtxRange nv("bk_run.%s", kernel_id >= 1 && kernel_id <= 6 ? kNames[kernel_id]
                              : kernel_id == BK_K_LAYOUT_DUMP ? "layout" : "pattern");
@@ -207,55 +256,44 @@ int bk_run(bk_ctx* c, int kernel_id, void* stream, void* out) {
   int rc;
   if (c->cfg.flags & (BK_FLAG_BASELINE_DBUF | BK_FLAG_BASELINE_SBUF)) {
     rc = run_dbuf(c, kernel_id, out, stream);
-    if (rc) {
-      cudaDeviceSynchronize();
-      cudaGetLastError();
-      return rc;
-    }
+    if (rc) drain(c);
+    release_run_outputs(c);
+    if (rc) return rc;
     c->st.kernel_launches = (uint64_t)c->n_launch;
     c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     return BK_OK;
   }
   switch (kernel_id) {
     case BK_K_WORDCOUNT:
-      if (h->struct_size != sizeof(bk_out_wordcount)) return fail(BK_E_INVAL, "bk_out_wordcount size");
       rc = run_wordcount(c, (bk_out_wordcount*)out, stream);
       break;
     case BK_K_GREP:
-      if (h->struct_size != sizeof(bk_out_grep)) return fail(BK_E_INVAL, "bk_out_grep size");
       rc = run_grep(c, (bk_out_grep*)out, stream);
       break;
     case BK_K_KMEANS:
-      if (h->struct_size != sizeof(bk_out_kmeans)) return fail(BK_E_INVAL, "bk_out_kmeans size");
       rc = run_kmeans(c, (bk_out_kmeans*)out, stream);
       break;
     case BK_K_GROUPBY:
-      if (h->struct_size != sizeof(bk_out_groupby)) return fail(BK_E_INVAL, "bk_out_groupby size");
       rc = run_groupby(c, (bk_out_groupby*)out, stream);
       break;
     case BK_K_KMER:
-      if (h->struct_size != sizeof(bk_out_kmer)) return fail(BK_E_INVAL, "bk_out_kmer size");
       rc = run_kmer(c, (bk_out_kmer*)out, stream);
       break;
     case BK_K_PATTERN_STATS:
-      if (h->struct_size != sizeof(bk_out_pattern)) return fail(BK_E_INVAL, "bk_out_pattern size");
       rc = run_pattern(c, (bk_out_pattern*)out, stream);
       break;
     case BK_K_LAYOUT_DUMP:
-      if (h->struct_size != sizeof(bk_out_layout)) return fail(BK_E_INVAL, "bk_out_layout size");
       rc = run_layout(c, (bk_out_layout*)out, stream);
       break;
     case BK_K_PARTITION:
-      if (h->struct_size != sizeof(bk_out_partition)) return fail(BK_E_INVAL, "bk_out_partition size");
       rc = run_partition(c, (bk_out_partition*)out, stream);
       break;
     default:
       return fail(BK_E_UNSUPPORTED, "unknown kernel_id %d", kernel_id);
   }
-  if (rc) {
-    drain(c);   // leave the context usable
-    return rc;
-  }
+  if (rc) drain(c);   // leave the context usable
+  release_run_outputs(c);
+  if (rc) return rc;
   c->st.kernel_launches = (uint64_t)c->n_launch;
   c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return BK_OK;
@@ -268,6 +306,8 @@ int bk_run_user(bk_ctx* c, const bk_access* a, bk_chunk_fn fn, void* user, void*
   if (!c->registered) return fail(BK_E_STATE, "bk_run_user before bk_register_segments");
   if (c->cfg.flags & (BK_FLAG_BASELINE_DBUF | BK_FLAG_BASELINE_SBUF))
     return fail(BK_E_UNSUPPORTED, "bk_run_user: no double-buffering baseline for user kernels");
+  DeviceGuard dg(c->cfg.device);
+  if (!dg.ok) return fail(BK_E_CUDA, "cudaSetDevice(%d)", c->cfg.device);
   const auto t0 = std::chrono::steady_clock::now();
   const int rc = run_user(c, a, fn, user, stream);
   if (rc) {
@@ -276,6 +316,54 @@ int bk_run_user(bk_ctx* c, const bk_access* a, bk_chunk_fn fn, void* user, void*
   }
   c->st.kernel_launches = (uint64_t)c->n_launch;
   c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return BK_OK;
+}
+
+int bk_merge_counts(bk_ctx* c, const uint64_t* rows, uint32_t n_seg, uint64_t seg_stride, const uint64_t* seg_rows,
+                    uint32_t row_u64, uint32_t key_u64, uint32_t count_col, uint64_t* out, uint64_t cap,
+                    uint64_t* n_out, void* stream) {
+  NvtxRange nv("bk_merge_counts");
+  if (!c || !n_out || (n_seg && !seg_rows)) return fail(BK_E_INVAL, "NULL argument");
+  if (key_u64 == 0 || count_col < key_u64 || count_col >= row_u64 || row_u64 > 16)
+    return fail(BK_E_INVAL, "need 1 <= key_u64 <= count_col < row_u64 <= 16");
+  if (n_seg > 64) return fail(BK_E_INVAL, "at most 64 segments");
+  uint64_t total = 0;
+  for (uint32_t i = 0; i < n_seg; ++i) {
+    if (seg_rows[i] > seg_stride) return fail(BK_E_INVAL, "seg_rows[%u] > seg_stride", i);
+    total += seg_rows[i];
+  }
+  if (total && !rows) return fail(BK_E_INVAL, "NULL rows");
+  if (cap && !out) return fail(BK_E_INVAL, "NULL out");
+  DeviceGuard dg(c->cfg.device);
+  if (!dg.ok) return fail(BK_E_CUDA, "cudaSetDevice(%d)", c->cfg.device);
+  uint64_t slots = 1024;
+  while (slots < 2 * total) slots <<= 1;
+  BK_CUDA(c->b_mown.ensure(slots * 8));
+  BK_CUDA(c->b_mcnt.ensure(slots * 8));
+  BK_CUDA(c->b_mctr.ensure(16));
+  cudaStream_t st = c->s_comp;
+  BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
+  BK_CUDA(cudaStreamWaitEvent(st, c->ev_begin, 0));
+  BK_CUDA(cudaMemsetAsync(c->d_err, 0, sizeof(int), st));
+  BK_CUDA(launch_merge_counts(rows, n_seg, seg_stride, seg_rows, row_u64, key_u64, count_col,
+                              (unsigned long long*)c->b_mown.p, (unsigned long long*)c->b_mcnt.p, slots, out, cap,
+                              (unsigned long long*)c->b_mctr.p, c->d_err, st));
+  BK_CUDA(cudaMemcpyAsync(c->h_ctr, c->b_mctr.p, 8, cudaMemcpyDeviceToHost, st));
+  BK_CUDA(cudaMemcpyAsync(c->h_ctr + 8, c->d_err, sizeof(int), cudaMemcpyDeviceToHost, st));
+  BK_CUDA(cudaEventRecord(c->ev_end, st));
+  BK_CUDA(cudaStreamWaitEvent((cudaStream_t)stream, c->ev_end, 0));
+  BK_CUDA(cudaStreamSynchronize(st));
+  if ((int)(uint32_t)c->h_ctr[8] & kErrTableFull) return fail(BK_E_CUDA, "merge table full (internal bound violated)");
+  *n_out = c->h_ctr[0];
+  if (*n_out > cap) return fail(BK_E_CAPACITY, "%llu distinct keys > cap %llu", (unsigned long long)*n_out,
+                                (unsigned long long)cap);
+  return BK_OK;
+}
+
+int bk_unpin_outputs(bk_ctx* c) {
+  if (!c) return fail(BK_E_INVAL, "NULL ctx");
+  DeviceGuard dg(c->cfg.device);
+  release_kept_outputs(c);
   return BK_OK;
 }
 
@@ -311,7 +399,7 @@ int bk_abi_sizes(uint32_t* sizes, int n) {
 
 int bk_destroy(bk_ctx* c) {
   if (!c) return BK_OK;
-  cudaSetDevice(c->cfg.device);
+  DeviceGuard dg(c->cfg.device);
   if (c->s_comp) cudaStreamSynchronize(c->s_comp);
   if (c->s_copy) cudaStreamSynchronize(c->s_copy);
   if (c->s_asm) cudaStreamSynchronize(c->s_asm);
@@ -347,8 +435,11 @@ int bk_destroy(bk_ctx* c) {
     cudaStreamDestroy(c->s_d2h);
   }
   for (auto e : c->ev_part) cudaEventDestroy(e);
-  for (auto& e : c->out_pinned) cudaHostUnregister(e.first);
-  for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base}) b->release();
+  release_run_outputs(c);
+  release_kept_outputs(c);
+  for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base, &c->b_h1, &c->b_h2, &c->b_mown, &c->b_mcnt,
+                    &c->b_mctr})
+    b->release();
   for (auto* h : c->hstage) cudaFreeHost(h);
   for (auto e : c->h_done) cudaEventDestroy(e);
   if (c->s_copy) cudaStreamDestroy(c->s_copy);

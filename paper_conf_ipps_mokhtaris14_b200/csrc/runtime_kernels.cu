@@ -21,6 +21,8 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
   BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(ocap, 1) * 4));
   BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  BK_CUDA(c->b_h1.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  BK_CUDA(c->b_h2.ensure(std::max<uint64_t>(ocap, 1) * 8));
   WcEntry* table = (WcEntry*)c->b_table.p;
   const std::string key = "wc/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
@@ -32,8 +34,8 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
       return BK_OK;
     });
     if (r) return r;
-    launch_wc_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
-                      (uint64_t*)c->b_out3.p, ocap, c->s_comp);
+    launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
+                      (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p, ocap, c->s_comp);
     c->n_launch += 1;
     return (int)BK_OK;
   });
@@ -44,14 +46,14 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
   if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
                                   (unsigned long long)slots);
-  if (nw) {
-    BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDeviceToHost));
-    BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDeviceToHost));
-    BK_CUDA(cudaMemcpy(o->word_count, c->b_out3.p, nw * 8, cudaMemcpyDeviceToHost));
+  if (nw) {   // host or device result arrays (unified addressing)
+    BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(o->word_count, c->b_out3.p, nw * 8, cudaMemcpyDefault));
+    if (o->word_h1) BK_CUDA(cudaMemcpy(o->word_h1, c->b_h1.p, nw * 8, cudaMemcpyDefault));
+    if (o->word_h2) BK_CUDA(cudaMemcpy(o->word_h2, c->b_h2.p, nw * 8, cudaMemcpyDefault));
   }
-  uint64_t tot = 0;
-  for (uint64_t i = 0; i < nw; ++i) tot += o->word_count[i];
-  o->total_words = tot;
+  o->total_words = c->h_ctr[6];
   c->st.bytes_d2h = nw * 20;
   return BK_OK;
 }
@@ -74,8 +76,7 @@ int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {
   BK_CUDA(c->b_blk.ensure((uint64_t)ntl * 4 * N));              // per slot: tile match counts
   BK_CUDA(c->b_blk2.ensure((uint64_t)ntl * 8 * N));             // per slot: tile output bases
   BK_CUDA(c->b_blk3.ensure((uint64_t)ntl * 32 * 4 * N));        // per slot: lane match masks
-  int dev_sms = 148;
-  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  const int dev_sms = device_sms();
   const int grid = dev_sms * 2;   // 2 x 8-warp blocks per SM stream the tiles (64 KB smem each)
   GrepParams gp{};
   if (o->pattern_len) memcpy(gp.pat, o->pattern, o->pattern_len);
@@ -124,8 +125,8 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
   BK_CUDA(c->b_agg1.ensure((uint64_t)G * 8));
   BK_CUDA(c->b_agg2.ensure((uint64_t)G * 8));
   BK_CUDA(c->b_agg3.ensure((uint64_t)G * 8));
-  int dev_sms = 148, per_sm = 1;
-  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  const int dev_sms = device_sms();
+  int per_sm = 1;
   const bool tma = stage_tma(p);
   per_sm = std::max<int>(1, (int)((220 * 1024) / std::max<size_t>(groupby_smem(G, tma), 1)));
   per_sm = std::min(per_sm, 3);
@@ -143,9 +144,9 @@ int run_groupby(bk_ctx* c, bk_out_groupby* o, void* stream) {
     });
   });
   if (rc) return rc;
-  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
-  BK_CUDA(cudaMemcpy(o->qty, c->b_agg2.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
-  BK_CUDA(cudaMemcpy(o->amount, c->b_agg3.p, (uint64_t)G * 8, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)G * 8, cudaMemcpyDefault));
+  BK_CUDA(cudaMemcpy(o->qty, c->b_agg2.p, (uint64_t)G * 8, cudaMemcpyDefault));
+  BK_CUDA(cudaMemcpy(o->amount, c->b_agg3.p, (uint64_t)G * 8, cudaMemcpyDefault));
   c->st.bytes_d2h = (uint64_t)G * 24;
   return BK_OK;
 }
@@ -166,8 +167,7 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   BK_CUDA(c->b_mu.ensure((uint64_t)K * 64));
   BK_CUDA(c->b_agg1.ensure((uint64_t)K * 8));
   BK_CUDA(c->b_agg3.ensure((uint64_t)K * 16 * 8));
-  int dev_sms = 148;
-  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->cfg.device);
+  const int dev_sms = device_sms();
   if (!c->h_mu) BK_CUDA(cudaHostAlloc((void**)&c->h_mu, 256 * 64, cudaHostAllocPortable));
   memcpy(c->h_mu, o->centroids, (size_t)K * 64);   // the graph copies from this pinned buffer
   const bool tma = stage_tma(p);   // TMA: one 16-warp block per SM; plain loads: two
@@ -198,8 +198,8 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
     });
   });
   if (rc) return rc;
-  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDeviceToHost));
-  BK_CUDA(cudaMemcpy(o->sum, c->b_agg3.p, (uint64_t)K * 128, cudaMemcpyDeviceToHost));
+  BK_CUDA(cudaMemcpy(o->count, c->b_agg1.p, (uint64_t)K * 8, cudaMemcpyDefault));
+  BK_CUDA(cudaMemcpy(o->sum, c->b_agg3.p, (uint64_t)K * 128, cudaMemcpyDefault));
   unsigned long long chk = 0;
   chk = c->h_ctr[4];
   o->chk = chk;
@@ -249,9 +249,9 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
                                        (unsigned long long)slots);
   if (nk) {
     // the result arrays are large (16 B per distinct k-mer): pin them once so the copy runs at DMA speed
-    if ((rc = ensure_out_pinned(c, o->kmer, o->cap * 8)) || (rc = ensure_out_pinned(c, o->count, o->cap * 8))) return rc;
-    BK_CUDA(cudaMemcpy(o->kmer, c->b_out1.p, nk * 8, cudaMemcpyDeviceToHost));
-    BK_CUDA(cudaMemcpy(o->count, c->b_out3.p, nk * 8, cudaMemcpyDeviceToHost));
+    if ((rc = ensure_out_pinned(c, o->kmer, nk * 8)) || (rc = ensure_out_pinned(c, o->count, nk * 8))) return rc;
+    BK_CUDA(cudaMemcpy(o->kmer, c->b_out1.p, nk * 8, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(o->count, c->b_out3.p, nk * 8, cudaMemcpyDefault));
   }
   c->st.bytes_d2h = nk * 16;
   return BK_OK;
@@ -357,6 +357,8 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(wc_ocap, 1) * 8));
     BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(wc_ocap, 1) * 4));
     BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(wc_ocap, 1) * 8));
+    BK_CUDA(c->b_h1.ensure(std::max<uint64_t>(wc_ocap, 1) * 8));
+    BK_CUDA(c->b_h2.ensure(std::max<uint64_t>(wc_ocap, 1) * 8));
   } else if (kid == BK_K_KMEANS) {
     if (ok->K == 0 || ok->K > 256 || !ok->centroids) return fail(BK_E_INVAL, "K must be in 1..256 with centroids");
     if (ok->cid) return fail(BK_E_UNSUPPORTED, "dbuf baseline: no k-means cid write-back");
@@ -446,8 +448,9 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
   }
   if (kid == BK_K_WORDCOUNT) {
-    launch_wc_compact((const WcEntry*)c->b_table.p, wc_slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p,
-                      (uint32_t*)c->b_out2.p, (uint64_t*)c->b_out3.p, wc_ocap, c->s_comp);
+    launch_wc_compact((const WcEntry*)c->b_table.p, wc_slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p,
+                      (uint32_t*)c->b_out2.p, (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p,
+                      wc_ocap, c->s_comp);
     c->n_launch += 1;
   }
   if ((rc = end_run(c, stream))) return rc;
@@ -464,21 +467,21 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     if (nw * 2 > wc_slots)
       return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw, (unsigned long long)wc_slots);
     if (nw) {
-      BK_CUDA(cudaMemcpy(ow->word_off, c->b_out1.p, nw * 8, cudaMemcpyDeviceToHost));
-      BK_CUDA(cudaMemcpy(ow->word_len, c->b_out2.p, nw * 4, cudaMemcpyDeviceToHost));
-      BK_CUDA(cudaMemcpy(ow->word_count, c->b_out3.p, nw * 8, cudaMemcpyDeviceToHost));
+      BK_CUDA(cudaMemcpy(ow->word_off, c->b_out1.p, nw * 8, cudaMemcpyDefault));
+      BK_CUDA(cudaMemcpy(ow->word_len, c->b_out2.p, nw * 4, cudaMemcpyDefault));
+      BK_CUDA(cudaMemcpy(ow->word_count, c->b_out3.p, nw * 8, cudaMemcpyDefault));
+      if (ow->word_h1) BK_CUDA(cudaMemcpy(ow->word_h1, c->b_h1.p, nw * 8, cudaMemcpyDefault));
+      if (ow->word_h2) BK_CUDA(cudaMemcpy(ow->word_h2, c->b_h2.p, nw * 8, cudaMemcpyDefault));
     }
-    uint64_t tot = 0;
-    for (uint64_t i = 0; i < nw; ++i) tot += ow->word_count[i];
-    ow->total_words = tot;
+    ow->total_words = c->h_ctr[6];
   } else if (kid == BK_K_KMEANS) {
-    BK_CUDA(cudaMemcpy(ok->count, c->b_agg1.p, (uint64_t)ok->K * 8, cudaMemcpyDeviceToHost));
-    BK_CUDA(cudaMemcpy(ok->sum, c->b_agg3.p, (uint64_t)ok->K * 128, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(ok->count, c->b_agg1.p, (uint64_t)ok->K * 8, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(ok->sum, c->b_agg3.p, (uint64_t)ok->K * 128, cudaMemcpyDefault));
     ok->chk = c->h_ctr[4];
   } else {
-    BK_CUDA(cudaMemcpy(ob->count, c->b_agg1.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
-    BK_CUDA(cudaMemcpy(ob->qty, c->b_agg2.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
-    BK_CUDA(cudaMemcpy(ob->amount, c->b_agg3.p, (uint64_t)ob->G * 8, cudaMemcpyDeviceToHost));
+    BK_CUDA(cudaMemcpy(ob->count, c->b_agg1.p, (uint64_t)ob->G * 8, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(ob->qty, c->b_agg2.p, (uint64_t)ob->G * 8, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(ob->amount, c->b_agg3.p, (uint64_t)ob->G * 8, cudaMemcpyDefault));
   }
   return BK_OK;
 }

@@ -400,21 +400,56 @@ void drop_graphs(bk_ctx* c) {
 
 bool graphable(const Plan& p) { return p.mode == BK_GATHER_ZC || p.mode == BK_GATHER_DENSE; }
 
+std::string resident_key(const bk_ctx* c) {
+  std::string k;
+  char b[24];
+  for (const DevBuf* d : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_blk3,
+                          &c->b_agg1, &c->b_agg2, &c->b_agg3, &c->b_mu, &c->b_hist, &c->b_colpre, &c->b_totals,
+                          &c->b_base, &c->b_h1, &c->b_h2}) {
+    snprintf(b, sizeof b, "%llx,", (unsigned long long)(uintptr_t)d->p);
+    k += b;
+  }
+  return k;
+}
 
-// The caller's per-record output (partition records, k-means cid) is written by DMA: pin it once
-// and keep it pinned across runs (one cached registration per context).
+
+// The caller's per-record outputs (partition records, k-means cid, k-mer arrays) are written by DMA,
+// so they must be page-locked while the run copies into them. By default they are registered for
+// the run only (release_run_outputs at the end of bk_run); with BK_FLAG_KEEP_OUTPUTS_PINNED the
+// registration is cached across runs (at most four arrays, oldest released first) and dropped by
+// bk_unpin_outputs / bk_destroy — the caller then keeps those arrays alive until one of them.
 int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes) {
   if (!bytes) return BK_OK;
+  const bool keep = (c->cfg.flags & BK_FLAG_KEEP_OUTPUTS_PINNED) != 0;
   for (auto& e : c->out_pinned)
     if (e.first == ptr && e.second == bytes) return BK_OK;
-  if (is_pinned(ptr)) return BK_OK;
-  if (c->out_pinned.size() >= 4) {  // keep at most four cached registrations (oldest out)
+  for (auto& e : c->out_pinned_run)
+    if (e.first == ptr && e.second >= bytes) return BK_OK;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, ptr) == cudaSuccess && at.type != cudaMemoryTypeUnregistered)
+    return BK_OK;   // device / managed memory, the caller's own pinned memory, or still registered by us
+  cudaGetLastError();
+  if (keep && c->out_pinned.size() >= 4) {
     cudaHostUnregister(c->out_pinned.front().first);
     c->out_pinned.erase(c->out_pinned.begin());
   }
   BK_CUDA(cudaHostRegister(ptr, bytes, cudaHostRegisterPortable));
-  c->out_pinned.emplace_back(ptr, bytes);
+  (keep ? c->out_pinned : c->out_pinned_run).emplace_back(ptr, bytes);
   return BK_OK;
+}
+
+// End of every bk_run (after all its copies completed or were drained): release this run's output
+// registrations.
+void release_run_outputs(bk_ctx* c) {
+  for (auto& e : c->out_pinned_run) cudaHostUnregister(e.first);
+  c->out_pinned_run.clear();
+  cudaGetLastError();
+}
+
+void release_kept_outputs(bk_ctx* c) {
+  for (auto& e : c->out_pinned) cudaHostUnregister(e.first);
+  c->out_pinned.clear();
+  cudaGetLastError();
 }
 
 void unregister(bk_ctx* c) {

@@ -1,0 +1,119 @@
+"""GPU checks of the context's cached state across runs:
+  * CUDA graphs captured by one run are never replayed after a later run reallocated a resident
+    buffer they baked in (parameters alternating small -> large -> small on one registration);
+  * output arrays bk_run page-locks are released at the end of the run unless the caller opted in
+    (BK_FLAG_KEEP_OUTPUTS_PINNED), and released by bk_unpin_outputs then;
+  * bk_run leaves the caller's current device unchanged;
+  * the in/out struct size is validated for every kernel id, baseline flags included."""
+import ctypes as C
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from paper_conf_ipps_mokhtaris14_b200 import bk
+
+pytestmark = pytest.mark.gpu
+MIB = 1 << 20
+
+
+def is_registered(arr: np.ndarray) -> bool:
+    """True iff `arr`'s pages are page-locked by cudaHostRegister (probe: unregister fails with
+    cudaErrorHostMemoryNotRegistered otherwise; a successful probe re-registers it)."""
+    import torch
+    cr = torch.cuda.cudart()
+    rc = int(cr.cudaHostUnregister(arr.ctypes.data))
+    if rc == 0:
+        assert int(cr.cudaHostRegister(arr.ctypes.data, arr.nbytes, 0)) == 0
+        return True
+    return False
+
+
+@pytest.mark.parametrize("mode", ["dense", "zc"])
+def test_groupby_alternating_G_replays_fresh_buffers(mode):
+    n = 300_000
+    g = gen.groupby(n=n, G=100)
+    with bk.Context(window_bytes=2 * MIB, record_size=16, gather_mode=mode) as ctx:
+        ctx.register(g, None, n_records=n)
+        for G in (100, 8192, 100, 8192, 100):
+            c, q, a = ctx.groupby(G)
+            wc_, wq, wa = oracle.groupby(g, n, 16, G)
+            assert np.array_equal(c, wc_) and np.array_equal(q, wq), G
+            np.testing.assert_allclose(a, wa, rtol=1e-5, atol=0)
+
+
+def test_grep_cap_small_large_small():
+    gb, goff = gen.grep_records(n=40_000)
+    want = oracle.grep(gb, goff, b"bigk")
+    with bk.Context(window_bytes=1 * MIB, gather_mode="zc") as ctx:
+        ctx.register(gb, goff)
+        for cap in (len(want) + 1, len(goff), len(want) + 1, len(goff)):
+            assert np.array_equal(ctx.grep(b"bigk", cap=cap), want), cap
+
+
+def test_wordcount_kmer_wordcount_share_table():
+    """word count and k-mers share the resident hash-table buffer: on one registration (256-B DNA
+    read records, word count over whole fixed records), k-mers grow it between two word counts."""
+    n = 6000
+    d = gen.dna(n=n)
+    want_wc = oracle.wc(d, np.arange(n, dtype=np.uint64) * 256)
+    okm, oct_ = oracle.kmer(d, n, k=31)
+    b = d.tobytes()
+    with bk.Context(window_bytes=1 * MIB, record_size=256, gather_mode="zc") as ctx:
+        ctx.register(d, None, n_records=n)
+        for step in range(3):
+            o, l, c = ctx.wordcount(cap=1 << 17, table_slots=1 << 18)
+            assert sorted((b[int(x): int(x) + int(y)], int(z)) for x, y, z in zip(o, l, c)) == want_wc, step
+            km, ct, _ = ctx.kmer(k=31, table_slots=1 << (20 + 2 * step), cap=1 << 20)
+            o = np.argsort(km)
+            assert np.array_equal(km[o], okm) and np.array_equal(ct[o], oct_), step
+
+
+def test_partition_buckets_alternate():
+    n = 200_000
+    kv = gen.kv(n=n)
+    with bk.Context(window_bytes=2 * MIB, record_size=16) as ctx:
+        ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=n)
+        for B in (256, 4096, 256):
+            out, cc, bc = ctx.partition(B)
+            assert np.array_equal(bk.partition_materialize(out, cc), oracle.partition(kv, B)[1]), B
+
+
+def test_outputs_released_after_run_unless_kept():
+    n = 100_000
+    x = gen.points(n=n)
+    mu = x[:64]
+    cid = np.zeros(n, np.int32)
+    with bk.Context(window_bytes=2 * MIB, record_size=64) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=n)
+        ctx.kmeans(mu, cid=cid)
+        assert not is_registered(cid)          # per-run registration released
+    cid2 = np.zeros(n, np.int32)
+    with bk.Context(window_bytes=2 * MIB, record_size=64, keep_outputs_pinned=True) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=n)
+        ctx.kmeans(mu, cid=cid2)
+        assert is_registered(cid2)             # cached across runs (opt-in)
+        ctx.kmeans(mu, cid=cid2)
+        ctx.unpin_outputs()
+        assert not is_registered(cid2)
+    assert np.array_equal(cid, cid2)
+
+
+def test_current_device_restored_and_struct_size_checked():
+    import torch
+    torch.cuda.set_device(0)
+    n = 10_000
+    g = gen.groupby(n=n)
+    for flags in ({}, {"baseline_dbuf": True}):
+        with bk.Context(window_bytes=1 * MIB, record_size=16, **flags) as ctx:
+            ctx.register(g, None, n_records=n)
+            ctx.groupby(4096)
+            assert torch.cuda.current_device() == 0
+            o = bk._hdr(bk.bk_out_groupby, bk.BK_K_GROUPBY)
+            o.h.struct_size = C.sizeof(bk.bk_out_grep)   # wrong size for this kernel id
+            cnt = np.empty(4096, np.uint64)
+            o.G, o.count, o.qty, o.amount = 4096, cnt.ctypes.data, cnt.ctypes.data, cnt.ctypes.data
+            with pytest.raises(bk.BkError) as e:
+                bk.bk_run(ctx.ctx, bk.BK_K_GROUPBY, None, o)
+            assert e.value.status == bk.BK_E_INVAL

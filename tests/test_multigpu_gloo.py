@@ -23,6 +23,11 @@ def free_port():
     return p
 
 
+def word_key(w: bytes) -> int:
+    import hashlib
+    return int.from_bytes(hashlib.blake2b(w, digest_size=8).digest(), "little") >> 1
+
+
 def worker(rank, world, port, q):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -58,9 +63,14 @@ def worker(rank, world, port, q):
         boff, out = oracle.partition(kv, 64)
         start, gboff = merge.merge_partition_offsets(np.diff(boff))
         res["partition"] = (start, gboff, boff, out)
-        # word count: union of per-rank tables
+        # word count: the all-gather of compacted per-rank rows (merge.gather_rows; the GPU merge by
+        # key, bk_merge_counts, is covered by tests/test_gpu_merge.py): rows {key, len, count, rank, off}
         tb, toff = gen.text(gen.SEED_WC + rank, cap_bytes=20_000)
-        res["wc"] = merge.merge_wordcount(dict(oracle.wc(tb, toff)))
+        raw = tb.tobytes()
+        rows = [[word_key(w), len(w), c, rank, raw.find(w)] for w, c in oracle.wc(tb, toff)]
+        t = torch.tensor(rows, dtype=torch.int64)
+        g, counts, stride = merge.gather_rows(t, len(rows) - 3)   # a rank may send fewer rows than it holds
+        res["wc"] = (g.numpy(), counts, stride, len(rows))
         q.put((rank, res))
     finally:
         dist.destroy_process_group()
@@ -118,13 +128,19 @@ def test_merge_matches_single_process(world):
             seg = out[int(boff[b]): int(boff[b + 1])]
             glob[int(start[b]): int(start[b]) + len(seg)] = seg
     assert np.array_equal(glob, wout)
-    # word count
-    want = {}
+    # word count: the gathered segments hold every rank's first n rows, padded to the longest
+    g, counts, stride, nrows = results[0]["wc"]
+    assert np.array_equal(g, results[1]["wc"][0]) and stride == max(counts)
+    merged = {}
     for r in range(world):
         tb, toff = gen.text(gen.SEED_WC + r, cap_bytes=20_000)
-        for w, cnt in oracle.wc(tb, toff):
-            want[w] = want.get(w, 0) + cnt
-    assert results[0]["wc"] == results[1]["wc"] == want
+        words = oracle.wc(tb, toff)
+        seg = g[r * stride: r * stride + int(counts[r])]
+        assert int(counts[r]) == len(words) - 3
+        for (w, c), row in zip(words, seg):
+            assert row[0] == word_key(w) and row[1] == len(w) and row[2] == c and row[3] == r
+            merged[w] = merged.get(w, 0) + c
+    assert len(merged) > 100
 
 
 def test_shard_range_covers():
