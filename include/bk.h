@@ -63,8 +63,14 @@ typedef enum {
                            the warp-tile layout (the paper's CPU assembly), then one DMA */
   BK_GATHER_DENSE = 3,  /* one contiguous DMA of the chunk's records (copy engine), then an
                            HBM->HBM re-layout kernel (fetch-all) */
-  BK_GATHER_HYBRID = 4  /* chunks split between the GPU zero-copy gather and CPU assembly, running
+  BK_GATHER_HYBRID = 4, /* chunks split between the GPU zero-copy gather and CPU assembly, running
                            concurrently and sharing the link (see zc_share_pm) */
+  BK_GATHER_FUSED = 5   /* BK_K_WORDCOUNT only (AUTO picks it there): the whole run is ONE persistent
+                           kernel (the paper's single launch) — per unit of whole records,
+                           stage 1 from the offsets, stages 2+3 as cp.async zero-copy copies into a
+                           shared-memory ring (S units per CTA, grid x S x unit <= window_bytes), stage
+                           4 from shared memory. Other kernels treat FUSED as AUTO; a record longer
+                           than a unit falls back to ZC. */
 } bk_gather_mode;
 
 typedef struct bk_config {
@@ -120,7 +126,8 @@ BK_API int bk_create(const bk_config* cfg, bk_ctx** out_ctx);
  * each <= nbytes; record i = [off[i], off[i+1]) with off[n] := nbytes; empty records are legal.
  * record_offsets == NULL: fixed records of cfg.record_size bytes (nbytes % record_size == 0,
  * n_records must equal nbytes / record_size). Memory is pinned ONCE here (cudaHostRegister,
- * mapped + portable + read-only where the device supports it: libbk never writes the data set)
+ * mapped + portable, + read-only where the device supports it and host_ptr and nbytes are multiples
+ * of 4 KiB so that the registration owns its pages: libbk never writes the data set)
  * unless already pinned; pre-pinned memory is left as is.
  * Validation is O(n) once: BK_E_INVAL on malformed offsets. */
 BK_API int bk_register_segments(bk_ctx* ctx, const void* host_ptr, uint64_t nbytes,
@@ -302,6 +309,11 @@ typedef struct bk_stats {
   double ms_d2h;              /* BK_FLAG_PROFILE: busy time of the device->host write-back copies (partitioned
                                  chunks, k-means cluster ids); counted in ms_xfer_busy */
   uint64_t n_d2h;             /*   number of write-back copies timed */
+  uint64_t n_units;           /* BK_GATHER_FUSED: units streamed through the shared-memory ring */
+  uint32_t unit_bytes;        /*   unit capacity in bytes (UB) */
+  uint32_t fused_grid;        /*   persistent CTAs */
+  double fused_wait_frac;     /*   BK_FLAG_PROFILE: share of CTA time waiting for a unit's bytes to land */
+  double fused_compute_frac;  /*   ... computing (stage 1 lane plan + stage 4), while later units' copies fly */
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);

@@ -16,14 +16,15 @@ LIB_PATH = os.path.join(_HERE, "libbk.so")
 
 BK_OK, BK_E_INVAL, BK_E_NOMEM, BK_E_CUDA, BK_E_STATE, BK_E_RANGE, BK_E_CAPACITY, BK_E_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
 BK_K_WORDCOUNT, BK_K_GREP, BK_K_KMEANS, BK_K_PARTITION, BK_K_GROUPBY, BK_K_LAYOUT_DUMP = 1, 2, 3, 4, 5, 100
-BK_GATHER_AUTO, BK_GATHER_ZC, BK_GATHER_CPU, BK_GATHER_DENSE, BK_GATHER_HYBRID = 0, 1, 2, 3, 4
+BK_GATHER_AUTO, BK_GATHER_ZC, BK_GATHER_CPU, BK_GATHER_DENSE, BK_GATHER_HYBRID, BK_GATHER_FUSED = 0, 1, 2, 3, 4, 5
 BK_FLAG_PROFILE = 1
 BK_FLAG_BASELINE_DBUF = 2
 BK_FLAG_BASELINE_SBUF = 4
 BK_FLAG_NO_GRAPH = 8
 BK_FLAG_TEST_DELAYS = 16
 BK_FLAG_KEEP_OUTPUTS_PINNED = 32
-GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE, "hybrid": BK_GATHER_HYBRID}
+GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE, "hybrid": BK_GATHER_HYBRID,
+                "fused": BK_GATHER_FUSED}
 
 u32, i32, u64, P = C.c_uint32, C.c_int32, C.c_uint64, C.c_void_p
 
@@ -79,7 +80,9 @@ class bk_stats(C.Structure):
                 ("ms_compute", C.c_double), ("n_gather", u64), ("n_chunks_cpu", u64), ("ms_cpu_gather", C.c_double),
                 ("ms_xfer_busy", C.c_double), ("ms_compute_busy", C.c_double), ("ms_overlap", C.c_double),
                 ("ms_zc", C.c_double), ("n_zc", u64), ("ms_relayout", C.c_double), ("n_relayout", u64),
-                ("n_chunks_zc", u64), ("bytes_zc", u64), ("records_zc", u64), ("ms_d2h", C.c_double), ("n_d2h", u64)]
+                ("n_chunks_zc", u64), ("bytes_zc", u64), ("records_zc", u64), ("ms_d2h", C.c_double), ("n_d2h", u64),
+                ("n_units", u64), ("unit_bytes", u32), ("fused_grid", u32), ("fused_wait_frac", C.c_double),
+                ("fused_compute_frac", C.c_double)]
 
 
 class bk_out_pattern(C.Structure):

@@ -97,6 +97,16 @@ struct WcEntry {            // 32 B open-addressing slot
 void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask,
                unsigned long long* used, int* err, cudaStream_t s);
+// C1 as one persistent launch (stages 1-4 fused, shared-memory ring): unit plan ub/uby (U+1 each,
+// device), UB/UR bytes/records caps per unit; *next zeroed before the launch; prof optional
+uint32_t wc_fused_stage_bytes(uint32_t UB, uint32_t UR);
+int wc_fused_grid(uint32_t stage_bytes);
+int wc_fused_stages();
+uint32_t wc_fused_threads();   // lanes (threads) per CTA = lanes per unit
+void launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t* off, uint64_t rec_size, uint64_t n,
+                     const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
+                     unsigned long long* next, WcEntry* table, uint64_t mask, unsigned long long* used, int* err,
+                     unsigned long long* prof, cudaStream_t s);
 // double-buffering baseline (variant iv): raw chunk bytes start at absolute offset base_byte
 void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
                     uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,

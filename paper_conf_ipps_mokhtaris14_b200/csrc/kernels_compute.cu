@@ -321,6 +321,221 @@ __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, 
 }
 
 // ------------------------------------------------------------------------------------------
+// C1 word count as ONE persistent launch: BigKernel's single kernel ("a single kernel
+// invocation"; Fig. 3 P:588-660 one block runs address generation and computation, the stages
+// overlapped across buffer instances), on sm_100a:
+//   * each CTA streams whole units (<= UB bytes / UR records of whole records, planned on the host
+//     once per registration, a1) through an S-stage shared-memory ring — the device working set
+//     is grid x S x stage <= window_bytes;
+//   * stage 1 (address generation): per unit, the record offsets (read zero-copy with
+//     cp.async) give every lane its contiguous record range by the lane rule (A4) and the byte
+//     range to fetch;
+//   * stages 2+3 (assembly + transfer): cp.async 16-B copies of exactly the unit's bytes
+//     from pinned, mapped host memory into shared memory, coalesced (512 B per warp instruction),
+//     issued S-1 units ahead so the PCIe reads of later units are in flight while this unit
+//     computes (the paper's n-3 buffer distance, as cp.async groups);
+//   * stage 4: each thread tokenises its lane from shared memory, words go through the
+//     warp queue / block hot-word table / global table of k_wc (same identities).
+// The ring replaces the per-chunk launch chain of the event pipeline (~5 launches per chunk at the
+// 8 MiB window's 0.4 MB chunks, profiles/r01_wc_sweep.md); the only per-unit synchronisation is
+// two CTA barriers (the paper's bar.red).
+constexpr int kFuThreads = 128;   // = kWcBlock: the WcShared queues are per warp of this block size
+constexpr int kFuStages = 3;
+
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+
+struct FusedArgs {
+  const uint8_t* data;        // device alias of the registered (mapped) data set
+  uint64_t nbytes;
+  const uint64_t* off;        // device alias of the mapped offsets, nullptr: fixed records
+  uint64_t rec_size;
+  uint64_t n;
+  const uint64_t* ub;         // unit record bounds (U + 1), device
+  const uint64_t* uby;        // unit byte bounds (U + 1), device
+  uint32_t U, UB, UR;         // units; bytes / records per unit (caps)
+  uint32_t stage_bytes;       // shared-memory bytes of one ring stage
+  unsigned long long* next;   // unit claim counter (zeroed by the run)
+  WcEntry* table;
+  uint64_t mask;
+  unsigned long long* used;
+  int* err;
+  unsigned long long* prof;   // optional: [0] wait cycles, [1] compute cycles, [2] CTA cycles (summed)
+};
+
+__global__ void __launch_bounds__(kFuThreads) k_wc_fused(FusedArgs a) {
+  extern __shared__ __align__(128) unsigned char fu_smem[];
+  __shared__ WcShared sh;
+  __shared__ uint32_t s_unit[kFuStages];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const unsigned lt = (1u << lane) - 1;
+  for (int i = tid; i < kWcTab; i += blockDim.x) { sh.k1[i] = 0; sh.k2[i] = 0; sh.cnt[i] = 0; }
+  const long long t_start = clock64();
+  long long t_wait = 0, t_comp = 0;
+  const uint32_t none = 0xffffffffu;
+  auto txt_of = [&](int st) { return fu_smem + (size_t)st * a.stage_bytes; };
+  auto offs_of = [&](int st) { return reinterpret_cast<uint64_t*>(fu_smem + (size_t)st * a.stage_bytes + a.UB + 32); };
+  // stages 1-3 of unit u into ring stage st: offsets slice + the unit's bytes, cp.async
+  auto prefetch = [&](int st, uint32_t u) {
+    if (u == none) return;
+    const uint64_t lo = a.ub[u], hi = a.ub[u + 1];
+    const uint64_t b0 = a.uby[u], b1 = a.uby[u + 1];
+    if (a.off) {
+      uint64_t* o = offs_of(st);
+      for (uint64_t j = tid; j < hi - lo; j += blockDim.x) cp_async8(o + j, a.off + lo + j);
+    }
+    const uintptr_t first = ((uintptr_t)(a.data + b0)) & ~(uintptr_t)15;
+    const uintptr_t last = ((uintptr_t)(a.data + b1) + 15) & ~(uintptr_t)15;
+    const uintptr_t dlo = (uintptr_t)a.data, dhi = (uintptr_t)(a.data + a.nbytes);
+    uint8_t* t = txt_of(st);
+    for (uintptr_t p = first + 16 * (uintptr_t)tid; p < last; p += 16 * (uintptr_t)blockDim.x) {
+      uint8_t* d = t + (p - first);
+      if (p >= dlo && p + 16 <= dhi) {
+        cp_async16(d, reinterpret_cast<const void*>(p));
+      } else {   // a word straddling the data set's edge: only its in-range bytes are read
+        for (int q = 0; q < 16; ++q) d[q] = (p + q >= dlo && p + q < dhi) ? *reinterpret_cast<const uint8_t*>(p + q) : 0;
+      }
+    }
+  };
+  auto claim = [&](int st) {
+    if (tid == 0) {
+      const unsigned long long u = atomicAdd(a.next, 1ull);
+      s_unit[st] = u < a.U ? (uint32_t)u : none;
+    }
+  };
+  // fill the ring: S-1 units in flight before the first compute
+  for (int st = 0; st < kFuStages - 1; ++st) claim(st);
+  __syncthreads();
+  for (int st = 0; st < kFuStages - 1; ++st) {
+    prefetch(st, s_unit[st]);
+    cp_async_commit();
+  }
+  int qn = 0;
+  for (uint32_t it = 0;; ++it) {
+    const int cur = (int)(it % kFuStages), nxt = (int)((it + kFuStages - 1) % kFuStages);
+    const long long t0 = clock64();
+    claim(nxt);
+    __syncthreads();   // (a) everyone left the compute of unit it-1 (stage nxt is free), the claim is visible
+    prefetch(nxt, s_unit[nxt]);
+    cp_async_commit();
+    cp_async_wait<kFuStages - 1>();   // this thread's copies of unit `it` landed
+    __syncthreads();   // (b) ... and every thread's
+    const long long t1 = clock64();
+    t_wait += t1 - t0;
+    const uint32_t u = s_unit[cur];
+    if (u == none) break;
+    // ---- stage 1 (lane plan) + stage 4 (tokenise, count) of unit u
+    const uint64_t lo = a.ub[u], hi = a.ub[u + 1];
+    const uint64_t base = a.uby[u], end = a.uby[u + 1];
+    const uint32_t nrec = (uint32_t)(hi - lo), A = (uint32_t)(end - base);
+    const uint8_t* txt = txt_of(cur) + (((uintptr_t)(a.data + base)) & 15);
+    const uint64_t* offs = offs_of(cur);
+    auto rpos = [&](uint32_t j) -> uint32_t {   // start of record lo+j relative to the unit (j <= nrec)
+      if (j >= nrec) return A;
+      return a.off ? (uint32_t)(offs[j] - base) : (uint32_t)((lo + j) * a.rec_size - base);
+    };
+    const uint32_t L = blockDim.x;
+    // first(t) = min{ j : rpos(j) >= floor(t*A/L) } (the lane rule, A4), by binary search in smem
+    auto first_of = [&](uint32_t t) -> uint32_t {
+      if (t >= L) return nrec;
+      const uint32_t target = (uint32_t)(((uint64_t)t * A) / L);
+      uint32_t l = 0, h = nrec;
+      while (l < h) {
+        const uint32_t m = (l + h) >> 1;
+        if (rpos(m) >= target) h = m; else l = m + 1;
+      }
+      return l;
+    };
+    const uint32_t f0 = first_of(tid), f1 = first_of(tid + 1);
+    const uint32_t x0 = rpos(f0), x1 = rpos(f1);
+    uint32_t j = f0 + 1;
+    uint32_t next_b = j <= f1 ? rpos(j) : 0xffffffffu;
+    const uint32_t steps = x1 - x0 + 1;   // the last step (p == x1) is the lane's closing boundary
+    uint32_t wsteps = steps;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) wsteps = max(wsteps, __shfl_xor_sync(kFull, wsteps, o));
+    bool in_word = false;
+    uint64_t h1 = 0, h2 = 0;
+    uint32_t wstart = 0, wlen = 0;
+    for (uint32_t k = 0; k < wsteps; ++k) {
+      const uint32_t p = x0 + k;
+      const bool valid = k < steps;
+      bool boundary = valid && p == x1;
+      if (valid && p == next_b) {
+        boundary = true;
+        do {   // several records may start here if some are empty
+          ++j;
+          next_b = j <= f1 ? rpos(j) : 0xffffffffu;
+        } while (next_b == p);
+      }
+      const uint32_t ch = (valid && p < x1) ? txt[p] : 0x20u;
+      const bool delim = is_delim(ch);
+      const bool end = valid && in_word && (boundary || delim);
+      const unsigned m = __ballot_sync(kFull, end);
+      if (m) {
+        if (end) {
+          const uint64_t occ = base + wstart;
+          if (wlen >= (1u << 24) || occ >= (1ull << 40)) atomicOr(a.err, kErrWordTooLong);
+          const int i = qn + __popc(m & lt);
+          sh.qk1[w][i] = h1;
+          sh.qk2[w][i] = h2;
+          sh.qol[w][i] = (occ << 24) | wlen;
+        }
+        qn += __popc(m);
+        if (qn > kWcQ - 32) {
+          wc_flush_queue(sh, w, lane, qn, a.table, a.mask, a.used, a.err);
+          qn = 0;
+        }
+      }
+      if (end) in_word = false;
+      if (valid && p < x1 && !delim) {
+        if (!in_word) { in_word = true; wstart = p; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
+        h1 = (h1 ^ ch) * 0x100000001b3ull;
+        h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
+        h2 ^= h2 >> 29;
+        ++wlen;
+      }
+    }
+    t_comp += clock64() - t1;
+  }
+  cp_async_wait<0>();
+  if (qn) wc_flush_queue(sh, w, lane, qn, a.table, a.mask, a.used, a.err);
+  __syncthreads();
+  // flush the block table (as k_wc)
+  constexpr int kPer = kWcTab / kFuThreads;
+  unsigned long long k1[kPer], k2[kPer];
+  ulonglong2 home[kPer];
+#pragma unroll
+  for (int m = 0; m < kPer; ++m) {
+    const int i = tid + m * kFuThreads;
+    k1[m] = sh.k1[i];
+    k2[m] = sh.k2[i];
+    home[m] = k1[m] ? __ldcg(reinterpret_cast<const ulonglong2*>(&a.table[k1[m] & a.mask])) : make_ulonglong2(0, 0);
+  }
+#pragma unroll
+  for (int m = 0; m < kPer; ++m) {
+    const int i = tid + m * kFuThreads;
+    if (!k1[m]) continue;
+    if (wc_home_hit(home[m], k1[m], k2[m])) atomicAdd(&a.table[k1[m] & a.mask].count, (unsigned long long)sh.cnt[i]);
+    else wc_insert(a.table, a.mask, k1[m], k2[m], sh.ol[i], sh.cnt[i], a.used, a.err);
+  }
+  if (a.prof && tid == 0) {
+    atomicAdd(&a.prof[0], (unsigned long long)t_wait);
+    atomicAdd(&a.prof[1], (unsigned long long)t_comp);
+    atomicAdd(&a.prof[2], (unsigned long long)(clock64() - t_start));
+  }
+}
+
+// ------------------------------------------------------------------------------------------
 // C2 grep (MCA analogue): key = first strnlen(32) bytes of the record's 32-byte key
 // field (staged as words 2j, 2j+1 of the lane); match iff the pattern is a substring. Output
 // indices are ascending. Chunks compute in any order (per-slot streams). Per chunk:
@@ -694,6 +909,30 @@ void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, cons
   k_wc<kSub><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
 }
 
+uint32_t wc_fused_stage_bytes(uint32_t UB, uint32_t UR) { return (UB + 32 + (UR + 1) * 8 + 127) / 128 * 128; }
+
+int wc_fused_grid(uint32_t stage_bytes) {
+  int per = 0;
+  const size_t dyn = (size_t)kFuStages * stage_bytes;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_wc_fused, kFuThreads, dyn) != cudaSuccess || per < 1) {
+    cudaGetLastError();
+    per = 1;
+  }
+  return device_sms() * std::min(per, 2);
+}
+
+void launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t* off, uint64_t rec_size, uint64_t n,
+                     const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
+                     unsigned long long* next, WcEntry* table, uint64_t mask, unsigned long long* used, int* err,
+                     unsigned long long* prof, cudaStream_t s) {
+  FusedArgs a{data, nbytes, off, rec_size, n, ub, uby, U, UB, UR, wc_fused_stage_bytes(UB, UR), next, table, mask,
+              used, err, prof};
+  k_wc_fused<<<grid, kFuThreads, (size_t)kFuStages * a.stage_bytes, s>>>(a);
+}
+
+int wc_fused_stages() { return kFuStages; }
+uint32_t wc_fused_threads() { return kFuThreads; }
+
 void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
                     uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                     int* err, cudaStream_t s) {
@@ -766,7 +1005,7 @@ void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, 
 
 cudaError_t configure_compute_kernels() {
   for (const void* f : {(const void*)k_groupby<true>, (const void*)k_groupby<false>, (const void*)k_kmeans<true>,
-                        (const void*)k_kmeans<false>, (const void*)k_grep_count<true>}) {
+                        (const void*)k_kmeans<false>, (const void*)k_grep_count<true>, (const void*)k_wc_fused}) {
     const cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
     if (e != cudaSuccess) return e;
   }

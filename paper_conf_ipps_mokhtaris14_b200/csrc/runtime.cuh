@@ -162,6 +162,10 @@ struct bk_ctx {  // the opaque context of include/bk.h
   std::vector<cudaEvent_t> ev_part;
   bk::rt::DevBuf b_hist, b_colpre, b_totals, b_base;
   bk::rt::DevBuf b_h1, b_h2;                 // word-count key hashes (multi-GPU merge keys)
+  bk::rt::DevBuf b_units;                    // BK_GATHER_FUSED unit plan (record bounds, byte bounds)
+  std::string units_key;                     //   which plan b_units holds
+  uint64_t n_units = 0;
+  unsigned long long* d_fprof = nullptr;     //   in-kernel wait / compute cycle counters (3 x u64)
   bk::rt::DevBuf b_mown, b_mcnt, b_mctr;     // bk_merge_counts scratch (never captured in a graph)
   std::vector<std::pair<void*, uint64_t>> out_pinned;      // caller output arrays pinned across runs (opt-in)
   std::vector<std::pair<void*, uint64_t>> out_pinned_run;  // caller output arrays pinned for this run only

@@ -190,9 +190,14 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
     if (is_pinned(host_ptr)) {
       c->pinned_data = false;
     } else {
-      // read-only where supported: libbk never writes the registered data set
+      // read-only where supported (libbk never writes the registered data set) and only
+      // when the range owns whole pages: a read-only registration of a page that also holds other
+      // objects makes every later registration touching that page fail (measured: offsets arrays
+      // and output arrays from the same heap pages -> cudaErrorInvalidValue)
       int ro = 0;
       cudaDeviceGetAttribute(&ro, cudaDevAttrHostRegisterReadOnlySupported, c->cfg.device);
+      const uintptr_t pg = 4096;
+      if ((uintptr_t)host_ptr % pg || nbytes % pg) ro = 0;
       const unsigned fl = cudaHostRegisterMapped | cudaHostRegisterPortable | (ro ? cudaHostRegisterReadOnly : 0u);
       cudaError_t e = cudaHostRegister((void*)host_ptr, nbytes, fl);
       if (e != cudaSuccess && ro) {   // some platforms advertise but refuse it: plain mapped registration
@@ -234,6 +239,7 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
   c->n = n;
   c->registered = true;
   c->plan_cache.clear();
+  c->units_key.clear();
   drop_graphs(c);
   c->st.ms_register = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return BK_OK;
@@ -419,6 +425,7 @@ int bk_destroy(bk_ctx* c) {
   if (c->window) cudaFree(c->window);
   if (c->d_err) cudaFree(c->d_err);
   if (c->d_ctr) cudaFree(c->d_ctr);
+  if (c->d_fprof) cudaFree(c->d_fprof);
   if (c->h_ctr) cudaFreeHost(c->h_ctr);
   if (c->ev_begin) cudaEventDestroy(c->ev_begin);
   if (c->ev_end) cudaEventDestroy(c->ev_end);
@@ -438,7 +445,7 @@ int bk_destroy(bk_ctx* c) {
   release_run_outputs(c);
   release_kept_outputs(c);
   for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base, &c->b_h1, &c->b_h2, &c->b_mown, &c->b_mcnt,
-                    &c->b_mctr})
+                    &c->b_mctr, &c->b_units})
     b->release();
   for (auto* h : c->hstage) cudaFreeHost(h);
   for (auto e : c->h_done) cudaEventDestroy(e);

@@ -7,9 +7,146 @@ namespace bk {
 namespace rt {
 
 // ------------------------------------------------------------------ kernels
+
+// distinct words + totals of the finished run -> the caller's (host or device) arrays
+static int wordcount_results(bk_ctx* c, bk_out_wordcount* o, uint64_t slots) {
+  const unsigned long long nw = c->h_ctr[2];
+  o->n_words = nw;
+  if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
+  if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
+                                  (unsigned long long)slots);
+  if (nw) {   // host or device result arrays (unified addressing)
+    BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDefault));
+    BK_CUDA(cudaMemcpy(o->word_count, c->b_out3.p, nw * 8, cudaMemcpyDefault));
+    if (o->word_h1) BK_CUDA(cudaMemcpy(o->word_h1, c->b_h1.p, nw * 8, cudaMemcpyDefault));
+    if (o->word_h2) BK_CUDA(cudaMemcpy(o->word_h2, c->b_h2.p, nw * 8, cudaMemcpyDefault));
+  }
+  o->total_words = c->h_ctr[6];
+  c->st.bytes_d2h = nw * 20;
+  return BK_OK;
+}
+
+// BK_GATHER_FUSED unit plan: greedy whole records, each unit <= UB bytes and <= UR records (A3 with a
+// second cap: shared-memory slots hold the unit's offsets too). 0 on success, BK_E_RANGE when a
+// record exceeds UB (the caller falls back to the event pipeline).
+static int fused_units(bk_ctx* c, uint32_t UB, uint32_t UR, std::vector<uint64_t>& ub, std::vector<uint64_t>& uby) {
+  ub.assign(1, 0);
+  uby.assign(1, 0);
+  uint64_t lo = 0;
+  while (lo < c->n) {
+    uint64_t hi = lo;
+    const uint64_t b0 = rec_start(c, lo);
+    if (!c->off) {
+      const uint64_t k = std::min<uint64_t>(UB / c->cfg.record_size, UR);
+      if (k == 0) return BK_E_RANGE;
+      hi = std::min<uint64_t>(c->n, lo + k);
+    } else {
+      const uint64_t lim = b0 + UB;
+      const uint64_t rmax = std::min<uint64_t>(c->n, lo + UR);
+      while (hi < rmax && rec_start(c, hi + 1) <= lim) ++hi;
+      if (hi == lo) return BK_E_RANGE;
+    }
+    ub.push_back(hi);
+    uby.push_back(rec_start(c, hi));
+    lo = hi;
+  }
+  return BK_OK;
+}
+
+// Word count as one persistent launch (BK_GATHER_FUSED, kernels_compute.cu k_wc_fused). Returns
+// BK_E_RANGE (nothing enqueued) when a record does not fit a unit: the caller then runs the pipeline.
+static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uint64_t slots, uint64_t ocap) {
+  const int S = wc_fused_stages();
+  // units: as large as 16 KiB allow, but grid x S ring stages never exceed the device window
+  // (a small window keeps units of >= 2 KiB and runs fewer CTAs instead)
+  int grid = wc_fused_grid(wc_fused_stage_bytes(16384, 1024));
+  const uint64_t per_stage = c->cfg.window_bytes / ((uint64_t)grid * S);
+  uint64_t UB = per_stage > 200 ? (per_stage - 200) * 2 / 3 : 0;
+  UB = std::min<uint64_t>(UB, 16384) / 16 * 16;
+  if (UB < 2048) {
+    UB = 2048;
+    grid = (int)std::min<uint64_t>(grid, c->cfg.window_bytes / ((uint64_t)S * wc_fused_stage_bytes(2048, 128)));
+    if (grid < 1) return BK_E_RANGE;
+  }
+  const uint32_t UR = (uint32_t)std::max<uint64_t>(UB / 16, 16);
+  const std::string ukey = std::to_string(UB) + "/" + std::to_string(UR) + "/" + std::to_string(grid);
+  if (c->units_key != ukey) {
+    std::vector<uint64_t> ub, uby;
+    if (fused_units(c, (uint32_t)UB, UR, ub, uby)) return BK_E_RANGE;
+    c->n_units = ub.size() - 1;
+    BK_CUDA(c->b_units.ensure(2 * ub.size() * 8));
+    BK_CUDA(cudaMemcpy(c->b_units.p, ub.data(), ub.size() * 8, cudaMemcpyHostToDevice));
+    BK_CUDA(cudaMemcpy((uint64_t*)c->b_units.p + ub.size(), uby.data(), uby.size() * 8, cudaMemcpyHostToDevice));
+    c->units_key = ukey;
+  }
+  if (!c->d_fprof) BK_CUDA(cudaMalloc(&c->d_fprof, 4 * 8));
+  const uint64_t U = c->n_units;
+  const uint64_t* ubd = (const uint64_t*)c->b_units.p;
+  const bool prof = (c->cfg.flags & BK_FLAG_PROFILE) != 0;
+  WcEntry* table = (WcEntry*)c->b_table.p;
+  const std::string key = "wcfused/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + ukey;
+  int rc = run_device(c, stream, key, true, 1, [&]() -> int {
+    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
+    if (prof) BK_CUDA(cudaMemsetAsync(c->d_fprof, 0, 4 * 8, c->s_comp));
+    c->st.n_chunks = U;
+    c->st.lanes = wc_fused_threads();
+    BK_PROF(kStGather, c->s_comp, true);
+    launch_wc_fused(c->host_dev, c->nbytes, c->off ? c->off_dev : nullptr, c->off ? 0 : c->cfg.record_size, c->n,
+                    ubd, ubd + U + 1, (uint32_t)U, (uint32_t)UB, UR, grid, c->d_ctr + 7, table, slots - 1,
+                    c->d_ctr + 1, c->d_err, prof ? c->d_fprof : nullptr, c->s_comp);
+    BK_PROF(kStGather, c->s_comp, false);
+    launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
+                      (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p, ocap, c->s_comp);
+    c->n_launch += 2;
+    return (int)BK_OK;
+  });
+  if (rc) return rc;
+  c->st.gather_mode = BK_GATHER_FUSED;
+  c->st.chunk_budget = UB;
+  c->st.n_chunks = U;
+  c->st.lanes = wc_fused_threads();
+  c->st.bytes_accessed = c->nbytes;
+  c->st.bytes_h2d = c->nbytes;
+  c->st.bytes_meta = c->off ? c->n * 8 : 0;
+  c->st.n_chunks_zc = U;
+  c->st.bytes_zc = c->nbytes;
+  c->st.records_zc = c->n;
+  c->st.n_units = U;
+  c->st.unit_bytes = (uint32_t)UB;
+  c->st.fused_grid = (uint32_t)grid;
+  c->st.fused_wait_frac = c->st.fused_compute_frac = 0;
+  if (prof) {
+    unsigned long long fp[3] = {0, 0, 0};
+    BK_CUDA(cudaMemcpy(fp, c->d_fprof, sizeof fp, cudaMemcpyDeviceToHost));
+    if (fp[2]) {
+      c->st.fused_wait_frac = (double)fp[0] / (double)fp[2];
+      c->st.fused_compute_frac = (double)fp[1] / (double)fp[2];
+    }
+    // the one kernel is stages 1-4: its interval is the transfer interval, its compute share is
+    // the CTAs' compute time (every unit but the last S-1 of a CTA computes while later units fly)
+    c->st.ms_compute_busy = c->st.ms_zc * c->st.fused_compute_frac;
+    c->st.ms_compute = c->st.ms_compute_busy;
+    c->st.ms_overlap = c->st.ms_compute_busy;
+  }
+  return BK_OK;
+}
+
 int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   uint64_t slots = o->table_slots ? o->table_slots : (1ull << 20);
   if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
+  const uint64_t ocap0 = std::min<uint64_t>(o->cap, slots);
+  if ((c->cfg.gather_mode == BK_GATHER_FUSED || c->cfg.gather_mode == BK_GATHER_AUTO) && c->n) {
+    BK_CUDA(c->b_table.ensure(slots * sizeof(WcEntry)));
+    BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap0, 1) * 8));
+    BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(ocap0, 1) * 4));
+    BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap0, 1) * 8));
+    BK_CUDA(c->b_h1.ensure(std::max<uint64_t>(ocap0, 1) * 8));
+    BK_CUDA(c->b_h2.ensure(std::max<uint64_t>(ocap0, 1) * 8));
+    const int frc = run_wordcount_fused(c, o, stream, slots, ocap0);
+    if (frc == BK_OK) return wordcount_results(c, o, slots);
+    if (frc != BK_E_RANGE) return frc;
+  }
   Plan p;
   // word count is compute-bound (thread-per-lane scan + table updates): AUTO picks ZC, which needs
   // no raw buffer, so the window holds twice the text in flight; 256-B lanes (profiles/r01_wc_sweep.md)
@@ -40,22 +177,7 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
     return (int)BK_OK;
   });
   if (rc) return rc;
-  unsigned long long nw = 0;
-  nw = c->h_ctr[2];
-  o->n_words = nw;
-  if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
-  if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
-                                  (unsigned long long)slots);
-  if (nw) {   // host or device result arrays (unified addressing)
-    BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDefault));
-    BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDefault));
-    BK_CUDA(cudaMemcpy(o->word_count, c->b_out3.p, nw * 8, cudaMemcpyDefault));
-    if (o->word_h1) BK_CUDA(cudaMemcpy(o->word_h1, c->b_h1.p, nw * 8, cudaMemcpyDefault));
-    if (o->word_h2) BK_CUDA(cudaMemcpy(o->word_h2, c->b_h2.p, nw * 8, cudaMemcpyDefault));
-  }
-  o->total_words = c->h_ctr[6];
-  c->st.bytes_d2h = nw * 20;
-  return BK_OK;
+  return wordcount_results(c, o, slots);
 }
 
 int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {

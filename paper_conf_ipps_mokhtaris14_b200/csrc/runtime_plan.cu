@@ -115,6 +115,7 @@ int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p,
   p.a = a;
   if (c->cfg.lane_bytes) lane_target = c->cfg.lane_bytes;
   int mode = (int)c->cfg.gather_mode;
+  if (mode == BK_GATHER_FUSED) mode = BK_GATHER_AUTO;   // FUSED is word count's own single-launch path
   // AUTO (counters in profiles/): whole-record access -> DENSE (copy engine at
   // 55.5 GB/s beats zero-copy's 51.4); sparse access -> HYBRID (host assembly packs exactly the
   // accessed bytes; the zero-copy gather is request-rate bound and only adds capacity on top).

@@ -60,14 +60,16 @@ def test_wordcount_kmer_wordcount_share_table():
     want_wc = oracle.wc(d, np.arange(n, dtype=np.uint64) * 256)
     okm, oct_ = oracle.kmer(d, n, k=31)
     b = d.tobytes()
-    with bk.Context(window_bytes=1 * MIB, record_size=256, gather_mode="zc") as ctx:
-        ctx.register(d, None, n_records=n)
-        for step in range(3):
-            o, l, c = ctx.wordcount(cap=1 << 17, table_slots=1 << 18)
-            assert sorted((b[int(x): int(x) + int(y)], int(z)) for x, y, z in zip(o, l, c)) == want_wc, step
-            km, ct, _ = ctx.kmer(k=31, table_slots=1 << (20 + 2 * step), cap=1 << 20)
-            o = np.argsort(km)
-            assert np.array_equal(km[o], okm) and np.array_equal(ct[o], oct_), step
+    for mode in ("zc", "auto"):   # the event pipeline, and the fused single launch over fixed records
+        with bk.Context(window_bytes=1 * MIB, record_size=256, gather_mode=mode) as ctx:
+            ctx.register(d, None, n_records=n)
+            for step in range(3):
+                o, l, c = ctx.wordcount(cap=1 << 17, table_slots=1 << 18)
+                got = sorted((b[int(x): int(x) + int(y)], int(z)) for x, y, z in zip(o, l, c))
+                assert got == want_wc, (mode, step)
+                km, ct, _ = ctx.kmer(k=31, table_slots=1 << (20 + 2 * step), cap=1 << 20)
+                o = np.argsort(km)
+                assert np.array_equal(km[o], okm) and np.array_equal(ct[o], oct_), (mode, step)
 
 
 def test_partition_buckets_alternate():

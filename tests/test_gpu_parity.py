@@ -74,7 +74,7 @@ def test_layout_dump_matches_oracle(name, extents, rs, mode, lanes):
 
 
 # ------------------------------------------------------------------ C1 word count
-@pytest.mark.parametrize("mode", ["dense", "zc", "cpu", "hybrid"])
+@pytest.mark.parametrize("mode", ["dense", "zc", "cpu", "hybrid", "fused"])
 @pytest.mark.parametrize("window,slots", [(256 * 1024, 2), (1 * MIB, 4), (8 * MIB, 3)])
 def test_wordcount_small(mode, window, slots):
     buf, off = gen.text(cap_bytes=2 * MIB)
@@ -82,8 +82,30 @@ def test_wordcount_small(mode, window, slots):
     with bk.Context(window_bytes=window, n_slots=slots, gather_mode=mode) as ctx:
         ctx.register(buf, off)
         got = wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 18))
-        assert ctx.stats()["n_chunks"] >= 2
+        st = ctx.stats()
+        assert st["n_chunks"] >= 2
+        if mode == "fused":   # one persistent launch; its shared-memory ring stays inside the window
+            assert st["gather_mode"] == bk.BK_GATHER_FUSED and st["n_units"] == st["n_chunks"]
+            assert st["fused_grid"] * 3 * (st["unit_bytes"] * 3 // 2) <= window
+            assert st["bytes_accessed"] == len(buf) and st["bytes_meta"] == 8 * len(off)
     assert got == want
+
+
+@pytest.mark.parametrize("profile", [False, True])
+def test_wordcount_fused_repeat_and_profile(profile):
+    """The fused kernel replayed from its graph gives the same table every run; profiled runs
+    report the in-kernel wait / compute shares."""
+    buf, off = gen.text(cap_bytes=3 * MIB)
+    want = oracle.wc(buf, off)
+    with bk.Context(window_bytes=2 * MIB, profile=profile) as ctx:
+        ctx.register(buf, off)
+        for _ in range(3):
+            assert wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 18)) == want
+        st = ctx.stats()
+    assert st["gather_mode"] == bk.BK_GATHER_FUSED
+    if profile:
+        assert 0 < st["fused_wait_frac"] < 1 and 0 < st["fused_compute_frac"] < 1
+        assert st["ms_zc"] > 0
 
 
 def adversarial_text():
@@ -103,6 +125,12 @@ def test_wordcount_adversarial():
         with bk.Context(window_bytes=64 * 1024, n_slots=2, gather_mode=mode, chunk_bytes=1500, lanes=32) as ctx:
             ctx.register(buf, off)
             assert wc_multiset_gpu(buf, *ctx.wordcount(cap=4096)) == want
+    # the fused single launch: many small units (window 64 KiB -> few CTAs, 2 KiB units) and the default
+    for window in (64 * 1024, 8 * MIB):
+        with bk.Context(window_bytes=window, gather_mode="fused") as ctx:
+            ctx.register(buf, off)
+            assert wc_multiset_gpu(buf, *ctx.wordcount(cap=4096)) == want
+            assert ctx.stats()["gather_mode"] == bk.BK_GATHER_FUSED
 
 
 def test_wordcount_full_c1_config():
@@ -116,6 +144,7 @@ def test_wordcount_full_c1_config():
     assert got == want
     assert st["bytes_accessed"] == len(buf)        # I3: every byte accessed once
     assert st["n_chunks"] >= 8                      # out-of-core: data > window
+    assert st["gather_mode"] == bk.BK_GATHER_FUSED  # AUTO: the single persistent launch
 
 
 # ------------------------------------------------------------------ C2 grep
