@@ -4,7 +4,7 @@ ARCH   := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -std=c++17 -O3 -lineinfo $(ARCH) -Xcompiler -fPIC,-fvisibility=hidden -Xptxas -v
 PKG    := paper_conf_ipps_mokhtaris14_b200
 CSRC   := $(PKG)/csrc
-OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/kernels_pattern.o build/kernels_kmer.o build/kernels_merge.o build/runtime_plan.o build/runtime_pipeline.o build/runtime_kernels.o build/runtime_api.o build/host_gather.o
+OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/kernels_pattern.o build/kernels_kmer.o build/kernels_merge.o build/kernels_addr.o build/runtime_plan.o build/runtime_pipeline.o build/runtime_kernels.o build/runtime_api.o build/host_gather.o
 
 all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so baselines/libbkmt.so tests/user/libbkuser.so
 

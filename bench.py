@@ -499,7 +499,7 @@ def main():
         pctx.close()
         for k in ("ms_h2d", "ms_addrgen", "ms_gather", "ms_compute", "n_gather", "ms_cpu_gather", "ms_xfer_busy",
                   "ms_zc", "n_zc", "ms_relayout", "n_relayout", "n_chunks_zc", "bytes_zc", "records_zc", "ms_d2h", "n_d2h",
-                  "ms_compute_busy", "ms_overlap"):
+                  "ms_compute_busy", "ms_overlap", "fused_wait_frac", "fused_compute_frac", "fused_loader_wait_frac"):
             st[k] = pst[k]
         st["profiled_ms_device"] = pst["ms_device"]
     total_bytes = nbytes * world * args.steps
@@ -524,7 +524,17 @@ def main():
         if st.get("n_d2h") and st.get("ms_d2h", 0.0) > st[{"zc": "ms_zc", "h2d": "ms_h2d"}[dom]]:
             dom = "d2h"  # write-back (partition's bucket-sorted chunks) is the busier direction
     stage_ms["d2h"] = st.get("ms_d2h", 0.0)
-    if dom == "d2h":
+    if st["gather_mode"] == 5:
+        dom = "fused"   # word count as one persistent launch: stages 1-4 in k_wc_fused
+    stage_ms["fused"] = st["ms_zc"]
+    if dom == "fused":
+        # the single launch pulls the text and the record offsets over PCIe (cp.async zero-copy into
+        # its shared-memory ring) and computes on them: algorithmic bytes = text + offsets
+        launches = max(st["n_zc"], 1)
+        per_launch = st["bytes_h2d"] + st["bytes_meta"]
+        roof = {"kernel": "k_wc_fused (stages 1-4, one persistent launch, zero-copy cp.async into shared memory)",
+                "bound": "host_link", "peak": peak_h2d, "unit": "GB/s"}
+    elif dom == "d2h":
         # copy-engine DMA of the per-chunk outputs back to the host, running full duplex with the
         # H2D stream: against the per-direction peak measured with both directions busy
         launches = max(st["n_d2h"], 1)
@@ -557,7 +567,7 @@ def main():
         avg_ms = float("nan")
     roof["achieved"] = per_launch / (avg_ms * 1e-3) / 1e9
     roof["peak_source"] = ("pinned H2D cudaMemcpyAsync measured live in this run (MEASURED_PEAKS.json has no "
-                           "host-link entry)") if dom in ("h2d", "zc") else (
+                           "host-link entry)") if dom in ("h2d", "zc", "fused") else (
         "pinned H2D + D2H cudaMemcpyAsync running concurrently, per direction, measured live in this run"
         if dom == "d2h" else None) if roof["bound"] == "host_link" else (
         "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6650 GB/s")
@@ -598,22 +608,14 @@ def main():
         roof["note"] = ("the zero-copy key gather is bound by outstanding PCIe read requests (one per 32-B key, "
                         "~84 B of read-completion traffic each), not by bytes: frac is against the H2D DMA byte "
                         "peak, request_rate.frac against the probed request-rate peak (DESIGN.md §6, §9)")
-    if dom == "compute" and args.workload == "wordcount":
-        roof["note"] = ("k_wc is latency-bound, not bandwidth-bound: an 8 MiB window gives ~0.44-MB chunks, "
-                        "0.15 waves of the kernel (6% achieved occupancy, issue IPC 0.43 under ncu); its launches "
-                        "overlap across slots, and dropping it entirely would raise the step by only ~12% "
-                        "(profiles/r01_wc_sweep.md). The step-level link fraction is link.frac")
-    if dom == "compute" and args.workload == "kmer" and box.get("kmer_windows") and st.get("ms_compute_busy"):
-        # k-mer table updates are random 16-B entry accesses in a 4 GiB table: the bound is the HBM
-        # random-update rate, probed on this GPU (profiles/r01_probe_random.txt: read the key of a
-        # random entry, then an 8-B atomic add to its count, 2^28 entries: 16.9 G updates/s).
-        # Launches of consecutive chunks overlap, so the rate uses the union of the compute intervals.
-        rate = box["kmer_windows"] / (st["ms_compute_busy"] * 1e-3) / 1e9
-        roof["random_update"] = {"bound": "hbm_random_update", "achieved": rate, "peak": 16.94,
-                                 "unit": "G updates/s", "frac": rate / 16.94,
-                                 "peak_source": "profiles/r01_probe_random.txt load+atomic, 148x4 blocks",
-                                 "note": "achieved counts every k-mer window; equal k-mers of one warp step are "
-                                         "merged into one update, so it can exceed the probe"}
+    if dom == "fused":
+        roof["fused"] = {"units": st["n_units"], "unit_bytes": st["unit_bytes"], "ctas": st["fused_grid"],
+                         "loader_ctas": st["fused_loaders"], "ring_slots": st["fused_ring_slots"],
+                         "consumer_wait_frac": round(st["fused_wait_frac"], 4),
+                         "consumer_compute_frac": round(st["fused_compute_frac"], 4),
+                         "loader_wait_frac": round(st["fused_loader_wait_frac"], 4),
+                         "note": "in-kernel %globaltimer shares (profiled pass): consumers waiting for a unit's flag "
+                                 "vs computing while loaders stream later units; loaders waiting for a free ring slot"}
     roof["avg_launch_ms"] = avg_ms
     roof["launches_per_step"] = launches
 
@@ -624,7 +626,7 @@ def main():
         "config": {"workload": args.workload, "desc": WORKLOADS[args.workload][2],
                    "bytes_per_gpu": nbytes, "records_per_gpu": shard["n"], "window_bytes": window,
                    "n_slots": st["n_slots"],
-                   "gather_mode": {1: "zc", 2: "cpu", 3: "dense", 4: "hybrid"}.get(st["gather_mode"], "?"),
+                   "gather_mode": {1: "zc", 2: "cpu", 3: "dense", 4: "hybrid", 5: "fused"}.get(st["gather_mode"], "?"),
                    "chunks_cpu_assembled": st["n_chunks_cpu"], "n_chunks": st["n_chunks"],
                    "lanes_per_chunk": st["lanes"], "chunk_budget_bytes": st["chunk_budget"],
                    "l2": "inputs (>=64 MiB per GPU, host-resident) exceed the 126 MB L2; streamed from host each step",

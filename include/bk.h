@@ -65,12 +65,20 @@ typedef enum {
                            HBM->HBM re-layout kernel (fetch-all) */
   BK_GATHER_HYBRID = 4, /* chunks split between the GPU zero-copy gather and CPU assembly, running
                            concurrently and sharing the link (see zc_share_pm) */
-  BK_GATHER_FUSED = 5   /* BK_K_WORDCOUNT only (AUTO picks it there): the whole run is ONE persistent
-                           kernel (the paper's single launch) — per unit of whole records,
-                           stage 1 from the offsets, stages 2+3 as cp.async zero-copy copies into a
-                           shared-memory ring (S units per CTA, grid x S x unit <= window_bytes), stage
-                           4 from shared memory. Other kernels treat FUSED as AUTO; a record longer
-                           than a unit falls back to ZC. */
+  BK_GATHER_FUSED = 5,  /* BK_K_WORDCOUNT only (AUTO picks it there): the whole run is ONE persistent,
+                           cooperative kernel (the paper's single launch): loader CTAs copy
+                           each unit of whole records (offsets + bytes, zero-copy) into a ring in the
+                           window and publish it with a flag, consumer CTAs count from shared memory.
+                           Other kernels treat FUSED as AUTO; a window too small for two units, or a
+                           record longer than a unit, falls back to ZC. */
+  BK_GATHER_ADDR = 6    /* the paper's own stages 1-3 (§IV.A):
+                           stage 1 on the GPU generates every element address of every lane (elements
+                           of addr_elem_bytes), recognises per-lane base + stride patterns online
+                           (T = 8 buffered addresses, periods <= 4, verify, fall back to explicit
+                           addresses; BK_FLAG_NO_PATTERNS: always explicit) and writes descriptors +
+                           explicit addresses into pinned host memory; the host pool assembles each
+                           lane's bytes from them in the warp-tile layout; one DMA H2D. Same staged
+                           bytes as every other mode. Never graph-replayed (host work per chunk). */
 } bk_gather_mode;
 
 typedef struct bk_config {
@@ -89,7 +97,9 @@ typedef struct bk_config {
   uint32_t zc_share_pm;   /* HYBRID: 0 = adaptive split (a zero-copy chunk is issued whenever fewer
                              than (n_slots-1)/2 are in flight); else per-mille of chunks gathered
                              zero-copy, deterministic: chunk i is zero-copy iff floor((i+1)s) > floor(i s) */
-  uint32_t _reserved;
+  uint32_t addr_elem_bytes; /* BK_GATHER_ADDR: bytes read per generated address (1, 2, 4, 8, 16); every
+                             accessed extent (or fixed record) length must be a multiple. 0 = the
+                             largest such power of two <= 8 (1 for whole variable-length records) */
 } bk_config;
 
 #define BK_FLAG_PROFILE 1u  /* time every stage of every chunk with CUDA events (bk_stats.ms_*); implies
@@ -106,6 +116,8 @@ typedef struct bk_config {
                                    host sleeps before CPU assembly, to expose missing ordering */
 #define BK_FLAG_BASELINE_SBUF 4u  /* the single-buffer variant: one buffer of the whole window,
                                      copy then compute, no overlap */
+#define BK_FLAG_NO_PATTERNS 64u  /* BK_GATHER_ADDR: no pattern recognition, every element address is sent
+                                    (the "addresses" column of the paper's Table II) */
 #define BK_FLAG_KEEP_OUTPUTS_PINNED 32u  /* caller-owned per-record output arrays that bk_run writes by DMA
                                      (bk_out_kmeans.cid, bk_out_partition.out_records, bk_out_kmer.kmer /
                                      .count) are page-locked (cudaHostRegister) by bk_run. Default: only for
@@ -311,9 +323,21 @@ typedef struct bk_stats {
   uint64_t n_d2h;             /*   number of write-back copies timed */
   uint64_t n_units;           /* BK_GATHER_FUSED: units streamed through the shared-memory ring */
   uint32_t unit_bytes;        /*   unit capacity in bytes (UB) */
-  uint32_t fused_grid;        /*   persistent CTAs */
-  double fused_wait_frac;     /*   BK_FLAG_PROFILE: share of CTA time waiting for a unit's bytes to land */
-  double fused_compute_frac;  /*   ... computing (stage 1 lane plan + stage 4), while later units' copies fly */
+  uint32_t fused_grid;        /*   persistent CTAs (one per SM) */
+  uint32_t fused_loaders;     /*   of which loaders (stages 1-3) */
+  uint32_t fused_ring_slots;  /*   HBM ring slots (R x slot <= window_bytes) */
+  double fused_wait_frac;     /*   BK_FLAG_PROFILE: consumers' share of time waiting for a unit's flag */
+  double fused_compute_frac;  /*   ... computing (stage 1 ranges + stage 4) while loaders stream later units */
+  double fused_loader_wait_frac; /* loaders' share of time waiting for a free ring slot */
+  uint64_t bytes_addr;        /* BK_GATHER_ADDR: address information the GPU wrote to host memory (48-B lane
+                                 descriptors + 8 B per explicit address + 8 B per chunk) */
+  uint64_t n_addr_lanes;      /*   lanes that generated addresses */
+  uint64_t n_pattern_lanes;   /*   ... of which sent a verified pattern instead of their addresses */
+  uint64_t n_addresses;       /*   element addresses generated */
+  uint64_t n_explicit_addr;   /*   ... of which sent explicitly */
+  uint32_t addr_elem_bytes;   /*   element size used */
+  uint32_t _pad_addr;
+  double ms_addr_wait;        /*   host time waiting for stage 1's address information */
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);
@@ -389,9 +413,43 @@ BK_API int bk_merge_counts(bk_ctx* ctx, const uint64_t* rows, uint32_t n_seg, ui
                            const uint64_t* seg_rows, uint32_t row_u64, uint32_t key_u64, uint32_t count_col,
                            uint64_t* out, uint64_t cap, uint64_t* n_out, void* stream);
 
+/* ---- user address generation (the paper's address mode with a caller-written stage 1) -----------
+ * BigKernel derives stage 1 from the kernel's own address computations; here the caller
+ * supplies that slice as a generator kernel. Per chunk libbk plans the lanes (contiguous record
+ * ranges balanced under `bound`, the access spec that bounds what the generator may touch), calls
+ * `gen` to enqueue the caller's kernel, which writes lane t's element addresses (byte offsets into
+ * the registered data set, in the order its stage-4 kernel will consume them) at
+ * addr[addr_base[t] + k], k < lane_desc[t].nbytes / elem_bytes, and the number written at
+ * addr_count[t] (counts start at 0). Then libbk runs the online pattern recogniser over those
+ * addresses, ships patterns / explicit addresses to the host, assembles the lanes (elem_bytes read
+ * at each address) in the warp-tile layout, DMAs them and calls `fn` (bk_run_user's stage-4
+ * callback) with lane_desc[t].nbytes = count x elem_bytes. Addresses outside the data set:
+ * BK_E_INVAL. All pointers in the view are DEVICE pointers valid for work enqueued on `stream`. */
+typedef struct bk_addr_view {
+  uint32_t struct_size;       /* = sizeof(bk_addr_view) */
+  uint32_t lanes;
+  uint64_t chunk_index, n_chunks, first_record, n_records;
+  const bk_lane* lane_desc;   /* lane t owns records [first, first + nrec); nbytes = its capacity in bytes */
+  const uint64_t* offsets;    /* record start offsets of the chunk's records (n_records), variable-length
+                                 records; NULL for fixed records (record r starts at r * record_size) */
+  uint64_t end_offset;        /* end of the chunk's last record */
+  uint64_t* addr;             /* out: element addresses, lane t's at addr[addr_base[t] + k] */
+  const uint64_t* addr_base;  /* lanes entries */
+  uint32_t* addr_count;       /* out: lanes entries, addresses lane t wrote */
+  uint32_t elem_bytes;
+  uint32_t _pad;
+} bk_addr_view;
+typedef int (*bk_addr_fn)(const bk_addr_view* view, void* stream, void* user);
+
+/* Ordered after `stream`; returns when every chunk's stage-4 work has completed. Always address
+ * mode (cfg.gather_mode is ignored; BK_FLAG_NO_PATTERNS applies). Errors as bk_run_user, plus
+ * BK_E_INVAL for a generator address outside the data set or a count above the lane's capacity. */
+BK_API int bk_run_user_addr(bk_ctx* ctx, const bk_access* bound, bk_addr_fn gen, void* gen_user, bk_chunk_fn fn,
+                            void* user, void* stream);
+
 /* ABI self-check for bindings: writes sizeof of bk_config, bk_out_wordcount, bk_out_grep,
  * bk_out_kmeans, bk_out_partition, bk_out_groupby, bk_out_layout, bk_stats, bk_out_pattern,
- * bk_out_kmer, bk_access, bk_chunk_view (in that order, up to n entries) and returns
+ * bk_out_kmer, bk_access, bk_chunk_view, bk_addr_view (in that order, up to n entries) and returns
  * BK_ABI_VERSION. Needs no GPU. */
 BK_API int bk_abi_sizes(uint32_t* sizes, int n);
 

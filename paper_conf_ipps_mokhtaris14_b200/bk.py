@@ -16,15 +16,17 @@ LIB_PATH = os.path.join(_HERE, "libbk.so")
 
 BK_OK, BK_E_INVAL, BK_E_NOMEM, BK_E_CUDA, BK_E_STATE, BK_E_RANGE, BK_E_CAPACITY, BK_E_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
 BK_K_WORDCOUNT, BK_K_GREP, BK_K_KMEANS, BK_K_PARTITION, BK_K_GROUPBY, BK_K_LAYOUT_DUMP = 1, 2, 3, 4, 5, 100
-BK_GATHER_AUTO, BK_GATHER_ZC, BK_GATHER_CPU, BK_GATHER_DENSE, BK_GATHER_HYBRID, BK_GATHER_FUSED = 0, 1, 2, 3, 4, 5
+BK_GATHER_AUTO, BK_GATHER_ZC, BK_GATHER_CPU, BK_GATHER_DENSE, BK_GATHER_HYBRID, BK_GATHER_FUSED, BK_GATHER_ADDR = (
+    0, 1, 2, 3, 4, 5, 6)
 BK_FLAG_PROFILE = 1
 BK_FLAG_BASELINE_DBUF = 2
 BK_FLAG_BASELINE_SBUF = 4
 BK_FLAG_NO_GRAPH = 8
 BK_FLAG_TEST_DELAYS = 16
 BK_FLAG_KEEP_OUTPUTS_PINNED = 32
+BK_FLAG_NO_PATTERNS = 64
 GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE, "hybrid": BK_GATHER_HYBRID,
-                "fused": BK_GATHER_FUSED}
+                "fused": BK_GATHER_FUSED, "addr": BK_GATHER_ADDR}
 
 u32, i32, u64, P = C.c_uint32, C.c_int32, C.c_uint64, C.c_void_p
 
@@ -33,7 +35,7 @@ class bk_config(C.Structure):
     _fields_ = [("struct_size", u32), ("device", i32), ("window_bytes", u64), ("n_slots", u32),
                 ("gather_mode", u32), ("chunk_bytes", u64), ("lanes", u32), ("host_threads", u32),
                 ("record_size", u64), ("flags", u32), ("lane_bytes", u32),
-                ("zc_share_pm", u32), ("_reserved", u32)]
+                ("zc_share_pm", u32), ("addr_elem_bytes", u32)]
 
 
 class bk_out_header(C.Structure):
@@ -81,8 +83,11 @@ class bk_stats(C.Structure):
                 ("ms_xfer_busy", C.c_double), ("ms_compute_busy", C.c_double), ("ms_overlap", C.c_double),
                 ("ms_zc", C.c_double), ("n_zc", u64), ("ms_relayout", C.c_double), ("n_relayout", u64),
                 ("n_chunks_zc", u64), ("bytes_zc", u64), ("records_zc", u64), ("ms_d2h", C.c_double), ("n_d2h", u64),
-                ("n_units", u64), ("unit_bytes", u32), ("fused_grid", u32), ("fused_wait_frac", C.c_double),
-                ("fused_compute_frac", C.c_double)]
+                ("n_units", u64), ("unit_bytes", u32), ("fused_grid", u32), ("fused_loaders", u32),
+                ("fused_ring_slots", u32), ("fused_wait_frac", C.c_double), ("fused_compute_frac", C.c_double),
+                ("fused_loader_wait_frac", C.c_double), ("bytes_addr", u64), ("n_addr_lanes", u64),
+                ("n_pattern_lanes", u64), ("n_addresses", u64), ("n_explicit_addr", u64), ("addr_elem_bytes", u32),
+                ("_pad_addr", u32), ("ms_addr_wait", C.c_double)]
 
 
 class bk_out_pattern(C.Structure):
@@ -113,16 +118,23 @@ class bk_chunk_view(C.Structure):
                 ("offsets", P), ("end_offset", u64)]
 
 
+class bk_addr_view(C.Structure):
+    _fields_ = [("struct_size", u32), ("lanes", u32), ("chunk_index", u64), ("n_chunks", u64),
+                ("first_record", u64), ("n_records", u64), ("lane_desc", P), ("offsets", P), ("end_offset", u64),
+                ("addr", P), ("addr_base", P), ("addr_count", P), ("elem_bytes", u32), ("_pad", u32)]
+
+
 # int (*bk_chunk_fn)(const bk_chunk_view* view, void* stream, void* user)
 bk_chunk_fn = C.CFUNCTYPE(C.c_int, C.POINTER(bk_chunk_view), P, P)
+bk_addr_fn = C.CFUNCTYPE(C.c_int, C.POINTER(bk_addr_view), P, P)
 
 BK_K_PATTERN_STATS = 101
 BK_K_KMER = 6
 ABI_STRUCTS = [bk_config, bk_out_wordcount, bk_out_grep, bk_out_kmeans, bk_out_partition, bk_out_groupby,
-               bk_out_layout, bk_stats, bk_out_pattern, bk_out_kmer, bk_access, bk_chunk_view]
+               bk_out_layout, bk_stats, bk_out_pattern, bk_out_kmer, bk_access, bk_chunk_view, bk_addr_view]
 EXPORTS = ["bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_strerror",
            "bk_last_error", "bk_get_stats", "bk_abi_sizes", "bk_partition_materialize", "bk_unpin_outputs",
-           "bk_merge_counts"]
+           "bk_merge_counts", "bk_run_user_addr"]
 
 _lib = None
 
@@ -155,8 +167,10 @@ def lib() -> C.CDLL:
         l.bk_partition_materialize.argtypes = [P, P, u64, u32, P, P, u32]
         l.bk_unpin_outputs.argtypes = [P]
         l.bk_merge_counts.argtypes = [P, P, u32, u64, P, u32, u32, u32, P, u64, C.POINTER(u64), P]
+        l.bk_run_user_addr.argtypes = [P, C.POINTER(bk_access), P, P, P, P, P]
         for name in ("bk_create", "bk_register_segments", "bk_run", "bk_run_user", "bk_destroy", "bk_get_stats",
-                     "bk_abi_sizes", "bk_partition_materialize", "bk_unpin_outputs", "bk_merge_counts"):
+                     "bk_abi_sizes", "bk_partition_materialize", "bk_unpin_outputs", "bk_merge_counts",
+                     "bk_run_user_addr"):
             getattr(l, name).restype = C.c_int
         _lib = l
     return _lib
@@ -191,7 +205,8 @@ def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_m
               chunk_bytes: int = 0, lanes: int = 0, record_size: int = 0, host_threads: int = 0,
               profile: bool = False, baseline_dbuf: bool = False, lane_bytes: int = 0,
               zc_share_pm: int = 0, baseline_sbuf: bool = False, no_graph: bool = False,
-              test_delays: bool = False, keep_outputs_pinned: bool = False) -> int:
+              test_delays: bool = False, keep_outputs_pinned: bool = False, no_patterns: bool = False,
+              addr_elem_bytes: int = 0) -> int:
     if isinstance(gather_mode, str):
         gather_mode = GATHER_NAMES[gather_mode]
     cfg = bk_config(C.sizeof(bk_config), device, window_bytes, n_slots, gather_mode, chunk_bytes, lanes,
@@ -199,9 +214,10 @@ def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_m
                     (BK_FLAG_PROFILE if profile else 0) | (BK_FLAG_BASELINE_DBUF if baseline_dbuf else 0) |
                     (BK_FLAG_BASELINE_SBUF if baseline_sbuf else 0) | (BK_FLAG_NO_GRAPH if no_graph else 0) |
                     (BK_FLAG_TEST_DELAYS if test_delays else 0) |
-                    (BK_FLAG_KEEP_OUTPUTS_PINNED if keep_outputs_pinned else 0),
+                    (BK_FLAG_KEEP_OUTPUTS_PINNED if keep_outputs_pinned else 0) |
+                    (BK_FLAG_NO_PATTERNS if no_patterns else 0),
                     lane_bytes,
-                    zc_share_pm, 0)
+                    zc_share_pm, addr_elem_bytes)
     ctx = P()
     check(lib().bk_create(C.byref(cfg), C.byref(ctx)), "bk_create")
     return ctx.value
@@ -422,6 +438,23 @@ class Context:
         fp = C.cast(fn, P)
         up = user if (user is None or isinstance(user, int)) else C.cast(C.pointer(user), P)
         check(lib().bk_run_user(self.ctx, C.byref(a), fp, up, stream), "bk_run_user")
+
+    def run_user_addr(self, gen, fn, gen_user=None, user=None, bound=None, lane_bytes: int = 0, stream=None):
+        """bk_run_user_addr: `gen` (a native bk_addr_fn) writes every lane's element addresses per chunk
+        (stage 1), libbk recognises patterns, ships addresses, assembles and DMAs (stages 2-3), then
+        `fn` (a native bk_chunk_fn) enqueues stage 4. `bound`: [(offset, length), ...] per record
+        bounding the lanes' capacities (None = whole records)."""
+        a = bk_access()
+        a.struct_size = C.sizeof(bk_access)
+        bound = bound or []
+        a.n_ext = len(bound)
+        for i, (eo, el) in enumerate(bound):
+            a.ext_off[i], a.ext_len[i] = eo, el
+        a.lane_bytes = lane_bytes
+        gu = gen_user if (gen_user is None or isinstance(gen_user, int)) else C.cast(C.pointer(gen_user), P)
+        up = user if (user is None or isinstance(user, int)) else C.cast(C.pointer(user), P)
+        check(lib().bk_run_user_addr(self.ctx, C.byref(a), C.cast(gen, P), gu, C.cast(fn, P), up, stream),
+              "bk_run_user_addr")
 
     def layout_dump(self, chunk: int, extents=None, stage_cap: int = 1 << 26, lane_cap: int = 1 << 20, stream=None):
         o = _hdr(bk_out_layout, BK_K_LAYOUT_DUMP)

@@ -48,6 +48,7 @@ enum : int {
   kErrKeyRange = 4,
   kErrWordTooLong = 8,
   kErrOutOverflow = 16,
+  kErrFusedTimeout = 32,   // a persistent kernel's producer/consumer wait exceeded its limit
 };
 
 // SM count of the current device (queried once per device, then cached): grids are sized in
@@ -97,16 +98,18 @@ struct WcEntry {            // 32 B open-addressing slot
 void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                const uint64_t* meta, uint64_t rec_size, WcEntry* table, uint64_t mask,
                unsigned long long* used, int* err, cudaStream_t s);
-// C1 as one persistent launch (stages 1-4 fused, shared-memory ring): unit plan ub/uby (U+1 each,
-// device), UB/UR bytes/records caps per unit; *next zeroed before the launch; prof optional
-uint32_t wc_fused_stage_bytes(uint32_t UB, uint32_t UR);
-int wc_fused_grid(uint32_t stage_bytes);
-int wc_fused_stages();
-uint32_t wc_fused_threads();   // lanes (threads) per CTA = lanes per unit
-void launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t* off, uint64_t rec_size, uint64_t n,
-                     const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
-                     unsigned long long* next, WcEntry* table, uint64_t mask, unsigned long long* used, int* err,
-                     unsigned long long* prof, cudaStream_t s);
+// C1 as one persistent launch (loader CTAs stream units into an HBM ring, consumer CTAs count):
+// unit plan ub/uby (U+1 each, device), UB/UR bytes/records caps per unit; ready/done: R flags each,
+// zeroed before the launch; prof optional (5 counters)
+uint32_t wc_fused_slot_bytes(uint32_t UB, uint32_t UR);
+size_t wc_fused_smem(uint32_t UB, uint32_t UR);
+int wc_fused_grid();
+uint32_t wc_fused_threads();
+cudaError_t launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t* off, uint64_t rec_size,
+                            const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
+                            uint32_t n_load, uint8_t* ring, uint32_t R, unsigned long long* ready,
+                            unsigned long long* done, WcEntry* table, uint64_t mask, unsigned long long* used,
+                            int* err, unsigned long long* prof, cudaStream_t s);
 // double-buffering baseline (variant iv): raw chunk bytes start at absolute offset base_byte
 void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
                     uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
@@ -188,7 +191,35 @@ cudaError_t launch_merge_counts(const uint64_t* rows, uint32_t n_seg, uint64_t s
                                 unsigned long long* cnt, uint64_t slots, uint64_t* out, uint64_t cap,
                                 unsigned long long* n_out, int* err, cudaStream_t s);
 
-// ---- online pattern recognition of stage 1 (kernels_pattern.cu, NEXT f2) ----
+// ---- stage 1 in address mode (kernels_addr.cu, BK_GATHER_ADDR) ----
+// One lane's address information as the host receives it (48 B): the element addresses are
+// base, base + stride[0], + stride[1], ... (strides repeat with period p) when p > 0; when p == 0
+// they are listed explicitly (count of them, in the chunk's compacted explicit-address buffer).
+struct AddrDesc {
+  uint64_t base;
+  int64_t stride[4];
+  uint32_t count;   // element addresses of the lane
+  int32_t p;        // period (1..4), 0 = explicit
+};
+// detect / verify per lane (descriptors to desc_host, mapped host memory), exclusive scan of the
+// explicit counts (total to *total_host), explicit addresses to exp_dev then exp_host (mapped).
+// user_addr != nullptr: addresses from a caller's generator (lane t: user_addr[user_base[t] + k],
+// k < user_count[t]); the kernel then also sets lanes[t].nbytes and tileK (run launch_tile_scan after).
+void launch_addr_stage1(const Chunk& c, const Access& a, const uint64_t* meta, LaneDesc* lanes, uint32_t* tileK,
+                        uint32_t elem, uint32_t T, uint32_t pmax, int patterns, const uint64_t* user_addr,
+                        const uint64_t* user_base, const uint32_t* user_count, AddrDesc* desc_host,
+                        uint32_t* ecount, uint64_t* epos, uint64_t* exp_dev, uint64_t* exp_host,
+                        uint64_t* total_host, cudaStream_t s);
+// bk_run_user_addr: lane t's address capacity lanes[t].nbytes / elem (into tmp) and its exclusive
+// scan base[t] (base[L] = total) — where the caller's generator writes lane t's addresses
+void launch_lane_bases(uint32_t L, const LaneDesc* lanes, uint32_t elem, uint32_t* tmp, uint64_t* base,
+                       cudaStream_t s);
+// tile bases from the per-tile word counts (the last kernel of launch_addrgen), for lane plans
+// whose byte counts were set after address generation
+void launch_tile_scan(const uint32_t* tileK, uint32_t ntiles, uint64_t* tile_base, uint64_t stage_cap, int* err,
+                      unsigned long long* staged_sum, cudaStream_t s);
+
+// ---- online pattern recognition (kernels_pattern.cu, NEXT f2) ----
 void launch_addr_patterns(const Chunk& c, const Access& a, const uint64_t* meta, const LaneDesc* lanes, uint32_t elem,
                           uint32_t T, uint32_t pmax, int32_t* lane_p, int64_t* lane_strides, uint64_t* lane_base,
                           uint64_t* lane_count, unsigned long long* totals, int dump, cudaStream_t s);

@@ -201,6 +201,85 @@ uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, c
   return size;
 }
 
+// Address mode (BK_GATHER_ADDR): the paper's CPU assembly loop, h_pBuf[i] = *(data + addrBuf[i])
+// (Fig. 3), per lane from its pattern (base + periodic strides) or its explicit address
+// list, in the lane's access order, written in the warp-tile layout. Reads are merged into runs of
+// contiguous elements (with a pattern the CPU reads each lane's data sequentially, §IV.B).
+uint64_t host_assemble_addr(HostPool& pool, const HostData& d, uint32_t L, uint32_t elem, const AddrDesc* desc,
+                            const uint64_t* exp, uint64_t n_exp, uint8_t* stage, uint64_t cap,
+                            std::vector<uint64_t>& epos, std::vector<uint64_t>& tbase) {
+  const uint32_t T = L / 32;
+  epos.resize((size_t)L + 1);
+  tbase.resize((size_t)T + 1);
+  for (uint32_t t = 0; t < L; ++t)
+    if (desc[t].count == 0xffffffffu) return UINT64_MAX - 1;   // a generator count above its lane's capacity
+  uint64_t e = 0, size = 0;
+  for (uint32_t w = 0; w < T; ++w) {
+    uint64_t K = 0;
+    for (uint32_t i = 0; i < 32; ++i) {
+      const AddrDesc& dd = desc[w * 32 + i];
+      epos[w * 32 + i] = e;
+      if (dd.p <= 0) e += dd.count;
+      K = std::max<uint64_t>(K, ((uint64_t)dd.count * elem + 15) / 16);
+    }
+    tbase[w] = size;
+    size += 512 * K;
+  }
+  tbase[T] = size;
+  epos[L] = e;
+  if (e != n_exp) return UINT64_MAX - 1;   // descriptors and explicit list disagree
+  if (size > cap) return UINT64_MAX;
+  std::atomic<uint32_t> next{0};
+  std::atomic<bool> bad{false};
+  pool.run([&](int) {
+    for (;;) {
+      const uint32_t w0 = next.fetch_add(8);
+      if (w0 >= T) break;
+      for (uint32_t w = w0; w < std::min(T, w0 + 8); ++w) {
+        uint8_t* tile = stage + tbase[w];
+        const uint64_t K = (tbase[w + 1] - tbase[w]) / 512;
+        for (int i = 0; i < 32; ++i) {
+          const uint32_t t = w * 32 + i;
+          const AddrDesc& dd = desc[t];
+          uint64_t b = 0;   // byte position in the lane's stream
+          auto put = [&](const uint8_t* src, uint64_t len) {
+            while (len) {
+              const uint64_t k = b >> 4, o = b & 15, m = std::min<uint64_t>(16 - o, len);
+              memcpy(tile + (k * 32 + i) * 16 + o, src, m);
+              b += m;
+              src += m;
+              len -= m;
+            }
+          };
+          uint64_t run0 = 0, runl = 0;   // current run of contiguous elements
+          auto elem_at = [&](uint64_t a) {
+            if (a > d.nbytes || elem > d.nbytes - a) { bad = true; return; }
+            if (runl && a == run0 + runl) { runl += elem; return; }
+            if (runl) put(d.base + run0, runl);
+            run0 = a;
+            runl = elem;
+          };
+          if (dd.p > 0) {
+            uint64_t a = dd.base;
+            for (uint32_t k = 0; k < dd.count; ++k) {
+              elem_at(a);
+              a += (uint64_t)dd.stride[k % (uint32_t)dd.p];
+            }
+          } else {
+            const uint64_t* x = exp + epos[t];
+            for (uint32_t k = 0; k < dd.count; ++k) elem_at(x[k]);
+          }
+          if (runl) put(d.base + run0, runl);
+          // zero the tail of the last word and the lane's holes up to the tile's longest lane
+          if (b & 15) memset(tile + ((b >> 4) * 32 + i) * 16 + (b & 15), 0, 16 - (b & 15));
+          for (uint64_t k = (b + 15) >> 4; k < K; ++k) memset(tile + (k * 32 + i) * 16, 0, 16);
+        }
+      }
+    }
+  });
+  return bad ? UINT64_MAX - 1 : size;
+}
+
 bool host_packable(const Access& a) { return !a.whole && a.n_ext == 1 && a.E > 0 && (a.E % 16) == 0; }
 
 uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* dst,

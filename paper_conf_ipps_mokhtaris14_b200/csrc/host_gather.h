@@ -49,6 +49,14 @@ uint64_t host_staged_size(const HostData& d, const Access& a, const Chunk& c);
 uint64_t host_gather_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* stage,
                            uint64_t cap, std::vector<uint64_t>& first_scratch, std::vector<uint64_t>& tile_scratch);
 
+// Address mode: assemble the chunk's L lanes from their address descriptors (desc, as stage 1 wrote
+// them) and the compacted explicit addresses (exp, n_exp entries) into `stage` (capacity cap), elem
+// bytes per address. Returns the staged size, UINT64_MAX if it exceeds cap, UINT64_MAX - 1 if an
+// address lies outside the data set or the descriptors disagree with n_exp.
+uint64_t host_assemble_addr(HostPool& pool, const HostData& d, uint32_t L, uint32_t elem, const AddrDesc* desc,
+                            const uint64_t* exp, uint64_t n_exp, uint8_t* stage, uint64_t cap,
+                            std::vector<uint64_t>& epos, std::vector<uint64_t>& tbase);
+
 // Single-extent access with E % 16 == 0 (host_packable): packs the chunk's accessed bytes in record
 // order, E bytes per record, into dst (16-B aligned) — a sequential read of the data set and a
 // sequential non-temporal write, the cheapest host gather there is. The warp-tile interleave is then

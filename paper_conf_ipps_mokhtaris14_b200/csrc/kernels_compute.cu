@@ -68,13 +68,17 @@ constexpr int kWcTab = 512;     // block table slots (a hot-word cache)
 constexpr int kWcQ = 256;       // per-warp queue of finished words
 constexpr int kWcProbes = 2;    // a crowded block-table slot sends the word to the global table
 
-struct WcShared {
+template <int NW, int Q>   // NW warps per block, Q queue entries per warp
+struct WcSharedT {
+  static constexpr int kQ = Q;
   unsigned long long k1[kWcTab], k2[kWcTab], ol[kWcTab];
   unsigned int cnt[kWcTab];
-  unsigned long long qk1[kWcBlock / 32][kWcQ], qk2[kWcBlock / 32][kWcQ], qol[kWcBlock / 32][kWcQ];
+  unsigned long long qk1[NW][Q], qk2[NW][Q], qol[NW][Q];
 };
+using WcShared = WcSharedT<kWcBlock / 32, kWcQ>;
 
-__device__ void tab_insert(WcShared& sh, WcEntry* table, uint64_t mask, unsigned long long k1,
+template <class SH>
+__device__ void tab_insert(SH& sh, WcEntry* table, uint64_t mask, unsigned long long k1,
                            unsigned long long k2, unsigned long long ol, unsigned int cnt,
                            unsigned long long* used, int* err) {
   uint32_t s = (uint32_t)(k1 >> 20) & (kWcTab - 1);
@@ -105,8 +109,9 @@ __device__ void tab_insert(WcShared& sh, WcEntry* table, uint64_t mask, unsigned
 
 // Insert the warp's n queued words, 32 at a time: finalise the identity here (every lane busy),
 // merge duplicates within a round by match_any, insert into the block table.
-__device__ __noinline__ void wc_flush_queue(WcShared& sh, int w, int lane, int n, WcEntry* table,
-                                               uint64_t mask, unsigned long long* used, int* err) {
+template <class SH>
+__device__ __noinline__ void wc_flush_queue(SH& sh, int w, int lane, int n, WcEntry* table,
+                                            uint64_t mask, unsigned long long* used, int* err) {
   __syncwarp();
   for (int base = 0; base < n; base += 32) {
     const int i = base + lane;
@@ -122,6 +127,30 @@ __device__ __noinline__ void wc_flush_queue(WcShared& sh, int w, int lane, int n
     if (v && lane == __ffs(m) - 1) tab_insert(sh, table, mask, k1, k2, ol, __popc(m), used, err);
   }
   __syncwarp();
+}
+
+// Block table -> global table: thread `tid` of `nthreads` moves its slots (all home-slot reads in
+// flight at once, then the adds), optionally clearing them for reuse.
+template <class SH, int kPer>
+__device__ __forceinline__ void wc_flush_block(SH& sh, int tid, int nthreads, WcEntry* table, uint64_t mask,
+                                               unsigned long long* used, int* err, bool clear) {
+  unsigned long long k1[kPer], k2[kPer];
+  ulonglong2 home[kPer];
+#pragma unroll
+  for (int m = 0; m < kPer; ++m) {
+    const int i = tid + m * nthreads;
+    k1[m] = sh.k1[i];
+    k2[m] = sh.k2[i];
+    home[m] = k1[m] ? __ldcg(reinterpret_cast<const ulonglong2*>(&table[k1[m] & mask])) : make_ulonglong2(0, 0);
+  }
+#pragma unroll
+  for (int m = 0; m < kPer; ++m) {
+    const int i = tid + m * nthreads;
+    if (!k1[m]) continue;
+    if (wc_home_hit(home[m], k1[m], k2[m])) atomicAdd(&table[k1[m] & mask].count, (unsigned long long)sh.cnt[i]);
+    else wc_insert(table, mask, k1[m], k2[m], sh.ol[i], sh.cnt[i], used, err);
+    if (clear) { sh.k1[i] = 0; sh.k2[i] = 0; sh.cnt[i] = 0; }
+  }
 }
 
 
@@ -240,23 +269,7 @@ __global__ void __launch_bounds__(kWcBlock) k_wc(Chunk c, const uint8_t* __restr
   }
   __syncthreads();
   // flush the block table: all of this thread's home-slot reads in flight at once, then adds
-  constexpr int kPer = kWcTab / kWcBlock;
-  unsigned long long k1[kPer], k2[kPer];
-  ulonglong2 home[kPer];
-#pragma unroll
-  for (int m = 0; m < kPer; ++m) {
-    const int i = threadIdx.x + m * kWcBlock;
-    k1[m] = sh.k1[i];
-    k2[m] = sh.k2[i];
-    home[m] = k1[m] ? __ldcg(reinterpret_cast<const ulonglong2*>(&table[k1[m] & mask])) : make_ulonglong2(0, 0);
-  }
-#pragma unroll
-  for (int m = 0; m < kPer; ++m) {
-    const int i = threadIdx.x + m * kWcBlock;
-    if (!k1[m]) continue;
-    if (wc_home_hit(home[m], k1[m], k2[m])) atomicAdd(&table[k1[m] & mask].count, (unsigned long long)sh.cnt[i]);
-    else wc_insert(table, mask, k1[m], k2[m], sh.ol[i], sh.cnt[i], used, err);
-  }
+  wc_flush_block<WcShared, kWcTab / kWcBlock>(sh, threadIdx.x, kWcBlock, table, mask, used, err, false);
 }
 
 // The paper's double-buffering baseline for word count (variant iv): the
@@ -322,165 +335,213 @@ __global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, 
 
 // ------------------------------------------------------------------------------------------
 // C1 word count as ONE persistent launch: BigKernel's single kernel ("a single kernel
-// invocation"; Fig. 3 P:588-660 one block runs address generation and computation, the stages
-// overlapped across buffer instances), on sm_100a:
-//   * each CTA streams whole units (<= UB bytes / UR records of whole records, planned on the host
-//     once per registration, a1) through an S-stage shared-memory ring — the device working set
-//     is grid x S x stage <= window_bytes;
-//   * stage 1 (address generation): per unit, the record offsets (read zero-copy with
-//     cp.async) give every lane its contiguous record range by the lane rule (A4) and the byte
-//     range to fetch;
-//   * stages 2+3 (assembly + transfer): cp.async 16-B copies of exactly the unit's bytes
-//     from pinned, mapped host memory into shared memory, coalesced (512 B per warp instruction),
-//     issued S-1 units ahead so the PCIe reads of later units are in flight while this unit
-//     computes (the paper's n-3 buffer distance, as cp.async groups);
-//   * stage 4: each thread tokenises its lane from shared memory, words go through the
-//     warp queue / block hot-word table / global table of k_wc (same identities).
-// The ring replaces the per-chunk launch chain of the event pipeline (~5 launches per chunk at the
-// 8 MiB window's 0.4 MB chunks, profiles/r01_wc_sweep.md); the only per-unit synchronisation is
-// two CTA barriers (the paper's bar.red).
-constexpr int kFuThreads = 128;   // = kWcBlock: the WcShared queues are per warp of this block size
-constexpr int kFuStages = 3;
-
-__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
-  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
-  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(d), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+// invocation"; Fig. 3: inside one launch, address-generation threads and compute threads
+// are specialised and synchronise through flags, the buffers ring across iterations, P:546-561,
+// P:790-860), specialised per CTA on sm_100a:
+//   * LOADER CTAs (stages 1-3): per unit of whole records (planned on the host once per
+//     registration, a1), copy the unit's record offsets and exactly its bytes from pinned, mapped
+//     host memory (zero-copy, coalesced 16-B loads, every byte once) into a ring slot in HBM, then
+//     publish the slot (release flag) — the paper's signal_dataReady;
+//   * CONSUMER CTAs (stage 4): wait for a unit's flag (acquire), copy the slot into shared memory,
+//     release the slot (the loader of unit u+R may refill it), derive each thread's byte range and
+//     record boundaries from the offsets (stage 1's lane plan), tokenise and count (warp queue ->
+//     block hot-word table -> global table, identities as k_wc).
+// Why split by CTA (= by SM, one CTA per SM): an SM's global loads queue behind its own
+// outstanding PCIe reads, which drain at that SM's share of the link (~0.35 GB/s): with zero-copy
+// traffic in flight a hash-table load took tens of microseconds (ncu, r02c: 36% of warp samples on
+// one unit-metadata load). Loader SMs only stream; consumer SMs never touch host memory.
+// The HBM ring (R slots, R x slot <= window_bytes) is the device working set; ring order and the
+// n - R reuse distance follow the paper's buffer-instance rule. Every spin has a
+// %globaltimer limit (error flag instead of a hang).
+constexpr int kFuThreads = 512;
+constexpr int kFuQ = 64;          // per-warp word queue (8 warps share the block)
+using FuShared = WcSharedT<kFuThreads / 32, kFuQ>;
+constexpr size_t kFuSmemForce = 120 * 1024;   // dynamic smem >= half an SM: one CTA per SM
 
 struct FusedArgs {
   const uint8_t* data;        // device alias of the registered (mapped) data set
   uint64_t nbytes;
   const uint64_t* off;        // device alias of the mapped offsets, nullptr: fixed records
   uint64_t rec_size;
-  uint64_t n;
   const uint64_t* ub;         // unit record bounds (U + 1), device
   const uint64_t* uby;        // unit byte bounds (U + 1), device
   uint32_t U, UB, UR;         // units; bytes / records per unit (caps)
-  uint32_t stage_bytes;       // shared-memory bytes of one ring stage
-  unsigned long long* next;   // unit claim counter (zeroed by the run)
+  uint32_t n_load;            // loader CTAs (blockIdx < n_load); the rest consume
+  uint8_t* ring;              // R slots of slot_bytes: [UB + 32 text][UR x 8 offsets]
+  uint32_t R, slot_bytes;
+  unsigned long long* ready;  // R: unit + 1 whose bytes the slot holds (zeroed by the run)
+  unsigned long long* done;   // R: unit + 1 the slot was last consumed for (zeroed by the run)
   WcEntry* table;
   uint64_t mask;
   unsigned long long* used;
   int* err;
-  unsigned long long* prof;   // optional: [0] wait cycles, [1] compute cycles, [2] CTA cycles (summed)
+  unsigned long long* prof;   // optional: [0] consumer wait ns, [1] consumer compute ns, [2] consumer ns,
+                              //           [3] loader wait ns, [4] loader copy ns
 };
 
-__global__ void __launch_bounds__(kFuThreads) k_wc_fused(FusedArgs a) {
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+constexpr unsigned long long kSpinLimitNs = 2000000000ull;   // 2 s: a stuck pipeline reports, never hangs
+
+__global__ void __launch_bounds__(kFuThreads, 1) k_wc_fused(FusedArgs a) {
   extern __shared__ __align__(128) unsigned char fu_smem[];
-  __shared__ WcShared sh;
-  __shared__ uint32_t s_unit[kFuStages];
+  __shared__ FuShared sh;
+  __shared__ int s_abort;
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (tid == 0) s_abort = 0;
+  __syncthreads();
+  const unsigned long long t_start = gtime();
+  if (blockIdx.x < a.n_load) {
+    // ------------------------------------------------------------ loader: stages 1-3
+    unsigned long long t_wait = 0;
+    for (uint32_t u = blockIdx.x; u < a.U; u += a.n_load) {
+      const uint32_t sl = u % a.R;
+      const unsigned long long tw = gtime();
+      if (tid == 0 && u >= a.R) {   // the slot's previous unit (u - R) must have been copied out
+        while (ld_acquire(&a.done[sl]) < u - a.R + 1)
+          if (gtime() - tw > kSpinLimitNs) { atomicOr(a.err, kErrFusedTimeout); s_abort = 1; break; }
+      }
+      __syncthreads();
+      if (s_abort) break;
+      t_wait += gtime() - tw;
+      uint8_t* slot = a.ring + (size_t)sl * a.slot_bytes;
+      const uint64_t lo = a.ub[u], hi = a.ub[u + 1];
+      const uint64_t b0 = a.uby[u], b1 = a.uby[u + 1];
+      if (a.off) {
+        uint64_t* o = reinterpret_cast<uint64_t*>(slot + a.UB + 32);
+        for (uint64_t j = tid; j < hi - lo; j += blockDim.x) o[j] = __ldcs(a.off + lo + j);
+      }
+      const uintptr_t first = ((uintptr_t)(a.data + b0)) & ~(uintptr_t)15;
+      const uintptr_t last = ((uintptr_t)(a.data + b1) + 15) & ~(uintptr_t)15;
+      const uintptr_t dlo = (uintptr_t)a.data, dhi = (uintptr_t)(a.data + a.nbytes);
+      const uint32_t nw = (uint32_t)((last - first) >> 4);
+      // 4 independent 16-B host loads per thread in flight, then their stores
+      for (uint32_t k0 = tid; k0 < nw; k0 += 4 * blockDim.x) {
+        uint4 v[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t k = k0 + q * blockDim.x;
+          const uintptr_t p = first + 16 * (uintptr_t)k;
+          v[q] = make_uint4(0, 0, 0, 0);
+          if (k < nw) {
+            if (p >= dlo && p + 16 <= dhi) {
+              v[q] = __ldcs(reinterpret_cast<const uint4*>(p));
+            } else {   // a word straddling the data set's edge: only its in-range bytes are read
+              uint32_t ww[4] = {0, 0, 0, 0};
+              for (int z = 0; z < 16; ++z)
+                if (p + z >= dlo && p + z < dhi) ww[z >> 2] |= (uint32_t)*reinterpret_cast<const uint8_t*>(p + z) << (8 * (z & 3));
+              v[q] = make_uint4(ww[0], ww[1], ww[2], ww[3]);
+            }
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t k = k0 + q * blockDim.x;
+          if (k < nw) __stcg(reinterpret_cast<uint4*>(slot) + k, v[q]);
+        }
+      }
+      __threadfence();
+      __syncthreads();
+      if (tid == 0) st_release(&a.ready[sl], (unsigned long long)u + 1);
+    }
+    if (a.prof && tid == 0) {
+      atomicAdd(&a.prof[3], t_wait);
+      atomicAdd(&a.prof[4], gtime() - t_start - t_wait);
+    }
+    return;
+  }
+  // -------------------------------------------------------------- consumer: stage 4
+  const uint32_t nc = gridDim.x - a.n_load, ci = blockIdx.x - a.n_load;
   const unsigned lt = (1u << lane) - 1;
   for (int i = tid; i < kWcTab; i += blockDim.x) { sh.k1[i] = 0; sh.k2[i] = 0; sh.cnt[i] = 0; }
-  const long long t_start = clock64();
-  long long t_wait = 0, t_comp = 0;
-  const uint32_t none = 0xffffffffu;
-  auto txt_of = [&](int st) { return fu_smem + (size_t)st * a.stage_bytes; };
-  auto offs_of = [&](int st) { return reinterpret_cast<uint64_t*>(fu_smem + (size_t)st * a.stage_bytes + a.UB + 32); };
-  // stages 1-3 of unit u into ring stage st: offsets slice + the unit's bytes, cp.async
-  auto prefetch = [&](int st, uint32_t u) {
-    if (u == none) return;
-    const uint64_t lo = a.ub[u], hi = a.ub[u + 1];
-    const uint64_t b0 = a.uby[u], b1 = a.uby[u + 1];
-    if (a.off) {
-      uint64_t* o = offs_of(st);
-      for (uint64_t j = tid; j < hi - lo; j += blockDim.x) cp_async8(o + j, a.off + lo + j);
+  uint8_t* txt_s = fu_smem;                                                   // UB + 32 bytes
+  uint64_t* offs = reinterpret_cast<uint64_t*>(fu_smem + a.UB + 32);          // UR entries
+  unsigned long long t_wait = 0, t_comp = 0;
+  for (uint32_t u = ci; u < a.U; u += nc) {
+    const uint32_t sl = u % a.R;
+    const unsigned long long tw = gtime();
+    if (tid == 0) {
+      while (ld_acquire(&a.ready[sl]) != (unsigned long long)u + 1)
+        if (gtime() - tw > kSpinLimitNs) { atomicOr(a.err, kErrFusedTimeout); s_abort = 1; break; }
     }
-    const uintptr_t first = ((uintptr_t)(a.data + b0)) & ~(uintptr_t)15;
-    const uintptr_t last = ((uintptr_t)(a.data + b1) + 15) & ~(uintptr_t)15;
-    const uintptr_t dlo = (uintptr_t)a.data, dhi = (uintptr_t)(a.data + a.nbytes);
-    uint8_t* t = txt_of(st);
-    for (uintptr_t p = first + 16 * (uintptr_t)tid; p < last; p += 16 * (uintptr_t)blockDim.x) {
-      uint8_t* d = t + (p - first);
-      if (p >= dlo && p + 16 <= dhi) {
-        cp_async16(d, reinterpret_cast<const void*>(p));
-      } else {   // a word straddling the data set's edge: only its in-range bytes are read
-        for (int q = 0; q < 16; ++q) d[q] = (p + q >= dlo && p + q < dhi) ? *reinterpret_cast<const uint8_t*>(p + q) : 0;
+    __syncthreads();
+    if (s_abort) break;
+    const unsigned long long t1 = gtime();
+    t_wait += t1 - tw;
+    const uint64_t lo = a.ub[u], hi = a.ub[u + 1];
+    const uint64_t base = a.uby[u];
+    const uint32_t nrec = (uint32_t)(hi - lo), A = (uint32_t)(a.uby[u + 1] - base);
+    const uint8_t* slot = a.ring + (size_t)sl * a.slot_bytes;
+    {   // slot -> shared memory (L2 reads: the flag's acquire orders them; .cg bypasses stale L1 lines)
+      const uint32_t sh0 = (uint32_t)(((uintptr_t)(a.data + base)) & 15);
+      const uint32_t nw = (sh0 + A + 15) >> 4;
+      for (uint32_t k = tid; k < nw; k += blockDim.x)
+        reinterpret_cast<uint4*>(txt_s)[k] = __ldcg(reinterpret_cast<const uint4*>(slot) + k);
+      if (a.off) {
+        const uint64_t* so = reinterpret_cast<const uint64_t*>(slot + a.UB + 32);
+        for (uint32_t j = tid; j < nrec; j += blockDim.x) offs[j] = __ldcg(so + j);
       }
     }
-  };
-  auto claim = [&](int st) {
-    if (tid == 0) {
-      const unsigned long long u = atomicAdd(a.next, 1ull);
-      s_unit[st] = u < a.U ? (uint32_t)u : none;
-    }
-  };
-  // fill the ring: S-1 units in flight before the first compute
-  for (int st = 0; st < kFuStages - 1; ++st) claim(st);
-  __syncthreads();
-  for (int st = 0; st < kFuStages - 1; ++st) {
-    prefetch(st, s_unit[st]);
-    cp_async_commit();
-  }
-  int qn = 0;
-  for (uint32_t it = 0;; ++it) {
-    const int cur = (int)(it % kFuStages), nxt = (int)((it + kFuStages - 1) % kFuStages);
-    const long long t0 = clock64();
-    claim(nxt);
-    __syncthreads();   // (a) everyone left the compute of unit it-1 (stage nxt is free), the claim is visible
-    prefetch(nxt, s_unit[nxt]);
-    cp_async_commit();
-    cp_async_wait<kFuStages - 1>();   // this thread's copies of unit `it` landed
-    __syncthreads();   // (b) ... and every thread's
-    const long long t1 = clock64();
-    t_wait += t1 - t0;
-    const uint32_t u = s_unit[cur];
-    if (u == none) break;
-    // ---- stage 1 (lane plan) + stage 4 (tokenise, count) of unit u
-    const uint64_t lo = a.ub[u], hi = a.ub[u + 1];
-    const uint64_t base = a.uby[u], end = a.uby[u + 1];
-    const uint32_t nrec = (uint32_t)(hi - lo), A = (uint32_t)(end - base);
-    const uint8_t* txt = txt_of(cur) + (((uintptr_t)(a.data + base)) & 15);
-    const uint64_t* offs = offs_of(cur);
+    __syncthreads();
+    if (tid == 0) st_release(&a.done[sl], (unsigned long long)u + 1);   // slot free for unit u + R
+    // ---- stage 1 (this thread's range) + stage 4. The unit's bytes are split evenly over the
+    // CTA's threads (parallel tokenisation): thread t owns the words that START in [x0, x1),
+    // finishes its last word past x1 and skips a word running into x0 (thread t-1's). Record starts
+    // are delimiters (A10/A19): the first one after x0 by binary search over the unit's offsets.
+    const uint8_t* txt = txt_s + (((uintptr_t)(a.data + base)) & 15);
     auto rpos = [&](uint32_t j) -> uint32_t {   // start of record lo+j relative to the unit (j <= nrec)
       if (j >= nrec) return A;
       return a.off ? (uint32_t)(offs[j] - base) : (uint32_t)((lo + j) * a.rec_size - base);
     };
-    const uint32_t L = blockDim.x;
-    // first(t) = min{ j : rpos(j) >= floor(t*A/L) } (the lane rule, A4), by binary search in smem
-    auto first_of = [&](uint32_t t) -> uint32_t {
-      if (t >= L) return nrec;
-      const uint32_t target = (uint32_t)(((uint64_t)t * A) / L);
-      uint32_t l = 0, h = nrec;
+    const uint32_t T = blockDim.x;
+    const uint32_t x0 = (uint32_t)(((uint64_t)tid * A) / T), x1 = (uint32_t)(((uint64_t)(tid + 1) * A) / T);
+    uint32_t j;   // first record index with rpos(j) > x0 (j in [1, nrec]; rpos(nrec) = A)
+    {
+      uint32_t l = 1, h = nrec;
       while (l < h) {
         const uint32_t m = (l + h) >> 1;
-        if (rpos(m) >= target) h = m; else l = m + 1;
+        if (rpos(m) > x0) h = m; else l = m + 1;
       }
-      return l;
-    };
-    const uint32_t f0 = first_of(tid), f1 = first_of(tid + 1);
-    const uint32_t x0 = rpos(f0), x1 = rpos(f1);
-    uint32_t j = f0 + 1;
-    uint32_t next_b = j <= f1 ? rpos(j) : 0xffffffffu;
-    const uint32_t steps = x1 - x0 + 1;   // the last step (p == x1) is the lane's closing boundary
-    uint32_t wsteps = steps;
-#pragma unroll
-    for (int o = 16; o; o >>= 1) wsteps = max(wsteps, __shfl_xor_sync(kFull, wsteps, o));
+      j = l;
+    }
+    const bool at_boundary = x0 == 0 || rpos(j - 1) == x0;
+    uint32_t next_b = j <= nrec ? rpos(j) : 0xffffffffu;
+    bool skip = x0 < A && !at_boundary && !is_delim(txt[x0 - 1]);
     bool in_word = false;
     uint64_t h1 = 0, h2 = 0;
     uint32_t wstart = 0, wlen = 0;
-    for (uint32_t k = 0; k < wsteps; ++k) {
-      const uint32_t p = x0 + k;
-      const bool valid = k < steps;
-      bool boundary = valid && p == x1;
-      if (valid && p == next_b) {
-        boundary = true;
-        do {   // several records may start here if some are empty
-          ++j;
-          next_b = j <= f1 ? rpos(j) : 0xffffffffu;
-        } while (next_b == p);
+    uint32_t p = x0;
+    bool go = x0 < x1;
+    int qn = 0;   // warp-uniform queue fill
+    while (__any_sync(kFull, go)) {
+      bool end = false, delim = true;
+      uint32_t ch = 0x20u;
+      if (go) {
+        bool boundary = false;
+        if (p == next_b) {
+          boundary = true;
+          do {   // several records may start here if some are empty
+            ++j;
+            next_b = j <= nrec ? rpos(j) : 0xffffffffu;
+          } while (next_b == p);
+        }
+        if (p < A) ch = txt[p];
+        delim = p >= A || is_delim(ch);
+        if (boundary || delim) skip = false;
+        end = in_word && (boundary || delim);
       }
-      const uint32_t ch = (valid && p < x1) ? txt[p] : 0x20u;
-      const bool delim = is_delim(ch);
-      const bool end = valid && in_word && (boundary || delim);
-      const unsigned m = __ballot_sync(kFull, end);
+      const unsigned m = __ballot_sync(kFull, end);   // the ended words go to the warp queue
       if (m) {
         if (end) {
           const uint64_t occ = base + wstart;
@@ -491,47 +552,36 @@ __global__ void __launch_bounds__(kFuThreads) k_wc_fused(FusedArgs a) {
           sh.qol[w][i] = (occ << 24) | wlen;
         }
         qn += __popc(m);
-        if (qn > kWcQ - 32) {
+        if (qn > kFuQ - 32) {
           wc_flush_queue(sh, w, lane, qn, a.table, a.mask, a.used, a.err);
           qn = 0;
         }
       }
-      if (end) in_word = false;
-      if (valid && p < x1 && !delim) {
-        if (!in_word) { in_word = true; wstart = p; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
-        h1 = (h1 ^ ch) * 0x100000001b3ull;
-        h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
-        h2 ^= h2 >> 29;
-        ++wlen;
+      if (go) {
+        if (end) in_word = false;
+        if (!delim && !skip && (in_word || p < x1)) {
+          if (!in_word) { in_word = true; wstart = p; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
+          h1 = (h1 ^ ch) * 0x100000001b3ull;
+          h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
+          h2 ^= h2 >> 29;
+          ++wlen;
+        }
+        ++p;
+        go = p <= A && (p < x1 || in_word);
       }
     }
-    t_comp += clock64() - t1;
-  }
-  cp_async_wait<0>();
-  if (qn) wc_flush_queue(sh, w, lane, qn, a.table, a.mask, a.used, a.err);
-  __syncthreads();
-  // flush the block table (as k_wc)
-  constexpr int kPer = kWcTab / kFuThreads;
-  unsigned long long k1[kPer], k2[kPer];
-  ulonglong2 home[kPer];
-#pragma unroll
-  for (int m = 0; m < kPer; ++m) {
-    const int i = tid + m * kFuThreads;
-    k1[m] = sh.k1[i];
-    k2[m] = sh.k2[i];
-    home[m] = k1[m] ? __ldcg(reinterpret_cast<const ulonglong2*>(&a.table[k1[m] & a.mask])) : make_ulonglong2(0, 0);
-  }
-#pragma unroll
-  for (int m = 0; m < kPer; ++m) {
-    const int i = tid + m * kFuThreads;
-    if (!k1[m]) continue;
-    if (wc_home_hit(home[m], k1[m], k2[m])) atomicAdd(&a.table[k1[m] & a.mask].count, (unsigned long long)sh.cnt[i]);
-    else wc_insert(a.table, a.mask, k1[m], k2[m], sh.ol[i], sh.cnt[i], a.used, a.err);
+    if (qn) wc_flush_queue(sh, w, lane, qn, a.table, a.mask, a.used, a.err);
+    // the block table caches this unit's hot words; empty it into the global table before the next
+    // unit (a table kept across units would fill with early words and send the hot ones global)
+    __syncthreads();
+    wc_flush_block<FuShared, kWcTab / kFuThreads>(sh, tid, kFuThreads, a.table, a.mask, a.used, a.err, true);
+    __syncthreads();
+    t_comp += gtime() - t1;
   }
   if (a.prof && tid == 0) {
-    atomicAdd(&a.prof[0], (unsigned long long)t_wait);
-    atomicAdd(&a.prof[1], (unsigned long long)t_comp);
-    atomicAdd(&a.prof[2], (unsigned long long)(clock64() - t_start));
+    atomicAdd(&a.prof[0], t_wait);
+    atomicAdd(&a.prof[1], t_comp);
+    atomicAdd(&a.prof[2], gtime() - t_start);
   }
 }
 
@@ -909,28 +959,35 @@ void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, cons
   k_wc<kSub><<<grid, kWcBlock, 0, s>>>(c, stage, lanes, tile_base, meta, rec_size, table, mask, used, err);
 }
 
-uint32_t wc_fused_stage_bytes(uint32_t UB, uint32_t UR) { return (UB + 32 + (UR + 1) * 8 + 127) / 128 * 128; }
+uint32_t wc_fused_slot_bytes(uint32_t UB, uint32_t UR) { return (UB + 32 + UR * 8 + 255) / 256 * 256; }
 
-int wc_fused_grid(uint32_t stage_bytes) {
-  int per = 0;
-  const size_t dyn = (size_t)kFuStages * stage_bytes;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_wc_fused, kFuThreads, dyn) != cudaSuccess || per < 1) {
-    cudaGetLastError();
-    per = 1;
-  }
-  return device_sms() * std::min(per, 2);
+size_t wc_fused_smem(uint32_t UB, uint32_t UR) {
+  return std::max<size_t>(kFuSmemForce, (size_t)UB + 32 + (size_t)UR * 8);
 }
 
-void launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t* off, uint64_t rec_size, uint64_t n,
-                     const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
-                     unsigned long long* next, WcEntry* table, uint64_t mask, unsigned long long* used, int* err,
-                     unsigned long long* prof, cudaStream_t s) {
-  FusedArgs a{data, nbytes, off, rec_size, n, ub, uby, U, UB, UR, wc_fused_stage_bytes(UB, UR), next, table, mask,
-              used, err, prof};
-  k_wc_fused<<<grid, kFuThreads, (size_t)kFuStages * a.stage_bytes, s>>>(a);
+int wc_fused_grid() { return device_sms(); }
+
+cudaError_t launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t* off, uint64_t rec_size,
+                            const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
+                            uint32_t n_load, uint8_t* ring, uint32_t R, unsigned long long* ready,
+                            unsigned long long* done, WcEntry* table, uint64_t mask, unsigned long long* used,
+                            int* err, unsigned long long* prof, cudaStream_t s) {
+  FusedArgs a{data, nbytes, off, rec_size, ub, uby, U, UB, UR, n_load, ring, R, wc_fused_slot_bytes(UB, UR),
+              ready, done, table, mask, used, err, prof};
+  // cooperative: every CTA is co-resident (loaders and consumers wait on each other)
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kFuThreads);
+  cfg.dynamicSmemBytes = wc_fused_smem(UB, UR);
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k_wc_fused, a);
 }
 
-int wc_fused_stages() { return kFuStages; }
 uint32_t wc_fused_threads() { return kFuThreads; }
 
 void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
@@ -1004,8 +1061,13 @@ void launch_kmeans(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, 
 }
 
 cudaError_t configure_compute_kernels() {
+  {   // the fused word count also holds its static FuShared tables: dynamic ring <= 227 KB - static
+    const cudaError_t e = cudaFuncSetAttribute((const void*)k_wc_fused, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                               227 * 1024 - (int)sizeof(FuShared) - 2048);
+    if (e != cudaSuccess) return e;
+  }
   for (const void* f : {(const void*)k_groupby<true>, (const void*)k_groupby<false>, (const void*)k_kmeans<true>,
-                        (const void*)k_kmeans<false>, (const void*)k_grep_count<true>, (const void*)k_wc_fused}) {
+                        (const void*)k_kmeans<false>, (const void*)k_grep_count<true>}) {
     const cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
     if (e != cudaSuccess) return e;
   }

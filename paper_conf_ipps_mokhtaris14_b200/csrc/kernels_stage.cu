@@ -429,6 +429,11 @@ void launch_addrgen(const Chunk& c, const Access& a, const uint64_t* meta, LaneD
   k_tile_scan<<<1, 1024, 0, s>>>(tileK, c.ntiles, tile_base, stage_cap, err, staged_sum);
 }
 
+void launch_tile_scan(const uint32_t* tileK, uint32_t ntiles, uint64_t* tile_base, uint64_t stage_cap, int* err,
+                      unsigned long long* staged_sum, cudaStream_t s) {
+  k_tile_scan<<<1, 1024, 0, s>>>(tileK, ntiles, tile_base, stage_cap, err, staged_sum);
+}
+
 template <bool kHost>
 static void gather_impl(const Chunk& c, const Access& a, const uint8_t* src, const uint64_t* meta,
                         const LaneDesc* lanes, const uint64_t* tile_base, uint8_t* stage, uint64_t cap,

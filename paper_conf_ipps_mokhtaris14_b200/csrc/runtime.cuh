@@ -59,6 +59,14 @@ struct Slot {
   uint32_t* tileK = nullptr;
   uint64_t* tile_base = nullptr;
   uint8_t* out = nullptr;       // per-chunk output (partition: the bucket-sorted chunk)
+  // BK_GATHER_ADDR: explicit addresses (device staging), per-lane explicit counts and their scan;
+  // bk_run_user_addr: the generator's address buffer, per-lane bases and counts
+  uint64_t* exp = nullptr;
+  uint32_t* ecount = nullptr;
+  uint64_t* epos = nullptr;
+  uint64_t* uaddr = nullptr;
+  uint64_t* ubase = nullptr;
+  uint32_t* ucount = nullptr;
   // descriptor sets (meta, lanes, tileK, tile_base); ZC plans keep two so that stage 1 of chunk
   // i+N can run while chunk i still computes from the other set. meta..tile_base above point at
   // the set of the chunk being issued.
@@ -102,6 +110,9 @@ struct Plan {
   uint64_t stage_cap = 0, raw_cap = 0, meta_cap = 0, out_cap = 0;
   uint32_t desc_sets = 1;              // descriptor sets per slot (2: ZC, stage 1 runs a chunk ahead)
   bool packed = false;                 // CPU chunks: host packs records' bytes, GPU interleaves (raw slot)
+  uint32_t elem = 0;                   // BK_GATHER_ADDR: bytes per element address
+  uint64_t exp_cap = 0;                // BK_GATHER_ADDR: bytes of one chunk's addresses (8 per element)
+  bool user_addr = false;              // bk_run_user_addr: the caller's generator writes the addresses
   std::vector<uint64_t> bounds;        // chunk record bounds
   std::string key;                     // plan-cache key (also part of the graph key)
 };
@@ -163,9 +174,20 @@ struct bk_ctx {  // the opaque context of include/bk.h
   bk::rt::DevBuf b_hist, b_colpre, b_totals, b_base;
   bk::rt::DevBuf b_h1, b_h2;                 // word-count key hashes (multi-GPU merge keys)
   bk::rt::DevBuf b_units;                    // BK_GATHER_FUSED unit plan (record bounds, byte bounds)
+  bk::rt::DevBuf b_flags;                    //   ring ready / done flags
   std::string units_key;                     //   which plan b_units holds
   uint64_t n_units = 0;
-  unsigned long long* d_fprof = nullptr;     //   in-kernel wait / compute cycle counters (3 x u64)
+  unsigned long long* d_fprof = nullptr;     //   in-kernel wait / compute counters
+  // BK_GATHER_ADDR: per slot, pinned + mapped host memory the GPU writes the address information to
+  // (the paper's CPU-side addrBuf), and the host's view of the chunk's tiles
+  std::vector<bk::AddrDesc*> a_desc_h, a_desc_d;
+  std::vector<uint64_t*> a_exp_h, a_exp_d, a_tot_h, a_tot_d;
+  uint64_t a_exp_cap = 0, a_L = 0;
+  std::vector<cudaEvent_t> a_ready;          // per slot: stage 1 (addresses) of its chunk finished
+  size_t addr_next = 0;                      // next chunk whose stage 1 is not yet issued
+  std::vector<uint64_t> a_epos, a_tbase;
+  bk_addr_fn a_gen = nullptr;                // bk_run_user_addr generator + its argument
+  void* a_gen_user = nullptr;
   bk::rt::DevBuf b_mown, b_mcnt, b_mctr;     // bk_merge_counts scratch (never captured in a graph)
   std::vector<std::pair<void*, uint64_t>> out_pinned;      // caller output arrays pinned across runs (opt-in)
   std::vector<std::pair<void*, uint64_t>> out_pinned_run;  // caller output arrays pinned for this run only
@@ -188,7 +210,7 @@ bool is_pinned(const void* p);
 uint64_t rec_start(const bk_ctx* c, uint64_t r);
 int make_chunks(const bk_ctx* c, Plan& p);
 int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t out_per_chunk = 0,
-             int auto_mode = BK_GATHER_AUTO);
+             int auto_mode = BK_GATHER_AUTO, bool user_addr = false);
 void carve(bk_ctx* c, const Plan& p);
 Chunk chunk_of(const bk_ctx* c, const Plan& p, size_t i);
 Access whole_access();
@@ -205,6 +227,9 @@ uint64_t test_rand(bk_ctx* c);
     if (c->cfg.flags & BK_FLAG_TEST_DELAYS) launch_spin((long long)(::bk::rt::test_rand(c) % 200000), stream); \
   } while (0)
 int ensure_host_side(bk_ctx* c, const Plan& p);
+int ensure_addr_side(bk_ctx* c, const Plan& p);
+int stage_chunk_addr(bk_ctx* c, const Plan& p, size_t i, Slot& s);
+void release_addr_side(bk_ctx* c);
 int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s);
 int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s);
 void note_plan(bk_ctx* c, const Plan& p);
@@ -249,10 +274,12 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
   note_plan(c, p);
   std::vector<cudaEvent_t> zc_inflight;
   const size_t zc_depth = std::max<size_t>(1, (c->cfg.n_slots - 1) / 2);
-  if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
+  if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID || p.mode == BK_GATHER_ADDR) {
     int rc = ensure_host_side(c, p);
+    if (!rc && p.mode == BK_GATHER_ADDR) rc = ensure_addr_side(c, p);
     if (rc) return rc;
   }
+  c->addr_next = 0;
   for (size_t i = 0; i < C; ++i) {
     Slot& s = c->slots[i % c->cfg.n_slots];
     cudaStream_t cs = concurrent ? c->s_slot[i % c->cfg.n_slots] : c->s_comp;
@@ -272,8 +299,9 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
     }
     int rc;
     {
-      NvtxRange r("chunk %zu %s", i, cpu ? "cpu" : p.zero_copy ? "zc" : "dense");
-      rc = cpu ? stage_chunk_cpu(c, p, i, s) : stage_chunk(c, p, i, s);
+      NvtxRange r("chunk %zu %s", i, p.mode == BK_GATHER_ADDR ? "addr" : cpu ? "cpu" : p.zero_copy ? "zc" : "dense");
+      rc = p.mode == BK_GATHER_ADDR ? stage_chunk_addr(c, p, i, s) : cpu ? stage_chunk_cpu(c, p, i, s)
+                                                                          : stage_chunk(c, p, i, s);
     }
     if (rc) return rc;
     if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(s.ready);
@@ -373,6 +401,8 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream);
 int run_pattern(bk_ctx* c, bk_out_pattern* o, void* stream);
 int run_layout(bk_ctx* c, bk_out_layout* o, void* stream);
 int run_user(bk_ctx* c, const bk_access* a, bk_chunk_fn fn, void* user, void* stream);
+int run_user_addr(bk_ctx* c, const bk_access* a, bk_addr_fn gen, void* gen_user, bk_chunk_fn fn, void* user,
+                  void* stream);
 
 }  // namespace rt
 }  // namespace bk

@@ -373,6 +373,27 @@ int bk_unpin_outputs(bk_ctx* c) {
   return BK_OK;
 }
 
+int bk_run_user_addr(bk_ctx* c, const bk_access* a, bk_addr_fn gen, void* gen_user, bk_chunk_fn fn, void* user,
+                     void* stream) {
+  NvtxRange nv("bk_run_user_addr");
+  if (!c || !a || !gen || !fn) return fail(BK_E_INVAL, "NULL argument");
+  if (a->struct_size != sizeof(bk_access)) return fail(BK_E_INVAL, "bk_access size");
+  if (!c->registered) return fail(BK_E_STATE, "bk_run_user_addr before bk_register_segments");
+  if (c->cfg.flags & (BK_FLAG_BASELINE_DBUF | BK_FLAG_BASELINE_SBUF))
+    return fail(BK_E_UNSUPPORTED, "bk_run_user_addr: no double-buffering baseline for user kernels");
+  DeviceGuard dg(c->cfg.device);
+  if (!dg.ok) return fail(BK_E_CUDA, "cudaSetDevice(%d)", c->cfg.device);
+  const auto t0 = std::chrono::steady_clock::now();
+  const int rc = run_user_addr(c, a, gen, gen_user, fn, user, stream);
+  if (rc) {
+    drain(c);
+    return rc;
+  }
+  c->st.kernel_launches = (uint64_t)c->n_launch;
+  c->st.ms_run = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return BK_OK;
+}
+
 int bk_get_stats(const bk_ctx* c, bk_stats* s) {
   if (!c || !s) return fail(BK_E_INVAL, "NULL argument");
   if (s->struct_size != sizeof(bk_stats)) return fail(BK_E_INVAL, "bk_stats size");
@@ -395,11 +416,12 @@ int bk_partition_materialize(const void* out_records, const uint64_t* chunk_coun
 }
 
 int bk_abi_sizes(uint32_t* sizes, int n) {
-  const uint32_t v[12] = {sizeof(bk_config),     sizeof(bk_out_wordcount), sizeof(bk_out_grep),
+  const uint32_t v[13] = {sizeof(bk_config),     sizeof(bk_out_wordcount), sizeof(bk_out_grep),
                           sizeof(bk_out_kmeans), sizeof(bk_out_partition), sizeof(bk_out_groupby),
                           sizeof(bk_out_layout), sizeof(bk_stats),         sizeof(bk_out_pattern),
-                          sizeof(bk_out_kmer),   sizeof(bk_access),        sizeof(bk_chunk_view)};
-  for (int i = 0; i < n && i < 12; ++i) sizes[i] = v[i];
+                          sizeof(bk_out_kmer),   sizeof(bk_access),        sizeof(bk_chunk_view),
+                          sizeof(bk_addr_view)};
+  for (int i = 0; i < n && i < 13; ++i) sizes[i] = v[i];
   return BK_ABI_VERSION;
 }
 
@@ -444,8 +466,9 @@ int bk_destroy(bk_ctx* c) {
   for (auto e : c->ev_part) cudaEventDestroy(e);
   release_run_outputs(c);
   release_kept_outputs(c);
+  release_addr_side(c);
   for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base, &c->b_h1, &c->b_h2, &c->b_mown, &c->b_mcnt,
-                    &c->b_mctr, &c->b_units})
+                    &c->b_mctr, &c->b_units, &c->b_flags})
     b->release();
   for (auto* h : c->hstage) cudaFreeHost(h);
   for (auto e : c->h_done) cudaEventDestroy(e);

@@ -54,23 +54,26 @@ static int fused_units(bk_ctx* c, uint32_t UB, uint32_t UR, std::vector<uint64_t
   return BK_OK;
 }
 
-// Word count as one persistent launch (BK_GATHER_FUSED, kernels_compute.cu k_wc_fused). Returns
-// BK_E_RANGE (nothing enqueued) when a record does not fit a unit: the caller then runs the pipeline.
+// Word count as one persistent launch (BK_GATHER_FUSED, kernels_compute.cu k_wc_fused): loader
+// CTAs stream units into an HBM ring carved from the window, consumer CTAs count. Returns
+// BK_E_RANGE (nothing enqueued) when the window cannot hold a ring of >= 2 units or a record does
+// not fit a unit: the caller then runs the event pipeline.
 static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uint64_t slots, uint64_t ocap) {
-  const int S = wc_fused_stages();
-  // units: as large as 16 KiB allow, but grid x S ring stages never exceed the device window
-  // (a small window keeps units of >= 2 KiB and runs fewer CTAs instead)
-  int grid = wc_fused_grid(wc_fused_stage_bytes(16384, 1024));
-  const uint64_t per_stage = c->cfg.window_bytes / ((uint64_t)grid * S);
-  uint64_t UB = per_stage > 200 ? (per_stage - 200) * 2 / 3 : 0;
-  UB = std::min<uint64_t>(UB, 16384) / 16 * 16;
-  if (UB < 2048) {
-    UB = 2048;
-    grid = (int)std::min<uint64_t>(grid, c->cfg.window_bytes / ((uint64_t)S * wc_fused_stage_bytes(2048, 128)));
-    if (grid < 1) return BK_E_RANGE;
-  }
+  (void)o;
+  const int grid = wc_fused_grid();
+  if (grid < 2) return BK_E_RANGE;
+  uint32_t n_load = (uint32_t)std::max(1, grid / 3);
+  if (const char* e = getenv("BK_FUSED_LOADERS")) n_load = (uint32_t)std::max(1, std::min(grid - 1, atoi(e)));
+  // units as large as 16 KiB allow while the ring keeps >= 2 slots per CTA; >= 2 KiB units and
+  // >= 2 slots in any case (R x slot <= window_bytes)
+  uint64_t UB = c->cfg.window_bytes / (2ull * grid);
+  UB = UB > 64 ? (UB - 64) * 2 / 3 : 0;
+  UB = std::max<uint64_t>(2048, std::min<uint64_t>(UB, 16384)) / 16 * 16;
   const uint32_t UR = (uint32_t)std::max<uint64_t>(UB / 16, 16);
-  const std::string ukey = std::to_string(UB) + "/" + std::to_string(UR) + "/" + std::to_string(grid);
+  const uint64_t slot_bytes = wc_fused_slot_bytes((uint32_t)UB, UR);
+  const uint64_t R = std::min<uint64_t>(c->cfg.window_bytes / slot_bytes, 1u << 20);
+  if (R < 2) return BK_E_RANGE;
+  const std::string ukey = std::to_string(UB) + "/" + std::to_string(UR);
   if (c->units_key != ukey) {
     std::vector<uint64_t> ub, uby;
     if (fused_units(c, (uint32_t)UB, UR, ub, uby)) return BK_E_RANGE;
@@ -80,21 +83,23 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
     BK_CUDA(cudaMemcpy((uint64_t*)c->b_units.p + ub.size(), uby.data(), uby.size() * 8, cudaMemcpyHostToDevice));
     c->units_key = ukey;
   }
-  if (!c->d_fprof) BK_CUDA(cudaMalloc(&c->d_fprof, 4 * 8));
+  if (!c->d_fprof) BK_CUDA(cudaMalloc(&c->d_fprof, 8 * 8));
+  BK_CUDA(c->b_flags.ensure(2 * R * 8));
   const uint64_t U = c->n_units;
   const uint64_t* ubd = (const uint64_t*)c->b_units.p;
+  unsigned long long* ready = (unsigned long long*)c->b_flags.p;
   const bool prof = (c->cfg.flags & BK_FLAG_PROFILE) != 0;
   WcEntry* table = (WcEntry*)c->b_table.p;
-  const std::string key = "wcfused/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + ukey;
-  int rc = run_device(c, stream, key, true, 1, [&]() -> int {
+  // eager issue (three operations): the cooperative launch is not graph-captured
+  int rc = run_device(c, stream, "wcfused", false, 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
-    if (prof) BK_CUDA(cudaMemsetAsync(c->d_fprof, 0, 4 * 8, c->s_comp));
-    c->st.n_chunks = U;
-    c->st.lanes = wc_fused_threads();
+    BK_CUDA(cudaMemsetAsync(ready, 0, 2 * R * 8, c->s_comp));
+    if (prof) BK_CUDA(cudaMemsetAsync(c->d_fprof, 0, 8 * 8, c->s_comp));
     BK_PROF(kStGather, c->s_comp, true);
-    launch_wc_fused(c->host_dev, c->nbytes, c->off ? c->off_dev : nullptr, c->off ? 0 : c->cfg.record_size, c->n,
-                    ubd, ubd + U + 1, (uint32_t)U, (uint32_t)UB, UR, grid, c->d_ctr + 7, table, slots - 1,
-                    c->d_ctr + 1, c->d_err, prof ? c->d_fprof : nullptr, c->s_comp);
+    BK_CUDA(launch_wc_fused(c->host_dev, c->nbytes, c->off ? c->off_dev : nullptr, c->off ? 0 : c->cfg.record_size,
+                            ubd, ubd + U + 1, (uint32_t)U, (uint32_t)UB, UR, grid, n_load, c->window, (uint32_t)R,
+                            ready, ready + R, table, slots - 1, c->d_ctr + 1, c->d_err, prof ? c->d_fprof : nullptr,
+                            c->s_comp));
     BK_PROF(kStGather, c->s_comp, false);
     launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
                       (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p, ocap, c->s_comp);
@@ -115,16 +120,19 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
   c->st.n_units = U;
   c->st.unit_bytes = (uint32_t)UB;
   c->st.fused_grid = (uint32_t)grid;
-  c->st.fused_wait_frac = c->st.fused_compute_frac = 0;
+  c->st.fused_loaders = n_load;
+  c->st.fused_ring_slots = (uint32_t)R;
+  c->st.fused_wait_frac = c->st.fused_compute_frac = c->st.fused_loader_wait_frac = 0;
   if (prof) {
-    unsigned long long fp[3] = {0, 0, 0};
+    unsigned long long fp[5] = {0, 0, 0, 0, 0};
     BK_CUDA(cudaMemcpy(fp, c->d_fprof, sizeof fp, cudaMemcpyDeviceToHost));
     if (fp[2]) {
       c->st.fused_wait_frac = (double)fp[0] / (double)fp[2];
       c->st.fused_compute_frac = (double)fp[1] / (double)fp[2];
     }
-    // the one kernel is stages 1-4: its interval is the transfer interval, its compute share is
-    // the CTAs' compute time (every unit but the last S-1 of a CTA computes while later units fly)
+    if (fp[3] + fp[4]) c->st.fused_loader_wait_frac = (double)fp[3] / (double)(fp[3] + fp[4]);
+    // the one kernel is stages 1-4: its interval is the transfer interval; the consumers' compute
+    // share of it overlaps the loaders' transfers of later units
     c->st.ms_compute_busy = c->st.ms_zc * c->st.fused_compute_frac;
     c->st.ms_compute = c->st.ms_compute_busy;
     c->st.ms_overlap = c->st.ms_compute_busy;
@@ -697,6 +705,43 @@ int run_user(bk_ctx* c, const bk_access* ua, bk_chunk_fn fn, void* user, void* s
   });
 }
 
+// bk_run_user_addr: the caller's generator is stage 1's address slice (address mode), stage 4 its
+// chunk callback. Always eager.
+int run_user_addr(bk_ctx* c, const bk_access* ua, bk_addr_fn gen, void* gen_user, bk_chunk_fn fn, void* user,
+                  void* stream) {
+  if (ua->n_ext > 8) return fail(BK_E_INVAL, "at most 8 extents");
+  Access a;
+  int rc = parse_access(c, ua->n_ext, ua->ext_off, ua->ext_len, a);
+  if (rc) return rc;
+  Plan p;
+  if ((rc = plan_run(c, a, ua->lane_bytes ? ua->lane_bytes : 256, p, 0, BK_GATHER_AUTO, true))) return rc;
+  carve(c, p);
+  c->a_gen = gen;
+  c->a_gen_user = gen_user;
+  const size_t C = p.bounds.size() - 1;
+  return run_device(c, stream, "useraddr", false, C, [&]() -> int {
+    size_t ci = 0;
+    return pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) -> int {
+      bk_chunk_view v{};
+      v.struct_size = sizeof(bk_chunk_view);
+      v.lanes = ch.L;
+      v.chunk_index = ci++;
+      v.n_chunks = C;
+      v.first_record = ch.lo;
+      v.n_records = ch.hi - ch.lo;
+      v.stage = s.stage;
+      v.lane_desc = reinterpret_cast<const bk_lane*>(s.lanes);
+      v.tile_base = s.tile_base;
+      v.offsets = c->off ? s.meta : nullptr;
+      v.end_offset = ch.end_byte;
+      const int r = fn(&v, (void*)cs, user);
+      if (r) return fail(BK_E_INVAL, "user chunk function returned %d for chunk %llu", r,
+                         (unsigned long long)v.chunk_index);
+      return (int)BK_OK;
+    });
+  });
+}
+
 int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
   Access a;
   int rc = parse_access(c, o->n_ext, o->ext_off, o->ext_len, a);
@@ -710,8 +755,13 @@ int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
   if (o->chunk >= o->n_chunks) return fail(BK_E_INVAL, "chunk %llu >= %llu chunks", (unsigned long long)o->chunk,
                                            (unsigned long long)o->n_chunks);
   if ((rc = begin_run(c, stream))) return rc;
-  Slot& s = c->slots[0];
-  if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
+  Slot& s = c->slots[p.mode == BK_GATHER_ADDR ? o->chunk % c->cfg.n_slots : 0];
+  if (p.mode == BK_GATHER_ADDR) {   // stage 1 of exactly this chunk (and the look-ahead one) in its slot
+    if ((rc = ensure_host_side(c, p)) || (rc = ensure_addr_side(c, p))) return rc;
+    c->addr_next = o->chunk;
+    if ((rc = stage_chunk_addr(c, p, o->chunk, s))) return rc;
+    BK_CUDA(cudaStreamSynchronize(c->s_asm));   // the look-ahead chunk's stage 1 too
+  } else if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID) {
     if ((rc = ensure_host_side(c, p))) return rc;
     if ((rc = stage_chunk_cpu(c, p, o->chunk, s))) return rc;
   } else if ((rc = stage_chunk(c, p, o->chunk, s))) {

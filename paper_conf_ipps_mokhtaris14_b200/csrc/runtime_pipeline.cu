@@ -135,6 +135,157 @@ int stage_chunk_cpu(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   return BK_OK;
 }
 
+// ---- BK_GATHER_ADDR: the paper's address-mode stages 1-3 ---------------------------------------
+// per slot: pinned, mapped host buffers for the lane descriptors, the explicit-address count and the
+// explicit addresses (the GPU writes them, the host reads them after the slot's a_ready event)
+void release_addr_side(bk_ctx* c) {
+  for (auto* v : {&c->a_exp_h, &c->a_tot_h})
+    for (auto* h : *v) cudaFreeHost(h);
+  for (auto* h : c->a_desc_h) cudaFreeHost(h);
+  c->a_desc_h.clear();
+  c->a_desc_d.clear();
+  c->a_exp_h.clear();
+  c->a_exp_d.clear();
+  c->a_tot_h.clear();
+  c->a_tot_d.clear();
+  for (auto e : c->a_ready) cudaEventDestroy(e);
+  c->a_ready.clear();
+  c->a_exp_cap = c->a_L = 0;
+}
+
+int ensure_addr_side(bk_ctx* c, const Plan& p) {
+  const size_t N = c->cfg.n_slots;
+  if (c->a_desc_h.size() == N && c->a_L >= p.L && c->a_exp_cap >= p.exp_cap) return BK_OK;
+  release_addr_side(c);
+  const unsigned fl = cudaHostAllocMapped | cudaHostAllocPortable;
+  c->a_desc_h.assign(N, nullptr);
+  c->a_desc_d.assign(N, nullptr);
+  c->a_exp_h.assign(N, nullptr);
+  c->a_exp_d.assign(N, nullptr);
+  c->a_tot_h.assign(N, nullptr);
+  c->a_tot_d.assign(N, nullptr);
+  c->a_ready.assign(N, nullptr);
+  for (size_t k = 0; k < N; ++k) {
+    BK_CUDA(cudaHostAlloc((void**)&c->a_desc_h[k], (size_t)p.L * sizeof(AddrDesc), fl));
+    BK_CUDA(cudaHostAlloc((void**)&c->a_exp_h[k], std::max<uint64_t>(p.exp_cap, 64), fl));
+    BK_CUDA(cudaHostAlloc((void**)&c->a_tot_h[k], 64, fl));
+    BK_CUDA(cudaHostGetDevicePointer((void**)&c->a_desc_d[k], c->a_desc_h[k], 0));
+    BK_CUDA(cudaHostGetDevicePointer((void**)&c->a_exp_d[k], c->a_exp_h[k], 0));
+    BK_CUDA(cudaHostGetDevicePointer((void**)&c->a_tot_d[k], c->a_tot_h[k], 0));
+    BK_CUDA(cudaEventCreateWithFlags(&c->a_ready[k], cudaEventDisableTiming));
+  }
+  c->a_L = p.L;
+  c->a_exp_cap = p.exp_cap;
+  return BK_OK;
+}
+
+// Stage 1 of chunk i on the GPU (s_asm): lane plan, then every lane's element addresses (from the
+// access spec, or the caller's generator), pattern recognition, descriptors + explicit addresses into
+// the slot's pinned host buffers; a_ready[slot] marks them complete (P:629-631 signal_addrReady).
+static int addr_issue(bk_ctx* c, const Plan& p, size_t i) {
+  const size_t k = i % c->cfg.n_slots;
+  Slot& s = c->slots[k];
+  const Chunk ch = chunk_of(c, p, i);
+  Access a = p.a;
+  a.rec_size = c->off ? 0 : c->cfg.record_size;
+  cudaStream_t st = c->s_asm;
+  if (s.used) BK_CUDA(cudaStreamWaitEvent(st, s.freed, 0));   // chunk i-N no longer reads the slot
+  BK_DELAY(st);
+  BK_PROF(kStAddrgen, st, true);
+  if (c->off && ch.hi > ch.lo) {
+    BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, st));
+    c->st.bytes_meta += (ch.hi - ch.lo) * 8;
+  }
+  launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err,
+                 p.user_addr ? c->d_ctr + 7 : c->d_ctr + 0, st);
+  c->n_launch += 3;
+  if (p.user_addr) {   // the caller's generator writes the addresses, within each lane's capacity
+    launch_lane_bases(ch.L, s.lanes, p.elem, s.ucount, s.ubase, st);
+    BK_CUDA(cudaMemsetAsync(s.ucount, 0, (size_t)ch.L * 4, st));
+    bk_addr_view v{};
+    v.struct_size = sizeof(bk_addr_view);
+    v.lanes = ch.L;
+    v.chunk_index = i;
+    v.n_chunks = p.bounds.size() - 1;
+    v.first_record = ch.lo;
+    v.n_records = ch.hi - ch.lo;
+    v.lane_desc = reinterpret_cast<const bk_lane*>(s.lanes);
+    v.offsets = c->off ? s.meta : nullptr;
+    v.end_offset = ch.end_byte;
+    v.addr = s.uaddr;
+    v.addr_base = s.ubase;
+    v.addr_count = s.ucount;
+    v.elem_bytes = p.elem;
+    const int r = c->a_gen(&v, (void*)st, c->a_gen_user);
+    if (r) return fail(BK_E_INVAL, "address generator returned %d for chunk %zu", r, i);
+    c->n_launch += 2;
+  }
+  launch_addr_stage1(ch, a, s.meta, s.lanes, s.tileK, p.elem, 8, 4, !(c->cfg.flags & BK_FLAG_NO_PATTERNS),
+                     p.user_addr ? s.uaddr : nullptr, s.ubase, s.ucount, c->a_desc_d[k], s.ecount, s.epos, s.exp,
+                     c->a_exp_d[k], c->a_tot_d[k], st);
+  c->n_launch += 4;
+  if (p.user_addr) {   // lane sizes are the generated counts: tile bases again
+    launch_tile_scan(s.tileK, ch.ntiles, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, st);
+    c->n_launch += 1;
+  }
+  BK_PROF(kStAddrgen, st, false);
+  BK_CUDA(cudaEventRecord(c->a_ready[k], st));
+  return BK_OK;
+}
+
+// Chunk i: stage 1 is issued one chunk ahead (the GPU generates chunk i+1's addresses while the host
+// assembles chunk i), the host waits for chunk i's addresses (P:691 wait_addrReady), assembles the
+// lanes from patterns / explicit addresses into pinned staging, one DMA.
+int stage_chunk_addr(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
+  const size_t C = p.bounds.size() - 1;
+  while (c->addr_next < C && c->addr_next <= i + 1) {
+    const int rc = addr_issue(c, p, c->addr_next++);
+    if (rc) return rc;
+  }
+  const size_t k = i % c->cfg.n_slots;
+  const Chunk ch = chunk_of(c, p, i);
+  const auto t0 = std::chrono::steady_clock::now();
+  BK_CUDA(cudaEventSynchronize(c->a_ready[k]));
+  const auto t1 = std::chrono::steady_clock::now();
+  c->st.ms_addr_wait += std::chrono::duration<double, std::milli>(t1 - t0).count();
+  const size_t hs = c->h_next++ % c->hstage.size();
+  if (c->h_used[hs]) BK_CUDA(cudaEventSynchronize(c->h_done[hs]));
+  if (c->cfg.flags & BK_FLAG_TEST_DELAYS) std::this_thread::sleep_for(std::chrono::microseconds(test_rand(c) % 200));
+  const uint64_t n_exp = *reinterpret_cast<volatile uint64_t*>(c->a_tot_h[k]);
+  HostData d{c->host, c->off, c->n, c->nbytes, c->cfg.record_size};
+  const auto t2 = std::chrono::steady_clock::now();
+  const uint64_t size = host_assemble_addr(*c->pool, d, ch.L, p.elem, c->a_desc_h[k], c->a_exp_h[k], n_exp,
+                                           c->hstage[hs], p.stage_cap, c->a_epos, c->a_tbase);
+  c->st.ms_cpu_gather += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t2).count();
+  if (size == UINT64_MAX) return fail(BK_E_RANGE, "address-mode chunk exceeds its slot (internal bound violated)");
+  if (size == UINT64_MAX - 1)
+    return fail(BK_E_INVAL, "chunk %zu: an element address lies outside the data set (or a count exceeds its lane)", i);
+  uint64_t pl = 0, na = 0;
+  for (uint32_t t = 0; t < ch.L; ++t) {
+    pl += c->a_desc_h[k][t].p > 0;
+    na += c->a_desc_h[k][t].count;
+  }
+  c->st.n_addr_lanes += ch.L;
+  c->st.n_pattern_lanes += pl;
+  c->st.n_addresses += na;
+  c->st.n_explicit_addr += n_exp;
+  c->st.bytes_addr += (uint64_t)ch.L * sizeof(AddrDesc) + n_exp * 8 + 8;
+  c->st.n_chunks_cpu += 1;
+  if (s.used) BK_CUDA(cudaStreamWaitEvent(c->s_copy, s.freed, 0));
+  BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->a_ready[k], 0));   // tile bases of this chunk are on the device
+  BK_DELAY(c->s_copy);
+  BK_PROF(kStH2D, c->s_copy, true);
+  if (size) BK_CUDA(cudaMemcpyAsync(s.stage, c->hstage[hs], size, cudaMemcpyHostToDevice, c->s_copy));
+  BK_CUDA(cudaEventRecord(c->h_done[hs], c->s_copy));
+  c->h_used[hs] = true;
+  BK_PROF(kStH2D, c->s_copy, false);
+  c->st.bytes_h2d += size;
+  c->st.bytes_accessed += ch.accessed;
+  BK_CUDA(cudaEventRecord(s.ready, c->s_copy));
+  s.used = true;
+  return BK_OK;
+}
+
 // Stages 1-3 of chunk i into slot s (on s_copy / s_asm); records s.ready.
 int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   const Chunk ch = chunk_of(c, p, i);
@@ -224,6 +375,7 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
 
 void note_plan(bk_ctx* c, const Plan& p) {
   c->st.gather_mode = (uint32_t)p.mode;
+  c->st.addr_elem_bytes = p.elem;
   c->st.chunk_budget = p.budget;
   c->st.lanes = p.L;
 }
@@ -234,6 +386,7 @@ int check_err(bk_ctx* c) {  // after end_host: the error bits arrived with the r
   if (herr & kErrKeyRange) return fail(BK_E_INVAL, "a group-by key is >= G");
   if (herr & kErrTableFull) return fail(BK_E_CAPACITY, "word-count hash table full; raise table_slots");
   if (herr & kErrWordTooLong) return fail(BK_E_RANGE, "a word is longer than 2^24 bytes or offset >= 2^40");
+  if (herr & kErrFusedTimeout) return fail(BK_E_CUDA, "persistent kernel: a loader/consumer wait timed out");
   return BK_OK;
 }
 
@@ -259,6 +412,8 @@ int begin_run(bk_ctx* c, void* stream) {
   c->st.n_chunks_cpu = 0;
   c->st.ms_cpu_gather = 0;
   c->st.n_chunks_zc = c->st.bytes_zc = c->st.records_zc = 0;
+  c->st.bytes_addr = c->st.n_addr_lanes = c->st.n_pattern_lanes = c->st.n_addresses = c->st.n_explicit_addr = 0;
+  c->st.ms_addr_wait = 0;
   return BK_OK;
 }
 
@@ -356,6 +511,8 @@ void host_reset(bk_ctx* c) {
   c->st.n_chunks_cpu = 0;
   c->st.ms_cpu_gather = 0;
   c->st.n_chunks_zc = c->st.bytes_zc = c->st.records_zc = 0;
+  c->st.bytes_addr = c->st.n_addr_lanes = c->st.n_pattern_lanes = c->st.n_addresses = c->st.n_explicit_addr = 0;
+  c->st.ms_addr_wait = 0;
 }
 
 int prof_reserve(bk_ctx* c, size_t pairs) {

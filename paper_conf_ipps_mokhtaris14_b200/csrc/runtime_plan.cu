@@ -61,7 +61,14 @@ uint64_t slot_need(const Plan& p) {
   const uint64_t ntiles = p.L / 32;
   const uint64_t desc = align_up(p.meta_cap * 8, kAlign) + align_up((uint64_t)p.L * sizeof(LaneDesc), kAlign) +
                         align_up(ntiles * 4, kAlign) + align_up((ntiles + 1) * 8, kAlign);
-  return align_up(p.raw_cap, kAlign) + align_up(p.stage_cap, kAlign) + p.desc_sets * desc + align_up(p.out_cap, kAlign);
+  uint64_t addr = 0;
+  if (p.mode == BK_GATHER_ADDR) {
+    addr = align_up(p.exp_cap, kAlign) + align_up((uint64_t)p.L * 4, kAlign) + align_up(((uint64_t)p.L + 1) * 8, kAlign);
+    if (p.user_addr)
+      addr += align_up(p.exp_cap, kAlign) + align_up((uint64_t)p.L * 8 + 8, kAlign) + align_up((uint64_t)p.L * 4, kAlign);
+  }
+  return align_up(p.raw_cap, kAlign) + align_up(p.stage_cap, kAlign) + p.desc_sets * desc + align_up(p.out_cap, kAlign) +
+         addr;
 }
 
 void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) {
@@ -108,21 +115,56 @@ void size_plan(const bk_ctx* c, Plan& p, uint64_t budget, uint32_t lane_target) 
   // = accessed bytes there)
   p.raw_cap = !p.zero_copy || p.packed ? budget + 64 : 0;
   p.meta_cap = c->off ? maxrecs + 1 : 0;
+  // address mode: 8 B per element address of the chunk with the most accessed bytes
+  p.exp_cap = p.mode == BK_GATHER_ADDR ? (acc / std::max<uint32_t>(p.elem, 1) + 2) * 8 : 0;
+}
+
+// BK_GATHER_ADDR element size: the configured one if every accessed length is a multiple of it, else
+// BK_E_INVAL; 0 = the largest power of two <= 8 dividing them (whole variable-length records: 1)
+static int addr_elem(const bk_ctx* c, const Access& a, uint32_t& el) {
+  std::vector<uint64_t> lens;
+  if (a.whole) {
+    if (c->off) lens.push_back(1);   // record lengths vary: bytes
+    else lens.push_back(c->cfg.record_size);
+  } else {
+    for (uint32_t e = 0; e < a.n_ext; ++e) lens.push_back(a.ext_len[e]);
+  }
+  auto divides = [&](uint32_t x) {
+    for (uint64_t l : lens)
+      if (l % x) return false;
+    return true;
+  };
+  el = c->cfg.addr_elem_bytes;
+  if (el == 0) {
+    el = 8;
+    while (el > 1 && !divides(el)) el >>= 1;
+    return BK_OK;
+  }
+  if ((el & (el - 1)) || el > 16 || !divides(el))
+    return fail(BK_E_INVAL, "addr_elem_bytes %u must be a power of two <= 16 dividing every accessed length", el);
+  return BK_OK;
 }
 
 int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t out_per_rec,
-                      int auto_mode) {
+                      int auto_mode, bool user_addr) {
   p.a = a;
+  p.user_addr = user_addr;
   if (c->cfg.lane_bytes) lane_target = c->cfg.lane_bytes;
   int mode = (int)c->cfg.gather_mode;
   if (mode == BK_GATHER_FUSED) mode = BK_GATHER_AUTO;   // FUSED is word count's own single-launch path
+  if (user_addr) mode = BK_GATHER_ADDR;
   // AUTO (counters in profiles/): whole-record access -> DENSE (copy engine at
   // 55.5 GB/s beats zero-copy's 51.4); sparse access -> HYBRID (host assembly packs exactly the
   // accessed bytes; the zero-copy gather is request-rate bound and only adds capacity on top).
   if (mode == BK_GATHER_AUTO) mode = auto_mode != BK_GATHER_AUTO ? auto_mode : a.whole ? BK_GATHER_DENSE : BK_GATHER_HYBRID;
-  if (mode != BK_GATHER_ZC && mode != BK_GATHER_DENSE && mode != BK_GATHER_CPU && mode != BK_GATHER_HYBRID)
+  if (mode != BK_GATHER_ZC && mode != BK_GATHER_DENSE && mode != BK_GATHER_CPU && mode != BK_GATHER_HYBRID &&
+      mode != BK_GATHER_ADDR)
     return fail(BK_E_INVAL, "bad gather_mode %d", mode);
   p.mode = mode;
+  if (mode == BK_GATHER_ADDR) {
+    const int rc = addr_elem(c, a, p.elem);
+    if (rc) return rc;
+  }
   p.zero_copy = mode != BK_GATHER_DENSE;
   p.desc_sets = mode == BK_GATHER_ZC ? 2 : 1;
   p.packed = (mode == BK_GATHER_CPU || mode == BK_GATHER_HYBRID) && host_packable(a);
@@ -155,10 +197,12 @@ int plan_run_uncached(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p,
               (unsigned long long)slot_need(p));
 }
 
-int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t out_per_chunk, int auto_mode) {
+int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t out_per_chunk, int auto_mode,
+             bool user_addr) {
   char key[256];
-  snprintf(key, sizeof key, "%u/%u/%u/%u/%u/%u/%u/%u/%u/%u/%d/%d", a.whole, a.n_ext, a.ext_off[0], a.ext_len[0],
-           a.ext_off[1], a.ext_len[1], a.ext_off[2], a.ext_len[2], a.E, lane_target, (int)out_per_chunk, auto_mode);
+  snprintf(key, sizeof key, "%u/%u/%u/%u/%u/%u/%u/%u/%u/%u/%d/%d/%d", a.whole, a.n_ext, a.ext_off[0], a.ext_len[0],
+           a.ext_off[1], a.ext_len[1], a.ext_off[2], a.ext_len[2], a.E, lane_target, (int)out_per_chunk, auto_mode,
+           (int)user_addr);
   std::string k(key);
   for (uint32_t e = 3; e < a.n_ext; ++e) k += "/" + std::to_string(a.ext_off[e]) + ":" + std::to_string(a.ext_len[e]);
   for (auto& kv : c->plan_cache)
@@ -166,7 +210,7 @@ int plan_run(bk_ctx* c, const Access& a, uint32_t lane_target, Plan& p, uint32_t
       p = kv.second;
       return BK_OK;
     }
-  const int rc = plan_run_uncached(c, a, lane_target, p, out_per_chunk, auto_mode);
+  const int rc = plan_run_uncached(c, a, lane_target, p, out_per_chunk, auto_mode, user_addr);
   p.key = k;
   if (rc == BK_OK) c->plan_cache.emplace_back(k, p);
   return rc;
@@ -204,6 +248,26 @@ void carve(bk_ctx* c, const Plan& p) {
     s.tileK = s.tileK_set[0];
     s.tile_base = s.tile_base_set[0];
     s.out = p.out_cap ? q : nullptr;
+    q += align_up(p.out_cap, kAlign);
+    s.exp = s.uaddr = s.ubase = nullptr;
+    s.ecount = s.ucount = nullptr;
+    s.epos = nullptr;
+    if (p.mode == BK_GATHER_ADDR) {
+      s.exp = reinterpret_cast<uint64_t*>(q);
+      q += align_up(p.exp_cap, kAlign);
+      s.ecount = reinterpret_cast<uint32_t*>(q);
+      q += align_up((uint64_t)p.L * 4, kAlign);
+      s.epos = reinterpret_cast<uint64_t*>(q);
+      q += align_up(((uint64_t)p.L + 1) * 8, kAlign);
+      if (p.user_addr) {
+        s.uaddr = reinterpret_cast<uint64_t*>(q);
+        q += align_up(p.exp_cap, kAlign);
+        s.ubase = reinterpret_cast<uint64_t*>(q);
+        q += align_up((uint64_t)p.L * 8 + 8, kAlign);
+        s.ucount = reinterpret_cast<uint32_t*>(q);
+        q += align_up((uint64_t)p.L * 4, kAlign);
+      }
+    }
     s.used = false;
   }
 }
