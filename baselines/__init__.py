@@ -33,6 +33,10 @@ def lib():
         l.mt_wordcount.argtypes = [p, u64, p, u64, p, p, p, u64]
         l.mt_kmer.restype = C.c_int64
         l.mt_kmer.argtypes = [p, u64, u32, u32, u32, u32, u64, p, p, u64]
+        l.mt_stream_copy.restype = C.c_double
+        l.mt_stream_copy.argtypes = [p, p, u64, C.c_int]
+        l.mt_stream_read.restype = C.c_double
+        l.mt_stream_read.argtypes = [p, u64, C.c_int, p]
         _lib = l
     return _lib
 
@@ -103,3 +107,16 @@ def wordcount(buf, off):
         if V >= 0:
             return wo[:V], wl[:V], wc[:V]
         cap = -V
+
+
+def host_stream(gib: float = 2.0, reps: int = 3) -> dict:
+    """Host DRAM bandwidth on all OpenMP threads (bench.py's host roofline): STREAM-style copy
+    (bytes read + written per second) and read-only, over buffers far larger than the LLC."""
+    n = int(gib * (1 << 30))
+    a = np.ones(n, np.uint8)
+    b = np.empty(n, np.uint8)
+    b.fill(1)
+    sink = np.zeros(1, np.uint64)
+    cp = lib().mt_stream_copy(a.ctypes.data, b.ctypes.data, n, reps)
+    rd = lib().mt_stream_read(a.ctypes.data, n, reps, sink.ctypes.data)
+    return {"copy_gbs": cp / 1e9, "read_gbs": rd / 1e9, "threads": threads(), "gib": gib}

@@ -325,3 +325,45 @@ int64_t mt_wordcount(const uint8_t* d, uint64_t nbytes, const uint64_t* off, uin
   free(pcnt);
   return (uint64_t)V > cap ? -V : V;
 }
+
+/* ---- host memory-system probes for bench.py's host roofline (not a paper variant) -------------
+ * STREAM-style, all OpenMP threads, each over its contiguous share: copy (read n + write n bytes,
+ * non-temporal-friendly 32-B vectors) and read (sum of u64). Return bytes moved per second. */
+double mt_stream_copy(const uint8_t* src, uint8_t* dst, uint64_t n, int reps) {
+  double best = 0;
+  for (int r = 0; r < reps; ++r) {
+    const double t0 = omp_get_wtime();
+#pragma omp parallel
+    {
+      const int T = omp_get_num_threads(), t = omp_get_thread_num();
+      const uint64_t lo = n * t / T / 64 * 64, hi = (t + 1 == T) ? n : n * (t + 1) / T / 64 * 64;
+      memcpy(dst + lo, src + lo, hi - lo);
+    }
+    const double dt = omp_get_wtime() - t0;
+    if (2.0 * n / dt > best) best = 2.0 * n / dt;
+  }
+  return best;
+}
+
+double mt_stream_read(const uint8_t* src, uint64_t n, int reps, uint64_t* sink) {
+  double best = 0;
+  uint64_t acc = 0;
+  for (int r = 0; r < reps; ++r) {
+    const double t0 = omp_get_wtime();
+#pragma omp parallel reduction(+ : acc)
+    {
+      const int T = omp_get_num_threads(), t = omp_get_thread_num();
+      const uint64_t lo = n / 8 * t / T, hi = n / 8 * (t + 1) / T;
+      const uint64_t* p = (const uint64_t*)src;
+      uint64_t a0 = 0, a1 = 0, a2 = 0, a3 = 0;
+      uint64_t i = lo;
+      for (; i + 4 <= hi; i += 4) { a0 += p[i]; a1 += p[i + 1]; a2 += p[i + 2]; a3 += p[i + 3]; }
+      for (; i < hi; ++i) a0 += p[i];
+      acc += a0 + a1 + a2 + a3;
+    }
+    const double dt = omp_get_wtime() - t0;
+    if (1.0 * n / dt > best) best = 1.0 * n / dt;
+  }
+  *sink = acc;
+  return best;
+}

@@ -244,8 +244,17 @@ uint64_t host_assemble_addr(HostPool& pool, const HostData& d, uint32_t L, uint3
           uint64_t b = 0;   // byte position in the lane's stream
           auto put = [&](const uint8_t* src, uint64_t len) {
             while (len) {
-              const uint64_t k = b >> 4, o = b & 15, m = std::min<uint64_t>(16 - o, len);
-              memcpy(tile + (k * 32 + i) * 16 + o, src, m);
+              const uint64_t k = b >> 4, o = b & 15;
+              uint8_t* dst = tile + (k * 32 + i) * 16;
+              if (o == 0 && len >= 16) {   // whole 16-B words: constant-size copies
+                memcpy(dst, src, 16);
+                b += 16;
+                src += 16;
+                len -= 16;
+                continue;
+              }
+              const uint64_t m = std::min<uint64_t>(16 - o, len);
+              memcpy(dst + o, src, m);
               b += m;
               src += m;
               len -= m;
@@ -259,7 +268,11 @@ uint64_t host_assemble_addr(HostPool& pool, const HostData& d, uint32_t L, uint3
             run0 = a;
             runl = elem;
           };
-          if (dd.p > 0) {
+          if (dd.p == 1 && dd.stride[0] == (int64_t)elem && dd.count) {   // one contiguous run
+            const uint64_t len = (uint64_t)dd.count * elem;
+            if (dd.base > d.nbytes || len > d.nbytes - dd.base) bad = true;
+            else put(d.base + dd.base, len);
+          } else if (dd.p > 0) {
             uint64_t a = dd.base;
             for (uint32_t k = 0; k < dd.count; ++k) {
               elem_at(a);

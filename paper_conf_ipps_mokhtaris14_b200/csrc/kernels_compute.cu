@@ -465,8 +465,10 @@ __global__ void __launch_bounds__(kFuThreads, 1) k_wc_fused(FusedArgs a) {
   const uint32_t nc = gridDim.x - a.n_load, ci = blockIdx.x - a.n_load;
   const unsigned lt = (1u << lane) - 1;
   for (int i = tid; i < kWcTab; i += blockDim.x) { sh.k1[i] = 0; sh.k2[i] = 0; sh.cnt[i] = 0; }
-  uint8_t* txt_s = fu_smem;                                                   // UB + 32 bytes
-  uint64_t* offs = reinterpret_cast<uint64_t*>(fu_smem + a.UB + 32);          // UR entries
+  uint8_t* txt_s = fu_smem;                                                   // UB + 64 bytes
+  uint64_t* offs = reinterpret_cast<uint64_t*>(fu_smem + a.UB + 64);          // UR entries
+  uint32_t* Dm = reinterpret_cast<uint32_t*>(offs + a.UR);                     // (UB + 64) / 32 + 2 entries
+  uint32_t* Bm = Dm + (a.UB + 64) / 32 + 2;
   unsigned long long t_wait = 0, t_comp = 0;
   for (uint32_t u = ci; u < a.U; u += nc) {
     const uint32_t sl = u % a.R;
@@ -495,79 +497,92 @@ __global__ void __launch_bounds__(kFuThreads, 1) k_wc_fused(FusedArgs a) {
     }
     __syncthreads();
     if (tid == 0) st_release(&a.done[sl], (unsigned long long)u + 1);   // slot free for unit u + R
-    // ---- stage 1 (this thread's range) + stage 4. The unit's bytes are split evenly over the
-    // CTA's threads (parallel tokenisation): thread t owns the words that START in [x0, x1),
-    // finishes its last word past x1 and skips a word running into x0 (thread t-1's). Record starts
-    // are delimiters (A10/A19): the first one after x0 by binary search over the unit's offsets.
-    const uint8_t* txt = txt_s + (((uintptr_t)(a.data + base)) & 15);
-    auto rpos = [&](uint32_t j) -> uint32_t {   // start of record lo+j relative to the unit (j <= nrec)
-      if (j >= nrec) return A;
-      return a.off ? (uint32_t)(offs[j] - base) : (uint32_t)((lo + j) * a.rec_size - base);
-    };
-    const uint32_t T = blockDim.x;
-    const uint32_t x0 = (uint32_t)(((uint64_t)tid * A) / T), x1 = (uint32_t)(((uint64_t)(tid + 1) * A) / T);
-    uint32_t j;   // first record index with rpos(j) > x0 (j in [1, nrec]; rpos(nrec) = A)
-    {
-      uint32_t l = 1, h = nrec;
-      while (l < h) {
-        const uint32_t m = (l + h) >> 1;
-        if (rpos(m) > x0) h = m; else l = m + 1;
-      }
-      j = l;
+    // ---- stage 1 (record boundaries -> break bits) + stage 4, word-parallel. Positions q are
+    // relative to the 16-B-aligned copy (the unit's byte 0 at q = sh0). Two bitmaps over the unit:
+    //   Dm: byte q is a delimiter (or outside the unit), Bm: a record starts at q (a word break, A10/A19);
+    // a word starts at q iff q is not a delimiter and q-1 is one or q starts a record, and ends at
+    // the next delimiter or record start. Each thread owns the words starting in its 32-byte segments,
+    // so the per-byte work is one SWAR classification and the hash of the word's bytes.
+    const uint32_t sh0 = (uint32_t)(((uintptr_t)(a.data + base)) & 15);
+    const uint32_t qend = sh0 + A;                       // first position past the unit
+    const uint32_t nseg = (qend + 31) >> 5;
+    for (uint32_t i = tid; i <= nseg; i += blockDim.x) Bm[i] = 0;
+    __syncthreads();
+    for (uint32_t j = 1 + tid; j < nrec; j += blockDim.x) {   // record starts after the unit's first
+      const uint32_t q = sh0 + (a.off ? (uint32_t)(offs[j] - base) : (uint32_t)((lo + j) * a.rec_size - base));
+      atomicOr(&Bm[q >> 5], 1u << (q & 31));
     }
-    const bool at_boundary = x0 == 0 || rpos(j - 1) == x0;
-    uint32_t next_b = j <= nrec ? rpos(j) : 0xffffffffu;
-    bool skip = x0 < A && !at_boundary && !is_delim(txt[x0 - 1]);
-    bool in_word = false;
-    uint64_t h1 = 0, h2 = 0;
-    uint32_t wstart = 0, wlen = 0;
-    uint32_t p = x0;
-    bool go = x0 < x1;
-    int qn = 0;   // warp-uniform queue fill
-    while (__any_sync(kFull, go)) {
-      bool end = false, delim = true;
-      uint32_t ch = 0x20u;
-      if (go) {
-        bool boundary = false;
-        if (p == next_b) {
-          boundary = true;
-          do {   // several records may start here if some are empty
-            ++j;
-            next_b = j <= nrec ? rpos(j) : 0xffffffffu;
-          } while (next_b == p);
+    for (uint32_t i = tid; i <= nseg; i += blockDim.x) {
+      uint32_t dm = 0xffffffffu;
+      if (i < nseg) {
+        dm = 0;
+        const uint32_t* wp = reinterpret_cast<const uint32_t*>(txt_s) + 8 * i;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const uint32_t x = wp[k];
+          // per byte 0xff where x == ' ' or 9 <= x <= 13, gathered to 4 bits
+          const uint32_t f = (__vcmpeq4(x, 0x20202020u) | (__vcmpgeu4(x, 0x09090909u) & __vcmpleu4(x, 0x0d0d0d0du)))
+                             & 0x01010101u;
+          dm |= ((f * 0x01020408u) >> 24) << (4 * k);
         }
-        if (p < A) ch = txt[p];
-        delim = p >= A || is_delim(ch);
-        if (boundary || delim) skip = false;
-        end = in_word && (boundary || delim);
+        const uint32_t q0 = 32 * i;   // positions outside [sh0, qend) count as delimiters
+        if (q0 < sh0) dm |= sh0 - q0 >= 32 ? 0xffffffffu : (1u << (sh0 - q0)) - 1;
+        if (q0 + 32 > qend) dm |= qend <= q0 ? 0xffffffffu : ~((1u << (qend - q0)) - 1);
       }
-      const unsigned m = __ballot_sync(kFull, end);   // the ended words go to the warp queue
-      if (m) {
-        if (end) {
-          const uint64_t occ = base + wstart;
-          if (wlen >= (1u << 24) || occ >= (1ull << 40)) atomicOr(a.err, kErrWordTooLong);
-          const int i = qn + __popc(m & lt);
-          sh.qk1[w][i] = h1;
-          sh.qk2[w][i] = h2;
-          sh.qol[w][i] = (occ << 24) | wlen;
+      Dm[i] = dm;
+    }
+    __syncthreads();
+    const uint8_t* tb = txt_s;
+    int qn = 0;   // warp-uniform queue fill
+    for (uint32_t i0 = 0; i0 < nseg; i0 += blockDim.x) {
+      const uint32_t i = i0 + tid;
+      uint32_t S = 0;
+      if (i < nseg) {
+        const uint32_t dm = Dm[i], bm = Bm[i];
+        const uint32_t prevd = i ? (Dm[i - 1] >> 31) : 1u;
+        S = ~dm & ((dm << 1) | prevd | bm);
+      }
+      // one word per lane per round: hash it, then the warp appends the round's words to its queue
+      while (__any_sync(kFull, S != 0)) {
+        const bool has = S != 0;
+        uint64_t h1 = 0, h2 = 0;
+        uint32_t q = 0, len = 0;
+        if (has) {
+          const uint32_t bit = __ffs(S) - 1;
+          S &= S - 1;
+          q = 32 * i + bit;
+          // end: the next break bit (delimiter or record start) after q
+          uint32_t seg = i;
+          uint32_t m = (Dm[seg] | Bm[seg]) & (bit == 31 ? 0u : ~((2u << bit) - 1));
+          while (!m) {
+            ++seg;
+            m = Dm[seg] | Bm[seg];   // Dm[nseg] is all ones: a word always ends
+          }
+          const uint32_t r = 32 * seg + __ffs(m) - 1;
+          len = r - q;
+          h1 = 0xcbf29ce484222325ull;
+          h2 = 0x84222325cbf29ce4ull;
+          for (uint32_t x = q; x < r; ++x) {
+            const uint32_t ch = tb[x];
+            h1 = (h1 ^ ch) * 0x100000001b3ull;
+            h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
+            h2 ^= h2 >> 29;
+          }
+        }
+        const unsigned m = __ballot_sync(kFull, has);
+        if (has) {
+          const uint64_t occ = base + (q - sh0);
+          if (len >= (1u << 24) || occ >= (1ull << 40)) atomicOr(a.err, kErrWordTooLong);
+          const int k = qn + __popc(m & lt);
+          sh.qk1[w][k] = h1;
+          sh.qk2[w][k] = h2;
+          sh.qol[w][k] = (occ << 24) | len;
         }
         qn += __popc(m);
         if (qn > kFuQ - 32) {
           wc_flush_queue(sh, w, lane, qn, a.table, a.mask, a.used, a.err);
           qn = 0;
         }
-      }
-      if (go) {
-        if (end) in_word = false;
-        if (!delim && !skip && (in_word || p < x1)) {
-          if (!in_word) { in_word = true; wstart = p; wlen = 0; h1 = 0xcbf29ce484222325ull; h2 = 0x84222325cbf29ce4ull; }
-          h1 = (h1 ^ ch) * 0x100000001b3ull;
-          h2 = (h2 + ch + 1) * 0x9E3779B97F4A7C15ull;
-          h2 ^= h2 >> 29;
-          ++wlen;
-        }
-        ++p;
-        go = p <= A && (p < x1 || in_word);
       }
     }
     if (qn) wc_flush_queue(sh, w, lane, qn, a.table, a.mask, a.used, a.err);
@@ -962,7 +977,7 @@ void launch_wc(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, cons
 uint32_t wc_fused_slot_bytes(uint32_t UB, uint32_t UR) { return (UB + 32 + UR * 8 + 255) / 256 * 256; }
 
 size_t wc_fused_smem(uint32_t UB, uint32_t UR) {
-  return std::max<size_t>(kFuSmemForce, (size_t)UB + 32 + (size_t)UR * 8);
+  return std::max<size_t>(kFuSmemForce, (size_t)UB + 64 + (size_t)UR * 8 + 2 * ((size_t)(UB + 64) / 32 + 2) * 4);
 }
 
 int wc_fused_grid() { return device_sms(); }

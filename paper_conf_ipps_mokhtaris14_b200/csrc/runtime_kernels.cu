@@ -15,6 +15,12 @@ static int wordcount_results(bk_ctx* c, bk_out_wordcount* o, uint64_t slots) {
   if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
   if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
                                   (unsigned long long)slots);
+  if (nw && (c->cfg.flags & BK_FLAG_KEEP_OUTPUTS_PINNED)) {   // cached registrations: DMA-speed result copies
+    int rc;
+    if ((rc = ensure_out_pinned(c, o->word_off, o->cap * 8)) || (rc = ensure_out_pinned(c, o->word_len, o->cap * 4)) ||
+        (rc = ensure_out_pinned(c, o->word_count, o->cap * 8)))
+      return rc;
+  }
   if (nw) {   // host or device result arrays (unified addressing)
     BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDefault));
     BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDefault));
@@ -62,14 +68,19 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
   (void)o;
   const int grid = wc_fused_grid();
   if (grid < 2) return BK_E_RANGE;
-  uint32_t n_load = (uint32_t)std::max(1, grid / 3);
+  uint32_t n_load = (uint32_t)std::max(1, grid / 6);   // sweep r02e: 16-32 of 148 (the link saturates)
   if (const char* e = getenv("BK_FUSED_LOADERS")) n_load = (uint32_t)std::max(1, std::min(grid - 1, atoi(e)));
   // units as large as 16 KiB allow while the ring keeps >= 2 slots per CTA; >= 2 KiB units and
   // >= 2 slots in any case (R x slot <= window_bytes)
   uint64_t UB = c->cfg.window_bytes / (2ull * grid);
   UB = UB > 64 ? (UB - 64) * 2 / 3 : 0;
-  UB = std::max<uint64_t>(2048, std::min<uint64_t>(UB, 16384)) / 16 * 16;
+  uint64_t ub_max = 16384;
+  if (const char* e = getenv("BK_FUSED_UNIT")) ub_max = std::max<uint64_t>(2048, std::min<uint64_t>(65536, atoll(e)));
+  UB = std::max<uint64_t>(2048, std::min<uint64_t>(UB, ub_max)) / 16 * 16;
+  if (c->cfg.chunk_bytes) UB = std::min<uint64_t>(UB, c->cfg.chunk_bytes / 16 * 16);   // explicit unit cap
+  if (UB < 16) return BK_E_RANGE;
   const uint32_t UR = (uint32_t)std::max<uint64_t>(UB / 16, 16);
+  if (c->cfg.flags & BK_FLAG_TEST_DELAYS) return BK_E_RANGE;   // delay injection targets the event pipeline
   const uint64_t slot_bytes = wc_fused_slot_bytes((uint32_t)UB, UR);
   const uint64_t R = std::min<uint64_t>(c->cfg.window_bytes / slot_bytes, 1u << 20);
   if (R < 2) return BK_E_RANGE;
@@ -90,8 +101,11 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
   unsigned long long* ready = (unsigned long long*)c->b_flags.p;
   const bool prof = (c->cfg.flags & BK_FLAG_PROFILE) != 0;
   WcEntry* table = (WcEntry*)c->b_table.p;
-  // eager issue (three operations): the cooperative launch is not graph-captured
-  int rc = run_device(c, stream, "wcfused", false, 1, [&]() -> int {
+  // captured once per (table, units, ring, loaders) and replayed: two memsets, the cooperative
+  // persistent kernel, the compaction
+  const std::string key = "wcfused/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + ukey + "/" +
+                          std::to_string(R) + "/" + std::to_string(n_load);
+  int rc = run_device(c, stream, key, true, 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
     BK_CUDA(cudaMemsetAsync(ready, 0, 2 * R * 8, c->s_comp));
     if (prof) BK_CUDA(cudaMemsetAsync(c->d_fprof, 0, 8 * 8, c->s_comp));
@@ -127,7 +141,7 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
     unsigned long long fp[5] = {0, 0, 0, 0, 0};
     BK_CUDA(cudaMemcpy(fp, c->d_fprof, sizeof fp, cudaMemcpyDeviceToHost));
     if (fp[2]) {
-      c->st.fused_wait_frac = (double)fp[0] / (double)fp[2];
+      c->st.fused_wait_frac = (double)fp[0] / (double)fp[2];   // consumers
       c->st.fused_compute_frac = (double)fp[1] / (double)fp[2];
     }
     if (fp[3] + fp[4]) c->st.fused_loader_wait_frac = (double)fp[3] / (double)(fp[3] + fp[4]);
@@ -144,7 +158,10 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   uint64_t slots = o->table_slots ? o->table_slots : (1ull << 20);
   if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
   const uint64_t ocap0 = std::min<uint64_t>(o->cap, slots);
-  if ((c->cfg.gather_mode == BK_GATHER_FUSED || c->cfg.gather_mode == BK_GATHER_AUTO) && c->n) {
+  // FUSED: when asked for, or AUTO's pick unless the caller fixed the chunking (chunk_bytes / lanes)
+  const bool fused = c->cfg.gather_mode == BK_GATHER_FUSED ||
+                     (c->cfg.gather_mode == BK_GATHER_AUTO && !c->cfg.chunk_bytes && !c->cfg.lanes);
+  if (fused && c->n) {
     BK_CUDA(c->b_table.ensure(slots * sizeof(WcEntry)));
     BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap0, 1) * 8));
     BK_CUDA(c->b_out2.ensure(std::max<uint64_t>(ocap0, 1) * 4));
@@ -755,6 +772,7 @@ int run_layout(bk_ctx* c, bk_out_layout* o, void* stream) {
   if (o->chunk >= o->n_chunks) return fail(BK_E_INVAL, "chunk %llu >= %llu chunks", (unsigned long long)o->chunk,
                                            (unsigned long long)o->n_chunks);
   if ((rc = begin_run(c, stream))) return rc;
+  note_plan(c, p);
   Slot& s = c->slots[p.mode == BK_GATHER_ADDR ? o->chunk % c->cfg.n_slots : 0];
   if (p.mode == BK_GATHER_ADDR) {   // stage 1 of exactly this chunk (and the look-ahead one) in its slot
     if ((rc = ensure_host_side(c, p)) || (rc = ensure_addr_side(c, p))) return rc;

@@ -562,7 +562,7 @@ std::string resident_key(const bk_ctx* c) {
   char b[24];
   for (const DevBuf* d : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_blk3,
                           &c->b_agg1, &c->b_agg2, &c->b_agg3, &c->b_mu, &c->b_hist, &c->b_colpre, &c->b_totals,
-                          &c->b_base, &c->b_h1, &c->b_h2, &c->b_units}) {
+                          &c->b_base, &c->b_h1, &c->b_h2, &c->b_units, &c->b_flags}) {
     snprintf(b, sizeof b, "%llx,", (unsigned long long)(uintptr_t)d->p);
     k += b;
   }
@@ -586,7 +586,7 @@ int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes) {
   if (cudaPointerGetAttributes(&at, ptr) == cudaSuccess && at.type != cudaMemoryTypeUnregistered)
     return BK_OK;   // device / managed memory, the caller's own pinned memory, or still registered by us
   cudaGetLastError();
-  if (keep && c->out_pinned.size() >= 4) {
+  if (keep && c->out_pinned.size() >= 8) {
     cudaHostUnregister(c->out_pinned.front().first);
     c->out_pinned.erase(c->out_pinned.begin());
   }
