@@ -4,11 +4,11 @@ ARCH   := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -std=c++17 -O3 -lineinfo $(ARCH) -Xcompiler -fPIC,-fvisibility=hidden -Xptxas -v
 PKG    := paper_conf_ipps_mokhtaris14_b200
 CSRC   := $(PKG)/csrc
-OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/kernels_pattern.o build/kernels_kmer.o build/kernels_merge.o build/kernels_addr.o build/runtime_plan.o build/runtime_pipeline.o build/runtime_kernels.o build/runtime_api.o build/host_gather.o
+OBJS   := build/kernels_stage.o build/kernels_compute.o build/kernels_partition.o build/kernels_baseline.o build/kernels_pattern.o build/kernels_kmer.o build/kernels_merge.o build/kernels_addr.o build/runtime_plan.o build/runtime_pipeline.o build/runtime_kernels.o build/runtime_api.o build/host_gather.o build/trace.o
 
 all: $(PKG)/libbk.so oracle/libbkoracle.so gen/libbkgen.so baselines/libbkmt.so tests/user/libbkuser.so
 
-build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh $(CSRC)/tma.cuh $(CSRC)/runtime.cuh $(CSRC)/host_gather.h include/bk.h
+build/%.o: $(CSRC)/%.cu $(CSRC)/bk_internal.cuh $(CSRC)/tma.cuh $(CSRC)/runtime.cuh $(CSRC)/host_gather.h $(CSRC)/trace.h include/bk.h
 	@mkdir -p build
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
 
@@ -16,8 +16,12 @@ build/host_gather.o: $(CSRC)/host_gather.cpp $(CSRC)/host_gather.h $(CSRC)/bk_in
 	@mkdir -p build
 	g++ -std=c++17 -O3 -march=x86-64-v3 -fPIC -fvisibility=hidden -Wall -I/usr/local/cuda/include -c $< -o $@
 
+build/trace.o: $(CSRC)/trace.cpp $(CSRC)/trace.h
+	@mkdir -p build
+	g++ -std=c++17 -O2 -fPIC -fvisibility=hidden -Wall -I/usr/local/cuda/include -c $< -o $@
+
 $(PKG)/libbk.so: $(OBJS)
-	$(NVCC) -shared $(ARCH) -cudart static -o $@ $(OBJS) -lpthread
+	$(NVCC) -shared $(ARCH) -cudart static -o $@ $(OBJS) -lpthread -ldl
 
 oracle/libbkoracle.so: oracle/oracle.c oracle/oracle.h
 	gcc -O2 -ffp-contract=off -fPIC -shared -Wall -o $@ oracle/oracle.c -lm

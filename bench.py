@@ -59,11 +59,13 @@ def parse():
     ap.add_argument("--host-threads", type=int, default=0)
     ap.add_argument("--lane-bytes", type=int, default=0)
     ap.add_argument("--zc-share", type=int, default=0, help="HYBRID zero-copy share of chunks, per mille")
+    ap.add_argument("--K", type=int, default=64, help="k-means clusters (C3: 64)")
     ap.add_argument("--pages", default="numpy", choices=["huge", "4k", "numpy"],
                     help="host data set pages: THP-backed mapping, 4 KiB mapping, or plain numpy")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-dbuf", action="store_true", help="skip the double-buffering baseline measurement")
     ap.add_argument("--no-profile", action="store_true", help="disable per-stage event timing")
+    ap.add_argument("--no-trace", action="store_true", help="skip the CUPTI-traced pass (BK_FLAG_TRACE)")
     ap.add_argument("--dump", default=None, help="after the timed steps, run one more step and write this rank's "
                                                  "(merged) result to DUMP/rank<r>.npz (the N>1 parity tests)")
     args = ap.parse_args()
@@ -121,7 +123,7 @@ def numa_local_cores(torch, local: int) -> list[int] | None:
     return part or None
 
 
-def make_shard(workload: str, gib: float, rank: int, world: int):
+def make_shard(workload: str, gib: float, rank: int, world: int, K: int = 64):
     """Rank r's contiguous shard of the weak-scaled data set. Returns dict."""
     nbytes = int(gib * GIB)
     if workload == "grep":
@@ -152,7 +154,7 @@ def make_shard(workload: str, gib: float, rank: int, world: int):
     n = nbytes // 64
     x = gen.points(gen.SEED_KMEANS, first=rank * n, n=n)
     return dict(buf=x.view(np.uint8).reshape(-1), off=None, n=n, first=rank * n, rec_size=64,
-                mu=gen.points(gen.SEED_KMEANS, first=0, n=64))
+                mu=gen.points(gen.SEED_KMEANS, first=0, n=K))
 
 
 # ------------------------------------------------------------------------------ helpers
@@ -272,6 +274,68 @@ def load_peaks():
         return {}
 
 
+# ------------------------------------------------------------------------------ host-side rooflines
+def host_rooflines(args, shard, st, step_s: float, peak_h2d: float, tr, pack_rate=None) -> dict:
+    """The two host-side resources a HYBRID step (CPU-packed + zero-copy chunks) is bound by,
+    against peaks measured in this run (the C2 line must name its binding roofline):
+      host_dram: bytes the host memory system moves per step / the live STREAM copy bandwidth (all
+        cores). Per packed record: its offset (8 B, variable records) + every 64-B line its accessed
+        extent touches (counted exactly from this shard's record addresses) + the packed bytes written
+        (non-temporal) + the same bytes read by the DMA; per zero-copy record: its lines + its offset
+        (DMA'd). Hardware prefetch may add lines, so this is a lower bound on the traffic.
+      pcie_wire: H2D completion bytes per step / the DMA wire peak. Zero-copy keys cost the PCIe read
+        bytes ncu measured per record (profiles/r01_traffic.json); DMAs carry their payload plus
+        one 24-B TLP header+framing per 256-B max payload (x 280/256), and so does the peak."""
+    import baselines
+    hs = baselines.host_stream(2.0, 3)
+    buf, off, n = shard["buf"], shard["off"], shard["n"]
+    eo, E = (16, 32) if args.workload == "grep" else (0, 16)
+    starts = (off.astype(np.uint64) if off is not None else np.arange(n, dtype=np.uint64) * np.uint64(shard["rec_size"]))
+    a0 = starts + np.uint64(buf.ctypes.data + eo)
+    lines = ((a0 + np.uint64(E - 1)) // np.uint64(64) - a0 // np.uint64(64) + np.uint64(1))
+    lines_per_rec = float(lines.mean())
+    rec_zc = st["records_zc"]
+    rec_cpu = n - rec_zc
+    off_b = 8 if off is not None else 0
+    host_bytes = rec_cpu * (off_b + 64 * lines_per_rec + 2 * E) + rec_zc * (off_b + 64 * lines_per_rec)
+    ach = host_bytes / step_s / 1e9
+    zc_wire = tr["pcie_read_per_unit"] if tr and tr.get("unit") == "record" else None
+    tlp = 280 / 256
+    wire = (rec_zc * zc_wire if zc_wire else 0.0) + (st["bytes_h2d"] - st["bytes_zc"] + st["bytes_meta"]) * tlp
+    wire_ach = wire / step_s / 1e9
+    out = {}
+    if pack_rate and st.get("ms_zc") and rec_zc:
+        # The HYBRID step as a two-resource schedule: the link carries the zero-copy keys (bound by the
+        # PCIe read-request rate: R_zc records/s, measured on the zero-copy gathers of this run's
+        # profiled pass), the packed keys and every record's offset by DMA (payload peak BW), while the
+        # host packs the rest at P records/s (measured alone in a CPU-assembly pass). With a share x of
+        # records zero-copy: link(x) = a + b x, host(x) = c (1 - x); the best split balances them, and
+        # T* = a + b x* is the least step time this host + link admit (DESIGN.md §9).
+        r_zc = rec_zc / (st["ms_zc"] * 1e-3)
+        a_ = (n * E + n * off_b) / (peak_h2d * 1e9)
+        b_ = n / r_zc - n * E / (peak_h2d * 1e9)
+        c_ = n / pack_rate
+        x_opt = min(1.0, max(0.0, (c_ - a_) / (b_ + c_)))
+        t_star = a_ + b_ * x_opt
+        out["hybrid_schedule"] = {
+            "bound": "link+host schedule", "t_bound_ms": round(t_star * 1e3, 3), "t_step_ms": round(step_s * 1e3, 3),
+            "frac": t_star / step_s, "x_zc_opt": round(x_opt, 4), "x_zc_run": round(rec_zc / n, 4),
+            "zc_records_per_s": r_zc, "pack_records_per_s": pack_rate, "dma_gbs": peak_h2d,
+            "note": "frac = least admissible step time / measured step time (1.0 = at the bound)"}
+    out.update({
+        "host_dram": {"bound": "host_dram", "achieved": ach, "peak": hs["copy_gbs"], "unit": "GB/s",
+                      "frac": ach / hs["copy_gbs"], "bytes_per_step": host_bytes,
+                      "lines_per_record": round(lines_per_rec, 4), "records_cpu": rec_cpu, "records_zc": rec_zc,
+                      "peak_source": f"STREAM copy (read + write bytes) on {hs['threads']} host threads, measured live "
+                                     f"(read-only: {hs['read_gbs']:.1f} GB/s)"},
+        "pcie_wire": {"bound": "pcie_wire", "achieved": wire_ach, "peak": peak_h2d * tlp, "unit": "GB/s",
+                      "frac": wire_ach / (peak_h2d * tlp), "bytes_per_step": wire,
+                      "zc_wire_bytes_per_record": zc_wire,
+                      "peak_source": "pinned H2D DMA payload peak (live) x 280/256 TLP framing"},
+    })
+    return out
+
+
 # ------------------------------------------------------------------------------ oracle timing
 def oracle_sample(workload: str, shard: dict, target_s: float):
     """Time the oracle (as it stands) on a bounded prefix of the shard; returns (GB/s, sample str, s)."""
@@ -347,7 +411,7 @@ def main():
                 args.host_threads = len(cores)
     if not args.host_threads:
         args.host_threads = max(1, (os.cpu_count() or 1) // int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
-    shard = make_shard(args.workload, gib, rank, world)
+    shard = make_shard(args.workload, gib, rank, world, args.K)
     peak_h2d = measure_h2d_peak(torch, dev)
     peak_bidir = measure_bidir_peak(torch, dev) if args.workload == "partition" else None
     ctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
@@ -381,8 +445,9 @@ def main():
         agg_out = ((cq[0], cq[1], torch.zeros(4096, dtype=torch.float64, device=dev), cq) if world > 1 else
                    (np.zeros(4096, np.uint64), np.zeros(4096, np.uint64), np.zeros(4096, np.float64)))
     if args.workload == "kmeans":
-        agg_out = ((torch.zeros(64, dtype=torch.int64, device=dev), torch.zeros(64, 16, dtype=torch.float64, device=dev))
-                   if world > 1 else (np.zeros(64, np.uint64), np.zeros((64, 16), np.float64)))
+        agg_out = ((torch.zeros(args.K, dtype=torch.int64, device=dev),
+                    torch.zeros(args.K, 16, dtype=torch.float64, device=dev))
+                   if world > 1 else (np.zeros(args.K, np.uint64), np.zeros((args.K, 16), np.float64)))
 
     from paper_conf_ipps_mokhtaris14_b200 import merge
 
@@ -502,6 +567,22 @@ def main():
                   "ms_compute_busy", "ms_overlap", "fused_wait_frac", "fused_compute_frac", "fused_loader_wait_frac"):
             st[k] = pst[k]
         st["profiled_ms_device"] = pst["ms_device"]
+    trace = None
+    if not args.no_profile and not args.no_trace:
+        # the timed pipeline itself (graph replay kept), every kernel and copy timed by CUPTI activity
+        # records: the stage breakdown and overlap of the pass that matches ms_per_step
+        try:
+            tctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode=args.gather,
+                              baseline_dbuf=args.impl == "dbuf", baseline_sbuf=args.impl == "sbuf",
+                              host_threads=args.host_threads, lane_bytes=args.lane_bytes, zc_share_pm=args.zc_share,
+                              trace=True, record_size=shard["rec_size"], keep_outputs_pinned=True)
+            tctx.register(shard["buf"], shard["off"], n_records=shard["n"])
+            for _ in range(3):
+                one_step(tctx)
+            trace = tctx.stats()
+            tctx.close()
+        except bk.BkError as e:
+            trace = {"unavailable": str(e)}
     total_bytes = nbytes * world * args.steps
     total_recs = shard["n"] * world * args.steps
     value = total_bytes / t_dev / 1e9
@@ -618,6 +699,17 @@ def main():
                                  "vs computing while loaders stream later units; loaders waiting for a free ring slot"}
     roof["avg_launch_ms"] = avg_ms
     roof["launches_per_step"] = launches
+    if rank == 0 and st.get("n_chunks_cpu") and args.workload in ("grep", "groupby_sparse") and args.impl == "ours":
+        # the host packers alone (CPU assembly of every chunk, no zero-copy traffic): their rate
+        cctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode="cpu",
+                          host_threads=args.host_threads, record_size=shard["rec_size"], keep_outputs_pinned=True)
+        cctx.register(shard["buf"], shard["off"], n_records=shard["n"])
+        one_step(cctx)
+        one_step(cctx)
+        cst = cctx.stats()
+        cctx.close()
+        pack_rate = shard["n"] / (cst["ms_cpu_gather"] * 1e-3) if cst["ms_cpu_gather"] else None
+        roof.update(host_rooflines(args, shard, st, t_dev / args.steps, peak_h2d, tr, pack_rate))
 
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
@@ -630,7 +722,8 @@ def main():
                    "chunks_cpu_assembled": st["n_chunks_cpu"], "n_chunks": st["n_chunks"],
                    "lanes_per_chunk": st["lanes"], "chunk_budget_bytes": st["chunk_budget"],
                    "l2": "inputs (>=64 MiB per GPU, host-resident) exceed the 126 MB L2; streamed from host each step",
-                   "parallelism": f"dp{world} (contiguous record shards, one PCIe link per GPU)"},
+                   "parallelism": f"dp{world} (contiguous record shards, one PCIe link per GPU)",
+                   **({"K": args.K} if args.workload == "kmeans" else {})},
         "records_per_s": total_recs / t_dev,
         "link_full_duplex": None if peak_bidir is None else {
             "peak_each_way_gbs": round(peak_bidir, 3), "achieved_each_way_gbs": round(link_gbs, 3),
@@ -647,6 +740,20 @@ def main():
                                "profiled_ms_device": round(st.get("profiled_ms_device", 0.0), 3),
                                "note": "per-stage busy sums from a profiled eager pass (CUDA events per stage "
                                        "per chunk); ms_device from the timed (graph-replayed when static) pass"},
+        "timed_pass_trace": None if trace is None else ({"unavailable": trace["unavailable"]} if "unavailable" in trace else {
+            "device_span_ms": round(trace["ms_trace_span"], 3), "records": trace["n_trace_records"],
+            "span_vs_ms_per_step": round(trace["ms_trace_span"] / (t_dev / args.steps * 1e3), 4),
+            "stages_ms": {k: round(trace[k], 3) for k in ("ms_h2d", "ms_addrgen", "ms_zc", "ms_relayout", "ms_compute",
+                                                          "ms_d2h")},
+            "launches": {"zc": trace["n_zc"], "relayout": trace["n_relayout"], "d2h": trace["n_d2h"]},
+            "xfer_busy_ms": round(trace["ms_xfer_busy"], 3), "compute_busy_ms": round(trace["ms_compute_busy"], 3),
+            "overlap_ms": round(trace["ms_overlap"], 3),
+            "overlap_frac": round(trace["ms_overlap"] / max(min(trace["ms_xfer_busy"], trace["ms_compute_busy"]), 1e-9), 4),
+            "link_busy_frac": round(trace["ms_xfer_busy"] / max(trace["ms_trace_span"], 1e-9), 4),
+            "max_busy_frac": round(max(trace["ms_xfer_busy"], trace["ms_compute_busy"]) / max(trace["ms_trace_span"], 1e-9), 4),
+            "how": "BK_FLAG_TRACE: CUPTI activity records of every kernel / copy of one graph-replayed (as timed) run; "
+                   "transfer = H2D/D2H copies + zero-copy gathers (+ k_wc_fused, stages 1-4), compute = stage-4 "
+                   "kernels; overlap_frac = |xfer n compute| / min(xfer, compute)"}),
         "overlap": {"xfer_busy_ms": round(st.get("ms_xfer_busy", 0.0), 3),
                     "compute_busy_ms": round(st.get("ms_compute_busy", 0.0), 3),
                     "overlap_ms": round(st.get("ms_overlap", 0.0), 3),

@@ -116,6 +116,10 @@ typedef struct bk_config {
                                    host sleeps before CPU assembly, to expose missing ordering */
 #define BK_FLAG_BASELINE_SBUF 4u  /* the single-buffer variant: one buffer of the whole window,
                                      copy then compute, no overlap */
+#define BK_FLAG_TRACE 128u  /* record every kernel and copy of a run with CUPTI activity records (libcupti
+                               loaded at run time; BK_E_UNSUPPORTED without it) and derive the bk_stats
+                               stage times / overlap from them — unlike BK_FLAG_PROFILE the run keeps its
+                               CUDA-graph replay, so the stats describe the timed pipeline */
 #define BK_FLAG_NO_PATTERNS 64u  /* BK_GATHER_ADDR: no pattern recognition, every element address is sent
                                     (the "addresses" column of the paper's Table II) */
 #define BK_FLAG_KEEP_OUTPUTS_PINNED 32u  /* caller-owned per-record output arrays that bk_run writes by DMA
@@ -338,6 +342,8 @@ typedef struct bk_stats {
   uint32_t addr_elem_bytes;   /*   element size used */
   uint32_t _pad_addr;
   double ms_addr_wait;        /*   host time waiting for stage 1's address information */
+  double ms_trace_span;       /* BK_FLAG_TRACE: first kernel/copy start to last end of the run (device) */
+  uint64_t n_trace_records;   /*   kernels + copies + memsets traced */
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);

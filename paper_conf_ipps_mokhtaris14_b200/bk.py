@@ -25,6 +25,7 @@ BK_FLAG_NO_GRAPH = 8
 BK_FLAG_TEST_DELAYS = 16
 BK_FLAG_KEEP_OUTPUTS_PINNED = 32
 BK_FLAG_NO_PATTERNS = 64
+BK_FLAG_TRACE = 128
 GATHER_NAMES = {"auto": BK_GATHER_AUTO, "zc": BK_GATHER_ZC, "cpu": BK_GATHER_CPU, "dense": BK_GATHER_DENSE, "hybrid": BK_GATHER_HYBRID,
                 "fused": BK_GATHER_FUSED, "addr": BK_GATHER_ADDR}
 
@@ -87,7 +88,8 @@ class bk_stats(C.Structure):
                 ("fused_ring_slots", u32), ("fused_wait_frac", C.c_double), ("fused_compute_frac", C.c_double),
                 ("fused_loader_wait_frac", C.c_double), ("bytes_addr", u64), ("n_addr_lanes", u64),
                 ("n_pattern_lanes", u64), ("n_addresses", u64), ("n_explicit_addr", u64), ("addr_elem_bytes", u32),
-                ("_pad_addr", u32), ("ms_addr_wait", C.c_double)]
+                ("_pad_addr", u32), ("ms_addr_wait", C.c_double), ("ms_trace_span", C.c_double),
+                ("n_trace_records", u64)]
 
 
 class bk_out_pattern(C.Structure):
@@ -206,7 +208,7 @@ def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_m
               profile: bool = False, baseline_dbuf: bool = False, lane_bytes: int = 0,
               zc_share_pm: int = 0, baseline_sbuf: bool = False, no_graph: bool = False,
               test_delays: bool = False, keep_outputs_pinned: bool = False, no_patterns: bool = False,
-              addr_elem_bytes: int = 0) -> int:
+              addr_elem_bytes: int = 0, trace: bool = False) -> int:
     if isinstance(gather_mode, str):
         gather_mode = GATHER_NAMES[gather_mode]
     cfg = bk_config(C.sizeof(bk_config), device, window_bytes, n_slots, gather_mode, chunk_bytes, lanes,
@@ -215,7 +217,7 @@ def bk_create(device: int = 0, window_bytes: int = 0, n_slots: int = 0, gather_m
                     (BK_FLAG_BASELINE_SBUF if baseline_sbuf else 0) | (BK_FLAG_NO_GRAPH if no_graph else 0) |
                     (BK_FLAG_TEST_DELAYS if test_delays else 0) |
                     (BK_FLAG_KEEP_OUTPUTS_PINNED if keep_outputs_pinned else 0) |
-                    (BK_FLAG_NO_PATTERNS if no_patterns else 0),
+                    (BK_FLAG_NO_PATTERNS if no_patterns else 0) | (BK_FLAG_TRACE if trace else 0),
                     lane_bytes,
                     zc_share_pm, addr_elem_bytes)
     ctx = P()

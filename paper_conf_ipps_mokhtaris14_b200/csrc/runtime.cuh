@@ -34,6 +34,7 @@
 #include "../../include/bk.h"
 #include "bk_internal.cuh"
 #include "host_gather.h"
+#include "trace.h"
 
 namespace bk {
 namespace rt {
@@ -186,6 +187,8 @@ struct bk_ctx {  // the opaque context of include/bk.h
   std::vector<cudaEvent_t> a_ready;          // per slot: stage 1 (addresses) of its chunk finished
   size_t addr_next = 0;                      // next chunk whose stage 1 is not yet issued
   std::vector<uint64_t> a_epos, a_tbase;
+  std::vector<bk::trace::Rec> trace_recs;    // BK_FLAG_TRACE: this run's CUPTI records
+  bool tracing = false;
   bk_addr_fn a_gen = nullptr;                // bk_run_user_addr generator + its argument
   void* a_gen_user = nullptr;
   bk::rt::DevBuf b_mown, b_mcnt, b_mctr;     // bk_merge_counts scratch (never captured in a graph)
@@ -241,6 +244,7 @@ int device_end(bk_ctx* c);
 void host_reset(bk_ctx* c);
 int prof_reserve(bk_ctx* c, size_t pairs);
 int end_host(bk_ctx* c, void* stream);
+int trace_begin(bk_ctx* c);
 void drop_graphs(bk_ctx* c);
 bool graphable(const Plan& p);
 // Stage 4 stages tiles through TMA bulk copies unless zero-copy gathers run alongside (ZC, HYBRID):
@@ -336,6 +340,7 @@ int run_device(bk_ctx* c, void* stream, const std::string& key_in, bool graphabl
   BK_CUDA(cudaSetDevice(c->cfg.device));
   const std::string key = key_in + "|" + resident_key(c);
   host_reset(c);
+  if (int rt = trace_begin(c)) return rt;
   BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
   BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_begin, 0));
   BK_CUDA(cudaEventRecord(c->t_begin, c->s_comp));

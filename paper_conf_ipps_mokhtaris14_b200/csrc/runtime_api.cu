@@ -30,6 +30,10 @@ using namespace bk::rt;
 // After a failed run: wait for everything already queued on the context's streams (no copy may
 // still target the caller's buffers, no kernel may still use the slots) and clear the error state.
 static void drain(bk_ctx* c) {
+  if (c->tracing) {   // a failed traced run: stop collecting
+    bk::trace::end();
+    c->tracing = false;
+  }
   for (cudaStream_t st : {c->s_copy, c->s_asm, c->s_comp, c->s_d2h})
     if (st) cudaStreamSynchronize(st);
   for (auto st : c->s_slot) cudaStreamSynchronize(st);

@@ -68,7 +68,7 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
   (void)o;
   const int grid = wc_fused_grid();
   if (grid < 2) return BK_E_RANGE;
-  uint32_t n_load = (uint32_t)std::max(1, grid / 6);   // sweep r02e: 16-32 of 148 (the link saturates)
+  uint32_t n_load = (uint32_t)std::max(1, grid / 4);   // sweeps r02e/r02h: 24-49 of 148 loaders saturate the link
   if (const char* e = getenv("BK_FUSED_LOADERS")) n_load = (uint32_t)std::max(1, std::min(grid - 1, atoi(e)));
   // units as large as 16 KiB allow while the ring keeps >= 2 slots per CTA; >= 2 KiB units and
   // >= 2 slots in any case (R x slot <= window_bytes)

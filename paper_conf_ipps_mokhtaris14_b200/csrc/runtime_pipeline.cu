@@ -397,6 +397,7 @@ int check_err(bk_ctx* c) {  // after end_host: the error bits arrived with the r
 
 int begin_run(bk_ctx* c, void* stream) {
   BK_CUDA(cudaSetDevice(c->cfg.device));
+  if (int rt = trace_begin(c)) return rt;
   BK_CUDA(cudaMemsetAsync(c->d_err, 0, sizeof(int), c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->d_ctr, 0, 8 * sizeof(unsigned long long), c->s_comp));
   BK_CUDA(cudaEventRecord(c->ev_begin, (cudaStream_t)stream));
@@ -417,28 +418,26 @@ int begin_run(bk_ctx* c, void* stream) {
   return BK_OK;
 }
 
-// Per-stage busy sums and, from the interval of every (stage, chunk) event pair relative to the
-// run start, the union of transfer intervals, the union of compute intervals and their overlap
-// (the north_star's copy/compute overlap, measured with CUDA events instead of nsys).
-int stage_stats(bk_ctx* c) {
+// Per-stage busy sums and, from (stage, begin, end) intervals relative to the run start, the union
+// of transfer intervals, the union of compute intervals and their overlap (the north_star's
+// copy/compute overlap). Intervals come from BK_FLAG_PROFILE's event pairs (eager issue) or from
+// BK_FLAG_TRACE's CUPTI records (the graph-replayed pipeline as timed).
+struct Interval { int stage; double b, e; };
+
+static void interval_stats(bk_ctx* c, const std::vector<Interval>& iv) {
   double acc[kNStages] = {};
   uint64_t cnt[kNStages] = {};
   std::vector<std::pair<double, double>> xfer, comp;
-  // BK_TIMELINE=<path>: append every profiled (stage, begin ms, end ms) interval of the run as CSV
-  // (a timeline for analysis where nsys is not available; stage ids as kSt* in runtime.cuh)
+  // BK_TIMELINE=<path>: append every interval of the run as CSV (stage ids as kSt* in runtime.cuh)
   const char* tl_path = getenv("BK_TIMELINE");
   FILE* tl = tl_path ? fopen(tl_path, "a") : nullptr;
   if (tl) fprintf(tl, "# run\n");
-  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
-    float e = 0, b0 = 0;
-    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
-    BK_CUDA(cudaEventElapsedTime(&b0, c->t_begin, c->prof[i]));
-    const int stg = c->prof_stage[i / 2];
-    if (tl) fprintf(tl, "%d,%.4f,%.4f\n", stg, b0, b0 + e);
-    acc[stg] += e;
-    cnt[stg] += 1;
-    if (stg == kStH2D || stg == kStGather || stg == kStD2H) xfer.emplace_back(b0, b0 + e);
-    if (stg == kStCompute) comp.emplace_back(b0, b0 + e);
+  for (const auto& x : iv) {
+    if (tl) fprintf(tl, "%d,%.4f,%.4f\n", x.stage, x.b, x.e);
+    acc[x.stage] += x.e - x.b;
+    cnt[x.stage] += 1;
+    if (x.stage == kStH2D || x.stage == kStGather || x.stage == kStD2H) xfer.emplace_back(x.b, x.e);
+    if (x.stage == kStCompute) comp.emplace_back(x.b, x.e);
   }
   if (tl) fclose(tl);
   auto merge = [](std::vector<std::pair<double, double>> v) {
@@ -473,7 +472,59 @@ int stage_stats(bk_ctx* c) {
   c->st.ms_xfer_busy = bx;
   c->st.ms_compute_busy = bc;
   c->st.ms_overlap = ov;
+}
+
+int stage_stats(bk_ctx* c) {
+  std::vector<Interval> iv;
+  for (size_t i = 0; i + 1 < c->prof_used + 1 && i < c->prof_used; i += 2) {
+    float e = 0, b0 = 0;
+    BK_CUDA(cudaEventElapsedTime(&e, c->prof[i], c->prof[i + 1]));
+    BK_CUDA(cudaEventElapsedTime(&b0, c->t_begin, c->prof[i]));
+    iv.push_back({c->prof_stage[i / 2], b0, b0 + e});
+  }
+  interval_stats(c, iv);
   return BK_OK;
+}
+
+// BK_FLAG_TRACE: stage of a traced kernel / copy, by the kernel's (mangled) name; -1 = not a stage
+// (memsets, finalize / compaction kernels, test spins)
+static int trace_stage(const trace::Rec& r) {
+  if (r.kind == trace::Rec::kMemcpy) return r.copy_kind == 1 ? kStH2D : r.copy_kind == 2 ? kStD2H : -1;
+  if (r.kind != trace::Rec::kKernel) return -1;
+  const std::string& n = r.name;
+  auto has = [&](const char* x) { return n.find(x) != std::string::npos; };
+  if (has("k_gather_")) return has("ILb1E") ? kStGather : kStRelayout;   // <kHost = true>: zero-copy
+  if (has("k_wc_fused")) return kStGather;                                 // stages 1-4 in one kernel
+  if (has("k_lane_first") || has("k_addrgen") || has("k_tile_scan") || has("k_addr_") || has("k_lane_caps"))
+    return kStAddrgen;
+  if (has("compact") || has("k_grep_order") || has("k_merge") || has("k_spin")) return -1;
+  return kStCompute;
+}
+
+int trace_begin(bk_ctx* c) {
+  c->tracing = false;
+  if (!(c->cfg.flags & BK_FLAG_TRACE)) return BK_OK;
+  if (trace::begin(&c->trace_recs)) return fail(BK_E_UNSUPPORTED, "BK_FLAG_TRACE: libcupti not available");
+  c->tracing = true;
+  return BK_OK;
+}
+
+static void trace_finish(bk_ctx* c) {
+  trace::end();
+  c->tracing = false;
+  std::vector<Interval> iv;
+  uint64_t t0 = UINT64_MAX, t1 = 0;
+  for (const auto& r : c->trace_recs) {
+    t0 = std::min(t0, r.start);
+    t1 = std::max(t1, r.end);
+  }
+  for (const auto& r : c->trace_recs) {
+    const int stg = trace_stage(r);
+    if (stg >= 0) iv.push_back({stg, (r.start - t0) * 1e-6, (r.end - t0) * 1e-6});
+  }
+  interval_stats(c, iv);
+  c->st.ms_trace_span = t1 > t0 ? (t1 - t0) * 1e-6 : 0.0;
+  c->st.n_trace_records = c->trace_recs.size();
 }
 
 int end_run(bk_ctx* c, void* stream) { return end_host(c, stream); }
@@ -540,8 +591,12 @@ int end_host(bk_ctx* c, void* stream) {
   float ms = 0;
   BK_CUDA(cudaEventElapsedTime(&ms, c->t_begin, c->t_end));
   c->st.ms_device = ms;
-  int rc = stage_stats(c);
-  if (rc) return rc;
+  if (c->tracing) {
+    trace_finish(c);
+  } else {
+    int rc = stage_stats(c);
+    if (rc) return rc;
+  }
   return check_err(c);
 }
 

@@ -119,3 +119,21 @@ def test_current_device_restored_and_struct_size_checked():
             with pytest.raises(bk.BkError) as e:
                 bk.bk_run(ctx.ctx, bk.BK_K_GROUPBY, None, o)
             assert e.value.status == bk.BK_E_INVAL
+
+
+@pytest.mark.parametrize("mode", ["dense", "zc", "hybrid"])
+def test_trace_flag_keeps_graph_replay_and_reports_stages(mode):
+    """BK_FLAG_TRACE (CUPTI activity records) on the graph-replayed pipeline: results unchanged, the
+    traced span is the run's device time, transfer and compute intervals are reported."""
+    n = 400_000
+    g = gen.groupby(n=n, stride=64)
+    want = oracle.groupby(g, n, 64, 4096)
+    with bk.Context(window_bytes=4 * MIB, record_size=64, gather_mode=mode, trace=True) as ctx:
+        ctx.register(g, None, n_records=n)
+        for _ in range(3):
+            c, q, a = ctx.groupby(4096)
+            assert np.array_equal(c, want[0]) and np.array_equal(q, want[1])
+        st = ctx.stats()
+    assert st["n_trace_records"] > st["n_chunks"] and st["ms_trace_span"] > 0
+    assert st["ms_xfer_busy"] > 0 and st["ms_compute_busy"] > 0
+    assert st["ms_trace_span"] <= st["ms_device"] * 1.05 + 0.05
