@@ -76,6 +76,7 @@ struct Slot {
   uint32_t* tileK_set[2] = {nullptr, nullptr};
   uint64_t* tile_base_set[2] = {nullptr, nullptr};
   cudaEvent_t copied = nullptr, ready = nullptr, freed = nullptr;
+  cudaEvent_t zt0 = nullptr, zt1 = nullptr;   // HYBRID: device time of the slot's zero-copy gather
   bool used = false;
 };
 
@@ -276,8 +277,13 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
   const size_t C = p.bounds.size() - 1;
   c->st.n_chunks = C;
   note_plan(c, p);
-  std::vector<cudaEvent_t> zc_inflight;
-  const size_t zc_depth = std::max<size_t>(1, (c->cfg.n_slots - 1) / 2);
+  // HYBRID adaptive split: zero-copy chunks in flight while the host packs one chunk. Starts at one
+  // (16 host threads pack a chunk faster than the link gathers one zero-copy: profiles/r01_hybrid_sweep.md)
+  // and follows the measured ratio (host time per packed chunk) / (time per zero-copy chunk), so a rank
+  // with few host cores (8 ranks on one host) lets the GPU gather more and never waits on slow packers.
+  std::vector<Slot*> zc_inflight;
+  size_t zc_depth = 1;
+  double t_zc_ms = 0, t_cpu_ms = 0;   // running estimates
   if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID || p.mode == BK_GATHER_ADDR) {
     int rc = ensure_host_side(c, p);
     if (!rc && p.mode == BK_GATHER_ADDR) rc = ensure_addr_side(c, p);
@@ -294,21 +300,32 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
       const uint64_t pm = std::min<uint32_t>(c->cfg.zc_share_pm, 1000);
       cpu = ((i + 1) * pm) / 1000 == (i * pm) / 1000;
     } else if (p.mode == BK_GATHER_HYBRID) {
-      // adaptive split (default): the GPU zero-copy gathers run asynchronously; keep one in flight
-      // and let the host pool assemble the next chunk while it is busy (profiles/r01_hybrid_sweep.md)
-      while (!zc_inflight.empty() && cudaEventQuery(zc_inflight.front()) == cudaSuccess)
+      // adaptive split (default): the GPU zero-copy gathers run asynchronously; keep zc_depth in
+      // flight and let the host pool assemble the next chunk while they are busy
+      while (!zc_inflight.empty() && cudaEventQuery(zc_inflight.front()->ready) == cudaSuccess) {
+        float ms = 0;   // the gather's own device time (timing events around it)
+        if (cudaEventElapsedTime(&ms, zc_inflight.front()->zt0, zc_inflight.front()->zt1) == cudaSuccess && ms > 0)
+          t_zc_ms = t_zc_ms > 0 ? 0.5 * (t_zc_ms + ms) : ms;
         zc_inflight.erase(zc_inflight.begin());
+      }
       cudaGetLastError();
+      if (t_zc_ms > 0 && t_cpu_ms > 0)
+        zc_depth = (size_t)std::max<long>(1, std::min<long>((long)c->cfg.n_slots - 1, std::lround(t_cpu_ms / t_zc_ms)));
       cpu = zc_inflight.size() >= zc_depth;
     }
     int rc;
     {
       NvtxRange r("chunk %zu %s", i, p.mode == BK_GATHER_ADDR ? "addr" : cpu ? "cpu" : p.zero_copy ? "zc" : "dense");
+      const auto t0 = std::chrono::steady_clock::now();
       rc = p.mode == BK_GATHER_ADDR ? stage_chunk_addr(c, p, i, s) : cpu ? stage_chunk_cpu(c, p, i, s)
                                                                           : stage_chunk(c, p, i, s);
+      if (cpu && p.mode == BK_GATHER_HYBRID) {
+        const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        t_cpu_ms = t_cpu_ms > 0 ? 0.5 * (t_cpu_ms + ms) : ms;
+      }
     }
     if (rc) return rc;
-    if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(s.ready);
+    if (p.mode == BK_GATHER_HYBRID && !cpu) zc_inflight.push_back(&s);
     BK_CUDA(cudaStreamWaitEvent(cs, s.ready, 0));
     BK_DELAY(cs);
     BK_PROF(kStCompute, cs, true);

@@ -150,7 +150,8 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
   for (auto& s : c->slots) {
     if (cudaEventCreateWithFlags(&s.copied, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&s.ready, cudaEventDisableTiming) != cudaSuccess ||
-        cudaEventCreateWithFlags(&s.freed, cudaEventDisableTiming) != cudaSuccess)
+        cudaEventCreateWithFlags(&s.freed, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreate(&s.zt0) != cudaSuccess || cudaEventCreate(&s.zt1) != cudaSuccess)
       return cleanup(fail(BK_E_CUDA, "slot events"));
   }
   c->st.struct_size = sizeof(bk_stats);
@@ -444,6 +445,8 @@ int bk_destroy(bk_ctx* c) {
     if (s.copied) cudaEventDestroy(s.copied);
     if (s.ready) cudaEventDestroy(s.ready);
     if (s.freed) cudaEventDestroy(s.freed);
+    if (s.zt0) cudaEventDestroy(s.zt0);
+    if (s.zt1) cudaEventDestroy(s.zt1);
   }
   for (DevBuf* b : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_blk3, &c->b_agg1, &c->b_agg2,
                     &c->b_agg3, &c->b_mu})

@@ -329,10 +329,12 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     if (s.used && early) BK_CUDA(cudaStreamWaitEvent(ss, s.freed, 0));   // the stage buffer
     BK_DELAY(ss);
     BK_PROF(kStGather, ss, true);
+    if (p.mode == BK_GATHER_HYBRID) BK_CUDA(cudaEventRecord(s.zt0, ss));
     Chunk gch = ch;   // readable source: the registered data set
     gch.guard_lo = ch.base_byte;
     gch.guard_hi = c->nbytes - ch.base_byte;
     launch_gather(gch, a, c->host_dev + ch.base_byte, s.meta, s.lanes, s.tile_base, s.stage, p.stage_cap, 1, ss);
+    if (p.mode == BK_GATHER_HYBRID) BK_CUDA(cudaEventRecord(s.zt1, ss));
     BK_PROF(kStGather, ss, false);
     c->n_launch += 3;
     c->st.bytes_h2d += ch.accessed;
