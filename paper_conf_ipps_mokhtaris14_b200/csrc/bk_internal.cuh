@@ -105,11 +105,22 @@ uint32_t wc_fused_slot_bytes(uint32_t UB, uint32_t UR);
 size_t wc_fused_smem(uint32_t UB, uint32_t UR);
 int wc_fused_grid();
 uint32_t wc_fused_threads();
+// DMA-fed variant: the copy engine fills K slots with batches of consecutive units (the host issues
+// copy + stream-ordered flag write per batch); every CTA consumes
+struct FusedDma {
+  const uint32_t* ubatch;   // U: unit -> batch
+  const uint64_t* bby;      // NB + 1: batch byte bounds
+  const uint64_t* brec;     // NB + 1: batch record bounds
+  const uint32_t* bunits;   // NB: units per batch
+  uint32_t K;
+  uint64_t bslot_bytes, btext;   // slot = [btext + 64 text][offsets]
+  unsigned int* bcnt;       // K (zeroed)
+};
 cudaError_t launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t* off, uint64_t rec_size,
                             const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
                             uint32_t n_load, uint8_t* ring, uint32_t R, unsigned long long* ready,
                             unsigned long long* done, WcEntry* table, uint64_t mask, unsigned long long* used,
-                            int* err, unsigned long long* prof, cudaStream_t s);
+                            int* err, unsigned long long* prof, const FusedDma* dma, cudaStream_t s);
 // double-buffering baseline (variant iv): raw chunk bytes start at absolute offset base_byte
 void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint64_t hi, uint64_t base_byte,
                     uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,

@@ -377,6 +377,17 @@ struct FusedArgs {
   int* err;
   unsigned long long* prof;   // optional: [0] consumer wait ns, [1] consumer compute ns, [2] consumer ns,
                               //           [3] loader wait ns, [4] loader copy ns
+  // DMA-fed mode (n_load == 0): the copy engine fills K batch slots (consecutive units), each followed
+  // by a stream-ordered flag write (ready[slot] = batch + 1); consumers count a batch's units done
+  // and the last one releases the slot (done[slot] = batch + 1) for the DMA of batch + K
+  const uint32_t* ubatch;     // U: unit -> batch
+  const uint64_t* bby;        // NB + 1: batch byte bounds
+  const uint64_t* brec;       // NB + 1: batch record bounds
+  const uint32_t* bunits;     // NB: units per batch
+  uint32_t K;                 // batch slots
+  uint64_t bslot_bytes;       // slot: [btext + 64 text][offsets]
+  uint64_t btext;
+  unsigned int* bcnt;         // K: units of the slot's batch consumed (zeroed by the run)
 };
 
 __device__ __forceinline__ unsigned long long gtime() {
@@ -470,11 +481,13 @@ __global__ void __launch_bounds__(kFuThreads, 1) k_wc_fused(FusedArgs a) {
   uint32_t* Dm = reinterpret_cast<uint32_t*>(offs + a.UR);                     // (UB + 64) / 32 + 2 entries
   uint32_t* Bm = Dm + (a.UB + 64) / 32 + 2;
   unsigned long long t_wait = 0, t_comp = 0;
+  const bool dma = a.n_load == 0;
   for (uint32_t u = ci; u < a.U; u += nc) {
-    const uint32_t sl = u % a.R;
+    const uint32_t b = dma ? a.ubatch[u] : u;      // what the flag names: the unit, or its batch
+    const uint32_t sl = dma ? b % a.K : u % a.R;
     const unsigned long long tw = gtime();
     if (tid == 0) {
-      while (ld_acquire(&a.ready[sl]) != (unsigned long long)u + 1)
+      while (ld_acquire(&a.ready[sl]) != (unsigned long long)b + 1)
         if (gtime() - tw > kSpinLimitNs) { atomicOr(a.err, kErrFusedTimeout); s_abort = 1; break; }
     }
     __syncthreads();
@@ -484,19 +497,34 @@ __global__ void __launch_bounds__(kFuThreads, 1) k_wc_fused(FusedArgs a) {
     const uint64_t lo = a.ub[u], hi = a.ub[u + 1];
     const uint64_t base = a.uby[u];
     const uint32_t nrec = (uint32_t)(hi - lo), A = (uint32_t)(a.uby[u + 1] - base);
-    const uint8_t* slot = a.ring + (size_t)sl * a.slot_bytes;
     {   // slot -> shared memory (L2 reads: the flag's acquire orders them; .cg bypasses stale L1 lines)
       const uint32_t sh0 = (uint32_t)(((uintptr_t)(a.data + base)) & 15);
       const uint32_t nw = (sh0 + A + 15) >> 4;
-      for (uint32_t k = tid; k < nw; k += blockDim.x)
-        reinterpret_cast<uint4*>(txt_s)[k] = __ldcg(reinterpret_cast<const uint4*>(slot) + k);
-      if (a.off) {
-        const uint64_t* so = reinterpret_cast<const uint64_t*>(slot + a.UB + 32);
-        for (uint32_t j = tid; j < nrec; j += blockDim.x) offs[j] = __ldcg(so + j);
+      const uint4* src;
+      const uint64_t* so;
+      if (dma) {   // the unit inside its batch: the batch's byte 0 sits at (data + bby[b]) mod 16
+        const uint8_t* bs = a.ring + (size_t)sl * a.bslot_bytes;
+        const uint64_t q = (((uintptr_t)(a.data + a.bby[b])) & 15) + (base - a.bby[b]);
+        src = reinterpret_cast<const uint4*>(bs + (q & ~15ull));
+        so = reinterpret_cast<const uint64_t*>(bs + a.btext + 64) + (lo - a.brec[b]);
+      } else {
+        const uint8_t* slot = a.ring + (size_t)sl * a.slot_bytes;
+        src = reinterpret_cast<const uint4*>(slot);
+        so = reinterpret_cast<const uint64_t*>(slot + a.UB + 32);
       }
+      for (uint32_t k = tid; k < nw; k += blockDim.x) reinterpret_cast<uint4*>(txt_s)[k] = __ldcg(src + k);
+      if (a.off)
+        for (uint32_t j = tid; j < nrec; j += blockDim.x) offs[j] = __ldcg(so + j);
     }
     __syncthreads();
-    if (tid == 0) st_release(&a.done[sl], (unsigned long long)u + 1);   // slot free for unit u + R
+    if (tid == 0) {
+      if (!dma) {
+        st_release(&a.done[sl], (unsigned long long)u + 1);   // slot free for unit u + R
+      } else if (atomicAdd(&a.bcnt[sl], 1u) + 1 == a.bunits[b]) {
+        a.bcnt[sl] = 0;                                       // last unit of the batch out of the slot:
+        st_release(&a.done[sl], (unsigned long long)b + 1);  // the DMA of batch b + K may refill it
+      }
+    }
     // ---- stage 1 (record boundaries -> break bits) + stage 4, word-parallel. Positions q are
     // relative to the 16-B-aligned copy (the unit's byte 0 at q = sh0). Two bitmaps over the unit:
     //   Dm: byte q is a delimiter (or outside the unit), Bm: a record starts at q (a word break, A10/A19);
@@ -919,7 +947,9 @@ __global__ void __launch_bounds__(kKmThreads) k_kmeans(Chunk c, const uint8_t* _
     const uint8_t* piece = ts.acquire(nw, np, nK);
     const uint32_t r0 = ts.p * kKmRows;
     const uint32_t j1 = min(min(ts.K, r0 + kKmRows) / 4, d.nrec);
-    for (uint32_t j = r0 / 4; j < j1; ++j) {
+    const uint32_t jw = __reduce_max_sync(kFull, j1);   // warp-uniform trip count (lanes past j1 idle)
+    for (uint32_t j = r0 / 4; j < jw; ++j) {
+      const bool valid = j < j1;
       float x[16];
 #pragma unroll
       for (int w = 0; w < 4; ++w) {
@@ -946,11 +976,34 @@ __global__ void __launch_bounds__(kKmThreads) k_kmeans(Chunk c, const uint8_t* _
         const float a0 = km_dist(x, s_mu + k * 16);
         if (k == 0 || a0 < bestd) { bestd = a0; best = k; }
       }
-      atomicAdd(&s_cnt[best], 1u);
+      // warp aggregation by cluster: lanes that chose the same centroid form a group; its leader pulls
+      // the members' coordinates (one fp32 shuffle each, summed exactly in fp64) and makes the group's
+      // 16 shared fp64 adds — no intra-warp contention on one cluster's sums, fewer CAS loops
+      const unsigned vmask = __ballot_sync(kFull, valid);
+      const unsigned grp = __match_any_sync(kFull, valid ? best : 0xffffffffu) & vmask;
+      const bool leader = valid && lane == __ffs(grp) - 1;
+      unsigned others = leader ? grp & ~(1u << lane) : 0u;
+      double acc[16];
 #pragma unroll
-      for (int q = 0; q < 16; ++q) atomicAdd(&s_sum[best * 16 + q], widen(x[q]));
-      chk += mix64(((first_index + d.first + j) << 8) ^ (uint64_t)best);
-      if (cid_out) cid_out[d.first + j - c.lo] = (int32_t)best;
+      for (int q = 0; q < 16; ++q) acc[q] = widen(x[q]);
+      while (__any_sync(kFull, others != 0)) {
+        const int src = others ? __ffs(others) - 1 : (int)lane;
+        others &= others - 1;
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+          const float y = __shfl_sync(kFull, x[q], src);
+          if (src != (int)lane) acc[q] += widen(y);
+        }
+      }
+      if (leader) {
+        atomicAdd(&s_cnt[best], (unsigned)__popc(grp));
+#pragma unroll
+        for (int q = 0; q < 16; ++q) atomicAdd(&s_sum[best * 16 + q], acc[q]);
+      }
+      if (valid) {
+        chk += mix64(((first_index + d.first + j) << 8) ^ (uint64_t)best);
+        if (cid_out) cid_out[d.first + j - c.lo] = (int32_t)best;
+      }
     }
     ts.release(nw, np, nK);
   }
@@ -986,9 +1039,20 @@ cudaError_t launch_wc_fused(const uint8_t* data, uint64_t nbytes, const uint64_t
                             const uint64_t* ub, const uint64_t* uby, uint32_t U, uint32_t UB, uint32_t UR, int grid,
                             uint32_t n_load, uint8_t* ring, uint32_t R, unsigned long long* ready,
                             unsigned long long* done, WcEntry* table, uint64_t mask, unsigned long long* used,
-                            int* err, unsigned long long* prof, cudaStream_t s) {
+                            int* err, unsigned long long* prof, const FusedDma* dma, cudaStream_t s) {
   FusedArgs a{data, nbytes, off, rec_size, ub, uby, U, UB, UR, n_load, ring, R, wc_fused_slot_bytes(UB, UR),
               ready, done, table, mask, used, err, prof};
+  if (dma) {
+    a.n_load = 0;
+    a.ubatch = dma->ubatch;
+    a.bby = dma->bby;
+    a.brec = dma->brec;
+    a.bunits = dma->bunits;
+    a.K = dma->K;
+    a.bslot_bytes = dma->bslot_bytes;
+    a.btext = dma->btext;
+    a.bcnt = dma->bcnt;
+  }
   // cooperative: every CTA is co-resident (loaders and consumers wait on each other)
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(grid);

@@ -177,6 +177,11 @@ struct bk_ctx {  // the opaque context of include/bk.h
   bk::rt::DevBuf b_h1, b_h2;                 // word-count key hashes (multi-GPU merge keys)
   bk::rt::DevBuf b_units;                    // BK_GATHER_FUSED unit plan (record bounds, byte bounds)
   bk::rt::DevBuf b_flags;                    //   ring ready / done flags
+  bk::rt::DevBuf b_batch;                    //   DMA feed: batch plan (byte / record bounds, unit -> batch)
+  std::string batch_key;
+  uint64_t n_batches = 0;
+  std::vector<uint64_t> h_bby, h_brec;
+  cudaEvent_t ev_fused = nullptr;
   std::string units_key;                     //   which plan b_units holds
   uint64_t n_units = 0;
   unsigned long long* d_fprof = nullptr;     //   in-kernel wait / compute counters

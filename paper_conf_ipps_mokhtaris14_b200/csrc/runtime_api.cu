@@ -133,7 +133,8 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
   if (cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "d2h stream"));
   if (configure_partition_kernels() != cudaSuccess || configure_baseline_kernels() != cudaSuccess)
     return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
-  if (cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess)
+  if (cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_fused, cudaEventDisableTiming) != cudaSuccess)
     return cleanup(fail(BK_E_CUDA, "events"));
   c->ev_join.assign(3 + 2 * c->cfg.n_slots, nullptr);
   for (auto& e : c->ev_join)
@@ -245,6 +246,7 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
   c->registered = true;
   c->plan_cache.clear();
   c->units_key.clear();
+  c->batch_key.clear();
   drop_graphs(c);
   c->st.ms_register = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return BK_OK;
@@ -463,6 +465,7 @@ int bk_destroy(bk_ctx* c) {
   for (cudaEvent_t e : c->prof) cudaEventDestroy(e);
   drop_graphs(c);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_fused) cudaEventDestroy(c->ev_fused);
   for (auto e : c->ev_join) cudaEventDestroy(e);
   if (c->h_mu) cudaFreeHost(c->h_mu);
   delete c->pool;
@@ -475,7 +478,7 @@ int bk_destroy(bk_ctx* c) {
   release_kept_outputs(c);
   release_addr_side(c);
   for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base, &c->b_h1, &c->b_h2, &c->b_mown, &c->b_mcnt,
-                    &c->b_mctr, &c->b_units, &c->b_flags})
+                    &c->b_mctr, &c->b_units, &c->b_flags, &c->b_batch})
     b->release();
   for (auto* h : c->hstage) cudaFreeHost(h);
   for (auto e : c->h_done) cudaEventDestroy(e);

@@ -3,6 +3,8 @@
 // baseline and the experiment kernels (layout dump, pattern statistics).
 #include "runtime.cuh"
 
+#include <cuda.h>   // CUstream / CUdeviceptr types of the stream memory operations
+
 namespace bk {
 namespace rt {
 
@@ -60,6 +62,33 @@ static int fused_units(bk_ctx* c, uint32_t UB, uint32_t UR, std::vector<uint64_t
   return BK_OK;
 }
 
+// Stream memory operations (driver API through the runtime's entry-point query, no -lcuda): the
+// copy stream writes a flag after each batch's DMA and waits for the consumers' release flag — the
+// paper's "DMA a flag right after the data" and its buffer-reuse distance.
+namespace {
+using PfnStreamValue64 = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+struct MemOps {
+  bool tried = false;
+  PfnStreamValue64 write = nullptr, wait = nullptr;
+};
+MemOps& memops() {
+  static MemOps m;
+  if (!m.tried) {
+    m.tried = true;
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuStreamWriteValue64", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      m.write = reinterpret_cast<PfnStreamValue64>(f);
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue64", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      m.wait = reinterpret_cast<PfnStreamValue64>(f);
+    cudaGetLastError();
+  }
+  return m;
+}
+}  // namespace
+
 // Word count as one persistent launch (BK_GATHER_FUSED, kernels_compute.cu k_wc_fused): loader
 // CTAs stream units into an HBM ring carved from the window, consumer CTAs count. Returns
 // BK_E_RANGE (nothing enqueued) when the window cannot hold a ring of >= 2 units or a record does
@@ -95,26 +124,105 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
     c->units_key = ukey;
   }
   if (!c->d_fprof) BK_CUDA(cudaMalloc(&c->d_fprof, 8 * 8));
-  BK_CUDA(c->b_flags.ensure(2 * R * 8));
+  // feed: "zc" (default): loader CTAs stream units with zero-copy loads; "dma" (BK_FUSED_FEED=dma):
+  // the copy engine fills K batch slots, each followed by a stream-ordered flag, every CTA consumes.
+  // Measured on the C1 config (profiles/r02_wc_fused.md): zc 1.74 ms/step, dma 1.88 (K=2) - 2.15 (K=4):
+  // the batch-granular release leaves the copy engine waiting at every batch boundary.
+  const char* fe = getenv("BK_FUSED_FEED");
+  const bool dma = fe && strcmp(fe, "dma") == 0 && memops().write && memops().wait;
+  uint32_t K = 3;
+  if (const char* e = getenv("BK_FUSED_BATCHES")) K = (uint32_t)std::max(2, std::min(8, atoi(e)));
+  const uint64_t bslot = c->cfg.window_bytes / K / 256 * 256;
+  const uint64_t btext = (bslot * 7 / 8 - 64) / 16 * 16;
+  const uint64_t brecs = (bslot - btext - 64) / 8;
+  FusedDma fd{};
+  if (dma) {
+    if (btext < UB || brecs < UR) return BK_E_RANGE;
+    const std::string bkey = ukey + "/" + std::to_string(K) + "/" + std::to_string(bslot);
+    if (c->batch_key != bkey) {
+      const uint64_t* hub = nullptr;
+      std::vector<uint64_t> ubh(c->n_units + 1), ubyh(c->n_units + 1);
+      BK_CUDA(cudaMemcpy(ubh.data(), c->b_units.p, ubh.size() * 8, cudaMemcpyDeviceToHost));
+      BK_CUDA(cudaMemcpy(ubyh.data(), (uint64_t*)c->b_units.p + ubh.size(), ubh.size() * 8, cudaMemcpyDeviceToHost));
+      (void)hub;
+      std::vector<uint32_t> ubatch(c->n_units), bunits;
+      std::vector<uint64_t> bby{0}, brec{0};
+      uint64_t u0 = 0;
+      while (u0 < c->n_units) {   // greedy: consecutive units while the batch's bytes and records fit a slot
+        uint64_t u1 = u0 + 1;
+        while (u1 < c->n_units && ubyh[u1 + 1] - ubyh[u0] + 16 <= btext && ubh[u1 + 1] - ubh[u0] <= brecs) ++u1;
+        for (uint64_t u = u0; u < u1; ++u) ubatch[u] = (uint32_t)bunits.size();
+        bunits.push_back((uint32_t)(u1 - u0));
+        bby.push_back(ubyh[u1]);
+        brec.push_back(ubh[u1]);
+        u0 = u1;
+      }
+      c->n_batches = bunits.size();
+      c->h_bby = bby;
+      c->h_brec = brec;
+      const size_t NB = c->n_batches;
+      BK_CUDA(c->b_batch.ensure(c->n_units * 4 + NB * 4 + 2 * (NB + 1) * 8 + 64));
+      uint8_t* q = (uint8_t*)c->b_batch.p;
+      BK_CUDA(cudaMemcpy(q, bby.data(), (NB + 1) * 8, cudaMemcpyHostToDevice));
+      BK_CUDA(cudaMemcpy(q + (NB + 1) * 8, brec.data(), (NB + 1) * 8, cudaMemcpyHostToDevice));
+      BK_CUDA(cudaMemcpy(q + 2 * (NB + 1) * 8, ubatch.data(), c->n_units * 4, cudaMemcpyHostToDevice));
+      BK_CUDA(cudaMemcpy(q + 2 * (NB + 1) * 8 + c->n_units * 4, bunits.data(), NB * 4, cudaMemcpyHostToDevice));
+      c->batch_key = bkey;
+    }
+    uint8_t* q = (uint8_t*)c->b_batch.p;
+    const size_t NB = c->n_batches;
+    fd.bby = (const uint64_t*)q;
+    fd.brec = (const uint64_t*)(q + (NB + 1) * 8);
+    fd.ubatch = (const uint32_t*)(q + 2 * (NB + 1) * 8);
+    fd.bunits = (const uint32_t*)(q + 2 * (NB + 1) * 8 + c->n_units * 4);
+    fd.K = K;
+    fd.bslot_bytes = bslot;
+    fd.btext = btext;
+  }
+  BK_CUDA(c->b_flags.ensure(2 * std::max<uint64_t>(R, K) * 8 + K * 4 + 64));
   const uint64_t U = c->n_units;
   const uint64_t* ubd = (const uint64_t*)c->b_units.p;
+  const uint64_t NF = dma ? K : R;   // flags per direction
   unsigned long long* ready = (unsigned long long*)c->b_flags.p;
+  fd.bcnt = (unsigned int*)(ready + 2 * NF);
   const bool prof = (c->cfg.flags & BK_FLAG_PROFILE) != 0;
   WcEntry* table = (WcEntry*)c->b_table.p;
   // captured once per (table, units, ring, loaders) and replayed: two memsets, the cooperative
   // persistent kernel, the compaction
   const std::string key = "wcfused/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + ukey + "/" +
                           std::to_string(R) + "/" + std::to_string(n_load);
-  int rc = run_device(c, stream, key, true, 1, [&]() -> int {
+  // the DMA feed issues eagerly (stream memory operations are not graph-captured here)
+  int rc = run_device(c, stream, key + (dma ? "/dma" : "/zc"), !dma, 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
-    BK_CUDA(cudaMemsetAsync(ready, 0, 2 * R * 8, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(ready, 0, 2 * NF * 8 + K * 4, c->s_comp));
     if (prof) BK_CUDA(cudaMemsetAsync(c->d_fprof, 0, 8 * 8, c->s_comp));
+    if (dma) {   // the copy stream starts after the flags are cleared
+      BK_CUDA(cudaEventRecord(c->ev_fused, c->s_comp));
+      BK_CUDA(cudaStreamWaitEvent(c->s_copy, c->ev_fused, 0));
+    }
     BK_PROF(kStGather, c->s_comp, true);
     BK_CUDA(launch_wc_fused(c->host_dev, c->nbytes, c->off ? c->off_dev : nullptr, c->off ? 0 : c->cfg.record_size,
-                            ubd, ubd + U + 1, (uint32_t)U, (uint32_t)UB, UR, grid, n_load, c->window, (uint32_t)R,
-                            ready, ready + R, table, slots - 1, c->d_ctr + 1, c->d_err, prof ? c->d_fprof : nullptr,
-                            c->s_comp));
+                            ubd, ubd + U + 1, (uint32_t)U, (uint32_t)UB, UR, grid, dma ? 0 : n_load, c->window,
+                            (uint32_t)R, ready, ready + NF, table, slots - 1, c->d_ctr + 1, c->d_err,
+                            prof ? c->d_fprof : nullptr, dma ? &fd : nullptr, c->s_comp));
     BK_PROF(kStGather, c->s_comp, false);
+    if (dma) {   // per batch: [wait for the slot's release] -> DMA text + offsets -> flag (stream order)
+      const MemOps& mo = memops();
+      for (size_t b = 0; b < c->n_batches; ++b) {
+        const uint64_t sl = b % K;
+        uint8_t* slot = c->window + sl * bslot;
+        if (b >= K && mo.wait((CUstream)c->s_copy, (CUdeviceptr)(ready + NF + sl), b - K + 1, CU_STREAM_WAIT_VALUE_GEQ))
+          return fail(BK_E_CUDA, "cuStreamWaitValue64");
+        const uint64_t b0 = c->h_bby[b], b1 = c->h_bby[b + 1];
+        BK_CUDA(cudaMemcpyAsync(slot + (((uintptr_t)(c->host_dev + b0)) & 15), c->host + b0, b1 - b0,
+                                cudaMemcpyHostToDevice, c->s_copy));
+        if (c->off)
+          BK_CUDA(cudaMemcpyAsync(slot + btext + 64, c->off + c->h_brec[b], (c->h_brec[b + 1] - c->h_brec[b]) * 8,
+                                  cudaMemcpyHostToDevice, c->s_copy));
+        if (mo.write((CUstream)c->s_copy, (CUdeviceptr)(ready + sl), b + 1, CU_STREAM_WRITE_VALUE_DEFAULT))
+          return fail(BK_E_CUDA, "cuStreamWriteValue64");
+      }
+    }
     launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
                       (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p, ocap, c->s_comp);
     c->n_launch += 2;
@@ -134,8 +242,8 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
   c->st.n_units = U;
   c->st.unit_bytes = (uint32_t)UB;
   c->st.fused_grid = (uint32_t)grid;
-  c->st.fused_loaders = n_load;
-  c->st.fused_ring_slots = (uint32_t)R;
+  c->st.fused_loaders = dma ? 0 : n_load;
+  c->st.fused_ring_slots = dma ? K : (uint32_t)R;
   c->st.fused_wait_frac = c->st.fused_compute_frac = c->st.fused_loader_wait_frac = 0;
   if (prof) {
     unsigned long long fp[5] = {0, 0, 0, 0, 0};
