@@ -258,12 +258,16 @@ DTYPE = {"grep": "u8", "wordcount": "u8 (u64 hashes, u64 counts)", "groupby": "u
 
 
 def load_traffic() -> dict:
-    """Per-unit traffic of the roofline kernels from one ncu --set full capture each (committed)."""
-    try:
-        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r01_traffic.json")) as f:
-            return json.load(f)
-    except (OSError, ValueError):
-        return {}
+    """Per-unit traffic of the roofline kernels from one ncu --set full capture each (committed;
+    the latest round's file wins per workload)."""
+    out = {}
+    for name in ("r01_traffic.json", "r02_traffic.json"):
+        try:
+            with open(os.path.join(ROOT, "profiles", name)) as f:
+                out.update(json.load(f))
+        except (OSError, ValueError):
+            pass
+    return out
 
 
 def load_peaks():
@@ -655,7 +659,15 @@ def main():
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["traffic"] = None
     tr = load_traffic().get(args.workload)
-    if tr and ((dom == "zc" and tr["unit"] == "record") or (dom == "compute")):
+    if tr and tr.get("kernel", "").endswith("k_wc_fused") != (dom == "fused"):
+        tr = None   # a capture of another kernel than this line's roofline kernel
+    if tr and dom == "fused":
+        units = st["bytes_accessed"]
+        roof["traffic"] = tr["traffic_per_unit"] * units
+        roof["traffic_source"] = (f"{tr['what']} of {tr['kernel']}, ncu --set full ({tr['capture']}): "
+                                  f"{tr['traffic_per_unit']:.3f} B per text byte x {units} bytes per launch; "
+                                  f"algorithmic bytes per launch {per_launch:.0f} (text + offsets)")
+    elif tr and ((dom == "zc" and tr["unit"] == "record") or (dom == "compute")):
         # bytes one launch moves, measured by ncu --set full on one launch of the same kernel
         # (profiles/r01_traffic.json, tools/gpu_traffic.sh), scaled to this run's units per launch
         if dom == "zc":

@@ -88,7 +88,143 @@ __global__ void k_kmer_compact(const KmerEntry* __restrict__ table, uint64_t slo
   }
 }
 
+// ---- two-phase counting (round 2): the table is split into R = 2^rb regions of S slots; a k-mer's
+// region is the top rb bits of mix64(key), its home slot the low bits. Phase A (stage 4, per chunk)
+// appends every k-mer window's key to its region's bucket in HBM (one L2 atomic on the bucket cursor
+// + one 8-B store; the L2 merges a bucket's consecutive appends into whole sectors). Phase B (flush)
+// gives each region to one CTA: the region is loaded into shared memory (S x 16 B <= 128 KiB), the
+// bucket's keys are counted with shared-memory atomics and the region is written back — DRAM traffic
+// ~24 B per k-mer (8 B appended, 8 B read back, the table read and written once per flush) instead of
+// a random 16-B table entry per k-mer (~146 B of DRAM per update measured in round 1). A bucket that
+// fills up sends the rest of its keys straight to the region in HBM (same slots), so any input is
+// counted exactly.
+
+__device__ __forceinline__ void region_insert(KmerEntry* region, uint64_t smask, uint64_t h,
+                                              unsigned long long key, unsigned long long cnt, int* err) {
+  uint64_t slot = h & smask;
+  for (uint64_t probe = 0; probe <= smask; ++probe, slot = (slot + 1) & smask) {
+    unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(&region[slot].key);
+    if (k == 0) k = atomicCAS(&region[slot].key, 0ull, key);
+    if (k == 0 || k == key) {
+      atomicAdd(&region[slot].count, cnt);
+      return;
+    }
+  }
+  atomicOr(err, kErrTableFull);
+}
+
+__global__ void __launch_bounds__(256) k_kmer_scatter(Chunk c, const uint8_t* __restrict__ stage,
+                                                      const LaneDesc* __restrict__ lanes,
+                                                      const uint64_t* __restrict__ tile_base, uint32_t k,
+                                                      uint32_t seq_words, KmerEntry* table, uint32_t rb,
+                                                      uint64_t smask, unsigned long long* __restrict__ bbuf,
+                                                      unsigned int* __restrict__ bcur, uint32_t bcap,
+                                                      unsigned long long* total, int* err) {
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= c.L) return;  // whole warps
+  const int lane = t & 31;
+  const LaneDesc d = lanes[t];
+  const uint8_t* tile = stage + tile_base[t >> 5];
+  const uint32_t R = __reduce_max_sync(kFull, d.nrec);
+  const uint64_t kmask = k == 32 ? ~0ull : ((1ull << (2 * k)) - 1);
+  unsigned long long mine = 0;
+  for (uint32_t j = 0; j < R; ++j) {
+    const bool rec = j < d.nrec;
+    uint64_t v = 0;
+    uint32_t valid = 0;
+    for (uint32_t w = 0; w < seq_words; ++w) {
+      uint4 q = make_uint4(0, 0, 0, 0);
+      if (rec) q = *reinterpret_cast<const uint4*>(tile + ((size_t)(j * seq_words + w) * 32 + lane) * 16);
+      const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+      for (int b = 0; b < 16; ++b) {
+        const uint32_t ch = (wd[b >> 2] >> (8 * (b & 3))) & 0xff;
+        const int code = ch == 'A' ? 0 : ch == 'C' ? 1 : ch == 'G' ? 2 : ch == 'T' ? 3 : -1;
+        if (code < 0) {
+          valid = 0;
+          v = 0;
+        } else {
+          v = ((v << 2) | (uint64_t)code) & kmask;
+          ++valid;
+        }
+        if (rec && valid >= k) {
+          const unsigned long long key = v + 1;
+          const uint64_t h = mix64(key);
+          const uint32_t r = rb ? (uint32_t)(h >> (64 - rb)) : 0u;
+          const unsigned pos = atomicAdd(&bcur[r], 1u);
+          if (pos < bcap) bbuf[(size_t)r * bcap + pos] = key;
+          else region_insert(table + (size_t)r * (smask + 1), smask, h, key, 1ull, err);   // bucket full
+          ++mine;
+        }
+      }
+    }
+  }
+  mine = __reduce_add_sync(kFull, (unsigned)mine);
+  if (lane == 0 && mine) atomicAdd(total, mine);
+}
+
+// one CTA per region: region -> shared memory, count its bucket, write back, reset the cursor
+__global__ void __launch_bounds__(512) k_kmer_flush(KmerEntry* table, uint32_t rb, uint64_t smask,
+                                                   const unsigned long long* __restrict__ bbuf,
+                                                   unsigned int* __restrict__ bcur, uint32_t bcap, int* err) {
+  extern __shared__ __align__(16) unsigned char km_smem[];
+  KmerEntry* sreg = reinterpret_cast<KmerEntry*>(km_smem);
+  const uint32_t r = blockIdx.x;
+  const uint64_t S = smask + 1;
+  KmerEntry* region = table + (size_t)r * S;
+  const uint32_t n = min(bcur[r], bcap);
+  if (n == 0) {   // nothing appended: the region in HBM is already current
+    __syncthreads();
+    if (threadIdx.x == 0) bcur[r] = 0;
+    return;
+  }
+  for (uint64_t i = threadIdx.x; i < S; i += blockDim.x)
+    reinterpret_cast<ulonglong2*>(sreg)[i] = reinterpret_cast<const ulonglong2*>(region)[i];
+  __syncthreads();
+  const unsigned long long* keys = bbuf + (size_t)r * bcap;
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const unsigned long long key = keys[i];
+    const uint64_t h = mix64(key);
+    uint64_t slot = h & smask;
+    bool done = false;
+    for (uint64_t probe = 0; probe <= smask; ++probe, slot = (slot + 1) & smask) {
+      unsigned long long kk = sreg[slot].key;
+      if (kk == 0) kk = atomicCAS(&sreg[slot].key, 0ull, key);
+      if (kk == 0 || kk == key) {
+        atomicAdd(&sreg[slot].count, 1ull);
+        done = true;
+        break;
+      }
+    }
+    if (!done) atomicOr(err, kErrTableFull);
+  }
+  __syncthreads();
+  for (uint64_t i = threadIdx.x; i < S; i += blockDim.x)
+    reinterpret_cast<ulonglong2*>(region)[i] = reinterpret_cast<const ulonglong2*>(sreg)[i];
+  if (threadIdx.x == 0) bcur[r] = 0;
+}
+
 }  // namespace
+
+size_t kmer_flush_smem(uint64_t region_slots) { return (size_t)region_slots * sizeof(KmerEntry); }
+
+void launch_kmer_scatter(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                         uint32_t k, uint32_t seq_words, KmerEntry* table, uint32_t rb, uint64_t region_slots,
+                         unsigned long long* bbuf, unsigned int* bcur, uint32_t bcap, unsigned long long* total,
+                         int* err, cudaStream_t s) {
+  k_kmer_scatter<<<(c.L + 255) / 256, 256, 0, s>>>(c, stage, lanes, tile_base, k, seq_words, table, rb,
+                                                    region_slots - 1, bbuf, bcur, bcap, total, err);
+}
+
+void launch_kmer_flush(KmerEntry* table, uint32_t rb, uint64_t region_slots, const unsigned long long* bbuf,
+                       unsigned int* bcur, uint32_t bcap, int* err, cudaStream_t s) {
+  k_kmer_flush<<<1u << rb, 512, kmer_flush_smem(region_slots), s>>>(table, rb, region_slots - 1, bbuf, bcur, bcap,
+                                                                      err);
+}
+
+cudaError_t configure_kmer_kernels() {
+  return cudaFuncSetAttribute((const void*)k_kmer_flush, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+}
 
 void launch_kmer(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base, uint32_t k,
                  uint32_t seq_words, KmerEntry* table, uint64_t mask, unsigned long long* used,

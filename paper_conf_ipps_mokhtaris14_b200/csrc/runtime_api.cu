@@ -131,7 +131,8 @@ int bk_create(const bk_config* cfg, bk_ctx** out_ctx) {
     return cleanup(fail(BK_E_NOMEM, "cudaHostAlloc counters"));
   c->slots.resize(c->cfg.n_slots);
   if (cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return cleanup(fail(BK_E_CUDA, "d2h stream"));
-  if (configure_partition_kernels() != cudaSuccess || configure_baseline_kernels() != cudaSuccess)
+  if (configure_partition_kernels() != cudaSuccess || configure_baseline_kernels() != cudaSuccess ||
+      configure_kmer_kernels() != cudaSuccess)
     return cleanup(fail(BK_E_CUDA, "cudaFuncSetAttribute"));
   if (cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev_fused, cudaEventDisableTiming) != cudaSuccess)

@@ -462,7 +462,9 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   return BK_OK;
 }
 
-// f4: k-mer counting (FIELD access to the sequence; the table is resident, outside the window)
+// f4: k-mer counting (FIELD access to the sequence; the table is resident, outside the window).
+// Two-phase (kernels_kmer.cu): per chunk every k-mer key is appended to its table region's bucket,
+// and flushes count whole buckets into their regions in shared memory.
 int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   const uint64_t slots = o->table_slots ? o->table_slots : (1ull << 24);
   if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
@@ -478,19 +480,44 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
   BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
   KmerEntry* table = (KmerEntry*)c->b_table.p;
+  // regions of <= 8192 slots (128 KiB of shared memory in the flush); buckets sized for the run's
+  // k-mer windows (an upper bound: every window of every record valid) within 16 GiB, else flushed
+  // every F chunks; a full bucket falls back to direct inserts
+  const uint64_t S = std::min<uint64_t>(slots, 8192);
+  uint32_t rb = 0;
+  while ((S << rb) < slots) ++rb;
+  const uint64_t R = 1ull << rb;
+  const uint64_t wpr = o->seq_len >= o->k ? o->seq_len - o->k + 1 : 0;   // windows per record (bound)
+  const uint64_t bound = c->n * wpr;
+  const uint64_t budget = std::min<uint64_t>(16ull << 30, (uint64_t)(bound * 1.15) * 8 + R * 8192 + 8);
+  const uint32_t bcap = (uint32_t)std::min<uint64_t>(budget / 8 / R, 0xffffffffull);
+  uint64_t per_chunk = 0;
+  for (size_t i = 0; i + 1 < p.bounds.size(); ++i) per_chunk = std::max<uint64_t>(per_chunk, (p.bounds[i + 1] - p.bounds[i]) * wpr);
+  const uint64_t F = per_chunk ? std::max<uint64_t>(1, (uint64_t)(0.8 * bcap * R) / per_chunk) : 1;
+  BK_CUDA(c->b_blk.ensure((uint64_t)bcap * R * 8));
+  BK_CUDA(c->b_blk2.ensure(R * 4));
+  unsigned long long* bbuf = (unsigned long long*)c->b_blk.p;
+  unsigned int* bcur = (unsigned int*)c->b_blk2.p;
   const std::string key = "kmer/" + std::to_string(o->k) + "/" + std::to_string(slots) + "/" + std::to_string(ocap) +
                           "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(KmerEntry), c->s_comp));
-    int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
-      launch_kmer(ch, s.stage, s.lanes, s.tile_base, o->k, o->seq_len / 16, table, slots - 1, c->d_ctr + 1,
-                  c->d_ctr + 5, c->d_err, cs);
+    BK_CUDA(cudaMemsetAsync(bcur, 0, R * 4, c->s_comp));
+    size_t ci = 0;
+    int r = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_kmer_scatter(ch, s.stage, s.lanes, s.tile_base, o->k, o->seq_len / 16, table, rb, S, bbuf, bcur, bcap,
+                          c->d_ctr + 5, c->d_err, cs);
       c->n_launch += 1;
+      if (++ci % F == 0 && ci + 1 < p.bounds.size()) {   // buckets near full: count them now
+        launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, c->d_err, cs);
+        c->n_launch += 1;
+      }
       return BK_OK;
     });
     if (r) return r;
+    launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, c->d_err, c->s_comp);
     launch_kmer_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint64_t*)c->b_out3.p, ocap, c->s_comp);
-    c->n_launch += 1;
+    c->n_launch += 2;
     return (int)BK_OK;
   });
   if (rc) return rc;

@@ -1,0 +1,37 @@
+#!/bin/bash
+# Round-2 evidence on one box (run through gpurun): every bench line (JSON -> gpurun_out/r02e_*),
+# the reference arm, ncu launch lists of the headline lines, the traffic captures behind
+# roofline.traffic, the sanitizers on the round-2 paths, measured Table II.
+# Copy what is judged into profiles/ afterwards (tools/README.md).
+mkdir -p gpurun_out
+T=${TAG:-r02z}
+line() {  # name bench-args...
+  name=$1; shift
+  timeout 1500 python bench.py "$@" > gpurun_out/${T}_bench_$name.json 2> gpurun_out/${T}_bench_$name.err
+  python3 -c "import json;d=json.loads(open('gpurun_out/${T}_bench_$name.json').read().splitlines()[-1]);print('$name', d['value'], d['ms_per_step'], round(d['roofline']['frac'],3), d['link']['frac'])" \
+    || tail -3 gpurun_out/${T}_bench_$name.err
+}
+line grep --steps 10 --warmup 3
+line wordcount --workload wordcount --steps 20 --warmup 5
+line groupby --workload groupby --steps 3 --warmup 3
+line groupby32 --workload groupby --gib 32 --steps 3 --warmup 3
+line groupby_sparse --workload groupby_sparse --steps 3 --warmup 3
+line kmeans --workload kmeans --steps 3 --warmup 3
+line kmeans256 --workload kmeans --K 256 --steps 3 --warmup 3 --no-dbuf
+line partition --workload partition --steps 3 --warmup 3
+line kmer --workload kmer --steps 3 --warmup 3
+line grep_addr --gather addr --gib 2 --steps 3 --warmup 3 --no-cpu-baseline --no-dbuf
+timeout 900 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/${T}_bench_reference.json 2> gpurun_out/${T}_bench_reference.err
+tail -c 300 gpurun_out/${T}_bench_reference.json
+# launch lists (serialised, cold): each kernel's share of the step
+for w in grep wordcount kmer; do
+  timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv \
+      --log-file gpurun_out/${T}_launches_$w.csv python bench.py --workload $w --steps 2 --warmup 1 \
+      --no-cpu-baseline --no-dbuf --no-profile --no-trace --gib $([ $w = grep ] && echo 2 || ([ $w = kmer ] && echo 1 || echo 0.0625)) \
+      > /dev/null 2>&1
+  echo "launches $w rc=$?"
+done
+TAG=${T} bash tools/gpu_traffic.sh
+TAG=${T} bash tools/sanitize.sh
+timeout 1200 python tools/table2_measured.py > gpurun_out/${T}_table2.jsonl 2> gpurun_out/${T}_table2.err
+echo table2 rc=$?

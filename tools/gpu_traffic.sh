@@ -4,8 +4,8 @@
 # tools/traffic_json.py turns them into profiles/r01_traffic.json, which bench.py scales into
 # roofline.traffic.
 mkdir -p gpurun_out
-TAG=${TAG:-r01x}
-B="python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-dbuf --no-profile"
+TAG=${TAG:-r02x}
+B="python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-dbuf --no-profile --no-trace"
 cap() {  # name kernel-regex skip bench-args
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$2" -s $3 -c 1 \
       -o gpurun_out/${TAG}_tr_$1 $B $4 > gpurun_out/${TAG}_tr_$1.json 2> gpurun_out/${TAG}_tr_$1.err
@@ -13,5 +13,5 @@ cap() {  # name kernel-regex skip bench-args
 }
 cap grep "k_gather_field" 6 "--workload grep --gib 4 --zc-share 1000"
 cap groupby_sparse "k_gather_field" 6 "--workload groupby_sparse --gib 4 --zc-share 1000"
-cap wordcount "k_wc" 40 "--workload wordcount --gather zc"
-cap kmer "k_kmer" 6 "--workload kmer --gib 1"
+cap wordcount "k_wc_fused" 3 "--workload wordcount"
+cap kmer "k_kmer_scatter" 6 "--workload kmer --gib 1"

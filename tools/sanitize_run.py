@@ -89,3 +89,30 @@ for n in (1, 33):
             if mode != "hybrid":
                 ctx.partition(64)
 print("sanitize run ok")
+# round 2: the fused single-launch word count (zero-copy loaders and the copy-engine feed), address
+# mode (patterns / explicit) incl. a layout dump, the GPU merge of count tables, two-phase k-mers
+import os  # noqa: E402
+for feed in ("zc", "dma"):
+    os.environ["BK_FUSED_FEED"] = feed
+    with bk.Context(window_bytes=256 << 10) as ctx:
+        ctx.register(buf, off)
+        ctx.wordcount(cap=1 << 16)
+        ctx.wordcount(cap=1 << 16)
+os.environ.pop("BK_FUSED_FEED")
+for nop in (False, True):
+    with bk.Context(window_bytes=512 << 10, gather_mode="addr", no_patterns=nop) as ctx:
+        ctx.register(buf, off)
+        ctx.wordcount(cap=1 << 16)
+        ctx.layout_dump(1)
+    with bk.Context(window_bytes=512 << 10, record_size=64, gather_mode="addr", no_patterns=nop) as ctx:
+        ctx.register(g, None, n_records=100_000)
+        ctx.groupby(4096)
+import torch  # noqa: E402
+rows = torch.randint(0, 1 << 20, (3 * 4096, 6), dtype=torch.int64, device="cuda")
+out = torch.empty(3 * 4096, 6, dtype=torch.int64, device="cuda")
+with bk.Context(window_bytes=1 << 20) as ctx:
+    ctx.merge_counts(rows, [4096, 100, 4000], 4096, 6, 3, 3, out)
+with bk.Context(window_bytes=1 << 20, record_size=256, gather_mode="zc") as ctx:
+    ctx.register(d, None, n_records=20_000)
+    ctx.kmer(k=31, table_slots=1 << 16)
+print("sanitize run (round 2) done")

@@ -1,10 +1,10 @@
 #!/usr/bin/env python3
 """Per-unit memory / link traffic of each bench line's roofline kernel, from one ncu --set full
 capture per kernel (tools/gpu_traffic.sh) plus the bench JSON line of the same command (units per
-launch). Writes profiles/r01_traffic.json; bench.py scales it to its own launch size into
+launch). Writes profiles/r02_traffic.json; bench.py scales it to its own launch size into
 roofline.traffic.
 
-    python tools/traffic_json.py r01x > profiles/r01_traffic.json
+    python tools/traffic_json.py r02x > profiles/r02_traffic.json
 """
 import csv
 import io
@@ -42,9 +42,10 @@ def main(tag: str) -> None:
         except Exception as e:  # noqa: BLE001 - report which capture is missing
             print(f"skip {w}: {e}", file=sys.stderr)
             continue
-        chunks = line["config"]["n_chunks"]
+        # launches per step: one per chunk, except the fused word count (one persistent launch)
+        chunks = 1 if line["config"].get("gather_mode") == "fused" else line["config"]["n_chunks"]
         units = (line["config"]["records_per_gpu"] if unit == "record" else line["config"]["bytes_per_gpu"]) / chunks
-        link = w in ("grep", "groupby_sparse")  # zero-copy gathers: the bound is the host link
+        link = w in ("grep", "groupby_sparse", "wordcount")  # zero-copy reads: the bound is the host link
         res[w] = {
             "kernel": k["kernel"], "capture": rep, "launch_ms": k["t"] * 1e3, "unit": unit,
             "units_per_launch": units,
