@@ -711,8 +711,10 @@ def main():
                                  "vs computing while loaders stream later units; loaders waiting for a free ring slot"}
     roof["avg_launch_ms"] = avg_ms
     roof["launches_per_step"] = launches
-    if rank == 0 and st.get("n_chunks_cpu") and args.workload in ("grep", "groupby_sparse") and args.impl == "ours":
-        # the host packers alone (CPU assembly of every chunk, no zero-copy traffic): their rate
+    if args.workload in ("grep", "groupby_sparse") and args.gather in ("auto", "hybrid") and args.impl == "ours" \
+            and not args.no_profile:
+        # the host packers alone (CPU assembly of every chunk, no zero-copy traffic): their rate. Every
+        # rank runs the pass (one_step holds the merge collective), rank 0 reports
         cctx = bk.Context(device=local, window_bytes=window, n_slots=args.slots, gather_mode="cpu",
                           host_threads=args.host_threads, record_size=shard["rec_size"], keep_outputs_pinned=True)
         cctx.register(shard["buf"], shard["off"], n_records=shard["n"])
@@ -721,7 +723,8 @@ def main():
         cst = cctx.stats()
         cctx.close()
         pack_rate = shard["n"] / (cst["ms_cpu_gather"] * 1e-3) if cst["ms_cpu_gather"] else None
-        roof.update(host_rooflines(args, shard, st, t_dev / args.steps, peak_h2d, tr, pack_rate))
+        if rank == 0 and st.get("n_chunks_cpu"):
+            roof.update(host_rooflines(args, shard, st, t_dev / args.steps, peak_h2d, tr, pack_rate))
 
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,

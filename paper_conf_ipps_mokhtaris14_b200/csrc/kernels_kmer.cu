@@ -136,6 +136,11 @@ __global__ void __launch_bounds__(256) k_kmer_scatter(Chunk c, const uint8_t* __
       uint4 q = make_uint4(0, 0, 0, 0);
       if (rec) q = *reinterpret_cast<const uint4*>(tile + ((size_t)(j * seq_words + w) * 32 + lane) * 16);
       const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+      // the word's up to 16 k-mers first, then their 16 independent cursor atomics, then the stores:
+      // one L2 round trip per 16 windows instead of one per window
+      unsigned long long key[16];
+      uint32_t bk[16];
+      uint32_t okm = 0;
 #pragma unroll
       for (int b = 0; b < 16; ++b) {
         const uint32_t ch = (wd[b >> 2] >> (8 * (b & 3))) & 0xff;
@@ -147,16 +152,20 @@ __global__ void __launch_bounds__(256) k_kmer_scatter(Chunk c, const uint8_t* __
           v = ((v << 2) | (uint64_t)code) & kmask;
           ++valid;
         }
-        if (rec && valid >= k) {
-          const unsigned long long key = v + 1;
-          const uint64_t h = mix64(key);
-          const uint32_t r = rb ? (uint32_t)(h >> (64 - rb)) : 0u;
-          const unsigned pos = atomicAdd(&bcur[r], 1u);
-          if (pos < bcap) bbuf[(size_t)r * bcap + pos] = key;
-          else region_insert(table + (size_t)r * (smask + 1), smask, h, key, 1ull, err);   // bucket full
-          ++mine;
-        }
+        key[b] = v + 1;
+        bk[b] = rb ? (uint32_t)(mix64(key[b]) >> (64 - rb)) : 0u;
+        if (rec && valid >= k) okm |= 1u << b;
       }
+      unsigned pos[16];
+#pragma unroll
+      for (int b = 0; b < 16; ++b) pos[b] = (okm >> b & 1) ? atomicAdd(&bcur[bk[b]], 1u) : 0u;
+#pragma unroll
+      for (int b = 0; b < 16; ++b) {
+        if (!(okm >> b & 1)) continue;
+        if (pos[b] < bcap) bbuf[(size_t)bk[b] * bcap + pos[b]] = key[b];
+        else region_insert(table + (size_t)bk[b] * (smask + 1), smask, mix64(key[b]), key[b], 1ull, err);   // full
+      }
+      mine += __popc(okm);
     }
   }
   mine = __reduce_add_sync(kFull, (unsigned)mine);

@@ -195,6 +195,7 @@ struct bk_ctx {  // the opaque context of include/bk.h
   std::vector<uint64_t> a_epos, a_tbase;
   std::vector<bk::trace::Rec> trace_recs;    // BK_FLAG_TRACE: this run's CUPTI records
   bool tracing = false;
+  double hy_t_zc_ms = 0, hy_t_cpu_ms = 0;    // HYBRID: measured ms per zero-copy / host-packed chunk
   bk_addr_fn a_gen = nullptr;                // bk_run_user_addr generator + its argument
   void* a_gen_user = nullptr;
   bk::rt::DevBuf b_mown, b_mcnt, b_mctr;     // bk_merge_counts scratch (never captured in a graph)
@@ -288,7 +289,8 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
   // with few host cores (8 ranks on one host) lets the GPU gather more and never waits on slow packers.
   std::vector<Slot*> zc_inflight;
   size_t zc_depth = 1;
-  double t_zc_ms = 0, t_cpu_ms = 0;   // running estimates
+  double& t_zc_ms = c->hy_t_zc_ms;    // running estimates, kept across runs of one registration
+  double& t_cpu_ms = c->hy_t_cpu_ms;
   if (p.mode == BK_GATHER_CPU || p.mode == BK_GATHER_HYBRID || p.mode == BK_GATHER_ADDR) {
     int rc = ensure_host_side(c, p);
     if (!rc && p.mode == BK_GATHER_ADDR) rc = ensure_addr_side(c, p);
@@ -317,6 +319,9 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
       if (t_zc_ms > 0 && t_cpu_ms > 0)
         zc_depth = (size_t)std::max<long>(1, std::min<long>((long)c->cfg.n_slots - 1, std::lround(t_cpu_ms / t_zc_ms)));
       cpu = zc_inflight.size() >= zc_depth;
+      // a packed chunk earns one chunk per t_cpu but idles the link for t_cpu - (N-1) t_zc once the
+      // zero-copy chunks in flight drain: pack only while that pays (t_cpu < N t_zc); else ZC only
+      if (t_zc_ms > 0 && t_cpu_ms > (double)c->cfg.n_slots * t_zc_ms) cpu = false;
     }
     int rc;
     {

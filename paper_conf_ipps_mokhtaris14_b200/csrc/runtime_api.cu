@@ -248,6 +248,7 @@ int bk_register_segments(bk_ctx* c, const void* host_ptr, uint64_t nbytes, const
   c->plan_cache.clear();
   c->units_key.clear();
   c->batch_key.clear();
+  c->hy_t_zc_ms = c->hy_t_cpu_ms = 0;
   drop_graphs(c);
   c->st.ms_register = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return BK_OK;

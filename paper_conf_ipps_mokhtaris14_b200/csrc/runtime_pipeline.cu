@@ -386,7 +386,7 @@ int check_err(bk_ctx* c) {  // after end_host: the error bits arrived with the r
   const int herr = (int)(uint32_t)c->h_ctr[8];
   if (herr & kErrStageOverflow) return fail(BK_E_RANGE, "staged chunk exceeded its slot (internal bound violated)");
   if (herr & kErrKeyRange) return fail(BK_E_INVAL, "a group-by key is >= G");
-  if (herr & kErrTableFull) return fail(BK_E_CAPACITY, "word-count hash table full; raise table_slots");
+  if (herr & kErrTableFull) return fail(BK_E_CAPACITY, "hash table full (word count / k-mers); raise table_slots");
   if (herr & kErrWordTooLong) return fail(BK_E_RANGE, "a word is longer than 2^24 bytes or offset >= 2^40");
   if (herr & kErrFusedTimeout) return fail(BK_E_CUDA, "persistent kernel: a loader/consumer wait timed out");
   return BK_OK;

@@ -94,16 +94,16 @@ def test_kmer_bench_scale_sampled():
     assert {int(key): int(h) for key, h in zip(keys, hits)} == want
 
 
-@pytest.mark.parametrize("slots", [1 << 13, 1 << 16, 1 << 22])
-def test_kmer_skewed_buckets_and_region_sizes(slots):
+@pytest.mark.parametrize("n,slots", [(60, 1 << 13), (6000, 1 << 18), (6000, 1 << 22)])
+def test_kmer_skewed_buckets_and_region_sizes(n, slots):
     """Two-phase counting under skew: half the reads are poly-A (one k-mer for every window: its
-    region's bucket overflows and the rest goes to the region directly), the rest random; tables of
+    region's bucket overflows and the rest goes to the region directly), the rest random; a table of
     one region (2^13 slots), a few regions, and many."""
-    n = 6000
     buf = gen.dna(n=n, genome_len=1 << 16, err_pm=2, n_pm=3).reshape(n, 256).copy()
     buf[::2, 16:112] = ord("A")
     buf = buf.reshape(-1)
     wk, wc = oracle.kmer(buf, n, 31)
+    assert len(wk) * 2 < slots
     with bk.Context(window_bytes=1 * MIB, record_size=256, gather_mode="zc") as ctx:
         ctx.register(buf, None, n_records=n)
         km, ct, total = ctx.kmer(k=31, table_slots=slots, cap=1 << 20)
