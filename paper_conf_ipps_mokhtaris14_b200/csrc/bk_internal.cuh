@@ -189,22 +189,19 @@ struct KmerEntry {            // 16 B exact-key slot
   unsigned long long key;     // k-mer + 1 (0 = empty)
   unsigned long long count;
 };
-void launch_kmer(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base, uint32_t k,
-                 uint32_t seq_words, KmerEntry* table, uint64_t mask, unsigned long long* used,
-                 unsigned long long* total, int* err, cudaStream_t s);
 // two-phase counting (kernels_kmer.cu): the table as 2^rb regions of region_slots slots; phase A
-// appends keys to per-region buckets (bbuf: 2^rb x bcap keys, bcur: 2^rb cursors, zeroed), phase B
-// (flush) counts each bucket into its region in shared memory and resets the cursors
+// appends keys to per-region buckets (bbuf: 2^rb x bcap keys, bcur: 2^rb cursors, dirty: 2^rb flags,
+// all zeroed), a flush counts each bucket into its region in shared memory; the final flush emits the
+// distinct k-mers to out_kmer / out_cnt (n_out, zeroed) instead of writing the regions back
 size_t kmer_flush_smem(uint64_t region_slots);
 void launch_kmer_scatter(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
                          uint32_t k, uint32_t seq_words, KmerEntry* table, uint32_t rb, uint64_t region_slots,
-                         unsigned long long* bbuf, unsigned int* bcur, uint32_t bcap, unsigned long long* total,
-                         int* err, cudaStream_t s);
+                         unsigned long long* bbuf, unsigned int* bcur, uint32_t bcap, unsigned char* dirty,
+                         unsigned long long* total, int* err, cudaStream_t s);
 void launch_kmer_flush(KmerEntry* table, uint32_t rb, uint64_t region_slots, const unsigned long long* bbuf,
-                       unsigned int* bcur, uint32_t bcap, int* err, cudaStream_t s);
+                       unsigned int* bcur, uint32_t bcap, unsigned char* dirty, int final_flush, uint64_t* out_kmer,
+                       uint64_t* out_cnt, uint64_t ocap, unsigned long long* n_out, int* err, cudaStream_t s);
 cudaError_t configure_kmer_kernels();
-void launch_kmer_compact(const KmerEntry* table, uint64_t slots, unsigned long long* n_out, uint64_t* kmer,
-                         uint64_t* cnt, uint64_t cap, cudaStream_t s);
 
 // ---- multi-GPU merge of count tables (kernels_merge.cu): rows of row_u64 words, key = words
 // [0, key_u64), count at count_col; owner/cnt: `slots` (power of two) scratch entries each

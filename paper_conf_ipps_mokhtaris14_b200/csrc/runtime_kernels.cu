@@ -495,29 +495,32 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   for (size_t i = 0; i + 1 < p.bounds.size(); ++i) per_chunk = std::max<uint64_t>(per_chunk, (p.bounds[i + 1] - p.bounds[i]) * wpr);
   const uint64_t F = per_chunk ? std::max<uint64_t>(1, (uint64_t)(0.8 * bcap * R) / per_chunk) : 1;
   BK_CUDA(c->b_blk.ensure((uint64_t)bcap * R * 8));
-  BK_CUDA(c->b_blk2.ensure(R * 4));
+  BK_CUDA(c->b_blk2.ensure(R * 5));
   unsigned long long* bbuf = (unsigned long long*)c->b_blk.p;
   unsigned int* bcur = (unsigned int*)c->b_blk2.p;
+  unsigned char* dirty = (unsigned char*)(bcur + R);
   const std::string key = "kmer/" + std::to_string(o->k) + "/" + std::to_string(slots) + "/" + std::to_string(ocap) +
                           "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(KmerEntry), c->s_comp));
-    BK_CUDA(cudaMemsetAsync(bcur, 0, R * 4, c->s_comp));
+    BK_CUDA(cudaMemsetAsync(bcur, 0, R * 5, c->s_comp));   // cursors + dirty flags
     size_t ci = 0;
-    int r = pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+    // appends commute: chunks scatter concurrently unless a mid-run flush must see all of them
+    const bool one_flush = F + 1 >= p.bounds.size();
+    int r = pipeline(c, p, one_flush, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
       launch_kmer_scatter(ch, s.stage, s.lanes, s.tile_base, o->k, o->seq_len / 16, table, rb, S, bbuf, bcur, bcap,
-                          c->d_ctr + 5, c->d_err, cs);
+                          dirty, c->d_ctr + 5, c->d_err, cs);
       c->n_launch += 1;
       if (++ci % F == 0 && ci + 1 < p.bounds.size()) {   // buckets near full: count them now
-        launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, c->d_err, cs);
+        launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, dirty, 0, nullptr, nullptr, 0, nullptr, c->d_err, cs);
         c->n_launch += 1;
       }
       return BK_OK;
     });
     if (r) return r;
-    launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, c->d_err, c->s_comp);
-    launch_kmer_compact(table, slots, c->d_ctr + 2, (uint64_t*)c->b_out1.p, (uint64_t*)c->b_out3.p, ocap, c->s_comp);
-    c->n_launch += 2;
+    launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, dirty, 1, (uint64_t*)c->b_out1.p, (uint64_t*)c->b_out3.p, ocap,
+                      c->d_ctr + 2, c->d_err, c->s_comp);   // final: emits the distinct k-mers
+    c->n_launch += 1;
     return (int)BK_OK;
   });
   if (rc) return rc;

@@ -5,6 +5,13 @@
 # Copy what is judged into profiles/ afterwards (tools/README.md).
 mkdir -p gpurun_out
 T=${TAG:-r02z}
+# the GPU suite, file by file (a hang or failure in one file does not hide the others)
+for f in tests/test_gpu_*.py; do
+  b=$(basename $f .py)
+  timeout 1500 python -m pytest $f -v --timeout 600 --tb=short -p no:cacheprovider > gpurun_out/${T}_$b.log 2>&1
+  echo "$b rc=$? $(grep -cE 'PASSED' gpurun_out/${T}_$b.log) passed $(grep -cE 'FAILED' gpurun_out/${T}_$b.log) failed"
+done
+timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${T}_smoke.log 2>&1; tail -1 gpurun_out/${T}_smoke.log
 line() {  # name bench-args...
   name=$1; shift
   timeout 1500 python bench.py "$@" > gpurun_out/${T}_bench_$name.json 2> gpurun_out/${T}_bench_$name.err
