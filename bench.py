@@ -52,7 +52,7 @@ def parse():
                          "buffering variants, for ablations)")
     ap.add_argument("--workload", default="grep", choices=["grep", "wordcount", "groupby", "groupby_sparse", "kmeans",
                                                              "partition", "kmer"])
-    ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense", "cpu", "hybrid"])
+    ap.add_argument("--gather", default="auto", choices=["auto", "zc", "dense", "cpu", "hybrid", "fused", "addr"])
     ap.add_argument("--gib", type=float, default=None, help="per-GPU data size override (GiB)")
     ap.add_argument("--window-mib", type=int, default=None)
     ap.add_argument("--slots", type=int, default=0)
@@ -733,7 +733,7 @@ def main():
         "config": {"workload": args.workload, "desc": WORKLOADS[args.workload][2],
                    "bytes_per_gpu": nbytes, "records_per_gpu": shard["n"], "window_bytes": window,
                    "n_slots": st["n_slots"],
-                   "gather_mode": {1: "zc", 2: "cpu", 3: "dense", 4: "hybrid", 5: "fused"}.get(st["gather_mode"], "?"),
+                   "gather_mode": {1: "zc", 2: "cpu", 3: "dense", 4: "hybrid", 5: "fused", 6: "addr"}.get(st["gather_mode"], "?"),
                    "chunks_cpu_assembled": st["n_chunks_cpu"], "n_chunks": st["n_chunks"],
                    "lanes_per_chunk": st["lanes"], "chunk_budget_bytes": st["chunk_budget"],
                    "l2": "inputs (>=64 MiB per GPU, host-resident) exceed the 126 MB L2; streamed from host each step",

@@ -194,10 +194,15 @@ struct KmerEntry {            // 16 B exact-key slot
 // all zeroed), a flush counts each bucket into its region in shared memory; the final flush emits the
 // distinct k-mers to out_kmer / out_cnt (n_out, zeroed) instead of writing the regions back
 size_t kmer_flush_smem(uint64_t region_slots);
-void launch_kmer_scatter(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
-                         uint32_t k, uint32_t seq_words, KmerEntry* table, uint32_t rb, uint64_t region_slots,
-                         unsigned long long* bbuf, unsigned int* bcur, uint32_t bcap, unsigned char* dirty,
-                         unsigned long long* total, int* err, cudaStream_t s);
+// phase A: k-mer keys -> 2^cb coarse bins (cb <= rb; cb == rb: the bins are the regions' buckets)
+void launch_kmer_bin(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                     uint32_t k, uint32_t seq_words, KmerEntry* table, uint32_t rb, uint32_t cb, uint64_t region_slots,
+                     unsigned long long* gbuf, unsigned int* gcur, uint32_t gcap, unsigned char* dirty,
+                     unsigned long long* total, int* err, cudaStream_t s);
+// flush, first half (cb < rb): coarse bins -> region buckets, coarse cursors reset (cdone: 2^cb, zeroed)
+void launch_kmer_split(const unsigned long long* cbuf, unsigned int* ccur, uint32_t ccap, unsigned int* cdone,
+                       uint32_t rb, uint32_t cb, unsigned long long* fbuf, unsigned int* fcur, uint32_t fcap,
+                       KmerEntry* table, uint64_t region_slots, unsigned char* dirty, int* err, cudaStream_t s);
 void launch_kmer_flush(KmerEntry* table, uint32_t rb, uint64_t region_slots, const unsigned long long* bbuf,
                        unsigned int* bcur, uint32_t bcap, unsigned char* dirty, int final_flush, uint64_t* out_kmer,
                        uint64_t* out_cnt, uint64_t ocap, unsigned long long* n_out, int* err, cudaStream_t s);

@@ -7,6 +7,7 @@
 #include <immintrin.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 namespace bk {
@@ -303,18 +304,32 @@ uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, con
   // sweep on the 16-core host (profiles/r01_hybrid_sweep.md): 16-record prefetch distance, grabs of
   // 4k-16k records read in order
   const uint64_t kGrab = grab ? grab : 16384;
-  constexpr uint64_t kPf = 16;        // software prefetch distance (records)
+  // prefetch: near (into L1) kPf records ahead, both ends of the field (a 32-B key crosses a 64-B line
+  // for 3 of 8 record alignments), and far (into L2) kPf2 records ahead. Sweep on the gpurun box's
+  // 16 vCPUs (tools/host_gather_bench.cpp, gpurun_out/r02s_hgb_*): near 16 only 0.58 G rec/s,
+  // near 8 + both ends + far 64 0.72 G rec/s (+23%). BK_PACK_PF / BK_PACK_PF2 / BK_PACK_PFEND
+  // override (sweep knobs).
+  static const uint64_t kPf = getenv("BK_PACK_PF") ? (uint64_t)atoll(getenv("BK_PACK_PF")) : 8;
+  static const uint64_t kPf2 = getenv("BK_PACK_PF2") ? (uint64_t)atoll(getenv("BK_PACK_PF2")) : 64;
+  static const bool kPfEnd = getenv("BK_PACK_PFEND") ? atoi(getenv("BK_PACK_PFEND")) != 0 : true;
   std::atomic<uint64_t> next{0};
   pool.run([&](int) {
     auto src = [&](uint64_t r) { return d.base + (d.off ? d.off[r] : r * d.rec_size) + eo; };
+    auto pf = [&](uint64_t r) {
+      const uint8_t* p = src(r);
+      __builtin_prefetch(p);
+      if (kPfEnd) __builtin_prefetch(p + E - 1);
+    };
     for (;;) {
       const uint64_t j0 = next.fetch_add(kGrab);
       if (j0 >= n) break;
       const uint64_t j1 = std::min(n, j0 + kGrab);
-      for (uint64_t j = j0; j < std::min(j1, j0 + kPf); ++j) __builtin_prefetch(src(c.lo + j));
+      for (uint64_t j = j0; j < std::min(j1, j0 + kPf); ++j) pf(c.lo + j);
+      for (uint64_t j = j0; kPf2 && j < std::min(j1, j0 + kPf2); ++j) _mm_prefetch((const char*)src(c.lo + j), _MM_HINT_T1);
       if (nt) {
         for (uint64_t j = j0; j < j1; ++j) {
-          if (j + kPf < j1) __builtin_prefetch(src(c.lo + j + kPf));
+          if (j + kPf < j1) pf(c.lo + j + kPf);
+          if (kPf2 && j + kPf2 < j1) _mm_prefetch((const char*)src(c.lo + j + kPf2), _MM_HINT_T1);
           const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
           __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
           for (uint32_t m = 0; m < EW; ++m) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
@@ -322,7 +337,8 @@ uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, con
         if (sink) _mm_sfence();
       } else {
         for (uint64_t j = j0; j < j1; ++j) {
-          if (j + kPf < j1) __builtin_prefetch(src(c.lo + j + kPf));
+          if (j + kPf < j1) pf(c.lo + j + kPf);
+          if (kPf2 && j + kPf2 < j1) _mm_prefetch((const char*)src(c.lo + j + kPf2), _MM_HINT_T1);
           const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
           __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
           for (uint32_t m = 0; m < EW; ++m) _mm_storeu_si128(o + m, _mm_loadu_si128(s + m));

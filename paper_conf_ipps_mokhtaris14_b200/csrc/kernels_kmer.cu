@@ -7,6 +7,8 @@
 // phases (below).
 #include "bk_internal.cuh"
 
+#include <algorithm>
+
 namespace bk {
 namespace {
 
@@ -38,21 +40,110 @@ __device__ __forceinline__ void region_insert(KmerEntry* region, uint64_t smask,
   atomicOr(err, kErrTableFull);
 }
 
-__global__ void __launch_bounds__(256) k_kmer_scatter(Chunk c, const uint8_t* __restrict__ stage,
-                                                      const LaneDesc* __restrict__ lanes,
-                                                      const uint64_t* __restrict__ tile_base, uint32_t k,
-                                                      uint32_t seq_words, KmerEntry* table, uint32_t rb,
-                                                      uint64_t smask, unsigned long long* __restrict__ bbuf,
-                                                      unsigned int* __restrict__ bcur, uint32_t bcap,
-                                                      unsigned char* __restrict__ dirty,
-                                                      unsigned long long* total, int* err) {
+// Block-level bucketing (phase A and the coarse -> fine split): a block stages up to kStep keys in
+// shared memory, sorts them by bin (shared-memory histogram + scan), reserves each bin's run in its
+// global bucket with ONE atomic per (block step, bin) and writes the runs coalesced. Keys of a full
+// bucket go to their table region in HBM directly (exact for any input).
+constexpr int kBinThreads = 256;
+constexpr uint32_t kStep = kBinThreads * 16;   // keys per block step (16 per thread: one staged word)
+constexpr uint32_t kMaxBins = 256;
+
+struct BinSmem {
+  unsigned int hist[kMaxBins], boff[kMaxBins + 1], gpos[kMaxBins];
+  unsigned long long key[kStep];
+  unsigned short bin[kStep];
+};
+
+// One block step: thread-local keys (okm bits of key[16], their bins in bn[16]) -> buckets
+// gbuf[bin * gcap ...] (cursors gcur[bin]); `region_of(key)` / `rbase` locate a key's table region
+// for the fallback. Every thread of the block must call it.
+template <class RegionOf>
+__device__ __forceinline__ void bin_step(BinSmem& sm, uint32_t nbins, const unsigned long long* key, const uint32_t* bn,
+                                         uint32_t okm, unsigned long long* gbuf, unsigned int* gcur, uint32_t gcap,
+                                         KmerEntry* table, uint64_t smask, unsigned char* dirty, int* err,
+                                         RegionOf&& region_of) {
+  const uint32_t tid = threadIdx.x;
+  for (uint32_t i = tid; i < nbins; i += blockDim.x) sm.hist[i] = 0;
+  __syncthreads();
+  unsigned lp[16];
+#pragma unroll
+  for (int b = 0; b < 16; ++b) lp[b] = (okm >> b & 1) ? atomicAdd(&sm.hist[bn[b]], 1u) : 0u;
+  __syncthreads();
+  if (tid < 32) {   // exclusive scan of the histogram (nbins <= 256: 8 per lane)
+    unsigned v[8], sum = 0;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t i = tid * 8 + q;
+      v[q] = i < nbins ? sm.hist[i] : 0u;
+      sum += v[q];
+    }
+    unsigned incl = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned y = __shfl_up_sync(kFull, incl, o);
+      if (tid >= (uint32_t)o) incl += y;
+    }
+    unsigned run = incl - sum;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t i = tid * 8 + q;
+      if (i < nbins) sm.boff[i] = run;
+      run += v[q];
+    }
+    if (tid == 31) sm.boff[nbins] = incl;
+  }
+  for (uint32_t i = tid; i < nbins; i += blockDim.x) sm.gpos[i] = sm.hist[i] ? atomicAdd(&gcur[i], sm.hist[i]) : 0u;
+  __syncthreads();
+#pragma unroll
+  for (int b = 0; b < 16; ++b) {
+    if (!(okm >> b & 1)) continue;
+    const uint32_t i = sm.boff[bn[b]] + lp[b];
+    sm.key[i] = key[b];
+    sm.bin[i] = (unsigned short)bn[b];
+  }
+  __syncthreads();
+  const uint32_t total = sm.boff[nbins];
+  for (uint32_t i = tid; i < total; i += blockDim.x) {
+    const uint32_t bi = sm.bin[i];
+    const unsigned long long kk = sm.key[i];
+    const uint64_t pos = (uint64_t)sm.gpos[bi] + (i - sm.boff[bi]);
+    if (pos < gcap) {
+      gbuf[(size_t)bi * gcap + pos] = kk;
+    } else {   // bucket full: straight into the key's region in HBM
+      const uint32_t r = region_of(kk);
+      region_insert(table + (size_t)r * (smask + 1), smask, mix64(kk), kk, 1ull, err);
+      dirty[r] = 1;
+    }
+  }
+  __syncthreads();
+}
+
+// Phase A (stage 4, per chunk): every k-mer window of the lane's reads -> its coarse bin (the top cb
+// bits of mix64(key); cb == rb: the bins are the regions' buckets themselves)
+__global__ void __launch_bounds__(kBinThreads) k_kmer_bin(Chunk c, const uint8_t* __restrict__ stage,
+                                                          const LaneDesc* __restrict__ lanes,
+                                                          const uint64_t* __restrict__ tile_base, uint32_t k,
+                                                          uint32_t seq_words, KmerEntry* table, uint32_t rb,
+                                                          uint32_t cb, uint64_t smask,
+                                                          unsigned long long* __restrict__ gbuf,
+                                                          unsigned int* __restrict__ gcur, uint32_t gcap,
+                                                          unsigned char* __restrict__ dirty,
+                                                          unsigned long long* total, int* err) {
+  __shared__ BinSmem sm;
+  __shared__ uint32_t s_rmax;
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-  if (t >= c.L) return;  // whole warps
-  const int lane = t & 31;
-  const LaneDesc d = lanes[t];
-  const uint8_t* tile = stage + tile_base[t >> 5];
-  const uint32_t R = __reduce_max_sync(kFull, d.nrec);
+  const int lane = threadIdx.x & 31;
+  const bool live = t < c.L;
+  LaneDesc d{0, 0, 0};
+  if (live) d = lanes[t];
+  const uint8_t* tile = stage + (live ? tile_base[t >> 5] : 0);
+  if (threadIdx.x == 0) s_rmax = 0;
+  __syncthreads();
+  atomicMax(&s_rmax, d.nrec);
+  __syncthreads();
+  const uint32_t R = s_rmax;   // block-uniform trip count (the steps synchronise the block)
   const uint64_t kmask = k == 32 ? ~0ull : ((1ull << (2 * k)) - 1);
+  auto region_of = [&](unsigned long long kk) -> uint32_t { return rb ? (uint32_t)(mix64(kk) >> (64 - rb)) : 0u; };
   unsigned long long mine = 0;
   for (uint32_t j = 0; j < R; ++j) {
     const bool rec = j < d.nrec;
@@ -62,10 +153,8 @@ __global__ void __launch_bounds__(256) k_kmer_scatter(Chunk c, const uint8_t* __
       uint4 q = make_uint4(0, 0, 0, 0);
       if (rec) q = *reinterpret_cast<const uint4*>(tile + ((size_t)(j * seq_words + w) * 32 + lane) * 16);
       const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
-      // the word's up to 16 k-mers first, then their 16 independent cursor atomics, then the stores:
-      // one L2 round trip per 16 windows instead of one per window
       unsigned long long key[16];
-      uint32_t bk[16];
+      uint32_t bn[16];
       uint32_t okm = 0;
 #pragma unroll
       for (int b = 0; b < 16; ++b) {
@@ -79,27 +168,52 @@ __global__ void __launch_bounds__(256) k_kmer_scatter(Chunk c, const uint8_t* __
           ++valid;
         }
         key[b] = v + 1;
-        bk[b] = rb ? (uint32_t)(mix64(key[b]) >> (64 - rb)) : 0u;
+        bn[b] = cb ? (uint32_t)(mix64(key[b]) >> (64 - cb)) : 0u;
         if (rec && valid >= k) okm |= 1u << b;
       }
-      unsigned pos[16];
-#pragma unroll
-      for (int b = 0; b < 16; ++b) pos[b] = (okm >> b & 1) ? atomicAdd(&bcur[bk[b]], 1u) : 0u;
-#pragma unroll
-      for (int b = 0; b < 16; ++b) {
-        if (!(okm >> b & 1)) continue;
-        if (pos[b] < bcap) {
-          bbuf[(size_t)bk[b] * bcap + pos[b]] = key[b];
-        } else {   // bucket full: straight into the region in HBM
-          region_insert(table + (size_t)bk[b] * (smask + 1), smask, mix64(key[b]), key[b], 1ull, err);
-          dirty[bk[b]] = 1;
-        }
-      }
       mine += __popc(okm);
+      bin_step(sm, 1u << cb, key, bn, okm, gbuf, gcur, gcap, table, smask, dirty, err, region_of);
     }
   }
-  mine = __reduce_add_sync(kFull, (unsigned)mine);
+  for (int o = 16; o; o >>= 1) mine += __shfl_down_sync(kFull, mine, o);
   if (lane == 0 && mine) atomicAdd(total, mine);
+}
+
+// Flush, first half (cb < rb): coarse bin b's keys -> the buckets of its 2^(rb-cb) regions. Grid
+// (slices, coarse bins); resets the coarse cursor when its last slice is done (a per-bin counter).
+__global__ void __launch_bounds__(kBinThreads) k_kmer_split(const unsigned long long* __restrict__ cbuf,
+                                                            unsigned int* __restrict__ ccur, uint32_t ccap,
+                                                            unsigned int* __restrict__ cdone, uint32_t rb, uint32_t cb,
+                                                            unsigned long long* __restrict__ fbuf,
+                                                            unsigned int* __restrict__ fcur, uint32_t fcap,
+                                                            KmerEntry* table, uint64_t smask,
+                                                            unsigned char* __restrict__ dirty, int* err) {
+  __shared__ BinSmem sm;
+  const uint32_t b = blockIdx.y, nslice = gridDim.x, sl = blockIdx.x;
+  const uint32_t n = min(ccur[b], ccap);
+  const uint32_t lo = (uint32_t)((uint64_t)n * sl / nslice), hi = (uint32_t)((uint64_t)n * (sl + 1) / nslice);
+  const uint32_t fb = rb - cb;   // fine bits within the coarse bin
+  const unsigned long long* keys = cbuf + (size_t)b * ccap;
+  auto region_of = [&](unsigned long long kk) -> uint32_t { return (uint32_t)(mix64(kk) >> (64 - rb)); };
+  for (uint32_t base = lo; base < hi; base += kStep) {
+    unsigned long long key[16];
+    uint32_t bn[16];
+    uint32_t okm = 0;
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const uint32_t i = base + q * blockDim.x + threadIdx.x;
+      key[q] = i < hi ? keys[i] : 0ull;
+      bn[q] = i < hi ? (uint32_t)(mix64(key[q]) >> (64 - rb)) & ((1u << fb) - 1) : 0u;
+      if (i < hi) okm |= 1u << q;
+    }
+    bin_step(sm, 1u << fb, key, bn, okm, fbuf + (size_t)b * (1ull << fb) * fcap, fcur + ((size_t)b << fb), fcap,
+             table, smask, dirty, err, region_of);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && atomicAdd(&cdone[b], 1u) + 1 == nslice) {   // the bin's last slice: reset it
+    ccur[b] = 0;
+    cdone[b] = 0;
+  }
 }
 
 // one CTA per region: the region -> shared memory (loaded only if its HBM copy holds counts: a direct
@@ -196,12 +310,21 @@ __global__ void __launch_bounds__(512) k_kmer_flush(KmerEntry* table, uint32_t r
 
 size_t kmer_flush_smem(uint64_t region_slots) { return (size_t)region_slots * sizeof(KmerEntry); }
 
-void launch_kmer_scatter(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
-                         uint32_t k, uint32_t seq_words, KmerEntry* table, uint32_t rb, uint64_t region_slots,
-                         unsigned long long* bbuf, unsigned int* bcur, uint32_t bcap, unsigned char* dirty,
-                         unsigned long long* total, int* err, cudaStream_t s) {
-  k_kmer_scatter<<<(c.L + 255) / 256, 256, 0, s>>>(c, stage, lanes, tile_base, k, seq_words, table, rb,
-                                                    region_slots - 1, bbuf, bcur, bcap, dirty, total, err);
+void launch_kmer_bin(const Chunk& c, const uint8_t* stage, const LaneDesc* lanes, const uint64_t* tile_base,
+                     uint32_t k, uint32_t seq_words, KmerEntry* table, uint32_t rb, uint32_t cb, uint64_t region_slots,
+                     unsigned long long* gbuf, unsigned int* gcur, uint32_t gcap, unsigned char* dirty,
+                     unsigned long long* total, int* err, cudaStream_t s) {
+  k_kmer_bin<<<(c.L + kBinThreads - 1) / kBinThreads, kBinThreads, 0, s>>>(c, stage, lanes, tile_base, k, seq_words,
+                                                                        table, rb, cb, region_slots - 1, gbuf, gcur,
+                                                                        gcap, dirty, total, err);
+}
+
+void launch_kmer_split(const unsigned long long* cbuf, unsigned int* ccur, uint32_t ccap, unsigned int* cdone,
+                       uint32_t rb, uint32_t cb, unsigned long long* fbuf, unsigned int* fcur, uint32_t fcap,
+                       KmerEntry* table, uint64_t region_slots, unsigned char* dirty, int* err, cudaStream_t s) {
+  const uint32_t slices = std::max(1, 2 * device_sms() / (1 << cb) + 1);
+  k_kmer_split<<<dim3(slices, 1u << cb), kBinThreads, 0, s>>>(cbuf, ccur, ccap, cdone, rb, cb, fbuf, fcur, fcap, table,
+                                                             region_slots - 1, dirty, err);
 }
 
 void launch_kmer_flush(KmerEntry* table, uint32_t rb, uint64_t region_slots, const unsigned long long* bbuf,

@@ -178,6 +178,7 @@ struct bk_ctx {  // the opaque context of include/bk.h
   bk::rt::DevBuf b_units;                    // BK_GATHER_FUSED unit plan (record bounds, byte bounds)
   bk::rt::DevBuf b_flags;                    //   ring ready / done flags
   bk::rt::DevBuf b_batch;                    //   DMA feed: batch plan (byte / record bounds, unit -> batch)
+  bk::rt::DevBuf b_kbin;                     // k-mers: coarse bins of phase A
   std::string batch_key;
   uint64_t n_batches = 0;
   std::vector<uint64_t> h_bby, h_brec;
@@ -326,11 +327,11 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
     int rc;
     {
       NvtxRange r("chunk %zu %s", i, p.mode == BK_GATHER_ADDR ? "addr" : cpu ? "cpu" : p.zero_copy ? "zc" : "dense");
-      const auto t0 = std::chrono::steady_clock::now();
+      const double packed0 = c->st.ms_cpu_gather;   // host time of the packing itself (no waits)
       rc = p.mode == BK_GATHER_ADDR ? stage_chunk_addr(c, p, i, s) : cpu ? stage_chunk_cpu(c, p, i, s)
                                                                           : stage_chunk(c, p, i, s);
-      if (cpu && p.mode == BK_GATHER_HYBRID) {
-        const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+      if (cpu && p.mode == BK_GATHER_HYBRID && !rc) {
+        const double ms = c->st.ms_cpu_gather - packed0;
         t_cpu_ms = t_cpu_ms > 0 ? 0.5 * (t_cpu_ms + ms) : ms;
       }
     }

@@ -480,7 +480,7 @@ int bk_destroy(bk_ctx* c) {
   release_kept_outputs(c);
   release_addr_side(c);
   for (DevBuf* b : {&c->b_hist, &c->b_colpre, &c->b_totals, &c->b_base, &c->b_h1, &c->b_h2, &c->b_mown, &c->b_mcnt,
-                    &c->b_mctr, &c->b_units, &c->b_flags, &c->b_batch})
+                    &c->b_mctr, &c->b_units, &c->b_flags, &c->b_batch, &c->b_kbin})
     b->release();
   for (auto* h : c->hstage) cudaFreeHost(h);
   for (auto e : c->h_done) cudaEventDestroy(e);

@@ -480,47 +480,68 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
   BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
   KmerEntry* table = (KmerEntry*)c->b_table.p;
-  // regions of <= 8192 slots (128 KiB of shared memory in the flush); buckets sized for the run's
-  // k-mer windows (an upper bound: every window of every record valid) within 16 GiB, else flushed
-  // every F chunks; a full bucket falls back to direct inserts
+  // regions of <= 8192 slots (128 KiB of shared memory in the flush). Phase A bins keys into 2^cb <= 256
+  // coarse bins (one global atomic per block step and bin); the flush splits them into the regions'
+  // buckets (cb < rb), then counts each bucket in its region. Buckets are sized for the run's k-mer
+  // windows (an upper bound: every window of every record valid) within 16 GiB each, else flushed every
+  // F chunks; a full bucket falls back to direct inserts
   const uint64_t S = std::min<uint64_t>(slots, 8192);
   uint32_t rb = 0;
   while ((S << rb) < slots) ++rb;
   const uint64_t R = 1ull << rb;
+  const uint32_t cb = std::min<uint32_t>(rb, 8);
+  const uint64_t NB = 1ull << cb;
+  const bool two = cb < rb;
   const uint64_t wpr = o->seq_len >= o->k ? o->seq_len - o->k + 1 : 0;   // windows per record (bound)
   const uint64_t bound = c->n * wpr;
-  const uint64_t budget = std::min<uint64_t>(16ull << 30, (uint64_t)(bound * 1.15) * 8 + R * 8192 + 8);
-  const uint32_t bcap = (uint32_t)std::min<uint64_t>(budget / 8 / R, 0xffffffffull);
+  const uint64_t fbudget = std::min<uint64_t>(16ull << 30, (uint64_t)(bound * 1.15) * 8 + R * 8192 + 8);
+  const uint32_t fcap = (uint32_t)std::min<uint64_t>(fbudget / 8 / R, 0xffffffffull);
+  const uint64_t cbudget = two ? std::min<uint64_t>(16ull << 30, (uint64_t)(bound * 1.1) * 8 + NB * 65536 + 8) : 0;
+  const uint32_t ccap = two ? (uint32_t)std::min<uint64_t>(cbudget / 8 / NB, 0xffffffffull) : 0;
   uint64_t per_chunk = 0;
   for (size_t i = 0; i + 1 < p.bounds.size(); ++i) per_chunk = std::max<uint64_t>(per_chunk, (p.bounds[i + 1] - p.bounds[i]) * wpr);
-  const uint64_t F = per_chunk ? std::max<uint64_t>(1, (uint64_t)(0.8 * bcap * R) / per_chunk) : 1;
-  BK_CUDA(c->b_blk.ensure((uint64_t)bcap * R * 8));
-  BK_CUDA(c->b_blk2.ensure(R * 5));
+  const uint64_t cap_keys = two ? std::min<uint64_t>((uint64_t)ccap * NB, (uint64_t)fcap * R) : (uint64_t)fcap * R;
+  uint64_t F = per_chunk ? std::max<uint64_t>(1, (uint64_t)(0.8 * cap_keys) / per_chunk) : 1;
+  if (getenv("BK_KMER_F")) F = std::max<uint64_t>(1, std::min<uint64_t>(F, (uint64_t)atoll(getenv("BK_KMER_F"))));
+  // split each chunk's coarse bins right after binning it (serial chunks) instead of once per flush
+  const bool split_each = two && getenv("BK_KMER_SPLIT_EACH") && atoi(getenv("BK_KMER_SPLIT_EACH"));
+  BK_CUDA(c->b_blk.ensure((uint64_t)fcap * R * 8));
+  if (two) BK_CUDA(c->b_kbin.ensure((uint64_t)ccap * NB * 8));
+  BK_CUDA(c->b_blk2.ensure(R * 5 + NB * 8 + 64));
   unsigned long long* bbuf = (unsigned long long*)c->b_blk.p;
   unsigned int* bcur = (unsigned int*)c->b_blk2.p;
   unsigned char* dirty = (unsigned char*)(bcur + R);
+  unsigned int* ccur = (unsigned int*)((uint8_t*)c->b_blk2.p + (R * 5 + 15) / 16 * 16);
+  unsigned int* cdone = ccur + NB;
+  unsigned long long* cbuf = two ? (unsigned long long*)c->b_kbin.p : bbuf;
   const std::string key = "kmer/" + std::to_string(o->k) + "/" + std::to_string(slots) + "/" + std::to_string(ocap) +
                           "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(KmerEntry), c->s_comp));
-    BK_CUDA(cudaMemsetAsync(bcur, 0, R * 5, c->s_comp));   // cursors + dirty flags
-    size_t ci = 0;
-    // appends commute: chunks scatter concurrently unless a mid-run flush must see all of them
-    const bool one_flush = F + 1 >= p.bounds.size();
-    int r = pipeline(c, p, one_flush, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
-      launch_kmer_scatter(ch, s.stage, s.lanes, s.tile_base, o->k, o->seq_len / 16, table, rb, S, bbuf, bcur, bcap,
-                          dirty, c->d_ctr + 5, c->d_err, cs);
+    BK_CUDA(cudaMemsetAsync(c->b_blk2.p, 0, R * 5 + NB * 8 + 64, c->s_comp));   // cursors, dirty flags
+    auto split = [&](cudaStream_t st) {
+      launch_kmer_split(cbuf, ccur, ccap, cdone, rb, cb, bbuf, bcur, fcap, table, S, dirty, c->d_err, st);
       c->n_launch += 1;
-      if (++ci % F == 0 && ci + 1 < p.bounds.size()) {   // buckets near full: count them now
-        launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, dirty, 0, nullptr, nullptr, 0, nullptr, c->d_err, cs);
-        c->n_launch += 1;
-      }
+    };
+    auto flush = [&](int final_flush, cudaStream_t st) {
+      if (two && !split_each) split(st);
+      launch_kmer_flush(table, rb, S, bbuf, bcur, fcap, dirty, final_flush, (uint64_t*)c->b_out1.p,
+                        (uint64_t*)c->b_out3.p, ocap, c->d_ctr + 2, c->d_err, st);
+      c->n_launch += 1;
+    };
+    size_t ci = 0;
+    // appends commute: chunks bin concurrently unless a mid-run flush must see all of them
+    const bool one_flush = F + 1 >= p.bounds.size() && !split_each;
+    int r = pipeline(c, p, one_flush, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
+      launch_kmer_bin(ch, s.stage, s.lanes, s.tile_base, o->k, o->seq_len / 16, table, rb, cb, S, cbuf,
+                      two ? ccur : bcur, two ? ccap : fcap, dirty, c->d_ctr + 5, c->d_err, cs);
+      c->n_launch += 1;
+      if (split_each) split(cs);
+      if (++ci % F == 0 && ci + 1 < p.bounds.size()) flush(0, cs);   // buckets near full: count them now
       return BK_OK;
     });
     if (r) return r;
-    launch_kmer_flush(table, rb, S, bbuf, bcur, bcap, dirty, 1, (uint64_t*)c->b_out1.p, (uint64_t*)c->b_out3.p, ocap,
-                      c->d_ctr + 2, c->d_err, c->s_comp);   // final: emits the distinct k-mers
-    c->n_launch += 1;
+    flush(1, c->s_comp);   // final: emits the distinct k-mers
     return (int)BK_OK;
   });
   if (rc) return rc;

@@ -619,7 +619,7 @@ std::string resident_key(const bk_ctx* c) {
   char b[24];
   for (const DevBuf* d : {&c->b_table, &c->b_out1, &c->b_out2, &c->b_out3, &c->b_blk, &c->b_blk2, &c->b_blk3,
                           &c->b_agg1, &c->b_agg2, &c->b_agg3, &c->b_mu, &c->b_hist, &c->b_colpre, &c->b_totals,
-                          &c->b_base, &c->b_h1, &c->b_h2, &c->b_units, &c->b_flags}) {
+                          &c->b_base, &c->b_h1, &c->b_h2, &c->b_units, &c->b_flags, &c->b_kbin}) {
     snprintf(b, sizeof b, "%llx,", (unsigned long long)(uintptr_t)d->p);
     k += b;
   }

@@ -1,7 +1,7 @@
 #!/bin/bash
 # One ncu --set full capture of the roofline kernel of each bench line whose dominant stage is a
 # kernel (not a copy-engine DMA), with the bench JSON of the same command (units per launch):
-# tools/traffic_json.py turns them into profiles/r01_traffic.json, which bench.py scales into
+# tools/traffic_json.py turns them into profiles/r0N_traffic.json, which bench.py scales into
 # roofline.traffic.
 mkdir -p gpurun_out
 TAG=${TAG:-r02x}
@@ -14,4 +14,4 @@ cap() {  # name kernel-regex skip bench-args
 cap grep "k_gather_field" 6 "--workload grep --gib 4 --zc-share 1000"
 cap groupby_sparse "k_gather_field" 6 "--workload groupby_sparse --gib 4 --zc-share 1000"
 cap wordcount "k_wc_fused" 3 "--workload wordcount"
-cap kmer "k_kmer_scatter" 6 "--workload kmer --gib 1"
+cap kmer "k_kmer_bin" 6 "--workload kmer --gib 1"

@@ -114,5 +114,6 @@ with bk.Context(window_bytes=1 << 20) as ctx:
     ctx.merge_counts(rows, [4096, 100, 4000], 4096, 6, 3, 3, out)
 with bk.Context(window_bytes=1 << 20, record_size=256, gather_mode="zc") as ctx:
     ctx.register(d, None, n_records=20_000)
-    ctx.kmer(k=31, table_slots=1 << 16)
+    ctx.kmer(k=31, table_slots=1 << 20)
+    ctx.kmer(k=31, table_slots=1 << 22)
 print("sanitize run (round 2) done")
