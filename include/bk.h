@@ -126,7 +126,7 @@ typedef struct bk_config {
                                      (bk_out_kmeans.cid, bk_out_partition.out_records, bk_out_kmer.kmer /
                                      .count) are page-locked (cudaHostRegister) by bk_run. Default: only for
                                      the duration of that bk_run (each run pays the registration, ~0.1 s per
-                                     GiB). With this flag the registration is cached across runs (at most four
+                                     GiB). With this flag the registration is cached across runs (at most eight
                                      arrays, oldest released first) and released by bk_unpin_outputs or
                                      bk_destroy: the caller must keep such arrays allocated until then. */
 
@@ -260,7 +260,11 @@ typedef struct bk_out_kmer {
   uint32_t _pad;
   uint64_t table_slots;     /* in: device table slots (power of two); 0 = 2^24 */
   uint64_t cap;             /* in: capacity of kmer / count */
-  uint64_t* kmer;           /* out: distinct k-mers, 2-bit packed (A=0 C=1 G=2 T=3), unordered */
+  uint64_t* kmer;           /* out: distinct k-mers, 2-bit packed (A=0 C=1 G=2 T=3), unordered. Device
+                               memory, caller-pinned host memory, or host memory kept pinned
+                               (BK_FLAG_KEEP_OUTPUTS_PINNED): the final flush kernel stores the results
+                               itself (over PCIe for host memory); other host memory receives a copy after
+                               the run. Both arrays are written up to min(cap, n_kmers) entries. */
   uint64_t* count;          /* out */
   uint64_t n_kmers;         /* out: distinct (> cap -> BK_E_CAPACITY) */
   uint64_t total;           /* out: k-mer occurrences */

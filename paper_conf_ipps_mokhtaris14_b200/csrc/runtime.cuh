@@ -259,6 +259,7 @@ bool graphable(const Plan& p);
 // those keep the SMs' sysmem path busy and the bulk copies were measured to stall behind them.
 inline bool stage_tma(const Plan& p) { return p.mode == BK_GATHER_DENSE || p.mode == BK_GATHER_CPU; }
 int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes);
+void* out_kernel_ptr(bk_ctx* c, void* ptr, uint64_t bytes);
 void release_run_outputs(bk_ctx* c);
 void release_kept_outputs(bk_ctx* c);
 void unregister(bk_ctx* c);

@@ -477,10 +477,20 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   carve(c, p);
   BK_CUDA(c->b_table.ensure(slots * sizeof(KmerEntry)));
   const uint64_t ocap = std::min<uint64_t>(o->cap, slots);
-  BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
-  BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
+  // the final flush stores the distinct k-mers straight into the caller's arrays when kernels can
+  // reach them (device memory, or pinned host memory through its mapped alias: the PCIe stores then
+  // overlap the flush instead of following it as a copy); else into HBM, copied after the run
+  uint64_t* dk = (uint64_t*)out_kernel_ptr(c, o->kmer, ocap * 8);
+  uint64_t* dc = dk ? (uint64_t*)out_kernel_ptr(c, o->count, ocap * 8) : nullptr;
+  const bool direct = dk && dc;
+  if (!direct) {
+    BK_CUDA(c->b_out1.ensure(std::max<uint64_t>(ocap, 1) * 8));
+    BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap, 1) * 8));
+    dk = (uint64_t*)c->b_out1.p;
+    dc = (uint64_t*)c->b_out3.p;
+  }
   KmerEntry* table = (KmerEntry*)c->b_table.p;
-  // regions of <= 8192 slots (128 KiB of shared memory in the flush). Phase A bins keys into 2^cb <= 256
+  // regions of <= 8192 slots (96 KiB of shared memory in the flush: 2 CTAs per SM). Phase A bins keys into 2^cb <= 256
   // coarse bins (one global atomic per block step and bin); the flush splits them into the regions'
   // buckets (cb < rb), then counts each bucket in its region. Buckets are sized for the run's k-mer
   // windows (an upper bound: every window of every record valid) within 16 GiB each, else flushed every
@@ -501,10 +511,15 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   uint64_t per_chunk = 0;
   for (size_t i = 0; i + 1 < p.bounds.size(); ++i) per_chunk = std::max<uint64_t>(per_chunk, (p.bounds[i + 1] - p.bounds[i]) * wpr);
   const uint64_t cap_keys = two ? std::min<uint64_t>((uint64_t)ccap * NB, (uint64_t)fcap * R) : (uint64_t)fcap * R;
-  uint64_t F = per_chunk ? std::max<uint64_t>(1, (uint64_t)(0.8 * cap_keys) / per_chunk) : 1;
+  // per_chunk is an upper bound (every window valid), so F chunks always fit the buckets on average;
+  // a region's share above its bucket's 15% + 8192-key margin goes to the region directly (exact)
+  uint64_t F = per_chunk ? std::max<uint64_t>(1, cap_keys / per_chunk) : 1;
   if (getenv("BK_KMER_F")) F = std::max<uint64_t>(1, std::min<uint64_t>(F, (uint64_t)atoll(getenv("BK_KMER_F"))));
-  // split each chunk's coarse bins right after binning it (serial chunks) instead of once per flush
-  const bool split_each = two && getenv("BK_KMER_SPLIT_EACH") && atoi(getenv("BK_KMER_SPLIT_EACH"));
+  // split each chunk's coarse bins right after binning it (chunks then run in order on one stream), so
+  // the split overlaps the transfer of later chunks instead of lengthening the final flush (measured:
+  // 60.3 vs 65.9 ms per 4-GiB step, profiles/r02_kmer.md); BK_KMER_SPLIT_EACH=0 splits once per flush
+  const char* se = getenv("BK_KMER_SPLIT_EACH");
+  const bool split_each = two && !(se && atoi(se) == 0);
   BK_CUDA(c->b_blk.ensure((uint64_t)fcap * R * 8));
   if (two) BK_CUDA(c->b_kbin.ensure((uint64_t)ccap * NB * 8));
   BK_CUDA(c->b_blk2.ensure(R * 5 + NB * 8 + 64));
@@ -515,7 +530,8 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   unsigned int* cdone = ccur + NB;
   unsigned long long* cbuf = two ? (unsigned long long*)c->b_kbin.p : bbuf;
   const std::string key = "kmer/" + std::to_string(o->k) + "/" + std::to_string(slots) + "/" + std::to_string(ocap) +
-                          "/" + p.key;
+                          "/" + std::to_string(F) + "/" + std::to_string(split_each) + "/" + std::to_string((uintptr_t)dk) + "/" +
+                          std::to_string((uintptr_t)dc) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(KmerEntry), c->s_comp));
     BK_CUDA(cudaMemsetAsync(c->b_blk2.p, 0, R * 5 + NB * 8 + 64, c->s_comp));   // cursors, dirty flags
@@ -525,8 +541,7 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
     };
     auto flush = [&](int final_flush, cudaStream_t st) {
       if (two && !split_each) split(st);
-      launch_kmer_flush(table, rb, S, bbuf, bcur, fcap, dirty, final_flush, (uint64_t*)c->b_out1.p,
-                        (uint64_t*)c->b_out3.p, ocap, c->d_ctr + 2, c->d_err, st);
+      launch_kmer_flush(table, rb, S, bbuf, bcur, fcap, dirty, final_flush, dk, dc, ocap, c->d_ctr + 2, c->d_err, st);
       c->n_launch += 1;
     };
     size_t ci = 0;
@@ -553,8 +568,8 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   if (nk > o->cap) return fail(BK_E_CAPACITY, "%llu distinct k-mers > cap %llu", nk, (unsigned long long)o->cap);
   if (nk * 10 > slots * 7) return fail(BK_E_CAPACITY, "k-mer table load %llu/%llu too high; raise table_slots", nk,
                                        (unsigned long long)slots);
-  if (nk) {
-    // the result arrays are large (16 B per distinct k-mer): pin them once so the copy runs at DMA speed
+  if (nk && !direct) {
+    // the result arrays are large (16 B per distinct k-mer): pin them so the copy runs at DMA speed
     if ((rc = ensure_out_pinned(c, o->kmer, nk * 8)) || (rc = ensure_out_pinned(c, o->count, nk * 8))) return rc;
     BK_CUDA(cudaMemcpy(o->kmer, c->b_out1.p, nk * 8, cudaMemcpyDefault));
     BK_CUDA(cudaMemcpy(o->count, c->b_out3.p, nk * 8, cudaMemcpyDefault));

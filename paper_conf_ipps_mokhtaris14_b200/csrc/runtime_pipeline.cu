@@ -647,9 +647,35 @@ int ensure_out_pinned(bk_ctx* c, void* ptr, uint64_t bytes) {
     cudaHostUnregister(c->out_pinned.front().first);
     c->out_pinned.erase(c->out_pinned.begin());
   }
-  BK_CUDA(cudaHostRegister(ptr, bytes, cudaHostRegisterPortable));
+  BK_CUDA(cudaHostRegister(ptr, bytes, cudaHostRegisterPortable | cudaHostRegisterMapped));
   (keep ? c->out_pinned : c->out_pinned_run).emplace_back(ptr, bytes);
   return BK_OK;
+}
+
+// A pointer kernels may store results through: device / managed memory as is, pinned host memory
+// through its mapped alias (kernel stores travel over PCIe, overlapping the kernel), host memory the
+// caller lets the context keep pinned (BK_FLAG_KEEP_OUTPUTS_PINNED: registered once); otherwise
+// nullptr (the caller stages the results in HBM and copies them after the run).
+void* out_kernel_ptr(bk_ctx* c, void* ptr, uint64_t bytes) {
+  if (!ptr || !bytes) return nullptr;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, ptr) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  if (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged) return ptr;
+  if (at.type == cudaMemoryTypeUnregistered) {
+    if (!(c->cfg.flags & BK_FLAG_KEEP_OUTPUTS_PINNED) || ensure_out_pinned(c, ptr, bytes)) {
+      cudaGetLastError();
+      return nullptr;
+    }
+  }
+  void* d = nullptr;
+  if (cudaHostGetDevicePointer(&d, ptr, 0) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return d;
 }
 
 // End of every bk_run (after all its copies completed or were drained): release this run's output

@@ -109,3 +109,46 @@ def test_kmer_skewed_buckets_and_region_sizes(n, slots):
         km, ct, total = ctx.kmer(k=31, table_slots=slots, cap=1 << 20)
     gk, gc = sorted_pairs(km, ct)
     assert np.array_equal(gk, wk) and np.array_equal(gc, wc) and total == int(wc.sum())
+
+
+@pytest.mark.parametrize("flush_every,split_each", [(1, "0"), (3, "0"), (1, "1"), (2, "1")])
+def test_kmer_mid_run_flushes(monkeypatch, flush_every, split_each):
+    """Mid-run flushes (every F chunks: the regions are written back with their 64-bit counts and
+    reloaded by the next flush) and the per-chunk coarse -> fine split give the oracle's table."""
+    monkeypatch.setenv("BK_KMER_F", str(flush_every))
+    monkeypatch.setenv("BK_KMER_SPLIT_EACH", split_each)
+    n = 30_000
+    buf = gen.dna(n=n, genome_len=1 << 16, err_pm=2, n_pm=3)
+    wk, wc = oracle.kmer(buf, n, 31)
+    with bk.Context(window_bytes=2 * MIB, record_size=256, gather_mode="hybrid") as ctx:
+        ctx.register(buf, None, n_records=n)
+        for _ in range(2):   # the second run replays the captured graph
+            km, ct, total = ctx.kmer(k=31, table_slots=1 << 22)
+            gk, gc = sorted_pairs(km, ct)
+            assert np.array_equal(gk, wk) and np.array_equal(gc, wc) and total == int(wc.sum())
+        assert ctx.stats()["n_chunks"] >= 4
+
+
+@pytest.mark.parametrize("where", ["pinned_host", "device"])
+def test_kmer_results_stored_by_the_flush(where):
+    """The final flush stores the distinct k-mers straight into the caller's arrays when kernels can
+    reach them: host arrays the context keeps pinned (mapped stores over PCIe) or device tensors."""
+    import torch
+    n = 20_000
+    buf = gen.dna(n=n, genome_len=1 << 16, err_pm=2, n_pm=3)
+    wk, wc = oracle.kmer(buf, n, 31)
+    cap = 1 << 20
+    if where == "device":
+        out = (torch.zeros(cap, dtype=torch.int64, device="cuda"), torch.zeros(cap, dtype=torch.int64, device="cuda"))
+    else:
+        out = (np.zeros(cap, np.uint64), np.zeros(cap, np.uint64))
+    with bk.Context(window_bytes=2 * MIB, record_size=256, keep_outputs_pinned=True) as ctx:
+        ctx.register(buf, None, n_records=n)
+        for _ in range(2):
+            km, ct, total = ctx.kmer(k=31, table_slots=1 << 22, out=out)
+            if where == "device":
+                km, ct = km.cpu().numpy().view(np.uint64), ct.cpu().numpy().view(np.uint64)
+            gk, gc = sorted_pairs(km, ct)
+            assert np.array_equal(gk, wk) and np.array_equal(gc, wc) and total == int(wc.sum())
+            out[0][:] = 0
+            out[1][:] = 0

@@ -1,8 +1,8 @@
 #!/usr/bin/env python3
-"""DESIGN.md §9 / README status rows from the committed bench lines (profiles/r01_bench_*.json).
+"""DESIGN.md §9 / README status rows from the committed bench lines (profiles/<round>_bench_*.json).
 
-    python tools/status_table.py design   # the §9 table rows
-    python tools/status_table.py readme   # the README table rows
+    python tools/status_table.py design [r02]   # the §9 table rows
+    python tools/status_table.py readme [r02]   # the README table rows
 """
 import json
 import os
@@ -12,16 +12,32 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 ROWS = [
     ("grep", "C2 grep 16 GiB (default bench)", "Grep, 16 GiB", "host-packing / PCIe-request-rate bound"),
     ("groupby", "C5 group-by 16 GiB dense", "Group-by, 16 GiB", ""),
+    ("groupby32", "C5 group-by 32 GiB dense (C5's per-GPU share at 8 GPUs)", "Group-by, 32 GiB", ""),
     ("groupby_sparse", "C5 group-by sparse 16 GiB (64-B records, 25% read)", "Group-by sparse (25% read), 16 GiB", ""),
     ("kmeans", "C3 k-means 16 GiB, K=64", "K-means, 16 GiB", ""),
+    ("kmeans256", "C3 k-means 16 GiB, K=256", "K-means K=256, 16 GiB", ""),
     ("partition", "C4 partition 8 GiB, 1024 buckets (D2H out)", "Partition, 8 GiB", ""),
     ("wordcount", "C1 word count 64 MiB, 8 MiB window, 8 slots", "Word count, 64 MiB (8 MiB window)", ""),
     ("kmer", "f4 k-mers 4 GiB (k = 31)", "k-mers, 4 GiB", "random-access bound table updates"),
 ]
 
 
+RND = sys.argv[2] if len(sys.argv) > 2 else "r01"
+
+
 def load(w):
-    return json.load(open(os.path.join(ROOT, "profiles", f"r01_bench_{w}.json")))
+    p = os.path.join(ROOT, "profiles", f"{RND}_bench_{w}.json")
+    return json.load(open(p)) if os.path.exists(p) else None
+
+
+def overlap(d):
+    """copy/compute overlap of the timed (graph-replayed) pass when traced, else the profiled pass"""
+    t = d.get("timed_pass_trace")
+    if d["config"].get("gather_mode") == "fused":
+        return "one launch"
+    if t and t.get("compute_busy_ms"):
+        return f"{t['overlap_frac']:.2f}"
+    return f"{d['overlap']['overlap_frac']:.2f}"
 
 
 def gbs(v):
@@ -31,6 +47,8 @@ def gbs(v):
 def design():
     for w, name, _, _ in ROWS:
         d = load(w)
+        if d is None:
+            continue
         fd = d.get("link_full_duplex")
         val = f"{d['value']:.1f} each way" if fd else f"{d['value']:.1f}"
         frac = (f"{d['link']['frac']:.2f} (H2D); {fd['frac']:.2f} of the {fd['peak_each_way_gbs']:.1f} GB/s "
@@ -39,13 +57,15 @@ def design():
         dbs = f"{db['bigkernel_speedup']:.2f}× ({db['value']:.1f})" if db else "—"
         mt = d.get("cpu_mt_baseline")
         print(f"| {name} | {d['config']['gather_mode'].upper()} | {val} | {d['ms_per_step']:.3g} | {frac} | "
-              f"{d['overlap']['overlap_frac']:.2f} | {dbs} | {gbs(mt['value']) if mt else '—'} | "
+              f"{overlap(d)} | {dbs} | {gbs(mt['value']) if mt else '—'} | "
               f"{gbs(d['cpu_baseline']['value'])} |")
 
 
 def readme():
     for w, _, name, note in ROWS:
         d = load(w)
+        if d is None:
+            continue
         fd = d.get("link_full_duplex")
         val = f"{d['value']:.1f} each way" if fd else f"{d['value']:.1f}"
         frac = f"{fd['frac']:.2f} of bidirectional" if fd else f"{d['link']['frac']:.2f}" + (f" ({note})" if note else "")
