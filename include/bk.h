@@ -174,7 +174,10 @@ typedef struct bk_out_header { uint32_t struct_size; int32_t kernel_id; } bk_out
 /* Result arrays of the aggregating kernels (word count, group-by, k-means, k-mers) may be HOST or
  * DEVICE pointers (device memory of the context's GPU): libbk copies with unified addressing, so a
  * multi-GPU caller can point them at the buffers its NCCL collectives reduce in place (SURVEY
- * §8(e)) with no host round trip. Host arrays need not be pinned. */
+ * §8(e)) with no host round trip. Host arrays need not be pinned. When every array of a word-count
+ * or k-mer result is reachable by kernels — device memory, caller-pinned host memory, or host
+ * memory kept pinned (BK_FLAG_KEEP_OUTPUTS_PINNED) — the final kernel stores the results into them
+ * directly (over PCIe for host memory) instead of staging them in HBM for a copy after the run. */
 typedef struct bk_out_wordcount {
   bk_out_header h;
   uint64_t table_slots;     /* in: device hash-table slots (power of two); 0 = 2^20 */

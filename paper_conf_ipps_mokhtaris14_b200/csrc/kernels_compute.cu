@@ -311,26 +311,69 @@ __global__ void __launch_bounds__(256) k_dbuf_wc(const uint8_t* __restrict__ raw
   }
 }
 
-__global__ void k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots, unsigned long long* n_out,
-                             unsigned long long* total, uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1,
-                             uint64_t* h2, uint64_t cap) {
+// Occupied slots -> the result arrays. Each block compacts 1024 consecutive slots into shared memory
+// (ballot + block scan, slot order), reserves its run with ONE atomic, and stores the run coalesced,
+// so the stores are long contiguous runs per array — the result arrays may be the caller's mapped
+// host memory, written over PCIe (a table is ~5% occupied: per-warp runs would be a few bytes each).
+// h1 / h2 (the word's two hashes, for the multi-GPU merge) are written only when asked for.
+constexpr int kCmpThreads = 256;
+constexpr uint32_t kCmpSlots = 1024;   // slots per block
+
+__global__ void __launch_bounds__(kCmpThreads) k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots,
+                                                            unsigned long long* n_out, unsigned long long* total,
+                                                            uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1,
+                                                            uint64_t* h2, uint64_t cap) {
+  __shared__ uint64_t s_off[kCmpSlots], s_cnt[kCmpSlots], s_h1[kCmpSlots], s_h2[kCmpSlots];
+  __shared__ uint32_t s_len[kCmpSlots];
+  __shared__ unsigned s_warp[kCmpThreads / 32];
+  __shared__ unsigned s_n;
+  __shared__ unsigned long long s_base;
+  const uint32_t tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const uint64_t lo = (uint64_t)blockIdx.x * kCmpSlots, hi = min(slots, lo + kCmpSlots);
+  if (tid == 0) s_n = 0;
   unsigned long long mine = 0;
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < slots; i += (uint64_t)gridDim.x * blockDim.x) {
-    const WcEntry e = table[i];
-    if (e.key1 == 0) continue;
-    mine += e.count;
-    const unsigned long long p = atomicAdd(n_out, 1ull);
-    if (p < cap) {
-      off[p] = e.offlen >> 24;
-      len[p] = (uint32_t)(e.offlen & 0xffffff);
-      cnt[p] = e.count;
-      h1[p] = e.key1;
-      h2[p] = e.key2;
+  for (uint64_t i0 = lo; i0 < hi; i0 += kCmpThreads) {
+    const uint64_t i = i0 + tid;
+    WcEntry e{};
+    if (i < hi) e = table[i];
+    const bool occ = e.key1 != 0;
+    const unsigned m = __ballot_sync(kFull, occ);
+    if (lane == 0) s_warp[w] = __popc(m);
+    __syncthreads();
+    unsigned before = s_n, tot = 0;
+    for (uint32_t q = 0; q < kCmpThreads / 32; ++q) {
+      before += q < w ? s_warp[q] : 0u;
+      tot += s_warp[q];
     }
+    if (occ) {
+      const unsigned p = before + __popc(m & ((1u << lane) - 1));
+      s_off[p] = e.offlen >> 24;
+      s_len[p] = (uint32_t)(e.offlen & 0xffffff);
+      s_cnt[p] = e.count;
+      s_h1[p] = e.key1;
+      s_h2[p] = e.key2;
+      mine += e.count;
+    }
+    __syncthreads();
+    if (tid == 0) s_n += tot;
+  }
+  __syncthreads();
+  const unsigned n = s_n;
+  if (tid == 0) s_base = n ? atomicAdd(n_out, (unsigned long long)n) : 0ull;
+  __syncthreads();
+  const unsigned long long base = s_base;
+  for (uint32_t j = tid; j < n; j += kCmpThreads) {
+    const unsigned long long p = base + j;
+    if (p >= cap) break;
+    off[p] = s_off[j];
+    len[p] = s_len[j];
+    cnt[p] = s_cnt[j];
+    if (h1) h1[p] = s_h1[j];
+    if (h2) h2[p] = s_h2[j];
   }
   // total words: one atomic per warp
   for (int o = 16; o; o >>= 1) mine += __shfl_down_sync(kFull, mine, o);
-  if ((threadIdx.x & 31) == 0 && mine) atomicAdd(total, mine);
+  if (lane == 0 && mine) atomicAdd(total, mine);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1078,7 +1121,8 @@ void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint6
 void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, unsigned long long* total,
                        uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1, uint64_t* h2, uint64_t cap,
                        cudaStream_t s) {
-  k_wc_compact<<<device_sms() * 4, 256, 0, s>>>(table, slots, n_out, total, off, len, cnt, h1, h2, cap);
+  k_wc_compact<<<(unsigned)((slots + kCmpSlots - 1) / kCmpSlots), kCmpThreads, 0, s>>>(table, slots, n_out, total, off,
+                                                                                     len, cnt, h1, h2, cap);
 }
 
 size_t grep_count_smem() { return stream_smem<true>(kGrepThreads / 32, kGrepRows); }

@@ -10,20 +10,50 @@ namespace rt {
 
 // ------------------------------------------------------------------ kernels
 
+// Where k_wc_compact stores the distinct words: straight into the caller's arrays when kernels can
+// reach all of them (device memory, or pinned / kept-pinned host memory through its mapped alias:
+// the PCIe stores replace a copy after the run), else into HBM staging copied by wordcount_results.
+struct WcOut {
+  uint64_t* off;
+  uint32_t* len;
+  uint64_t* cnt;
+  uint64_t* h1;
+  uint64_t* h2;
+  bool direct;
+  std::string key() const {
+    return direct ? "/d" + std::to_string((uintptr_t)off) + "." + std::to_string((uintptr_t)len) + "." +
+                        std::to_string((uintptr_t)cnt) + "." + std::to_string((uintptr_t)h1) + "." +
+                        std::to_string((uintptr_t)h2)
+                  : "/s" + std::to_string(h1 != nullptr);
+  }
+};
+
+static WcOut wordcount_out(bk_ctx* c, bk_out_wordcount* o, uint64_t ocap) {
+  WcOut w{};
+  w.off = (uint64_t*)out_kernel_ptr(c, o->word_off, ocap * 8);
+  w.len = w.off ? (uint32_t*)out_kernel_ptr(c, o->word_len, ocap * 4) : nullptr;
+  w.cnt = w.len ? (uint64_t*)out_kernel_ptr(c, o->word_count, ocap * 8) : nullptr;
+  w.h1 = o->word_h1 && w.cnt ? (uint64_t*)out_kernel_ptr(c, o->word_h1, ocap * 8) : nullptr;
+  w.h2 = o->word_h2 && w.cnt ? (uint64_t*)out_kernel_ptr(c, o->word_h2, ocap * 8) : nullptr;
+  w.direct = w.cnt && (!o->word_h1 || w.h1) && (!o->word_h2 || w.h2);
+  if (!w.direct) {
+    w.off = (uint64_t*)c->b_out1.p;
+    w.len = (uint32_t*)c->b_out2.p;
+    w.cnt = (uint64_t*)c->b_out3.p;
+    w.h1 = o->word_h1 ? (uint64_t*)c->b_h1.p : nullptr;
+    w.h2 = o->word_h2 ? (uint64_t*)c->b_h2.p : nullptr;
+  }
+  return w;
+}
+
 // distinct words + totals of the finished run -> the caller's (host or device) arrays
-static int wordcount_results(bk_ctx* c, bk_out_wordcount* o, uint64_t slots) {
+static int wordcount_results(bk_ctx* c, bk_out_wordcount* o, uint64_t slots, bool direct) {
   const unsigned long long nw = c->h_ctr[2];
   o->n_words = nw;
   if (nw > o->cap) return fail(BK_E_CAPACITY, "%llu distinct words > cap %llu", nw, (unsigned long long)o->cap);
   if (nw * 2 > slots) return fail(BK_E_CAPACITY, "table load %llu/%llu too high; raise table_slots", nw,
                                   (unsigned long long)slots);
-  if (nw && (c->cfg.flags & BK_FLAG_KEEP_OUTPUTS_PINNED)) {   // cached registrations: DMA-speed result copies
-    int rc;
-    if ((rc = ensure_out_pinned(c, o->word_off, o->cap * 8)) || (rc = ensure_out_pinned(c, o->word_len, o->cap * 4)) ||
-        (rc = ensure_out_pinned(c, o->word_count, o->cap * 8)))
-      return rc;
-  }
-  if (nw) {   // host or device result arrays (unified addressing)
+  if (nw && !direct) {   // host or device result arrays (unified addressing)
     BK_CUDA(cudaMemcpy(o->word_off, c->b_out1.p, nw * 8, cudaMemcpyDefault));
     BK_CUDA(cudaMemcpy(o->word_len, c->b_out2.p, nw * 4, cudaMemcpyDefault));
     BK_CUDA(cudaMemcpy(o->word_count, c->b_out3.p, nw * 8, cudaMemcpyDefault));
@@ -31,7 +61,7 @@ static int wordcount_results(bk_ctx* c, bk_out_wordcount* o, uint64_t slots) {
     if (o->word_h2) BK_CUDA(cudaMemcpy(o->word_h2, c->b_h2.p, nw * 8, cudaMemcpyDefault));
   }
   o->total_words = c->h_ctr[6];
-  c->st.bytes_d2h = nw * 20;
+  c->st.bytes_d2h = nw * (20 + (o->word_h1 ? 8 : 0) + (o->word_h2 ? 8 : 0));
   return BK_OK;
 }
 
@@ -93,7 +123,8 @@ MemOps& memops() {
 // CTAs stream units into an HBM ring carved from the window, consumer CTAs count. Returns
 // BK_E_RANGE (nothing enqueued) when the window cannot hold a ring of >= 2 units or a record does
 // not fit a unit: the caller then runs the event pipeline.
-static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uint64_t slots, uint64_t ocap) {
+static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uint64_t slots, uint64_t ocap,
+                               const WcOut& wo) {
   (void)o;
   const int grid = wc_fused_grid();
   if (grid < 2) return BK_E_RANGE;
@@ -190,7 +221,7 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
   // captured once per (table, units, ring, loaders) and replayed: two memsets, the cooperative
   // persistent kernel, the compaction
   const std::string key = "wcfused/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + ukey + "/" +
-                          std::to_string(R) + "/" + std::to_string(n_load);
+                          std::to_string(R) + "/" + std::to_string(n_load) + wo.key();
   // the DMA feed issues eagerly (stream memory operations are not graph-captured here)
   int rc = run_device(c, stream, key + (dma ? "/dma" : "/zc"), !dma, 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
@@ -223,8 +254,7 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
           return fail(BK_E_CUDA, "cuStreamWriteValue64");
       }
     }
-    launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
-                      (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p, ocap, c->s_comp);
+    launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, wo.off, wo.len, wo.cnt, wo.h1, wo.h2, ocap, c->s_comp);
     c->n_launch += 2;
     return (int)BK_OK;
   });
@@ -276,8 +306,9 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
     BK_CUDA(c->b_out3.ensure(std::max<uint64_t>(ocap0, 1) * 8));
     BK_CUDA(c->b_h1.ensure(std::max<uint64_t>(ocap0, 1) * 8));
     BK_CUDA(c->b_h2.ensure(std::max<uint64_t>(ocap0, 1) * 8));
-    const int frc = run_wordcount_fused(c, o, stream, slots, ocap0);
-    if (frc == BK_OK) return wordcount_results(c, o, slots);
+    const WcOut wo = wordcount_out(c, o, ocap0);
+    const int frc = run_wordcount_fused(c, o, stream, slots, ocap0, wo);
+    if (frc == BK_OK) return wordcount_results(c, o, slots, wo.direct);
     if (frc != BK_E_RANGE) return frc;
   }
   Plan p;
@@ -294,7 +325,8 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   BK_CUDA(c->b_h1.ensure(std::max<uint64_t>(ocap, 1) * 8));
   BK_CUDA(c->b_h2.ensure(std::max<uint64_t>(ocap, 1) * 8));
   WcEntry* table = (WcEntry*)c->b_table.p;
-  const std::string key = "wc/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + p.key;
+  const WcOut wo = wordcount_out(c, o, ocap);
+  const std::string key = "wc/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + p.key + wo.key();
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
     int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
@@ -304,13 +336,12 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
       return BK_OK;
     });
     if (r) return r;
-    launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p, (uint32_t*)c->b_out2.p,
-                      (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p, ocap, c->s_comp);
+    launch_wc_compact(table, slots, c->d_ctr + 2, c->d_ctr + 6, wo.off, wo.len, wo.cnt, wo.h1, wo.h2, ocap, c->s_comp);
     c->n_launch += 1;
     return (int)BK_OK;
   });
   if (rc) return rc;
-  return wordcount_results(c, o, slots);
+  return wordcount_results(c, o, slots, wo.direct);
 }
 
 int run_grep(bk_ctx* c, bk_out_grep* o, void* stream) {

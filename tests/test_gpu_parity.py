@@ -625,3 +625,34 @@ def test_results_survive_random_stage_delays(mode):
         ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=len(kv))
         out, cc, bc = ctx.partition(1024)
         assert np.array_equal(global_from_runs(out, cc), wout)
+
+
+@pytest.mark.parametrize("mode", ["fused", "zc"])
+@pytest.mark.parametrize("where", ["kept_pinned_host", "device", "pageable_host"])
+def test_wordcount_results_stored_by_the_compaction(mode, where):
+    """k_wc_compact stores the distinct words straight into the caller's arrays when kernels can reach
+    all of them (kept-pinned host memory through its mapped alias, device tensors); pageable host
+    arrays get a copy after the run. Same multiset either way, replayed graphs included."""
+    import torch
+    buf, off = gen.text(cap_bytes=3 * MIB)
+    want = oracle.wc(buf, off)
+    cap = 1 << 18
+    if where == "device":
+        out = (torch.zeros(cap, dtype=torch.int64, device="cuda"), torch.zeros(cap, dtype=torch.int32, device="cuda"),
+               torch.zeros(cap, dtype=torch.int64, device="cuda"), torch.zeros(cap, dtype=torch.int64, device="cuda"),
+               torch.zeros(cap, dtype=torch.int64, device="cuda"))
+    else:
+        out = (np.zeros(cap, np.uint64), np.zeros(cap, np.uint32), np.zeros(cap, np.uint64))
+    with bk.Context(window_bytes=2 * MIB, gather_mode=mode, keep_outputs_pinned=where == "kept_pinned_host") as ctx:
+        ctx.register(buf, off)
+        for _ in range(3):
+            r = ctx.wordcount(out=out)
+            o, ln, cnt = r[:3]
+            if where == "device":
+                o, ln, cnt = (o.cpu().numpy().view(np.uint64), ln.cpu().numpy().view(np.uint32),
+                              cnt.cpu().numpy().view(np.uint64))
+                h1, h2 = r[3].cpu().numpy(), r[4].cpu().numpy()
+                assert len(h1) == len(o) and np.all(h1 != 0)
+            assert wc_multiset_gpu(buf, o, ln, cnt) == want
+            for a in out:
+                a[:] = 0

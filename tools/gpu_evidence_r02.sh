@@ -32,6 +32,7 @@ line grep_addr --gather addr --gib 2 --steps 3 --warmup 3 --no-cpu-baseline --no
 line grep_ht2_hybrid --host-threads 2 --gib 4 --steps 3 --warmup 3 --no-cpu-baseline --no-dbuf
 line grep_ht2_zc --gather zc --host-threads 2 --gib 4 --steps 3 --warmup 3 --no-cpu-baseline --no-dbuf
 line grep_ht8_hybrid --host-threads 8 --gib 4 --steps 3 --warmup 3 --no-cpu-baseline --no-dbuf
+line grep_ht8_zc --gather zc --host-threads 8 --gib 4 --steps 3 --warmup 3 --no-cpu-baseline --no-dbuf
 timeout 900 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/${T}_bench_reference.json 2> gpurun_out/${T}_bench_reference.err
 tail -c 300 gpurun_out/${T}_bench_reference.json
 # launch lists (serialised, cold): each kernel's share of the step

@@ -14,4 +14,4 @@ cap() {  # name kernel-regex skip bench-args
 cap grep "k_gather_field" 6 "--workload grep --gib 4 --zc-share 1000"
 cap groupby_sparse "k_gather_field" 6 "--workload groupby_sparse --gib 4 --zc-share 1000"
 cap wordcount "k_wc_fused" 3 "--workload wordcount"
-cap kmer "k_kmer_bin" 6 "--workload kmer --gib 1"
+# k-mers: three kernels per chunk, per-kernel DRAM bytes in profiles/r02_kmer.md (no single roofline kernel)

@@ -116,4 +116,20 @@ with bk.Context(window_bytes=1 << 20, record_size=256, gather_mode="zc") as ctx:
     ctx.register(d, None, n_records=20_000)
     ctx.kmer(k=31, table_slots=1 << 20)
     ctx.kmer(k=31, table_slots=1 << 22)
+# results stored by the final kernels straight into kept-pinned host arrays (mapped) and device tensors;
+# a mid-run flush
+import numpy as np  # noqa: E402
+os.environ["BK_KMER_F"] = "1"
+with bk.Context(window_bytes=1 << 20, record_size=256, keep_outputs_pinned=True) as ctx:
+    ctx.register(d, None, n_records=20_000)
+    kout = (np.zeros(1 << 20, np.uint64), np.zeros(1 << 20, np.uint64))
+    ctx.kmer(k=31, table_slots=1 << 22, out=kout)
+    ctx.kmer(k=31, table_slots=1 << 22, out=(torch.zeros(1 << 20, dtype=torch.int64, device="cuda"),
+                                             torch.zeros(1 << 20, dtype=torch.int64, device="cuda")))
+os.environ.pop("BK_KMER_F")
+with bk.Context(window_bytes=256 << 10, keep_outputs_pinned=True) as ctx:
+    ctx.register(buf, off)
+    wout = (np.zeros(1 << 16, np.uint64), np.zeros(1 << 16, np.uint32), np.zeros(1 << 16, np.uint64))
+    ctx.wordcount(out=wout)
+    ctx.wordcount(out=wout)
 print("sanitize run (round 2) done")
