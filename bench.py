@@ -733,7 +733,8 @@ def main():
 
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": round(t_dev / args.steps * 1e3, 3), "higher_is_better": True,
+        "warmup": args.warmup, "ms_per_step": round(t_dev / args.steps * 1e3, 3),
+        "step_ms": [round(x, 3) for x in dev_ms], "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": DTYPE[args.workload], "data": "synthetic (seeded counter RNG, gen/)",
         "config": {"workload": args.workload, "desc": WORKLOADS[args.workload][2],
                    "bytes_per_gpu": nbytes, "records_per_gpu": shard["n"], "window_bytes": window,

@@ -296,58 +296,93 @@ uint64_t host_assemble_addr(HostPool& pool, const HostData& d, uint32_t L, uint3
 
 bool host_packable(const Access& a) { return !a.whole && a.n_ext == 1 && a.E > 0 && (a.E % 16) == 0; }
 
+// One packer thread: grabs of kGrab records from a shared counter, each record's E accessed bytes
+// copied in record order. Prefetch: near (into L1) PF records ahead — with END both ends of the
+// field (a 32-B key crosses a 64-B line for 3 of 8 record alignments) — and far (into L2) PF2
+// records ahead. Distances and the 16-B word count are template constants: the same distances read
+// from variables cost 15-24% of the packing rate in the bench (gpurun_out/r02bis3_*).
+namespace {
+using PackSink = std::function<void(uint64_t, uint64_t)>;
+using PackFn = void (*)(const HostData&, uint32_t, uint64_t, uint32_t, const Chunk&, uint8_t*, uint64_t, uint64_t, bool,
+                        const PackSink*, std::atomic<uint64_t>&);
+
+template <int PF, int PF2, bool END, int EWC>
+void pack_worker(const HostData& d, uint32_t eo, uint64_t E, uint32_t ew, const Chunk& c, uint8_t* dst, uint64_t n,
+                 uint64_t kGrab, bool nt, const PackSink* sink, std::atomic<uint64_t>& next) {
+  const uint32_t EW = EWC ? (uint32_t)EWC : ew;
+  auto src = [&](uint64_t r) { return d.base + (d.off ? d.off[r] : r * d.rec_size) + eo; };
+  auto pf = [&](uint64_t r) {
+    const uint8_t* p = src(r);
+    __builtin_prefetch(p);
+    if (END) __builtin_prefetch(p + E - 1);
+  };
+  for (;;) {
+    const uint64_t j0 = next.fetch_add(kGrab);
+    if (j0 >= n) break;
+    const uint64_t j1 = std::min(n, j0 + kGrab);
+    for (uint64_t j = j0; j < std::min<uint64_t>(j1, j0 + PF); ++j) pf(c.lo + j);
+    if (PF2)
+      for (uint64_t j = j0; j < std::min<uint64_t>(j1, j0 + PF2); ++j) _mm_prefetch((const char*)src(c.lo + j), _MM_HINT_T1);
+    if (nt) {
+      for (uint64_t j = j0; j < j1; ++j) {
+        if (j + PF < j1) pf(c.lo + j + PF);
+        if (PF2 && j + PF2 < j1) _mm_prefetch((const char*)src(c.lo + j + PF2), _MM_HINT_T1);
+        const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
+        __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
+        for (uint32_t m = 0; m < EW; ++m) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
+      }
+      if (sink) _mm_sfence();
+    } else {
+      for (uint64_t j = j0; j < j1; ++j) {
+        if (j + PF < j1) pf(c.lo + j + PF);
+        if (PF2 && j + PF2 < j1) _mm_prefetch((const char*)src(c.lo + j + PF2), _MM_HINT_T1);
+        const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
+        __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
+        for (uint32_t m = 0; m < EW; ++m) _mm_storeu_si128(o + m, _mm_loadu_si128(s + m));
+      }
+    }
+    if (sink) (*sink)(j0 * E, (j1 - j0) * E);
+  }
+  _mm_sfence();
+}
+
+template <int PF, int PF2, bool END>
+PackFn pack_for_ew(uint32_t ew) {
+  switch (ew) {
+    case 1: return pack_worker<PF, PF2, END, 1>;
+    case 2: return pack_worker<PF, PF2, END, 2>;
+    case 6: return pack_worker<PF, PF2, END, 6>;
+    default: return pack_worker<PF, PF2, END, 0>;
+  }
+}
+
+// prefetch configurations {near, far, both ends}; BK_PACK_CFG selects one (sweep knob). In the bench
+// (HYBRID, zero-copy gathers running; profiles/r02_packer.md): grep 16/0/- 205.7 GB/s, 8/64/ends
+// 208.7, 16/64/ends 210.0, 16/0/ends 199.8, 32/128/ends 205.0, 8/0/ends 201.5; sparse group-by
+// 16/0/- 108.9, 8/64/ends 115.3, 16/0/ends 111.5. Default: 8/64/ends.
+PackFn pack_fn(uint32_t ew) {
+  static const int cfg = getenv("BK_PACK_CFG") ? atoi(getenv("BK_PACK_CFG")) : 2;
+  switch (cfg) {
+    case 1: return pack_for_ew<16, 0, false>(ew);   // round 1
+    case 3: return pack_for_ew<16, 64, true>(ew);
+    case 4: return pack_for_ew<16, 0, true>(ew);
+    case 5: return pack_for_ew<32, 128, true>(ew);
+    case 6: return pack_for_ew<8, 0, true>(ew);
+    default: return pack_for_ew<8, 64, true>(ew);
+  }
+}
+}  // namespace
+
 uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, const Chunk& c, uint8_t* dst,
                          uint64_t cap, uint64_t grab, bool nt, const std::function<void(uint64_t, uint64_t)>* sink) {
   const uint64_t E = a.E, n = c.hi - c.lo, size = n * E;
   if (size > cap) return UINT64_MAX;
   const uint32_t eo = a.ext_off[0], EW = (uint32_t)(E / 16);
-  // sweep on the 16-core host (profiles/r01_hybrid_sweep.md): 16-record prefetch distance, grabs of
-  // 4k-16k records read in order
+  // sweep on the 16-core host (profiles/r01_hybrid_sweep.md): grabs of 4k-16k records read in order
   const uint64_t kGrab = grab ? grab : 16384;
-  // prefetch: near (into L1) kPf records ahead, both ends of the field (a 32-B key crosses a 64-B line
-  // for 3 of 8 record alignments), and far (into L2) kPf2 records ahead. Sweep on the gpurun box's
-  // 16 vCPUs (tools/host_gather_bench.cpp, gpurun_out/r02s_hgb_*): near 16 only 0.58 G rec/s,
-  // near 8 + both ends + far 64 0.72 G rec/s (+23%). BK_PACK_PF / BK_PACK_PF2 / BK_PACK_PFEND
-  // override (sweep knobs).
-  static const uint64_t kPf = getenv("BK_PACK_PF") ? (uint64_t)atoll(getenv("BK_PACK_PF")) : 8;
-  static const uint64_t kPf2 = getenv("BK_PACK_PF2") ? (uint64_t)atoll(getenv("BK_PACK_PF2")) : 64;
-  static const bool kPfEnd = getenv("BK_PACK_PFEND") ? atoi(getenv("BK_PACK_PFEND")) != 0 : true;
+  const PackFn fn = pack_fn(EW);
   std::atomic<uint64_t> next{0};
-  pool.run([&](int) {
-    auto src = [&](uint64_t r) { return d.base + (d.off ? d.off[r] : r * d.rec_size) + eo; };
-    auto pf = [&](uint64_t r) {
-      const uint8_t* p = src(r);
-      __builtin_prefetch(p);
-      if (kPfEnd) __builtin_prefetch(p + E - 1);
-    };
-    for (;;) {
-      const uint64_t j0 = next.fetch_add(kGrab);
-      if (j0 >= n) break;
-      const uint64_t j1 = std::min(n, j0 + kGrab);
-      for (uint64_t j = j0; j < std::min(j1, j0 + kPf); ++j) pf(c.lo + j);
-      for (uint64_t j = j0; kPf2 && j < std::min(j1, j0 + kPf2); ++j) _mm_prefetch((const char*)src(c.lo + j), _MM_HINT_T1);
-      if (nt) {
-        for (uint64_t j = j0; j < j1; ++j) {
-          if (j + kPf < j1) pf(c.lo + j + kPf);
-          if (kPf2 && j + kPf2 < j1) _mm_prefetch((const char*)src(c.lo + j + kPf2), _MM_HINT_T1);
-          const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
-          __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
-          for (uint32_t m = 0; m < EW; ++m) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
-        }
-        if (sink) _mm_sfence();
-      } else {
-        for (uint64_t j = j0; j < j1; ++j) {
-          if (j + kPf < j1) pf(c.lo + j + kPf);
-          if (kPf2 && j + kPf2 < j1) _mm_prefetch((const char*)src(c.lo + j + kPf2), _MM_HINT_T1);
-          const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
-          __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
-          for (uint32_t m = 0; m < EW; ++m) _mm_storeu_si128(o + m, _mm_loadu_si128(s + m));
-        }
-      }
-      if (sink) (*sink)(j0 * E, (j1 - j0) * E);
-    }
-    _mm_sfence();
-  });
+  pool.run([&](int) { fn(d, eo, E, EW, c, dst, n, kGrab, nt, sink, next); });
   return size;
 }
 
