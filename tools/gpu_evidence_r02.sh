@@ -18,6 +18,10 @@ line() {  # name bench-args...
   python3 -c "import json;d=json.loads(open('gpurun_out/${T}_bench_$name.json').read().splitlines()[-1]);print('$name', d['value'], d['ms_per_step'], round(d['roofline']['frac'],3), d['link']['frac'])" \
     || tail -3 gpurun_out/${T}_bench_$name.err
 }
+# the round-1 tree on the same box (ab_r01/: git archive of the round-1 head, built in place), grep only
+(cd ab_r01 2>/dev/null && timeout 900 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-dbuf \
+    > ../gpurun_out/${T}_bench_grep_r01tree.json 2> ../gpurun_out/${T}_bench_grep_r01tree.err) && \
+  python3 -c "import json;d=json.loads(open('gpurun_out/${T}_bench_grep_r01tree.json').read().splitlines()[-1]);print('grep_r01tree', d['value'], d['ms_per_step'])"
 line grep --steps 10 --warmup 3
 line wordcount --workload wordcount --steps 20 --warmup 5
 line groupby --workload groupby --steps 3 --warmup 3
