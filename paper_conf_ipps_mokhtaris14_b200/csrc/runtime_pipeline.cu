@@ -670,8 +670,15 @@ void* out_kernel_ptr(bk_ctx* c, void* ptr, uint64_t bytes) {
       return nullptr;
     }
   }
-  void* d = nullptr;
-  if (cudaHostGetDevicePointer(&d, ptr, 0) != cudaSuccess) {
+  // pinned host memory: both ends of the range must be mapped, at the same distance on the device
+  // (a registration covers whole pages, so an array can start inside another array's registered page
+  // and run past it; kernels would then store through an unmapped address)
+  uint8_t* last = static_cast<uint8_t*>(ptr) + bytes - 1;
+  cudaPointerAttributes at_last;
+  void *d = nullptr, *d_last = nullptr;
+  if (cudaPointerGetAttributes(&at_last, last) != cudaSuccess || at_last.type != cudaMemoryTypeHost ||
+      cudaHostGetDevicePointer(&d, ptr, 0) != cudaSuccess || cudaHostGetDevicePointer(&d_last, last, 0) != cudaSuccess ||
+      static_cast<uint8_t*>(d_last) - static_cast<uint8_t*>(d) != (ptrdiff_t)(bytes - 1)) {
     cudaGetLastError();
     return nullptr;
   }

@@ -152,3 +152,21 @@ def test_kmer_results_stored_by_the_flush(where):
             assert np.array_equal(gk, wk) and np.array_equal(gc, wc) and total == int(wc.sum())
             out[0][:] = 0
             out[1][:] = 0
+
+
+def test_kmer_direct_store_capacity_error_then_recovers():
+    """Kept-pinned result arrays smaller than the distinct k-mers: BK_E_CAPACITY (the flush stored only
+    what fits), then a run into large enough arrays on the same context is exact."""
+    n = 5000
+    buf = gen.dna(n=n, genome_len=1 << 16, err_pm=2, n_pm=3)
+    wk, wc = oracle.kmer(buf, n, 31)
+    small = (np.zeros(len(wk) // 2, np.uint64), np.zeros(len(wk) // 2, np.uint64))
+    big = (np.zeros(len(wk) + 10, np.uint64), np.zeros(len(wk) + 10, np.uint64))
+    with bk.Context(window_bytes=1 * MIB, record_size=256, keep_outputs_pinned=True) as ctx:
+        ctx.register(buf, None, n_records=n)
+        with pytest.raises(bk.BkError) as e:
+            ctx.kmer(k=31, table_slots=1 << 20, out=small)
+        assert e.value.status == bk.BK_E_CAPACITY
+        km, ct, total = ctx.kmer(k=31, table_slots=1 << 20, out=big)
+        gk, gc = sorted_pairs(km, ct)
+        assert np.array_equal(gk, wk) and np.array_equal(gc, wc) and total == int(wc.sum())

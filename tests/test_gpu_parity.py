@@ -656,3 +656,18 @@ def test_wordcount_results_stored_by_the_compaction(mode, where):
             assert wc_multiset_gpu(buf, o, ln, cnt) == want
             for a in out:
                 a[:] = 0
+
+
+def test_wordcount_direct_store_capacity_error_then_recovers():
+    """Kept-pinned result arrays smaller than the vocabulary: BK_E_CAPACITY, then the same context
+    with large enough arrays (another captured graph) is exact."""
+    buf, off = gen.text(cap_bytes=1 * MIB)
+    want = oracle.wc(buf, off)
+    small = (np.zeros(100, np.uint64), np.zeros(100, np.uint32), np.zeros(100, np.uint64))
+    big = (np.zeros(1 << 17, np.uint64), np.zeros(1 << 17, np.uint32), np.zeros(1 << 17, np.uint64))
+    with bk.Context(window_bytes=2 * MIB, keep_outputs_pinned=True) as ctx:
+        ctx.register(buf, off)
+        with pytest.raises(bk.BkError) as e:
+            ctx.wordcount(out=small)
+        assert e.value.status == bk.BK_E_CAPACITY
+        assert wc_multiset_gpu(buf, *ctx.wordcount(out=big)) == want
