@@ -71,6 +71,8 @@ def parse():
     args = ap.parse_args()
     if args.slots == 0 and args.workload == "wordcount":
         args.slots = 8   # the 8 MiB window: more, smaller chunks in flight (profiles/r01_wc_sweep.md)
+    if args.slots == 0 and args.workload == "partition":
+        args.slots = 12  # smaller chunks shorten the one-direction fill and drain (profiles/r02_partition.md)
     return args
 
 

@@ -361,7 +361,8 @@ PackFn pack_for_ew(uint32_t ew) {
 // 208.7, 16/64/ends 210.0, 16/0/ends 199.8, 32/128/ends 205.0, 8/0/ends 201.5; sparse group-by
 // 16/0/- 108.9, 8/64/ends 115.3, 16/0/ends 111.5. Default: 8/64/ends.
 PackFn pack_fn(uint32_t ew) {
-  static const int cfg = getenv("BK_PACK_CFG") ? atoi(getenv("BK_PACK_CFG")) : 2;
+  const char* e = getenv("BK_PACK_CFG");   // read per chunk (one call), so a process can switch
+  const int cfg = e ? atoi(e) : 2;
   switch (cfg) {
     case 1: return pack_for_ew<16, 0, false>(ew);   // round 1
     case 3: return pack_for_ew<16, 64, true>(ew);

@@ -671,3 +671,37 @@ def test_wordcount_direct_store_capacity_error_then_recovers():
             ctx.wordcount(out=small)
         assert e.value.status == bk.BK_E_CAPACITY
         assert wc_multiset_gpu(buf, *ctx.wordcount(out=big)) == want
+
+
+@pytest.mark.parametrize("env", [{"BK_FUSED_FEED": "dma", "BK_FUSED_BATCHES": "2"},
+                                 {"BK_FUSED_FEED": "dma", "BK_FUSED_BATCHES": "5"},
+                                 {"BK_FUSED_LOADERS": "1", "BK_FUSED_UNIT": "4096"},
+                                 {"BK_FUSED_LOADERS": "9", "BK_FUSED_UNIT": "65536"}])
+def test_wordcount_fused_knobs(monkeypatch, env):
+    """The single launch's tuning knobs (copy-engine feed and its batch slots, loader count, unit
+    size) change the schedule, never the table."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    buf, off = gen.text(cap_bytes=3 * MIB)
+    want = oracle.wc(buf, off)
+    with bk.Context(window_bytes=2 * MIB, gather_mode="fused") as ctx:
+        ctx.register(buf, off)
+        for _ in range(2):
+            assert wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 18)) == want
+
+
+@pytest.mark.parametrize("cfg", ["1", "2", "3", "4", "5", "6"])
+def test_host_packer_prefetch_configs(monkeypatch, cfg):
+    """Every host-packer prefetch configuration (BK_PACK_CFG) packs the same bytes: grep keys of
+    variable records (2 words per field) and sparse group-by fields (1 word) through CPU assembly."""
+    monkeypatch.setenv("BK_PACK_CFG", cfg)
+    gb, goff = gen.grep_records(max_bytes=4 * MIB)
+    with bk.Context(window_bytes=1 * MIB, gather_mode="cpu") as ctx:
+        ctx.register(gb, goff)
+        assert np.array_equal(ctx.grep(b"bigk", cap=len(goff)), oracle.grep(gb, goff, b"bigk"))
+    g = gen.groupby(n=60_000, stride=64)
+    wc_, wq, wa = oracle.groupby(g, 60_000, 64, 4096)
+    with bk.Context(window_bytes=1 * MIB, record_size=64, gather_mode="cpu") as ctx:
+        ctx.register(g, None, n_records=60_000)
+        c, q, a = ctx.groupby(4096)
+        assert np.array_equal(c, wc_) and np.array_equal(q, wq) and np.allclose(a, wa, rtol=1e-5, atol=0)
