@@ -126,7 +126,7 @@ void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint6
                     uint64_t end_byte, uint64_t rec_size, WcEntry* table, uint64_t mask, unsigned long long* used,
                     int* err, cudaStream_t s);
 // distinct words -> (occurrence offset, length, count, key1, key2) rows; *total += every count
-void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, unsigned long long* total,
+void launch_wc_compact(WcEntry* table, uint64_t slots, unsigned long long* n_out, unsigned long long* total,
                        uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1, uint64_t* h2, uint64_t cap,
                        cudaStream_t s);
 

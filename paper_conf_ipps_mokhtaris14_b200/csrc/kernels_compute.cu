@@ -311,7 +311,7 @@ __global__ void __launch_bounds__(256) k_dbuf_wc(const uint8_t* __restrict__ raw
   }
 }
 
-// Occupied slots -> the result arrays. Each block compacts 1024 consecutive slots into shared memory
+// Occupied slots -> the result arrays, each drained slot zeroed. Each block compacts 1024 consecutive slots into shared memory
 // (ballot + block scan, slot order), reserves its run with ONE atomic, and stores the run coalesced,
 // so the stores are long contiguous runs per array — the result arrays may be the caller's mapped
 // host memory, written over PCIe (a table is ~5% occupied: per-warp runs would be a few bytes each).
@@ -319,7 +319,7 @@ __global__ void __launch_bounds__(256) k_dbuf_wc(const uint8_t* __restrict__ raw
 constexpr int kCmpThreads = 256;
 constexpr uint32_t kCmpSlots = 1024;   // slots per block
 
-__global__ void __launch_bounds__(kCmpThreads) k_wc_compact(const WcEntry* __restrict__ table, uint64_t slots,
+__global__ void __launch_bounds__(kCmpThreads) k_wc_compact(WcEntry* __restrict__ table, uint64_t slots,
                                                             unsigned long long* n_out, unsigned long long* total,
                                                             uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1,
                                                             uint64_t* h2, uint64_t cap) {
@@ -346,6 +346,7 @@ __global__ void __launch_bounds__(kCmpThreads) k_wc_compact(const WcEntry* __res
       tot += s_warp[q];
     }
     if (occ) {
+      table[i] = WcEntry{};   // drained: the table is all zero for the next run (no memset)
       const unsigned p = before + __popc(m & ((1u << lane) - 1));
       s_off[p] = e.offlen >> 24;
       s_len[p] = (uint32_t)(e.offlen & 0xffffff);
@@ -1118,7 +1119,7 @@ void launch_dbuf_wc(const uint8_t* raw, const uint64_t* meta, uint64_t lo, uint6
   k_dbuf_wc<<<device_sms() * 4, 256, 0, s>>>(raw, meta, lo, hi, base_byte, end_byte, rec_size, table, mask, used, err);
 }
 
-void launch_wc_compact(const WcEntry* table, uint64_t slots, unsigned long long* n_out, unsigned long long* total,
+void launch_wc_compact(WcEntry* table, uint64_t slots, unsigned long long* n_out, unsigned long long* total,
                        uint64_t* off, uint32_t* len, uint64_t* cnt, uint64_t* h1, uint64_t* h2, uint64_t cap,
                        cudaStream_t s) {
   k_wc_compact<<<(unsigned)((slots + kCmpSlots - 1) / kCmpSlots), kCmpThreads, 0, s>>>(table, slots, n_out, total, off,

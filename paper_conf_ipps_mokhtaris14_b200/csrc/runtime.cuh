@@ -198,6 +198,8 @@ struct bk_ctx {  // the opaque context of include/bk.h
   std::vector<bk::trace::Rec> trace_recs;    // BK_FLAG_TRACE: this run's CUPTI records
   bool tracing = false;
   double hy_t_zc_ms = 0, hy_t_cpu_ms = 0;    // HYBRID: measured ms per zero-copy / host-packed chunk
+  void* wc_clean_ptr = nullptr;              // word count: b_table is all zero in its first
+  uint64_t wc_clean_slots = 0;               //   wc_clean_slots entries (drained by the last run)
   bk_addr_fn a_gen = nullptr;                // bk_run_user_addr generator + its argument
   void* a_gen_user = nullptr;
   bk::rt::DevBuf b_mown, b_mcnt, b_mctr;     // bk_merge_counts scratch (never captured in a graph)

@@ -65,6 +65,21 @@ static int wordcount_results(bk_ctx* c, bk_out_wordcount* o, uint64_t slots, boo
   return BK_OK;
 }
 
+// The word-count table between runs: k_wc_compact zeroes every slot it drains, so after a completed
+// run the table's first `slots` entries are zero and the next run skips the 32-MB memset. The memset
+// runs (eagerly, ahead of the run's graph on the compute stream) when the table is new or grown, was
+// used by another kernel (k-mers, the baselines), or the last run did not complete.
+static int wc_table_begin(bk_ctx* c, uint64_t slots) {
+  const bool clean = c->wc_clean_ptr == c->b_table.p && c->wc_clean_slots >= slots;
+  c->wc_clean_ptr = nullptr;   // dirty until this run's compaction has completed
+  if (!clean) BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
+  return BK_OK;
+}
+static void wc_table_end(bk_ctx* c, uint64_t slots) {
+  c->wc_clean_ptr = c->b_table.p;
+  c->wc_clean_slots = slots;
+}
+
 // BK_GATHER_FUSED unit plan: greedy whole records, each unit <= UB bytes and <= UR records (A3 with a
 // second cap: shared-memory slots hold the unit's offsets too). 0 on success, BK_E_RANGE when a
 // record exceeds UB (the caller falls back to the event pipeline).
@@ -223,8 +238,8 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
   const std::string key = "wcfused/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + ukey + "/" +
                           std::to_string(R) + "/" + std::to_string(n_load) + wo.key();
   // the DMA feed issues eagerly (stream memory operations are not graph-captured here)
+  if (int r0 = wc_table_begin(c, slots)) return r0;
   int rc = run_device(c, stream, key + (dma ? "/dma" : "/zc"), !dma, 1, [&]() -> int {
-    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
     BK_CUDA(cudaMemsetAsync(ready, 0, 2 * NF * 8 + K * 4, c->s_comp));
     if (prof) BK_CUDA(cudaMemsetAsync(c->d_fprof, 0, 8 * 8, c->s_comp));
     if (dma) {   // the copy stream starts after the flags are cleared
@@ -259,6 +274,7 @@ static int run_wordcount_fused(bk_ctx* c, bk_out_wordcount* o, void* stream, uin
     return (int)BK_OK;
   });
   if (rc) return rc;
+  wc_table_end(c, slots);
   c->st.gather_mode = BK_GATHER_FUSED;
   c->st.chunk_budget = UB;
   c->st.n_chunks = U;
@@ -327,8 +343,8 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
   WcEntry* table = (WcEntry*)c->b_table.p;
   const WcOut wo = wordcount_out(c, o, ocap);
   const std::string key = "wc/" + std::to_string(slots) + "/" + std::to_string(ocap) + "/" + p.key + wo.key();
+  if ((rc = wc_table_begin(c, slots))) return rc;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
-    BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(WcEntry), c->s_comp));
     int r = pipeline(c, p, true, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t&) {
       launch_wc(ch, s.stage, s.lanes, s.tile_base, s.meta, c->off ? 0 : c->cfg.record_size, table, slots - 1,
                 c->d_ctr + 1, c->d_err, cs);
@@ -341,6 +357,7 @@ int run_wordcount(bk_ctx* c, bk_out_wordcount* o, void* stream) {
     return (int)BK_OK;
   });
   if (rc) return rc;
+  wc_table_end(c, slots);
   return wordcount_results(c, o, slots, wo.direct);
 }
 
@@ -497,6 +514,7 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
 // Two-phase (kernels_kmer.cu): per chunk every k-mer key is appended to its table region's bucket,
 // and flushes count whole buckets into their regions in shared memory.
 int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
+  c->wc_clean_ptr = nullptr;   // the table buffer holds k-mer regions now
   const uint64_t slots = o->table_slots ? o->table_slots : (1ull << 24);
   if (slots & (slots - 1)) return fail(BK_E_INVAL, "table_slots must be a power of two");
   if (o->k < 1 || o->k > 31) return fail(BK_E_INVAL, "k must be in 1..31");
@@ -667,6 +685,7 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
 
 // ---- BK_FLAG_BASELINE_DBUF: the traditional chunked loop with two buffers ----
 int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
+  c->wc_clean_ptr = nullptr;   // the baselines use the table buffer with their own memset
   if (kid != BK_K_GREP && kid != BK_K_GROUPBY && kid != BK_K_KMEANS && kid != BK_K_WORDCOUNT)
     return fail(BK_E_UNSUPPORTED, "dbuf baseline: word count / grep / group-by / k-means only");
   Plan p;
@@ -800,7 +819,7 @@ int run_dbuf(bk_ctx* c, int kid, void* out, void* stream) {
     BK_CUDA(cudaStreamWaitEvent(c->s_comp, c->ev_end, 0));
   }
   if (kid == BK_K_WORDCOUNT) {
-    launch_wc_compact((const WcEntry*)c->b_table.p, wc_slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p,
+    launch_wc_compact((WcEntry*)c->b_table.p, wc_slots, c->d_ctr + 2, c->d_ctr + 6, (uint64_t*)c->b_out1.p,
                       (uint32_t*)c->b_out2.p, (uint64_t*)c->b_out3.p, (uint64_t*)c->b_h1.p, (uint64_t*)c->b_h2.p,
                       wc_ocap, c->s_comp);
     c->n_launch += 1;
