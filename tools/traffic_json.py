@@ -4,7 +4,7 @@ capture per kernel (tools/gpu_traffic.sh) plus the bench JSON line of the same c
 launch). Writes profiles/r02_traffic.json; bench.py scales it to its own launch size into
 roofline.traffic.
 
-    python tools/traffic_json.py r02f > profiles/r02_traffic.json
+    python tools/traffic_json.py r02h > profiles/r02_traffic.json
 """
 import csv
 import io
