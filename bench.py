@@ -398,10 +398,14 @@ def main():
 
     # one process per GPU; BK_BENCH_BACKEND=gloo lets several ranks share one GPU for a smoke test
     backend = os.environ.get("BK_BENCH_BACKEND", "nccl")
+    # BK_BENCH_DIST=1 runs the distributed path (process group, device-resident results, merge.py's
+    # collectives) even at world size 1: `torchrun --nproc-per-node 1` exercises the real NCCL calls
+    # on a one-GPU box (tests/test_gpu_nccl.py)
+    dist_on = world > 1 or os.environ.get("BK_BENCH_DIST") == "1"
     local = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
+    if dist_on:
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=dev)
         else:
@@ -439,21 +443,21 @@ def main():
     if args.workload == "kmer":
         kcap = 1 << 27
         kmer_out = ((torch.zeros(kcap, dtype=torch.int64, device=dev), torch.zeros(kcap, dtype=torch.int64, device=dev))
-                    if world > 1 else (np.zeros(kcap, np.uint64), np.zeros(kcap, np.uint64)))
+                    if dist_on else (np.zeros(kcap, np.uint64), np.zeros(kcap, np.uint64)))
     if args.workload == "wordcount":
         wcap = 1 << 20
         wc_out = ((torch.zeros(wcap, dtype=torch.int64, device=dev), torch.zeros(wcap, dtype=torch.int32, device=dev),
                    torch.zeros(wcap, dtype=torch.int64, device=dev), torch.zeros(wcap, dtype=torch.int64, device=dev),
                    torch.zeros(wcap, dtype=torch.int64, device=dev))
-                  if world > 1 else (np.zeros(wcap, np.uint64), np.zeros(wcap, np.uint32), np.zeros(wcap, np.uint64)))
+                  if dist_on else (np.zeros(wcap, np.uint64), np.zeros(wcap, np.uint32), np.zeros(wcap, np.uint64)))
     if args.workload in ("groupby", "groupby_sparse"):
         cq = torch.zeros(2, 4096, dtype=torch.int64, device=dev)
-        agg_out = ((cq[0], cq[1], torch.zeros(4096, dtype=torch.float64, device=dev), cq) if world > 1 else
+        agg_out = ((cq[0], cq[1], torch.zeros(4096, dtype=torch.float64, device=dev), cq) if dist_on else
                    (np.zeros(4096, np.uint64), np.zeros(4096, np.uint64), np.zeros(4096, np.float64)))
     if args.workload == "kmeans":
         agg_out = ((torch.zeros(args.K, dtype=torch.int64, device=dev),
                     torch.zeros(args.K, 16, dtype=torch.float64, device=dev))
-                   if world > 1 else (np.zeros(args.K, np.uint64), np.zeros((args.K, 16), np.float64)))
+                   if dist_on else (np.zeros(args.K, np.uint64), np.zeros((args.K, 16), np.float64)))
 
     from paper_conf_ipps_mokhtaris14_b200 import merge
 
@@ -465,36 +469,36 @@ def main():
         cs = stream.cuda_stream
         if args.workload == "grep":
             res = ctx.grep(b"bigk", first_index=shard["first"], stream=cs, out=idx_out)
-            return {"idx": res, "place": merge.merge_grep_offsets(len(res)) if world > 1 else (0, len(res))}
+            return {"idx": res, "place": merge.merge_grep_offsets(len(res)) if dist_on else (0, len(res))}
         if args.workload == "wordcount":
             r = ctx.wordcount(stream=cs, out=wc_out)
-            if world > 1:   # all-gather of compacted {h1, h2, len, count, rank, off} rows, merged on the GPU
+            if dist_on:   # all-gather of compacted {h1, h2, len, count, rank, off} rows, merged on the GPU
                 rows = merge.merge_wordcount(ctx, *r)
                 return {"rows": rows.cpu().numpy()}
             return {"off": r[0], "len": r[1], "count": r[2]}
         if args.workload == "kmer":
             km, ct, total = ctx.kmer(k=31, table_slots=1 << 28, stream=cs, out=kmer_out)
             box["kmer_windows"] = total
-            if world > 1:
+            if dist_on:
                 rows = merge.merge_kmer(ctx, km, ct)
                 return {"rows": rows.cpu().numpy()}
             return {"kmer": km, "count": ct}
         if args.workload == "partition":
             out, cc, bc = ctx.partition(1024, out=shard["out"], stream=cs)
             box["part_cc"] = cc
-            if world > 1:
+            if dist_on:
                 start, boff = merge.merge_partition_offsets(bc)
                 return {"start": start, "boff": boff, "cc": cc}
             return {"cc": cc, "bc": bc}
         if args.workload in ("groupby", "groupby_sparse"):
             c, q, a = ctx.groupby(4096, stream=cs, out=agg_out[:3])
-            if world > 1:   # in place on the device buffers bk_run wrote
+            if dist_on:   # in place on the device buffers bk_run wrote
                 merge.merge_sum(agg_out[3])
                 merge.merge_sum(a)
                 return {"count": c.cpu().numpy(), "qty": q.cpu().numpy(), "amount": a.cpu().numpy()}
             return {"count": c, "qty": q, "amount": a}
         c, s_, chk = ctx.kmeans(shard["mu"], first_index=shard["first"], stream=cs, out=agg_out)
-        if world > 1:
+        if dist_on:
             merge.merge_sum(c)
             merge.merge_sum(s_)
             chk = merge.merge_checksum(chk)
@@ -504,13 +508,13 @@ def main():
     for _ in range(args.warmup):
         one_step()
     torch.cuda.synchronize()
-    if world > 1:
+    if dist_on:
         dist.barrier()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     wall, dev_ms, stats = [], [], []
     with ClockSampler(local) as clk:
         torch.cuda.synchronize()
-        if world > 1:
+        if dist_on:
             dist.barrier()
         for k in range(args.steps):
             h0 = time.perf_counter()
@@ -521,12 +525,12 @@ def main():
             wall.append(time.perf_counter() - h0)
             stats.append(ctx.stats())
         torch.cuda.synchronize()
-        if world > 1:
+        if dist_on:
             dist.barrier()
     dev_ms = [a.elapsed_time(b) for a, b in ev]
     t_dev = sum(dev_ms) / 1e3
     t_wall = sum(wall)
-    if world > 1:  # max over ranks
+    if dist_on:  # max over ranks
         tt = torch.tensor([t_dev, t_wall], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t_dev, t_wall = tt.tolist()
@@ -834,7 +838,7 @@ def main():
         b_.record(stream)
         b_.synchronize()
         dt = a_.elapsed_time(b_) / 1e3
-        if world > 1:
+        if dist_on:
             tt = torch.tensor([dt], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             dt = tt.item()
@@ -892,7 +896,7 @@ def main():
     if rank == 0:
         print(json.dumps(line), flush=True)
     ctx.close()
-    if world > 1:
+    if dist_on:
         dist.barrier()
         dist.destroy_process_group()
 
