@@ -306,7 +306,28 @@ using PackSink = std::function<void(uint64_t, uint64_t)>;
 using PackFn = void (*)(const HostData&, uint32_t, uint64_t, uint32_t, const Chunk&, uint8_t*, uint64_t, uint64_t, bool,
                         const PackSink*, std::atomic<uint64_t>&);
 
-template <int PF, int PF2, bool END, int EWC>
+// copies one record's EW 16-B words: with W32 (EW even, 32-B aligned destination) as 32-B AVX2
+// loads / stores, half the memory instructions of the 16-B loop
+template <int EWC, bool W32, bool NT>
+inline void copy_field(const uint8_t* sp, uint8_t* op, uint32_t EW) {
+  if (W32) {
+    const __m256i* s = reinterpret_cast<const __m256i*>(sp);
+    __m256i* o = reinterpret_cast<__m256i*>(op);
+    for (uint32_t m = 0; m < EW / 2; ++m) {
+      if (NT) _mm256_stream_si256(o + m, _mm256_loadu_si256(s + m));
+      else _mm256_storeu_si256(o + m, _mm256_loadu_si256(s + m));
+    }
+  } else {
+    const __m128i* s = reinterpret_cast<const __m128i*>(sp);
+    __m128i* o = reinterpret_cast<__m128i*>(op);
+    for (uint32_t m = 0; m < EW; ++m) {
+      if (NT) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
+      else _mm_storeu_si128(o + m, _mm_loadu_si128(s + m));
+    }
+  }
+}
+
+template <int PF, int PF2, bool END, int EWC, bool W32>
 void pack_worker(const HostData& d, uint32_t eo, uint64_t E, uint32_t ew, const Chunk& c, uint8_t* dst, uint64_t n,
                  uint64_t kGrab, bool nt, const PackSink* sink, std::atomic<uint64_t>& next) {
   const uint32_t EW = EWC ? (uint32_t)EWC : ew;
@@ -327,18 +348,14 @@ void pack_worker(const HostData& d, uint32_t eo, uint64_t E, uint32_t ew, const 
       for (uint64_t j = j0; j < j1; ++j) {
         if (j + PF < j1) pf(c.lo + j + PF);
         if (PF2 && j + PF2 < j1) _mm_prefetch((const char*)src(c.lo + j + PF2), _MM_HINT_T1);
-        const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
-        __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
-        for (uint32_t m = 0; m < EW; ++m) _mm_stream_si128(o + m, _mm_loadu_si128(s + m));
+        copy_field<EWC, W32, true>(src(c.lo + j), dst + j * E, EW);
       }
       if (sink) _mm_sfence();
     } else {
       for (uint64_t j = j0; j < j1; ++j) {
         if (j + PF < j1) pf(c.lo + j + PF);
         if (PF2 && j + PF2 < j1) _mm_prefetch((const char*)src(c.lo + j + PF2), _MM_HINT_T1);
-        const __m128i* s = reinterpret_cast<const __m128i*>(src(c.lo + j));
-        __m128i* o = reinterpret_cast<__m128i*>(dst + j * E);
-        for (uint32_t m = 0; m < EW; ++m) _mm_storeu_si128(o + m, _mm_loadu_si128(s + m));
+        copy_field<EWC, W32, false>(src(c.lo + j), dst + j * E, EW);
       }
     }
     if (sink) (*sink)(j0 * E, (j1 - j0) * E);
@@ -346,13 +363,13 @@ void pack_worker(const HostData& d, uint32_t eo, uint64_t E, uint32_t ew, const 
   _mm_sfence();
 }
 
-template <int PF, int PF2, bool END>
+template <int PF, int PF2, bool END, bool W32 = false>
 PackFn pack_for_ew(uint32_t ew) {
   switch (ew) {
-    case 1: return pack_worker<PF, PF2, END, 1>;
-    case 2: return pack_worker<PF, PF2, END, 2>;
-    case 6: return pack_worker<PF, PF2, END, 6>;
-    default: return pack_worker<PF, PF2, END, 0>;
+    case 1: return pack_worker<PF, PF2, END, 1, false>;
+    case 2: return pack_worker<PF, PF2, END, 2, W32>;
+    case 6: return pack_worker<PF, PF2, END, 6, W32>;
+    default: return pack_worker<PF, PF2, END, 0, false>;
   }
 }
 
@@ -360,15 +377,18 @@ PackFn pack_for_ew(uint32_t ew) {
 // (HYBRID, zero-copy gathers running; profiles/r02_packer.md): grep 16/0/- 205.7 GB/s, 8/64/ends
 // 208.7, 16/64/ends 210.0, 16/0/ends 199.8, 32/128/ends 205.0, 8/0/ends 201.5; sparse group-by
 // 16/0/- 108.9, 8/64/ends 115.3, 16/0/ends 111.5. Default: 8/64/ends.
-PackFn pack_fn(uint32_t ew) {
+PackFn pack_fn(uint32_t ew, bool dst32) {
   const char* e = getenv("BK_PACK_CFG");   // read per chunk (one call), so a process can switch
-  const int cfg = e ? atoi(e) : 2;
+  int cfg = e ? atoi(e) : 2;
+  if (cfg >= 7 && !dst32) cfg = 2;   // 32-B stores need a 32-B aligned destination
   switch (cfg) {
     case 1: return pack_for_ew<16, 0, false>(ew);   // round 1
     case 3: return pack_for_ew<16, 64, true>(ew);
     case 4: return pack_for_ew<16, 0, true>(ew);
     case 5: return pack_for_ew<32, 128, true>(ew);
     case 6: return pack_for_ew<8, 0, true>(ew);
+    case 7: return pack_for_ew<8, 64, true, true>(ew);    // default distances, 32-B AVX2 copies
+    case 8: return pack_for_ew<16, 64, true, true>(ew);
     default: return pack_for_ew<8, 64, true>(ew);
   }
 }
@@ -381,7 +401,7 @@ uint64_t host_pack_chunk(HostPool& pool, const HostData& d, const Access& a, con
   const uint32_t eo = a.ext_off[0], EW = (uint32_t)(E / 16);
   // sweep on the 16-core host (profiles/r01_hybrid_sweep.md): grabs of 4k-16k records read in order
   const uint64_t kGrab = grab ? grab : 16384;
-  const PackFn fn = pack_fn(EW);
+  const PackFn fn = pack_fn(EW, ((uintptr_t)dst & 31) == 0);
   std::atomic<uint64_t> next{0};
   pool.run([&](int) { fn(d, eo, E, EW, c, dst, n, kGrab, nt, sink, next); });
   return size;

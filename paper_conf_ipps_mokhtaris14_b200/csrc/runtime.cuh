@@ -254,6 +254,7 @@ int device_begin(bk_ctx* c);
 int device_end(bk_ctx* c);
 void host_reset(bk_ctx* c);
 int prof_reserve(bk_ctx* c, size_t pairs);
+int refork(bk_ctx* c);   // side streams wait for everything enqueued on s_comp so far
 int end_host(bk_ctx* c, void* stream);
 int trace_begin(bk_ctx* c);
 void drop_graphs(bk_ctx* c);
@@ -302,6 +303,7 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
     if (rc) return rc;
   }
   c->addr_next = 0;
+  if (int rf = refork(c)) return rf;   // the driver's setup on s_comp happens-before every chunk
   for (size_t i = 0; i < C; ++i) {
     Slot& s = c->slots[i % c->cfg.n_slots];
     cudaStream_t cs = concurrent ? c->s_slot[i % c->cfg.n_slots] : c->s_comp;
@@ -365,6 +367,7 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
 // reallocated by a later run with larger parameters, so their current addresses are part of the key
 // and a graph whose buffers moved is never replayed (it would touch freed memory).
 std::string resident_key(const bk_ctx* c);
+std::string mem_key(const void* p);   // address + CUDA allocation id of a caller buffer a graph bakes in
 constexpr size_t kMaxGraphs = 16;   // cached graphs per context (oldest dropped first)
 
 template <class Enqueue>
@@ -378,7 +381,9 @@ int run_device(bk_ctx* c, void* stream, const std::string& key_in, bool graphabl
   BK_CUDA(cudaEventRecord(c->t_begin, c->s_comp));
   int rc;
   // per-stage profiling events must be real stream events (timestamps), so BK_FLAG_PROFILE issues eagerly
-  if (!graphable || (c->cfg.flags & (BK_FLAG_NO_GRAPH | BK_FLAG_PROFILE))) {
+  // outputs registered for this run only are unregistered at its end: a graph of their copies could
+  // never be replayed (mem_key differs next run), so such runs issue eagerly instead of capturing
+  if (!graphable || !c->out_pinned_run.empty() || (c->cfg.flags & (BK_FLAG_NO_GRAPH | BK_FLAG_PROFILE))) {
     if ((rc = device_begin(c)) || (rc = enqueue()) || (rc = device_end(c))) return rc;
     return end_host(c, stream);
   }

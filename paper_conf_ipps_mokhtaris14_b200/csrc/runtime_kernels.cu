@@ -21,9 +21,7 @@ struct WcOut {
   uint64_t* h2;
   bool direct;
   std::string key() const {
-    return direct ? "/d" + std::to_string((uintptr_t)off) + "." + std::to_string((uintptr_t)len) + "." +
-                        std::to_string((uintptr_t)cnt) + "." + std::to_string((uintptr_t)h1) + "." +
-                        std::to_string((uintptr_t)h2)
+    return direct ? "/d" + mem_key(off) + "." + mem_key(len) + "." + mem_key(cnt) + "." + mem_key(h1) + "." + mem_key(h2)
                   : "/s" + std::to_string(h1 != nullptr);
   }
 };
@@ -476,7 +474,7 @@ int run_kmeans(bk_ctx* c, bk_out_kmeans* o, void* stream) {
   const bool tma = stage_tma(p);   // TMA: one 16-warp block per SM; plain loads: two
   const int grid = std::max(1, std::min<int>((p.L + 255) / 256, dev_sms * (tma ? 1 : 2)));
   const std::string key = "kmeans/" + std::to_string(K) + "/" + std::to_string(o->first_index) + "/" +
-                          std::to_string((uintptr_t)o->cid) + "/" + p.key;
+                          mem_key(o->cid) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     BK_CUDA(cudaMemcpyAsync(c->b_mu.p, c->h_mu, (uint64_t)K * 64, cudaMemcpyHostToDevice, c->s_comp));
     BK_CUDA(cudaMemsetAsync(c->b_agg1.p, 0, (uint64_t)K * 8, c->s_comp));
@@ -579,8 +577,7 @@ int run_kmer(bk_ctx* c, bk_out_kmer* o, void* stream) {
   unsigned int* cdone = ccur + NB;
   unsigned long long* cbuf = two ? (unsigned long long*)c->b_kbin.p : bbuf;
   const std::string key = "kmer/" + std::to_string(o->k) + "/" + std::to_string(slots) + "/" + std::to_string(ocap) +
-                          "/" + std::to_string(F) + "/" + std::to_string(split_each) + "/" + std::to_string((uintptr_t)dk) + "/" +
-                          std::to_string((uintptr_t)dc) + "/" + p.key;
+                          "/" + std::to_string(F) + "/" + std::to_string(split_each) + "/" + mem_key(dk) + "/" + mem_key(dc) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     BK_CUDA(cudaMemsetAsync(c->b_table.p, 0, slots * sizeof(KmerEntry), c->s_comp));
     BK_CUDA(cudaMemsetAsync(c->b_blk2.p, 0, R * 5 + NB * 8 + 64, c->s_comp));   // cursors, dirty flags
@@ -649,7 +646,7 @@ int run_partition(bk_ctx* c, bk_out_partition* o, void* stream) {
   BK_CUDA(c->b_totals.ensure(std::max<uint64_t>(C, 1) * B * 8));
   BK_CUDA(c->b_base.ensure((uint64_t)B * 8));
   if ((rc = ensure_out_pinned(c, o->out_records, c->n * 16))) return rc;
-  const std::string key = "part/" + std::to_string(B) + "/" + std::to_string((uintptr_t)o->out_records) + "/" + p.key;
+  const std::string key = "part/" + std::to_string(B) + "/" + mem_key(o->out_records) + "/" + p.key;
   rc = run_device(c, stream, key, graphable(p), p.bounds.size() - 1, [&]() -> int {
     size_t ci = 0;
     return pipeline(c, p, false, [&](const Chunk& ch, Slot& s, cudaStream_t cs, cudaStream_t& rel) -> int {

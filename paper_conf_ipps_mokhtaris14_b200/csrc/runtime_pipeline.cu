@@ -1,6 +1,8 @@
 // runtime_pipeline.cu — stages 1-3 of a chunk (ZC / DENSE on the GPU, CPU assembly on the host pool),
 // profiling and delay-injection hooks, fork/join of the context's streams, stage statistics and
 // the CUDA-graph cache.
+#include <cuda.h>   // CU_POINTER_ATTRIBUTE_BUFFER_ID (driver entry point, no -lcuda)
+
 #include "runtime.cuh"
 
 namespace bk {
@@ -544,6 +546,20 @@ int device_begin(bk_ctx* c) {
   BK_CUDA(cudaMemsetAsync(c->d_ctr, 0, 8 * sizeof(unsigned long long), c->s_comp));
   BK_CUDA(cudaEventRecord(c->ev_fork, c->s_comp));
   for (auto st : side_streams(c)) BK_CUDA(cudaStreamWaitEvent(st, c->ev_fork, 0));
+  // test delays: s_comp lags the side streams by ~2 ms here, so a chunk stage that does not wait
+  // for the driver's setup on s_comp (centroids, memsets) reads it uninitialised
+  if (c->cfg.flags & BK_FLAG_TEST_DELAYS) launch_spin(4000000, c->s_comp);
+  return BK_OK;
+}
+
+// Work a kernel driver enqueues on s_comp after device_begin (centroid upload, aggregate / table /
+// cursor memsets) must precede every chunk's stages on the side streams: the pipeline forks them from
+// s_comp again before its first chunk. Without it the slot streams depended only on the first fork
+// (gpurun_out/r02s: eager k-means at 2.5e8 points computed its first chunks against the zeroed
+// centroid buffer; graph replays had hidden the missing edge by timing).
+int refork(bk_ctx* c) {
+  BK_CUDA(cudaEventRecord(c->ev_fork, c->s_comp));
+  for (auto st : side_streams(c)) BK_CUDA(cudaStreamWaitEvent(st, c->ev_fork, 0));
   return BK_OK;
 }
 
@@ -626,6 +642,31 @@ std::string resident_key(const bk_ctx* c) {
   return k;
 }
 
+
+// Identity of a caller-owned buffer a captured graph bakes in (a D2H destination, a mapped result
+// array): its address AND the CUDA allocation it belongs to (CU_POINTER_ATTRIBUTE_BUFFER_ID, unique
+// per allocation / registration in the process). A graph whose copy targets a registration that was
+// since released — or memory freed and reallocated at the same address — must never be replayed:
+// the driver resolved its DMA mapping at capture (a replay after re-registration crashed in the
+// driver, gpurun_out/r02f1: partition run twice on one registration). Unknown memory: address only.
+std::string mem_key(const void* p) {
+  using PfnPtrAttr = CUresult (*)(void*, CUpointer_attribute, CUdeviceptr);
+  static PfnPtrAttr attr = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    PfnPtrAttr r = nullptr;
+    if (cudaGetDriverEntryPoint("cuPointerGetAttribute", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      r = reinterpret_cast<PfnPtrAttr>(f);
+    cudaGetLastError();
+    return r;
+  }();
+  unsigned long long id = 0;
+  if (p && attr && attr(&id, CU_POINTER_ATTRIBUTE_BUFFER_ID, (CUdeviceptr)(uintptr_t)p) != CUDA_SUCCESS) id = 0;
+  char b[48];
+  snprintf(b, sizeof b, "%llx#%llx", (unsigned long long)(uintptr_t)p, id);
+  return b;
+}
 
 // The caller's per-record outputs (partition records, k-means cid, k-mer arrays) are written by DMA,
 // so they must be page-locked while the run copies into them. By default they are registered for

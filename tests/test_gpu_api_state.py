@@ -104,6 +104,44 @@ def test_outputs_released_after_run_unless_kept():
     assert np.array_equal(cid, cid2)
 
 
+@pytest.mark.parametrize("keep", [False, True])
+def test_outputs_reregistered_across_runs_never_replay_stale_graphs(keep):
+    """A captured graph's D2H copies target the output registration of the run that captured it. Runs
+    that re-register the same array (per-run pinning), arrays freed and reallocated at the same
+    address (fresh k-means cid arrays), and kept registrations released by bk_unpin_outputs must
+    never replay a graph bound to a released registration (gpurun_out/r02f1: partition run twice on
+    one registration crashed inside the driver). Many repetitions: the failure was intermittent."""
+    n = 120_000
+    kv = gen.kv(n=n)
+    _, wout = oracle.partition(kv, 256)
+    x = gen.points(n=60_000)
+    _, _, kchk, kcid = oracle.kmeans(x, x[:64], want_cid=True)
+    out = np.empty_like(kv)
+    # kept registrations require the caller to keep the arrays alive (bk.h): then only the arrays
+    # unpinned by bk_unpin_outputs and pinned again change; per-run pinning also sees fresh arrays
+    out2, cid_kept = np.empty_like(kv), np.empty(60_000, np.int32)
+    with bk.Context(window_bytes=1 * MIB, record_size=16, keep_outputs_pinned=keep) as pctx, \
+            bk.Context(window_bytes=1 * MIB, record_size=64, keep_outputs_pinned=keep) as kctx:
+        pctx.register(kv.view(np.uint8).reshape(-1), None, n_records=n)
+        kctx.register(x.view(np.uint8).reshape(-1), None, n_records=60_000)
+        for it in range(12):
+            out[:] = 0
+            o, cc, _ = pctx.partition(256, out=out)
+            assert np.array_equal(bk.partition_materialize(o, cc), wout), it
+            fresh = out2 if keep else np.empty_like(kv)   # a new array, often at a recycled address
+            o2, cc2, _ = pctx.partition(256, out=fresh)
+            assert np.array_equal(bk.partition_materialize(o2, cc2), wout), it
+            del fresh, o2
+            cid = cid_kept if keep else np.empty(60_000, np.int32)
+            cid[:] = -1
+            _, _, chk = kctx.kmeans(x[:64], cid=cid)
+            assert chk == kchk and np.array_equal(cid, kcid), it
+            del cid
+            if keep and it % 3 == 2:
+                pctx.unpin_outputs()
+                kctx.unpin_outputs()
+
+
 def test_current_device_restored_and_struct_size_checked():
     import torch
     torch.cuda.set_device(0)

@@ -625,6 +625,28 @@ def test_results_survive_random_stage_delays(mode):
         ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=len(kv))
         out, cc, bc = ctx.partition(1024)
         assert np.array_equal(global_from_runs(out, cc), wout)
+    # the drivers' setup on the compute stream (centroid upload, aggregate / table / cursor memsets)
+    # is delayed ~2 ms behind the chunk streams: every chunk stage must still wait for it
+    g = gen.groupby(n=100_000, stride=64)
+    wc_, wq, wa = oracle.groupby(g, 100_000, 64, 4096)
+    with bk.Context(window_bytes=512 * 1024, n_slots=2, gather_mode=mode, test_delays=True, record_size=64) as ctx:
+        ctx.register(g, None, n_records=100_000)
+        c, q, a = ctx.groupby(4096)
+        assert np.array_equal(c, wc_) and np.array_equal(q, wq) and np.allclose(a, wa, rtol=1e-5, atol=0)
+    x = gen.points(n=50_000)
+    kc, _, kchk, kcid = oracle.kmeans(x, x[:64], want_cid=True)
+    with bk.Context(window_bytes=512 * 1024, n_slots=2, gather_mode=mode, test_delays=True, record_size=64) as ctx:
+        ctx.register(x.view(np.uint8).reshape(-1), None, n_records=50_000)
+        cid = np.full(50_000, -1, np.int32)
+        c, _, chk = ctx.kmeans(x[:64], cid=cid)
+        assert np.array_equal(cid, kcid) and chk == kchk and np.array_equal(c, kc)
+    d = gen.dna(n=4_000)
+    okm, oct_ = oracle.kmer(d, 4_000, k=31)
+    with bk.Context(window_bytes=256 * 1024, n_slots=2, gather_mode=mode, test_delays=True, record_size=256) as ctx:
+        ctx.register(d, None, n_records=4_000)
+        km, ct, _ = ctx.kmer(k=31, cap=1 << 20)
+    o = np.argsort(km)
+    assert np.array_equal(km[o], okm) and np.array_equal(ct[o], oct_)
 
 
 @pytest.mark.parametrize("mode", ["fused", "zc"])
@@ -690,10 +712,11 @@ def test_wordcount_fused_knobs(monkeypatch, env):
             assert wc_multiset_gpu(buf, *ctx.wordcount(cap=1 << 18)) == want
 
 
-@pytest.mark.parametrize("cfg", ["1", "2", "3", "4", "5", "6"])
+@pytest.mark.parametrize("cfg", ["1", "2", "3", "4", "5", "6", "7", "8"])
 def test_host_packer_prefetch_configs(monkeypatch, cfg):
-    """Every host-packer prefetch configuration (BK_PACK_CFG) packs the same bytes: grep keys of
-    variable records (2 words per field) and sparse group-by fields (1 word) through CPU assembly."""
+    """Every host-packer configuration (BK_PACK_CFG: prefetch distances; 7, 8 with 32-B AVX2 copies)
+    packs the same bytes: grep keys of variable records (2 words per field), sparse group-by fields
+    (1 word) and k-mer sequence fields (6 words) through CPU assembly."""
     monkeypatch.setenv("BK_PACK_CFG", cfg)
     gb, goff = gen.grep_records(max_bytes=4 * MIB)
     with bk.Context(window_bytes=1 * MIB, gather_mode="cpu") as ctx:
@@ -705,3 +728,10 @@ def test_host_packer_prefetch_configs(monkeypatch, cfg):
         ctx.register(g, None, n_records=60_000)
         c, q, a = ctx.groupby(4096)
         assert np.array_equal(c, wc_) and np.array_equal(q, wq) and np.allclose(a, wa, rtol=1e-5, atol=0)
+    d = gen.dna(n=6_000)
+    okm, oct_ = oracle.kmer(d, 6_000, k=31)
+    with bk.Context(window_bytes=1 * MIB, record_size=256, gather_mode="cpu") as ctx:
+        ctx.register(d, None, n_records=6_000)
+        km, ct, _ = ctx.kmer(k=31, cap=1 << 20)
+    o = np.argsort(km)
+    assert np.array_equal(km[o], okm) and np.array_equal(ct[o], oct_)
