@@ -387,7 +387,9 @@ PackFn pack_fn(uint32_t ew, bool dst32) {
     case 4: return pack_for_ew<16, 0, true>(ew);
     case 5: return pack_for_ew<32, 128, true>(ew);
     case 6: return pack_for_ew<8, 0, true>(ew);
-    case 7: return pack_for_ew<8, 64, true, true>(ew);    // default distances, 32-B AVX2 copies
+    // 32-B AVX2 copies (round 2, interleaved on one box, gpurun_out/r02u): grep 200.1-201.5 GB/s vs
+    // 208.2-211.1 with the default 16-B loop; sparse group-by (16-B fields, no 32-B path) unchanged
+    case 7: return pack_for_ew<8, 64, true, true>(ew);
     case 8: return pack_for_ew<16, 64, true, true>(ew);
     default: return pack_for_ew<8, 64, true>(ew);
   }

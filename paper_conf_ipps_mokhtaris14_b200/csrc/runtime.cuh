@@ -254,7 +254,7 @@ int device_begin(bk_ctx* c);
 int device_end(bk_ctx* c);
 void host_reset(bk_ctx* c);
 int prof_reserve(bk_ctx* c, size_t pairs);
-int refork(bk_ctx* c);   // side streams wait for everything enqueued on s_comp so far
+int refork(bk_ctx* c);   // compute streams wait for everything enqueued on s_comp so far
 int end_host(bk_ctx* c, void* stream);
 int trace_begin(bk_ctx* c);
 void drop_graphs(bk_ctx* c);
@@ -303,7 +303,7 @@ int pipeline(bk_ctx* c, const Plan& p, bool concurrent, Compute&& compute) {
     if (rc) return rc;
   }
   c->addr_next = 0;
-  if (int rf = refork(c)) return rf;   // the driver's setup on s_comp happens-before every chunk
+  if (int rf = refork(c)) return rf;   // the driver's setup on s_comp happens-before every chunk's compute
   for (size_t i = 0; i < C; ++i) {
     Slot& s = c->slots[i % c->cfg.n_slots];
     cudaStream_t cs = concurrent ? c->s_slot[i % c->cfg.n_slots] : c->s_comp;

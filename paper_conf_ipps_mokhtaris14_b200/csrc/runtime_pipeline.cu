@@ -553,13 +553,14 @@ int device_begin(bk_ctx* c) {
 }
 
 // Work a kernel driver enqueues on s_comp after device_begin (centroid upload, aggregate / table /
-// cursor memsets) must precede every chunk's stages on the side streams: the pipeline forks them from
-// s_comp again before its first chunk. Without it the slot streams depended only on the first fork
+// cursor memsets) must precede every chunk's compute: the pipeline makes the per-slot compute streams
+// wait for s_comp again before its first chunk (stages 1-3 do not read that state, so the first DMAs
+// and gathers still start at once). Without it the compute streams depended only on the first fork
 // (gpurun_out/r02s: eager k-means at 2.5e8 points computed its first chunks against the zeroed
 // centroid buffer; graph replays had hidden the missing edge by timing).
 int refork(bk_ctx* c) {
   BK_CUDA(cudaEventRecord(c->ev_fork, c->s_comp));
-  for (auto st : side_streams(c)) BK_CUDA(cudaStreamWaitEvent(st, c->ev_fork, 0));
+  for (auto st : c->s_slot) BK_CUDA(cudaStreamWaitEvent(st, c->ev_fork, 0));
   return BK_OK;
 }
 
