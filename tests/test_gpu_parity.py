@@ -603,7 +603,7 @@ def test_api_errors():
 
 
 # ------------------------------------------------------------------ delay injection
-@pytest.mark.parametrize("mode", ["zc", "dense", "cpu", "hybrid"])
+@pytest.mark.parametrize("mode", ["zc", "dense", "cpu", "hybrid", "addr"])
 def test_results_survive_random_stage_delays(mode):
     """Random spin kernels before every stage on every stream (and host sleeps before CPU
     assembly) reorder the stages' timing; with a 2-slot ring any missing event dependency
