@@ -27,7 +27,7 @@ def test_reference_arm_json_line():
     assert d["config"]["workload"] == "grep" and d["unit"] == "GB/s"
 
 
-@pytest.mark.parametrize("path", sorted(glob.glob(os.path.join(ROOT, "profiles", "r01_bench_*.json"))))
+@pytest.mark.parametrize("path", sorted(glob.glob(os.path.join(ROOT, "profiles", "r0*_bench_*.json"))))
 def test_committed_bench_lines_carry_the_contract(path):
     d = json.loads(open(path).read().strip().splitlines()[-1])
     assert BASE <= set(d), set(BASE) - set(d)
