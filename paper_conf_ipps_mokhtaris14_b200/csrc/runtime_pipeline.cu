@@ -294,13 +294,17 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   Access a = p.a;
   a.rec_size = c->off ? 0 : c->cfg.record_size;
   if (p.zero_copy) {
-    // ZC mode: stages 1-3 of slot k's chunks on slot k's own staging stream, so consecutive
-    // chunks' zero-copy gathers overlap (one gather's ramp-up and tail hide under the next one's
-    // transfer). HYBRID: stage 1 on s_asm runs ahead, and the gathers share s_copy with the DMAs
-    // of CPU-assembled chunks so chunks become ready in order (grep's compute is ordered).
-    const bool per_slot = p.mode != BK_GATHER_HYBRID;
-    cudaStream_t s1 = per_slot ? c->s_stage[i % c->cfg.n_slots] : c->s_asm;
-    cudaStream_t ss = per_slot ? s1 : c->s_copy;
+    // ZC: stages 1-3 of slot k's chunks on slot k's own staging stream, so consecutive zero-copy
+    // gathers overlap (one gather's ramp-up and tail hide under the next one's transfer).
+    // HYBRID: the zero-copy chunks on one stream of their own (s_asm), so a gather shares the link
+    // with the DMAs of host-packed chunks instead of queueing behind them on s_copy — the
+    // request-bound gather leaves wire capacity the DMAs use (grep +4-6%, sparse group-by +6% on one
+    // box, gpurun_out/r02x) — while zero-copy gathers still run one at a time (several at once
+    // slowed a 2-packer rank by 10%, r02x). Chunks then become ready out of order, which every
+    // compute path allows (per-chunk outputs are indexed by chunk; ordered computes wait for each
+    // chunk's ready event in chunk order).
+    cudaStream_t s1 = p.mode == BK_GATHER_HYBRID ? c->s_asm : c->s_stage[i % c->cfg.n_slots];
+    cudaStream_t ss = s1;
     // two descriptor sets: stage 1 of this chunk writes the set chunk i-2N used, whose compute
     // ended before chunk i-N's gather started (that gather waited for it, earlier on this stream)
     const int set = p.desc_sets == 2 ? (int)((i / c->cfg.n_slots) & 1) : 0;
@@ -308,7 +312,7 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     s.lanes = s.lanes_set[set];
     s.tileK = s.tileK_set[set];
     s.tile_base = s.tile_base_set[set];
-    const bool early = per_slot && p.desc_sets == 2;   // stage 1 need not wait for the slot
+    const bool early = p.desc_sets == 2;   // stage 1 need not wait for the slot
     if (s.used && !early) BK_CUDA(cudaStreamWaitEvent(s1, s.freed, 0));
     BK_DELAY(s1);
     // whole variable-length records: stage 1 reads the offsets zero-copy itself (no DMA in the chain)
@@ -324,10 +328,6 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, s1,
                    meta_zc ? c->off_dev + ch.lo : nullptr);
     BK_PROF(kStAddrgen, s1, false);
-    if (!per_slot) {
-      BK_CUDA(cudaEventRecord(s.copied, s1));
-      BK_CUDA(cudaStreamWaitEvent(ss, s.copied, 0));
-    }
     if (s.used && early) BK_CUDA(cudaStreamWaitEvent(ss, s.freed, 0));   // the stage buffer
     BK_DELAY(ss);
     BK_PROF(kStGather, ss, true);
