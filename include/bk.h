@@ -94,9 +94,13 @@ typedef struct bk_config {
   uint64_t record_size;   /* fixed record length when record_offsets == NULL */
   uint32_t flags;         /* BK_FLAG_* */
   uint32_t lane_bytes;    /* target accessed bytes per lane when lanes == 0; 0 = the kernel's default */
-  uint32_t zc_share_pm;   /* HYBRID: 0 = adaptive split (a zero-copy chunk is issued whenever fewer
-                             than (n_slots-1)/2 are in flight); else per-mille of chunks gathered
-                             zero-copy, deterministic: chunk i is zero-copy iff floor((i+1)s) > floor(i s) */
+  uint32_t zc_share_pm;   /* HYBRID: 0 = adaptive split (a chunk is gathered zero-copy whenever fewer
+                             zero-copy chunks are in flight than max(1, min(n_slots-1, round(t_pack /
+                             t_zc))) of the measured per-chunk host-packing and gather times, and
+                             every chunk is when packing one costs more than n_slots gathers); else
+                             per-mille of chunks gathered zero-copy, deterministic: chunk i is zero-copy
+                             iff floor((i+1)s) > floor(i s). Zero-copy chunks run one at a time on their
+                             own stream, concurrently with the DMAs of host-packed chunks */
   uint32_t addr_elem_bytes; /* BK_GATHER_ADDR: bytes read per generated address (1, 2, 4, 8, 16); every
                              accessed extent (or fixed record) length must be a multiple. 0 = the
                              largest such power of two <= 8 (1 for whole variable-length records) */
