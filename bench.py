@@ -804,6 +804,8 @@ def main():
                         "input byte of every step crosses the host link inside bk_run, in both measurements"},
         "roofline": roof,
         "gpu_launches": int(st["kernel_launches"]) * args.steps,
+        # how the timed steps issued their device work (bk_stats.graph_issue of the last step)
+        "graph_issue": {0: "eager", 1: "captured", 2: "replayed"}.get(int(st.get("graph_issue", 0)), "?"),
         "clocks": clk.summary(),
         "register_s": round(reg_s, 3),
         **({"materialize": box["materialize"]} if "materialize" in box else {}),

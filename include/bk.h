@@ -355,6 +355,10 @@ typedef struct bk_stats {
   double ms_addr_wait;        /*   host time waiting for stage 1's address information */
   double ms_trace_span;       /* BK_FLAG_TRACE: first kernel/copy start to last end of the run (device) */
   uint64_t n_trace_records;   /*   kernels + copies + memsets traced */
+  uint32_t graph_issue;       /* how the run's device work was issued: 0 eager (BK_FLAG_NO_GRAPH /
+                                 PROFILE, host work per chunk, or outputs page-locked for this run only),
+                                 1 captured as a CUDA graph and launched, 2 a cached graph replayed */
+  uint32_t _pad_graph;
 } bk_stats;
 
 BK_API int bk_get_stats(const bk_ctx* ctx, bk_stats* s);

@@ -89,7 +89,7 @@ class bk_stats(C.Structure):
                 ("fused_loader_wait_frac", C.c_double), ("bytes_addr", u64), ("n_addr_lanes", u64),
                 ("n_pattern_lanes", u64), ("n_addresses", u64), ("n_explicit_addr", u64), ("addr_elem_bytes", u32),
                 ("_pad_addr", u32), ("ms_addr_wait", C.c_double), ("ms_trace_span", C.c_double),
-                ("n_trace_records", u64)]
+                ("n_trace_records", u64), ("graph_issue", u32), ("_pad_graph", u32)]
 
 
 class bk_out_pattern(C.Structure):

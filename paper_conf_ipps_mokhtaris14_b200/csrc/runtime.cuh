@@ -385,11 +385,13 @@ int run_device(bk_ctx* c, void* stream, const std::string& key_in, bool graphabl
   // never be replayed (mem_key differs next run), so such runs issue eagerly instead of capturing
   if (!graphable || !c->out_pinned_run.empty() || (c->cfg.flags & (BK_FLAG_NO_GRAPH | BK_FLAG_PROFILE))) {
     if ((rc = device_begin(c)) || (rc = enqueue()) || (rc = device_end(c))) return rc;
+    c->st.graph_issue = 0;
     return end_host(c, stream);
   }
   GraphEntry* ge = nullptr;
   for (auto& g : c->graphs)
     if (g.key == key) ge = &g;
+  const bool replay = ge != nullptr;
   if (ge) {
     const double reg = c->st.ms_register;
     c->st = ge->st;
@@ -427,6 +429,7 @@ int run_device(bk_ctx* c, void* stream, const std::string& key_in, bool graphabl
     c->graphs.push_back(std::move(g));
     ge = &c->graphs.back();
   }
+  c->st.graph_issue = replay ? 2 : 1;
   BK_CUDA(cudaGraphLaunch(ge->exec, c->s_comp));
   return end_host(c, stream);
 }

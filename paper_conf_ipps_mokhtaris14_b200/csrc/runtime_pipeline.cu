@@ -401,6 +401,7 @@ int check_err(bk_ctx* c) {  // after end_host: the error bits arrived with the r
 
 int begin_run(bk_ctx* c, void* stream) {
   BK_CUDA(cudaSetDevice(c->cfg.device));
+  c->st.graph_issue = 0;   // the baselines issue eagerly
   if (int rt = trace_begin(c)) return rt;
   BK_CUDA(cudaMemsetAsync(c->d_err, 0, sizeof(int), c->s_comp));
   BK_CUDA(cudaMemsetAsync(c->d_ctr, 0, 8 * sizeof(unsigned long long), c->s_comp));

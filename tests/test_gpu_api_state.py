@@ -142,6 +142,38 @@ def test_outputs_reregistered_across_runs_never_replay_stale_graphs(keep):
                 kctx.unpin_outputs()
 
 
+def test_graph_issue_reported():
+    """bk_stats.graph_issue: static pipelines capture a graph on the first run and replay it later
+    (kept-pinned or no per-record outputs); outputs page-locked for one run only, NO_GRAPH and
+    host-assembled (HYBRID) runs issue eagerly."""
+    n = 100_000
+    kv = gen.kv(n=n)
+    out = np.empty_like(kv)
+    g = gen.groupby(n=n)
+    for keep, want in ((True, [1, 2, 2]), (False, [0, 0, 0])):
+        with bk.Context(window_bytes=1 * MIB, record_size=16, keep_outputs_pinned=keep) as ctx:
+            ctx.register(kv.view(np.uint8).reshape(-1), None, n_records=n)
+            got = []
+            for _ in range(3):
+                ctx.partition(256, out=out)
+                got.append(ctx.stats()["graph_issue"])
+            assert got == want, (keep, got)
+    for flags, want in (({}, [1, 2]), ({"no_graph": True}, [0, 0])):
+        with bk.Context(window_bytes=1 * MIB, record_size=16, **flags) as ctx:
+            ctx.register(g, None, n_records=n)
+            got = []
+            for _ in range(2):
+                ctx.groupby(4096)
+                got.append(ctx.stats()["graph_issue"])
+            assert got == want, (flags, got)
+    g64 = gen.groupby(n=n, stride=64)
+    with bk.Context(window_bytes=1 * MIB, record_size=64, gather_mode="hybrid") as ctx:
+        ctx.register(g64, None, n_records=n)
+        ctx.groupby(4096)
+        ctx.groupby(4096)
+        assert ctx.stats()["graph_issue"] == 0
+
+
 def test_current_device_restored_and_struct_size_checked():
     import torch
     torch.cuda.set_device(0)
