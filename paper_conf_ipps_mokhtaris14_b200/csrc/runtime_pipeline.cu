@@ -288,7 +288,7 @@ int stage_chunk_addr(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   return BK_OK;
 }
 
-// Stages 1-3 of chunk i into slot s (on s_copy / s_asm); records s.ready.
+// Stages 1-3 of chunk i into slot s (ZC: a staging stream; DENSE: s_copy + s_asm); records s.ready.
 int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
   const Chunk ch = chunk_of(c, p, i);
   Access a = p.a;
@@ -298,13 +298,12 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     // gathers overlap (one gather's ramp-up and tail hide under the next one's transfer).
     // HYBRID: the zero-copy chunks on one stream of their own (s_asm), so a gather shares the link
     // with the DMAs of host-packed chunks instead of queueing behind them on s_copy — the
-    // request-bound gather leaves wire capacity the DMAs use (grep +4-6%, sparse group-by +6% on one
-    // box, gpurun_out/r02x) — while zero-copy gathers still run one at a time (several at once
-    // slowed a 2-packer rank by 10%, r02x). Chunks then become ready out of order, which every
+    // request-bound gather leaves wire capacity the DMAs use (grep +3-10% on two boxes,
+    // profiles/r02_hybrid_streams.md) — while zero-copy gathers still run one at a time (several at
+    // once slowed a 2-packer rank by 10%). Chunks then become ready out of order, which every
     // compute path allows (per-chunk outputs are indexed by chunk; ordered computes wait for each
     // chunk's ready event in chunk order).
-    cudaStream_t s1 = p.mode == BK_GATHER_HYBRID ? c->s_asm : c->s_stage[i % c->cfg.n_slots];
-    cudaStream_t ss = s1;
+    cudaStream_t ss = p.mode == BK_GATHER_HYBRID ? c->s_asm : c->s_stage[i % c->cfg.n_slots];
     // two descriptor sets: stage 1 of this chunk writes the set chunk i-2N used, whose compute
     // ended before chunk i-N's gather started (that gather waited for it, earlier on this stream)
     const int set = p.desc_sets == 2 ? (int)((i / c->cfg.n_slots) & 1) : 0;
@@ -313,21 +312,21 @@ int stage_chunk(bk_ctx* c, const Plan& p, size_t i, Slot& s) {
     s.tileK = s.tileK_set[set];
     s.tile_base = s.tile_base_set[set];
     const bool early = p.desc_sets == 2;   // stage 1 need not wait for the slot
-    if (s.used && !early) BK_CUDA(cudaStreamWaitEvent(s1, s.freed, 0));
-    BK_DELAY(s1);
+    if (s.used && !early) BK_CUDA(cudaStreamWaitEvent(ss, s.freed, 0));
+    BK_DELAY(ss);
     // whole variable-length records: stage 1 reads the offsets zero-copy itself (no DMA in the chain)
     const bool meta_zc = a.whole && c->off && c->off_dev;
-    BK_PROF(kStH2D, s1, true);
+    BK_PROF(kStH2D, ss, true);
     if (c->off && ch.hi > ch.lo) {
       if (!meta_zc)
-        BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, s1));
+        BK_CUDA(cudaMemcpyAsync(s.meta, c->off + ch.lo, (ch.hi - ch.lo) * 8, cudaMemcpyHostToDevice, ss));
       c->st.bytes_meta += (ch.hi - ch.lo) * 8;
     }
-    BK_PROF(kStH2D, s1, false);
-    BK_PROF(kStAddrgen, s1, true);
-    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, s1,
+    BK_PROF(kStH2D, ss, false);
+    BK_PROF(kStAddrgen, ss, true);
+    launch_addrgen(ch, a, s.meta, s.lanes, s.tileK, s.tile_base, p.stage_cap, c->d_err, c->d_ctr + 0, ss,
                    meta_zc ? c->off_dev + ch.lo : nullptr);
-    BK_PROF(kStAddrgen, s1, false);
+    BK_PROF(kStAddrgen, ss, false);
     if (s.used && early) BK_CUDA(cudaStreamWaitEvent(ss, s.freed, 0));   // the stage buffer
     BK_DELAY(ss);
     BK_PROF(kStGather, ss, true);
