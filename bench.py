@@ -712,6 +712,23 @@ def main():
         roof["note"] = ("the zero-copy key gather is bound by outstanding PCIe read requests (one per 32-B key, "
                         "~84 B of read-completion traffic each), not by bytes: frac is against the H2D DMA byte "
                         "peak, request_rate.frac against the probed request-rate peak (DESIGN.md §6, §9)")
+    if dom != "zc" and args.workload == "grep" and st.get("n_chunks_zc") and st.get("ms_zc"):
+        # HYBRID with the packed chunks' DMA as the busiest stage: the zero-copy gather kernel (the
+        # dominant KERNEL of the ncu launch list) still runs beside it, sharing the link; its own
+        # per-launch rooflines, from the profiled pass
+        zc_ms = st["ms_zc"] / st["n_chunks_zc"]
+        recs = st["records_zc"] / st["n_chunks_zc"]
+        key_gbs = recs * 32 / (zc_ms * 1e-3) / 1e9
+        req = recs * 1.1875 / (zc_ms * 1e-3)
+        roof["zc_gather"] = {"kernel": "k_gather_field<zero-copy> (stages 2+3)", "avg_launch_ms": zc_ms,
+                             "launches_per_step": st["n_chunks_zc"], "achieved": key_gbs, "unit": "GB/s",
+                             "frac": key_gbs / peak_h2d, "peak": peak_h2d,
+                             "request_rate": {"bound": "pcie_read_requests", "achieved": req / 1e9, "peak": 0.562,
+                                              "unit": "G requests/s", "frac": req / 0.562e9,
+                                              "peak_source": "profiles/r01_box_probe.txt zc_sparse"},
+                             "note": "runs concurrently with the DMAs of host-packed chunks (the two share the "
+                                     "link), so both per-launch rates are below their solo rates; "
+                                     "hybrid_schedule.frac is the step against the least time this host + link admit"}
     if dom == "fused":
         roof["fused"] = {"units": st["n_units"], "unit_bytes": st["unit_bytes"], "ctas": st["fused_grid"],
                          "loader_ctas": st["fused_loaders"], "ring_slots": st["fused_ring_slots"],
